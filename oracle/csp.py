@@ -1,0 +1,249 @@
+"""CSP scheduling oracle (plus the balanced partition).
+
+Definitions followed:
+* Def.2 dependency preservation: if SN_x and SN_y (x < y) choose the same layer l,
+  SN_y's READ and WRITE of l wait for SN_x's WRITE of l.
+* Alg.2: a queued forward ``qval`` on stage K is blocked if any earlier
+  ``wval`` not in L_f has one of qval's stage-K layers.
+* Alg.1 + P:L154/P:L225: backward first, lower ID first.
+
+Readings: layer id = globally unique (block, choice) (A1); strict
+backward-first with lowest-ID pending backward (A5); queued forwards scanned in ascending ID
+(A6); the stage-0 window W over the lowest unfinished ID (A7); logical integer time with
+completions/deliveries applied before decisions (A8); fixed contiguous partition (A12).
+"""
+from itertools import combinations
+
+import numpy as np
+
+
+# --------------------------------------------------------------------------------------
+# O3: dependency table
+# --------------------------------------------------------------------------------------
+def dep_table(choices):
+    """dep[y][b] = the latest x < y with c_x[b] == c_y[b], else -1 (written out as a scan)."""
+    N, m = len(choices), len(choices[0])
+    dep = np.full((N, m), -1, dtype=np.int64)
+    for y in range(N):
+        for b in range(m):
+            for x in range(y - 1, -1, -1):
+                if choices[x][b] == choices[y][b]:
+                    dep[y, b] = x
+                    break
+    return dep
+
+
+def stage_blocks(stage_of_block, K):
+    return [b for b, s in enumerate(stage_of_block) if s == K]
+
+
+def deps(choices, stage_of_block, y, K):
+    """deps(y,K) = {dep[y][b] : b in blocks(K)} minus {-1} (O3)."""
+    dep = dep_table(choices[: y + 1])
+    return {int(dep[y, b]) for b in stage_blocks(stage_of_block, K)} - {-1}
+
+
+# --------------------------------------------------------------------------------------
+# O5: Algorithm 2, verbatim
+# --------------------------------------------------------------------------------------
+def literal_alg2(Lq, Lf, L_SN, K, stage_of_block):
+    """Algorithm 2 line by line.
+
+    Lq: queue list of subnet ids (scanned in the given order); Lf: finished list;
+    L_SN[y]: subnet y as a list of layer ids (b, c); K: stage.  Returns (qidx, qval)."""
+    for qidx, qval in enumerate(Lq):                          # line 2
+        scheduled = True                                     # line 3
+        for wval in range(0, qval):                          # line 4: [0, qval-1]
+            if wval in Lf:                                   # line 5
+                continue                                     # line 6
+            layers_w = set(L_SN[wval])
+            for l in L_SN[qval]:                             # line 7: l in L_SN[qval][K]
+                if stage_of_block[l[0]] != K:
+                    continue
+                if l in layers_w:                            # line 8
+                    scheduled = False                        # line 9
+                    break                                    # line 10
+            if not scheduled:
+                break
+        if scheduled:                                        # line 11
+            return qidx, qval                                # line 12
+    return -1, -1                                            # line 13
+
+
+# --------------------------------------------------------------------------------------
+# Partition ("D-partition ... roughly the same execution time"; reading A12)
+# --------------------------------------------------------------------------------------
+def balanced_partition(block_cost, D):
+    """Contiguous partition of blocks into D non-empty stages minimising the max stage
+    cost; ties -> lexicographically smallest split points.  Brute force over all splits."""
+    m = len(block_cost)
+    assert 1 <= D <= m
+    best, best_splits = None, None
+    for splits in combinations(range(1, m), D - 1):          # lexicographic order
+        bounds = (0,) + splits + (m,)
+        worst = max(sum(block_cost[bounds[i]:bounds[i + 1]]) for i in range(D))
+        if best is None or worst < best:
+            best, best_splits = worst, bounds
+    sob = np.zeros(m, dtype=np.int32)
+    for K in range(D):
+        sob[best_splits[K]:best_splits[K + 1]] = K
+    return sob
+
+
+def block_partition_cost(cost_f, cost_b):
+    """Per-block partition weight: sum over choices of (cf + cb) (n * the mean, A12)."""
+    return [int(np.sum(cost_f[b]) + np.sum(cost_b[b])) for b in range(len(cost_f))]
+
+
+# --------------------------------------------------------------------------------------
+# O2: logical-time discrete-event CSP schedule
+# --------------------------------------------------------------------------------------
+def task_costs(choices, stage_of_block, cost_f, cost_b, D):
+    """cf[K][y] = max(1, sum_{b in blocks(K)} cost_f[b][c_y[b]]) (same for cb)."""
+    N = len(choices)
+    cf = np.zeros((D, N), dtype=np.int64)
+    cb = np.zeros((D, N), dtype=np.int64)
+    for K in range(D):
+        for y in range(N):
+            sf = sum(int(cost_f[b][choices[y][b]]) for b in stage_blocks(stage_of_block, K))
+            sb = sum(int(cost_b[b][choices[y][b]]) for b in stage_blocks(stage_of_block, K))
+            cf[K, y], cb[K, y] = max(1, sf), max(1, sb)
+    return cf, cb
+
+
+def simulate_csp(choices, stage_of_block, D, W, cf, cb, lam=0, policy=0, ignore_deps=False,
+                 admit=None):
+    """O2.  Returns dict(trace=[(t, K, kind, y)], makespan, order=[[(kind, y)] per stage]).
+
+    kind: 0 = F (forward), 1 = B (backward).  cf, cb: int [D][N] task costs (>= 1).
+    policy 0: strict backward-first (A5).  policy 1: after a backward, try one forward
+    first (Alg.1's alternation).  ``ignore_deps`` gives the no-dependency upper bound used
+    in the sweep report (not CSP).  ``admit(K, inF_K, fin_K) -> y or None`` replaces the
+    dependency-table admission rule (used to cross-check against Algorithm 2 verbatim)."""
+    N = len(choices)
+    dep_sets = [[set() if ignore_deps else deps(choices, stage_of_block, y, K)
+                 for y in range(N)] for K in range(D)]
+    fin = [set() for _ in range(D)]
+    inF = [set() for _ in range(D)]
+    inB = [set() for _ in range(D)]
+    started0 = set()
+    busy = [None] * D              # (end_time, kind, y)
+    last_kind = [None] * D
+    deliveries = []                # (time, kind, K, y): kind 0 -> inF[K], 1 -> inB[K]
+    trace, order = [], [[] for _ in range(D)]
+    t = 0
+    done0 = 0
+    while True:
+        # (1) completions at t, then deliveries with time <= t
+        for K in range(D):
+            if busy[K] is not None and busy[K][0] == t:
+                _, kind, y = busy[K]
+                busy[K] = None
+                if kind == 0:
+                    if K < D - 1:
+                        deliveries.append((t + lam, 0, K + 1, y))
+                    else:
+                        inB[K].add(y)
+                else:
+                    fin[K].add(y)
+                    if K > 0:
+                        deliveries.append((t + lam, 1, K - 1, y))
+                    else:
+                        done0 += 1
+        keep = []
+        for dv in deliveries:
+            if dv[0] <= t:
+                (inF if dv[1] == 0 else inB)[dv[2]].add(dv[3])
+            else:
+                keep.append(dv)
+        deliveries = keep
+        if done0 == N:
+            return dict(trace=trace, makespan=t, order=order)
+        # (2) stage-0 source under the window
+        wm0 = min([y for y in range(N) if y not in fin[0]], default=N)
+        for y in range(N):
+            if y < wm0 + W and y not in started0:
+                inF[0].add(y)
+        # (3) decisions on idle stages
+        for K in range(D):
+            if busy[K] is not None:
+                continue
+            if admit is None:
+                admissible = sorted(y for y in inF[K] if dep_sets[K][y] <= fin[K])
+                first = admissible[0] if admissible else None
+            else:
+                first = admit(K, set(inF[K]), set(fin[K]))
+            choose = None
+            if policy == 1 and last_kind[K] == 1 and first is not None:
+                choose = (0, first)
+            elif inB[K]:
+                choose = (1, min(inB[K]))
+            elif first is not None:
+                choose = (0, first)
+            if choose is None:
+                continue
+            kind, y = choose
+            if kind == 0:
+                inF[K].discard(y)
+                if K == 0:
+                    started0.add(y)
+                busy[K] = (t + int(cf[K][y]), 0, y)
+            else:
+                inB[K].discard(y)
+                busy[K] = (t + int(cb[K][y]), 1, y)
+            last_kind[K] = kind
+            trace.append((t, K, kind, y))
+            order[K].append((kind, y))
+        # (4) advance time
+        nxt = [b[0] for b in busy if b is not None] + [dv[0] for dv in deliveries]
+        assert nxt, "CSP simulation stalled (no pending event)"
+        t = min(nxt)
+
+
+# --------------------------------------------------------------------------------------
+# O4: trace checker (precedence + Table 4 access pattern)
+# --------------------------------------------------------------------------------------
+def check_trace(trace, choices, stage_of_block, D):
+    """Returns a list of violations (empty == valid CSP trace).
+
+    trace: [(t, K, kind, y)] task starts in nondecreasing t, or per-stage order lists
+    converted by the caller.  Checks: F(y,K) before B(y,K); F(y,K) after F(y,K-1);
+    B(y,K) after B(y,K+1); for every candidate l its accesses read F(x1) B(x1) F(x2) B(x2)...
+    with x1 < x2 < ... (Table 4)."""
+    errs = []
+    pos = {}
+    for idx, (t, K, kind, y) in enumerate(trace):
+        pos[(kind, y, K)] = (t, idx)
+    N = len(choices)
+    for y in range(N):
+        for K in range(D):
+            if (0, y, K) not in pos or (1, y, K) not in pos:
+                errs.append(f"missing task y={y} K={K}")
+                continue
+            if pos[(0, y, K)] >= pos[(1, y, K)]:
+                errs.append(f"B before F y={y} K={K}")
+            if K > 0 and pos[(0, y, K)] <= pos[(0, y, K - 1)]:
+                errs.append(f"F({y},{K}) not after F({y},{K-1})")
+            if K < D - 1 and pos[(1, y, K)] <= pos[(1, y, K + 1)]:
+                errs.append(f"B({y},{K}) not after B({y},{K+1})")
+    # per-candidate access sequence in trace order on its owning stage
+    acc = {}
+    for (t, K, kind, y) in trace:
+        for b in stage_blocks(stage_of_block, K):
+            acc.setdefault((b, int(choices[y][b])), []).append((kind, y))
+    for l, seq in acc.items():
+        users = sorted({y for _, y in seq})
+        expect = [(k, y) for y in users for k in (0, 1)]
+        if seq != expect:
+            errs.append(f"candidate {l} access order {seq} != {expect}")
+    return errs
+
+
+def expected_versions(choices):
+    """Version invariant: v(y, (b,c)) = #{x < y : c_x[b] == c}."""
+    N, m = len(choices), len(choices[0])
+    v = np.zeros((N, m), dtype=np.int64)
+    for y in range(N):
+        for b in range(m):
+            v[y, b] = sum(1 for x in range(y) if choices[x][b] == choices[y][b])
+    return v

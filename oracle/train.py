@@ -1,0 +1,126 @@
+"""Sequential supernet training: the numeric oracle.
+
+PAPER.md Def.1: the result of training is the parameters of all layers, bitwise.
+P:L107: inter-subnet reproducibility "requires that the read-write interleaving among
+subnets is equivalent to training each subnet sequentially, one at a time, according to the
+order provided by the exploration algorithm".  P:L96: a later subnet reads a shared layer
+"with the update made in the backward pass (with optimizer step) of the former".  CSP
+(Def.2) reaches exactly this sequential result, so the oracle IS the sequential
+definition:
+
+    for y in 0..N-1 (chronological order):
+        forward SN_y's active candidates in block order, loss, backward,
+        theta[b, c_y[b]] -= lr * dL_y/dtheta[b, c_y[b]]   for every block b
+
+Readings: plain SGD, constant lr, no momentum/weight decay, only active candidates change
+(A3); dgrad uses pre-update weights (A4); loss = mean((y - t)^2) over all elements (A18);
+no stem/head for the MLP/transformer families (A2).
+"""
+import numpy as np
+
+from . import mlp, transformer
+
+FAMILIES = {"mlp": mlp, "transformer": transformer}
+
+
+def candidate_layout(cfg, b, c):
+    if cfg["family"] == "mlp":
+        return mlp.layout(cfg)
+    if cfg["family"] == "transformer":
+        return transformer.layout(cfg, c)
+    raise ValueError(cfg["family"])
+
+
+def candidate_size(cfg, b, c):
+    return sum(int(np.prod(s)) for _, s, _, _ in candidate_layout(cfg, b, c))
+
+
+def unpack(cfg, b, c, vec):
+    """Packed float vector -> dict of float64 arrays (packing order of the layout)."""
+    out, off = {}, 0
+    for name, shape, _, _ in candidate_layout(cfg, b, c):
+        n = int(np.prod(shape))
+        out[name] = np.asarray(vec[off:off + n], dtype=np.float64).reshape(shape)
+        off += n
+    assert off == len(vec)
+    return out
+
+
+def pack(cfg, b, c, params):
+    return np.concatenate([np.asarray(params[name], dtype=np.float64).ravel()
+                           for name, _, _, _ in candidate_layout(cfg, b, c)])
+
+
+def mse_loss(y, t):
+    """A18: mean((y - t)^2) over all elements, and its gradient."""
+    diff = y - t
+    return float(np.mean(diff * diff)), 2.0 * diff / diff.size
+
+
+def _block_fwd(cfg, p, x, c):
+    if cfg["family"] == "mlp":
+        return mlp.forward(p, x)
+    return transformer.forward(p, x, cfg["choice_heads"][c])
+
+
+def _block_bwd(cfg, p, tape, dy):
+    if cfg["family"] == "mlp":
+        return mlp.backward(p, tape, dy)
+    return transformer.backward(p, tape, dy)
+
+
+def subnet_step(cfg, theta, choice, x, t):
+    """One subnet's forward + backward.  Returns (loss, grads{(b,c): dict}).
+
+    Does not modify theta.  All gradients are taken at the pre-update parameters.
+    """
+    h = np.asarray(x, dtype=np.float64)
+    tapes = []
+    for b, c in enumerate(choice):
+        p = theta[(b, int(c))]
+        h, tape = _block_fwd(cfg, p, h, int(c))
+        tapes.append(tape)
+    loss, dy = mse_loss(h, np.asarray(t, dtype=np.float64))
+    grads = {}
+    for b in reversed(range(len(choice))):
+        c = int(choice[b])
+        dy, g = _block_bwd(cfg, theta[(b, c)], tapes[b], dy)
+        grads[(b, c)] = g
+    return loss, grads
+
+
+def sgd_apply(theta, grads, lr):
+    for key, g in grads.items():
+        p = theta[key]
+        for name in g:
+            p[name] = p[name] - lr * g[name]
+
+
+def train_sequential(cfg, theta0, choices, batches, order=None):
+    """O1.  theta0: {(b,c): packed vector}; choices: int [N, m]; batches: list of (x, t).
+
+    ``order`` (default chronological 0..N-1) exists only for the reordering-invariance
+    property test: any linear extension of the conflict order must give identical results.
+    Returns (theta {(b,c): packed float64 vector}, losses [N]).
+    """
+    theta = {k: unpack(cfg, k[0], k[1], v) for k, v in theta0.items()}
+    N = len(choices)
+    losses = np.zeros(N)
+    for y in (range(N) if order is None else order):
+        x, t = batches[y]
+        loss, grads = subnet_step(cfg, theta, choices[y], x, t)
+        sgd_apply(theta, grads, cfg["lr"])
+        losses[y] = loss
+    return {k: pack(cfg, k[0], k[1], v) for k, v in theta.items()}, losses
+
+
+def initial_theta(cfg):
+    """theta0 from the shared counter hash (synth.init_packed), every candidate."""
+    from synth import init_packed
+    n = cfg["n_choices"]
+    theta = {}
+    for b in range(cfg["n_blocks"]):
+        for c in range(n):
+            segs = [(int(np.prod(s)), kind, fan) for _, s, kind, fan in candidate_layout(cfg, b, c)]
+            theta[(b, c)] = init_packed(cfg["init_seed"], b * n + c, segs)
+    return theta

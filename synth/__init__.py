@@ -1,0 +1,158 @@
+"""Seeded synthetic workload generators shared by the tests, the oracle harness and bench.py.
+
+This module holds NO arithmetic of the method (no forward/backward, no scheduling, no
+update rule).  It only produces inputs: workload configurations, subnet choice vectors,
+input batches and the counter-based initial parameter values.  Both sides of every parity
+test receive what this module generates:
+
+* the CUDA path receives choice vectors and batches through the C ABI and generates its own
+  initial parameters with its own C++ implementation of the same counter hash;
+* the oracle (``oracle/``) receives the same choice vectors and batches, and the initial
+  parameters from :func:`init_packed` below.
+
+Workload recipe:
+* choices: uniform per choice block (§3 "Preliminaries": "per choice block
+  uniform sampling"), NumPy PCG64 ``default_rng(arch_seed)``, arch_seed = 0;
+* batch y: inputs and targets N(0,1) float32 from ``default_rng([data_seed, y])``,
+  data_seed = 1, so batch y does not depend on how many subnets are generated;
+* parameters: U(-1/sqrt(fan_in), 1/sqrt(fan_in)) from a splitmix64 counter hash keyed by
+  (init_seed, candidate uid = b*n + c, element index i); LayerNorm gamma = 1, beta = 0.
+"""
+from __future__ import annotations
+
+import copy
+import numpy as np
+
+ARCH_SEED = 0
+DATA_SEED = 1
+INIT_SEED = 2
+
+# ----------------------------------------------------------------------------------------
+# Workload configurations (BASELINE.json "configs").  Plain dicts so the
+# oracle and the binding each interpret them with their own code.
+# ----------------------------------------------------------------------------------------
+CONFIGS = {
+    # configs[0]: "toy supernet: 4 layers x 4 MLP choice blocks (width 64), 2 stages,
+    # 16 subnets, batch 8, fp32"
+    "toy": dict(family="mlp", n_blocks=4, n_choices=4, batch=8, width=64, lr=0.05,
+                compute_dtype="fp32", n_stages=2, n_subnets=16),
+    # configs[2]: "Transformer supernet (24 layers, choices over FFN width/heads, seq 128,
+    # batch 32) bf16".  n = 4 = {h 8,16} x {f 2048,4096}.
+    "transformer": dict(family="transformer", n_blocks=24, n_choices=4, batch=32,
+                        d_model=1024, seq_len=128,
+                        choice_heads=[8, 8, 16, 16], choice_ffn=[2048, 4096, 2048, 4096],
+                        lr=0.01, compute_dtype="bf16", n_stages=8, n_subnets=256),
+    # configs[3]: "large Transformer supernet (48 layers x 8 choices)".
+    "large_transformer": dict(family="transformer", n_blocks=48, n_choices=8, batch=32,
+                              d_model=2048, seq_len=128,
+                              choice_heads=[16] * 4 + [32] * 4,
+                              choice_ffn=[4096, 8192, 12288, 16384] * 2,
+                              lr=0.01, compute_dtype="bf16", n_stages=8, n_subnets=64),
+    # Small transformer used by the parity tests: several GEMM tiles in every dimension
+    # and ragged tails (d=192 is 1.5 x 128; f=320 is 2.5 x 128), seq 128 like the real one.
+    "tiny_transformer": dict(family="transformer", n_blocks=4, n_choices=3, batch=2,
+                             d_model=192, seq_len=128,
+                             choice_heads=[3, 2, 3], choice_ffn=[320, 384, 192],
+                             lr=0.01, compute_dtype="bf16", n_stages=2, n_subnets=8),
+}
+
+
+def sweep_config(n_choices: int) -> dict:
+    """configs[4]: search-space sweep; C3 with a uniform candidate shape (h=16, f=3072)."""
+    return dict(family="transformer", n_blocks=24, n_choices=n_choices, batch=32,
+                d_model=1024, seq_len=128, choice_heads=[16] * n_choices,
+                choice_ffn=[3072] * n_choices, lr=0.01, compute_dtype="bf16",
+                n_stages=8, n_subnets=256)
+
+
+def get_config(name: str, **overrides) -> dict:
+    cfg = copy.deepcopy(CONFIGS[name])
+    cfg.update(overrides)
+    cfg.setdefault("init_seed", INIT_SEED)
+    return cfg
+
+
+# ----------------------------------------------------------------------------------------
+# Subnet choice vectors
+# ----------------------------------------------------------------------------------------
+def sample_choices(n_subnets: int, n_blocks: int, n_choices: int,
+                   seed: int = ARCH_SEED) -> np.ndarray:
+    """Uniform per-block sampling.  Row y is subnet SN_y's choice vector."""
+    rng = np.random.default_rng(seed)
+    return rng.integers(0, n_choices, size=(n_subnets, n_blocks), dtype=np.int64).astype(np.int32)
+
+
+# ----------------------------------------------------------------------------------------
+# Batches
+# ----------------------------------------------------------------------------------------
+def batch_shape(cfg: dict) -> tuple:
+    if cfg["family"] == "mlp":
+        return (cfg["batch"], cfg["width"])
+    if cfg["family"] == "transformer":
+        return (cfg["batch"], cfg["seq_len"], cfg["d_model"])
+    raise ValueError(cfg["family"])
+
+
+def make_batch(cfg: dict, y: int, seed: int = DATA_SEED):
+    """Input and target for subnet y: N(0,1) float32, independent of N."""
+    rng = np.random.default_rng([seed, int(y)])
+    shp = batch_shape(cfg)
+    x = rng.standard_normal(shp, dtype=np.float32)
+    t = rng.standard_normal(shp, dtype=np.float32)
+    return x, t
+
+
+# ----------------------------------------------------------------------------------------
+# Counter-based initial parameters (SURVEY §8c reading A21)
+# ----------------------------------------------------------------------------------------
+_M64 = np.uint64(0xFFFFFFFFFFFFFFFF)
+_GOLD = np.uint64(0x9E3779B97F4A7C15)
+
+
+def _splitmix64(x: np.ndarray) -> np.ndarray:
+    with np.errstate(over="ignore"):
+        z = x + _GOLD
+        z = (z ^ (z >> np.uint64(30))) * np.uint64(0xBF58476D1CE4E5B9)
+        z = (z ^ (z >> np.uint64(27))) * np.uint64(0x94D049BB133111EB)
+        z = z ^ (z >> np.uint64(31))
+    return z
+
+
+def hash_uniform(seed: int, uid: int, start: int, count: int) -> np.ndarray:
+    """u_i = (splitmix64(seed ^ (uid*GOLD + i)) >> 40) * 2^-24 for i in [start, start+count)."""
+    i = np.arange(start, start + count, dtype=np.uint64)
+    with np.errstate(over="ignore"):
+        key = np.uint64(seed) ^ (np.uint64(uid) * _GOLD + i)
+    z = _splitmix64(key)
+    return (z >> np.uint64(40)).astype(np.float32) * np.float32(2.0 ** -24)
+
+
+def init_packed(seed: int, uid: int, segments) -> np.ndarray:
+    """Packed float32 parameter vector of one candidate.
+
+    ``segments`` is a list of (size, kind, fan_in) in packing order, kind in
+    {"uniform", "ones", "zeros"}.  Element i of the packed vector (counted over all
+    segments) uses counter i, so the value does not depend on how segments are grouped.
+    """
+    total = sum(s for s, _, _ in segments)
+    out = np.empty(total, dtype=np.float32)
+    off = 0
+    for size, kind, fan_in in segments:
+        if kind == "uniform":
+            bound = np.float32(1.0) / np.sqrt(np.float32(fan_in))
+            u = hash_uniform(seed, uid, off, size)
+            out[off:off + size] = bound * (np.float32(2.0) * u - np.float32(1.0))
+        elif kind == "ones":
+            out[off:off + size] = 1.0
+        elif kind == "zeros":
+            out[off:off + size] = 0.0
+        else:
+            raise ValueError(kind)
+        off += size
+    return out
+
+
+def cost_table_uniform(n_blocks: int, n_choices: int, cf: int = 1, cb: int = 2):
+    """The canonical unit cost table of SURVEY §8c A8 (cf=1, cb=2 per block)."""
+    return (np.full((n_blocks, n_choices), cf, dtype=np.int32),
+            np.full((n_blocks, n_choices), cb, dtype=np.int32))

@@ -1,0 +1,186 @@
+"""Pins for oracle/csp.py.
+
+* the hand-worked example of SURVEY §8c (fixture tests/golden/csp_worked_example.json);
+* special cases: n=1 (every subnet shares everything) degenerates to strictly sequential
+  execution; D=1 gives F0 B0 F1 B1 ...;
+* the dependency table agrees with Algorithm 2 executed verbatim on every
+  decision of random CSP runs;
+* every simulated trace satisfies the Table 4 access pattern and the checker
+  rejects mutated traces;
+* the partition follows its definition on hand cases.
+"""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import synth
+from oracle import csp
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def _unit_costs(choices, sob, D, cf=1, cb=2):
+    m, n = len(sob), int(np.max(choices)) + 1
+    return csp.task_costs(choices, sob, np.full((m, n), cf), np.full((m, n), cb), D)
+
+
+def test_worked_example():
+    with open(os.path.join(GOLD, "csp_worked_example.json")) as f:
+        g = json.load(f)
+    choices = np.array(g["choices"])
+    sob = np.array(g["stage_of_block"])
+    D = g["D"]
+    cf, cb = _unit_costs(choices, sob, D, g["cf"], g["cb"])
+    for K in range(D):
+        got = [sorted(csp.deps(choices, sob, y, K)) for y in range(len(choices))]
+        assert got == g["deps"][K]
+    res = csp.simulate_csp(choices, sob, D, g["W"], cf, cb, lam=0, policy=0)
+    assert res["makespan"] == g["makespan"]
+    for K in range(D):
+        got = [("F" if k == 0 else "B") + f"{y}@{t}" for (t, KK, k, y) in res["trace"] if KK == K]
+        assert got == g["stage_order"][K]
+    assert csp.check_trace(res["trace"], choices, sob, D) == []
+
+
+def test_worked_example_variants():
+    sob = np.array([0, 1])
+    ch = np.zeros((3, 2), dtype=int)             # every subnet identical: fully serial
+    cf, cb = csp.task_costs(ch, sob, np.ones((2, 2)), np.full((2, 2), 2), 2)
+    assert csp.simulate_csp(ch, sob, 2, 4, cf, cb)["makespan"] == 18   # = 3 * 2 * 3
+    ch4 = np.array([[0, 0], [1, 0], [0, 1], [1, 1]])
+    sob1 = np.array([0, 0])
+    cf, cb = csp.task_costs(ch4, sob1, np.full((2, 2), 0), np.full((2, 2), 0), 1)
+    # D = 1 with a stage cost of 1 / 2 ticks (costs are per stage here)
+    cf[:] = 1
+    cb[:] = 2
+    res = csp.simulate_csp(ch4, sob1, 1, 4, cf, cb)
+    assert res["makespan"] == 12
+    assert res["order"][0] == [(0, 0), (1, 0), (0, 1), (1, 1), (0, 2), (1, 2), (0, 3), (1, 3)]
+
+
+@pytest.mark.parametrize("D", [1, 2, 3, 4])
+def test_single_choice_is_sequential(D):
+    """n = 1: every subnet depends on its predecessor everywhere -> makespan = N*D*(cf+cb)."""
+    N, m = 5, 4
+    ch = np.zeros((N, m), dtype=int)
+    sob = np.array([b * D // m for b in range(m)])
+    cf = np.ones((D, N), dtype=int)
+    cb = np.full((D, N), 2)
+    res = csp.simulate_csp(ch, sob, D, 4 * D, cf, cb)
+    assert res["makespan"] == N * D * 3
+    # strictly sequential: subnet y+1 starts only after subnet y's last backward
+    starts = {(k, y, K): t for t, K, k, y in res["trace"]}
+    for y in range(N - 1):
+        assert starts[(0, y + 1, 0)] >= starts[(1, y, 0)] + 2
+
+
+def test_disjoint_subnets_pipeline_fully():
+    """No shared candidates: F tasks stream back to back on stage 0 (limited by W)."""
+    N, m, D = 6, 2, 2
+    ch = np.array([[y, y] for y in range(N)])
+    sob = np.array([0, 1])
+    cf = np.ones((D, N), dtype=int)
+    cb = np.full((D, N), 2)
+    res = csp.simulate_csp(ch, sob, D, 8, cf, cb)
+    f0 = [t for t, K, k, y in res["trace"] if K == 0 and k == 0]
+    assert f0[:2] == [0, 1]
+    assert res["makespan"] < N * D * 3
+
+
+def _alg2_admit(choices, sob):
+    L_SN = [[(b, int(c)) for b, c in enumerate(row)] for row in choices]
+
+    def admit(K, inF, fin):
+        Lq = sorted(inF)
+        _, qval = csp.literal_alg2(Lq, fin, L_SN, K, sob)
+        return None if qval < 0 else qval
+    return admit
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_dep_table_equals_literal_alg2(seed):
+    rng = np.random.default_rng(seed)
+    N = int(rng.integers(4, 14))
+    m = int(rng.integers(1, 6))
+    n = int(rng.integers(1, 4))
+    D = int(rng.integers(1, m + 1))
+    W = int(rng.integers(1, 3 * D + 2))
+    ch = synth.sample_choices(N, m, n, seed)
+    _, sob = np.unique(np.sort(rng.integers(0, D, size=m)), return_inverse=True)
+    Dn = int(sob.max()) + 1
+    cf = rng.integers(1, 4, size=(Dn, N))
+    cb = rng.integers(1, 5, size=(Dn, N))
+    lam = int(rng.integers(0, 2))
+    ref = csp.simulate_csp(ch, sob, Dn, W, cf, cb, lam=lam)
+    alt = csp.simulate_csp(ch, sob, Dn, W, cf, cb, lam=lam, admit=_alg2_admit(ch, sob))
+    assert ref["trace"] == alt["trace"]
+    assert csp.check_trace(ref["trace"], ch, sob, Dn) == []
+
+
+@pytest.mark.parametrize("policy", [0, 1])
+def test_random_traces_are_csp_valid(policy):
+    for seed in range(10):
+        rng = np.random.default_rng(100 + seed)
+        N, m, n, D = 10, 4, int(rng.integers(2, 5)), int(rng.integers(1, 5))
+        ch = synth.sample_choices(N, m, n, seed)
+        sob = np.array([b * D // m for b in range(m)])
+        cf = rng.integers(1, 4, size=(D, N))
+        cb = rng.integers(1, 5, size=(D, N))
+        res = csp.simulate_csp(ch, sob, D, 2 * D, cf, cb, policy=policy)
+        assert csp.check_trace(res["trace"], ch, sob, D) == []
+        # the version invariant holds along the trace
+        v = csp.expected_versions(ch)
+        ver = {}
+        for t, K, k, y in res["trace"]:
+            for b in csp.stage_blocks(sob, K):
+                l = (b, int(ch[y][b]))
+                assert ver.get(l, 0) == v[y, b]
+                if k == 1:
+                    ver[l] = ver.get(l, 0) + 1
+
+
+def test_checker_rejects_mutations():
+    ch = np.array([[0, 0], [1, 0], [0, 1], [1, 1]])
+    sob = np.array([0, 1])
+    cf, cb = _unit_costs(ch, sob, 2)
+    tr = csp.simulate_csp(ch, sob, 2, 4, cf, cb)["trace"]
+    assert csp.check_trace(tr, ch, sob, 2) == []
+    # move F(2,0) before B(0,0): subnet 2 reads candidate (0,0) before subnet 0 wrote it
+    i_f2 = next(i for i, e in enumerate(tr) if e[1] == 0 and e[2] == 0 and e[3] == 2)
+    i_b0 = next(i for i, e in enumerate(tr) if e[1] == 0 and e[2] == 1 and e[3] == 0)
+    bad = list(tr)
+    bad.insert(i_b0, bad.pop(i_f2))
+    assert csp.check_trace(bad, ch, sob, 2) != []
+    # drop a task
+    assert csp.check_trace(tr[:-1], ch, sob, 2) != []
+
+
+def test_table4_pattern_example():
+    """Table 4: a layer used by subnets 2, 5, 7 is accessed 2F-2B-5F-5B-7F-7B."""
+    N, m = 8, 3
+    ch = np.array([[y, 0 if y in (2, 5, 7) else y + 1, y] for y in range(N)])
+    for D in (1, 3):
+        sob = np.array([b * D // m for b in range(m)])
+        cf = np.ones((D, N), dtype=int)
+        cb = np.full((D, N), 2)
+        tr = csp.simulate_csp(ch, sob, D, 4 * D, cf, cb)["trace"]
+        K1 = sob[1]
+        seq = [("F" if k == 0 else "B") + str(y) for t, K, k, y in tr if K == K1 and y in (2, 5, 7)]
+        assert seq == ["F2", "B2", "F5", "B5", "F7", "B7"]
+
+
+def test_partition_hand_cases():
+    assert list(csp.balanced_partition([1, 1, 1, 1], 2)) == [0, 0, 1, 1]
+    assert list(csp.balanced_partition([3, 1, 1, 1], 2)) == [0, 1, 1, 1]
+    assert list(csp.balanced_partition([1, 1, 1], 2)) == [0, 1, 1]          # tie -> earliest
+    assert list(csp.balanced_partition([5, 1, 1, 1, 1, 5], 3)) == [0, 1, 1, 1, 1, 2]
+    assert list(csp.balanced_partition([2, 2, 2], 3)) == [0, 1, 2]
+    assert list(csp.balanced_partition([7], 1)) == [0]
+
+
+def test_dep_table_small():
+    ch = np.array([[0, 1], [0, 0], [1, 1], [0, 1]])
+    np.testing.assert_array_equal(csp.dep_table(ch), [[-1, -1], [0, -1], [-1, 0], [1, 2]])
+    np.testing.assert_array_equal(csp.expected_versions(ch), [[0, 0], [1, 0], [0, 1], [2, 2]])
