@@ -1,0 +1,217 @@
+/*
+ * naspipe.h — C ABI of the B200-native NASPipe hot path.
+ *
+ * What it computes (PAPER.md = /root/reference/PAPER.md, cited P:L<line>):
+ *   Causal-synchronous-parallel (CSP) pipelined training of sampled subnets over a
+ *   supernet partitioned into stages (Def.2; Alg.1/Alg.2).
+ *   A supernet is a sequence of m choice blocks with n candidates each; a subnet
+ *   y picks one candidate per block; subnets are trained in the chronological order of
+ *   their submission.  The result (every candidate's parameters and every subnet's loss)
+ *   equals training the subnets one at a time in that order (Def.1), with
+ *   plain SGD on the active candidates (reading A3).
+ *
+ * Conventions
+ *   - Every function returns naspipe_status (0 = OK, < 0 = error) unless stated otherwise.
+ *     naspipe_last_error() returns a thread-local message for the last error.
+ *   - Invalid arguments -> NASPIPE_EINVAL with no state change (a rejected submit does not
+ *     consume a sequence id).  CUDA / NCCL faults are sticky: every later call on the
+ *     handle returns the same code.
+ *   - Pointers are host pointers unless a field says "device".  No torch types.
+ *   - Handles are not thread-safe; one handle per process (multi-process mode: one per rank).
+ *   - Parameters are exchanged as float32 "packed candidate vectors" in the canonical
+ *     order of the family (weights row-major [out,in], then biases, then norm gamma/beta):
+ *       MLP:          W[d,d], b[d]
+ *       TRANSFORMER:  Wqkv[3d,d], bqkv[3d], Wo[d,d], bo[d], ln1.g[d], ln1.b[d],
+ *                     W1[f,d], b1[f], W2[d,f], b2[d], ln2.g[d], ln2.b[d]
+ */
+#ifndef NASPIPE_H_
+#define NASPIPE_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+#if defined(__GNUC__)
+#pragma GCC visibility push(default) /* the library builds with -fvisibility=hidden */
+#endif
+
+#define NASPIPE_ABI_VERSION 1
+
+typedef enum {
+  NASPIPE_OK = 0,
+  NASPIPE_EINVAL = -1,   /* invalid argument / inconsistent spec                        */
+  NASPIPE_ESTATE = -2,   /* call not valid in the current state (e.g. get before drain) */
+  NASPIPE_ENOMEM = -3,   /* host or device allocation failed                            */
+  NASPIPE_ECUDA = -4,    /* CUDA runtime / driver error (sticky)                        */
+  NASPIPE_ENCCL = -5,    /* NCCL error (sticky)                                         */
+  NASPIPE_EBUDGET = -6,  /* HBM weight budget cannot hold one task's candidates         */
+  NASPIPE_EINTERNAL = -7 /* internal invariant violated (e.g. version check) (sticky)   */
+} naspipe_status;
+
+typedef enum { NASPIPE_MLP = 0, NASPIPE_TRANSFORMER = 1, NASPIPE_SPOS_CNN = 2 } naspipe_family;
+typedef enum { NASPIPE_FP32 = 0, NASPIPE_BF16 = 1 } naspipe_dtype; /* compute dtype; masters fp32 */
+
+/* spec.flags */
+#define NASPIPE_FLAG_TRACE 1         /* keep the executed task trace (naspipe_get_trace)      */
+#define NASPIPE_FLAG_VERSION_CHECK 2 /* assert candidate versions at every task start        */
+#define NASPIPE_FLAG_NULL_KERNELS 4  /* run planner/transport only; kernels become no-ops     */
+#define NASPIPE_FLAG_TIMING 8        /* CUDA-event timing of the dominant kernel (GEMM)      */
+
+/*
+ * Supernet specification.  naspipe_create deep-copies it and every array it points to.
+ *   family, n_blocks (m), n_choices (n), batch (B), compute_dtype   — all families
+ *   width                                                          — MLP (d)
+ *   d_model, seq_len, choice_heads[n], choice_ffn[n]               — TRANSFORMER
+ *   lr            plain SGD learning rate (reading A3)
+ *   init_seed     counter-hash initialisation (reading A21): w = bound*(2u-1),
+ *                 u = (splitmix64(seed ^ (uid*0x9E3779B97F4A7C15 + i)) >> 40) * 2^-24,
+ *                 uid = b*n + c, i = index in the packed vector, bound = 1/sqrt(fan_in);
+ *                 LayerNorm gamma = 1, beta = 0.
+ *   stage_of_block [m] optional, non-decreasing, 0..n_stages-1 each used; NULL = balanced
+ *                 partition (reading A12) of the cost table.
+ *   cost_fwd, cost_bwd [m*n] optional integer ticks >= 0 per (block, choice); NULL =
+ *                 naspipe_default_costs.  A stage task costs max(1, sum over its blocks).
+ *   window        W: stage 0 starts F(y,0) only for y < (lowest unfinished id) + W
+ *                 (reading A7); 0 = 4 * n_stages.
+ *   lookahead     residency prefetch depth L in tasks ("2"); 0 = 2.
+ *   hbm_weight_budget_bytes  per-stage device budget for candidate fp32 masters; 0 = all
+ *                 candidates resident (no context switching).
+ *   bwd_policy    0 = strict backward-first (reading A5); 1 = Alg.1 alternation.
+ *   link_latency  lambda ticks for stage-boundary deliveries in the planner (reading A8).
+ */
+typedef struct {
+  int32_t abi_version; /* = NASPIPE_ABI_VERSION */
+  int32_t family;
+  int32_t n_blocks;
+  int32_t n_choices;
+  int32_t batch;
+  int32_t compute_dtype;
+  int32_t width;
+  int32_t d_model;
+  int32_t seq_len;
+  const int32_t* choice_heads;
+  const int32_t* choice_ffn;
+  float lr;
+  uint64_t init_seed;
+  const int32_t* stage_of_block;
+  const int32_t* cost_fwd;
+  const int32_t* cost_bwd;
+  int32_t window;
+  int32_t lookahead;
+  int64_t hbm_weight_budget_bytes;
+  int32_t bwd_policy;
+  int32_t link_latency;
+  int32_t flags;
+} naspipe_supernet_spec;
+
+/* naspipe_batch.where */
+#define NASPIPE_BATCH_HOST 0      /* input/target are host float32 buffers; read
+                                     asynchronously, must stay valid until naspipe_drain */
+#define NASPIPE_BATCH_DEVICE 1    /* device float32 buffers on the stage-0 / last-stage
+                                     device; borrowed until naspipe_drain                */
+#define NASPIPE_BATCH_SYNTHETIC 2 /* generated on the device from synth_seed (perf only)  */
+
+/* One subnet's batch: input [batch x sample] and target [batch x sample] float32, where
+ * sample = width (MLP) or seq_len*d_model (TRANSFORMER), row-major. */
+typedef struct {
+  const void* input;
+  const void* target;
+  int32_t where;
+  uint64_t synth_seed;
+} naspipe_batch;
+
+typedef struct naspipe_handle naspipe_t;
+
+/* ---------------------------------------------------------------------------------------
+ * Engine (the hot path)
+ * ------------------------------------------------------------------------------------- */
+
+/* Single-process engine: all n_stages stages live in this process; stage K runs on CUDA
+ * device (current_device + K) % device_count.  Allocates all device memory, initialises
+ * every candidate from init_seed.  EBUDGET if the budget cannot hold one task's need. */
+int naspipe_create(const naspipe_supernet_spec* spec, int32_t n_stages, naspipe_t** out);
+
+/* Multi-process engine (one process per GPU): this process runs stage `stage_rank` on CUDA
+ * device `device`.  nccl_ids points to 2*(n_stages-1) ncclUniqueId blobs (128 bytes each):
+ * [2k] = activation channel k -> k+1, [2k+1] = gradient channel k+1 -> k, identical on every
+ * rank.  Every rank must make the same sequence of naspipe_submit / naspipe_drain calls. */
+int naspipe_create_rank(const naspipe_supernet_spec* spec, int32_t n_stages, int32_t stage_rank,
+                        int32_t device, const void* nccl_ids, naspipe_t** out);
+
+/* Submit the next subnet in chronological order.  subnet_choice_vec [m] with entries in
+ * [0, n).  Assigns and returns its sequence id (0, 1, 2, ...).  Plans as far as the
+ * streaming rule allows and issues the planned tasks asynchronously. */
+int naspipe_submit(naspipe_t* h, const int32_t* subnet_choice_vec, const naspipe_batch* batch,
+                   int64_t* seq_id_out);
+
+/* Fix N = number of submitted subnets, plan and run everything, wait for the devices. */
+int naspipe_drain(naspipe_t* h);
+
+/* Copy candidate (block, choice)'s fp32 master parameters (packed order above) into dst.
+ * Only on the rank that owns the block.  ESTATE before naspipe_drain. */
+int naspipe_get_params(naspipe_t* h, int32_t block, int32_t choice, float* dst, size_t n_floats);
+int naspipe_set_params(naspipe_t* h, int32_t block, int32_t choice, const float* src,
+                       size_t n_floats);
+
+/* Per-subnet losses (last stage's rank), seq ids [0, n). ESTATE before drain. */
+int naspipe_get_losses(naspipe_t* h, float* dst, int64_t n);
+
+/* Executed tasks in issue order: 4 int64 per task (tick, stage, kind 0=F/1=B, seq id). */
+int naspipe_get_trace(naspipe_t* h, int64_t* dst, size_t cap_tasks, size_t* n_tasks);
+
+/* Statistics, 16 doubles: [0] tasks, [1] kernel launches, [2] h2d bytes, [3] d2h bytes,
+ * [4] p2p bytes, [5] makespan ticks, [6] dominant-kernel launches, [7] dominant-kernel
+ * flops, [8] dominant-kernel ms (TIMING flag), [9] residency loads, [10] residency evicts,
+ * [11] writebacks, [12] version checks passed, [13..15] reserved. */
+int naspipe_get_stats(naspipe_t* h, double* dst16);
+
+/* Residency trace: 4 int64 per event (stage, task index, op 0=LOAD/1=EVICT, uid=b*n+c). */
+int naspipe_get_residency_trace(naspipe_t* h, int64_t* dst, size_t cap, size_t* n);
+
+void naspipe_destroy(naspipe_t* h); /* implies drain; NULL is a no-op */
+
+/* ---------------------------------------------------------------------------------------
+ * Host-only helpers (no device needed): spec queries and the deterministic CSP planner.
+ * ------------------------------------------------------------------------------------- */
+int naspipe_param_count(const naspipe_supernet_spec* spec, int32_t block, int32_t choice,
+                        size_t* n_floats);
+/* Analytic integer tick table (1 tick = 1 us): cost_fwd/cost_bwd [m*n]. */
+int naspipe_default_costs(const naspipe_supernet_spec* spec, int32_t* cost_fwd, int32_t* cost_bwd);
+/* Stage of each block for n_stages (the spec's or the balanced partition). */
+int naspipe_partition(const naspipe_supernet_spec* spec, int32_t n_stages, int32_t* stage_of_block);
+/* Initial packed parameters of one candidate (same generator the engine uses). */
+int naspipe_init_params(const naspipe_supernet_spec* spec, int32_t block, int32_t choice,
+                        float* dst, size_t n_floats);
+
+typedef struct naspipe_plan_handle naspipe_plan_t;
+/* Plan N subnets (choices [N*m]) on n_stages stages: the logical-time CSP schedule
+ * using the spec's window, costs, policy and latency. */
+int naspipe_plan_create(const naspipe_supernet_spec* spec, int32_t n_stages,
+                        const int32_t* choices, int64_t n_subnets, naspipe_plan_t** out);
+int naspipe_plan_trace(const naspipe_plan_t* p, int64_t* dst, size_t cap_tasks, size_t* n_tasks);
+int naspipe_plan_makespan(const naspipe_plan_t* p, int64_t* makespan);
+/* deps(y, K): ids of the latest earlier users of y's stage-K candidates (dependency table). */
+int naspipe_plan_deps(const naspipe_plan_t* p, int64_t y, int32_t stage, int64_t* dst, size_t cap,
+                      size_t* n);
+/* Belady residency of stage K under budget bytes (0 = all resident), depth L (0 = spec's);
+ * 4 int64 per event (stage, task index, op, uid); writebacks counted in *n_writebacks. */
+int naspipe_plan_residency(const naspipe_plan_t* p, int32_t stage, int64_t budget_bytes,
+                           int32_t depth, int64_t* dst, size_t cap, size_t* n,
+                           int64_t* n_writebacks);
+void naspipe_plan_destroy(naspipe_plan_t* p);
+
+/* Fill 128 bytes with a fresh ncclUniqueId (for naspipe_create_rank's nccl_ids). */
+int naspipe_nccl_unique_id(void* out128);
+
+const char* naspipe_last_error(void);
+int naspipe_abi_version(void);
+
+#if defined(__GNUC__)
+#pragma GCC visibility pop
+#endif
+#ifdef __cplusplus
+}
+#endif
+#endif /* NASPIPE_H_ */

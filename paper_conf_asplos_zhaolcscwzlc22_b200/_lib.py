@@ -1,0 +1,313 @@
+"""ctypes marshalling for include/naspipe.h.  No computation happens here."""
+import ctypes as C
+import os
+
+import numpy as np
+
+LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libnaspipe.so")
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"{LIB_PATH} is missing: build it with "
+                      "`python -m paper_conf_asplos_zhaolcscwzlc22_b200.build` (no CPU fallback exists)")
+lib = C.CDLL(LIB_PATH)
+
+ABI_VERSION = 1
+FAMILY = {"mlp": 0, "transformer": 1, "spos": 2}
+DTYPE = {"fp32": 0, "bf16": 1}
+BATCH_HOST, BATCH_DEVICE, BATCH_SYNTHETIC = 0, 1, 2
+FLAG_TRACE, FLAG_VERSION_CHECK, FLAG_NULL_KERNELS, FLAG_TIMING = 1, 2, 4, 8
+STATS_FIELDS = ["tasks", "kernel_launches", "h2d_bytes", "d2h_bytes", "p2p_bytes", "makespan_ticks",
+                "dominant_launches", "dominant_flops", "dominant_ms", "res_loads", "res_evicts",
+                "writebacks", "version_checks", "r13", "r14", "r15"]
+
+_i32p = C.POINTER(C.c_int32)
+_i64p = C.POINTER(C.c_int64)
+
+
+class _SpecStruct(C.Structure):
+    _fields_ = [("abi_version", C.c_int32), ("family", C.c_int32), ("n_blocks", C.c_int32),
+                ("n_choices", C.c_int32), ("batch", C.c_int32), ("compute_dtype", C.c_int32),
+                ("width", C.c_int32), ("d_model", C.c_int32), ("seq_len", C.c_int32),
+                ("choice_heads", _i32p), ("choice_ffn", _i32p), ("lr", C.c_float),
+                ("init_seed", C.c_uint64), ("stage_of_block", _i32p), ("cost_fwd", _i32p),
+                ("cost_bwd", _i32p), ("window", C.c_int32), ("lookahead", C.c_int32),
+                ("hbm_weight_budget_bytes", C.c_int64), ("bwd_policy", C.c_int32),
+                ("link_latency", C.c_int32), ("flags", C.c_int32)]
+
+
+class _BatchStruct(C.Structure):
+    _fields_ = [("input", C.c_void_p), ("target", C.c_void_p), ("where", C.c_int32),
+                ("synth_seed", C.c_uint64)]
+
+
+def _sig(name, res, args):
+    f = getattr(lib, name)
+    f.restype = res
+    f.argtypes = args
+    return f
+
+
+_SP = C.POINTER(_SpecStruct)
+_sig("naspipe_last_error", C.c_char_p, [])
+_sig("naspipe_abi_version", C.c_int, [])
+_sig("naspipe_create", C.c_int, [_SP, C.c_int32, C.POINTER(C.c_void_p)])
+_sig("naspipe_create_rank", C.c_int, [_SP, C.c_int32, C.c_int32, C.c_int32, C.c_void_p, C.POINTER(C.c_void_p)])
+_sig("naspipe_submit", C.c_int, [C.c_void_p, _i32p, C.POINTER(_BatchStruct), _i64p])
+_sig("naspipe_drain", C.c_int, [C.c_void_p])
+_sig("naspipe_get_params", C.c_int, [C.c_void_p, C.c_int32, C.c_int32, C.POINTER(C.c_float), C.c_size_t])
+_sig("naspipe_set_params", C.c_int, [C.c_void_p, C.c_int32, C.c_int32, C.POINTER(C.c_float), C.c_size_t])
+_sig("naspipe_get_losses", C.c_int, [C.c_void_p, C.POINTER(C.c_float), C.c_int64])
+_sig("naspipe_get_trace", C.c_int, [C.c_void_p, _i64p, C.c_size_t, C.POINTER(C.c_size_t)])
+_sig("naspipe_get_stats", C.c_int, [C.c_void_p, C.POINTER(C.c_double)])
+_sig("naspipe_get_residency_trace", C.c_int, [C.c_void_p, _i64p, C.c_size_t, C.POINTER(C.c_size_t)])
+_sig("naspipe_destroy", None, [C.c_void_p])
+_sig("naspipe_param_count", C.c_int, [_SP, C.c_int32, C.c_int32, C.POINTER(C.c_size_t)])
+_sig("naspipe_default_costs", C.c_int, [_SP, _i32p, _i32p])
+_sig("naspipe_partition", C.c_int, [_SP, C.c_int32, _i32p])
+_sig("naspipe_init_params", C.c_int, [_SP, C.c_int32, C.c_int32, C.POINTER(C.c_float), C.c_size_t])
+_sig("naspipe_plan_create", C.c_int, [_SP, C.c_int32, _i32p, C.c_int64, C.POINTER(C.c_void_p)])
+_sig("naspipe_plan_trace", C.c_int, [C.c_void_p, _i64p, C.c_size_t, C.POINTER(C.c_size_t)])
+_sig("naspipe_plan_makespan", C.c_int, [C.c_void_p, _i64p])
+_sig("naspipe_plan_deps", C.c_int, [C.c_void_p, C.c_int64, C.c_int32, _i64p, C.c_size_t, C.POINTER(C.c_size_t)])
+_sig("naspipe_plan_residency", C.c_int, [C.c_void_p, C.c_int32, C.c_int64, C.c_int32, _i64p, C.c_size_t,
+                                         C.POINTER(C.c_size_t), _i64p])
+_sig("naspipe_plan_destroy", None, [C.c_void_p])
+_sig("naspipe_nccl_unique_id", C.c_int, [C.c_void_p])
+
+EXPORTED_SYMBOLS = [
+    "naspipe_create", "naspipe_create_rank", "naspipe_submit", "naspipe_drain", "naspipe_get_params",
+    "naspipe_set_params", "naspipe_get_losses", "naspipe_get_trace", "naspipe_get_stats",
+    "naspipe_get_residency_trace", "naspipe_destroy", "naspipe_param_count", "naspipe_default_costs",
+    "naspipe_partition", "naspipe_init_params", "naspipe_plan_create", "naspipe_plan_trace",
+    "naspipe_plan_makespan", "naspipe_plan_deps", "naspipe_plan_residency", "naspipe_plan_destroy",
+    "naspipe_nccl_unique_id", "naspipe_last_error", "naspipe_abi_version"]
+
+
+class NaspipeError(RuntimeError):
+    def __init__(self, code, msg):
+        super().__init__(f"naspipe error {code}: {msg}")
+        self.code = code
+
+
+def _check(rc):
+    if rc != 0:
+        raise NaspipeError(rc, lib.naspipe_last_error().decode(errors="replace"))
+
+
+def _i32(a):
+    a = np.ascontiguousarray(a, dtype=np.int32)
+    return a, a.ctypes.data_as(_i32p)
+
+
+class Spec:
+    """naspipe_supernet_spec built from a workload dict (synth.CONFIGS style)."""
+
+    def __init__(self, cfg, **over):
+        cfg = dict(cfg, **over)
+        s = _SpecStruct()
+        s.abi_version = ABI_VERSION
+        s.family = FAMILY[cfg["family"]]
+        s.n_blocks, s.n_choices, s.batch = cfg["n_blocks"], cfg["n_choices"], cfg["batch"]
+        s.compute_dtype = DTYPE[cfg.get("compute_dtype", "fp32")]
+        s.width = cfg.get("width", 0)
+        s.d_model, s.seq_len = cfg.get("d_model", 0), cfg.get("seq_len", 0)
+        self._keep = []
+        for name in ("choice_heads", "choice_ffn", "stage_of_block", "cost_fwd", "cost_bwd"):
+            if cfg.get(name) is not None:
+                arr, ptr = _i32(np.asarray(cfg[name]).ravel())
+                self._keep.append(arr)
+                setattr(s, name, ptr)
+        s.lr = cfg.get("lr", 0.01)
+        s.init_seed = cfg.get("init_seed", 2)
+        s.window = cfg.get("window", 0)
+        s.lookahead = cfg.get("lookahead", 0)
+        s.hbm_weight_budget_bytes = cfg.get("hbm_weight_budget_bytes", 0)
+        s.bwd_policy = cfg.get("bwd_policy", 0)
+        s.link_latency = cfg.get("link_latency", 0)
+        s.flags = cfg.get("flags", 0)
+        self.struct = s
+        self.cfg = cfg
+
+    @property
+    def ptr(self):
+        return C.byref(self.struct)
+
+
+class Handle:
+    def __init__(self, ptr, spec):
+        self.ptr = ptr
+        self.spec = spec
+        self.keep = []   # host buffers borrowed until the next drain
+
+    def __del__(self):
+        if getattr(self, "ptr", None):
+            lib.naspipe_destroy(self.ptr)
+            self.ptr = None
+
+
+def naspipe_abi_version():
+    return lib.naspipe_abi_version()
+
+
+def naspipe_create(spec: Spec, n_stages: int) -> Handle:
+    h = C.c_void_p()
+    _check(lib.naspipe_create(spec.ptr, n_stages, C.byref(h)))
+    return Handle(h, spec)
+
+
+def naspipe_create_rank(spec: Spec, n_stages: int, stage_rank: int, device: int, nccl_ids: bytes) -> Handle:
+    h = C.c_void_p()
+    buf = C.create_string_buffer(bytes(nccl_ids), max(1, len(nccl_ids)))
+    _check(lib.naspipe_create_rank(spec.ptr, n_stages, stage_rank, device, buf, C.byref(h)))
+    return Handle(h, spec)
+
+
+def naspipe_nccl_unique_id() -> bytes:
+    buf = C.create_string_buffer(128)
+    _check(lib.naspipe_nccl_unique_id(buf))
+    return buf.raw
+
+
+def _ptr_of(x, keep):
+    if x is None:
+        return None
+    if isinstance(x, int):
+        return x
+    if hasattr(x, "data_ptr"):          # torch tensor (pinned host or device)
+        keep.append(x)
+        return x.data_ptr()
+    a = np.ascontiguousarray(x, dtype=np.float32)
+    keep.append(a)
+    return a.ctypes.data
+
+
+def naspipe_submit(h: Handle, choice, input=None, target=None, where=BATCH_HOST, synth_seed=0) -> int:
+    ch, chp = _i32(np.asarray(choice).ravel())
+    b = _BatchStruct()
+    b.input = _ptr_of(input, h.keep)
+    b.target = _ptr_of(target, h.keep)
+    b.where = where
+    b.synth_seed = synth_seed
+    y = C.c_int64()
+    _check(lib.naspipe_submit(h.ptr, chp, C.byref(b), C.byref(y)))
+    return y.value
+
+
+def naspipe_drain(h: Handle):
+    _check(lib.naspipe_drain(h.ptr))
+    h.keep.clear()
+
+
+def naspipe_destroy(h: Handle):
+    if h.ptr:
+        lib.naspipe_destroy(h.ptr)
+        h.ptr = None
+
+
+def naspipe_param_count(spec: Spec, block: int, choice: int) -> int:
+    n = C.c_size_t()
+    _check(lib.naspipe_param_count(spec.ptr, block, choice, C.byref(n)))
+    return n.value
+
+
+def naspipe_get_params(h: Handle, block: int, choice: int) -> np.ndarray:
+    n = naspipe_param_count(h.spec, block, choice)
+    out = np.empty(n, dtype=np.float32)
+    _check(lib.naspipe_get_params(h.ptr, block, choice, out.ctypes.data_as(C.POINTER(C.c_float)), n))
+    return out
+
+
+def naspipe_set_params(h: Handle, block: int, choice: int, src):
+    a = np.ascontiguousarray(src, dtype=np.float32)
+    _check(lib.naspipe_set_params(h.ptr, block, choice, a.ctypes.data_as(C.POINTER(C.c_float)), a.size))
+
+
+def naspipe_get_losses(h: Handle, n: int) -> np.ndarray:
+    out = np.empty(n, dtype=np.float32)
+    _check(lib.naspipe_get_losses(h.ptr, out.ctypes.data_as(C.POINTER(C.c_float)), n))
+    return out
+
+
+def _get_rows(fn, *args, width=4):
+    n = C.c_size_t()
+    _check(fn(*args, None, 0, C.byref(n)))
+    out = np.zeros((n.value, width), dtype=np.int64)
+    if n.value:
+        _check(fn(*args, out.ctypes.data_as(_i64p), n.value, C.byref(n)))
+    return out
+
+
+def naspipe_get_trace(h: Handle) -> np.ndarray:
+    """(tick, stage, kind 0=F/1=B, seq id) per executed task, in issue order."""
+    return _get_rows(lib.naspipe_get_trace, h.ptr)
+
+
+def naspipe_get_residency_trace(h: Handle) -> np.ndarray:
+    return _get_rows(lib.naspipe_get_residency_trace, h.ptr)
+
+
+def naspipe_get_stats(h: Handle) -> dict:
+    out = (C.c_double * 16)()
+    _check(lib.naspipe_get_stats(h.ptr, out))
+    return dict(zip(STATS_FIELDS, list(out)))
+
+
+def naspipe_default_costs(spec: Spec):
+    m, n = spec.struct.n_blocks, spec.struct.n_choices
+    cf = np.zeros(m * n, dtype=np.int32)
+    cb = np.zeros(m * n, dtype=np.int32)
+    _check(lib.naspipe_default_costs(spec.ptr, cf.ctypes.data_as(_i32p), cb.ctypes.data_as(_i32p)))
+    return cf.reshape(m, n), cb.reshape(m, n)
+
+
+def naspipe_partition(spec: Spec, n_stages: int) -> np.ndarray:
+    out = np.zeros(spec.struct.n_blocks, dtype=np.int32)
+    _check(lib.naspipe_partition(spec.ptr, n_stages, out.ctypes.data_as(_i32p)))
+    return out
+
+
+def naspipe_init_params(spec: Spec, block: int, choice: int) -> np.ndarray:
+    n = naspipe_param_count(spec, block, choice)
+    out = np.empty(n, dtype=np.float32)
+    _check(lib.naspipe_init_params(spec.ptr, block, choice, out.ctypes.data_as(C.POINTER(C.c_float)), n))
+    return out
+
+
+class Plan:
+    """Host-only CSP plan (naspipe_plan_create): trace, makespan, deps, residency."""
+
+    def __init__(self, spec: Spec, n_stages: int, choices):
+        ch, chp = _i32(np.asarray(choices).reshape(-1, spec.struct.n_blocks))
+        self.spec = spec
+        self.n_subnets = ch.shape[0]
+        self.ptr = C.c_void_p()
+        _check(lib.naspipe_plan_create(spec.ptr, n_stages, chp, ch.shape[0], C.byref(self.ptr)))
+
+    def __del__(self):
+        if getattr(self, "ptr", None):
+            lib.naspipe_plan_destroy(self.ptr)
+            self.ptr = None
+
+    def trace(self) -> np.ndarray:
+        return _get_rows(lib.naspipe_plan_trace, self.ptr)
+
+    def makespan(self) -> int:
+        v = C.c_int64()
+        _check(lib.naspipe_plan_makespan(self.ptr, C.byref(v)))
+        return v.value
+
+    def deps(self, y: int, stage: int):
+        return [int(v) for v in _get_rows(lib.naspipe_plan_deps, self.ptr, y, stage, width=1).ravel()]
+
+    def residency(self, stage: int, budget_bytes: int, depth: int = 0):
+        n = C.c_size_t()
+        wb = C.c_int64()
+        _check(lib.naspipe_plan_residency(self.ptr, stage, budget_bytes, depth, None, 0, C.byref(n), C.byref(wb)))
+        out = np.zeros((n.value, 4), dtype=np.int64)
+        if n.value:
+            _check(lib.naspipe_plan_residency(self.ptr, stage, budget_bytes, depth, out.ctypes.data_as(_i64p),
+                                              n.value, C.byref(n), C.byref(wb)))
+        return out, wb.value
+
+
+def naspipe_plan(spec: Spec, n_stages: int, choices) -> Plan:
+    return Plan(spec, n_stages, choices)

@@ -1,0 +1,514 @@
+// Stage executor (see engine.h).  The host walks the CSP plan in tick order and enqueues
+// every task on its stage's compute stream; cross-stage dependencies are CUDA events
+// (single process) or NCCL send/recv on dedicated per-direction channels (multi-process),
+// so execution follows the plan exactly while the devices run asynchronously.
+#include <dlfcn.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <cstring>
+
+#include "engine.h"
+
+namespace naspipe {
+
+#define CU(call)                                                                                 \
+  do {                                                                                           \
+    cudaError_t e_ = (call);                                                                     \
+    NP_REQUIRE(e_ == cudaSuccess, NASPIPE_ECUDA, "%s: %s", #call, cudaGetErrorString(e_));       \
+  } while (0)
+
+// ------------------------------------------------------------------------------ NCCL (dlopen)
+namespace {
+struct NcclApi {
+  void* h = nullptr;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId*) = nullptr;
+  ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+  ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+  ncclResult_t (*Send)(const void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*Recv)(void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*GroupStart)() = nullptr;
+  ncclResult_t (*GroupEnd)() = nullptr;
+  const char* (*GetErrorString)(ncclResult_t) = nullptr;
+};
+NcclApi& nccl() {
+  static NcclApi api;
+  static bool tried = false;
+  if (!tried) {
+    tried = true;
+    const char* env = getenv("NASPIPE_NCCL_LIB");
+    const char* names[] = {env ? env : "libnccl.so.2", "libnccl.so.2", "libnccl.so"};
+    for (const char* n : names) {
+      api.h = dlopen(n, RTLD_NOW | RTLD_GLOBAL);
+      if (api.h) break;
+    }
+    if (api.h) {
+      api.GetUniqueId = (decltype(api.GetUniqueId))dlsym(api.h, "ncclGetUniqueId");
+      api.CommInitRank = (decltype(api.CommInitRank))dlsym(api.h, "ncclCommInitRank");
+      api.CommDestroy = (decltype(api.CommDestroy))dlsym(api.h, "ncclCommDestroy");
+      api.Send = (decltype(api.Send))dlsym(api.h, "ncclSend");
+      api.Recv = (decltype(api.Recv))dlsym(api.h, "ncclRecv");
+      api.GroupStart = (decltype(api.GroupStart))dlsym(api.h, "ncclGroupStart");
+      api.GroupEnd = (decltype(api.GroupEnd))dlsym(api.h, "ncclGroupEnd");
+      api.GetErrorString = (decltype(api.GetErrorString))dlsym(api.h, "ncclGetErrorString");
+    }
+  }
+  NP_REQUIRE(api.h && api.Send && api.Recv && api.CommInitRank, NASPIPE_ENCCL, "libnccl.so.2 not loadable");
+  return api;
+}
+#define NC(call)                                                                                     \
+  do {                                                                                               \
+    ncclResult_t r_ = (call);                                                                        \
+    NP_REQUIRE(r_ == ncclSuccess, NASPIPE_ENCCL, "%s: %s", #call, nccl().GetErrorString(r_));        \
+  } while (0)
+}  // namespace
+
+int nccl_unique_id(void* out) {
+  ncclUniqueId id;
+  NC(nccl().GetUniqueId(&id));
+  std::memcpy(out, &id, sizeof id);
+  return 0;
+}
+
+// Per-rank NCCL channels: activation K-1 -> K (recv) and K -> K+1 (send); gradient K+1 -> K
+// (recv) and K -> K-1 (send).  Each channel is a 2-rank communicator (sender = rank 0) used
+// on its own stream, so the two directions never serialise behind each other.
+struct Transport {
+  ncclComm_t act_in = nullptr, act_out = nullptr, grad_in = nullptr, grad_out = nullptr;
+  cudaStream_t s_act_in, s_act_out, s_grad_in, s_grad_out;
+  std::vector<cudaEvent_t> ev_act_rx, ev_grad_rx, ev_act_tx, ev_grad_tx;  // per slot
+  ~Transport() {
+    for (ncclComm_t c : {act_in, act_out, grad_in, grad_out})
+      if (c) nccl().CommDestroy(c);
+  }
+};
+
+// ------------------------------------------------------------------------------ construction
+Engine::Engine(const Spec& spec, int D) : spec_(spec), D_(D), W_(spec.window(D)), planner_(spec_, D) {
+  NP_REQUIRE(spec_.raw.hbm_weight_budget_bytes == 0, NASPIPE_EINVAL,
+             "hbm_weight_budget_bytes > 0 (context switching) is not enabled in this build");
+  version_.assign((size_t)spec_.m() * spec_.n(), 0);
+  timer_.on = (spec_.raw.flags & NASPIPE_FLAG_TIMING) != 0;
+}
+
+std::unique_ptr<Engine> Engine::create_local(const Spec& spec, int D) {
+  spec.validate_stages(D);
+  int ndev = 0, cur = 0;
+  CU(cudaGetDeviceCount(&ndev));
+  NP_REQUIRE(ndev >= 1, NASPIPE_ECUDA, "no CUDA device");
+  CU(cudaGetDevice(&cur));
+  std::unique_ptr<Engine> e(new Engine(spec, D));
+  e->st_.resize(D);
+  for (int K = 0; K < D; ++K) e->setup_stage(K, (cur + K) % ndev, true);
+  e->link_local_buffers();
+  CU(cudaSetDevice(cur));
+  return e;
+}
+
+std::unique_ptr<Engine> Engine::create_rank(const Spec& spec, int D, int rank, int device, const void* ids) {
+  spec.validate_stages(D);
+  NP_REQUIRE(rank >= 0 && rank < D, NASPIPE_EINVAL, "stage_rank %d not in [0,%d)", rank, D);
+  NP_REQUIRE(D == 1 || ids != nullptr, NASPIPE_EINVAL, "nccl_ids NULL");
+  std::unique_ptr<Engine> e(new Engine(spec, D));
+  e->rank_ = rank;
+  e->st_.resize(D);
+  for (int K = 0; K < D; ++K) {
+    e->st_[K].K = K;
+    e->st_[K].dev = device;
+  }
+  e->setup_stage(rank, device, true);
+  e->link_local_buffers();
+  if (D > 1) {
+    auto tx = std::make_unique<Transport>();
+    CU(cudaSetDevice(device));
+    for (cudaStream_t* s : {&tx->s_act_in, &tx->s_act_out, &tx->s_grad_in, &tx->s_grad_out})
+      CU(cudaStreamCreateWithFlags(s, cudaStreamNonBlocking));
+    for (auto* v : {&tx->ev_act_rx, &tx->ev_grad_rx, &tx->ev_act_tx, &tx->ev_grad_tx}) {
+      v->resize(e->W_);
+      for (auto& ev : *v) CU(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+    }
+    const ncclUniqueId* id = static_cast<const ncclUniqueId*>(ids);
+    // channel k uses ids[2k] (activation k -> k+1, sender rank 0) and ids[2k+1]
+    // (gradient k+1 -> k, sender rank 0).  Initialise channel rank-1 then channel rank: a
+    // chain that cannot deadlock.
+    if (rank > 0) {
+      NC(nccl().GroupStart());
+      NC(nccl().CommInitRank(&tx->act_in, 2, id[2 * (rank - 1)], 1));
+      NC(nccl().CommInitRank(&tx->grad_out, 2, id[2 * (rank - 1) + 1], 0));
+      NC(nccl().GroupEnd());
+    }
+    if (rank < D - 1) {
+      NC(nccl().GroupStart());
+      NC(nccl().CommInitRank(&tx->act_out, 2, id[2 * rank], 0));
+      NC(nccl().CommInitRank(&tx->grad_in, 2, id[2 * rank + 1], 1));
+      NC(nccl().GroupEnd());
+    }
+    e->tx_ = std::move(tx);
+  }
+  return e;
+}
+
+void Engine::setup_stage(int K, int dev, bool local) {
+  StageRt& st = st_[K];
+  st.K = K;
+  st.dev = dev;
+  st.local = local;
+  CU(cudaSetDevice(dev));
+  CU(cudaStreamCreateWithFlags(&st.comp, cudaStreamNonBlocking));
+  CU(cudaStreamCreateWithFlags(&st.copy, cudaStreamNonBlocking));
+  st.arena = std::make_unique<DevArena>(dev);
+  st.fam = make_family(spec_, planner_.blocks_of(K), W_, *st.arena, st.comp);
+  st.fam->timer = &timer_;
+  const size_t n = spec_.batch_elems();
+  st.in.assign(W_, nullptr);
+  st.gout.assign(W_, nullptr);
+  st.out.resize(W_);
+  st.gin.assign(W_, nullptr);
+  for (int s = 0; s < W_; ++s) {
+    st.out[s] = st.arena->alloc<float>(n);
+    if (K > 0) st.gin[s] = st.arena->alloc<float>(n);
+    if (K == 0) st.in[s] = st.arena->alloc<float>(n);
+    if (K == D_ - 1) st.gout[s] = st.arena->alloc<float>(n);
+  }
+  if (K == D_ - 1) {
+    st.target.resize(W_);
+    for (auto& p : st.target) p = st.arena->alloc<float>(n);
+    st.loss = st.arena->alloc<float>(loss_cap_);
+    st.mse_part = st.arena->alloc<float>(mse_blocks(n));
+    CU(cudaMemsetAsync(st.loss, 0, loss_cap_ * sizeof(float), st.comp));
+  }
+  for (auto* v : {&st.ev_f, &st.ev_b, &st.ev_in, &st.ev_tgt}) {
+    v->resize(W_);
+    for (auto& ev : *v) CU(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+  }
+  CU(cudaStreamSynchronize(st.comp));
+}
+
+// Same-device neighbours share boundary buffers (zero copy); otherwise each side owns a
+// receive buffer filled by a peer copy (single process) or NCCL (multi-process).
+void Engine::link_local_buffers() {
+  const size_t n = spec_.batch_elems();
+  for (int K = 0; K < D_; ++K) {
+    StageRt& st = st_[K];
+    if (!st.local) continue;
+    CU(cudaSetDevice(st.dev));
+    for (int s = 0; s < W_; ++s) {
+      if (K > 0) {
+        const StageRt& p = st_[K - 1];
+        st.in[s] = (p.local && p.dev == st.dev) ? p.out[s] : st.arena->alloc<float>(n);
+      }
+      if (K < D_ - 1) {
+        const StageRt& q = st_[K + 1];
+        st.gout[s] = (q.local && q.dev == st.dev) ? q.gin[s] : st.arena->alloc<float>(n);
+      }
+    }
+  }
+}
+
+Engine::~Engine() { shutdown(); }
+
+void Engine::shutdown() {
+  for (auto& st : st_) {
+    if (!st.local || !st.comp) continue;
+    cudaSetDevice(st.dev);
+    cudaStreamSynchronize(st.comp);
+    cudaStreamSynchronize(st.copy);
+  }
+  if (tx_) {
+    for (cudaStream_t s : {tx_->s_act_in, tx_->s_act_out, tx_->s_grad_in, tx_->s_grad_out}) cudaStreamSynchronize(s);
+  }
+  tx_.reset();
+  for (auto& st : st_) {
+    if (!st.local || !st.comp) continue;
+    cudaSetDevice(st.dev);
+    st.fam.reset();
+    st.arena.reset();
+    for (auto* v : {&st.ev_f, &st.ev_b, &st.ev_in, &st.ev_tgt})
+      for (auto ev : *v) cudaEventDestroy(ev);
+    cudaStreamDestroy(st.comp);
+    cudaStreamDestroy(st.copy);
+    st.comp = st.copy = nullptr;
+  }
+}
+
+void Engine::check_sticky() const {
+  if (sticky_code_) throw Error(sticky_code_, "sticky error: " + sticky_msg_);
+}
+void Engine::set_sticky(int code, const std::string& msg) {
+  if (!sticky_code_) {
+    sticky_code_ = code;
+    sticky_msg_ = msg;
+  }
+}
+
+void Engine::cuda_check(const char* what) {
+  cudaError_t e = cudaGetLastError();
+  NP_REQUIRE(e == cudaSuccess, NASPIPE_ECUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+// ------------------------------------------------------------------------------ submit / issue
+int64_t Engine::submit(const int32_t* choice, const naspipe_batch* batch) {
+  NP_REQUIRE(choice && batch, NASPIPE_EINVAL, "choice/batch NULL");
+  NP_REQUIRE(batch->where >= NASPIPE_BATCH_HOST && batch->where <= NASPIPE_BATCH_SYNTHETIC, NASPIPE_EINVAL,
+             "batch.where %d", batch->where);
+  NP_REQUIRE(batch->where == NASPIPE_BATCH_SYNTHETIC || (batch->input && batch->target), NASPIPE_EINVAL,
+             "batch input/target NULL");
+  NP_REQUIRE(planner_.n_subnets() < loss_cap_, NASPIPE_EINVAL, "more than %lld subnets", (long long)loss_cap_);
+  for (int b = 0; b < spec_.m(); ++b)
+    NP_REQUIRE(choice[b] >= 0 && choice[b] < spec_.n(), NASPIPE_EINVAL, "choice[%d]=%d outside [0,%d)", b,
+               choice[b], spec_.n());
+  if (drained_) {
+    planner_.reopen();
+    drained_ = false;
+  }
+  const int64_t y = planner_.add_subnet(choice);
+  batches_.push_back({*batch});
+  planner_.advance();
+  issue_planned();
+  return y;
+}
+
+void Engine::drain() {
+  if (!drained_) {
+    planner_.finalize();
+    planner_.advance();
+    NP_REQUIRE(planner_.done(), NASPIPE_EINTERNAL, "planner did not finish");
+    issue_planned();
+  }
+  for (auto& st : st_) {
+    if (!st.local) continue;
+    CU(cudaSetDevice(st.dev));
+    CU(cudaStreamSynchronize(st.copy));
+    CU(cudaStreamSynchronize(st.comp));
+  }
+  if (tx_)
+    for (cudaStream_t s : {tx_->s_act_in, tx_->s_act_out, tx_->s_grad_in, tx_->s_grad_out})
+      CU(cudaStreamSynchronize(s));
+  cuda_check("drain");
+  timer_.collect();
+  drained_ = true;
+}
+
+void Engine::issue_planned() {
+  const auto& tasks = planner_.tasks();
+  while (issued_ < tasks.size()) issue(tasks[issued_++]);
+}
+
+void Engine::version_check(const Task& t) {
+  // Expected version of candidate (b, c_y[b]) at any task of y = #{x < y : c_x[b] == c_y[b]}
+  // (SURVEY §8c "version invariant"); the backward's update makes it v + 1.
+  for (int b : planner_.blocks_of(t.K)) {
+    const size_t key = (size_t)b * spec_.n() + planner_.choice(t.y, b);
+    NP_REQUIRE(version_[key] == planner_.version(t.y, b), NASPIPE_EINTERNAL,
+               "version check: subnet %lld stage %d block %d sees version %lld, expected %lld", (long long)t.y, t.K,
+               b, (long long)version_[key], (long long)planner_.version(t.y, b));
+    ++version_checks_;
+    if (t.kind == 1) version_[key] += 1;
+  }
+}
+
+void Engine::issue(const Task& t) {
+  const int slot = (int)(t.y % W_);
+  StageRt& st = st_[t.K];
+  if (rank_ >= 0 && tx_) {
+    // multi-process: post receives for the neighbours' tasks in their plan order
+    StageRt& me = st_[rank_];
+    const size_t n = spec_.batch_elems();
+    if (t.kind == 0 && t.K == rank_ - 1) {
+      CU(cudaSetDevice(me.dev));
+      CU(cudaStreamWaitEvent(tx_->s_act_in, me.ev_b[slot], 0));  // slot free (B(y-W) done)
+      NC(nccl().Recv(me.in[slot], n, ncclFloat32, 0, tx_->act_in, tx_->s_act_in));
+      CU(cudaEventRecord(tx_->ev_act_rx[slot], tx_->s_act_in));
+      p2p_bytes_ += 4.0 * n;
+    } else if (t.kind == 1 && t.K == rank_ + 1) {
+      CU(cudaSetDevice(me.dev));
+      CU(cudaStreamWaitEvent(tx_->s_grad_in, me.ev_b[slot], 0));
+      NC(nccl().Recv(me.gout[slot], n, ncclFloat32, 0, tx_->grad_in, tx_->s_grad_in));
+      CU(cudaEventRecord(tx_->ev_grad_rx[slot], tx_->s_grad_in));
+      p2p_bytes_ += 4.0 * n;
+    }
+  }
+  if (!st.local) return;
+  if (spec_.raw.flags & NASPIPE_FLAG_VERSION_CHECK) version_check(t);
+  if (spec_.raw.flags & NASPIPE_FLAG_TRACE) trace_.push_back(t);
+  CU(cudaSetDevice(st.dev));
+  if (t.kind == 0) issue_forward(st, t.y, slot);
+  else issue_backward(st, t.y, slot);
+}
+
+void Engine::issue_forward(StageRt& st, int64_t y, int slot) {
+  const int K = st.K;
+  const size_t n = spec_.batch_elems();
+  const naspipe_batch& bt = batches_[y].b;
+  const bool null_k = (spec_.raw.flags & NASPIPE_FLAG_NULL_KERNELS) != 0;
+  const float* xin = nullptr;
+  if (K == 0) {
+    if (bt.where == NASPIPE_BATCH_HOST) {
+      CU(cudaStreamWaitEvent(st.copy, st.ev_b[slot], 0));
+      CU(cudaMemcpyAsync(st.in[slot], bt.input, n * 4, cudaMemcpyHostToDevice, st.copy));
+      CU(cudaEventRecord(st.ev_in[slot], st.copy));
+      CU(cudaStreamWaitEvent(st.comp, st.ev_in[slot], 0));
+      h2d_bytes_ += 4.0 * n;
+      xin = st.in[slot];
+    } else if (bt.where == NASPIPE_BATCH_DEVICE) {
+      xin = static_cast<const float*>(bt.input);
+    } else {
+      if (!null_k) synth_fill(st.comp, st.in[slot], n, bt.synth_seed * 2 + 0);
+      xin = st.in[slot];
+    }
+  } else if (rank_ < 0) {
+    StageRt& p = st_[K - 1];
+    CU(cudaStreamWaitEvent(st.comp, p.ev_f[slot], 0));
+    if (p.dev != st.dev) {
+      CU(cudaMemcpyPeerAsync(st.in[slot], st.dev, p.out[slot], p.dev, n * 4, st.comp));
+      p2p_bytes_ += 4.0 * n;
+    }
+    xin = st.in[slot];
+  } else {
+    CU(cudaStreamWaitEvent(st.comp, tx_->ev_act_rx[slot], 0));
+    xin = st.in[slot];
+  }
+  const float* tgt = nullptr;
+  if (K == D_ - 1) {
+    if (bt.where == NASPIPE_BATCH_HOST) {
+      CU(cudaStreamWaitEvent(st.copy, st.ev_f[slot], 0));  // previous user's loss done
+      CU(cudaMemcpyAsync(st.target[slot], bt.target, n * 4, cudaMemcpyHostToDevice, st.copy));
+      CU(cudaEventRecord(st.ev_tgt[slot], st.copy));
+      h2d_bytes_ += 4.0 * n;
+      tgt = st.target[slot];
+    } else if (bt.where == NASPIPE_BATCH_DEVICE) {
+      tgt = static_cast<const float*>(bt.target);
+    } else {
+      if (!null_k) synth_fill(st.comp, st.target[slot], n, bt.synth_seed * 2 + 1);
+      tgt = st.target[slot];
+    }
+  }
+  if (rank_ >= 0 && tx_ && K < D_ - 1)  // out[slot] free once the previous send left
+    CU(cudaStreamWaitEvent(st.comp, tx_->ev_act_tx[slot], 0));
+  // stage forward: the candidates chosen by y in this stage's blocks
+  if (!null_k) st.fam->forward(slot, planner_.choice_row(y), xin, st.out[slot], st.comp);
+  if (K == D_ - 1) {
+    if (bt.where == NASPIPE_BATCH_HOST) CU(cudaStreamWaitEvent(st.comp, st.ev_tgt[slot], 0));
+    if (!null_k) mse_loss(st.comp, st.out[slot], tgt, st.gout[slot], st.mse_part, st.loss + y, n);
+  }
+  CU(cudaEventRecord(st.ev_f[slot], st.comp));
+  if (rank_ >= 0 && tx_ && K < D_ - 1) {
+    CU(cudaStreamWaitEvent(tx_->s_act_out, st.ev_f[slot], 0));
+    NC(nccl().Send(st.out[slot], n, ncclFloat32, 1, tx_->act_out, tx_->s_act_out));
+    CU(cudaEventRecord(tx_->ev_act_tx[slot], tx_->s_act_out));
+  }
+  cuda_check("forward");
+}
+
+void Engine::issue_backward(StageRt& st, int64_t y, int slot) {
+  const int K = st.K;
+  const size_t n = spec_.batch_elems();
+  const bool null_k = (spec_.raw.flags & NASPIPE_FLAG_NULL_KERNELS) != 0;
+  if (K < D_ - 1) {
+    if (rank_ < 0) {
+      StageRt& q = st_[K + 1];
+      CU(cudaStreamWaitEvent(st.comp, q.ev_b[slot], 0));
+      if (q.dev != st.dev) {
+        CU(cudaMemcpyPeerAsync(st.gout[slot], st.dev, q.gin[slot], q.dev, n * 4, st.comp));
+        p2p_bytes_ += 4.0 * n;
+      }
+    } else {
+      CU(cudaStreamWaitEvent(st.comp, tx_->ev_grad_rx[slot], 0));
+    }
+  }
+  if (rank_ >= 0 && tx_ && K > 0) CU(cudaStreamWaitEvent(st.comp, tx_->ev_grad_tx[slot], 0));
+  float* dx = K > 0 ? st.gin[slot] : nullptr;
+  if (!null_k) st.fam->backward(slot, planner_.choice_row(y), st.gout[slot], dx, st.comp);
+  CU(cudaEventRecord(st.ev_b[slot], st.comp));
+  if (rank_ >= 0 && tx_ && K > 0) {
+    CU(cudaStreamWaitEvent(tx_->s_grad_out, st.ev_b[slot], 0));
+    NC(nccl().Send(st.gin[slot], n, ncclFloat32, 0, tx_->grad_out, tx_->s_grad_out));
+    CU(cudaEventRecord(tx_->ev_grad_tx[slot], tx_->s_grad_out));
+  }
+  cuda_check("backward");
+}
+
+// ------------------------------------------------------------------------------ read-out
+static int owner_local_index(const std::vector<int>& blocks, int b) {
+  for (size_t j = 0; j < blocks.size(); ++j)
+    if (blocks[j] == b) return (int)j;
+  return -1;
+}
+
+void Engine::get_params(int block, int choice, float* dst, size_t n) {
+  NP_REQUIRE(block >= 0 && block < spec_.m() && choice >= 0 && choice < spec_.n(), NASPIPE_EINVAL,
+             "candidate (%d,%d) out of range", block, choice);
+  NP_REQUIRE(dst && n == spec_.param_count(block, choice), NASPIPE_EINVAL, "n_floats %zu != %zu", n,
+             spec_.param_count(block, choice));
+  NP_REQUIRE(drained_ || planner_.n_subnets() == 0, NASPIPE_ESTATE, "get_params before naspipe_drain");
+  const int K = planner_.stage_of_block()[block];
+  StageRt& st = st_[K];
+  NP_REQUIRE(st.local, NASPIPE_EINVAL, "block %d lives on stage %d, not on this rank", block, K);
+  CU(cudaSetDevice(st.dev));
+  const int j = owner_local_index(planner_.blocks_of(K), block);
+  CU(cudaMemcpy(dst, st.fam->master(j, choice), n * 4, cudaMemcpyDeviceToHost));
+  d2h_bytes_ += 4.0 * n;
+}
+
+void Engine::set_params(int block, int choice, const float* src, size_t n) {
+  NP_REQUIRE(block >= 0 && block < spec_.m() && choice >= 0 && choice < spec_.n(), NASPIPE_EINVAL,
+             "candidate (%d,%d) out of range", block, choice);
+  NP_REQUIRE(src && n == spec_.param_count(block, choice), NASPIPE_EINVAL, "n_floats %zu != %zu", n,
+             spec_.param_count(block, choice));
+  NP_REQUIRE(drained_ || planner_.n_subnets() == 0, NASPIPE_ESTATE, "set_params with work in flight");
+  const int K = planner_.stage_of_block()[block];
+  StageRt& st = st_[K];
+  NP_REQUIRE(st.local, NASPIPE_EINVAL, "block %d lives on stage %d, not on this rank", block, K);
+  CU(cudaSetDevice(st.dev));
+  const int j = owner_local_index(planner_.blocks_of(K), block);
+  CU(cudaMemcpy(st.fam->master(j, choice), src, n * 4, cudaMemcpyHostToDevice));
+  st.fam->refresh_shadow(j, choice, st.comp);
+  CU(cudaStreamSynchronize(st.comp));
+}
+
+void Engine::get_losses(float* dst, int64_t n) {
+  NP_REQUIRE(dst && n >= 0 && n <= planner_.n_subnets(), NASPIPE_EINVAL, "bad loss count %lld", (long long)n);
+  NP_REQUIRE(drained_, NASPIPE_ESTATE, "get_losses before naspipe_drain");
+  StageRt& st = st_[D_ - 1];
+  NP_REQUIRE(st.local, NASPIPE_EINVAL, "losses live on the last stage's rank");
+  CU(cudaSetDevice(st.dev));
+  if (n) CU(cudaMemcpy(dst, st.loss, n * 4, cudaMemcpyDeviceToHost));
+}
+
+void Engine::get_trace(int64_t* dst, size_t cap, size_t* n) {
+  NP_REQUIRE(n, NASPIPE_EINVAL, "n NULL");
+  *n = trace_.size();
+  for (size_t i = 0; i < trace_.size() && i < cap && dst; ++i) {
+    dst[4 * i] = trace_[i].t;
+    dst[4 * i + 1] = trace_[i].K;
+    dst[4 * i + 2] = trace_[i].kind;
+    dst[4 * i + 3] = trace_[i].y;
+  }
+}
+
+void Engine::get_stats(double* o) {
+  NP_REQUIRE(o, NASPIPE_EINVAL, "dst NULL");
+  std::fill(o, o + 16, 0.0);
+  double launches = 0;
+  for (auto& st : st_)
+    if (st.local && st.fam) launches += (double)st.fam->counters.launches;
+  o[0] = (double)issued_;
+  o[1] = launches;
+  o[2] = h2d_bytes_;
+  o[3] = d2h_bytes_;
+  o[4] = p2p_bytes_;
+  o[5] = (double)planner_.makespan();
+  o[6] = timer_.launches;
+  o[7] = timer_.flops;
+  o[8] = timer_.ms;
+  o[12] = (double)version_checks_;
+}
+
+void Engine::get_residency_trace(int64_t* dst, size_t cap, size_t* n) {
+  (void)dst;
+  (void)cap;
+  NP_REQUIRE(n, NASPIPE_EINVAL, "n NULL");
+  *n = 0;  // all candidates resident (hbm_weight_budget_bytes == 0)
+}
+
+}  // namespace naspipe

@@ -1,0 +1,89 @@
+// Stage executor: turns the CSP plan into device work.  Each stage owns one compute stream
+// (tasks in plan order), an input-copy stream, per-slot boundary buffers and events.  Slots
+// are indexed y mod W: every in-flight subnet lies in [wm0, wm0 + W) (reading A7), so slot
+// reuse is ordered by the plan itself.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "family.h"
+#include "planner.h"
+
+namespace naspipe {
+
+struct Transport;  // NCCL channels (multi-process mode)
+int nccl_unique_id(void* out128);
+
+struct StageRt {
+  int K = 0, dev = 0;
+  bool local = false;
+  cudaStream_t comp = nullptr, copy = nullptr;
+  std::unique_ptr<DevArena> arena;
+  std::unique_ptr<Family> fam;
+  // boundary buffers per slot (device, on dev)
+  std::vector<float*> in, out, gin, gout, target;
+  std::vector<cudaEvent_t> ev_f, ev_b, ev_in, ev_tgt;
+  float* loss = nullptr;  // [loss_cap] on the last stage
+  float* mse_part = nullptr;
+};
+
+struct BatchRec {
+  naspipe_batch b;
+};
+
+class Engine {
+ public:
+  static std::unique_ptr<Engine> create_local(const Spec& spec, int D);
+  static std::unique_ptr<Engine> create_rank(const Spec& spec, int D, int rank, int device, const void* nccl_ids);
+  ~Engine();
+
+  int64_t submit(const int32_t* choice, const naspipe_batch* batch);
+  void drain();
+  void get_params(int block, int choice, float* dst, size_t n);
+  void set_params(int block, int choice, const float* src, size_t n);
+  void get_losses(float* dst, int64_t n);
+  void get_trace(int64_t* dst, size_t cap, size_t* n);
+  void get_stats(double* dst16);
+  void get_residency_trace(int64_t* dst, size_t cap, size_t* n);
+  void shutdown();
+
+  void check_sticky() const;
+  void set_sticky(int code, const std::string& msg);
+
+ private:
+  Engine(const Spec& spec, int D);
+  void setup_stage(int K, int dev, bool local);
+  void link_local_buffers();
+  void issue_planned();
+  void issue(const Task& t);
+  void issue_forward(StageRt& st, int64_t y, int slot);
+  void issue_backward(StageRt& st, int64_t y, int slot);
+  void version_check(const Task& t);
+  void cuda_check(const char* what);
+
+  Spec spec_;
+  int D_, W_;
+  int rank_ = -1;  // -1: single process, all stages local
+  Planner planner_;
+  std::vector<StageRt> st_;
+  std::unique_ptr<Transport> tx_;
+  std::vector<BatchRec> batches_;
+  std::vector<int32_t> stage_choice_;  // scratch
+  size_t issued_ = 0;
+  bool drained_ = false;
+  int64_t loss_cap_ = 1 << 20;
+  int sticky_code_ = 0;
+  std::string sticky_msg_;
+  // version counters per candidate (host mirror, VERSION_CHECK)
+  std::vector<int64_t> version_;
+  uint64_t version_checks_ = 0;
+  // stats
+  double h2d_bytes_ = 0, d2h_bytes_ = 0, p2p_bytes_ = 0;
+  std::vector<Task> trace_;
+  KernelTimer timer_;
+};
+
+}  // namespace naspipe

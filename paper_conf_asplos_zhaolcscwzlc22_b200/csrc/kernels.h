@@ -1,0 +1,87 @@
+// Host-side launchers of the sm_100a kernels (implemented in *.cu).  All launchers are
+// asynchronous on the given stream, deterministic (fixed tiling and reduction order, no
+// floating-point atomics) and throw naspipe::Error(NASPIPE_ECUDA) on launch failure.
+#pragma once
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+
+#include <cstddef>
+#include <cstdint>
+
+namespace naspipe {
+
+using bf16 = __nv_bfloat16;
+
+// ------------------------------------------------------------------ tcgen05 GEMM
+// C[M,N] = sum_k A[m,k] * B[n,k], bf16 operands, fp32 accumulation in TMEM.
+//   A K-major: A stored [M][lda] (k contiguous);  A MN-major: stored [K][lda] (m contiguous)
+//   B K-major: B stored [N][ldb];                 B MN-major: stored [K][ldb] (n contiguous)
+// Epilogues (row m, column n, acc = C[m,n]):
+enum GemmEpi {
+  EPI_BF16 = 0,           // out16 = bf16(acc)
+  EPI_F32 = 1,            // out32 = acc
+  EPI_BIAS_BF16 = 2,      // out16 = bf16(acc + bias[n])
+  EPI_BIAS_RESID_F32 = 3, // out32 = acc + bias[n] + resid[m,n]
+  EPI_BIAS_GELU = 4,      // z = acc + bias[n]; out16 = bf16(z); out2 = bf16(gelu_tanh(z))
+  EPI_DGELU = 5,          // out16 = bf16(acc * gelu_tanh'(aux16[m,n]))
+  EPI_SGD = 6,            // w32[m,n] -= lr * acc; w16[m,n] = bf16(w32[m,n])   (the WRITE)
+};
+struct GemmEpiParams {
+  const float* bias = nullptr;
+  const float* resid = nullptr;
+  const bf16* aux16 = nullptr;
+  void* out = nullptr;
+  bf16* out2 = nullptr;
+  float* w32 = nullptr;
+  bf16* w16 = nullptr;
+  float lr = 0.f;
+};
+void gemm_bf16_tc(cudaStream_t s, int M, int N, int K, const bf16* A, bool a_mn, int lda, const bf16* B,
+                  bool b_mn, int ldb, int epi, const GemmEpiParams& ep);
+// number of tcgen05 GEMM launches so far in this process (stats)
+uint64_t gemm_launch_count();
+
+// ------------------------------------------------------------------ attention (S <= 128)
+// qkv [B*S, 3d] bf16 (q | k | v thirds, head j = columns [j*hd, (j+1)*hd) of each third);
+// o [B*S, d] bf16; lse [B*h*S] f32 (natural log of the softmax denominator incl. scale).
+void attn_fwd(cudaStream_t s, const bf16* qkv, bf16* o, float* lse, int B, int S, int d, int h);
+// do_ [B*S, d] bf16 -> dqkv [B*S, 3d] bf16
+void attn_bwd(cudaStream_t s, const bf16* qkv, const bf16* o, const float* lse, const bf16* do_,
+              bf16* dqkv, int B, int S, int d, int h);
+
+// ------------------------------------------------------------------ LayerNorm (eps 1e-5)
+// y16 = bf16(g * (x - mu) * rstd + b); saves mean, rstd [T]
+void ln_fwd(cudaStream_t s, const float* x, const float* g, const float* b, bf16* y16, float* mean,
+            float* rstd, int T, int d);
+// dx = resid + LN'(dy); dx16 = bf16(dx) (optional); per-row-block partials of
+// dgamma, dbeta [nblk, d] and of colsum(dx) [nblk, d] (optional).
+int ln_bwd_blocks(int T);
+void ln_bwd(cudaStream_t s, const float* dy, const float* x, const float* mean, const float* rstd,
+            const float* g, const float* resid, float* dx, bf16* dx16, float* part_dg, float* part_db,
+            float* part_colsum, int T, int d);
+
+// ------------------------------------------------------------------ reductions / elementwise
+int colsum_blocks(int T);
+// per-row-block column partial sums of X [T, N] (bf16 or f32) -> part [nblk, N]
+void colsum_bf16(cudaStream_t s, const bf16* X, float* part, int T, int N);
+// f32 -> bf16 copy plus column partial sums [ln_bwd_blocks(T), N] (ln_bwd's grouping)
+void cast_colsum(cudaStream_t s, const float* X, bf16* X16, float* part, int T, int N);
+// p[i] -= lr * sum_{j < nblk} part[j * n + i]   (fixed order)
+void sgd_from_partials(cudaStream_t s, float* p, const float* part, int nblk, int n, float lr);
+// w16 = bf16(w32), n elements
+void f32_to_bf16(cudaStream_t s, const float* w32, bf16* w16, size_t n);
+// loss[0] = mean((y - t)^2); dy = 2 (y - t) / n.  part: workspace of mse_blocks(n) floats
+int mse_blocks(size_t n);
+void mse_loss(cudaStream_t s, const float* y, const float* t, float* dy, float* part, float* loss,
+              size_t n);
+// synthetic N(0,1)-like data from a counter hash (perf runs only)
+void synth_fill(cudaStream_t s, float* x, size_t n, uint64_t seed);
+
+// ------------------------------------------------------------------ MLP family (fp32)
+// y = x + tanh(x W^T + b), x [B, d]; saves h = tanh(.) for backward
+void mlp_fwd(cudaStream_t s, const float* x, const float* W, const float* b, float* y, float* h, int B, int d);
+// dz = dy (1 - h^2); dx = dy + dz W (pre-update W); then W -= lr dz^T x, b -= lr sum dz
+void mlp_bwd_sgd(cudaStream_t s, const float* x, const float* h, const float* dy, float* dx, float* W,
+                 float* b, float lr, int B, int d);
+
+}  // namespace naspipe

@@ -1,0 +1,216 @@
+// CSP planner and Belady residency planner (see planner.h).
+#include "planner.h"
+
+#include <algorithm>
+#include <limits>
+#include <map>
+
+namespace naspipe {
+
+Planner::Planner(const Spec& spec, int D)
+    : D_(D), m_(spec.m()), n_(spec.n()), W_(spec.window(D)), policy_(spec.raw.bwd_policy),
+      lambda_(spec.raw.link_latency) {
+  sob_ = spec.partition(D);
+  blocks_.assign(D, {});
+  for (int b = 0; b < m_; ++b) blocks_[sob_[b]].push_back(b);
+  spec.costs(cf_tab_, cb_tab_);
+  last_user_.assign((size_t)m_ * n_, -1);
+  use_count_.assign((size_t)m_ * n_, 0);
+  inF_.assign(D, {});
+  inB_.assign(D, {});
+  fin_.assign(D, {});
+  fin_wm_.assign(D, 0);
+  busy_.assign(D, {});
+  last_kind_.assign(D, -1);
+  stage_tasks_.assign(D, {});
+}
+
+int64_t Planner::add_subnet(const int32_t* choice) {
+  NP_REQUIRE(!finalized_, NASPIPE_ESTATE, "stream already finalised (drained)");
+  for (int b = 0; b < m_; ++b)
+    NP_REQUIRE(choice[b] >= 0 && choice[b] < n_, NASPIPE_EINVAL,
+               "choice[%d]=%d outside [0,%d)", b, choice[b], n_);
+  const int64_t y = n_subnets();
+  for (int b = 0; b < m_; ++b) {
+    const size_t key = (size_t)b * n_ + choice[b];
+    choices_.push_back(choice[b]);
+    dep_.push_back(last_user_[key]);      // dependency table (D8)
+    ver_.push_back(use_count_[key]);
+    last_user_[key] = y;
+    use_count_[key] += 1;
+  }
+  for (int K = 0; K < D_; ++K) fin_[K].push_back(0);
+  return y;
+}
+
+void Planner::reopen() {
+  NP_REQUIRE(done_, NASPIPE_ESTATE, "reopen before the plan finished");
+  finalized_ = false;
+  done_ = false;
+  phase_ = 0;
+}
+
+std::vector<int64_t> Planner::deps(int64_t y, int K) const {
+  std::vector<int64_t> out;
+  for (int b : blocks_[K]) {
+    const int64_t d = dep(y, b);
+    if (d >= 0) out.push_back(d);
+  }
+  std::sort(out.begin(), out.end());
+  out.erase(std::unique(out.begin(), out.end()), out.end());
+  return out;
+}
+
+int64_t Planner::cost(int K, int64_t y, int kind) const {
+  int64_t s = 0;
+  const auto& tab = kind == 0 ? cf_tab_ : cb_tab_;
+  for (int b : blocks_[K]) s += tab[(size_t)b * n_ + choice(y, b)];
+  return std::max<int64_t>(1, s);
+}
+
+bool Planner::admissible(int K, int64_t y) const {
+  for (int b : blocks_[K]) {
+    const int64_t d = dep(y, b);
+    if (d >= 0 && !fin_[K][d]) return false;
+  }
+  return true;
+}
+
+void Planner::start(int K, int kind, int64_t y) {
+  busy_[K] = {true, t_ + cost(K, y, kind), kind, y};
+  last_kind_[K] = kind;
+  stage_tasks_[K].push_back((int64_t)tasks_.size());
+  tasks_.push_back({t_, K, kind, y});
+}
+
+void Planner::advance() {
+  while (!done_) {
+    if (phase_ == 0) {
+      // (1) completions at t, then deliveries with time <= t
+      for (int K = 0; K < D_; ++K) {
+        Busy& bz = busy_[K];
+        if (!bz.on || bz.end != t_) continue;
+        bz.on = false;
+        if (bz.kind == 0) {
+          if (K < D_ - 1) deliveries_.push_back({t_ + lambda_, 0, K + 1, bz.y});
+          else inB_[K].insert(bz.y);
+        } else {
+          fin_[K][bz.y] = 1;
+          while (fin_wm_[K] < (int64_t)fin_[K].size() && fin_[K][fin_wm_[K]]) ++fin_wm_[K];
+          if (K > 0) deliveries_.push_back({t_ + lambda_, 1, K - 1, bz.y});
+          else ++done0_;
+        }
+      }
+      std::vector<Delivery> keep;
+      for (auto& dv : deliveries_) {
+        if (dv.time <= t_) (dv.to_B ? inB_ : inF_)[dv.K].insert(dv.y);
+        else keep.push_back(dv);
+      }
+      deliveries_.swap(keep);
+      phase_ = 1;
+    }
+    // the stream may have been finalised while suspended at this tick
+    if (finalized_ && done0_ == n_subnets()) {
+      done_ = true;
+      makespan_ = t_;
+      return;
+    }
+    // (2) stage-0 source under the window: y < wm0 + W (reading A7)
+    const int64_t N = n_subnets();
+    const int64_t wm0 = fin_wm_[0];
+    const int64_t hi = wm0 + W_;
+    if (!finalized_ && N < hi) return;  // streaming rule: wait for more subnets
+    const int64_t lim = std::min(hi, N);
+    for (; src_next_ < lim; ++src_next_) inF_[0].insert(src_next_);
+    // (3) decisions on idle stages
+    for (int K = 0; K < D_; ++K) {
+      if (busy_[K].on) continue;
+      int64_t first = -1;
+      for (int64_t y : inF_[K])
+        if (admissible(K, y)) { first = y; break; }  // ascending id (reading A6)
+      if (policy_ == 1 && last_kind_[K] == 1 && first >= 0) {
+        inF_[K].erase(first);
+        start(K, 0, first);
+      } else if (!inB_[K].empty()) {                  // backward first, lowest id (A5)
+        const int64_t y = *inB_[K].begin();
+        inB_[K].erase(inB_[K].begin());
+        start(K, 1, y);
+      } else if (first >= 0) {
+        inF_[K].erase(first);
+        start(K, 0, first);
+      }
+    }
+    // (4) advance time
+    int64_t nxt = std::numeric_limits<int64_t>::max();
+    for (auto& bz : busy_) if (bz.on) nxt = std::min(nxt, bz.end);
+    for (auto& dv : deliveries_) nxt = std::min(nxt, dv.time);
+    NP_REQUIRE(nxt != std::numeric_limits<int64_t>::max(), NASPIPE_EINTERNAL,
+               "CSP planner stalled at tick %lld", (long long)t_);
+    t_ = nxt;
+    phase_ = 0;
+  }
+}
+
+ResidencyPlan plan_residency(int K, const std::vector<std::vector<int64_t>>& uses,
+                             const std::vector<int>& kinds, const std::vector<int64_t>& bytes,
+                             int64_t budget, int L) {
+  ResidencyPlan out;
+  const int64_t T = (int64_t)uses.size();
+  const int64_t NEVER = std::numeric_limits<int64_t>::max();
+  std::map<int64_t, std::vector<int64_t>> when;  // uid -> task indices using it
+  for (int64_t i = 0; i < T; ++i)
+    for (int64_t u : uses[i]) when[u].push_back(i);
+  auto next_use = [&](int64_t u, int64_t i) -> int64_t {
+    auto& v = when[u];
+    auto it = std::lower_bound(v.begin(), v.end(), i);
+    return it == v.end() ? NEVER : *it;
+  };
+  auto size_of = [&](const std::set<int64_t>& s) {
+    int64_t t = 0;
+    for (int64_t u : s) t += bytes[u];
+    return t;
+  };
+  std::set<int64_t> resident, dirty;
+  for (int64_t i = 0; i < T; ++i) {
+    std::set<int64_t> need(uses[i].begin(), uses[i].end());
+    NP_REQUIRE(size_of(need) <= budget, NASPIPE_EBUDGET,
+               "stage %d task %lld needs %lld bytes > budget %lld", K, (long long)i,
+               (long long)size_of(need), (long long)budget);
+    for (int depth = 2; depth <= L; ++depth) {
+      if (i + depth - 1 >= T) break;
+      std::set<int64_t> cand = need;
+      cand.insert(uses[i + depth - 1].begin(), uses[i + depth - 1].end());
+      if (size_of(cand) > budget) break;
+      need.swap(cand);
+    }
+    for (;;) {
+      std::set<int64_t> uni = resident;
+      uni.insert(need.begin(), need.end());
+      if (size_of(uni) <= budget) break;
+      int64_t victim = -1, far = -1;
+      for (int64_t u : resident) {  // ascending uid: ties keep the lowest
+        if (need.count(u)) continue;
+        const int64_t nu = next_use(u, i);
+        if (nu > far) { far = nu; victim = u; }
+      }
+      resident.erase(victim);
+      out.events.push_back({K, i, 1, victim});
+      if (dirty.count(victim)) {
+        out.writebacks.push_back({i, victim});
+        dirty.erase(victim);
+      }
+    }
+    std::vector<std::pair<int64_t, int64_t>> loads;
+    for (int64_t u : need)
+      if (!resident.count(u)) loads.push_back({next_use(u, i), u});
+    std::sort(loads.begin(), loads.end());
+    for (auto& lu : loads) {
+      resident.insert(lu.second);
+      out.events.push_back({K, i, 0, lu.second});
+    }
+    if (kinds[i] == 1) dirty.insert(uses[i].begin(), uses[i].end());
+  }
+  return out;
+}
+
+}  // namespace naspipe

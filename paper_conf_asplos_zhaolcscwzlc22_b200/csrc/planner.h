@@ -1,0 +1,98 @@
+// Deterministic CSP planner: dependency table over (block, choice) keyed by chronological
+// subnet order, and a logical-time discrete-event schedule of Alg.1 + Alg.2 (PAPER.md
+// P:L170-221) under readings A5-A8.  Streaming: subnets are appended one at a
+// time; a stage-0 decision at tick t is taken only once every y < wm0 + W has been
+// submitted or the stream has been finalised, so the plan never depends on submit pace.
+#pragma once
+#include <cstdint>
+#include <deque>
+#include <set>
+#include <vector>
+
+#include "spec.h"
+
+namespace naspipe {
+
+struct Task {
+  int64_t t;    // start tick
+  int32_t K;    // stage
+  int32_t kind; // 0 = F, 1 = B
+  int64_t y;    // subnet sequence id
+};
+
+class Planner {
+ public:
+  Planner(const Spec& spec, int D);
+
+  int D() const { return D_; }
+  const std::vector<int32_t>& stage_of_block() const { return sob_; }
+  const std::vector<int>& blocks_of(int K) const { return blocks_[K]; }
+
+  // Append subnet (choice vector of length m).  Returns its id.
+  int64_t add_subnet(const int32_t* choice);
+  // Fix N = number of added subnets.
+  void finalize() { finalized_ = true; }
+  // After done(): accept more subnets; the continuation starts at the previous makespan with
+  // every earlier subnet finished (a drain is a pipeline flush).
+  void reopen();
+  // Advance the simulation as far as allowed; newly planned tasks are appended to tasks().
+  void advance();
+  bool done() const { return done_; }
+  int64_t makespan() const { return makespan_; }
+  int64_t n_subnets() const { return (int64_t)choices_.size() / m_; }
+
+  const std::vector<Task>& tasks() const { return tasks_; }
+  // per-stage planned order: indices into tasks()
+  const std::vector<std::vector<int64_t>>& stage_tasks() const { return stage_tasks_; }
+
+  int32_t choice(int64_t y, int b) const { return choices_[(size_t)y * m_ + b]; }
+  const int32_t* choice_row(int64_t y) const { return choices_.data() + (size_t)y * m_; }
+  // dependency table: dep[y][b] = latest x < y with c_x[b] == c_y[b], else -1
+  int64_t dep(int64_t y, int b) const { return dep_[(size_t)y * m_ + b]; }
+  // version of candidate (b, c_y[b]) seen by subnet y = #{x < y : c_x[b] == c_y[b]}
+  int64_t version(int64_t y, int b) const { return ver_[(size_t)y * m_ + b]; }
+  std::vector<int64_t> deps(int64_t y, int K) const;
+  int64_t cost(int K, int64_t y, int kind) const;
+
+ private:
+  bool admissible(int K, int64_t y) const;
+  void start(int K, int kind, int64_t y);
+
+  int D_, m_, n_, W_, policy_, lambda_;
+  std::vector<int32_t> sob_;
+  std::vector<std::vector<int>> blocks_;
+  std::vector<int32_t> cf_tab_, cb_tab_;  // [m*n]
+
+  std::vector<int32_t> choices_;   // [N*m]
+  std::vector<int64_t> dep_, ver_; // [N*m]
+  std::vector<int64_t> last_user_, use_count_;  // [m*n]
+
+  // simulation state
+  struct Busy { bool on = false; int64_t end = 0; int kind = 0; int64_t y = 0; };
+  struct Delivery { int64_t time; int to_B; int K; int64_t y; };
+  std::vector<std::set<int64_t>> inF_, inB_;
+  std::vector<std::vector<uint8_t>> fin_;  // fin_[K][y]
+  std::vector<int64_t> fin_wm_;            // all y < fin_wm_[K] finished on K
+  std::vector<Busy> busy_;
+  std::vector<int> last_kind_;
+  std::vector<Delivery> deliveries_;
+  int64_t t_ = 0, src_next_ = 0, done0_ = 0, makespan_ = -1;
+  int phase_ = 0;
+  bool finalized_ = false, done_ = false;
+
+  std::vector<Task> tasks_;
+  std::vector<std::vector<int64_t>> stage_tasks_;
+};
+
+// Belady residency over one stage's planned order (reading A9).
+struct ResidencyEvent { int32_t K; int64_t i; int32_t op; int64_t uid; };  // op 0 LOAD 1 EVICT
+struct ResidencyPlan {
+  std::vector<ResidencyEvent> events;
+  std::vector<std::pair<int64_t, int64_t>> writebacks;  // (task index, uid)
+};
+// uses[i] = sorted uids used by task i; kinds[i] = 0/1; bytes[uid]; budget > 0.
+ResidencyPlan plan_residency(int K, const std::vector<std::vector<int64_t>>& uses,
+                             const std::vector<int>& kinds, const std::vector<int64_t>& bytes,
+                             int64_t budget, int L);
+
+}  // namespace naspipe

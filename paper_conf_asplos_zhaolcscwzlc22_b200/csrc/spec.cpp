@@ -1,0 +1,245 @@
+// Spec validation, layouts, analytic costs, balanced partition (reading A12) and the
+// counter-hash initialiser (reading A21).
+#include "spec.h"
+
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <limits>
+
+namespace naspipe {
+
+std::string strfmt(const char* fmt, ...) {
+  char buf[1024];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  return buf;
+}
+
+uint64_t splitmix64(uint64_t x) {
+  uint64_t z = x + 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
+Spec::Spec(const naspipe_supernet_spec* s) {
+  NP_REQUIRE(s != nullptr, NASPIPE_EINVAL, "spec is NULL");
+  NP_REQUIRE(s->abi_version == NASPIPE_ABI_VERSION, NASPIPE_EINVAL, "abi_version %d != %d",
+             s->abi_version, NASPIPE_ABI_VERSION);
+  raw = *s;
+  NP_REQUIRE(raw.family == NASPIPE_MLP || raw.family == NASPIPE_TRANSFORMER, NASPIPE_EINVAL,
+             "unsupported family %d", raw.family);
+  NP_REQUIRE(raw.n_blocks >= 1 && raw.n_blocks <= 4096, NASPIPE_EINVAL, "n_blocks %d", raw.n_blocks);
+  NP_REQUIRE(raw.n_choices >= 1 && raw.n_choices <= 4096, NASPIPE_EINVAL, "n_choices %d",
+             raw.n_choices);
+  NP_REQUIRE(raw.batch >= 1, NASPIPE_EINVAL, "batch %d", raw.batch);
+  NP_REQUIRE(std::isfinite(raw.lr), NASPIPE_EINVAL, "lr not finite");
+  NP_REQUIRE(raw.window >= 0 && raw.lookahead >= 0 && raw.bwd_policy >= 0 && raw.bwd_policy <= 1 &&
+                 raw.link_latency >= 0 && raw.hbm_weight_budget_bytes >= 0,
+             NASPIPE_EINVAL, "bad window/lookahead/policy/latency/budget");
+  const int n = raw.n_choices, m = raw.n_blocks;
+  if (raw.family == NASPIPE_MLP) {
+    NP_REQUIRE(raw.width >= 1 && raw.width <= 1024, NASPIPE_EINVAL, "width %d", raw.width);
+    NP_REQUIRE(raw.compute_dtype == NASPIPE_FP32, NASPIPE_EINVAL, "MLP computes in fp32");
+  } else {
+    NP_REQUIRE(raw.compute_dtype == NASPIPE_BF16, NASPIPE_EINVAL, "transformer computes in bf16");
+    NP_REQUIRE(raw.d_model >= 16 && raw.d_model % 16 == 0, NASPIPE_EINVAL,
+               "d_model %d must be a positive multiple of 16", raw.d_model);
+    NP_REQUIRE(raw.seq_len >= 1 && raw.seq_len <= 128, NASPIPE_EINVAL, "seq_len %d (1..128)",
+               raw.seq_len);
+    NP_REQUIRE(raw.choice_heads && raw.choice_ffn, NASPIPE_EINVAL, "choice_heads/choice_ffn NULL");
+    heads.assign(raw.choice_heads, raw.choice_heads + n);
+    ffn.assign(raw.choice_ffn, raw.choice_ffn + n);
+    for (int c = 0; c < n; ++c) {
+      NP_REQUIRE(heads[c] >= 1 && raw.d_model % heads[c] == 0, NASPIPE_EINVAL,
+                 "heads[%d]=%d must divide d_model", c, heads[c]);
+      const int hd = raw.d_model / heads[c];
+      NP_REQUIRE(hd % 16 == 0 && hd <= 128, NASPIPE_EINVAL, "head dim %d must be 16..128, %%16", hd);
+      NP_REQUIRE(ffn[c] >= 16 && ffn[c] % 16 == 0, NASPIPE_EINVAL, "ffn[%d]=%d must be a multiple of 16",
+                 c, ffn[c]);
+    }
+  }
+  if (raw.stage_of_block) {
+    stage_of_block.assign(raw.stage_of_block, raw.stage_of_block + m);
+    has_partition = true;
+  }
+  NP_REQUIRE((raw.cost_fwd == nullptr) == (raw.cost_bwd == nullptr), NASPIPE_EINVAL,
+             "cost_fwd and cost_bwd must both be given or both NULL");
+  if (raw.cost_fwd) {
+    cost_fwd.assign(raw.cost_fwd, raw.cost_fwd + (size_t)m * n);
+    cost_bwd.assign(raw.cost_bwd, raw.cost_bwd + (size_t)m * n);
+    for (size_t i = 0; i < cost_fwd.size(); ++i)
+      NP_REQUIRE(cost_fwd[i] >= 0 && cost_bwd[i] >= 0, NASPIPE_EINVAL, "negative cost");
+    has_costs = true;
+  }
+  raw.choice_heads = heads.empty() ? nullptr : heads.data();
+  raw.choice_ffn = ffn.empty() ? nullptr : ffn.data();
+  raw.stage_of_block = has_partition ? stage_of_block.data() : nullptr;
+  raw.cost_fwd = has_costs ? cost_fwd.data() : nullptr;
+  raw.cost_bwd = has_costs ? cost_bwd.data() : nullptr;
+}
+
+Spec::Spec(const Spec& o)
+    : raw(o.raw), heads(o.heads), ffn(o.ffn), stage_of_block(o.stage_of_block),
+      cost_fwd(o.cost_fwd), cost_bwd(o.cost_bwd), has_partition(o.has_partition),
+      has_costs(o.has_costs) {
+  raw.choice_heads = heads.empty() ? nullptr : heads.data();
+  raw.choice_ffn = ffn.empty() ? nullptr : ffn.data();
+  raw.stage_of_block = has_partition ? stage_of_block.data() : nullptr;
+  raw.cost_fwd = has_costs ? cost_fwd.data() : nullptr;
+  raw.cost_bwd = has_costs ? cost_bwd.data() : nullptr;
+}
+
+size_t Spec::sample_elems() const {
+  return family() == NASPIPE_MLP ? (size_t)raw.width : (size_t)raw.seq_len * raw.d_model;
+}
+
+int Spec::rows() const { return family() == NASPIPE_MLP ? raw.batch : raw.batch * raw.seq_len; }
+
+TfOffsets Spec::tf_offsets(int c) const {
+  const size_t d = raw.d_model, f = ffn[c];
+  TfOffsets o{};
+  size_t off = 0;
+  auto take = [&](size_t n) { size_t r = off; off += n; return r; };
+  o.Wqkv = take(3 * d * d); o.bqkv = take(3 * d);
+  o.Wo = take(d * d); o.bo = take(d);
+  o.ln1g = take(d); o.ln1b = take(d);
+  o.W1 = take(f * d); o.b1 = take(f);
+  o.W2 = take(d * f); o.b2 = take(d);
+  o.ln2g = take(d); o.ln2b = take(d);
+  o.total = off;
+  return o;
+}
+
+std::vector<Segment> Spec::segments(int b, int c) const {
+  (void)b;
+  std::vector<Segment> s;
+  if (family() == NASPIPE_MLP) {
+    const size_t d = raw.width;
+    s.push_back({0, d * d, 0, (int)d});
+    s.push_back({d * d, d, 0, (int)d});
+    return s;
+  }
+  const TfOffsets o = tf_offsets(c);
+  const size_t d = raw.d_model, f = ffn[c];
+  s.push_back({o.Wqkv, 3 * d * d, 0, (int)d});
+  s.push_back({o.bqkv, 3 * d, 0, (int)d});
+  s.push_back({o.Wo, d * d, 0, (int)d});
+  s.push_back({o.bo, d, 0, (int)d});
+  s.push_back({o.ln1g, d, 1, 0});
+  s.push_back({o.ln1b, d, 2, 0});
+  s.push_back({o.W1, f * d, 0, (int)d});
+  s.push_back({o.b1, f, 0, (int)d});
+  s.push_back({o.W2, d * f, 0, (int)f});
+  s.push_back({o.b2, d, 0, (int)f});
+  s.push_back({o.ln2g, d, 1, 0});
+  s.push_back({o.ln2b, d, 2, 0});
+  return s;
+}
+
+size_t Spec::param_count(int b, int c) const {
+  size_t t = 0;
+  for (auto& s : segments(b, c)) t += s.size;
+  return t;
+}
+
+void Spec::init_params(int b, int c, float* dst) const {
+  const uint64_t uid = (uint64_t)b * (uint64_t)n() + (uint64_t)c;
+  for (auto& s : segments(b, c)) {
+    if (s.kind == 1) { std::fill(dst + s.offset, dst + s.offset + s.size, 1.0f); continue; }
+    if (s.kind == 2) { std::fill(dst + s.offset, dst + s.offset + s.size, 0.0f); continue; }
+    const float bound = 1.0f / std::sqrt((float)s.fan_in);
+    for (size_t k = 0; k < s.size; ++k) {
+      const uint64_t i = s.offset + k;
+      const uint64_t z = splitmix64(raw.init_seed ^ (uid * 0x9E3779B97F4A7C15ull + i));
+      const float u = (float)(z >> 40) * 5.9604644775390625e-08f;  // 2^-24
+      const float two_u_m1 = 2.0f * u - 1.0f;                       // exact
+      dst[s.offset + k] = bound * two_u_m1;
+    }
+  }
+}
+
+// Analytic per-(block, choice) tick table (1 tick = 1 us), SURVEY §8c "Cost tables":
+// cf = ceil(max(flops / (0.6 * 1378e12), bytes / (0.8 * 6544e9))), cb = ceil(2 * tf + update).
+void Spec::default_costs(int32_t* cf, int32_t* cb) const {
+  const double peak = 0.6 * 1378e12, bw = 0.8 * 6544e9;
+  for (int b = 0; b < m(); ++b)
+    for (int c = 0; c < n(); ++c) {
+      double flops, bytes;
+      const double P = (double)param_count(b, c);
+      if (family() == NASPIPE_MLP) {
+        const double d = raw.width, T = raw.batch;
+        flops = 2.0 * T * d * d;
+        bytes = 4.0 * (3.0 * T * d + d * d + d);
+      } else {
+        const double d = raw.d_model, f = ffn[c], T = (double)raw.batch * raw.seq_len,
+                     S = raw.seq_len;
+        flops = 2.0 * T * (4.0 * d * d + 2.0 * d * f) + 4.0 * T * S * d;
+        bytes = 2.0 * T * (12.0 * d + 3.0 * f) + 2.0 * P;
+      }
+      const double tf = std::max(flops / peak, bytes / bw) * 1e6;
+      const double tb = 2.0 * tf + 10.0 * P / bw * 1e6;
+      cf[b * n() + c] = (int32_t)std::max(1.0, std::ceil(tf));
+      cb[b * n() + c] = (int32_t)std::max(1.0, std::ceil(tb));
+    }
+}
+
+void Spec::costs(std::vector<int32_t>& cf, std::vector<int32_t>& cb) const {
+  if (has_costs) { cf = cost_fwd; cb = cost_bwd; return; }
+  cf.assign((size_t)m() * n(), 0);
+  cb.assign((size_t)m() * n(), 0);
+  default_costs(cf.data(), cb.data());
+}
+
+void Spec::validate_stages(int D) const {
+  NP_REQUIRE(D >= 1 && D <= m(), NASPIPE_EINVAL, "n_stages %d not in 1..n_blocks=%d", D, m());
+  if (!has_partition) return;
+  NP_REQUIRE(stage_of_block[0] == 0 && stage_of_block[m() - 1] == D - 1, NASPIPE_EINVAL,
+             "stage_of_block must start at 0 and end at n_stages-1");
+  for (int b = 1; b < m(); ++b)
+    NP_REQUIRE(stage_of_block[b] == stage_of_block[b - 1] || stage_of_block[b] == stage_of_block[b - 1] + 1,
+               NASPIPE_EINVAL, "stage_of_block must be contiguous and non-decreasing");
+}
+
+// Balanced contiguous partition: minimise the max stage weight, weight(b) = sum_c (cf+cb);
+// ties -> lexicographically smallest split points (reading A12).  Exact integer DP.
+std::vector<int32_t> Spec::partition(int D) const {
+  validate_stages(D);
+  if (has_partition) return stage_of_block;
+  std::vector<int32_t> cf, cb;
+  costs(cf, cb);
+  const int M = m();
+  std::vector<int64_t> pre(M + 1, 0);
+  for (int b = 0; b < M; ++b) {
+    int64_t w = 0;
+    for (int c = 0; c < n(); ++c) w += (int64_t)cf[b * n() + c] + cb[b * n() + c];
+    pre[b + 1] = pre[b] + w;
+  }
+  auto seg = [&](int i, int e) { return pre[e] - pre[i]; };
+  const int64_t INF = std::numeric_limits<int64_t>::max();
+  // g[k][i]: min over splits of blocks [i, M) into k non-empty stages of the max weight
+  std::vector<std::vector<int64_t>> g(D + 1, std::vector<int64_t>(M + 1, INF));
+  for (int i = 0; i < M; ++i) g[1][i] = seg(i, M);
+  for (int k = 2; k <= D; ++k)
+    for (int i = 0; i + k <= M; ++i)
+      for (int e = i + 1; e + (k - 1) <= M; ++e)
+        g[k][i] = std::min(g[k][i], std::max(seg(i, e), g[k - 1][e]));
+  const int64_t best = g[D][0];
+  std::vector<int32_t> sob(M, 0);
+  int start = 0;
+  for (int k = 0; k < D - 1; ++k) {
+    const int r = D - k;  // stages left including this one
+    int e = start + 1;
+    for (; e + (r - 1) <= M; ++e)
+      if (seg(start, e) <= best && g[r - 1][e] <= best) break;
+    for (int b = start; b < e; ++b) sob[b] = k;
+    start = e;
+  }
+  for (int b = start; b < M; ++b) sob[b] = D - 1;
+  return sob;
+}
+
+}  // namespace naspipe

@@ -1,0 +1,60 @@
+// Supernet specification: validated deep copy of naspipe_supernet_spec, parameter layouts,
+// the analytic cost table, the balanced partition and the counter-hash initialiser.
+#pragma once
+#include <cstddef>
+#include <cstdint>
+#include <vector>
+
+#include "common.h"
+
+namespace naspipe {
+
+// One tensor of a candidate's packed parameter vector.
+struct Segment {
+  size_t offset, size;
+  int kind;      // 0 = uniform(+-1/sqrt(fan_in)), 1 = ones, 2 = zeros
+  int fan_in;
+};
+
+// Offsets (in floats) of the transformer candidate tensors in the packed vector
+// (packing order of include/naspipe.h).
+struct TfOffsets {
+  size_t Wqkv, bqkv, Wo, bo, ln1g, ln1b, W1, b1, W2, b2, ln2g, ln2b, total;
+};
+
+struct Spec {
+  naspipe_supernet_spec raw{};  // scalar fields; pointer fields re-pointed into vectors below
+  std::vector<int32_t> heads, ffn, stage_of_block, cost_fwd, cost_bwd;
+  bool has_partition = false, has_costs = false;
+
+  explicit Spec(const naspipe_supernet_spec* s);
+  Spec(const Spec& o);
+
+  int family() const { return raw.family; }
+  int m() const { return raw.n_blocks; }
+  int n() const { return raw.n_choices; }
+  int B() const { return raw.batch; }
+  int window(int D) const { return raw.window > 0 ? raw.window : 4 * D; }
+  int lookahead() const { return raw.lookahead > 0 ? raw.lookahead : 2; }
+  // elements of one sample of input / output (the residual stream width per batch row)
+  size_t sample_elems() const;
+  size_t batch_elems() const { return (size_t)B() * sample_elems(); }
+  int rows() const;  // GEMM rows T: B (MLP) or B*S (transformer)
+  int d() const { return family() == NASPIPE_MLP ? raw.width : raw.d_model; }
+
+  std::vector<Segment> segments(int b, int c) const;
+  size_t param_count(int b, int c) const;
+  TfOffsets tf_offsets(int c) const;
+  void init_params(int b, int c, float* dst) const;
+
+  void default_costs(int32_t* cf, int32_t* cb) const;
+  // cost tables actually used by the planner (spec's or default), [m*n]
+  void costs(std::vector<int32_t>& cf, std::vector<int32_t>& cb) const;
+  std::vector<int32_t> partition(int D) const;
+  void validate_stages(int D) const;
+};
+
+// splitmix64 counter hash (reading A21)
+uint64_t splitmix64(uint64_t x);
+
+}  // namespace naspipe

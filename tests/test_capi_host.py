@@ -1,0 +1,152 @@
+"""Host-side C ABI tests (no GPU): the library loads and exports every declared symbol; the
+C++ planner, dependency table, partition, residency planner and initialiser agree
+bit-exactly with the oracle (SURVEY §4 tier T1)."""
+import os
+import re
+
+import numpy as np
+import pytest
+
+import synth
+from oracle import csp, residency, train
+
+npipe = pytest.importorskip("paper_conf_asplos_zhaolcscwzlc22_b200")
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def test_exports_every_declared_symbol():
+    hdr = open(os.path.join(ROOT, "include", "naspipe.h")).read()
+    declared = set(re.findall(r"^(?:int|void|const char\s*\*)\s+(naspipe_[a-z_0-9]+)\s*\(", hdr, re.M))
+    assert declared, "no declarations parsed"
+    for name in sorted(declared):
+        assert hasattr(npipe.lib, name), name
+    assert declared == set(npipe.EXPORTED_SYMBOLS)
+    assert npipe.naspipe_abi_version() == 1
+
+
+@pytest.mark.parametrize("name", ["toy", "tiny_transformer", "transformer"])
+def test_init_params_match_shared_hash(name):
+    cfg = synth.get_config(name)
+    spec = npipe.Spec(cfg)
+    n = cfg["n_choices"]
+    for (b, c) in [(0, 0), (1, n - 1), (cfg["n_blocks"] - 1, n // 2)]:
+        got = npipe.naspipe_init_params(spec, b, c)
+        segs = [(int(np.prod(s)), kind, fan) for _, s, kind, fan in train.candidate_layout(cfg, b, c)]
+        assert npipe.naspipe_param_count(spec, b, c) == sum(s for s, _, _ in segs)
+        if name == "transformer" and (b, c) != (0, 0):
+            continue  # one full-size candidate is enough (12.6 M floats)
+        ref = synth.init_packed(cfg["init_seed"], b * n + c, segs)
+        assert np.array_equal(got.view(np.uint32), ref.view(np.uint32)), (b, c)
+
+
+def _random_case(seed):
+    rng = np.random.default_rng(seed)
+    N = int(rng.integers(3, 40))
+    m = int(rng.integers(1, 9))
+    n = int(rng.integers(1, 6))
+    D = int(rng.integers(1, m + 1))
+    W = int(rng.integers(1, 4 * D + 3))
+    lam = int(rng.integers(0, 3))
+    policy = int(rng.integers(0, 2))
+    cf = rng.integers(0, 5, size=(m, n)).astype(np.int32)
+    cb = rng.integers(0, 7, size=(m, n)).astype(np.int32)
+    ch = synth.sample_choices(N, m, n, seed)
+    cfg = dict(family="mlp", n_blocks=m, n_choices=n, batch=2, width=8, lr=0.05, compute_dtype="fp32",
+               window=W, link_latency=lam, bwd_policy=policy, cost_fwd=cf, cost_bwd=cb)
+    return cfg, ch, D
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_planner_matches_oracle_bit_exact(seed):
+    cfg, ch, D = _random_case(seed)
+    spec = npipe.Spec(cfg)
+    sob = npipe.naspipe_partition(spec, D)
+    wts = csp.block_partition_cost(cfg["cost_fwd"], cfg["cost_bwd"])
+    np.testing.assert_array_equal(sob, csp.balanced_partition(wts, D))
+    plan = npipe.naspipe_plan(spec, D, ch)
+    tf, tb = csp.task_costs(ch, sob, cfg["cost_fwd"], cfg["cost_bwd"], D)
+    ref = csp.simulate_csp(ch, sob, D, cfg["window"], tf, tb, lam=cfg["link_latency"], policy=cfg["bwd_policy"])
+    got = [tuple(int(v) for v in row) for row in plan.trace()]
+    assert got == [tuple(r) for r in ref["trace"]]
+    assert plan.makespan() == ref["makespan"]
+    for y in range(len(ch)):
+        for K in range(D):
+            assert plan.deps(y, K) == sorted(csp.deps(ch, sob, y, K))
+
+
+def test_worked_example_through_c_abi():
+    ch = np.array([[0, 0], [1, 0], [0, 1], [1, 1]])
+    cfg = dict(family="mlp", n_blocks=2, n_choices=2, batch=2, width=8, compute_dtype="fp32", window=4,
+               cost_fwd=np.ones((2, 2)), cost_bwd=np.full((2, 2), 2), stage_of_block=[0, 1])
+    plan = npipe.naspipe_plan(npipe.Spec(cfg), 2, ch)
+    assert plan.makespan() == 15
+    s0 = [("F" if k == 0 else "B") + f"{y}@{t}" for t, K, k, y in plan.trace() if K == 0]
+    assert s0 == ["F0@0", "F1@1", "B0@4", "F2@6", "B1@7", "F3@9", "B2@10", "B3@13"]
+    # residency worked example 2 needs unit candidate sizes: check ordering semantics via
+    # the oracle on the library's own plan at D = 1 with bytes = 4 * params (all equal)
+    plan1 = npipe.naspipe_plan(npipe.Spec(dict(cfg, stage_of_block=[0, 0])), 1, ch)
+    P = 4 * npipe.naspipe_param_count(npipe.Spec(cfg), 0, 0)
+    ev, wb = plan1.residency(0, 3 * P, 2)
+    got = [("LOAD" if op == 0 else "EVICT") + f"({i},{u})" for _, i, op, u in ev]
+    assert got == ["LOAD(0,0)", "LOAD(0,2)", "LOAD(1,1)", "EVICT(4,2)", "LOAD(4,3)"]
+    assert wb == 1
+
+
+@pytest.mark.parametrize("seed", range(15))
+def test_residency_matches_oracle(seed):
+    cfg, ch, D = _random_case(100 + seed)
+    cfg = dict(cfg, family="transformer", d_model=16, seq_len=16, compute_dtype="bf16",
+               choice_heads=[1] * cfg["n_choices"],
+               choice_ffn=[16 * (1 + c % 3) for c in range(cfg["n_choices"])])
+    spec = npipe.Spec(cfg)
+    plan = npipe.naspipe_plan(spec, D, ch)
+    sob = npipe.naspipe_partition(spec, D)
+    tr = plan.trace()
+    n, m = cfg["n_choices"], cfg["n_blocks"]
+    nbytes = {b * n + c: 4 * npipe.naspipe_param_count(spec, b, c) for b in range(m) for c in range(n)}
+    rng = np.random.default_rng(seed)
+    for K in range(D):
+        order = [(int(k), int(y)) for t, KK, k, y in tr if KK == K]
+        blocks = [b for b in range(m) if sob[b] == K]
+        uses = residency.stage_uses(order, ch, blocks, n)
+        need = max(sum(nbytes[u] for u in us) for us in uses)
+        budget = int(need * rng.uniform(1.0, 3.0))
+        for depth in (1, 2, 3):
+            ref = residency.simulate_residency(uses, [k for k, _ in order], nbytes, budget, L=depth)
+            ev, wb = plan.residency(K, budget, depth)
+            got = [("LOAD" if op == 0 else "EVICT", int(i), int(u)) for _, i, op, u in ev]
+            assert got == ref["events"], (K, depth)
+            assert wb == len(ref["writebacks"])
+
+
+def test_budget_error_and_invalid_args():
+    cfg = dict(family="mlp", n_blocks=2, n_choices=2, batch=2, width=8, compute_dtype="fp32")
+    spec = npipe.Spec(cfg)
+    plan = npipe.naspipe_plan(spec, 1, np.array([[0, 0], [1, 1]]))
+    P = 4 * npipe.naspipe_param_count(spec, 0, 0)
+    with pytest.raises(npipe.NaspipeError) as e:
+        plan.residency(0, P, 2)            # one task needs 2 candidates
+    assert e.value.code == -6
+    with pytest.raises(npipe.NaspipeError) as e:
+        npipe.naspipe_plan(spec, 1, np.array([[0, 2]]))   # choice out of range
+    assert e.value.code == -1
+    with pytest.raises(npipe.NaspipeError):
+        npipe.naspipe_plan(spec, 3, np.array([[0, 0]]))   # more stages than blocks
+    bad = npipe.Spec(dict(cfg, family="transformer", d_model=24, seq_len=8, compute_dtype="bf16",
+                          choice_heads=[1, 1], choice_ffn=[16, 16]))   # d_model % 16 != 0
+    with pytest.raises(npipe.NaspipeError) as e:
+        npipe.naspipe_param_count(bad, 0, 0)
+    assert e.value.code == -1
+
+
+def test_default_costs_and_partition_of_real_configs():
+    for name, D in [("transformer", 8), ("large_transformer", 8), ("toy", 2)]:
+        cfg = synth.get_config(name)
+        spec = npipe.Spec(cfg)
+        cf, cb = npipe.naspipe_default_costs(spec)
+        assert (cf >= 1).all() and (cb >= cf).all()
+        sob = npipe.naspipe_partition(spec, D)
+        assert sob[0] == 0 and sob[-1] == D - 1 and np.all(np.diff(sob) >= 0)
+        if name == "toy":
+            assert list(sob) == [0, 0, 1, 1]

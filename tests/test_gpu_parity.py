@@ -1,0 +1,163 @@
+"""End-to-end parity of the CUDA path against the sequential CPU oracle (SURVEY §4 tier T3),
+through the C ABI (naspipe_create / submit / drain / get_params).
+
+Bars (BASELINE.json north_star, reading A15):
+* parameters: max over candidates of max|gpu - ref| / max|ref| <= 1e-3 after 1 step,
+  <= 1e-2 after 100 steps;  diagnostic on the update Delta = theta_t - theta_0 (the params
+  alone are dominated by theta_0), normwise per tensor: <= 1e-5 (fp32 MLP), <= 1e-1 (bf16
+  transformer; derivation in DESIGN.md "Tolerances");
+* schedule decisions bit-exact: the executed task trace equals the oracle CSP schedule;
+* two GPU runs bitwise identical; runs at different stage counts D bitwise identical
+  (Table 3, artifact P:L557-561) — all stages of a run share one GPU here.
+"""
+import numpy as np
+import pytest
+
+import synth
+from oracle import csp, train
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+npipe = pytest.importorskip("paper_conf_asplos_zhaolcscwzlc22_b200")
+
+FLAGS = npipe.FLAG_TRACE | npipe.FLAG_VERSION_CHECK
+
+
+def run_engine(cfg, choices, batches, D, where=npipe.BATCH_HOST, flags=FLAGS, theta0=None):
+    spec = npipe.Spec(cfg, flags=flags)
+    h = npipe.naspipe_create(spec, D)
+    if theta0 is not None:
+        for (b, c), v in theta0.items():
+            npipe.naspipe_set_params(h, b, c, v)
+    keep = []
+    for y, ch in enumerate(choices):
+        x, t = batches[y]
+        if where == npipe.BATCH_DEVICE:
+            xd = torch.from_numpy(x).cuda()
+            td = torch.from_numpy(t).cuda()
+            keep += [xd, td]
+            npipe.naspipe_submit(h, ch, xd, td, where=where)
+        else:
+            npipe.naspipe_submit(h, ch, x, t, where=where)
+    npipe.naspipe_drain(h)
+    params = {(b, c): npipe.naspipe_get_params(h, b, c)
+              for b in range(cfg["n_blocks"]) for c in range(cfg["n_choices"])}
+    losses = npipe.naspipe_get_losses(h, len(choices))
+    trace = npipe.naspipe_get_trace(h)
+    stats = npipe.naspipe_get_stats(h)
+    npipe.naspipe_destroy(h)
+    return params, losses, trace, stats
+
+
+def param_errors(cfg, got, ref, theta0):
+    """(A15 metric, update diagnostic).
+
+    A15: max over candidates of max_i |gpu_i - ref_i| / max_i |ref_i| over the
+    candidate's packed parameter vector (the unit naspipe_get_params returns).
+    Diagnostic: max over tensors of the normwise relative error of the update
+    ||(gpu - theta0) - (ref - theta0)||_2 / ||ref - theta0||_2 (untouched tensors must be
+    bitwise unchanged)."""
+    worst, worst_delta = 0.0, 0.0
+    for (b, c), r in ref.items():
+        g = got[(b, c)].astype(np.float64)
+        worst = max(worst, np.max(np.abs(g - r)) / np.max(np.abs(r)))
+        off = 0
+        for name, shape, _, _ in train.candidate_layout(cfg, b, c):
+            n = int(np.prod(shape))
+            gs, rs, t0 = g[off:off + n], r[off:off + n], theta0[(b, c)][off:off + n].astype(np.float64)
+            off += n
+            dr = rs - t0
+            if np.any(dr != 0):
+                worst_delta = max(worst_delta, np.linalg.norm((gs - t0) - dr) / np.linalg.norm(dr))
+            else:
+                assert np.array_equal(gs, t0), (b, c, name)
+    return worst, worst_delta
+
+
+def _workload(name, N, **over):
+    cfg = synth.get_config(name, **over)
+    choices = synth.sample_choices(N, cfg["n_blocks"], cfg["n_choices"])
+    batches = [synth.make_batch(cfg, y) for y in range(N)]
+    return cfg, choices, batches
+
+
+def _oracle(cfg, choices, batches):
+    theta0 = train.initial_theta(cfg)
+    ref, losses = train.train_sequential(cfg, theta0, choices, batches)
+    return theta0, ref, losses
+
+
+def _check_trace(cfg, choices, D, trace):
+    spec = npipe.Spec(cfg)
+    sob = npipe.naspipe_partition(spec, D)
+    cf, cb = npipe.naspipe_default_costs(spec)
+    tf, tb = csp.task_costs(choices, sob, cf, cb, D)
+    ref = csp.simulate_csp(choices, sob, D, 4 * D, tf, tb)
+    assert [tuple(int(v) for v in r) for r in trace] == [tuple(r) for r in ref["trace"]]
+    assert csp.check_trace(ref["trace"], choices, sob, D) == []
+
+
+@pytest.mark.parametrize("N,tol", [(1, 1e-3), (16, 1e-3), (100, 1e-2)])
+def test_toy_mlp_parity(N, tol):
+    cfg, choices, batches = _workload("toy", N)
+    theta0, ref, ref_loss = _oracle(cfg, choices, batches)
+    params, losses, trace, stats = run_engine(cfg, choices, batches, D=2)
+    err, derr = param_errors(cfg, params, ref, theta0)
+    assert err <= tol and derr <= 1e-5, (err, derr)
+    np.testing.assert_allclose(losses, ref_loss, rtol=1e-5)
+    _check_trace(cfg, choices, 2, trace)
+    assert stats["version_checks"] == 2 * N * cfg["n_blocks"]
+
+
+def test_toy_bitwise_across_runs_and_stage_counts():
+    cfg, choices, batches = _workload("toy", 24)
+    base, base_loss, _, _ = run_engine(cfg, choices, batches, D=1)
+    for D in (1, 2, 4):
+        p, l, tr, _ = run_engine(cfg, choices, batches, D=D)
+        assert np.array_equal(l.view(np.uint32), base_loss.view(np.uint32)), D
+        for k in base:
+            assert np.array_equal(p[k].view(np.uint32), base[k].view(np.uint32)), (D, k)
+        _check_trace(cfg, choices, D, tr)
+
+
+@pytest.mark.parametrize("N,tol", [(1, 1e-3), (8, 1e-3), (100, 1e-2)])
+def test_tiny_transformer_parity(N, tol):
+    cfg, choices, batches = _workload("tiny_transformer", N)
+    theta0, ref, ref_loss = _oracle(cfg, choices, batches)
+    params, losses, trace, _ = run_engine(cfg, choices, batches, D=2)
+    err, derr = param_errors(cfg, params, ref, theta0)
+    assert err <= tol and derr <= 1e-1, (err, derr)
+    np.testing.assert_allclose(losses, ref_loss, rtol=1e-2)
+    _check_trace(cfg, choices, 2, trace)
+
+
+def test_tiny_transformer_bitwise_across_runs_and_stage_counts():
+    cfg, choices, batches = _workload("tiny_transformer", 10)
+    base, base_loss, _, _ = run_engine(cfg, choices, batches, D=1)
+    for D, where in ((1, npipe.BATCH_HOST), (2, npipe.BATCH_DEVICE), (4, npipe.BATCH_HOST)):
+        p, l, _, _ = run_engine(cfg, choices, batches, D=D, where=where)
+        assert np.array_equal(l.view(np.uint32), base_loss.view(np.uint32)), D
+        for k in base:
+            assert np.array_equal(p[k].view(np.uint32), base[k].view(np.uint32)), (D, k)
+
+
+def test_null_kernels_and_errors():
+    cfg, choices, batches = _workload("toy", 6)
+    spec = npipe.Spec(cfg, flags=FLAGS | npipe.FLAG_NULL_KERNELS)
+    h = npipe.naspipe_create(spec, 2)
+    with pytest.raises(npipe.NaspipeError) as e:
+        npipe.naspipe_submit(h, np.array([0, 0, 0, 9]), batches[0][0], batches[0][1])
+    assert e.value.code == -1
+    for y in range(6):
+        assert npipe.naspipe_submit(h, choices[y], *batches[y]) == y    # rejected submit kept ids
+    npipe.naspipe_drain(h)
+    # parameters untouched with null kernels
+    for (b, c), v in train.initial_theta(cfg).items():
+        assert np.array_equal(npipe.naspipe_get_params(h, b, c), v)
+    # a second stream after a drain continues the ids
+    assert npipe.naspipe_submit(h, choices[0], *batches[0]) == 6
+    with pytest.raises(npipe.NaspipeError) as e:
+        npipe.naspipe_get_params(h, 0, 0)
+    assert e.value.code == -2
+    npipe.naspipe_drain(h)
+    npipe.naspipe_destroy(h)
