@@ -1,0 +1,293 @@
+#!/usr/bin/env python
+"""Benchmark of the NASPipe hot path on B200 (contract: see DESIGN.md "Measurement").
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--workload NAME]
+
+One step = one subnet trained through the whole pipeline (forward, loss, backward and the
+SGD WRITE of every active candidate on every stage) on one synthetic batch.  N = 1 runs the
+whole supernet as one stage on one GPU; N > 1 (torchrun, one process per GPU) runs an
+N-stage CSP pipeline with NCCL send/recv between stages.
+
+Printed by rank 0 as ONE JSON line: value = samples/s of the whole job with the inputs
+already resident in HBM (device batches); e2e = the same through the C ABI with pinned HOST
+buffers (H2D of input+target inside the timed region, D2H of the step losses);
+roofline = the tcgen05 GEMM (the dominant kernel) timed by CUDA events on its stream;
+cpu_baseline = the fp64 NumPy oracle on a bounded sample, on this host's cores.
+"""
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=12)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="transformer")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    return ap.parse_args()
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return dict(bf16=d["bf16_tflops"], bf16_sustained=d.get("bf16_tflops_sustained", d["bf16_tflops"]),
+                    hbm=d["hbm_gbs"], source="MEASURED_PEAKS.json")
+    return dict(bf16=1590.0, bf16_sustained=1400.0, hbm=6650.0, source="fallback (B200_PROFILING.md)")
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device):
+        self.device, self.rows, self.proc = device, [], None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([v.strip() for v in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            self.proc.wait()
+
+    def summary(self):
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        sm = [float(r[0]) for r in self.rows if len(r) >= 6 and r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if len(r) >= 6 and r[1].replace(".", "").isdigit()]
+        reasons = sorted({names[i] for r in self.rows if len(r) >= 6 for i in range(4)
+                          if r[2 + i].lower() == "active"})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(sm)}
+
+
+# ------------------------------------------------------------------------------ CPU oracle
+def oracle_block_sample(cfg, n_blocks_sample):
+    """Time the fp64 oracle on `n_blocks_sample` full-size blocks (fwd + bwd + SGD) of
+    subnet 0.  Returns (seconds, sample description)."""
+    from oracle import train, transformer, mlp   # noqa: F401  (test infrastructure, timing only)
+    ch = synth.sample_choices(1, cfg["n_blocks"], cfg["n_choices"])[0]
+    x, t = synth.make_batch(cfg, 0)
+    theta = {}
+    for b in range(n_blocks_sample):
+        c = int(ch[b])
+        segs = [(int(np.prod(s)), kind, fan) for _, s, kind, fan in train.candidate_layout(cfg, b, c)]
+        theta[(b, c)] = train.unpack(cfg, b, c, synth.init_packed(cfg["init_seed"], b * cfg["n_choices"] + c, segs))
+    t0 = time.perf_counter()
+    sub = dict(cfg, n_blocks=n_blocks_sample)
+    loss, grads = train.subnet_step(sub, theta, ch[:n_blocks_sample], x, t)
+    train.sgd_apply(theta, grads, cfg["lr"])
+    return time.perf_counter() - t0
+
+
+def cpu_threads():
+    try:
+        from threadpoolctl import threadpool_info
+        return max((i.get("num_threads", 1) for i in threadpool_info()), default=os.cpu_count())
+    except Exception:
+        return os.cpu_count()
+
+
+def cpu_baseline(cfg, n_blocks_sample):
+    secs = oracle_block_sample(cfg, n_blocks_sample)
+    per_subnet = secs * cfg["n_blocks"] / n_blocks_sample
+    return {"value": cfg["batch"] / per_subnet, "unit": "samples/s", "cores": cpu_threads(), "kind": "oracle",
+            "sample": f"fp64 NumPy oracle, {n_blocks_sample} of {cfg['n_blocks']} blocks of subnet 0 "
+                      f"(fwd+bwd+SGD, full B={cfg['batch']}, shape of {cfg.get('d_model', cfg.get('width'))}), "
+                      f"{secs:.2f} s, scaled x{cfg['n_blocks'] / n_blocks_sample:g} to one subnet"}
+
+
+def run_reference(args, cfg, rank, world):
+    """--impl reference: the oracle as it stands, on host cores, rank 0 only."""
+    if rank != 0:
+        return
+    nb = 1 if cfg["family"] == "transformer" else cfg["n_blocks"]
+    for _ in range(args.warmup):
+        oracle_block_sample(cfg, nb)
+    ts = [oracle_block_sample(cfg, nb) for _ in range(args.steps)]
+    per_subnet = float(np.mean(ts)) * cfg["n_blocks"] / nb
+    value = cfg["batch"] / per_subnet
+    cores = cpu_threads()
+    sample = (f"each step = {nb} full-size block(s) fwd+bwd+SGD of subnet 0 in the fp64 oracle, "
+              f"scaled x{cfg['n_blocks'] / nb:g} to one subnet")
+    print(json.dumps({
+        "impl": "reference", "metric": "supernet samples/sec", "value": value, "unit": "samples/s",
+        "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * per_subnet,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": workload_config(args, cfg, world),
+        "cpu_baseline": {"kind": "oracle", "cores": cores, "sample": sample, "value": value, "unit": "samples/s"},
+        "e2e": {"value": value, "unit": "samples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}))
+
+
+def workload_config(args, cfg, world):
+    c = {"workload": f"configs[2] {args.workload}" if args.workload == "transformer" else args.workload,
+         "n_blocks": cfg["n_blocks"], "n_choices": cfg["n_choices"], "batch": cfg["batch"],
+         "stages": world, "parallelism": f"pp{world}" if world > 1 else "single stage",
+         "l2": "working set > L2 (active weights + activations per step >> 126 MB)"}
+    if cfg["family"] == "transformer":
+        c.update(seq_len=cfg["seq_len"], d_model=cfg["d_model"], heads=cfg["choice_heads"], ffn=cfg["choice_ffn"])
+    return c
+
+
+# ------------------------------------------------------------------------------ GPU arm
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    cfg = synth.get_config(args.workload)
+    if args.impl == "reference":
+        run_reference(args, cfg, rank, world)
+        return
+
+    import torch
+    import torch.distributed as dist
+    import paper_conf_asplos_zhaolcscwzlc22_b200 as npipe
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    D = world
+    m, n, B = cfg["n_blocks"], cfg["n_choices"], cfg["batch"]
+    total = args.warmup + 2 * args.steps
+    choices = synth.sample_choices(total, m, n)
+    # device-resident input pool (value run) and pinned host pool (e2e run)
+    pool = [synth.make_batch(cfg, y) for y in range(4)]
+    dev_pool = [(torch.from_numpy(x).cuda(), torch.from_numpy(t).cuda()) for x, t in pool]
+    host_pool = [(torch.from_numpy(x).pin_memory(), torch.from_numpy(t).pin_memory()) for x, t in pool]
+    spec = npipe.Spec(cfg, flags=npipe.FLAG_TIMING)
+    if world == 1:
+        h = npipe.naspipe_create(spec, 1)
+    else:
+        ids = [None]
+        if rank == 0:
+            ids[0] = b"".join(npipe.naspipe_nccl_unique_id() for _ in range(2 * (D - 1)))
+        dist.broadcast_object_list(ids, src=0)
+        h = npipe.naspipe_create_rank(spec, D, rank, local, ids[0])
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+
+    def max_over_ranks(v):
+        if world == 1:
+            return v
+        t = torch.tensor([v], device="cuda", dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    y = 0
+    for _ in range(args.warmup):
+        x, t = dev_pool[y % 4]
+        npipe.naspipe_submit(h, choices[y], x, t, where=npipe.BATCH_DEVICE)
+        y += 1
+    npipe.naspipe_drain(h)
+
+    # ---- timed region 1: inputs resident in HBM
+    s0 = npipe.naspipe_get_stats(h)
+    barrier()
+    with ClockSampler(local) as clk:
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        t_wall = time.perf_counter()
+        e0.record()
+        for _ in range(args.steps):
+            x, t = dev_pool[y % 4]
+            npipe.naspipe_submit(h, choices[y], x, t, where=npipe.BATCH_DEVICE)
+            y += 1
+        npipe.naspipe_drain(h)
+        e1.record()
+        torch.cuda.synchronize()
+        t_wall = time.perf_counter() - t_wall
+    s1 = npipe.naspipe_get_stats(h)
+    # the default-stream events bracket the drain (host waits for every stage stream), so
+    # the elapsed time covers all device work of the K steps
+    ms = max_over_ranks(e0.elapsed_time(e1))
+    value = args.steps * B / (ms / 1000)
+
+    # ---- roofline of the dominant kernel (tcgen05 GEMM), CUDA events on its stream
+    g_flops = s1["dominant_flops"] - s0["dominant_flops"]
+    g_ms = s1["dominant_ms"] - s0["dominant_ms"]
+    g_n = s1["dominant_launches"] - s0["dominant_launches"]
+    pk = peaks()
+    achieved = (g_flops / g_n) / ((g_ms / g_n) / 1000) / 1e12 if g_n else None
+    traffic = None
+    prof = os.path.join(ROOT, "profiles", "gemm_traffic.json")
+    if os.path.exists(prof):
+        with open(prof) as f:
+            traffic = json.load(f).get("dram_bytes_per_launch_by_shape")
+    roofline = {"bound": "tensor", "kernel": "gemm_tc_kernel (tcgen05, all shapes of the step)",
+                "achieved": achieved, "peak": pk["bf16_sustained"], "unit": "TFLOP/s",
+                "frac": achieved / pk["bf16_sustained"] if achieved else None, "traffic": traffic,
+                "peak_source": pk["source"] + " bf16_tflops_sustained (kernel timed inside a long step)",
+                "launches": g_n, "gemm_share_of_step": g_ms / ms if ms else None,
+                "algorithmic_flops_per_step": g_flops / args.steps}
+    launches = (s1["kernel_launches"] - s0["kernel_launches"])
+
+    # ---- timed region 2: end to end through the C ABI with pinned host buffers
+    e2e = None
+    if not args.no_e2e:
+        barrier()
+        e0.record()
+        for k in range(args.steps):
+            x, t = host_pool[y % 4]
+            npipe.naspipe_submit(h, choices[y], x, t, where=npipe.BATCH_HOST)
+            y += 1
+        npipe.naspipe_drain(h)
+        if rank == world - 1:
+            npipe.naspipe_get_losses(h, y)[-args.steps:]   # D2H of the step results
+        e1.record()
+        torch.cuda.synchronize()
+        ms2 = max_over_ranks(e0.elapsed_time(e1))
+        per = x.numel() * 4
+        e2e = {"value": args.steps * B / (ms2 / 1000), "unit": "samples/s",
+               "h2d_bytes_per_step": 2 * per, "d2h_bytes_per_step": 4}
+    losses = npipe.naspipe_get_losses(h, y) if rank == world - 1 else None
+    npipe.naspipe_destroy(h)
+
+    if rank != 0:
+        return
+    cpu = None
+    if world == 1 and not args.no_cpu:
+        cpu = cpu_baseline(cfg, 2 if cfg["family"] == "transformer" else cfg["n_blocks"])
+    out = {"metric": "supernet samples/sec", "value": value, "unit": "samples/s", "n_gpus": world,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+           "scaling": "strong", "vs_baseline": None, "dtype": "bf16" if cfg["family"] == "transformer" else "f32",
+           "data": "synthetic (N(0,1) inputs/targets, counter-hash init, uniform per-block choices)",
+           "config": workload_config(args, cfg, world), "clocks": clk.summary(), "e2e": e2e,
+           "gpu_launches": int(launches), "roofline": roofline, "cpu_baseline": cpu,
+           "loss_finite": bool(losses is None or np.all(np.isfinite(losses)))}
+    print(json.dumps(out))
+
+
+if __name__ == "__main__":
+    main()

@@ -353,7 +353,7 @@ void Engine::issue_forward(StageRt& st, int64_t y, int slot) {
     } else if (bt.where == NASPIPE_BATCH_DEVICE) {
       xin = static_cast<const float*>(bt.input);
     } else {
-      if (!null_k) synth_fill(st.comp, st.in[slot], n, bt.synth_seed * 2 + 0);
+      if (!null_k) { synth_fill(st.comp, st.in[slot], n, bt.synth_seed * 2 + 0); ++engine_launches_; }
       xin = st.in[slot];
     }
   } else if (rank_ < 0) {
@@ -379,7 +379,7 @@ void Engine::issue_forward(StageRt& st, int64_t y, int slot) {
     } else if (bt.where == NASPIPE_BATCH_DEVICE) {
       tgt = static_cast<const float*>(bt.target);
     } else {
-      if (!null_k) synth_fill(st.comp, st.target[slot], n, bt.synth_seed * 2 + 1);
+      if (!null_k) { synth_fill(st.comp, st.target[slot], n, bt.synth_seed * 2 + 1); ++engine_launches_; }
       tgt = st.target[slot];
     }
   }
@@ -389,7 +389,7 @@ void Engine::issue_forward(StageRt& st, int64_t y, int slot) {
   if (!null_k) st.fam->forward(slot, planner_.choice_row(y), xin, st.out[slot], st.comp);
   if (K == D_ - 1) {
     if (bt.where == NASPIPE_BATCH_HOST) CU(cudaStreamWaitEvent(st.comp, st.ev_tgt[slot], 0));
-    if (!null_k) mse_loss(st.comp, st.out[slot], tgt, st.gout[slot], st.mse_part, st.loss + y, n);
+    if (!null_k) { mse_loss(st.comp, st.out[slot], tgt, st.gout[slot], st.mse_part, st.loss + y, n); engine_launches_ += 2; }
   }
   CU(cudaEventRecord(st.ev_f[slot], st.comp));
   if (rank_ >= 0 && tx_ && K < D_ - 1) {
@@ -493,7 +493,7 @@ void Engine::get_stats(double* o) {
   for (auto& st : st_)
     if (st.local && st.fam) launches += (double)st.fam->counters.launches;
   o[0] = (double)issued_;
-  o[1] = launches;
+  o[1] = launches + (double)engine_launches_;
   o[2] = h2d_bytes_;
   o[3] = d2h_bytes_;
   o[4] = p2p_bytes_;

@@ -82,6 +82,7 @@ class Engine {
   uint64_t version_checks_ = 0;
   // stats
   double h2d_bytes_ = 0, d2h_bytes_ = 0, p2p_bytes_ = 0;
+  uint64_t engine_launches_ = 0;  // kernels launched by the engine itself (loss, synthetic data)
   std::vector<Task> trace_;
   KernelTimer timer_;
 };
