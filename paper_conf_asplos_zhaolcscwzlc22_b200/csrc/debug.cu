@@ -40,8 +40,24 @@ int naspipe_debug_gemm(int M, int N, int K, const void* A, int a_mn, int lda, co
     ep.w32 = w32;
     ep.w16 = static_cast<bf16*>(w16);
     ep.lr = lr;
-    gemm_bf16_tc((cudaStream_t)stream, M, N, K, static_cast<const bf16*>(A), a_mn != 0, lda,
-                 static_cast<const bf16*>(B), b_mn != 0, ldb, epi, ep);
+    // exercise split-K exactly as the engine would (workspace of splits * M * N floats)
+    const int splits = gemm_splitk_factor(M, N, K);
+    cudaStream_t s = (cudaStream_t)stream;
+    static float* ws = nullptr;  // grown on demand, kept for the process (test helper)
+    static size_t ws_cap = 0;
+    if (splits > 1 && (epi == EPI_F32 || epi == EPI_SGD)) {
+      const size_t need = (size_t)splits * M * N;
+      if (need > ws_cap) {
+        cudaDeviceSynchronize();
+        if (ws) cudaFree(ws);
+        NP_REQUIRE(cudaMalloc(&ws, need * 4) == cudaSuccess, NASPIPE_ENOMEM, "ws");
+        ws_cap = need;
+      }
+      ep.ws = ws;
+      ep.ws_elems = ws_cap;
+    }
+    gemm_bf16_tc(s, M, N, K, static_cast<const bf16*>(A), a_mn != 0, lda, static_cast<const bf16*>(B), b_mn != 0,
+                 ldb, epi, ep);
   });
 }
 

@@ -162,6 +162,31 @@ __global__ void sgd_partials_kernel(float* __restrict__ p, const float* __restri
   p[i] -= lr * g;
 }
 
+// 32 columns x 8 row-groups per block; group g sums partials [g*G, (g+1)*G) in order, the 8
+// group sums are added in group order.
+__global__ void sgd_multi_kernel(SgdJobs jobs) {
+  const SgdJob jb = jobs.job[blockIdx.y];
+  const int lane = threadIdx.x & 31, grp = threadIdx.x >> 5;
+  const int col = blockIdx.x * 32 + lane;
+  if (blockIdx.x * 32 >= jb.n) return;  // block-uniform
+  __shared__ float red[8][33];
+  float acc = 0.f;
+  if (col < jb.n) {
+    const int G = (jb.nblk + 7) / 8;
+    const int j0 = grp * G, j1 = min(jb.nblk, j0 + G);
+#pragma unroll 8
+    for (int j = j0; j < j1; ++j) acc += jb.part[(size_t)j * jb.n + col];
+  }
+  red[grp][lane] = acc;
+  __syncthreads();
+  if (grp == 0 && col < jb.n) {
+    float g = 0.f;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) g += red[k][lane];
+    jb.p[col] -= jobs.lr * g;
+  }
+}
+
 __global__ void f2bf_kernel(const float* __restrict__ a, bf16* __restrict__ b, size_t n) {
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x)
     b[i] = __float2bfloat16_rn(a[i]);
@@ -295,6 +320,14 @@ void cast_colsum(cudaStream_t s, const float* X, bf16* X16, float* part, int T, 
 void sgd_from_partials(cudaStream_t s, float* p, const float* part, int nblk, int n, float lr) {
   sgd_partials_kernel<<<(n + 255) / 256, 256, 0, s>>>(p, part, nblk, n, lr);
   check_launch("sgd_from_partials");
+}
+
+void sgd_multi(cudaStream_t s, const SgdJobs& jobs) {
+  int nmax = 0;
+  for (int i = 0; i < jobs.count; ++i) nmax = std::max(nmax, jobs.job[i].n);
+  dim3 grid((nmax + 31) / 32, jobs.count);
+  sgd_multi_kernel<<<grid, 256, 0, s>>>(jobs);
+  check_launch("sgd_multi");
 }
 
 void f32_to_bf16(cudaStream_t s, const float* w32, bf16* w16, size_t n) {

@@ -188,6 +188,15 @@ class TfFamily : public Family {
     dqkv_ = A.alloc<bf16>(3 * Td);
     gb_[0] = A.alloc<float>(Td);
     gb_[1] = A.alloc<float>(Td);
+    // split-K workspace: the largest splits * M * N over this stage's GEMMs
+    ws_elems_ = 0;
+    for (int c = 0; c < n; ++c) {
+      const int f = spec.ffn[c], T = T_, d = d_;
+      const int shp[6][3] = {{d, f, T}, {f, d, T}, {d, d, T}, {3 * d, d, T}, {T, d, f}, {T, d, 3 * d}};
+      for (auto& q : shp)
+        ws_elems_ = std::max(ws_elems_, (size_t)gemm_splitk_factor(q[0], q[1], q[2]) * q[0] * q[1]);
+    }
+    ws_ = A.alloc<float>(ws_elems_);
     csb_ = colsum_blocks(T_);
     lnb_ = ln_bwd_blocks(T_);
     const int pb = std::max(csb_, lnb_);
@@ -252,7 +261,10 @@ class TfFamily : public Family {
   void gemm(cudaStream_t s, int M, int N, int K, const bf16* A, bool amn, int lda, const bf16* B, bool bmn, int ldb,
             int epi, const GemmEpiParams& ep) {
     if (timer) timer->begin(s);
-    gemm_bf16_tc(s, M, N, K, A, amn, lda, B, bmn, ldb, epi, ep);
+    GemmEpiParams e = ep;
+    e.ws = ws_;
+    e.ws_elems = ws_elems_;
+    gemm_bf16_tc(s, M, N, K, A, amn, lda, B, bmn, ldb, epi, e);
     if (timer) timer->end(s, 2.0 * M * N * K);
     counters.launches++;
   }
@@ -338,18 +350,26 @@ class TfFamily : public Family {
     e.lr = lr_;
     gemm(s, 3 * d, d, T, dqkv_, true, 3 * d, t.a, true, d, EPI_SGD, e);    // Wqkv -= lr dqkv^T a
     // bias / LN2 updates (their partials are complete; LN1 partials come next)
-    sgd_from_partials(s, P + o.b2, p_db2_, db2_nblk, d, lr_);
-    sgd_from_partials(s, P + o.b1, p_db1_, csb_, f, lr_);
-    sgd_from_partials(s, P + o.bo, p_dbo_, lnb_, d, lr_);
-    sgd_from_partials(s, P + o.bqkv, p_dbqkv_, csb_, 3 * d, lr_);
-    sgd_from_partials(s, P + o.ln2g, p_g2_, lnb_, d, lr_);
-    sgd_from_partials(s, P + o.ln2b, p_b2_, lnb_, d, lr_);
+    SgdJobs j1{};
+    j1.lr = lr_;
+    j1.job[0] = {P + o.b2, p_db2_, db2_nblk, d};
+    j1.job[1] = {P + o.b1, p_db1_, csb_, f};
+    j1.job[2] = {P + o.bo, p_dbo_, lnb_, d};
+    j1.job[3] = {P + o.bqkv, p_dbqkv_, csb_, 3 * d};
+    j1.job[4] = {P + o.ln2g, p_g2_, lnb_, d};
+    j1.job[5] = {P + o.ln2b, p_b2_, lnb_, d};
+    j1.count = 6;
+    sgd_multi(s, j1);
     // LN1 backward: dx = dx1 + LN1'(da); bf16 copy / column partials feed block j-1
     ln_bwd(s, da_, t.xin, t.mean1, t.rstd1, P + o.ln1g, dx1_, dx, want_next ? dy16_ : nullptr, p_g1_, p_b1_,
            want_next ? p_db2_ : nullptr, T, d);
-    sgd_from_partials(s, P + o.ln1g, p_g1_, lnb_, d, lr_);
-    sgd_from_partials(s, P + o.ln1b, p_b1_, lnb_, d, lr_);
-    counters.launches += 13;
+    SgdJobs j2{};
+    j2.lr = lr_;
+    j2.job[0] = {P + o.ln1g, p_g1_, lnb_, d};
+    j2.job[1] = {P + o.ln1b, p_b1_, lnb_, d};
+    j2.count = 2;
+    sgd_multi(s, j2);
+    counters.launches += 7;
   }
 
   const Spec& spec_;
@@ -360,7 +380,8 @@ class TfFamily : public Family {
   std::vector<bf16*> w16_;
   std::vector<TfSlot> slots_;
   bf16 *dy16_, *dz_, *dx1_16_, *do16_, *dqkv_;
-  float *da_, *dx1_, *gb_[2];
+  float *da_, *dx1_, *gb_[2], *ws_ = nullptr;
+  size_t ws_elems_ = 0;
   float *p_db2_, *p_db1_, *p_dbo_, *p_dbqkv_, *p_g1_, *p_b1_, *p_g2_, *p_b2_;
 };
 

@@ -1,15 +1,19 @@
-// tcgen05 GEMM for sm_100a: TMA (128B swizzle) -> shared memory ring -> single-thread
-// tcgen05.mma (M=128, N=BN, K=16 per instruction) accumulating in TMEM -> fused epilogue
-// (bias / residual / GELU / GELU' / SGD update) from tcgen05.ld.
+// tcgen05 GEMM for sm_100a (persistent, warp-specialised).
 //
-// Warp roles (128 threads): warp 0 lane 0 = TMA producer, warp 1 lane 0 = MMA issuer,
-// warp 2 = TMEM allocator; after the main loop all four warps run the epilogue, warp w
-// owning accumulator rows (TMEM lanes) 32w..32w+31.  One output tile per CTA; the kernel
-// is sized so that two CTAs co-reside per SM, overlapping one CTA's epilogue with the
-// other's main loop.  Every output element is produced by exactly one CTA with a fixed K
-// order, so results are bitwise deterministic.
+//   TMA (128B swizzle) -> 4-stage shared-memory ring -> single-thread tcgen05.mma
+//   (M=128, N=256, K=16 per instruction) accumulating in TMEM (2 x 256 columns, double
+//   buffered) -> tcgen05.ld epilogue with fused bias / residual / GELU / GELU' / SGD update.
+//
+// One CTA per SM (192 KB ring), 6 warps: warp 0 = TMA producer, warp 1 = MMA issuer (also
+// allocates TMEM), warps 2-5 = epilogue (warp w reads TMEM lanes 32*(w%4)..+31).  Tiles are
+// assigned statically (tile = blockIdx.x + i*gridDim.x), so the epilogue of tile i overlaps
+// the main loop of tile i+1.  Deterministic split-K (for the wgrad GEMMs, K = B*S, whose
+// outputs are too small to fill 148 SMs): each K slice writes an fp32 partial tile to a
+// workspace and a second kernel sums the slices in fixed order and applies the epilogue.
+// Every output element is produced with a fixed K order: results are bitwise reproducible.
 #include <cuda.h>
 
+#include <algorithm>
 #include <atomic>
 #include <mutex>
 
@@ -22,43 +26,142 @@ namespace naspipe {
 namespace {
 
 constexpr int BM = 128;
+constexpr int BN = 256;
 constexpr int BK = 64;  // 64 bf16 = 128 B = one swizzle row
+constexpr int STAGES = 4;
+constexpr int A_BYTES = BM * BK * 2;               // 16 KB
+constexpr int B_BYTES = BN * BK * 2;               // 32 KB
+constexpr int STAGE_BYTES = A_BYTES + B_BYTES;     // 48 KB
+constexpr int BAR_OFF = STAGES * STAGE_BYTES;
+constexpr int SMEM_TOTAL = BAR_OFF + (2 * STAGES + 4) * 8 + 16 + 1024;  // + alignment slack
+constexpr int THREADS = 320;  // 2 control warps + 8 epilogue warps
+constexpr int EPI_PARTIAL = 100;  // internal: fp32 partial tile of one K slice
 
 __device__ __forceinline__ float gelu_tanh(float z) {
   const float c = 0.7978845608028654f;
   const float u = c * (z + 0.044715f * z * z * z);
-  return 0.5f * z * (1.f + tanhf(u));
+  return 0.5f * z * (1.f + ptx::tanh_fast(u));
 }
 __device__ __forceinline__ float gelu_tanh_grad(float z) {
   const float c = 0.7978845608028654f;
-  const float t = tanhf(c * (z + 0.044715f * z * z * z));
+  const float t = ptx::tanh_fast(c * (z + 0.044715f * z * z * z));
   return 0.5f * (1.f + t) + 0.5f * z * (1.f - t * t) * c * (1.f + 3.f * 0.044715f * z * z);
 }
 
-template <int BN, int STAGES>
-struct GemmSmem {
-  static constexpr int A_BYTES = BM * BK * 2;
-  static constexpr int B_BYTES = BN * BK * 2;
-  static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int BAR_OFF = STAGES * STAGE_BYTES;
-  static constexpr int TOTAL = BAR_OFF + (2 * STAGES + 1) * 8 + 16 + 1024;  // +1024 alignment slack
+__device__ __forceinline__ void store16_bf16(bf16* dst, const float (&v)[16]) {
+  uint32_t p[8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) p[i] = ptx::pack_bf16(v[2 * i], v[2 * i + 1]);
+  uint4* o4 = reinterpret_cast<uint4*>(dst);
+  o4[0] = make_uint4(p[0], p[1], p[2], p[3]);
+  o4[1] = make_uint4(p[4], p[5], p[6], p[7]);
+}
+__device__ __forceinline__ void store16_f32(float* dst, const float (&v)[16]) {
+  float4* o4 = reinterpret_cast<float4*>(dst);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) o4[i] = make_float4(v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
+}
+
+// Operands of the epilogue that live in global memory, loaded BEFORE the TMEM read so that
+// their latency overlaps it (residual / fp32 master / pre-activation).
+struct Pre16 {
+  float4 q[4];
+  uint4 z[2];
+};
+template <int EPI>
+__device__ __forceinline__ void preload16(Pre16& p, size_t off, const GemmEpiParams& ep) {
+  if constexpr (EPI == EPI_BIAS_RESID_F32) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i) p.q[i] = reinterpret_cast<const float4*>(ep.resid + off)[i];
+  }
+  if constexpr (EPI == EPI_SGD) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i) p.q[i] = reinterpret_cast<const float4*>(ep.w32 + off)[i];
+  }
+  if constexpr (EPI == EPI_DGELU) {
+#pragma unroll
+    for (int i = 0; i < 2; ++i) p.z[i] = reinterpret_cast<const uint4*>(ep.aux16 + off)[i];
+  }
+}
+
+// Apply epilogue EPI to 16 consecutive accumulator columns (row, col..col+15), N = ld.
+template <int EPI>
+__device__ __forceinline__ void epilogue16(float (&v)[16], const Pre16& pre, size_t off, int col,
+                                           const GemmEpiParams& ep, int split) {
+  if constexpr (EPI == EPI_PARTIAL) {
+    store16_f32(ep.ws + (size_t)split * ep.ws_stride + off, v);
+    return;
+  }
+  if constexpr (EPI == EPI_BIAS_BF16 || EPI == EPI_BIAS_RESID_F32 || EPI == EPI_BIAS_GELU) {
+    const float4* b4 = reinterpret_cast<const float4*>(ep.bias + col);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const float4 b = b4[i];
+      v[4 * i] += b.x; v[4 * i + 1] += b.y; v[4 * i + 2] += b.z; v[4 * i + 3] += b.w;
+    }
+  }
+  if constexpr (EPI == EPI_BIAS_RESID_F32) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      v[4 * i] += pre.q[i].x; v[4 * i + 1] += pre.q[i].y; v[4 * i + 2] += pre.q[i].z; v[4 * i + 3] += pre.q[i].w;
+    }
+  }
+  if constexpr (EPI == EPI_DGELU) {
+#pragma unroll
+    for (int i = 0; i < 2; ++i) {
+      const bf16* zz = reinterpret_cast<const bf16*>(&pre.z[i]);
+#pragma unroll
+      for (int j = 0; j < 8; ++j) v[8 * i + j] *= gelu_tanh_grad(__bfloat162float(zz[j]));
+    }
+  }
+  if constexpr (EPI == EPI_F32 || EPI == EPI_BIAS_RESID_F32) {
+    store16_f32(reinterpret_cast<float*>(ep.out) + off, v);
+  } else if constexpr (EPI == EPI_SGD) {
+    float w[16];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      float4 x = pre.q[i];
+      x.x -= ep.lr * v[4 * i]; x.y -= ep.lr * v[4 * i + 1];
+      x.z -= ep.lr * v[4 * i + 2]; x.w -= ep.lr * v[4 * i + 3];
+      reinterpret_cast<float4*>(ep.w32 + off)[i] = x;
+      w[4 * i] = x.x; w[4 * i + 1] = x.y; w[4 * i + 2] = x.z; w[4 * i + 3] = x.w;
+    }
+    store16_bf16(ep.w16 + off, w);
+  } else {
+    store16_bf16(reinterpret_cast<bf16*>(ep.out) + off, v);
+    if constexpr (EPI == EPI_BIAS_GELU) {
+      float g[16];
+#pragma unroll
+      for (int i = 0; i < 16; ++i) g[i] = gelu_tanh(v[i]);
+      store16_bf16(ep.out2 + off, g);
+    }
+  }
+}
+
+struct TileSpace {
+  int MT, NT, splits, nk_per_split, nk;
+  __device__ __forceinline__ void decode(int t, int& tm, int& tn, int& ks) const {
+    ks = t % splits;
+    const int r = t / splits;
+    tm = r % MT;
+    tn = r / MT;
+  }
 };
 
-template <int BN, int STAGES, bool A_MN, bool B_MN, int EPI>
-__global__ void __launch_bounds__(128, 2)
-    gemm_tc_kernel(const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb, int M,
-                   int N, int K, GemmEpiParams ep) {
-  using L = GemmSmem<BN, STAGES>;
+template <bool A_MN, bool B_MN, int EPI>
+__global__ void __launch_bounds__(THREADS, 1)
+    gemm_tc_kernel(const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb, int M, int N,
+                   TileSpace ts, GemmEpiParams ep) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + L::BAR_OFF);
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + BAR_OFF);
   uint64_t* empty = full + STAGES;
-  uint64_t* tmem_full = empty + STAGES;
-  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(tmem_full + 1);
+  uint64_t* tfull = empty + STAGES;  // [2]
+  uint64_t* tempty = tfull + 2;      // [2]
+  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(tempty + 2);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int m0 = blockIdx.y * BM, n0 = blockIdx.x * BN;
-  const int nk = (K + BK - 1) / BK;
+  const int n_tiles = ts.MT * ts.NT * ts.splits;
 
   if (threadIdx.x == 0) {
     ptx::tma_prefetch(&ta);
@@ -67,143 +170,155 @@ __global__ void __launch_bounds__(128, 2)
       ptx::mbar_init(&full[s], 1);
       ptx::mbar_init(&empty[s], 1);
     }
-    ptx::mbar_init(tmem_full, 1);
+    for (int a = 0; a < 2; ++a) {
+      ptx::mbar_init(&tfull[a], 1);
+      ptx::mbar_init(&tempty[a], 8);
+    }
     ptx::fence_mbar_init();
   }
-  if (warp == 2) ptx::tmem_alloc<BN>(tmem_holder);
+  if (warp == 1) ptx::tmem_alloc<512>(tmem_holder);
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_holder;
 
-  if (warp == 0 && lane == 0) {
-    // ---------------- TMA producer
-    for (int kb = 0; kb < nk; ++kb) {
-      const int s = kb % STAGES;
-      if (kb >= STAGES) ptx::mbar_wait(&empty[s], ((kb / STAGES) - 1) & 1);
-      uint8_t* sa = smem + s * L::STAGE_BYTES;
-      uint8_t* sb = sa + L::A_BYTES;
-      ptx::mbar_arrive_expect_tx(&full[s], L::STAGE_BYTES);
-      const int k0 = kb * BK;
-      if (!A_MN) {
-        ptx::tma_load_2d(sa, &ta, &full[s], k0, m0);
-      } else {
+  if (warp == 0) {
+    if (lane == 0) {  // ---------------- TMA producer
+      int s = 0, ph = 0;
+      for (int t = blockIdx.x; t < n_tiles; t += gridDim.x) {
+        int tm, tn, ks;
+        ts.decode(t, tm, tn, ks);
+        const int m0 = tm * BM, n0 = tn * BN;
+        const int kb0 = ks * ts.nk_per_split, kb1 = min(ts.nk, kb0 + ts.nk_per_split);
+        for (int kb = kb0; kb < kb1; ++kb) {
+          ptx::mbar_wait(&empty[s], ph ^ 1);
+          uint8_t* sa = smem + s * STAGE_BYTES;
+          uint8_t* sb = sa + A_BYTES;
+          ptx::mbar_arrive_expect_tx(&full[s], STAGE_BYTES);
+          const int k0 = kb * BK;
+          if (!A_MN) {
+            ptx::tma_load_2d(sa, &ta, &full[s], k0, m0);
+          } else {
 #pragma unroll
-        for (int j = 0; j < BM / 64; ++j) ptx::tma_load_2d(sa + j * 8192, &ta, &full[s], m0 + 64 * j, k0);
-      }
-      if (!B_MN) {
-        ptx::tma_load_2d(sb, &tb, &full[s], k0, n0);
-      } else {
+            for (int j = 0; j < BM / 64; ++j) ptx::tma_load_2d(sa + j * 8192, &ta, &full[s], m0 + 64 * j, k0);
+          }
+          if (!B_MN) {
+            ptx::tma_load_2d(sb, &tb, &full[s], k0, n0);
+          } else {
 #pragma unroll
-        for (int j = 0; j < BN / 64; ++j) ptx::tma_load_2d(sb + j * 8192, &tb, &full[s], n0 + 64 * j, k0);
+            for (int j = 0; j < BN / 64; ++j) ptx::tma_load_2d(sb + j * 8192, &tb, &full[s], n0 + 64 * j, k0);
+          }
+          if (++s == STAGES) { s = 0; ph ^= 1; }
+        }
       }
     }
-  } else if (warp == 1 && lane == 0) {
-    // ---------------- MMA issuer
-    constexpr uint32_t idesc = ptx::umma_idesc_bf16(BM, BN, A_MN ? 1 : 0, B_MN ? 1 : 0);
-    for (int kb = 0; kb < nk; ++kb) {
-      const int s = kb % STAGES;
-      ptx::mbar_wait(&full[s], (kb / STAGES) & 1);
+  } else if (warp == 1) {
+    if (lane == 0) {  // ---------------- MMA issuer
+      constexpr uint32_t idesc = ptx::umma_idesc_bf16(BM, BN, A_MN ? 1 : 0, B_MN ? 1 : 0);
+      int s = 0, ph = 0, it = 0;
+      for (int t = blockIdx.x; t < n_tiles; t += gridDim.x, ++it) {
+        int tm, tn, ks;
+        ts.decode(t, tm, tn, ks);
+        const int kb0 = ks * ts.nk_per_split, kb1 = min(ts.nk, kb0 + ts.nk_per_split);
+        const int acc = it & 1;
+        ptx::mbar_wait(&tempty[acc], ((it >> 1) & 1) ^ 1);  // epilogue drained this buffer
+        ptx::tc_fence_after();
+        const uint32_t d = tmem + acc * BN;
+        for (int kb = kb0; kb < kb1; ++kb) {
+          ptx::mbar_wait(&full[s], ph);
+          ptx::tc_fence_after();
+          const uint32_t sa = ptx::smem_u32(smem + s * STAGE_BYTES);
+          const uint32_t sb = sa + A_BYTES;
+#pragma unroll
+          for (int k = 0; k < BK / 16; ++k) {
+            // K-major: 128-B rows, 8-row groups 1024 B apart (SBO); a K step of 16 = +32 B.
+            // MN-major: 64-element MN chunks 8 KB apart (LBO), 8 K-rows = 1024 B (SBO);
+            //           a K step of 16 rows = +2048 B.
+            const uint64_t ad = A_MN ? ptx::umma_desc_sw128(sa + k * 2048, 8192, 1024)
+                                     : ptx::umma_desc_sw128(sa + k * 32, 16, 1024);
+            const uint64_t bd = B_MN ? ptx::umma_desc_sw128(sb + k * 2048, 8192, 1024)
+                                     : ptx::umma_desc_sw128(sb + k * 32, 16, 1024);
+            ptx::umma_bf16(d, ad, bd, idesc, (kb > kb0 || k > 0) ? 1u : 0u);
+          }
+          ptx::umma_commit(&empty[s]);  // frees the smem stage when these MMAs complete
+          if (++s == STAGES) { s = 0; ph ^= 1; }
+        }
+        ptx::umma_commit(&tfull[acc]);  // accumulator ready for the epilogue
+      }
+    }
+  } else {
+    // ---------------- epilogue warps 2..9: TMEM lane quarter (warp % 4), column half
+    const int lane_base = 32 * (warp & 3);
+    const int cbeg = ((warp - 2) >> 2) * (BN / 2);
+    int it = 0;
+    for (int t = blockIdx.x; t < n_tiles; t += gridDim.x, ++it) {
+      int tm, tn, ks;
+      ts.decode(t, tm, tn, ks);
+      const int acc = it & 1;
+      ptx::mbar_wait(&tfull[acc], (it >> 1) & 1);
       ptx::tc_fence_after();
-      const uint32_t sa = ptx::smem_u32(smem + s * L::STAGE_BYTES);
-      const uint32_t sb = sa + L::A_BYTES;
-#pragma unroll
-      for (int k = 0; k < BK / 16; ++k) {
-        // K-major: rows of 128 B, 8-row groups 1024 B apart; a K step of 16 = +32 B.
-        // MN-major: 64-element MN chunks 8 KB apart (LBO), 8 K-rows = 1024 B (SBO);
-        //           a K step of 16 rows = +2048 B.
-        const uint64_t ad = A_MN ? ptx::umma_desc_sw128(sa + k * 2048, 8192, 1024)
-                                 : ptx::umma_desc_sw128(sa + k * 32, 16, 1024);
-        const uint64_t bd = B_MN ? ptx::umma_desc_sw128(sb + k * 2048, 8192, 1024)
-                                 : ptx::umma_desc_sw128(sb + k * 32, 16, 1024);
-        ptx::umma_bf16(tmem, ad, bd, idesc, (kb | k) != 0 ? 1u : 0u);
-      }
-      ptx::umma_commit(&empty[s]);  // frees the smem stage when these MMAs complete
-    }
-    ptx::umma_commit(tmem_full);
-  }
-  __syncwarp();
-
-  // ---------------- epilogue: all 4 warps
-  ptx::mbar_wait(tmem_full, 0);
-  ptx::tc_fence_after();
-  const int row = m0 + warp * 32 + lane;
-  const bool row_ok = row < M;
+      const int row = tm * BM + lane_base + lane;
+      const bool row_ok = row < M;
+      const uint32_t taddr = tmem + ((uint32_t)lane_base << 16) + acc * BN;
 #pragma unroll 1
-  for (int c0 = 0; c0 < BN; c0 += 16) {
-    uint32_t r[16];
-    ptx::tmem_ld16(tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)c0, r);
-    ptx::tmem_ld_wait();
-    const int col = n0 + c0;
-    if (!row_ok || col >= N) continue;
-    float v[16];
+      for (int c0 = cbeg; c0 < cbeg + BN / 2; c0 += 32) {
+        const int col = tn * BN + c0;
+        if (col >= N) break;               // warp-uniform
+        const bool two = col + 16 < N;     // N % 16 == 0: the chunk is 16 or 32 columns
+        const size_t off = (size_t)row * N + col;
+        Pre16 p0, p1;
+        if (row_ok) {
+          preload16<EPI>(p0, off, ep);
+          if (two) preload16<EPI>(p1, off + 16, ep);
+        }
+        uint32_t r[32];
+        ptx::tmem_ld32(taddr + c0, r);
+        ptx::tmem_ld_wait();
+        if (!row_ok) continue;
+        float v[16];
 #pragma unroll
-    for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
-    const size_t off = (size_t)row * N + col;
-    if constexpr (EPI == EPI_BIAS_BF16 || EPI == EPI_BIAS_RESID_F32 || EPI == EPI_BIAS_GELU) {
-      const float4* b4 = reinterpret_cast<const float4*>(ep.bias + col);
+        for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
+        epilogue16<EPI>(v, p0, off, col, ep, ks);
+        if (two) {
 #pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const float4 b = b4[i];
-        v[4 * i] += b.x; v[4 * i + 1] += b.y; v[4 * i + 2] += b.z; v[4 * i + 3] += b.w;
+          for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[16 + i]);
+          epilogue16<EPI>(v, p1, off + 16, col + 16, ep, ks);
+        }
       }
-    }
-    if constexpr (EPI == EPI_BIAS_RESID_F32) {
-      const float4* r4 = reinterpret_cast<const float4*>(ep.resid + off);
-#pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const float4 q = r4[i];
-        v[4 * i] += q.x; v[4 * i + 1] += q.y; v[4 * i + 2] += q.z; v[4 * i + 3] += q.w;
-      }
-    }
-    if constexpr (EPI == EPI_DGELU) {
-      const uint4* z4 = reinterpret_cast<const uint4*>(ep.aux16 + off);
-#pragma unroll
-      for (int i = 0; i < 2; ++i) {
-        uint4 q = z4[i];
-        const __nv_bfloat16* zz = reinterpret_cast<const __nv_bfloat16*>(&q);
-#pragma unroll
-        for (int j = 0; j < 8; ++j) v[8 * i + j] *= gelu_tanh_grad(__bfloat162float(zz[j]));
-      }
-    }
-    if constexpr (EPI == EPI_F32 || EPI == EPI_BIAS_RESID_F32) {
-      float4* o4 = reinterpret_cast<float4*>(reinterpret_cast<float*>(ep.out) + off);
-#pragma unroll
-      for (int i = 0; i < 4; ++i) o4[i] = make_float4(v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
-    } else if constexpr (EPI == EPI_SGD) {
-      float4* w4 = reinterpret_cast<float4*>(ep.w32 + off);
-      uint32_t p[8];
-#pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        float4 w = w4[i];
-        w.x -= ep.lr * v[4 * i]; w.y -= ep.lr * v[4 * i + 1];
-        w.z -= ep.lr * v[4 * i + 2]; w.w -= ep.lr * v[4 * i + 3];
-        w4[i] = w;
-        p[2 * i] = ptx::pack_bf16(w.x, w.y);
-        p[2 * i + 1] = ptx::pack_bf16(w.z, w.w);
-      }
-      uint4* o4 = reinterpret_cast<uint4*>(ep.w16 + off);
-      o4[0] = make_uint4(p[0], p[1], p[2], p[3]);
-      o4[1] = make_uint4(p[4], p[5], p[6], p[7]);
-    } else {
-      uint32_t p[8];
-#pragma unroll
-      for (int i = 0; i < 8; ++i) p[i] = ptx::pack_bf16(v[2 * i], v[2 * i + 1]);
-      uint4* o4 = reinterpret_cast<uint4*>(reinterpret_cast<bf16*>(ep.out) + off);
-      o4[0] = make_uint4(p[0], p[1], p[2], p[3]);
-      o4[1] = make_uint4(p[4], p[5], p[6], p[7]);
-      if constexpr (EPI == EPI_BIAS_GELU) {
-#pragma unroll
-        for (int i = 0; i < 8; ++i) p[i] = ptx::pack_bf16(gelu_tanh(v[2 * i]), gelu_tanh(v[2 * i + 1]));
-        uint4* g4 = reinterpret_cast<uint4*>(ep.out2 + off);
-        g4[0] = make_uint4(p[0], p[1], p[2], p[3]);
-        g4[1] = make_uint4(p[4], p[5], p[6], p[7]);
-      }
+      ptx::tc_fence_before();
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(&tempty[acc]);
     }
   }
-  ptx::tc_fence_before();
   __syncthreads();
-  if (warp == 2) ptx::tmem_dealloc<BN>(tmem);
+  if (warp == 1) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc<512>(tmem);
+  }
+}
+
+// Fixed-order sum of the split-K partial tiles, then the final epilogue (EPI_F32 / EPI_SGD).
+template <int EPI>
+__global__ void splitk_reduce_kernel(int M, int N, int splits, GemmEpiParams ep) {
+  const size_t total = (size_t)M * N / 4;
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < total; i += (size_t)gridDim.x * blockDim.x) {
+    float4 acc = reinterpret_cast<const float4*>(ep.ws)[i];
+    for (int k = 1; k < splits; ++k) {
+      const float4 p = reinterpret_cast<const float4*>(ep.ws + (size_t)k * ep.ws_stride)[i];
+      acc.x += p.x; acc.y += p.y; acc.z += p.z; acc.w += p.w;
+    }
+    if constexpr (EPI == EPI_F32) {
+      reinterpret_cast<float4*>(ep.out)[i] = acc;
+    } else {
+      float4 w = reinterpret_cast<float4*>(ep.w32)[i];
+      w.x -= ep.lr * acc.x; w.y -= ep.lr * acc.y; w.z -= ep.lr * acc.z; w.w -= ep.lr * acc.w;
+      reinterpret_cast<float4*>(ep.w32)[i] = w;
+      uint2 o;
+      o.x = ptx::pack_bf16(w.x, w.y);
+      o.y = ptx::pack_bf16(w.z, w.w);
+      reinterpret_cast<uint2*>(ep.w16)[i] = o;
+    }
+  }
 }
 
 // ---------------------------------------------------------------- host side
@@ -244,35 +359,48 @@ CUtensorMap make_map(const bf16* base, uint64_t inner, uint64_t outer, uint64_t 
 
 std::atomic<uint64_t> g_gemm_launches{0};
 
-template <int BN, int STAGES, bool A_MN, bool B_MN, int EPI>
-void launch(cudaStream_t s, int M, int N, int K, const CUtensorMap& ta, const CUtensorMap& tb,
-            const GemmEpiParams& ep) {
-  using L = GemmSmem<BN, STAGES>;
-  auto kern = gemm_tc_kernel<BN, STAGES, A_MN, B_MN, EPI>;
-  static bool configured = false;  // per instantiation
-  if (!configured) {
-    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, L::TOTAL);
-    configured = true;
+int num_sms() {
+  static int n = 0;
+  if (!n) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    if (n <= 0) n = 148;
   }
-  dim3 grid((N + BN - 1) / BN, (M + BM - 1) / BM);
-  kern<<<grid, 128, L::TOTAL, s>>>(ta, tb, M, N, K, ep);
+  return n;
+}
+
+template <bool A_MN, bool B_MN, int EPI>
+void launch(cudaStream_t s, int M, int N, const TileSpace& ts, const CUtensorMap& ta, const CUtensorMap& tb,
+            const GemmEpiParams& ep) {
+  auto kern = gemm_tc_kernel<A_MN, B_MN, EPI>;
+  static uint32_t configured = 0;  // per instantiation, per device bit
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (!(configured & (1u << dev))) {
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_TOTAL);
+    configured |= 1u << dev;
+  }
+  const int tiles = ts.MT * ts.NT * ts.splits;
+  const int grid = std::min(tiles, num_sms());
+  kern<<<grid, THREADS, SMEM_TOTAL, s>>>(ta, tb, M, N, ts, ep);
   cudaError_t e = cudaGetLastError();
   NP_REQUIRE(e == cudaSuccess, NASPIPE_ECUDA, "gemm launch: %s", cudaGetErrorString(e));
   g_gemm_launches.fetch_add(1, std::memory_order_relaxed);
 }
 
 template <bool A_MN, bool B_MN>
-void dispatch_epi(cudaStream_t s, int M, int N, int K, const CUtensorMap& ta, const CUtensorMap& tb, int epi,
-                  const GemmEpiParams& ep) {
-  constexpr int BN = 128, ST = 3;
+void dispatch_epi(cudaStream_t s, int M, int N, const TileSpace& ts, const CUtensorMap& ta, const CUtensorMap& tb,
+                  int epi, const GemmEpiParams& ep) {
   switch (epi) {
-    case EPI_BF16: return launch<BN, ST, A_MN, B_MN, EPI_BF16>(s, M, N, K, ta, tb, ep);
-    case EPI_F32: return launch<BN, ST, A_MN, B_MN, EPI_F32>(s, M, N, K, ta, tb, ep);
-    case EPI_BIAS_BF16: return launch<BN, ST, A_MN, B_MN, EPI_BIAS_BF16>(s, M, N, K, ta, tb, ep);
-    case EPI_BIAS_RESID_F32: return launch<BN, ST, A_MN, B_MN, EPI_BIAS_RESID_F32>(s, M, N, K, ta, tb, ep);
-    case EPI_BIAS_GELU: return launch<BN, ST, A_MN, B_MN, EPI_BIAS_GELU>(s, M, N, K, ta, tb, ep);
-    case EPI_DGELU: return launch<BN, ST, A_MN, B_MN, EPI_DGELU>(s, M, N, K, ta, tb, ep);
-    case EPI_SGD: return launch<BN, ST, A_MN, B_MN, EPI_SGD>(s, M, N, K, ta, tb, ep);
+    case EPI_BF16: return launch<A_MN, B_MN, EPI_BF16>(s, M, N, ts, ta, tb, ep);
+    case EPI_F32: return launch<A_MN, B_MN, EPI_F32>(s, M, N, ts, ta, tb, ep);
+    case EPI_BIAS_BF16: return launch<A_MN, B_MN, EPI_BIAS_BF16>(s, M, N, ts, ta, tb, ep);
+    case EPI_BIAS_RESID_F32: return launch<A_MN, B_MN, EPI_BIAS_RESID_F32>(s, M, N, ts, ta, tb, ep);
+    case EPI_BIAS_GELU: return launch<A_MN, B_MN, EPI_BIAS_GELU>(s, M, N, ts, ta, tb, ep);
+    case EPI_DGELU: return launch<A_MN, B_MN, EPI_DGELU>(s, M, N, ts, ta, tb, ep);
+    case EPI_SGD: return launch<A_MN, B_MN, EPI_SGD>(s, M, N, ts, ta, tb, ep);
+    case EPI_PARTIAL: return launch<A_MN, B_MN, EPI_PARTIAL>(s, M, N, ts, ta, tb, ep);
     default: NP_REQUIRE(false, NASPIPE_EINVAL, "bad epilogue %d", epi);
   }
 }
@@ -281,18 +409,54 @@ void dispatch_epi(cudaStream_t s, int M, int N, int K, const CUtensorMap& ta, co
 
 uint64_t gemm_launch_count() { return g_gemm_launches.load(); }
 
+int gemm_splitk_factor(int M, int N, int K) {
+  const int tiles = ((M + BM - 1) / BM) * ((N + BN - 1) / BN);
+  const int nk = (K + BK - 1) / BK;
+  const int sms = num_sms();
+  // cost in k-block rounds (~0.3 us each): rounds * k-blocks per round, plus the fp32
+  // round trip of the split-K reduction ((s + 2.5) * M * N * 4 bytes at ~6 TB/s)
+  auto cost = [&](int s) {
+    const double rounds = (double)((tiles * s + sms - 1) / sms);
+    const double red_us = s > 1 ? (s + 2.5) * 4.0 * M * (double)N / 6e12 * 1e6 : 0.0;
+    return rounds * ((nk + s - 1) / s) + red_us / 0.3;
+  };
+  int best = 1;
+  for (int s = 2; s <= 4; s *= 2)
+    if (nk / s >= 8 && cost(s) < 0.9 * cost(best)) best = s;
+  return best;
+}
+
 void gemm_bf16_tc(cudaStream_t s, int M, int N, int K, const bf16* A, bool a_mn, int lda, const bf16* B,
-                  bool b_mn, int ldb, int epi, const GemmEpiParams& ep) {
+                  bool b_mn, int ldb, int epi, const GemmEpiParams& ep_in) {
   NP_REQUIRE(M > 0 && N > 0 && K > 0 && N % 16 == 0, NASPIPE_EINVAL, "gemm dims M=%d N=%d K=%d (N%%16)", M, N, K);
-  constexpr int BN = 128;
+  GemmEpiParams ep = ep_in;
   const CUtensorMap ta = a_mn ? make_map(A, (uint64_t)M, (uint64_t)K, (uint64_t)lda, BK)
                               : make_map(A, (uint64_t)K, (uint64_t)M, (uint64_t)lda, BM);
   const CUtensorMap tb = b_mn ? make_map(B, (uint64_t)N, (uint64_t)K, (uint64_t)ldb, BK)
                               : make_map(B, (uint64_t)K, (uint64_t)N, (uint64_t)ldb, BN);
-  if (!a_mn && !b_mn) return dispatch_epi<false, false>(s, M, N, K, ta, tb, epi, ep);
-  if (!a_mn && b_mn) return dispatch_epi<false, true>(s, M, N, K, ta, tb, epi, ep);
-  if (a_mn && b_mn) return dispatch_epi<true, true>(s, M, N, K, ta, tb, epi, ep);
-  return dispatch_epi<true, false>(s, M, N, K, ta, tb, epi, ep);
+  TileSpace ts;
+  ts.MT = (M + BM - 1) / BM;
+  ts.NT = (N + BN - 1) / BN;
+  ts.nk = (K + BK - 1) / BK;
+  ts.splits = 1;
+  if ((epi == EPI_SGD || epi == EPI_F32) && ep.ws != nullptr) {
+    ts.splits = gemm_splitk_factor(M, N, K);
+    if ((size_t)ts.splits * M * N > ep.ws_elems || (M * (size_t)N) % 4 != 0) ts.splits = 1;
+  }
+  ts.nk_per_split = (ts.nk + ts.splits - 1) / ts.splits;
+  const int run_epi = ts.splits > 1 ? EPI_PARTIAL : epi;
+  ep.ws_stride = (size_t)M * N;
+  if (!a_mn && !b_mn) dispatch_epi<false, false>(s, M, N, ts, ta, tb, run_epi, ep);
+  else if (!a_mn && b_mn) dispatch_epi<false, true>(s, M, N, ts, ta, tb, run_epi, ep);
+  else if (a_mn && b_mn) dispatch_epi<true, true>(s, M, N, ts, ta, tb, run_epi, ep);
+  else dispatch_epi<true, false>(s, M, N, ts, ta, tb, run_epi, ep);
+  if (ts.splits > 1) {
+    const int blocks = std::min<size_t>(((size_t)M * N / 4 + 255) / 256, 4 * (size_t)num_sms());
+    if (epi == EPI_F32) splitk_reduce_kernel<EPI_F32><<<blocks, 256, 0, s>>>(M, N, ts.splits, ep);
+    else splitk_reduce_kernel<EPI_SGD><<<blocks, 256, 0, s>>>(M, N, ts.splits, ep);
+    cudaError_t e = cudaGetLastError();
+    NP_REQUIRE(e == cudaSuccess, NASPIPE_ECUDA, "splitk reduce: %s", cudaGetErrorString(e));
+  }
 }
 
 }  // namespace naspipe

@@ -35,7 +35,13 @@ struct GemmEpiParams {
   float* w32 = nullptr;
   bf16* w16 = nullptr;
   float lr = 0.f;
+  // optional fp32 workspace enabling deterministic split-K for EPI_F32 / EPI_SGD
+  float* ws = nullptr;
+  size_t ws_elems = 0;
+  size_t ws_stride = 0;  // set by the launcher
 };
+// split-K factor the launcher uses for an (M, N, K) GEMM given a large enough workspace
+int gemm_splitk_factor(int M, int N, int K);
 void gemm_bf16_tc(cudaStream_t s, int M, int N, int K, const bf16* A, bool a_mn, int lda, const bf16* B,
                   bool b_mn, int ldb, int epi, const GemmEpiParams& ep);
 // number of tcgen05 GEMM launches so far in this process (stats)
@@ -68,6 +74,21 @@ void colsum_bf16(cudaStream_t s, const bf16* X, float* part, int T, int N);
 void cast_colsum(cudaStream_t s, const float* X, bf16* X16, float* part, int T, int N);
 // p[i] -= lr * sum_{j < nblk} part[j * n + i]   (fixed order)
 void sgd_from_partials(cudaStream_t s, float* p, const float* part, int nblk, int n, float lr);
+// Several of the above in one launch.  The sum is split into 8 fixed row groups of
+// ceil(nblk/8) partials each, combined in group order — fixed for a given (nblk, n), so a
+// parameter's update is bitwise independent of which stage or launch computes it.
+struct SgdJob {
+  float* p;
+  const float* part;
+  int nblk, n;
+};
+constexpr int kMaxSgdJobs = 8;
+struct SgdJobs {
+  SgdJob job[kMaxSgdJobs];
+  int count;
+  float lr;
+};
+void sgd_multi(cudaStream_t s, const SgdJobs& jobs);
 // w16 = bf16(w32), n elements
 void f32_to_bf16(cudaStream_t s, const float* w32, bf16* w16, size_t n);
 // loss[0] = mean((y - t)^2); dy = 2 (y - t) / n.  part: workspace of mse_blocks(n) floats

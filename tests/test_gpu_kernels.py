@@ -56,7 +56,7 @@ def _gemm(M, N, K, A, a_mn, B, b_mn, epi, **kw):
     torch.cuda.synchronize()
 
 
-SHAPES = [(128, 128, 64), (256, 384, 512), (304, 208, 200), (4096, 1024, 1024)]
+SHAPES = [(128, 128, 64), (256, 384, 512), (304, 208, 200), (4096, 1024, 1024), (256, 512, 4096)]  # last: split-K
 
 
 @pytest.mark.parametrize("M,N,K", SHAPES)
