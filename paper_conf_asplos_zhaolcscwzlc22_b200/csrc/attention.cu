@@ -20,15 +20,22 @@ struct AttnCfg {
   static constexpr int LDS = SMAX + 8;
 };
 
-// cooperative copy of S rows x HD cols (bf16) from global (row pitch ld) into smem (pitch LDH)
+// cooperative asynchronous copy (cp.async, 16 B per request, all requests in flight) of S
+// rows x HD cols (bf16) from global (row pitch ld) into smem (pitch LDH); completes at
+// cp_async_wait_all() + __syncthreads()
 template <int HD>
 __device__ __forceinline__ void load_tile(bf16* dst, const bf16* src, int S, int ld) {
   constexpr int CH = HD / 8;  // 16-byte chunks per row
   for (int i = threadIdx.x; i < S * CH; i += blockDim.x) {
     const int r = i / CH, c = i % CH;
-    *reinterpret_cast<uint4*>(dst + r * AttnCfg<HD>::LDH + c * 8) =
-        *reinterpret_cast<const uint4*>(src + (size_t)r * ld + c * 8);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(
+                     ptx::smem_u32(dst + r * AttnCfg<HD>::LDH + c * 8)),
+                 "l"(src + (size_t)r * ld + c * 8)
+                 : "memory");
   }
+}
+__device__ __forceinline__ void cp_async_wait_all() {
+  asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
 }
 
 // A fragment (16x16) at rows r0, cols k0 of a row-major smem tile with pitch ld
@@ -93,6 +100,7 @@ __global__ void __launch_bounds__(256) attn_fwd_kernel(const bf16* __restrict__ 
   load_tile<HD>(Qs, base, S, (int)ld);
   load_tile<HD>(Ks, base + d, S, (int)ld);
   load_tile<HD>(Vs, base + 2 * d, S, (int)ld);
+  cp_async_wait_all();
   __syncthreads();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
   const int r0 = warp * 16;
@@ -184,13 +192,31 @@ __global__ void __launch_bounds__(256) attn_bwd_kernel(const bf16* __restrict__ 
   load_tile<HD>(Ks, base + d, S, (int)ld);
   load_tile<HD>(Vs, base + 2 * d, S, (int)ld);
   load_tile<HD>(dOs, dout + (size_t)b * S * d + hh * HD, S, d);
+  bf16* Os = Ps;  // O is staged in the P buffer (free until phase 1 writes P)
+  static_assert(C::LDS >= C::LDH, "O staging must fit the P rows");
+  {
+    constexpr int CH = HD / 8;
+    const bf16* osrc = o + (size_t)b * S * d + hh * HD;
+    for (int i = threadIdx.x; i < S * CH; i += blockDim.x) {
+      const int r = i / CH, c = i % CH;
+      asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(ptx::smem_u32(Os + r * C::LDS + c * 8)),
+                   "l"(osrc + (size_t)r * d + c * 8)
+                   : "memory");
+    }
+  }
+  cp_async_wait_all();
+  __syncthreads();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
   // Di = rowsum(dO * O) (fp32), one warp per row, fixed lane order
   for (int r = warp; r < S; r += NWARP) {
-    const bf16* orow = o + ((size_t)b * S + r) * d + hh * HD;
-    const bf16* drow = dout + ((size_t)b * S + r) * d + hh * HD;
+    const bf16* orow = Os + r * C::LDS;
+    const bf16* drow = dOs + r * C::LDH;
     float acc = 0.f;
-    for (int c = lane; c < HD; c += 32) acc += __bfloat162float(orow[c]) * __bfloat162float(drow[c]);
+    for (int c = 2 * lane; c < HD; c += 64) {
+      const float2 ov = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(orow + c));
+      const float2 dv = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(drow + c));
+      acc += ov.x * dv.x + ov.y * dv.y;
+    }
 #pragma unroll
     for (int s = 16; s >= 1; s >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, s);
     if (lane == 0) Di[r] = acc;

@@ -9,7 +9,6 @@
 namespace naspipe {
 namespace {
 
-constexpr int LN_ROWS = 16;    // rows per block in ln_bwd partials
 constexpr int CS_ROWS = 64;    // rows per block in colsum partials
 
 inline void check_launch(const char* what) {
@@ -23,103 +22,6 @@ __device__ __forceinline__ float warp_sum(float v) {
   return v;
 }
 
-// ---------------------------------------------------------------- LayerNorm forward
-// one warp per row; d % 4 == 0
-__global__ void ln_fwd_kernel(const float* __restrict__ x, const float* __restrict__ g, const float* __restrict__ b,
-                              bf16* __restrict__ y, float* __restrict__ mean, float* __restrict__ rstd, int T, int d) {
-  const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
-  if (warp >= T) return;
-  const float4* xr = reinterpret_cast<const float4*>(x + (size_t)warp * d);
-  const int n4 = d / 4;
-  float s = 0.f;
-  for (int i = lane; i < n4; i += 32) {
-    const float4 v = xr[i];
-    s += (v.x + v.y) + (v.z + v.w);
-  }
-  const float mu = warp_sum(s) / (float)d;
-  float q = 0.f;
-  for (int i = lane; i < n4; i += 32) {
-    const float4 v = xr[i];
-    const float a = v.x - mu, bb = v.y - mu, c = v.z - mu, e = v.w - mu;
-    q += (a * a + bb * bb) + (c * c + e * e);
-  }
-  const float var = warp_sum(q) / (float)d;
-  const float rs = rsqrtf(var + 1e-5f);
-  const float4* g4 = reinterpret_cast<const float4*>(g);
-  const float4* b4 = reinterpret_cast<const float4*>(b);
-  uint2* yr = reinterpret_cast<uint2*>(y + (size_t)warp * d);
-  for (int i = lane; i < n4; i += 32) {
-    const float4 v = xr[i], gg = g4[i], bb = b4[i];
-    uint2 o;
-    o.x = ptx::pack_bf16((v.x - mu) * rs * gg.x + bb.x, (v.y - mu) * rs * gg.y + bb.y);
-    o.y = ptx::pack_bf16((v.z - mu) * rs * gg.z + bb.z, (v.w - mu) * rs * gg.w + bb.w);
-    yr[i] = o;
-  }
-  if (lane == 0) {
-    mean[warp] = mu;
-    rstd[warp] = rs;
-  }
-}
-
-// ---------------------------------------------------------------- LayerNorm backward
-// Phase 1 (warp per row): dx = resid + rstd (dxh - mean(dxh) - xhat mean(dxh xhat)), dxh = dy g.
-// Phase 2 (thread per column): partial dgamma, dbeta, colsum(dx) over the block's rows.
-__global__ void ln_bwd_kernel(const float* __restrict__ dy, const float* __restrict__ x,
-                              const float* __restrict__ mean, const float* __restrict__ rstd,
-                              const float* __restrict__ g, const float* __restrict__ resid, float* __restrict__ dx,
-                              bf16* __restrict__ dx16, float* __restrict__ pdg, float* __restrict__ pdb,
-                              float* __restrict__ pcs, int T, int d) {
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
-  const int r_begin = blockIdx.x * LN_ROWS, r_end = min(T, r_begin + LN_ROWS);
-  const int n4 = d / 4;
-  for (int r = r_begin + warp; r < r_end; r += nw) {
-    const float mu = mean[r], rs = rstd[r];
-    const float4* xr = reinterpret_cast<const float4*>(x + (size_t)r * d);
-    const float4* dr = reinterpret_cast<const float4*>(dy + (size_t)r * d);
-    const float4* g4 = reinterpret_cast<const float4*>(g);
-    float s1 = 0.f, s2 = 0.f;
-    for (int i = lane; i < n4; i += 32) {
-      const float4 v = xr[i], dv = dr[i], gg = g4[i];
-      const float h0 = (v.x - mu) * rs, h1 = (v.y - mu) * rs, h2 = (v.z - mu) * rs, h3 = (v.w - mu) * rs;
-      const float e0 = dv.x * gg.x, e1 = dv.y * gg.y, e2 = dv.z * gg.z, e3 = dv.w * gg.w;
-      s1 += (e0 + e1) + (e2 + e3);
-      s2 += (e0 * h0 + e1 * h1) + (e2 * h2 + e3 * h3);
-    }
-    const float m1 = warp_sum(s1) / (float)d, m2 = warp_sum(s2) / (float)d;
-    const float4* rr = reinterpret_cast<const float4*>(resid + (size_t)r * d);
-    float4* outr = reinterpret_cast<float4*>(dx + (size_t)r * d);
-    for (int i = lane; i < n4; i += 32) {
-      const float4 v = xr[i], dv = dr[i], gg = g4[i], re = rr[i];
-      float4 o;
-      o.x = re.x + rs * (dv.x * gg.x - m1 - (v.x - mu) * rs * m2);
-      o.y = re.y + rs * (dv.y * gg.y - m1 - (v.y - mu) * rs * m2);
-      o.z = re.z + rs * (dv.z * gg.z - m1 - (v.z - mu) * rs * m2);
-      o.w = re.w + rs * (dv.w * gg.w - m1 - (v.w - mu) * rs * m2);
-      outr[i] = o;
-      if (dx16) {
-        uint2 p;
-        p.x = ptx::pack_bf16(o.x, o.y);
-        p.y = ptx::pack_bf16(o.z, o.w);
-        reinterpret_cast<uint2*>(dx16 + (size_t)r * d)[i] = p;
-      }
-    }
-  }
-  __syncthreads();
-  for (int c = threadIdx.x; c < d; c += blockDim.x) {
-    float ag = 0.f, ab = 0.f, ac = 0.f;
-    for (int r = r_begin; r < r_end; ++r) {
-      const float dv = dy[(size_t)r * d + c];
-      const float xh = (x[(size_t)r * d + c] - mean[r]) * rstd[r];
-      ag += dv * xh;
-      ab += dv;
-      if (pcs) ac += dx[(size_t)r * d + c];
-    }
-    pdg[(size_t)blockIdx.x * d + c] = ag;
-    pdb[(size_t)blockIdx.x * d + c] = ab;
-    if (pcs) pcs[(size_t)blockIdx.x * d + c] = ac;
-  }
-}
-
 // ---------------------------------------------------------------- column sums
 template <typename T>
 __device__ __forceinline__ float to_f(T v);
@@ -128,30 +30,26 @@ __device__ __forceinline__ float to_f<float>(float v) { return v; }
 template <>
 __device__ __forceinline__ float to_f<bf16>(bf16 v) { return __bfloat162float(v); }
 
-template <typename T>
-__global__ void colsum_kernel(const T* __restrict__ X, float* __restrict__ part, int T_rows, int N) {
-  const int c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= N) return;
+// thread = 8 consecutive bf16 columns (one 16-byte load per row), rows of the block in order
+__global__ void colsum_bf16_kernel(const bf16* __restrict__ X, float* __restrict__ part, int T_rows, int N) {
+  const int c8 = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c8 * 8 >= N) return;
   const int r0 = blockIdx.y * CS_ROWS, r1 = min(T_rows, r0 + CS_ROWS);
-  float acc = 0.f;
-  for (int r = r0; r < r1; ++r) acc += to_f<T>(X[(size_t)r * N + c]);
-  part[(size_t)blockIdx.y * N + c] = acc;
-}
-
-__global__ void cast_colsum_kernel(const float* __restrict__ X, bf16* __restrict__ X16, float* __restrict__ part,
-                                   int T_rows, int N) {
-  const int c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= N) return;
-  // same row grouping and order as ln_bwd's colsum partials, so a bias gradient is
-  // bitwise independent of whether its block sits at a stage boundary
-  const int r0 = blockIdx.y * LN_ROWS, r1 = min(T_rows, r0 + LN_ROWS);
-  float acc = 0.f;
+  float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+#pragma unroll 8
   for (int r = r0; r < r1; ++r) {
-    const float v = X[(size_t)r * N + c];
-    X16[(size_t)r * N + c] = __float2bfloat16_rn(v);
-    acc += v;
+    uint4 q = reinterpret_cast<const uint4*>(X + (size_t)r * N)[c8];
+    const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&q);
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const float2 f = __bfloat1622float2(h[j]);
+      acc[2 * j] += f.x;
+      acc[2 * j + 1] += f.y;
+    }
   }
-  part[(size_t)blockIdx.y * N + c] = acc;
+  float4* o = reinterpret_cast<float4*>(part + (size_t)blockIdx.y * N + c8 * 8);
+  o[0] = make_float4(acc[0], acc[1], acc[2], acc[3]);
+  o[1] = make_float4(acc[4], acc[5], acc[6], acc[7]);
 }
 
 __global__ void sgd_partials_kernel(float* __restrict__ p, const float* __restrict__ part, int nblk, int n, float lr) {
@@ -284,37 +182,13 @@ __global__ void mlp_bwd_kernel(const float* __restrict__ x, const float* __restr
 
 }  // namespace
 
-void ln_fwd(cudaStream_t s, const float* x, const float* g, const float* b, bf16* y16, float* mean, float* rstd,
-            int T, int d) {
-  NP_REQUIRE(d % 4 == 0, NASPIPE_EINVAL, "ln d %% 4");
-  const int warps_per_block = 8;
-  ln_fwd_kernel<<<(T + warps_per_block - 1) / warps_per_block, 32 * warps_per_block, 0, s>>>(x, g, b, y16, mean,
-                                                                                              rstd, T, d);
-  check_launch("ln_fwd");
-}
-
-int ln_bwd_blocks(int T) { return (T + LN_ROWS - 1) / LN_ROWS; }
-
-void ln_bwd(cudaStream_t s, const float* dy, const float* x, const float* mean, const float* rstd, const float* g,
-            const float* resid, float* dx, bf16* dx16, float* part_dg, float* part_db, float* part_colsum, int T,
-            int d) {
-  ln_bwd_kernel<<<ln_bwd_blocks(T), 256, 0, s>>>(dy, x, mean, rstd, g, resid, dx, dx16, part_dg, part_db,
-                                                 part_colsum, T, d);
-  check_launch("ln_bwd");
-}
-
 int colsum_blocks(int T) { return (T + CS_ROWS - 1) / CS_ROWS; }
 
 void colsum_bf16(cudaStream_t s, const bf16* X, float* part, int T, int N) {
-  dim3 grid((N + 255) / 256, colsum_blocks(T));
-  colsum_kernel<bf16><<<grid, 256, 0, s>>>(X, part, T, N);
+  NP_REQUIRE(N % 8 == 0, NASPIPE_EINVAL, "colsum width %d must be a multiple of 8", N);
+  dim3 grid((N / 8 + 127) / 128, colsum_blocks(T));
+  colsum_bf16_kernel<<<grid, 128, 0, s>>>(X, part, T, N);
   check_launch("colsum");
-}
-
-void cast_colsum(cudaStream_t s, const float* X, bf16* X16, float* part, int T, int N) {
-  dim3 grid((N + 255) / 256, ln_bwd_blocks(T));
-  cast_colsum_kernel<<<grid, 256, 0, s>>>(X, X16, part, T, N);
-  check_launch("cast_colsum");
 }
 
 void sgd_from_partials(cudaStream_t s, float* p, const float* part, int nblk, int n, float lr) {
