@@ -178,36 +178,49 @@ class TfFamily : public Family {
         t.lse = A.alloc<float>((size_t)B_ * hmax_ * S_);
         t.x1 = A.alloc<float>(Td);
       }
-    // backward workspace (tasks on a stage are serialised on its stream)
-    dy16_ = A.alloc<bf16>(Td);
-    dz_ = A.alloc<bf16>((size_t)T_ * fmax_);
+    // backward workspace (tasks on a stage are serialised on its stream).  Buffers the side
+    // stream reads are double buffered by block parity (see backward()).
+    for (int p = 0; p < 2; ++p) {
+      dy16_[p] = A.alloc<bf16>(Td);
+      dz_[p] = A.alloc<bf16>((size_t)T_ * fmax_);
+      dx1_16_[p] = A.alloc<bf16>(Td);
+      dqkv_[p] = A.alloc<bf16>(3 * Td);
+    }
     da_ = A.alloc<float>(Td);
     dx1_ = A.alloc<float>(Td);
-    dx1_16_ = A.alloc<bf16>(Td);
     do16_ = A.alloc<bf16>(Td);
-    dqkv_ = A.alloc<bf16>(3 * Td);
     gb_[0] = A.alloc<float>(Td);
     gb_[1] = A.alloc<float>(Td);
-    // split-K workspace: the largest splits * M * N over this stage's GEMMs
+    // split-K workspace (side stream only): the largest splits * M * N of the wgrad GEMMs
     ws_elems_ = 0;
     for (int c = 0; c < n; ++c) {
       const int f = spec.ffn[c], T = T_, d = d_;
-      const int shp[6][3] = {{d, f, T}, {f, d, T}, {d, d, T}, {3 * d, d, T}, {T, d, f}, {T, d, 3 * d}};
+      const int shp[4][3] = {{d, f, T}, {f, d, T}, {d, d, T}, {3 * d, d, T}};
       for (auto& q : shp)
         ws_elems_ = std::max(ws_elems_, (size_t)gemm_splitk_factor(q[0], q[1], q[2]) * q[0] * q[1]);
     }
     ws_ = A.alloc<float>(ws_elems_);
     csb_ = colsum_blocks(T_);
     lnb_ = ln_bwd_blocks(T_);
-    const int pb = std::max(csb_, lnb_);
-    p_db2_ = A.alloc<float>((size_t)pb * d_);
-    p_db1_ = A.alloc<float>((size_t)csb_ * fmax_);
-    p_dbo_ = A.alloc<float>((size_t)lnb_ * d_);
-    p_dbqkv_ = A.alloc<float>((size_t)csb_ * 3 * d_);
+    for (int p = 0; p < 2; ++p) {
+      p_db2_[p] = A.alloc<float>((size_t)lnb_ * d_);
+      p_db1_[p] = A.alloc<float>((size_t)csb_ * fmax_);
+      p_dbo_[p] = A.alloc<float>((size_t)lnb_ * d_);
+      p_dbqkv_[p] = A.alloc<float>((size_t)csb_ * 3 * d_);
+      p_g2_[p] = A.alloc<float>((size_t)lnb_ * d_);
+      p_b2_[p] = A.alloc<float>((size_t)lnb_ * d_);
+    }
     p_g1_ = A.alloc<float>((size_t)lnb_ * d_);
     p_b1_ = A.alloc<float>((size_t)lnb_ * d_);
-    p_g2_ = A.alloc<float>((size_t)lnb_ * d_);
-    p_b2_ = A.alloc<float>((size_t)lnb_ * d_);
+    cudaStreamCreateWithFlags(&side_, cudaStreamNonBlocking);
+    for (auto* e : {&ev_dz_, &ev_da2_, &ev_do_, &ev_da_, &ev_done_[0], &ev_done_[1], &ev_join_})
+      cudaEventCreateWithFlags(e, cudaEventDisableTiming);
+  }
+
+  ~TfFamily() override {
+    cudaStreamSynchronize(side_);
+    for (auto e : {ev_dz_, ev_da2_, ev_do_, ev_da_, ev_done_[0], ev_done_[1], ev_join_}) cudaEventDestroy(e);
+    cudaStreamDestroy(side_);
   }
 
   float* master(int j, int c) override { return w32_[(size_t)j * spec_.n() + c]; }
@@ -236,34 +249,45 @@ class TfFamily : public Family {
     }
   }
 
+  // Backward of the stage.  The dgrad chain (dz -> da2 -> LN2' -> do -> attention' -> da ->
+  // LN1') runs on the stage stream; each weight-gradient GEMM (with its fused SGD WRITE),
+  // the bias column sums and the bias/LN2 updates run on a side stream as soon as the dgrad
+  // that read the pre-update weight is done (reading A4), filling the SMs the dgrad chain
+  // leaves idle.  Buffers the side stream reads are double-buffered by block parity; the
+  // stage stream joins the side stream before the task ends.
   void backward(int slot, const int32_t* ch, const float* dy, float* dx, cudaStream_t s) override {
     const int nb = (int)blocks_.size();
     const float* g = dy;
     int db2_nblk = 0;
     for (int j = nb - 1; j >= 0; --j) {
       const int c = ch[blocks_[j]];
+      const int p = j & 1;
       TfSlot& t = slots_[(size_t)slot * nb + j];
       if (j == nb - 1) {  // grad entering the stage: bf16 copy + colsum for b2
-        cast_colsum(s, g, dy16_, p_db2_, T_, d_);
+        cast_colsum(s, g, dy16_[p], p_db2_[p], T_, d_);
         counters.launches++;
         db2_nblk = lnb_;
       }
       // stage 0 needs no input gradient, but LN1's backward still runs (dgamma/dbeta):
       // its dx goes to a scratch buffer (gb_[0] is free: block 1 wrote gb_[1])
       float* out = (j == 0) ? (dx ? dx : gb_[0]) : gb_[j & 1];
-      block_bwd(j, c, t, g, out, /*want_next=*/j > 0, db2_nblk, s);
+      block_bwd(j, c, t, g, out, /*want_next=*/j > 0, db2_nblk, p, s);
       db2_nblk = lnb_;
       g = out;
     }
+    cudaEventRecord(ev_join_, side_);
+    cudaStreamWaitEvent(s, ev_join_, 0);
   }
 
  private:
   void gemm(cudaStream_t s, int M, int N, int K, const bf16* A, bool amn, int lda, const bf16* B, bool bmn, int ldb,
-            int epi, const GemmEpiParams& ep) {
+            int epi, const GemmEpiParams& ep, bool split_ok = false) {
     if (timer) timer->begin(s);
     GemmEpiParams e = ep;
-    e.ws = ws_;
-    e.ws_elems = ws_elems_;
+    if (split_ok) {  // only the side stream owns the split-K workspace
+      e.ws = ws_;
+      e.ws_elems = ws_elems_;
+    }
     gemm_bf16_tc(s, M, N, K, A, amn, lda, B, bmn, ldb, epi, e);
     if (timer) timer->end(s, 2.0 * M * N * K);
     counters.launches++;
@@ -301,68 +325,70 @@ class TfFamily : public Family {
     counters.launches += 3;
   }
 
-  // dy: f32 grad of the block output (its bf16 copy is in dy16_, its column partials in
-  // p_db2_[0..db2_nblk)); writes dx (f32); if want_next also dy16_/p_db2_ for block j-1.
-  void block_bwd(int j, int c, TfSlot& t, const float* dy, float* dx, bool want_next, int db2_nblk,
+  // dy: f32 grad of the block output (its bf16 copy is in dy16_[p], its column partials in
+  // p_db2_[p][0..db2_nblk)); writes dx (f32); if want_next also dy16_/p_db2_[p^1] for block j-1.
+  void block_bwd(int j, int c, TfSlot& t, const float* dy, float* dx, bool want_next, int db2_nblk, int p,
                  cudaStream_t s) {
     const TfOffsets o = spec_.tf_offsets(c);
     const int d = d_, f = spec_.ffn[c], h = spec_.heads[c], T = T_;
     float* P = master(j, c);
     bf16* W = w16_[(size_t)j * spec_.n() + c];
     bf16 *Wqkv = W, *Wo = W + 3 * (size_t)d * d, *W1 = W + 4 * (size_t)d * d, *W2 = W1 + (size_t)f * d;
-    // FFN half
+    auto sgd_ep = [&](float* w32, bf16* w16) {
+      GemmEpiParams e;
+      e.w32 = w32;
+      e.w16 = w16;
+      e.lr = lr_;
+      return e;
+    };
+    // ---- FFN half
     GemmEpiParams e;
     e.aux16 = t.z;
-    e.out = dz_;
-    gemm(s, T, f, d, dy16_, false, d, W2, true, f, EPI_DGELU, e);          // dz = (dy W2) * gelu'(z)
-    e = GemmEpiParams();
-    e.w32 = P + o.W2;
-    e.w16 = W2;
-    e.lr = lr_;
-    gemm(s, d, f, T, dy16_, true, d, t.g, true, f, EPI_SGD, e);            // W2 -= lr dy^T g
-    colsum_bf16(s, dz_, p_db1_, T, f);
+    e.out = dz_[p];
+    gemm(s, T, f, d, dy16_[p], false, d, W2, true, f, EPI_DGELU, e);        // dz = (dy W2) * gelu'(z)
+    cudaEventRecord(ev_dz_, s);
+    cudaStreamWaitEvent(side_, ev_dz_, 0);
+    gemm(side_, d, f, T, dy16_[p], true, d, t.g, true, f, EPI_SGD, sgd_ep(P + o.W2, W2), true);  // W2 -= lr dy^T g
+    colsum_bf16(side_, dz_[p], p_db1_[p], T, f);
     e = GemmEpiParams();
     e.out = da_;
-    gemm(s, T, d, f, dz_, false, f, W1, true, d, EPI_F32, e);               // da2 = dz W1
-    e = GemmEpiParams();
-    e.w32 = P + o.W1;
-    e.w16 = W1;
-    e.lr = lr_;
-    gemm(s, f, d, T, dz_, true, f, t.a2, true, d, EPI_SGD, e);             // W1 -= lr dz^T a2
-    ln_bwd(s, da_, t.x1, t.mean2, t.rstd2, P + o.ln2g, dy, dx1_, dx1_16_, p_g2_, p_b2_, p_dbo_, T, d);
-    // attention half
+    gemm(s, T, d, f, dz_[p], false, f, W1, true, d, EPI_F32, e);             // da2 = dz W1
+    cudaEventRecord(ev_da2_, s);
+    cudaStreamWaitEvent(side_, ev_da2_, 0);
+    gemm(side_, f, d, T, dz_[p], true, f, t.a2, true, d, EPI_SGD, sgd_ep(P + o.W1, W1), true);  // W1 -= lr dz^T a2
+    ln_bwd(s, da_, t.x1, t.mean2, t.rstd2, P + o.ln2g, dy, dx1_, dx1_16_[p], p_g2_[p], p_b2_[p], p_dbo_[p], T, d);
+    // ---- attention half
     e = GemmEpiParams();
     e.out = do16_;
-    gemm(s, T, d, d, dx1_16_, false, d, Wo, true, d, EPI_BF16, e);          // do = dx1 Wo
-    e = GemmEpiParams();
-    e.w32 = P + o.Wo;
-    e.w16 = Wo;
-    e.lr = lr_;
-    gemm(s, d, d, T, dx1_16_, true, d, t.o, true, d, EPI_SGD, e);          // Wo -= lr dx1^T o
-    attn_bwd(s, t.qkv, t.o, t.lse, do16_, dqkv_, B_, S_, d, h);
-    colsum_bf16(s, dqkv_, p_dbqkv_, T, 3 * d);
+    gemm(s, T, d, d, dx1_16_[p], false, d, Wo, true, d, EPI_BF16, e);        // do = dx1 Wo
+    cudaEventRecord(ev_do_, s);
+    cudaStreamWaitEvent(side_, ev_do_, 0);
+    gemm(side_, d, d, T, dx1_16_[p], true, d, t.o, true, d, EPI_SGD, sgd_ep(P + o.Wo, Wo), true);  // Wo -= lr dx1^T o
+    attn_bwd(s, t.qkv, t.o, t.lse, do16_, dqkv_[p], B_, S_, d, h);
     e = GemmEpiParams();
     e.out = da_;
-    gemm(s, T, d, 3 * d, dqkv_, false, 3 * d, Wqkv, true, d, EPI_F32, e);  // da = dqkv Wqkv
-    e = GemmEpiParams();
-    e.w32 = P + o.Wqkv;
-    e.w16 = Wqkv;
-    e.lr = lr_;
-    gemm(s, 3 * d, d, T, dqkv_, true, 3 * d, t.a, true, d, EPI_SGD, e);    // Wqkv -= lr dqkv^T a
-    // bias / LN2 updates (their partials are complete; LN1 partials come next)
+    gemm(s, T, d, 3 * d, dqkv_[p], false, 3 * d, Wqkv, true, d, EPI_F32, e);  // da = dqkv Wqkv
+    cudaEventRecord(ev_da_, s);
+    cudaStreamWaitEvent(side_, ev_da_, 0);
+    colsum_bf16(side_, dqkv_[p], p_dbqkv_[p], T, 3 * d);
+    gemm(side_, 3 * d, d, T, dqkv_[p], true, 3 * d, t.a, true, d, EPI_SGD, sgd_ep(P + o.Wqkv, Wqkv), true);
+    // bias / LN2 updates (all their partials are complete)
     SgdJobs j1{};
     j1.lr = lr_;
-    j1.job[0] = {P + o.b2, p_db2_, db2_nblk, d};
-    j1.job[1] = {P + o.b1, p_db1_, csb_, f};
-    j1.job[2] = {P + o.bo, p_dbo_, lnb_, d};
-    j1.job[3] = {P + o.bqkv, p_dbqkv_, csb_, 3 * d};
-    j1.job[4] = {P + o.ln2g, p_g2_, lnb_, d};
-    j1.job[5] = {P + o.ln2b, p_b2_, lnb_, d};
+    j1.job[0] = {P + o.b2, p_db2_[p], db2_nblk, d};
+    j1.job[1] = {P + o.b1, p_db1_[p], csb_, f};
+    j1.job[2] = {P + o.bo, p_dbo_[p], lnb_, d};
+    j1.job[3] = {P + o.bqkv, p_dbqkv_[p], csb_, 3 * d};
+    j1.job[4] = {P + o.ln2g, p_g2_[p], lnb_, d};
+    j1.job[5] = {P + o.ln2b, p_b2_[p], lnb_, d};
     j1.count = 6;
-    sgd_multi(s, j1);
-    // LN1 backward: dx = dx1 + LN1'(da); bf16 copy / column partials feed block j-1
-    ln_bwd(s, da_, t.xin, t.mean1, t.rstd1, P + o.ln1g, dx1_, dx, want_next ? dy16_ : nullptr, p_g1_, p_b1_,
-           want_next ? p_db2_ : nullptr, T, d);
+    sgd_multi(side_, j1);
+    cudaEventRecord(ev_done_[p], side_);
+    // LN1 backward: dx = dx1 + LN1'(da); its bf16 copy / column partials feed block j-1 and
+    // go to the other parity's buffers, whose last reader (block j+1's side work) must be done
+    cudaStreamWaitEvent(s, ev_done_[p ^ 1], 0);
+    ln_bwd(s, da_, t.xin, t.mean1, t.rstd1, P + o.ln1g, dx1_, dx, want_next ? dy16_[p ^ 1] : nullptr, p_g1_, p_b1_,
+           want_next ? p_db2_[p ^ 1] : nullptr, T, d);
     SgdJobs j2{};
     j2.lr = lr_;
     j2.job[0] = {P + o.ln1g, p_g1_, lnb_, d};
@@ -379,10 +405,12 @@ class TfFamily : public Family {
   std::vector<float*> w32_;
   std::vector<bf16*> w16_;
   std::vector<TfSlot> slots_;
-  bf16 *dy16_, *dz_, *dx1_16_, *do16_, *dqkv_;
+  bf16 *dy16_[2], *dz_[2], *dx1_16_[2], *dqkv_[2], *do16_;
   float *da_, *dx1_, *gb_[2], *ws_ = nullptr;
   size_t ws_elems_ = 0;
-  float *p_db2_, *p_db1_, *p_dbo_, *p_dbqkv_, *p_g1_, *p_b1_, *p_g2_, *p_b2_;
+  float *p_db2_[2], *p_db1_[2], *p_dbo_[2], *p_dbqkv_[2], *p_g2_[2], *p_b2_[2], *p_g1_, *p_b1_;
+  cudaStream_t side_ = nullptr;
+  cudaEvent_t ev_dz_, ev_da2_, ev_do_, ev_da_, ev_done_[2], ev_join_;
 };
 
 }  // namespace
