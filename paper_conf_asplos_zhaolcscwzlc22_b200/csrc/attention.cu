@@ -6,6 +6,7 @@
 // tcgen05 path.
 #include "common.h"
 #include "kernels.h"
+#include "launch.h"
 #include "ptx.cuh"
 
 namespace naspipe {
@@ -97,6 +98,7 @@ __global__ void __launch_bounds__(256) attn_fwd_kernel(const bf16* __restrict__ 
   const int bh = blockIdx.x, b = bh / h, hh = bh % h;
   const size_t ld = 3 * (size_t)d;
   const bf16* base = qkv + (size_t)b * S * ld + hh * HD;
+  ptx::pdl_wait();
   load_tile<HD>(Qs, base, S, (int)ld);
   load_tile<HD>(Ks, base + d, S, (int)ld);
   load_tile<HD>(Vs, base + 2 * d, S, (int)ld);
@@ -188,6 +190,7 @@ __global__ void __launch_bounds__(256) attn_bwd_kernel(const bf16* __restrict__ 
   const int bh = blockIdx.x, b = bh / h, hh = bh % h;
   const size_t ld = 3 * (size_t)d;
   const bf16* base = qkv + (size_t)b * S * ld + hh * HD;
+  ptx::pdl_wait();
   load_tile<HD>(Qs, base, S, (int)ld);
   load_tile<HD>(Ks, base + d, S, (int)ld);
   load_tile<HD>(Vs, base + 2 * d, S, (int)ld);
@@ -330,14 +333,14 @@ template <int HD>
 void fwd_launch(cudaStream_t s, const bf16* qkv, bf16* o, float* lse, int B, int S, int d, int h) {
   const int smem = 3 * SMAX * AttnCfg<HD>::LDH * 2;
   cudaFuncSetAttribute(attn_fwd_kernel<HD>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  attn_fwd_kernel<HD><<<B * h, 256, smem, s>>>(qkv, o, lse, S, d, h);
+  launch_pdl(attn_fwd_kernel<HD>, dim3(B * h), dim3(256), smem, s, qkv, o, lse, S, d, h);
 }
 template <int HD>
 void bwd_launch(cudaStream_t s, const bf16* qkv, const bf16* o, const float* lse, const bf16* dout, bf16* dqkv,
                 int B, int S, int d, int h) {
   const int smem = 4 * SMAX * AttnCfg<HD>::LDH * 2 + 2 * SMAX * AttnCfg<HD>::LDS * 2 + SMAX * 4;
   cudaFuncSetAttribute(attn_bwd_kernel<HD>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  attn_bwd_kernel<HD><<<B * h, 256, smem, s>>>(qkv, o, lse, dout, dqkv, S, d, h);
+  launch_pdl(attn_bwd_kernel<HD>, dim3(B * h), dim3(256), smem, s, qkv, o, lse, dout, dqkv, S, d, h);
 }
 
 #define NP_HD_DISPATCH(HDV, CALL) \

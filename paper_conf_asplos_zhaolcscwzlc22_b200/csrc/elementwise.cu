@@ -4,6 +4,7 @@
 // floating-point atomics, so every result is bitwise reproducible.
 #include "common.h"
 #include "kernels.h"
+#include "launch.h"
 #include "ptx.cuh"
 
 namespace naspipe {
@@ -32,6 +33,7 @@ __device__ __forceinline__ float to_f<bf16>(bf16 v) { return __bfloat162float(v)
 
 // thread = 8 consecutive bf16 columns (one 16-byte load per row), rows of the block in order
 __global__ void colsum_bf16_kernel(const bf16* __restrict__ X, float* __restrict__ part, int T_rows, int N) {
+  ptx::pdl_wait();
   const int c8 = blockIdx.x * blockDim.x + threadIdx.x;
   if (c8 * 8 >= N) return;
   const int r0 = blockIdx.y * CS_ROWS, r1 = min(T_rows, r0 + CS_ROWS);
@@ -63,6 +65,7 @@ __global__ void sgd_partials_kernel(float* __restrict__ p, const float* __restri
 // 32 columns x 8 row-groups per block; group g sums partials [g*G, (g+1)*G) in order, the 8
 // group sums are added in group order.
 __global__ void sgd_multi_kernel(SgdJobs jobs) {
+  ptx::pdl_wait();
   const SgdJob jb = jobs.job[blockIdx.y];
   const int lane = threadIdx.x & 31, grp = threadIdx.x >> 5;
   const int col = blockIdx.x * 32 + lane;
@@ -94,6 +97,7 @@ __global__ void f2bf_kernel(const float* __restrict__ a, bf16* __restrict__ b, s
 constexpr int MSE_THREADS = 256, MSE_PER_BLOCK = 8192;
 __global__ void mse_part_kernel(const float* __restrict__ y, const float* __restrict__ t, float* __restrict__ dy,
                                 float* __restrict__ part, size_t n, float two_over_n) {
+  ptx::pdl_wait();
   __shared__ float red[MSE_THREADS / 32];
   const size_t base = (size_t)blockIdx.x * MSE_PER_BLOCK;
   float acc = 0.f;
@@ -115,6 +119,7 @@ __global__ void mse_part_kernel(const float* __restrict__ y, const float* __rest
   }
 }
 __global__ void mse_final_kernel(const float* __restrict__ part, int nblk, float* __restrict__ loss, float inv_n) {
+  ptx::pdl_wait();
   if (threadIdx.x != 0) return;
   double s = 0.0;  // fixed order
   for (int j = 0; j < nblk; ++j) s += part[j];
@@ -187,7 +192,7 @@ int colsum_blocks(int T) { return (T + CS_ROWS - 1) / CS_ROWS; }
 void colsum_bf16(cudaStream_t s, const bf16* X, float* part, int T, int N) {
   NP_REQUIRE(N % 8 == 0, NASPIPE_EINVAL, "colsum width %d must be a multiple of 8", N);
   dim3 grid((N / 8 + 127) / 128, colsum_blocks(T));
-  colsum_bf16_kernel<<<grid, 128, 0, s>>>(X, part, T, N);
+  launch_pdl(colsum_bf16_kernel, grid, dim3(128), 0, s, X, part, T, N);
   check_launch("colsum");
 }
 
@@ -200,7 +205,7 @@ void sgd_multi(cudaStream_t s, const SgdJobs& jobs) {
   int nmax = 0;
   for (int i = 0; i < jobs.count; ++i) nmax = std::max(nmax, jobs.job[i].n);
   dim3 grid((nmax + 31) / 32, jobs.count);
-  sgd_multi_kernel<<<grid, 256, 0, s>>>(jobs);
+  launch_pdl(sgd_multi_kernel, grid, dim3(256), 0, s, jobs);
   check_launch("sgd_multi");
 }
 
@@ -214,8 +219,8 @@ int mse_blocks(size_t n) { return (int)((n + MSE_PER_BLOCK - 1) / MSE_PER_BLOCK)
 
 void mse_loss(cudaStream_t s, const float* y, const float* t, float* dy, float* part, float* loss, size_t n) {
   const int nb = mse_blocks(n);
-  mse_part_kernel<<<nb, MSE_THREADS, 0, s>>>(y, t, dy, part, n, 2.0f / (float)n);
-  mse_final_kernel<<<1, 32, 0, s>>>(part, nb, loss, (float)(1.0 / (double)n));
+  launch_pdl(mse_part_kernel, dim3(nb), dim3(MSE_THREADS), 0, s, y, t, dy, part, n, 2.0f / (float)n);
+  launch_pdl(mse_final_kernel, dim3(1), dim3(32), 0, s, part, nb, loss, (float)(1.0 / (double)n));
   check_launch("mse_loss");
 }
 

@@ -19,6 +19,7 @@
 
 #include "common.h"
 #include "kernels.h"
+#include "launch.h"
 #include "ptx.cuh"
 
 namespace naspipe {
@@ -181,6 +182,7 @@ __global__ void __launch_bounds__(THREADS, 1)
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_holder;
+  ptx::pdl_wait();  // predecessors' outputs (A, B, residual, ...) are visible from here
 
   if (warp == 0) {
     if (lane == 0) {  // ---------------- TMA producer
@@ -212,6 +214,7 @@ __global__ void __launch_bounds__(THREADS, 1)
         }
       }
     }
+    ptx::pdl_trigger();
   } else if (warp == 1) {
     if (lane == 0) {  // ---------------- MMA issuer
       constexpr uint32_t idesc = ptx::umma_idesc_bf16(BM, BN, A_MN ? 1 : 0, B_MN ? 1 : 0);
@@ -246,6 +249,7 @@ __global__ void __launch_bounds__(THREADS, 1)
         ptx::umma_commit(&tfull[acc]);  // accumulator ready for the epilogue
       }
     }
+    ptx::pdl_trigger();
   } else {
     // ---------------- epilogue warps 2..9: TMEM lane quarter (warp % 4), column half
     const int lane_base = 32 * (warp & 3);
@@ -257,6 +261,7 @@ __global__ void __launch_bounds__(THREADS, 1)
       const int acc = it & 1;
       ptx::mbar_wait(&tfull[acc], (it >> 1) & 1);
       ptx::tc_fence_after();
+      if (t + (int)gridDim.x >= n_tiles) ptx::pdl_trigger();  // last tile: let the next kernel launch
       const int row = tm * BM + lane_base + lane;
       const bool row_ok = row < M;
       const uint32_t taddr = tmem + ((uint32_t)lane_base << 16) + acc * BN;
@@ -300,6 +305,7 @@ __global__ void __launch_bounds__(THREADS, 1)
 // Fixed-order sum of the split-K partial tiles, then the final epilogue (EPI_F32 / EPI_SGD).
 template <int EPI>
 __global__ void splitk_reduce_kernel(int M, int N, int splits, GemmEpiParams ep) {
+  ptx::pdl_wait();
   const size_t total = (size_t)M * N / 4;
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < total; i += (size_t)gridDim.x * blockDim.x) {
     float4 acc = reinterpret_cast<const float4*>(ep.ws)[i];
@@ -383,9 +389,7 @@ void launch(cudaStream_t s, int M, int N, const TileSpace& ts, const CUtensorMap
   }
   const int tiles = ts.MT * ts.NT * ts.splits;
   const int grid = std::min(tiles, num_sms());
-  kern<<<grid, THREADS, SMEM_TOTAL, s>>>(ta, tb, M, N, ts, ep);
-  cudaError_t e = cudaGetLastError();
-  NP_REQUIRE(e == cudaSuccess, NASPIPE_ECUDA, "gemm launch: %s", cudaGetErrorString(e));
+  launch_pdl(kern, dim3(grid), dim3(THREADS), SMEM_TOTAL, s, ta, tb, M, N, ts, ep);
   g_gemm_launches.fetch_add(1, std::memory_order_relaxed);
 }
 
@@ -452,10 +456,8 @@ void gemm_bf16_tc(cudaStream_t s, int M, int N, int K, const bf16* A, bool a_mn,
   else dispatch_epi<true, false>(s, M, N, ts, ta, tb, run_epi, ep);
   if (ts.splits > 1) {
     const int blocks = std::min<size_t>(((size_t)M * N / 4 + 255) / 256, 4 * (size_t)num_sms());
-    if (epi == EPI_F32) splitk_reduce_kernel<EPI_F32><<<blocks, 256, 0, s>>>(M, N, ts.splits, ep);
-    else splitk_reduce_kernel<EPI_SGD><<<blocks, 256, 0, s>>>(M, N, ts.splits, ep);
-    cudaError_t e = cudaGetLastError();
-    NP_REQUIRE(e == cudaSuccess, NASPIPE_ECUDA, "splitk reduce: %s", cudaGetErrorString(e));
+    if (epi == EPI_F32) launch_pdl(splitk_reduce_kernel<EPI_F32>, dim3(blocks), dim3(256), 0, s, M, N, ts.splits, ep);
+    else launch_pdl(splitk_reduce_kernel<EPI_SGD>, dim3(blocks), dim3(256), 0, s, M, N, ts.splits, ep);
   }
 }
 

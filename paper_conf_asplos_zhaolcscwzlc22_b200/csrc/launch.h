@@ -1,0 +1,28 @@
+// Kernel launch with programmatic dependent launch (PDL) enabled: the launch of a kernel
+// overlaps the tail of the previous kernel in the stream; the kernel itself waits
+// (ptx::pdl_wait) before reading its predecessors' outputs.
+#pragma once
+#include <cuda_runtime.h>
+
+#include "common.h"
+
+namespace naspipe {
+
+template <typename... KArgs, typename... Args>
+inline void launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                       Args&&... args) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  const cudaError_t e = cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+  NP_REQUIRE(e == cudaSuccess, NASPIPE_ECUDA, "kernel launch: %s", cudaGetErrorString(e));
+}
+
+}  // namespace naspipe

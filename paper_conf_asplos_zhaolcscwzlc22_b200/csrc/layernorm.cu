@@ -11,6 +11,7 @@
 
 #include "common.h"
 #include "kernels.h"
+#include "launch.h"
 #include "ptx.cuh"
 
 namespace naspipe {
@@ -38,6 +39,7 @@ __global__ void __launch_bounds__(256) ln_fwd_kernel(const float* __restrict__ x
                                                      const float* __restrict__ b, bf16* __restrict__ y,
                                                      float* __restrict__ mean, float* __restrict__ rstd, int T, int d) {
   const int row = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  ptx::pdl_wait();
   if (row >= T) return;
   const int n4 = d / 4;
   const float4* xr = reinterpret_cast<const float4*>(x + (size_t)row * d);
@@ -92,6 +94,7 @@ __global__ void __launch_bounds__(256) ln_bwd_kernel(const float* __restrict__ d
                                                      float* __restrict__ pdg, float* __restrict__ pdb,
                                                      float* __restrict__ pcs, int T, int d) {
   __shared__ float s_m1[LN_ROWS], s_m2[LN_ROWS], s_mu[LN_ROWS], s_rs[LN_ROWS];
+  ptx::pdl_wait();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int n4 = d / 4, r0 = blockIdx.x * LN_ROWS;
   const int nrows = min(LN_ROWS, T - r0);
@@ -157,6 +160,7 @@ __global__ void __launch_bounds__(256) ln_bwd_kernel(const float* __restrict__ d
 // (ln_bwd's colsum order)
 __global__ void __launch_bounds__(256) cast_colsum_kernel(const float* __restrict__ X, bf16* __restrict__ X16,
                                                           float* __restrict__ part, int T, int d) {
+  ptx::pdl_wait();
   const int n4 = d / 4, r0 = blockIdx.x * LN_ROWS;
   const int nrows = min(LN_ROWS, T - r0);
   for (int c = threadIdx.x; c < n4; c += blockDim.x) {
@@ -189,11 +193,11 @@ void ln_fwd(cudaStream_t s, const float* x, const float* g, const float* b, bf16
             int T, int d) {
   const int grid = (T + 7) / 8;
   switch (vpl_for(d)) {
-    case 1: ln_fwd_kernel<1><<<grid, 256, 0, s>>>(x, g, b, y16, mean, rstd, T, d); break;
-    case 2: ln_fwd_kernel<2><<<grid, 256, 0, s>>>(x, g, b, y16, mean, rstd, T, d); break;
-    case 4: ln_fwd_kernel<4><<<grid, 256, 0, s>>>(x, g, b, y16, mean, rstd, T, d); break;
-    case 8: ln_fwd_kernel<8><<<grid, 256, 0, s>>>(x, g, b, y16, mean, rstd, T, d); break;
-    default: ln_fwd_kernel<16><<<grid, 256, 0, s>>>(x, g, b, y16, mean, rstd, T, d); break;
+    case 1: launch_pdl(ln_fwd_kernel<1>, dim3(grid), dim3(256), 0, s, x, g, b, y16, mean, rstd, T, d); break;
+    case 2: launch_pdl(ln_fwd_kernel<2>, dim3(grid), dim3(256), 0, s, x, g, b, y16, mean, rstd, T, d); break;
+    case 4: launch_pdl(ln_fwd_kernel<4>, dim3(grid), dim3(256), 0, s, x, g, b, y16, mean, rstd, T, d); break;
+    case 8: launch_pdl(ln_fwd_kernel<8>, dim3(grid), dim3(256), 0, s, x, g, b, y16, mean, rstd, T, d); break;
+    default: launch_pdl(ln_fwd_kernel<16>, dim3(grid), dim3(256), 0, s, x, g, b, y16, mean, rstd, T, d); break;
   }
   check_launch("ln_fwd");
 }
@@ -202,14 +206,14 @@ void ln_bwd(cudaStream_t s, const float* dy, const float* x, const float* mean, 
             const float* resid, float* dx, bf16* dx16, float* part_dg, float* part_db, float* part_colsum, int T,
             int d) {
   NP_REQUIRE(d % 4 == 0, NASPIPE_EINVAL, "LayerNorm width %d must be a multiple of 4", d);
-  ln_bwd_kernel<<<ln_bwd_blocks(T), 256, 0, s>>>(dy, x, mean, rstd, g, resid, dx, dx16, part_dg, part_db, part_colsum,
-                                                 T, d);
+  launch_pdl(ln_bwd_kernel, dim3(ln_bwd_blocks(T)), dim3(256), 0, s, dy, x, mean, rstd, g, resid, dx, dx16, part_dg,
+             part_db, part_colsum, T, d);
   check_launch("ln_bwd");
 }
 
 void cast_colsum(cudaStream_t s, const float* X, bf16* X16, float* part, int T, int N) {
   NP_REQUIRE(N % 4 == 0, NASPIPE_EINVAL, "cast_colsum width %d must be a multiple of 4", N);
-  cast_colsum_kernel<<<ln_bwd_blocks(T), 256, 0, s>>>(X, X16, part, T, N);
+  launch_pdl(cast_colsum_kernel, dim3(ln_bwd_blocks(T)), dim3(256), 0, s, X, X16, part, T, N);
   check_launch("cast_colsum");
 }
 

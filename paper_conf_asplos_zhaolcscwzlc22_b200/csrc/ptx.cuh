@@ -124,6 +124,13 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
 }
 __device__ __forceinline__ void tmem_ld_wait() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
 
+// Programmatic dependent launch: a kernel launched with the PDL attribute may start while
+// its predecessor in the stream is finishing; pdl_wait() blocks until the predecessor has
+// completed and its writes are visible.  Every PDL-launched kernel calls pdl_wait() before
+// touching memory its predecessors produce.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 // hardware tanh (MUFU.TANH), max relative error ~2^-11: below bf16 output resolution
 __device__ __forceinline__ float tanh_fast(float x) {
   float y;
