@@ -25,9 +25,12 @@ def stage_uses(order_K, choices, blocks_K, n):
     return [{b * n + int(choices[y][b]) for b in blocks_K} for _, y in order_K]
 
 
-def simulate_residency(uses, kinds, nbytes, budget, L=2):
+def simulate_residency(uses, kinds, nbytes, budget, L=2, horizon=None):
     """uses: list of uid sets per task; kinds: 0/1 per task (B writes => dirty);
     nbytes: {uid: bytes}; budget: bytes (0 = everything resident, no traffic).
+    horizon: reading A26 — "next use" only looks at tasks [i, i + horizon) (None = the whole
+    plan), so the decision before task i needs only the plan up to i + horizon - 1, which a
+    streaming executor knows without waiting for the end of the stream.
 
     Returns dict(events=[(op, i, uid)], writebacks=[(i, uid)]) with op in {"LOAD", "EVICT"}.
     """
@@ -38,7 +41,8 @@ def simulate_residency(uses, kinds, nbytes, budget, L=2):
     resident, dirty = set(), set()
 
     def next_use(uid, i):
-        for j in range(i, T):
+        end = T if horizon is None else min(T, i + horizon)
+        for j in range(i, end):
             if uid in uses[j]:
                 return j
         return INF

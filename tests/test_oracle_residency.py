@@ -71,6 +71,19 @@ def test_large_budget_loads_once(seed):
     assert all(op == "LOAD" for op, _, _ in ev)
 
 
+def test_horizon_reading():
+    """A26: a horizon covering the whole plan is the unbounded rule; horizon 1 sees only the
+    current task, so every non-needed candidate is 'never used again' and ties go to the
+    lowest uid (worked example, budget 3: at task 4 uid 1 is evicted instead of uid 2)."""
+    uses, kinds = _worked_plan()
+    nbytes = {u: 1 for u in range(4)}
+    full = residency.simulate_residency(uses, kinds, nbytes, 3)
+    assert residency.simulate_residency(uses, kinds, nbytes, 3, horizon=len(uses)) == full
+    short = residency.simulate_residency(uses, kinds, nbytes, 3, L=1, horizon=1)["events"]
+    assert [f"{op}({i},{u})" for op, i, u in short] == [
+        "LOAD(0,0)", "LOAD(0,2)", "LOAD(2,1)", "EVICT(4,1)", "LOAD(4,3)", "EVICT(6,0)", "LOAD(6,1)"]
+
+
 @pytest.mark.parametrize("seed", range(6))
 def test_belady_optimal_on_unit_sizes(seed):
     """Unit sizes, L=1: Belady's rule minimises loads; compare against exhaustive search
