@@ -76,6 +76,8 @@ typedef enum { NASPIPE_FP32 = 0, NASPIPE_BF16 = 1 } naspipe_dtype; /* compute dt
  *   window        W: stage 0 starts F(y,0) only for y < (lowest unfinished id) + W
  *                 (reading A7); 0 = 4 * n_stages.
  *   lookahead     residency prefetch depth L in tasks ("2"); 0 = 2.
+ *   residency_horizon  H: Belady's "next use" looks at the stage's next H tasks only
+ *                 (reading A26); 0 = 64, < 0 = unbounded (decisions wait for the final plan).
  *   hbm_weight_budget_bytes  per-stage device budget for candidate fp32 masters; 0 = all
  *                 candidates resident (no context switching).
  *   bwd_policy    0 = strict backward-first (reading A5); 1 = Alg.1 alternation.
@@ -100,6 +102,7 @@ typedef struct {
   const int32_t* cost_bwd;
   int32_t window;
   int32_t lookahead;
+  int32_t residency_horizon;
   int64_t hbm_weight_budget_bytes;
   int32_t bwd_policy;
   int32_t link_latency;
@@ -195,10 +198,11 @@ int naspipe_plan_makespan(const naspipe_plan_t* p, int64_t* makespan);
 /* deps(y, K): ids of the latest earlier users of y's stage-K candidates (dependency table). */
 int naspipe_plan_deps(const naspipe_plan_t* p, int64_t y, int32_t stage, int64_t* dst, size_t cap,
                       size_t* n);
-/* Belady residency of stage K under budget bytes (0 = all resident), depth L (0 = spec's);
- * 4 int64 per event (stage, task index, op, uid); writebacks counted in *n_writebacks. */
+/* Belady residency of stage K under budget bytes of fp32 masters (0 = all resident), depth
+ * L (0 = spec's), next-use horizon H (0 = spec's, < 0 = unbounded); 4 int64 per event
+ * (stage, task index, op 0=LOAD/1=EVICT, uid); writebacks counted in *n_writebacks. */
 int naspipe_plan_residency(const naspipe_plan_t* p, int32_t stage, int64_t budget_bytes,
-                           int32_t depth, int64_t* dst, size_t cap, size_t* n,
+                           int32_t depth, int32_t horizon, int64_t* dst, size_t cap, size_t* n,
                            int64_t* n_writebacks);
 void naspipe_plan_destroy(naspipe_plan_t* p);
 

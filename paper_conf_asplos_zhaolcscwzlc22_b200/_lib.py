@@ -30,6 +30,7 @@ class _SpecStruct(C.Structure):
                 ("choice_heads", _i32p), ("choice_ffn", _i32p), ("lr", C.c_float),
                 ("init_seed", C.c_uint64), ("stage_of_block", _i32p), ("cost_fwd", _i32p),
                 ("cost_bwd", _i32p), ("window", C.c_int32), ("lookahead", C.c_int32),
+                ("residency_horizon", C.c_int32),
                 ("hbm_weight_budget_bytes", C.c_int64), ("bwd_policy", C.c_int32),
                 ("link_latency", C.c_int32), ("flags", C.c_int32)]
 
@@ -68,8 +69,8 @@ _sig("naspipe_plan_create", C.c_int, [_SP, C.c_int32, _i32p, C.c_int64, C.POINTE
 _sig("naspipe_plan_trace", C.c_int, [C.c_void_p, _i64p, C.c_size_t, C.POINTER(C.c_size_t)])
 _sig("naspipe_plan_makespan", C.c_int, [C.c_void_p, _i64p])
 _sig("naspipe_plan_deps", C.c_int, [C.c_void_p, C.c_int64, C.c_int32, _i64p, C.c_size_t, C.POINTER(C.c_size_t)])
-_sig("naspipe_plan_residency", C.c_int, [C.c_void_p, C.c_int32, C.c_int64, C.c_int32, _i64p, C.c_size_t,
-                                         C.POINTER(C.c_size_t), _i64p])
+_sig("naspipe_plan_residency", C.c_int, [C.c_void_p, C.c_int32, C.c_int64, C.c_int32, C.c_int32, _i64p,
+                                         C.c_size_t, C.POINTER(C.c_size_t), _i64p])
 _sig("naspipe_plan_destroy", None, [C.c_void_p])
 _sig("naspipe_nccl_unique_id", C.c_int, [C.c_void_p])
 
@@ -120,6 +121,7 @@ class Spec:
         s.init_seed = cfg.get("init_seed", 2)
         s.window = cfg.get("window", 0)
         s.lookahead = cfg.get("lookahead", 0)
+        s.residency_horizon = cfg.get("residency_horizon", 0)
         s.hbm_weight_budget_bytes = cfg.get("hbm_weight_budget_bytes", 0)
         s.bwd_policy = cfg.get("bwd_policy", 0)
         s.link_latency = cfg.get("link_latency", 0)
@@ -298,13 +300,15 @@ class Plan:
     def deps(self, y: int, stage: int):
         return [int(v) for v in _get_rows(lib.naspipe_plan_deps, self.ptr, y, stage, width=1).ravel()]
 
-    def residency(self, stage: int, budget_bytes: int, depth: int = 0):
+    def residency(self, stage: int, budget_bytes: int, depth: int = 0, horizon: int = -1):
+        """horizon: -1 unbounded, 0 the spec's, > 0 reading A26's H."""
         n = C.c_size_t()
         wb = C.c_int64()
-        _check(lib.naspipe_plan_residency(self.ptr, stage, budget_bytes, depth, None, 0, C.byref(n), C.byref(wb)))
+        _check(lib.naspipe_plan_residency(self.ptr, stage, budget_bytes, depth, horizon, None, 0, C.byref(n),
+                                          C.byref(wb)))
         out = np.zeros((n.value, 4), dtype=np.int64)
         if n.value:
-            _check(lib.naspipe_plan_residency(self.ptr, stage, budget_bytes, depth, out.ctypes.data_as(_i64p),
+            _check(lib.naspipe_plan_residency(self.ptr, stage, budget_bytes, depth, horizon, out.ctypes.data_as(_i64p),
                                               n.value, C.byref(n), C.byref(wb)))
         return out, wb.value
 

@@ -133,7 +133,7 @@ int naspipe_plan_deps(const naspipe_plan_t* p, int64_t y, int32_t stage, int64_t
 }
 
 int naspipe_plan_residency(const naspipe_plan_t* p, int32_t stage, int64_t budget_bytes, int32_t depth,
-                           int64_t* dst, size_t cap, size_t* n, int64_t* n_writebacks) {
+                           int32_t horizon, int64_t* dst, size_t cap, size_t* n, int64_t* n_writebacks) {
   return guarded([&] {
     NP_REQUIRE(p && n && stage >= 0 && stage < p->planner->D() && budget_bytes >= 0 && depth >= 0,
                NASPIPE_EINVAL, "bad args");
@@ -154,7 +154,8 @@ int naspipe_plan_residency(const naspipe_plan_t* p, int32_t stage, int64_t budge
       for (int c = 0; c < s.n(); ++c) bytes[(size_t)b * s.n() + c] = 4 * (int64_t)s.param_count(b, c);
     ResidencyPlan rp;
     if (budget_bytes > 0)
-      rp = plan_residency(stage, uses, kinds, bytes, budget_bytes, depth > 0 ? depth : s.lookahead());
+      rp = plan_residency(stage, uses, kinds, bytes, budget_bytes, depth > 0 ? depth : s.lookahead(),
+                          horizon == 0 ? s.residency_horizon() : horizon);
     *n = rp.events.size();
     if (n_writebacks) *n_writebacks = (int64_t)rp.writebacks.size();
     for (size_t i = 0; i < rp.events.size() && i < cap && dst; ++i) {

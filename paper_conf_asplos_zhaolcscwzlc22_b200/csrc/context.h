@@ -1,0 +1,70 @@
+// Candidate storage of one stage and the context switch (PAPER.md P:L156,
+// P:L160-162; readings A9, A26).
+//
+// Budget 0: every candidate of the stage is resident in HBM for the whole run.
+// Budget > 0: all candidates live in a pinned host stash (fp32 masters, "by default,
+// the supernet's operators all reside in CPU storage"); before each task the Belady plan
+// (BeladyResidency: farthest next use within the horizon, depth-L prefetch that fits the
+// budget) issues EVICTs (D2H write-back only if updated since load) and LOADs (H2D + bf16
+// shadow refresh) on the stage's copy stream; the compute stream waits only for the
+// candidates of the task it is about to run, so prefetches for later tasks overlap compute.
+// Numerics are unaffected by residency: a candidate's bytes are the same wherever it lives.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <memory>
+#include <vector>
+
+#include "family.h"
+#include "planner.h"
+
+namespace naspipe {
+
+class CandidateStore {
+ public:
+  CandidateStore(const Spec& spec, const Planner& planner, int K, int dev, Family* fam, DevArena* arena,
+                 int64_t budget);
+  ~CandidateStore();
+  bool managed() const { return budget_ > 0; }
+
+  // plan feed (host thread)
+  void push_task(const Task& t);
+  void set_final();
+  bool ready() const;  // the next stage task's residency can be decided
+
+  // issue hooks, in the stage's plan order
+  void before_task(const Task& t, cudaStream_t comp, cudaStream_t copy);
+  void after_task(const Task& t, cudaStream_t comp);
+
+  // read-out (streams idle)
+  void get(int b, int c, float* dst);
+  void set(int b, int c, const float* src, cudaStream_t s);
+
+  uint64_t loads = 0, evicts = 0, writebacks = 0;
+  double h2d_bytes = 0, d2h_bytes = 0;
+  std::vector<ResidencyEvent> log;
+
+ private:
+  struct Cand {
+    int j = -1, c = -1;  // local block, choice
+    size_t n32 = 0, n16 = 0;
+    float* stash = nullptr;  // pinned host fp32 master (managed mode)
+    float* w32 = nullptr;    // device, when resident
+    bf16* w16 = nullptr;
+    cudaEvent_t ready = nullptr, last_use = nullptr;
+  };
+  int uid_of(int b, int c) const { return b * n_ + c; }
+  std::vector<int64_t> task_uids(const Task& t) const;
+  void load(Cand& cd, cudaStream_t copy);
+  void evict(Cand& cd, bool writeback, cudaStream_t copy);
+
+  const Spec& spec_;
+  const Planner& planner_;
+  int K_, dev_, n_;
+  Family* fam_;
+  int64_t budget_;
+  std::vector<Cand> cands_;  // indexed by uid (only this stage's blocks are populated)
+  std::unique_ptr<BeladyResidency> belady_;
+};
+
+}  // namespace naspipe

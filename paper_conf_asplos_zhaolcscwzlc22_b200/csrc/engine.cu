@@ -85,8 +85,6 @@ struct Transport {
 
 // ------------------------------------------------------------------------------ construction
 Engine::Engine(const Spec& spec, int D) : spec_(spec), D_(D), W_(spec.window(D)), planner_(spec_, D) {
-  NP_REQUIRE(spec_.raw.hbm_weight_budget_bytes == 0, NASPIPE_EINVAL,
-             "hbm_weight_budget_bytes > 0 (context switching) is not enabled in this build");
   version_.assign((size_t)spec_.m() * spec_.n(), 0);
   timer_.on = (spec_.raw.flags & NASPIPE_FLAG_TIMING) != 0;
 }
@@ -159,6 +157,8 @@ void Engine::setup_stage(int K, int dev, bool local) {
   st.arena = std::make_unique<DevArena>(dev);
   st.fam = make_family(spec_, planner_.blocks_of(K), W_, *st.arena, st.comp);
   st.fam->timer = &timer_;
+  st.store = std::make_unique<CandidateStore>(spec_, planner_, K, dev, st.fam.get(), st.arena.get(),
+                                              spec_.raw.hbm_weight_budget_bytes);
   const size_t n = spec_.batch_elems();
   st.in.assign(W_, nullptr);
   st.gout.assign(W_, nullptr);
@@ -221,6 +221,7 @@ void Engine::shutdown() {
   for (auto& st : st_) {
     if (!st.local || !st.comp) continue;
     cudaSetDevice(st.dev);
+    st.store.reset();
     st.fam.reset();
     st.arena.reset();
     for (auto* v : {&st.ev_f, &st.ev_b, &st.ev_in, &st.ev_tgt})
@@ -264,6 +265,7 @@ int64_t Engine::submit(const int32_t* choice, const naspipe_batch* batch) {
   const int64_t y = planner_.add_subnet(choice);
   batches_.push_back({*batch});
   planner_.advance();
+  feed_stores();
   issue_planned();
   return y;
 }
@@ -273,7 +275,11 @@ void Engine::drain() {
     planner_.finalize();
     planner_.advance();
     NP_REQUIRE(planner_.done(), NASPIPE_EINTERNAL, "planner did not finish");
+    feed_stores();
+    for (auto& st : st_)
+      if (st.local) st.store->set_final();
     issue_planned();
+    NP_REQUIRE(issued_ == planner_.tasks().size(), NASPIPE_EINTERNAL, "tasks left unissued at drain");
   }
   for (auto& st : st_) {
     if (!st.local) continue;
@@ -289,9 +295,24 @@ void Engine::drain() {
   drained_ = true;
 }
 
+// Append newly planned stage tasks to the local stages' candidate stores (residency plan).
+void Engine::feed_stores() {
+  for (auto& st : st_) {
+    if (!st.local) continue;
+    const auto& idx = planner_.stage_tasks()[st.K];
+    for (; st.pushed < idx.size(); ++st.pushed) st.store->push_task(planner_.tasks()[idx[st.pushed]]);
+  }
+}
+
+// Issue planned tasks in tick order; a local stage whose next residency decision needs more
+// of the plan (reading A26's horizon) holds the issue point until more subnets arrive.
 void Engine::issue_planned() {
   const auto& tasks = planner_.tasks();
-  while (issued_ < tasks.size()) issue(tasks[issued_++]);
+  while (issued_ < tasks.size()) {
+    const Task& t = tasks[issued_];
+    if (st_[t.K].local && !st_[t.K].store->ready()) break;
+    issue(tasks[issued_++]);
+  }
 }
 
 void Engine::version_check(const Task& t) {
@@ -332,8 +353,10 @@ void Engine::issue(const Task& t) {
   if (spec_.raw.flags & NASPIPE_FLAG_VERSION_CHECK) version_check(t);
   if (spec_.raw.flags & NASPIPE_FLAG_TRACE) trace_.push_back(t);
   CU(cudaSetDevice(st.dev));
+  st.store->before_task(t, st.comp, st.copy);  // context switch: LOAD/EVICT, wait for this task's candidates
   if (t.kind == 0) issue_forward(st, t.y, slot);
   else issue_backward(st, t.y, slot);
+  st.store->after_task(t, st.comp);
 }
 
 void Engine::issue_forward(StageRt& st, int64_t y, int slot) {
@@ -429,12 +452,6 @@ void Engine::issue_backward(StageRt& st, int64_t y, int slot) {
 }
 
 // ------------------------------------------------------------------------------ read-out
-static int owner_local_index(const std::vector<int>& blocks, int b) {
-  for (size_t j = 0; j < blocks.size(); ++j)
-    if (blocks[j] == b) return (int)j;
-  return -1;
-}
-
 void Engine::get_params(int block, int choice, float* dst, size_t n) {
   NP_REQUIRE(block >= 0 && block < spec_.m() && choice >= 0 && choice < spec_.n(), NASPIPE_EINVAL,
              "candidate (%d,%d) out of range", block, choice);
@@ -444,9 +461,7 @@ void Engine::get_params(int block, int choice, float* dst, size_t n) {
   const int K = planner_.stage_of_block()[block];
   StageRt& st = st_[K];
   NP_REQUIRE(st.local, NASPIPE_EINVAL, "block %d lives on stage %d, not on this rank", block, K);
-  CU(cudaSetDevice(st.dev));
-  const int j = owner_local_index(planner_.blocks_of(K), block);
-  CU(cudaMemcpy(dst, st.fam->master(j, choice), n * 4, cudaMemcpyDeviceToHost));
+  st.store->get(block, choice, dst);
   d2h_bytes_ += 4.0 * n;
 }
 
@@ -459,11 +474,7 @@ void Engine::set_params(int block, int choice, const float* src, size_t n) {
   const int K = planner_.stage_of_block()[block];
   StageRt& st = st_[K];
   NP_REQUIRE(st.local, NASPIPE_EINVAL, "block %d lives on stage %d, not on this rank", block, K);
-  CU(cudaSetDevice(st.dev));
-  const int j = owner_local_index(planner_.blocks_of(K), block);
-  CU(cudaMemcpy(st.fam->master(j, choice), src, n * 4, cudaMemcpyHostToDevice));
-  st.fam->refresh_shadow(j, choice, st.comp);
-  CU(cudaStreamSynchronize(st.comp));
+  st.store->set(block, choice, src, st.comp);
 }
 
 void Engine::get_losses(float* dst, int64_t n) {
@@ -492,10 +503,22 @@ void Engine::get_stats(double* o) {
   double launches = 0;
   for (auto& st : st_)
     if (st.local && st.fam) launches += (double)st.fam->counters.launches;
+  double loads = 0, evicts = 0, wbs = 0, rh2d = 0, rd2h = 0;
+  for (auto& st : st_)
+    if (st.local && st.store) {
+      loads += (double)st.store->loads;
+      evicts += (double)st.store->evicts;
+      wbs += (double)st.store->writebacks;
+      rh2d += st.store->h2d_bytes;
+      rd2h += st.store->d2h_bytes;
+    }
   o[0] = (double)issued_;
   o[1] = launches + (double)engine_launches_;
-  o[2] = h2d_bytes_;
-  o[3] = d2h_bytes_;
+  o[2] = h2d_bytes_ + rh2d;
+  o[3] = d2h_bytes_ + rd2h;
+  o[9] = loads;
+  o[10] = evicts;
+  o[11] = wbs;
   o[4] = p2p_bytes_;
   o[5] = (double)planner_.makespan();
   o[6] = timer_.launches;
@@ -505,10 +528,21 @@ void Engine::get_stats(double* o) {
 }
 
 void Engine::get_residency_trace(int64_t* dst, size_t cap, size_t* n) {
-  (void)dst;
-  (void)cap;
   NP_REQUIRE(n, NASPIPE_EINVAL, "n NULL");
-  *n = 0;  // all candidates resident (hbm_weight_budget_bytes == 0)
+  size_t k = 0;
+  for (auto& st : st_) {
+    if (!st.local || !st.store) continue;
+    for (const auto& e : st.store->log) {
+      if (dst && k < cap) {
+        dst[4 * k] = e.K;
+        dst[4 * k + 1] = e.i;
+        dst[4 * k + 2] = e.op;
+        dst[4 * k + 3] = e.uid;
+      }
+      ++k;
+    }
+  }
+  *n = k;
 }
 
 }  // namespace naspipe

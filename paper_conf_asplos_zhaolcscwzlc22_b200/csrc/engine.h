@@ -9,6 +9,7 @@
 #include <string>
 #include <vector>
 
+#include "context.h"
 #include "family.h"
 #include "planner.h"
 
@@ -23,6 +24,8 @@ struct StageRt {
   cudaStream_t comp = nullptr, copy = nullptr;
   std::unique_ptr<DevArena> arena;
   std::unique_ptr<Family> fam;
+  std::unique_ptr<CandidateStore> store;  // candidate parameters (resident or context-switched)
+  size_t pushed = 0;                      // stage tasks fed to the store
   // boundary buffers per slot (device, on dev)
   std::vector<float*> in, out, gin, gout, target;
   std::vector<cudaEvent_t> ev_f, ev_b, ev_in, ev_tgt;
@@ -57,6 +60,7 @@ class Engine {
   Engine(const Spec& spec, int D);
   void setup_stage(int K, int dev, bool local);
   void link_local_buffers();
+  void feed_stores();
   void issue_planned();
   void issue(const Task& t);
   void issue_forward(StageRt& st, int64_t y, int slot);

@@ -71,17 +71,9 @@ class MlpFamily : public Family {
   MlpFamily(const Spec& spec, const std::vector<int>& blocks, int W, DevArena& A, cudaStream_t s)
       : spec_(spec), blocks_(blocks), W_(W), B_(spec.B()), d_(spec.raw.width), lr_(spec.raw.lr) {
     const int nb = (int)blocks.size(), n = spec.n();
-    const size_t P = spec.param_count(0, 0), act = (size_t)B_ * d_;
-    params_.resize((size_t)nb * n);
-    std::vector<float> host(P);
-    for (int j = 0; j < nb; ++j)
-      for (int c = 0; c < n; ++c) {
-        float* p = A.alloc<float>(P);
-        spec.init_params(blocks[j], c, host.data());
-        cudaMemcpyAsync(p, host.data(), P * 4, cudaMemcpyHostToDevice, s);
-        cudaStreamSynchronize(s);
-        params_[(size_t)j * n + c] = p;
-      }
+    (void)s;
+    const size_t act = (size_t)B_ * d_;
+    params_.assign((size_t)nb * n, nullptr);
     h_.resize((size_t)W * nb);
     act_.resize((size_t)W * nb);
     xin_.assign((size_t)W * nb, nullptr);
@@ -90,6 +82,8 @@ class MlpFamily : public Family {
     g_[0] = A.alloc<float>(act);
     g_[1] = A.alloc<float>(act);
   }
+  void bind(int j, int c, float* w32, bf16*) override { params_[(size_t)j * spec_.n() + c] = w32; }
+  size_t shadow_elems(int) const override { return 0; }
   float* master(int j, int c) override { return params_[(size_t)j * spec_.n() + c]; }
   void refresh_shadow(int, int, cudaStream_t) override {}
 
@@ -144,21 +138,9 @@ class TfFamily : public Family {
     const int nb = (int)blocks.size(), n = spec.n();
     fmax_ = *std::max_element(spec.ffn.begin(), spec.ffn.end());
     hmax_ = *std::max_element(spec.heads.begin(), spec.heads.end());
-    w32_.resize((size_t)nb * n);
-    w16_.resize((size_t)nb * n);
-    for (int j = 0; j < nb; ++j)
-      for (int c = 0; c < n; ++c) {
-        const TfOffsets o = spec.tf_offsets(c);
-        const size_t f = spec.ffn[c];
-        float* p = A.alloc<float>(o.total);
-        std::vector<float> host(o.total);
-        spec.init_params(blocks[j], c, host.data());
-        cudaMemcpyAsync(p, host.data(), o.total * 4, cudaMemcpyHostToDevice, s);
-        cudaStreamSynchronize(s);
-        w32_[(size_t)j * n + c] = p;
-        w16_[(size_t)j * n + c] = A.alloc<bf16>(4 * (size_t)d_ * d_ + 2 * (size_t)d_ * f);
-        refresh_shadow(j, c, s);
-      }
+    (void)s;
+    w32_.assign((size_t)nb * n, nullptr);
+    w16_.assign((size_t)nb * n, nullptr);
     const size_t Td = (size_t)T_ * d_;
     slots_.resize((size_t)W * nb);
     for (int sl = 0; sl < W; ++sl)
@@ -223,6 +205,11 @@ class TfFamily : public Family {
     cudaStreamDestroy(side_);
   }
 
+  void bind(int j, int c, float* w32, bf16* w16) override {
+    w32_[(size_t)j * spec_.n() + c] = w32;
+    w16_[(size_t)j * spec_.n() + c] = w16;
+  }
+  size_t shadow_elems(int c) const override { return 4 * (size_t)d_ * d_ + 2 * (size_t)d_ * spec_.ffn[c]; }
   float* master(int j, int c) override { return w32_[(size_t)j * spec_.n() + c]; }
 
   void refresh_shadow(int j, int c, cudaStream_t s) override {

@@ -53,7 +53,13 @@ class Family {
   // dy: grad w.r.t. the stage output; dx: grad w.r.t. the stage input (nullptr: not needed)
   virtual void backward(int slot, const int32_t* choice_of_block, const float* dy, float* dx,
                         cudaStream_t s) = 0;
-  virtual float* master(int local_block, int c) = 0;   // device fp32 packed vector
+  // Candidate (local block j, choice c) parameters live in buffers the engine owns (resident
+  // for the whole run, or loaded/evicted by the context switch); bind() points the family at
+  // them (nullptr = not resident).  master() is the packed fp32 vector, the bf16 shadow holds
+  // the GEMM operands (shadow_elems(c) elements; 0 for fp32 families).
+  virtual void bind(int local_block, int c, float* w32, bf16* w16) = 0;
+  virtual size_t shadow_elems(int c) const = 0;
+  virtual float* master(int local_block, int c) = 0;
   virtual void refresh_shadow(int local_block, int c, cudaStream_t s) = 0;  // bf16 <- fp32
   FamilyCounters counters;
   KernelTimer* timer = nullptr;

@@ -151,65 +151,77 @@ void Planner::advance() {
   }
 }
 
+bool BeladyResidency::can_decide() const {
+  if (next_ >= known()) return false;
+  if (final_) return true;
+  if (H_ <= 0) return false;
+  return known() >= next_ + std::max<int64_t>(L_, H_);
+}
+
+int64_t BeladyResidency::next_use(int64_t u, int64_t i) const {
+  const int64_t end = H_ > 0 ? std::min(known(), i + H_) : known();
+  for (int64_t j = i; j < end; ++j)
+    if (std::binary_search(uses_[j].begin(), uses_[j].end(), u)) return j;
+  return std::numeric_limits<int64_t>::max();
+}
+
+int64_t BeladyResidency::size_of(const std::set<int64_t>& s) const {
+  int64_t t = 0;
+  for (int64_t u : s) t += bytes_[u];
+  return t;
+}
+
+void BeladyResidency::decide_next(std::vector<ResidencyEvent>& events,
+                                  std::vector<std::pair<int64_t, int64_t>>& writebacks) {
+  const int64_t i = next_;
+  const int64_t T = known();
+  std::set<int64_t> need(uses_[i].begin(), uses_[i].end());
+  NP_REQUIRE(size_of(need) <= budget_, NASPIPE_EBUDGET, "stage %d task %lld needs %lld bytes > budget %lld", K_,
+             (long long)i, (long long)size_of(need), (long long)budget_);
+  for (int depth = 2; depth <= L_; ++depth) {  // prefetch depth L' <= L that fits the budget
+    if (i + depth - 1 >= T) break;
+    std::set<int64_t> cand = need;
+    cand.insert(uses_[i + depth - 1].begin(), uses_[i + depth - 1].end());
+    if (size_of(cand) > budget_) break;
+    need.swap(cand);
+  }
+  for (;;) {
+    std::set<int64_t> uni = resident_;
+    uni.insert(need.begin(), need.end());
+    if (size_of(uni) <= budget_) break;
+    int64_t victim = -1, far = -1;
+    for (int64_t u : resident_) {  // ascending uid: ties keep the lowest
+      if (need.count(u)) continue;
+      const int64_t nu = next_use(u, i);
+      if (nu > far) { far = nu; victim = u; }
+    }
+    resident_.erase(victim);
+    events.push_back({K_, i, 1, victim});
+    if (dirty_.count(victim)) {
+      writebacks.push_back({i, victim});
+      dirty_.erase(victim);
+    }
+  }
+  std::vector<std::pair<int64_t, int64_t>> loads;
+  for (int64_t u : need)
+    if (!resident_.count(u)) loads.push_back({next_use(u, i), u});
+  std::sort(loads.begin(), loads.end());
+  for (auto& lu : loads) {
+    resident_.insert(lu.second);
+    events.push_back({K_, i, 0, lu.second});
+  }
+  if (kinds_[i] == 1) dirty_.insert(uses_[i].begin(), uses_[i].end());
+  ++next_;
+}
+
 ResidencyPlan plan_residency(int K, const std::vector<std::vector<int64_t>>& uses,
                              const std::vector<int>& kinds, const std::vector<int64_t>& bytes,
-                             int64_t budget, int L) {
+                             int64_t budget, int L, int64_t horizon) {
   ResidencyPlan out;
-  const int64_t T = (int64_t)uses.size();
-  const int64_t NEVER = std::numeric_limits<int64_t>::max();
-  std::map<int64_t, std::vector<int64_t>> when;  // uid -> task indices using it
-  for (int64_t i = 0; i < T; ++i)
-    for (int64_t u : uses[i]) when[u].push_back(i);
-  auto next_use = [&](int64_t u, int64_t i) -> int64_t {
-    auto& v = when[u];
-    auto it = std::lower_bound(v.begin(), v.end(), i);
-    return it == v.end() ? NEVER : *it;
-  };
-  auto size_of = [&](const std::set<int64_t>& s) {
-    int64_t t = 0;
-    for (int64_t u : s) t += bytes[u];
-    return t;
-  };
-  std::set<int64_t> resident, dirty;
-  for (int64_t i = 0; i < T; ++i) {
-    std::set<int64_t> need(uses[i].begin(), uses[i].end());
-    NP_REQUIRE(size_of(need) <= budget, NASPIPE_EBUDGET,
-               "stage %d task %lld needs %lld bytes > budget %lld", K, (long long)i,
-               (long long)size_of(need), (long long)budget);
-    for (int depth = 2; depth <= L; ++depth) {
-      if (i + depth - 1 >= T) break;
-      std::set<int64_t> cand = need;
-      cand.insert(uses[i + depth - 1].begin(), uses[i + depth - 1].end());
-      if (size_of(cand) > budget) break;
-      need.swap(cand);
-    }
-    for (;;) {
-      std::set<int64_t> uni = resident;
-      uni.insert(need.begin(), need.end());
-      if (size_of(uni) <= budget) break;
-      int64_t victim = -1, far = -1;
-      for (int64_t u : resident) {  // ascending uid: ties keep the lowest
-        if (need.count(u)) continue;
-        const int64_t nu = next_use(u, i);
-        if (nu > far) { far = nu; victim = u; }
-      }
-      resident.erase(victim);
-      out.events.push_back({K, i, 1, victim});
-      if (dirty.count(victim)) {
-        out.writebacks.push_back({i, victim});
-        dirty.erase(victim);
-      }
-    }
-    std::vector<std::pair<int64_t, int64_t>> loads;
-    for (int64_t u : need)
-      if (!resident.count(u)) loads.push_back({next_use(u, i), u});
-    std::sort(loads.begin(), loads.end());
-    for (auto& lu : loads) {
-      resident.insert(lu.second);
-      out.events.push_back({K, i, 0, lu.second});
-    }
-    if (kinds[i] == 1) dirty.insert(uses[i].begin(), uses[i].end());
-  }
+  BeladyResidency r(K, bytes, budget, L, horizon);
+  for (size_t i = 0; i < uses.size(); ++i) r.push_task(uses[i], kinds[i]);
+  r.set_final();
+  while (r.can_decide()) r.decide_next(out.events, out.writebacks);
   return out;
 }
 

@@ -90,9 +90,45 @@ struct ResidencyPlan {
   std::vector<ResidencyEvent> events;
   std::vector<std::pair<int64_t, int64_t>> writebacks;  // (task index, uid)
 };
-// uses[i] = sorted uids used by task i; kinds[i] = 0/1; bytes[uid]; budget > 0.
+// Incremental Belady residency of one stage (SURVEY §8c O6 with the next-use horizon of
+// reading A26).  Tasks are appended as the plan grows; the decision before task i is taken
+// once tasks [i, i + max(L, H)) are known or the plan is final, so it never depends on how
+// far the planner happened to be.  horizon <= 0: unbounded (needs the final plan).
+class BeladyResidency {
+ public:
+  BeladyResidency(int K, std::vector<int64_t> bytes, int64_t budget, int L, int64_t horizon)
+      : K_(K), bytes_(std::move(bytes)), budget_(budget), L_(L), H_(horizon) {}
+  void push_task(std::vector<int64_t> sorted_uids, int kind) {
+    uses_.push_back(std::move(sorted_uids));
+    kinds_.push_back(kind);
+  }
+  void set_final() { final_ = true; }
+  bool can_decide() const;
+  // Decide the next task: appends its LOAD/EVICT events and write-backs.  Throws EBUDGET.
+  void decide_next(std::vector<ResidencyEvent>& events, std::vector<std::pair<int64_t, int64_t>>& writebacks);
+  int64_t decided() const { return next_; }
+  int64_t known() const { return (int64_t)uses_.size(); }
+  const std::vector<int64_t>& uses(int64_t i) const { return uses_[i]; }
+  int kind(int64_t i) const { return kinds_[i]; }
+
+ private:
+  int64_t next_use(int64_t u, int64_t i) const;
+  int64_t size_of(const std::set<int64_t>& s) const;
+  int K_;
+  std::vector<int64_t> bytes_;
+  int64_t budget_;
+  int L_;
+  int64_t H_;
+  bool final_ = false;
+  int64_t next_ = 0;
+  std::vector<std::vector<int64_t>> uses_;
+  std::vector<int> kinds_;
+  std::set<int64_t> resident_, dirty_;
+};
+
+// Whole-plan convenience wrapper (host planner API).
 ResidencyPlan plan_residency(int K, const std::vector<std::vector<int64_t>>& uses,
                              const std::vector<int>& kinds, const std::vector<int64_t>& bytes,
-                             int64_t budget, int L);
+                             int64_t budget, int L, int64_t horizon);
 
 }  // namespace naspipe

@@ -36,6 +36,7 @@ struct Spec {
   int B() const { return raw.batch; }
   int window(int D) const { return raw.window > 0 ? raw.window : 4 * D; }
   int lookahead() const { return raw.lookahead > 0 ? raw.lookahead : 2; }
+  int64_t residency_horizon() const { return raw.residency_horizon == 0 ? 64 : raw.residency_horizon; }
   // elements of one sample of input / output (the residual stream width per batch row)
   size_t sample_elems() const;
   size_t batch_elems() const { return (size_t)B() * sample_elems(); }

@@ -113,11 +113,13 @@ def test_residency_matches_oracle(seed):
         need = max(sum(nbytes[u] for u in us) for us in uses)
         budget = int(need * rng.uniform(1.0, 3.0))
         for depth in (1, 2, 3):
-            ref = residency.simulate_residency(uses, [k for k, _ in order], nbytes, budget, L=depth)
-            ev, wb = plan.residency(K, budget, depth)
-            got = [("LOAD" if op == 0 else "EVICT", int(i), int(u)) for _, i, op, u in ev]
-            assert got == ref["events"], (K, depth)
-            assert wb == len(ref["writebacks"])
+            for horizon in (None, 1, 3, 8):
+                ref = residency.simulate_residency(uses, [k for k, _ in order], nbytes, budget, L=depth,
+                                                   horizon=horizon)
+                ev, wb = plan.residency(K, budget, depth, -1 if horizon is None else horizon)
+                got = [("LOAD" if op == 0 else "EVICT", int(i), int(u)) for _, i, op, u in ev]
+                assert got == ref["events"], (K, depth, horizon)
+                assert wb == len(ref["writebacks"])
 
 
 def test_budget_error_and_invalid_args():
