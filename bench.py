@@ -39,7 +39,23 @@ def parse():
     ap.add_argument("--workload", default="transformer")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--budget-x", type=float, default=0.0,
+                    help="HBM weight budget per stage as a multiple of one subnet's mean stage slice "
+                         "(0 = all candidates resident; P:L337 uses ~3)")
+    ap.add_argument("--n-choices", type=int, default=0, help="override n (search-space sweep, configs[4])")
+    ap.add_argument("--lookahead", type=int, default=0, help="residency prefetch depth L in tasks (0 = 2, P:L156)")
     return ap.parse_args()
+
+
+def stage_budget(cfg, D, x, npipe):
+    """x times the mean fp32 bytes of one subnet's slice on the largest stage."""
+    spec = npipe.Spec(cfg)
+    sob = npipe.naspipe_partition(spec, D)
+    n = cfg["n_choices"]
+    per_stage = [0.0] * D
+    for b in range(cfg["n_blocks"]):
+        per_stage[sob[b]] += np.mean([4 * npipe.naspipe_param_count(spec, b, c) for c in range(n)])
+    return int(x * max(per_stage))
 
 
 def peaks():
@@ -149,7 +165,10 @@ def run_reference(args, cfg, rank, world):
 
 
 def workload_config(args, cfg, world):
-    c = {"workload": f"configs[2] {args.workload}" if args.workload == "transformer" else args.workload,
+    names = {"transformer": "configs[2] transformer", "large_transformer": "configs[3] large_transformer",
+             "toy": "configs[0] toy"}
+    c = {"workload": names.get(args.workload, args.workload) if not args.n_choices
+         else f"configs[4] sweep n={args.n_choices}",
          "n_blocks": cfg["n_blocks"], "n_choices": cfg["n_choices"], "batch": cfg["batch"],
          "stages": world, "parallelism": f"pp{world}" if world > 1 else "single stage",
          "l2": "working set > L2 (active weights + activations per step >> 126 MB)"}
@@ -164,7 +183,7 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    cfg = synth.get_config(args.workload)
+    cfg = synth.get_config(args.workload) if args.n_choices == 0 else synth.sweep_config(args.n_choices)
     if args.impl == "reference":
         run_reference(args, cfg, rank, world)
         return
@@ -184,7 +203,8 @@ def main():
     pool = [synth.make_batch(cfg, y) for y in range(4)]
     dev_pool = [(torch.from_numpy(x).cuda(), torch.from_numpy(t).cuda()) for x, t in pool]
     host_pool = [(torch.from_numpy(x).pin_memory(), torch.from_numpy(t).pin_memory()) for x, t in pool]
-    spec = npipe.Spec(cfg, flags=npipe.FLAG_TIMING)
+    budget = stage_budget(cfg, D, args.budget_x, npipe) if args.budget_x > 0 else 0
+    spec = npipe.Spec(cfg, flags=npipe.FLAG_TIMING, hbm_weight_budget_bytes=budget, lookahead=args.lookahead)
     if world == 1:
         h = npipe.naspipe_create(spec, 1)
     else:
@@ -278,13 +298,20 @@ def main():
         return
     cpu = None
     if world == 1 and not args.no_cpu:
-        cpu = cpu_baseline(cfg, 2 if cfg["family"] == "transformer" else cfg["n_blocks"])
+        nb = (2 if cfg["d_model"] <= 1024 else 1) if cfg["family"] == "transformer" else cfg["n_blocks"]
+        cpu = cpu_baseline(cfg, nb)
     out = {"metric": "supernet samples/sec", "value": value, "unit": "samples/s", "n_gpus": world,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
            "scaling": "strong", "vs_baseline": None, "dtype": "bf16" if cfg["family"] == "transformer" else "f32",
            "data": "synthetic (N(0,1) inputs/targets, counter-hash init, uniform per-block choices)",
            "config": workload_config(args, cfg, world), "clocks": clk.summary(), "e2e": e2e,
            "gpu_launches": int(launches), "roofline": roofline, "cpu_baseline": cpu,
+           "context_switch": {"budget_bytes_per_stage": budget, "budget_x": args.budget_x,
+                              "lookahead": args.lookahead or 2,
+                              "loads": s1["res_loads"] - s0["res_loads"], "evicts": s1["res_evicts"] - s0["res_evicts"],
+                              "writebacks": s1["writebacks"] - s0["writebacks"],
+                              "h2d_GBps": (s1["h2d_bytes"] - s0["h2d_bytes"]) / (ms / 1000) / 1e9,
+                              "d2h_GBps": (s1["d2h_bytes"] - s0["d2h_bytes"]) / (ms / 1000) / 1e9} if budget else None,
            "loss_finite": bool(losses is None or np.all(np.isfinite(losses)))}
     print(json.dumps(out))
 

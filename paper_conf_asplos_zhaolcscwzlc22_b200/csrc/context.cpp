@@ -48,12 +48,24 @@ CandidateStore::CandidateStore(const Spec& spec, const Planner& planner, int K, 
       CU(cudaHostAlloc(reinterpret_cast<void**>(&cands_[u].stash), cands_[u].n32 * 4, cudaHostAllocDefault));
       CU(cudaEventCreateWithFlags(&cands_[u].ready, cudaEventDisableTiming));
       CU(cudaEventCreateWithFlags(&cands_[u].last_use, cudaEventDisableTiming));
+      CU(cudaEventCreateWithFlags(&cands_[u].wb_done, cudaEventDisableTiming));
     }
+    CU(cudaStreamCreateWithFlags(&evict_, cudaStreamNonBlocking));
     // keep freed blocks in the stream-ordered pool: loads reuse evicted memory
     cudaMemPool_t pool;
     CU(cudaDeviceGetDefaultMemPool(&pool, dev));
     uint64_t thr = UINT64_MAX;
     CU(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
+    // reserve the pool up front (fp32 masters + bf16 shadows of a full budget, plus the
+    // in-flight loads/evictions) so no load pays for growing the pool mid-run
+    void* reserve = nullptr;
+    const size_t rbytes = (size_t)(2.0 * (double)budget_);
+    if (cudaMallocAsync(&reserve, rbytes, 0) == cudaSuccess) {
+      cudaFreeAsync(reserve, 0);
+      cudaStreamSynchronize(0);
+    } else {
+      cudaGetLastError();  // not fatal: the pool grows on demand
+    }
   } else {
     for (int u : uids) {
       cands_[u].w32 = arena->alloc<float>(cands_[u].n32);
@@ -92,12 +104,18 @@ CandidateStore::CandidateStore(const Spec& spec, const Planner& planner, int K, 
 
 CandidateStore::~CandidateStore() {
   cudaSetDevice(dev_);
+  if (evict_) cudaStreamSynchronize(evict_);  // write-backs into the stash have landed
   for (auto& cd : cands_) {
     if (cd.stash) cudaFreeHost(cd.stash);
     if (managed() && cd.w32) cudaFree(cd.w32);
     if (managed() && cd.w16) cudaFree(cd.w16);
     if (cd.ready) cudaEventDestroy(cd.ready);
     if (cd.last_use) cudaEventDestroy(cd.last_use);
+    if (cd.wb_done) cudaEventDestroy(cd.wb_done);
+  }
+  if (evict_) {
+    cudaStreamSynchronize(evict_);
+    cudaStreamDestroy(evict_);
   }
 }
 
@@ -117,6 +135,7 @@ void CandidateStore::set_final() {
 bool CandidateStore::ready() const { return !managed() || belady_->can_decide(); }
 
 void CandidateStore::load(Cand& cd, cudaStream_t copy) {
+  CU(cudaStreamWaitEvent(copy, cd.wb_done, 0));  // a reload reads the written-back stash
   CU(cudaMallocAsync(reinterpret_cast<void**>(&cd.w32), cd.n32 * 4, copy));
   if (cd.n16) CU(cudaMallocAsync(reinterpret_cast<void**>(&cd.w16), cd.n16 * 2, copy));
   CU(cudaMemcpyAsync(cd.w32, cd.stash, cd.n32 * 4, cudaMemcpyHostToDevice, copy));
@@ -127,15 +146,17 @@ void CandidateStore::load(Cand& cd, cudaStream_t copy) {
   ++loads;
 }
 
-void CandidateStore::evict(Cand& cd, bool writeback, cudaStream_t copy) {
-  CU(cudaStreamWaitEvent(copy, cd.last_use, 0));  // the last task reading/updating it is done
+void CandidateStore::evict(Cand& cd, bool writeback, cudaStream_t) {
+  CU(cudaStreamWaitEvent(evict_, cd.last_use, 0));  // the last task reading/updating it is done
+  CU(cudaStreamWaitEvent(evict_, cd.ready, 0));     // (and its load finished)
   if (writeback) {
-    CU(cudaMemcpyAsync(cd.stash, cd.w32, cd.n32 * 4, cudaMemcpyDeviceToHost, copy));
+    CU(cudaMemcpyAsync(cd.stash, cd.w32, cd.n32 * 4, cudaMemcpyDeviceToHost, evict_));
     d2h_bytes += 4.0 * cd.n32;
     ++writebacks;
   }
-  CU(cudaFreeAsync(cd.w32, copy));
-  if (cd.w16) CU(cudaFreeAsync(cd.w16, copy));
+  CU(cudaEventRecord(cd.wb_done, evict_));
+  CU(cudaFreeAsync(cd.w32, evict_));
+  if (cd.w16) CU(cudaFreeAsync(cd.w16, evict_));
   cd.w32 = nullptr;
   cd.w16 = nullptr;
   fam_->bind(cd.j, cd.c, nullptr, nullptr);
@@ -166,6 +187,10 @@ void CandidateStore::before_task(const Task& t, cudaStream_t comp, cudaStream_t 
 void CandidateStore::after_task(const Task& t, cudaStream_t comp) {
   if (!managed()) return;
   for (int64_t u : task_uids(t)) CU(cudaEventRecord(cands_[u].last_use, comp));
+}
+
+void CandidateStore::sync() {
+  if (evict_) CU(cudaStreamSynchronize(evict_));
 }
 
 void CandidateStore::get(int b, int c, float* dst) {

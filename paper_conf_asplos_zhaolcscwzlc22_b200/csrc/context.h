@@ -6,7 +6,8 @@
 // the supernet's operators all reside in CPU storage"); before each task the Belady plan
 // (BeladyResidency: farthest next use within the horizon, depth-L prefetch that fits the
 // budget) issues EVICTs (D2H write-back only if updated since load) and LOADs (H2D + bf16
-// shadow refresh) on the stage's copy stream; the compute stream waits only for the
+// shadow refresh) on the stage's copy stream (write-backs on their own stream, so both PCIe
+// directions run concurrently); the compute stream waits only for the
 // candidates of the task it is about to run, so prefetches for later tasks overlap compute.
 // Numerics are unaffected by residency: a candidate's bytes are the same wherever it lives.
 #pragma once
@@ -36,6 +37,7 @@ class CandidateStore {
   void before_task(const Task& t, cudaStream_t comp, cudaStream_t copy);
   void after_task(const Task& t, cudaStream_t comp);
 
+  void sync();  // wait for outstanding write-backs
   // read-out (streams idle)
   void get(int b, int c, float* dst);
   void set(int b, int c, const float* src, cudaStream_t s);
@@ -51,7 +53,7 @@ class CandidateStore {
     float* stash = nullptr;  // pinned host fp32 master (managed mode)
     float* w32 = nullptr;    // device, when resident
     bf16* w16 = nullptr;
-    cudaEvent_t ready = nullptr, last_use = nullptr;
+    cudaEvent_t ready = nullptr, last_use = nullptr, wb_done = nullptr;
   };
   int uid_of(int b, int c) const { return b * n_ + c; }
   std::vector<int64_t> task_uids(const Task& t) const;
@@ -64,6 +66,7 @@ class CandidateStore {
   Family* fam_;
   int64_t budget_;
   std::vector<Cand> cands_;  // indexed by uid (only this stage's blocks are populated)
+  cudaStream_t evict_ = nullptr;  // D2H write-backs + frees, concurrent with the H2D loads
   std::unique_ptr<BeladyResidency> belady_;
 };
 

@@ -286,6 +286,7 @@ void Engine::drain() {
     CU(cudaSetDevice(st.dev));
     CU(cudaStreamSynchronize(st.copy));
     CU(cudaStreamSynchronize(st.comp));
+    st.store->sync();
   }
   if (tx_)
     for (cudaStream_t s : {tx_->s_act_in, tx_->s_act_out, tx_->s_grad_in, tx_->s_grad_out})
