@@ -167,6 +167,24 @@ int naspipe_plan_residency(const naspipe_plan_t* p, int32_t stage, int64_t budge
   });
 }
 
+int naspipe_plan_comm_schedule(const naspipe_plan_t* p, int32_t rank, int64_t* dst, size_t cap, size_t* n) {
+  return guarded([&] {
+    NP_REQUIRE(p && n && rank >= 0 && rank < p->planner->D(), NASPIPE_EINVAL, "bad args");
+    size_t k = 0;
+    for (const Task& t : p->planner->tasks()) {
+      CommStep ops[2];
+      const int m = comm_ops(t, rank, p->planner->D(), ops);
+      for (int i = 0; i < m; ++i, ++k)
+        if (dst && k < cap) {
+          dst[3 * k] = ops[i].op;
+          dst[3 * k + 1] = ops[i].peer;
+          dst[3 * k + 2] = ops[i].y;
+        }
+    }
+    *n = k;
+  });
+}
+
 void naspipe_plan_destroy(naspipe_plan_t* p) { delete p; }
 
 int naspipe_nccl_unique_id(void* out128) {

@@ -333,21 +333,26 @@ void Engine::issue(const Task& t) {
   const int slot = (int)(t.y % W_);
   StageRt& st = st_[t.K];
   if (rank_ >= 0 && tx_) {
-    // multi-process: post receives for the neighbours' tasks in their plan order
+    // multi-process: post receives for the neighbours' tasks in their plan order (the sends
+    // follow the same rules inside issue_forward / issue_backward; see comm_ops)
     StageRt& me = st_[rank_];
     const size_t n = spec_.batch_elems();
-    if (t.kind == 0 && t.K == rank_ - 1) {
-      CU(cudaSetDevice(me.dev));
-      CU(cudaStreamWaitEvent(tx_->s_act_in, me.ev_b[slot], 0));  // slot free (B(y-W) done)
-      NC(nccl().Recv(me.in[slot], n, ncclFloat32, 0, tx_->act_in, tx_->s_act_in));
-      CU(cudaEventRecord(tx_->ev_act_rx[slot], tx_->s_act_in));
-      p2p_bytes_ += 4.0 * n;
-    } else if (t.kind == 1 && t.K == rank_ + 1) {
-      CU(cudaSetDevice(me.dev));
-      CU(cudaStreamWaitEvent(tx_->s_grad_in, me.ev_b[slot], 0));
-      NC(nccl().Recv(me.gout[slot], n, ncclFloat32, 0, tx_->grad_in, tx_->s_grad_in));
-      CU(cudaEventRecord(tx_->ev_grad_rx[slot], tx_->s_grad_in));
-      p2p_bytes_ += 4.0 * n;
+    CommStep ops[2];
+    const int nops = comm_ops(t, rank_, D_, ops);
+    for (int k = 0; k < nops; ++k) {
+      if (ops[k].op == RECV_ACT) {
+        CU(cudaSetDevice(me.dev));
+        CU(cudaStreamWaitEvent(tx_->s_act_in, me.ev_b[slot], 0));  // slot free (B(y-W) done)
+        NC(nccl().Recv(me.in[slot], n, ncclFloat32, 0, tx_->act_in, tx_->s_act_in));
+        CU(cudaEventRecord(tx_->ev_act_rx[slot], tx_->s_act_in));
+        p2p_bytes_ += 4.0 * n;
+      } else if (ops[k].op == RECV_GRAD) {
+        CU(cudaSetDevice(me.dev));
+        CU(cudaStreamWaitEvent(tx_->s_grad_in, me.ev_b[slot], 0));
+        NC(nccl().Recv(me.gout[slot], n, ncclFloat32, 0, tx_->grad_in, tx_->s_grad_in));
+        CU(cudaEventRecord(tx_->ev_grad_rx[slot], tx_->s_grad_in));
+        p2p_bytes_ += 4.0 * n;
+      }
     }
   }
   if (!st.local) return;

@@ -84,6 +84,26 @@ class Planner {
   std::vector<std::vector<int64_t>> stage_tasks_;
 };
 
+// Point-to-point operations rank `rank` performs for global task t in multi-process mode
+// (one process per stage), in the order the executor walks the plan: it posts the receive
+// of an activation when the upstream F(y, rank-1) starts and of a gradient when the
+// downstream B(y, rank+1) starts, and sends after its own F (to rank+1) and B (to rank-1).
+// Each channel therefore carries y in the sender's plan order, which is exactly the
+// receiver's posting order (test: tests/test_dist_gloo.py).
+enum CommOp { SEND_ACT = 0, RECV_ACT = 1, SEND_GRAD = 2, RECV_GRAD = 3 };
+struct CommStep {
+  int op, peer;
+  int64_t y;
+};
+inline int comm_ops(const Task& t, int rank, int D, CommStep out[2]) {
+  int n = 0;
+  if (t.kind == 0 && t.K == rank - 1) out[n++] = {RECV_ACT, rank - 1, t.y};
+  if (t.kind == 1 && t.K == rank + 1) out[n++] = {RECV_GRAD, rank + 1, t.y};
+  if (t.K == rank && t.kind == 0 && rank < D - 1) out[n++] = {SEND_ACT, rank + 1, t.y};
+  if (t.K == rank && t.kind == 1 && rank > 0) out[n++] = {SEND_GRAD, rank - 1, t.y};
+  return n;
+}
+
 // Belady residency over one stage's planned order (reading A9).
 struct ResidencyEvent { int32_t K; int64_t i; int32_t op; int64_t uid; };  // op 0 LOAD 1 EVICT
 struct ResidencyPlan {
