@@ -204,6 +204,9 @@ int naspipe_plan_deps(const naspipe_plan_t* p, int64_t y, int32_t stage, int64_t
 int naspipe_plan_residency(const naspipe_plan_t* p, int32_t stage, int64_t budget_bytes,
                            int32_t depth, int32_t horizon, int64_t* dst, size_t cap, size_t* n,
                            int64_t* n_writebacks);
+/* Idle ticks per stage [n_stages]: stalled (a queued forward is blocked by a dependency)
+ * and bubble (nothing queued).  busy + stall + bubble = makespan on every stage. */
+int naspipe_plan_idle(const naspipe_plan_t* p, int64_t* stall, int64_t* bubble);
 /* Multi-process point-to-point schedule of one rank (= stage) in the order the executor
  * issues it: 3 int64 per operation (op 0=SEND_ACT to rank+1, 1=RECV_ACT from rank-1,
  * 2=SEND_GRAD to rank-1, 3=RECV_GRAD from rank+1; peer rank; subnet id). */

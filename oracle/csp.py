@@ -113,7 +113,10 @@ def task_costs(choices, stage_of_block, cost_f, cost_b, D):
 
 def simulate_csp(choices, stage_of_block, D, W, cf, cb, lam=0, policy=0, ignore_deps=False,
                  admit=None):
-    """O2.  Returns dict(trace=[(t, K, kind, y)], makespan, order=[[(kind, y)] per stage]).
+    """O2.  Returns dict(trace=[(t, K, kind, y)], makespan, order=[[(kind, y)] per stage],
+    stall=[ticks per stage], bubble=[ticks per stage]).  An idle stage is *stalled* while a
+    queued forward is blocked by a dependency and in a *bubble* while nothing is queued
+    (dependency stall vs bubble).
 
     kind: 0 = F (forward), 1 = B (backward).  cf, cb: int [D][N] task costs (>= 1).
     policy 0: strict backward-first (A5).  policy 1: after a backward, try one forward
@@ -131,6 +134,7 @@ def simulate_csp(choices, stage_of_block, D, W, cf, cb, lam=0, policy=0, ignore_
     last_kind = [None] * D
     deliveries = []                # (time, kind, K, y): kind 0 -> inF[K], 1 -> inB[K]
     trace, order = [], [[] for _ in range(D)]
+    stall, bubble = [0] * D, [0] * D
     t = 0
     done0 = 0
     while True:
@@ -158,7 +162,7 @@ def simulate_csp(choices, stage_of_block, D, W, cf, cb, lam=0, policy=0, ignore_
                 keep.append(dv)
         deliveries = keep
         if done0 == N:
-            return dict(trace=trace, makespan=t, order=order)
+            return dict(trace=trace, makespan=t, order=order, stall=stall, bubble=bubble)
         # (2) stage-0 source under the window
         wm0 = min([y for y in range(N) if y not in fin[0]], default=N)
         for y in range(N):
@@ -197,6 +201,13 @@ def simulate_csp(choices, stage_of_block, D, W, cf, cb, lam=0, policy=0, ignore_
         # (4) advance time
         nxt = [b[0] for b in busy if b is not None] + [dv[0] for dv in deliveries]
         assert nxt, "CSP simulation stalled (no pending event)"
+        dt = min(nxt) - t
+        for K in range(D):
+            if busy[K] is None:
+                if inF[K]:
+                    stall[K] += dt
+                else:
+                    bubble[K] += dt
         t = min(nxt)
 
 

@@ -71,6 +71,7 @@ _sig("naspipe_plan_makespan", C.c_int, [C.c_void_p, _i64p])
 _sig("naspipe_plan_deps", C.c_int, [C.c_void_p, C.c_int64, C.c_int32, _i64p, C.c_size_t, C.POINTER(C.c_size_t)])
 _sig("naspipe_plan_residency", C.c_int, [C.c_void_p, C.c_int32, C.c_int64, C.c_int32, C.c_int32, _i64p,
                                          C.c_size_t, C.POINTER(C.c_size_t), _i64p])
+_sig("naspipe_plan_idle", C.c_int, [C.c_void_p, _i64p, _i64p])
 _sig("naspipe_plan_comm_schedule", C.c_int, [C.c_void_p, C.c_int32, _i64p, C.c_size_t, C.POINTER(C.c_size_t)])
 _sig("naspipe_plan_destroy", None, [C.c_void_p])
 _sig("naspipe_nccl_unique_id", C.c_int, [C.c_void_p])
@@ -81,7 +82,7 @@ EXPORTED_SYMBOLS = [
     "naspipe_get_residency_trace", "naspipe_destroy", "naspipe_param_count", "naspipe_default_costs",
     "naspipe_partition", "naspipe_init_params", "naspipe_plan_create", "naspipe_plan_trace",
     "naspipe_plan_makespan", "naspipe_plan_deps", "naspipe_plan_residency", "naspipe_plan_destroy",
-    "naspipe_plan_comm_schedule",
+    "naspipe_plan_comm_schedule", "naspipe_plan_idle",
     "naspipe_nccl_unique_id", "naspipe_last_error", "naspipe_abi_version"]
 
 
@@ -301,6 +302,13 @@ class Plan:
 
     def deps(self, y: int, stage: int):
         return [int(v) for v in _get_rows(lib.naspipe_plan_deps, self.ptr, y, stage, width=1).ravel()]
+
+    def idle(self, n_stages: int):
+        """(stall ticks [D], bubble ticks [D])."""
+        st = np.zeros(n_stages, dtype=np.int64)
+        bu = np.zeros(n_stages, dtype=np.int64)
+        _check(lib.naspipe_plan_idle(self.ptr, st.ctypes.data_as(_i64p), bu.ctypes.data_as(_i64p)))
+        return st, bu
 
     def comm_schedule(self, rank: int) -> np.ndarray:
         """(op, peer, subnet id) rows: the p2p operations rank `rank` issues, in order."""

@@ -167,6 +167,16 @@ int naspipe_plan_residency(const naspipe_plan_t* p, int32_t stage, int64_t budge
   });
 }
 
+int naspipe_plan_idle(const naspipe_plan_t* p, int64_t* stall, int64_t* bubble) {
+  return guarded([&] {
+    NP_REQUIRE(p && stall && bubble, NASPIPE_EINVAL, "bad args");
+    for (int K = 0; K < p->planner->D(); ++K) {
+      stall[K] = p->planner->stall_ticks()[K];
+      bubble[K] = p->planner->bubble_ticks()[K];
+    }
+  });
+}
+
 int naspipe_plan_comm_schedule(const naspipe_plan_t* p, int32_t rank, int64_t* dst, size_t cap, size_t* n) {
   return guarded([&] {
     NP_REQUIRE(p && n && rank >= 0 && rank < p->planner->D(), NASPIPE_EINVAL, "bad args");

@@ -23,6 +23,8 @@ Planner::Planner(const Spec& spec, int D)
   busy_.assign(D, {});
   last_kind_.assign(D, -1);
   stage_tasks_.assign(D, {});
+  stall_.assign(D, 0);
+  bubble_.assign(D, 0);
 }
 
 int64_t Planner::add_subnet(const int32_t* choice) {
@@ -146,6 +148,8 @@ void Planner::advance() {
     for (auto& dv : deliveries_) nxt = std::min(nxt, dv.time);
     NP_REQUIRE(nxt != std::numeric_limits<int64_t>::max(), NASPIPE_EINTERNAL,
                "CSP planner stalled at tick %lld", (long long)t_);
+    for (int K = 0; K < D_; ++K)
+      if (!busy_[K].on) (inF_[K].empty() ? bubble_ : stall_)[K] += nxt - t_;
     t_ = nxt;
     phase_ = 0;
   }

@@ -53,6 +53,10 @@ class Planner {
   int64_t version(int64_t y, int b) const { return ver_[(size_t)y * m_ + b]; }
   std::vector<int64_t> deps(int64_t y, int K) const;
   int64_t cost(int K, int64_t y, int kind) const;
+  // idle ticks per stage: stalled (a queued forward is blocked by a dependency) / bubble
+  // (nothing queued) — SURVEY §8d C5
+  const std::vector<int64_t>& stall_ticks() const { return stall_; }
+  const std::vector<int64_t>& bubble_ticks() const { return bubble_; }
 
  private:
   bool admissible(int K, int64_t y) const;
@@ -76,6 +80,7 @@ class Planner {
   std::vector<Busy> busy_;
   std::vector<int> last_kind_;
   std::vector<Delivery> deliveries_;
+  std::vector<int64_t> stall_, bubble_;
   int64_t t_ = 0, src_next_ = 0, done0_ = 0, makespan_ = -1;
   int phase_ = 0;
   bool finalized_ = false, done_ = false;

@@ -70,6 +70,8 @@ def test_planner_matches_oracle_bit_exact(seed):
     got = [tuple(int(v) for v in row) for row in plan.trace()]
     assert got == [tuple(r) for r in ref["trace"]]
     assert plan.makespan() == ref["makespan"]
+    st, bu = plan.idle(D)
+    assert list(st) == ref["stall"] and list(bu) == ref["bubble"]
     for y in range(len(ch)):
         for K in range(D):
             assert plan.deps(y, K) == sorted(csp.deps(ch, sob, y, K))

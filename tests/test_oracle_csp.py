@@ -38,6 +38,7 @@ def test_worked_example():
         assert got == g["deps"][K]
     res = csp.simulate_csp(choices, sob, D, g["W"], cf, cb, lam=0, policy=0)
     assert res["makespan"] == g["makespan"]
+    assert res["stall"] == g["stall"] and res["bubble"] == g["bubble"]
     for K in range(D):
         got = [("F" if k == 0 else "B") + f"{y}@{t}" for (t, KK, k, y) in res["trace"] if KK == K]
         assert got == g["stage_order"][K]
@@ -117,6 +118,23 @@ def test_dep_table_equals_literal_alg2(seed):
     alt = csp.simulate_csp(ch, sob, Dn, W, cf, cb, lam=lam, admit=_alg2_admit(ch, sob))
     assert ref["trace"] == alt["trace"]
     assert csp.check_trace(ref["trace"], ch, sob, Dn) == []
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_idle_accounting_identity(seed):
+    """Per stage: busy + stall + bubble = makespan; n = 1 on D = 1 has no idle time."""
+    rng = np.random.default_rng(seed)
+    N, m, n, D = 9, 4, int(rng.integers(1, 4)), int(rng.integers(1, 5))
+    ch = synth.sample_choices(N, m, n, seed)
+    sob = np.array([b * D // m for b in range(m)])
+    cf = rng.integers(1, 4, size=(D, N))
+    cb = rng.integers(1, 5, size=(D, N))
+    res = csp.simulate_csp(ch, sob, D, 2 * D, cf, cb, lam=int(rng.integers(0, 2)))
+    for K in range(D):
+        busy = int(cf[K].sum() + cb[K].sum())
+        assert busy + res["stall"][K] + res["bubble"][K] == res["makespan"]
+    if D == 1:
+        assert res["stall"] == [0] and res["bubble"] == [0]
 
 
 @pytest.mark.parametrize("policy", [0, 1])
