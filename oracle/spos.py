@@ -1,0 +1,254 @@
+"""SPOS-style CNN supernet (configs[1]: "SPOS-style CNN supernet (20 layers x 4 choices,
+synthetic 224x224 images, batch 64)").  TEST INFRASTRUCTURE ONLY (see oracle/__init__.py).
+
+The paper names the CV candidate ops (Table 5: Conv 3x3, Sep Conv 3x3/5x5, Dil
+Conv 3x3) and cites SPOS [9] for the sampling; block internals follow SPOS's
+ShuffleNetV2 search space — reading SURVEY §8c "C2 SPOS candidate" (A16/A17):
+
+* NHWC tensors; every conv is bias-free and followed by BatchNorm in training mode (batch
+  statistics over N*H*W, biased variance, eps 1e-5, trainable gamma/beta, no running stats).
+* Stages: repeats [4,4,8,4], C_out [64,160,320,640]; the first block of a stage has stride 2,
+  inp = C_prev, mid = C_out/2, out_main = C_out - inp; other blocks stride 1 with
+  inp = mid = out_main = C_out/2.
+* Stride 1: x_proj = even channels (passed through), x_main = odd channels;
+  y = concat(x_proj, main(x_main)).
+* Stride 2: y = concat(proj(x), main(x)), proj = dw k s2 -> BN -> pw inp->inp -> BN -> ReLU.
+* Choices 0/1/2 (Shuffle k = 3/5/7): main = pw inp->mid -> BN -> ReLU -> dw k (stride s) -> BN
+  -> pw mid->out_main -> BN -> ReLU.
+* Choice 3 (Xception, k=3): main = dw3 (s) -> BN -> pw inp->mid -> BN -> ReLU -> dw3 -> BN ->
+  pw mid->mid -> BN -> ReLU -> dw3 -> BN -> pw mid->out_main -> BN -> ReLU.
+* Frozen stem: conv3x3 s2 pad 1 3->C0 -> BN(gamma=1, beta=0) -> ReLU.  Frozen head: pw ->
+  BN(1, 0) -> ReLU -> global average pool -> FC (no bias) -> mean cross-entropy.  Frozen
+  parts are never updated (reading A2); their weights use the counter hash with reserved uids.
+* Packing of a candidate: the proj branch's convs (stride-2 blocks) then the main branch's, in
+  order, each conv weight followed by its BN gamma, beta.  pw weights [out, in]; dw weights
+  [C, k, k]; the stem weight [out, kh, kw, in].
+"""
+import numpy as np
+
+EPS = 1e-5
+
+
+# ------------------------------------------------------------------ shapes / layout
+def block_dims(cfg, b):
+    """(stride, inp, mid, out_main, C_out, H_in) of block b."""
+    reps, chans = cfg["stage_repeats"], cfg["stage_channels"]
+    c_prev, H = cfg["stem_channels"], cfg["image_hw"] // 2
+    k = 0
+    for st, (r, co) in enumerate(zip(reps, chans)):
+        for i in range(r):
+            if k == b:
+                if i == 0:
+                    return 2, c_prev, co // 2, co - c_prev, co, H
+                return 1, co // 2, co // 2, co // 2, co, H
+            if i == 0:
+                H //= 2
+            k += 1
+        c_prev = co
+    raise IndexError(b)
+
+
+def convs(cfg, b, c):
+    """Ordered conv list of candidate (b, c): (name, kind 'pw'|'dw', cin, cout, k, stride)."""
+    s, inp, mid, out, _, _ = block_dims(cfg, b)
+    k = cfg["choice_kernel"][c]
+    L = []
+    if s == 2:
+        L += [("p_dw", "dw", inp, inp, k, 2), ("p_pw", "pw", inp, inp, 1, 1)]
+    if not cfg["choice_xception"][c]:
+        L += [("m_pw1", "pw", inp, mid, 1, 1), ("m_dw", "dw", mid, mid, k, s), ("m_pw2", "pw", mid, out, 1, 1)]
+    else:
+        L += [("x_dw1", "dw", inp, inp, 3, s), ("x_pw1", "pw", inp, mid, 1, 1), ("x_dw2", "dw", mid, mid, 3, 1),
+              ("x_pw2", "pw", mid, mid, 1, 1), ("x_dw3", "dw", mid, mid, 3, 1), ("x_pw3", "pw", mid, out, 1, 1)]
+    return L
+
+
+def layout(cfg, b, c):
+    out = []
+    for name, kind, cin, cout, k, _ in convs(cfg, b, c):
+        if kind == "pw":
+            out.append((name, (cout, cin), "uniform", cin))
+        else:
+            out.append((name, (cout, k, k), "uniform", k * k))
+        out.append((name + "_g", (cout,), "ones", 0))
+        out.append((name + "_b", (cout,), "zeros", 0))
+    return out
+
+
+def frozen_layout(cfg):
+    C0, Ch = cfg["stem_channels"], cfg["head_channels"]
+    Clast = cfg["stage_channels"][-1]
+    return {"stem": [("w", (C0, 3, 3, 3), "uniform", 27)],
+            "head": [("w", (Ch, Clast), "uniform", Clast)],
+            "fc": [("w", (cfg["num_classes"], Ch), "uniform", Ch)]}
+
+
+# ------------------------------------------------------------------ primitive ops
+def pad_hw(x, p):
+    return np.pad(x, ((0, 0), (p, p), (p, p), (0, 0)))
+
+
+def dw_fwd(x, w, s):
+    """Depthwise conv, pad k//2: y[b,i,j,c] = sum_{u,v} xpad[b, i*s+u, j*s+v, c] w[c,u,v]."""
+    k = w.shape[1]
+    p = k // 2
+    xp = pad_hw(x, p)
+    B, H, W, C = x.shape
+    Ho, Wo = (H + 2 * p - k) // s + 1, (W + 2 * p - k) // s + 1
+    y = np.zeros((B, Ho, Wo, C))
+    for u in range(k):
+        for v in range(k):
+            y += xp[:, u:u + s * (Ho - 1) + 1:s, v:v + s * (Wo - 1) + 1:s, :] * w[:, u, v]
+    return y
+
+
+def dw_bwd(x, w, s, dy):
+    k = w.shape[1]
+    p = k // 2
+    xp = pad_hw(x, p)
+    B, Ho, Wo, C = dy.shape
+    dxp = np.zeros_like(xp)
+    dw = np.zeros_like(w)
+    for u in range(k):
+        for v in range(k):
+            sl = (slice(None), slice(u, u + s * (Ho - 1) + 1, s), slice(v, v + s * (Wo - 1) + 1, s), slice(None))
+            dxp[sl] += dy * w[:, u, v]
+            dw[:, u, v] = np.sum(dy * xp[sl], axis=(0, 1, 2))
+    return dxp[:, p:p + x.shape[1], p:p + x.shape[2], :], dw
+
+
+def conv_fwd(x, w, s):
+    """Dense conv (stem): w [Cout, k, k, Cin], pad k//2."""
+    k = w.shape[1]
+    p = k // 2
+    xp = pad_hw(x, p)
+    B, H, W, _ = x.shape
+    Ho, Wo = (H + 2 * p - k) // s + 1, (W + 2 * p - k) // s + 1
+    y = np.zeros((B, Ho, Wo, w.shape[0]))
+    for u in range(k):
+        for v in range(k):
+            y += xp[:, u:u + s * (Ho - 1) + 1:s, v:v + s * (Wo - 1) + 1:s, :] @ w[:, u, v, :].T
+    return y
+
+
+def bn_fwd(x, g, b):
+    mu = x.mean(axis=(0, 1, 2))
+    var = ((x - mu) ** 2).mean(axis=(0, 1, 2))
+    rstd = 1.0 / np.sqrt(var + EPS)
+    xh = (x - mu) * rstd
+    return g * xh + b, (xh, rstd)
+
+
+def bn_bwd(dy, g, cache):
+    xh, rstd = cache
+    dxh = dy * g
+    dx = rstd * (dxh - dxh.mean(axis=(0, 1, 2)) - xh * (dxh * xh).mean(axis=(0, 1, 2)))
+    return dx, (dy * xh).sum(axis=(0, 1, 2)), dy.sum(axis=(0, 1, 2))
+
+
+# ------------------------------------------------------------------ conv -> BN [-> ReLU] unit
+def _unit_fwd(p, name, kind, s, relu, x):
+    w = p[name]
+    z = dw_fwd(x, w, s) if kind == "dw" else x @ w.T
+    y, cb = bn_fwd(z, p[name + "_g"], p[name + "_b"])
+    if relu:
+        y = np.maximum(y, 0.0)
+    return y, (x, cb, y if relu else None)
+
+
+def _unit_bwd(p, name, kind, s, dy, tape, grads):
+    x, cb, yr = tape
+    if yr is not None:
+        dy = dy * (yr > 0)
+    dz, grads[name + "_g"], grads[name + "_b"] = bn_bwd(dy, p[name + "_g"], cb)
+    if kind == "dw":
+        dx, grads[name] = dw_bwd(x, p[name], s, dz)
+    else:
+        grads[name] = np.einsum("bhwo,bhwi->oi", dz, x)
+        dx = dz @ p[name]
+    return dx
+
+
+def _chain(cfg, b, c, which):
+    """Units of the proj ('p') or main branch: (name, kind, stride, relu)."""
+    out = []
+    cl = [u for u in convs(cfg, b, c) if u[0].startswith(which)]
+    for i, (name, kind, _, _, _, s) in enumerate(cl):
+        relu = kind == "pw" and (which == "p" or i == len(cl) - 1 or name in ("m_pw1", "x_pw1", "x_pw2"))
+        out.append((name, kind, s, relu))
+    return out
+
+
+def block_fwd(cfg, b, c, p, x):
+    s = block_dims(cfg, b)[0]
+    main_key = "x" if cfg["choice_xception"][c] else "m"
+    if s == 1:
+        xp, xm = x[..., 0::2], x[..., 1::2]
+    else:
+        xp = xm = x
+    tapes = {"p": [], main_key: []}
+    h = xm
+    for name, kind, st, relu in _chain(cfg, b, c, main_key):
+        h, t = _unit_fwd(p, name, kind, st, relu, h)
+        tapes[main_key].append(t)
+    main = h
+    if s == 2:
+        h = xp
+        for name, kind, st, relu in _chain(cfg, b, c, "p"):
+            h, t = _unit_fwd(p, name, kind, st, relu, h)
+            tapes["p"].append(t)
+        xp = h
+    return np.concatenate([xp, main], axis=-1), tapes
+
+
+def block_bwd(cfg, b, c, p, tapes, dy):
+    s, inp = block_dims(cfg, b)[:2]
+    main_key = "x" if cfg["choice_xception"][c] else "m"
+    cp = inp if s == 2 else dy.shape[-1] // 2
+    d_proj, d_main = dy[..., :cp], dy[..., cp:]
+    grads = {}
+    h = d_main
+    chain = _chain(cfg, b, c, main_key)
+    for (name, kind, st, relu), t in zip(reversed(chain), reversed(tapes[main_key])):
+        h = _unit_bwd(p, name, kind, st, h, t, grads)
+    if s == 1:
+        dx = np.zeros(d_proj.shape[:-1] + (2 * cp,))
+        dx[..., 0::2] = d_proj
+        dx[..., 1::2] = h
+        return dx, grads
+    g = d_proj
+    for (name, kind, st, relu), t in zip(reversed(_chain(cfg, b, c, "p")), reversed(tapes["p"])):
+        g = _unit_bwd(p, name, kind, st, g, t, grads)
+    return h + g, grads
+
+
+# ------------------------------------------------------------------ frozen stem / head
+def stem_fwd(fz, x):
+    z = conv_fwd(x, fz["stem"]["w"], 2)
+    C = z.shape[-1]
+    y, _ = bn_fwd(z, np.ones(C), np.zeros(C))
+    return np.maximum(y, 0.0)
+
+
+def head_loss(fz, x, labels):
+    """Returns (loss, dL/dx) through pw -> BN -> ReLU -> GAP -> FC -> mean CE (frozen)."""
+    wh, wf = fz["head"]["w"], fz["fc"]["w"]
+    z = x @ wh.T
+    C = z.shape[-1]
+    y, cb = bn_fwd(z, np.ones(C), np.zeros(C))
+    r = np.maximum(y, 0.0)
+    gap = r.mean(axis=(1, 2))
+    logits = gap @ wf.T
+    mx = logits.max(axis=1, keepdims=True)
+    lse = mx[:, 0] + np.log(np.exp(logits - mx).sum(axis=1))
+    B = x.shape[0]
+    loss = float(np.mean(lse - logits[np.arange(B), labels]))
+    prob = np.exp(logits - lse[:, None])
+    dlog = prob
+    dlog[np.arange(B), labels] -= 1.0
+    dlog /= B
+    dgap = dlog @ wf
+    dr = np.broadcast_to(dgap[:, None, None, :] / (r.shape[1] * r.shape[2]), r.shape)
+    dy = dr * (r > 0)
+    dz, _, _ = bn_bwd(dy, np.ones(C), cb)
+    return loss, dz @ wh

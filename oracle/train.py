@@ -18,9 +18,9 @@ no stem/head for the MLP/transformer families (A2).
 """
 import numpy as np
 
-from . import mlp, transformer
+from . import mlp, spos, transformer
 
-FAMILIES = {"mlp": mlp, "transformer": transformer}
+FAMILIES = {"mlp": mlp, "transformer": transformer, "spos": spos}
 
 
 def candidate_layout(cfg, b, c):
@@ -28,6 +28,8 @@ def candidate_layout(cfg, b, c):
         return mlp.layout(cfg)
     if cfg["family"] == "transformer":
         return transformer.layout(cfg, c)
+    if cfg["family"] == "spos":
+        return spos.layout(cfg, b, c)
     raise ValueError(cfg["family"])
 
 
@@ -69,11 +71,42 @@ def _block_bwd(cfg, p, tape, dy):
     return transformer.backward(p, tape, dy)
 
 
+def frozen_theta(cfg):
+    """SPOS frozen stem / head / FC weights: counter hash with reserved uids m*n + {0,1,2}."""
+    from synth import init_packed
+    base = cfg["n_blocks"] * cfg["n_choices"]
+    out = {}
+    for k, (part, segs) in enumerate(spos.frozen_layout(cfg).items()):
+        name, shape, kind, fan = segs[0]
+        v = init_packed(cfg["init_seed"], base + k, [(int(np.prod(shape)), kind, fan)])
+        out[part] = {name: v.astype(np.float64).reshape(shape)}
+    return out
+
+
+def _spos_step(cfg, theta, choice, x, labels):
+    fz = frozen_theta(cfg)
+    h = spos.stem_fwd(fz, np.asarray(x, dtype=np.float64))
+    tapes = []
+    for b, c in enumerate(choice):
+        h, tp = spos.block_fwd(cfg, b, int(c), theta[(b, int(c))], h)
+        tapes.append(tp)
+    loss, dy = spos.head_loss(fz, h, np.asarray(labels, dtype=np.int64))
+    grads = {}
+    for b in reversed(range(len(choice))):
+        c = int(choice[b])
+        dy, g = spos.block_bwd(cfg, b, c, theta[(b, c)], tapes[b], dy)
+        grads[(b, c)] = g
+    return loss, grads
+
+
 def subnet_step(cfg, theta, choice, x, t):
     """One subnet's forward + backward.  Returns (loss, grads{(b,c): dict}).
 
     Does not modify theta.  All gradients are taken at the pre-update parameters.
+    SPOS: t is the integer label vector; the loss is the frozen head's mean cross-entropy.
     """
+    if cfg["family"] == "spos":
+        return _spos_step(cfg, theta, choice, x, t)
     h = np.asarray(x, dtype=np.float64)
     tapes = []
     for b, c in enumerate(choice):

@@ -54,6 +54,17 @@ CONFIGS = {
                              d_model=192, seq_len=128,
                              choice_heads=[3, 2, 3], choice_ffn=[320, 384, 192],
                              lr=0.01, compute_dtype="bf16", n_stages=2, n_subnets=8),
+    # configs[1]: "SPOS-style CNN supernet (20 layers x 4 choices, synthetic 224x224 images,
+    # batch 64)": repeats [4,4,8,4], C_out [64,160,320,640], choices {Shuffle 3/5/7, Xception}
+    "spos": dict(family="spos", n_blocks=20, n_choices=4, batch=64, image_hw=224, num_classes=1000,
+                 stage_repeats=[4, 4, 8, 4], stage_channels=[64, 160, 320, 640], stem_channels=16,
+                 head_channels=1024, choice_kernel=[3, 5, 7, 3], choice_xception=[0, 0, 0, 1],
+                 lr=0.01, compute_dtype="bf16", n_stages=8, n_subnets=256),
+    # small SPOS supernet for parity tests: every channel count a multiple of 16
+    "tiny_spos": dict(family="spos", n_blocks=5, n_choices=4, batch=4, image_hw=64, num_classes=10,
+                      stage_repeats=[1, 2, 1, 1], stage_channels=[32, 64, 96, 128], stem_channels=16,
+                      head_channels=64, choice_kernel=[3, 5, 7, 3], choice_xception=[0, 0, 0, 1],
+                      lr=0.01, compute_dtype="bf16", n_stages=2, n_subnets=8),
 }
 
 
@@ -90,15 +101,21 @@ def batch_shape(cfg: dict) -> tuple:
         return (cfg["batch"], cfg["width"])
     if cfg["family"] == "transformer":
         return (cfg["batch"], cfg["seq_len"], cfg["d_model"])
+    if cfg["family"] == "spos":
+        return (cfg["batch"], cfg["image_hw"], cfg["image_hw"], 3)
     raise ValueError(cfg["family"])
 
 
 def make_batch(cfg: dict, y: int, seed: int = DATA_SEED):
-    """Input and target for subnet y: N(0,1) float32, independent of N."""
+    """Input and target for subnet y: N(0,1) float32, independent of N.
+    SPOS: the target is an int32 label vector, uniform in [0, num_classes)."""
     rng = np.random.default_rng([seed, int(y)])
     shp = batch_shape(cfg)
     x = rng.standard_normal(shp, dtype=np.float32)
-    t = rng.standard_normal(shp, dtype=np.float32)
+    if cfg["family"] == "spos":
+        t = rng.integers(0, cfg["num_classes"], size=cfg["batch"], dtype=np.int64).astype(np.int32)
+    else:
+        t = rng.standard_normal(shp, dtype=np.float32)
     return x, t
 
 

@@ -1,0 +1,143 @@
+"""Pins for oracle/spos.py (configs[1] SPOS CNN family).
+
+* depthwise and dense convolutions against their definition written as explicit loops, and
+  special cases (1x1 depthwise = per-channel scaling, centred delta kernel = identity);
+* BatchNorm output statistics (closed form);
+* central finite differences (fp64) of every block variant (stride 1/2 x Shuffle 3/5/7 and
+  Xception) for the input and every parameter, and of the frozen head's cross-entropy;
+* the trainer's SGD step on a tiny SPOS supernet changes exactly the active candidates.
+"""
+import numpy as np
+import pytest
+
+import synth
+from oracle import spos, train
+
+
+def _dw_loops(x, w, s):
+    B, H, W, C = x.shape
+    k = w.shape[1]
+    p = k // 2
+    Ho, Wo = (H + 2 * p - k) // s + 1, (W + 2 * p - k) // s + 1
+    y = np.zeros((B, Ho, Wo, C))
+    for b in range(B):
+        for i in range(Ho):
+            for j in range(Wo):
+                for c in range(C):
+                    acc = 0.0
+                    for u in range(k):
+                        for v in range(k):
+                            ii, jj = i * s + u - p, j * s + v - p
+                            if 0 <= ii < H and 0 <= jj < W:
+                                acc += x[b, ii, jj, c] * w[c, u, v]
+                    y[b, i, j, c] = acc
+    return y
+
+
+@pytest.mark.parametrize("k,s", [(3, 1), (5, 2), (7, 1), (3, 2)])
+def test_depthwise_matches_loops(k, s):
+    rng = np.random.default_rng(k * 10 + s)
+    x = rng.standard_normal((2, 6, 6, 3))
+    w = rng.standard_normal((3, k, k))
+    np.testing.assert_allclose(spos.dw_fwd(x, w, s), _dw_loops(x, w, s), rtol=1e-12, atol=1e-12)
+
+
+def test_depthwise_special_cases():
+    rng = np.random.default_rng(0)
+    x = rng.standard_normal((2, 5, 5, 4))
+    w1 = rng.standard_normal((4, 1, 1))
+    np.testing.assert_allclose(spos.dw_fwd(x, w1, 1), x * w1[:, 0, 0], rtol=1e-14)
+    delta = np.zeros((4, 3, 3))
+    delta[:, 1, 1] = 1.0
+    np.testing.assert_allclose(spos.dw_fwd(x, delta, 1), x, rtol=1e-14)
+    np.testing.assert_allclose(spos.dw_fwd(x, delta, 2), x[:, ::2, ::2, :], rtol=1e-14)
+
+
+def test_dense_conv_matches_loops():
+    rng = np.random.default_rng(1)
+    x = rng.standard_normal((1, 6, 6, 3))
+    w = rng.standard_normal((4, 3, 3, 3))
+    y = spos.conv_fwd(x, w, 2)
+    ref = np.zeros_like(y)
+    for i in range(3):
+        for j in range(3):
+            for o in range(4):
+                for u in range(3):
+                    for v in range(3):
+                        ii, jj = 2 * i + u - 1, 2 * j + v - 1
+                        if 0 <= ii < 6 and 0 <= jj < 6:
+                            ref[0, i, j, o] += x[0, ii, jj, :] @ w[o, u, v, :]
+    np.testing.assert_allclose(y, ref, rtol=1e-12)
+
+
+def test_batchnorm_closed_form():
+    rng = np.random.default_rng(2)
+    x = rng.standard_normal((3, 4, 4, 5)) * 3 + 2
+    y, _ = spos.bn_fwd(x, np.ones(5), np.zeros(5))
+    var = x.var(axis=(0, 1, 2))
+    np.testing.assert_allclose(y.mean(axis=(0, 1, 2)), 0, atol=1e-12)
+    np.testing.assert_allclose(y.var(axis=(0, 1, 2)), var / (var + 1e-5), rtol=1e-10)
+
+
+MINI = dict(family="spos", n_blocks=2, n_choices=4, batch=2, image_hw=16, num_classes=5,
+            stage_repeats=[2], stage_channels=[8], stem_channels=4, head_channels=6,
+            choice_kernel=[3, 5, 7, 3], choice_xception=[0, 0, 0, 1], lr=0.01, init_seed=2)
+
+
+def _check_fd(f, analytic, arr, rng, n=6, eps=1e-6):
+    idxs = rng.choice(arr.size, size=min(n, arr.size), replace=False)
+    for fi in idxs:
+        i = np.unravel_index(fi, arr.shape)
+        old = arr[i]
+        arr[i] = old + eps
+        fp = f()
+        arr[i] = old - eps
+        fm = f()
+        arr[i] = old
+        num = (fp - fm) / (2 * eps)
+        assert abs(num - analytic[i]) <= 1e-5 * max(abs(num), abs(analytic[i])) + 1e-7, (i, num, analytic[i])
+
+
+@pytest.mark.parametrize("b", [0, 1])          # block 0: stride 2 (proj branch), block 1: stride 1
+@pytest.mark.parametrize("c", [0, 1, 2, 3])    # Shuffle 3/5/7, Xception
+def test_block_fd(b, c):
+    rng = np.random.default_rng(10 * b + c)
+    s, inp, mid, out, cout, H = spos.block_dims(MINI, b)
+    p = {}
+    for name, shape, kind, _ in spos.layout(MINI, b, c):
+        if kind == "uniform":
+            p[name] = rng.standard_normal(shape) * 0.5
+        else:
+            p[name] = (1.0 if kind == "ones" else 0.0) + 0.2 * rng.standard_normal(shape)
+    cin = inp if s == 2 else cout
+    x = rng.standard_normal((2, H, H, cin))
+    y, tapes = spos.block_fwd(MINI, b, c, p, x)
+    assert y.shape == (2, H // s, H // s, cout)
+    R = rng.standard_normal(y.shape)
+    dx, g = spos.block_bwd(MINI, b, c, p, tapes, R)
+    loss = lambda: float(np.sum(spos.block_fwd(MINI, b, c, p, x)[0] * R))   # noqa: E731
+    _check_fd(loss, dx, x, rng)
+    for name in p:
+        _check_fd(loss, g[name], p[name], rng, n=3)
+
+
+def test_head_loss_fd():
+    rng = np.random.default_rng(5)
+    fz = train.frozen_theta(MINI)
+    x = rng.standard_normal((2, 4, 4, 8))
+    labels = np.array([1, 3])
+    _, dx = spos.head_loss(fz, x, labels)
+    _check_fd(lambda: spos.head_loss(fz, x, labels)[0], dx, x, rng, n=10)
+
+
+def test_tiny_spos_training_updates_only_active():
+    cfg = synth.get_config("tiny_spos")
+    ch = synth.sample_choices(2, cfg["n_blocks"], cfg["n_choices"])
+    batches = [synth.make_batch(cfg, y) for y in range(2)]
+    th0 = train.initial_theta(cfg)
+    th, losses = train.train_sequential(cfg, th0, ch, batches)
+    assert np.all(np.isfinite(losses)) and abs(losses[0] - np.log(cfg["num_classes"])) < 1.0
+    used = {(b, int(ch[y][b])) for y in range(2) for b in range(cfg["n_blocks"])}
+    for k in th:
+        changed = not np.array_equal(th[k], th0[k].astype(np.float64))
+        assert changed == (k in used), k
