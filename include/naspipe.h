@@ -23,6 +23,12 @@
  *       MLP:          W[d,d], b[d]
  *       TRANSFORMER:  Wqkv[3d,d], bqkv[3d], Wo[d,d], bo[d], ln1.g[d], ln1.b[d],
  *                     W1[f,d], b1[f], W2[d,f], b2[d], ln2.g[d], ln2.b[d]
+ *       SPOS_CNN:     for each conv of the candidate in order (stride-2 blocks: the proj
+ *                     branch's dw, pw first; then the main branch's convs), the conv weight
+ *                     (pw [out,in]; dw [C,k,k]) followed by its BatchNorm gamma[out], beta[out].
+ *                     Main branch, choices with kernel k (SURVEY §8c "C2 SPOS candidate",
+ *                     DESIGN.md A16/A27): Shuffle = pw in->mid, dw k (stride s), pw mid->out;
+ *                     Xception = dw3 (s), pw in->mid, dw3, pw mid->mid, dw3, pw mid->out.
  */
 #ifndef NASPIPE_H_
 #define NASPIPE_H_
@@ -37,7 +43,7 @@ extern "C" {
 #pragma GCC visibility push(default) /* the library builds with -fvisibility=hidden */
 #endif
 
-#define NASPIPE_ABI_VERSION 1
+#define NASPIPE_ABI_VERSION 2
 
 typedef enum {
   NASPIPE_OK = 0,
@@ -82,6 +88,18 @@ typedef enum { NASPIPE_FP32 = 0, NASPIPE_BF16 = 1 } naspipe_dtype; /* compute dt
  *                 candidates resident (no context switching).
  *   bwd_policy    0 = strict backward-first (reading A5); 1 = Alg.1 alternation.
  *   link_latency  lambda ticks for stage-boundary deliveries in the planner (reading A8).
+ *   SPOS_CNN only (SPOS [9] search space; op types of Table 5):
+ *   image_hw      input resolution (square), divisible by 2^(1 + n_cnn_stages)
+ *   num_classes   classes of the frozen FC head
+ *   stem_channels frozen stem conv3x3 s2 3->stem_channels (+BN(1,0)+ReLU), % 16 == 0
+ *   head_channels frozen head pw Clast->head_channels, BN(1,0), ReLU, GAP, FC (no bias)
+ *   n_cnn_stages, stage_repeats[n_cnn_stages] (sum = n_blocks), stage_channels[..] (% 32,
+ *                 strictly increasing, first > stem_channels): the first block of each
+ *                 stage has stride 2, inp = C_prev, mid = C/2, out = C - C_prev; the
+ *                 others stride 1 with inp = mid = out = C/2 (channel split).
+ *   choice_kernel[n] (3, 5 or 7), choice_xception[n] (0 = Shuffle, 1 = Xception k=3)
+ *   Frozen stem/head/FC weights use the counter hash with uids m*n + {0, 1, 2}, fan_in
+ *   27 / C_last / head_channels; they are never updated (reading A2).
  */
 typedef struct {
   int32_t abi_version; /* = NASPIPE_ABI_VERSION */
@@ -107,6 +125,16 @@ typedef struct {
   int32_t bwd_policy;
   int32_t link_latency;
   int32_t flags;
+  /* SPOS_CNN (ignored otherwise) */
+  int32_t image_hw;
+  int32_t num_classes;
+  int32_t stem_channels;
+  int32_t head_channels;
+  int32_t n_cnn_stages;
+  const int32_t* stage_repeats;
+  const int32_t* stage_channels;
+  const int32_t* choice_kernel;
+  const int32_t* choice_xception;
 } naspipe_supernet_spec;
 
 /* naspipe_batch.where */
@@ -117,7 +145,9 @@ typedef struct {
 #define NASPIPE_BATCH_SYNTHETIC 2 /* generated on the device from synth_seed (perf only)  */
 
 /* One subnet's batch: input [batch x sample] and target [batch x sample] float32, where
- * sample = width (MLP) or seq_len*d_model (TRANSFORMER), row-major. */
+ * sample = width (MLP) or seq_len*d_model (TRANSFORMER), row-major.  SPOS_CNN: input is
+ * float32 NHWC [batch, image_hw, image_hw, 3], target is int32 labels [batch] in
+ * [0, num_classes) (loss = mean cross-entropy of the frozen head, reading A18). */
 typedef struct {
   const void* input;
   const void* target;
@@ -187,6 +217,12 @@ int naspipe_partition(const naspipe_supernet_spec* spec, int32_t n_stages, int32
 /* Initial packed parameters of one candidate (same generator the engine uses). */
 int naspipe_init_params(const naspipe_supernet_spec* spec, int32_t block, int32_t choice,
                         float* dst, size_t n_floats);
+
+/* SPOS_CNN frozen (never-updated, reading A2) weights: part 0 = stem [C0,3,3,3] ([out, kh,
+ * kw, in]), 1 = head 1x1 conv [head_channels, C_last], 2 = FC [num_classes, head_channels];
+ * the counter hash of init_seed with uid = n_blocks*n_choices + part.  EINVAL for other
+ * families or a size mismatch. */
+int naspipe_init_frozen(const naspipe_supernet_spec* spec, int32_t part, float* dst, size_t n_floats);
 
 typedef struct naspipe_plan_handle naspipe_plan_t;
 /* Plan N subnets (choices [N*m]) on n_stages stages: the logical-time CSP schedule

@@ -23,10 +23,38 @@ ShuffleNetV2 search space — reading SURVEY §8c "C2 SPOS candidate" (DESIGN.md
 * Packing of a candidate: the proj branch's convs (stride-2 blocks) then the main branch's, in
   order, each conv weight followed by its BN gamma, beta.  pw weights [out, in]; dw weights
   [C, k, k]; the stem weight [out, kh, kw, in].
+
+Storage precision (reading A28).  Every function takes an optional ``q``: the
+rounding applied where a stored tensor is written.  ``q = None`` (default) is the plain fp64
+definition.  ``q = to_bf16`` rounds exactly the tensors the bf16 path stores (conv outputs
+z, BN/ReLU outputs y, 1x1-conv weight operands, the head's operands, and the gradients dz,
+dx between units and blocks) with round-to-nearest-even, and computes everything else in
+fp64.  Reason: the ReLU masks are decisions taken from floating point; the task fixes that
+both sides take such decisions in the same precision, and without it a 2^-9 perturbation
+of the activations flips ~0.2 % of the masks, which moves the fp64 weight update of this
+family by ~20 % (tools/diag_spos.py; A28) -- no bf16 implementation can meet
+1e-3 against the plain definition.
 """
 import numpy as np
 
 EPS = 1e-5
+
+
+def to_bf16(x):
+    """Round to the nearest bfloat16 (ties to even), returned as float64.  fp64 -> fp32 is
+    round-to-nearest first (the kernels hold fp32 values when they store bf16)."""
+    a = np.ascontiguousarray(x, dtype=np.float32)
+    u = a.view(np.uint32).astype(np.uint64)
+    r = ((u + np.uint64(0x7FFF) + ((u >> np.uint64(16)) & np.uint64(1))) >> np.uint64(16)) << np.uint64(16)
+    out = r.astype(np.uint32).view(np.float32).astype(np.float64)
+    nan = np.isnan(a)
+    if np.any(nan):
+        out[nan] = np.nan
+    return out
+
+
+def _id(x):
+    return x
 
 
 # ------------------------------------------------------------------ shapes / layout
@@ -147,26 +175,30 @@ def bn_bwd(dy, g, cache):
 
 
 # ------------------------------------------------------------------ conv -> BN [-> ReLU] unit
-def _unit_fwd(p, name, kind, s, relu, x):
+def _unit_fwd(p, name, kind, s, relu, x, q=_id):
     w = p[name]
-    z = dw_fwd(x, w, s) if kind == "dw" else x @ w.T
+    z = q(dw_fwd(x, w, s) if kind == "dw" else x @ q(w).T)
     y, cb = bn_fwd(z, p[name + "_g"], p[name + "_b"])
     if relu:
         y = np.maximum(y, 0.0)
+    y = q(y)
     return y, (x, cb, y if relu else None)
 
 
-def _unit_bwd(p, name, kind, s, dy, tape, grads):
+def _unit_bwd(p, name, kind, s, dy, tape, grads, q=_id, add=None):
+    """dx of the unit (+ add, the other branch's gradient of the same input, before the
+    storage rounding), accumulating the parameter gradients into grads."""
     x, cb, yr = tape
     if yr is not None:
         dy = dy * (yr > 0)
     dz, grads[name + "_g"], grads[name + "_b"] = bn_bwd(dy, p[name + "_g"], cb)
+    dz = q(dz)
     if kind == "dw":
         dx, grads[name] = dw_bwd(x, p[name], s, dz)
     else:
         grads[name] = np.einsum("bhwo,bhwi->oi", dz, x)
-        dx = dz @ p[name]
-    return dx
+        dx = dz @ q(p[name])
+    return q(dx if add is None else dx + add)
 
 
 def _chain(cfg, b, c, which):
@@ -179,7 +211,7 @@ def _chain(cfg, b, c, which):
     return out
 
 
-def block_fwd(cfg, b, c, p, x):
+def block_fwd(cfg, b, c, p, x, q=_id):
     s = block_dims(cfg, b)[0]
     main_key = "x" if cfg["choice_xception"][c] else "m"
     if s == 1:
@@ -189,19 +221,19 @@ def block_fwd(cfg, b, c, p, x):
     tapes = {"p": [], main_key: []}
     h = xm
     for name, kind, st, relu in _chain(cfg, b, c, main_key):
-        h, t = _unit_fwd(p, name, kind, st, relu, h)
+        h, t = _unit_fwd(p, name, kind, st, relu, h, q)
         tapes[main_key].append(t)
     main = h
     if s == 2:
         h = xp
         for name, kind, st, relu in _chain(cfg, b, c, "p"):
-            h, t = _unit_fwd(p, name, kind, st, relu, h)
+            h, t = _unit_fwd(p, name, kind, st, relu, h, q)
             tapes["p"].append(t)
         xp = h
     return np.concatenate([xp, main], axis=-1), tapes
 
 
-def block_bwd(cfg, b, c, p, tapes, dy):
+def block_bwd(cfg, b, c, p, tapes, dy, q=_id):
     s, inp = block_dims(cfg, b)[:2]
     main_key = "x" if cfg["choice_xception"][c] else "m"
     cp = inp if s == 2 else dy.shape[-1] // 2
@@ -210,33 +242,35 @@ def block_bwd(cfg, b, c, p, tapes, dy):
     h = d_main
     chain = _chain(cfg, b, c, main_key)
     for (name, kind, st, relu), t in zip(reversed(chain), reversed(tapes[main_key])):
-        h = _unit_bwd(p, name, kind, st, h, t, grads)
+        h = _unit_bwd(p, name, kind, st, h, t, grads, q)
     if s == 1:
         dx = np.zeros(d_proj.shape[:-1] + (2 * cp,))
         dx[..., 0::2] = d_proj
         dx[..., 1::2] = h
         return dx, grads
     g = d_proj
-    for (name, kind, st, relu), t in zip(reversed(_chain(cfg, b, c, "p")), reversed(tapes["p"])):
-        g = _unit_bwd(p, name, kind, st, g, t, grads)
-    return h + g, grads
+    pchain = list(zip(reversed(_chain(cfg, b, c, "p")), reversed(tapes["p"])))
+    for i, ((name, kind, st, relu), t) in enumerate(pchain):
+        last = i == len(pchain) - 1     # the proj branch's first unit: add the main branch's dx
+        g = _unit_bwd(p, name, kind, st, g, t, grads, q, add=h if last else None)
+    return g, grads
 
 
 # ------------------------------------------------------------------ frozen stem / head
-def stem_fwd(fz, x):
-    z = conv_fwd(x, fz["stem"]["w"], 2)
+def stem_fwd(fz, x, q=_id):
+    z = q(conv_fwd(x, fz["stem"]["w"], 2))
     C = z.shape[-1]
     y, _ = bn_fwd(z, np.ones(C), np.zeros(C))
-    return np.maximum(y, 0.0)
+    return q(np.maximum(y, 0.0))
 
 
-def head_loss(fz, x, labels):
+def head_loss(fz, x, labels, q=_id):
     """Returns (loss, dL/dx) through pw -> BN -> ReLU -> GAP -> FC -> mean CE (frozen)."""
-    wh, wf = fz["head"]["w"], fz["fc"]["w"]
-    z = x @ wh.T
+    wh, wf = q(fz["head"]["w"]), fz["fc"]["w"]
+    z = q(x @ wh.T)
     C = z.shape[-1]
     y, cb = bn_fwd(z, np.ones(C), np.zeros(C))
-    r = np.maximum(y, 0.0)
+    r = q(np.maximum(y, 0.0))
     gap = r.mean(axis=(1, 2))
     logits = gap @ wf.T
     mx = logits.max(axis=1, keepdims=True)
@@ -248,7 +282,7 @@ def head_loss(fz, x, labels):
     dlog[np.arange(B), labels] -= 1.0
     dlog /= B
     dgap = dlog @ wf
-    dr = np.broadcast_to(dgap[:, None, None, :] / (r.shape[1] * r.shape[2]), r.shape)
+    dr = q(np.broadcast_to(dgap[:, None, None, :] / (r.shape[1] * r.shape[2]), r.shape))
     dy = dr * (r > 0)
     dz, _, _ = bn_bwd(dy, np.ones(C), cb)
-    return loss, dz @ wh
+    return loss, q(q(dz) @ wh)

@@ -84,17 +84,20 @@ def frozen_theta(cfg):
 
 
 def _spos_step(cfg, theta, choice, x, labels):
+    """SPOS step; cfg["storage"] == "bf16" selects the kernel-precision storage rounding of
+    reading A28 (spos.to_bf16 at every stored tensor), default plain fp64."""
+    q = spos.to_bf16 if cfg.get("storage") == "bf16" else spos._id
     fz = frozen_theta(cfg)
-    h = spos.stem_fwd(fz, np.asarray(x, dtype=np.float64))
+    h = spos.stem_fwd(fz, np.asarray(x, dtype=np.float64), q)
     tapes = []
     for b, c in enumerate(choice):
-        h, tp = spos.block_fwd(cfg, b, int(c), theta[(b, int(c))], h)
+        h, tp = spos.block_fwd(cfg, b, int(c), theta[(b, int(c))], h, q)
         tapes.append(tp)
-    loss, dy = spos.head_loss(fz, h, np.asarray(labels, dtype=np.int64))
+    loss, dy = spos.head_loss(fz, h, np.asarray(labels, dtype=np.int64), q)
     grads = {}
     for b in reversed(range(len(choice))):
         c = int(choice[b])
-        dy, g = spos.block_bwd(cfg, b, c, theta[(b, c)], tapes[b], dy)
+        dy, g = spos.block_bwd(cfg, b, c, theta[(b, c)], tapes[b], dy, q)
         grads[(b, c)] = g
     return loss, grads
 

@@ -10,7 +10,7 @@ if not os.path.exists(LIB_PATH):
                       "`python -m paper_conf_asplos_zhaolcscwzlc22_b200.build` (no CPU fallback exists)")
 lib = C.CDLL(LIB_PATH)
 
-ABI_VERSION = 1
+ABI_VERSION = 2
 FAMILY = {"mlp": 0, "transformer": 1, "spos": 2}
 DTYPE = {"fp32": 0, "bf16": 1}
 BATCH_HOST, BATCH_DEVICE, BATCH_SYNTHETIC = 0, 1, 2
@@ -32,7 +32,10 @@ class _SpecStruct(C.Structure):
                 ("cost_bwd", _i32p), ("window", C.c_int32), ("lookahead", C.c_int32),
                 ("residency_horizon", C.c_int32),
                 ("hbm_weight_budget_bytes", C.c_int64), ("bwd_policy", C.c_int32),
-                ("link_latency", C.c_int32), ("flags", C.c_int32)]
+                ("link_latency", C.c_int32), ("flags", C.c_int32),
+                ("image_hw", C.c_int32), ("num_classes", C.c_int32), ("stem_channels", C.c_int32),
+                ("head_channels", C.c_int32), ("n_cnn_stages", C.c_int32), ("stage_repeats", _i32p),
+                ("stage_channels", _i32p), ("choice_kernel", _i32p), ("choice_xception", _i32p)]
 
 
 class _BatchStruct(C.Structure):
@@ -65,6 +68,7 @@ _sig("naspipe_param_count", C.c_int, [_SP, C.c_int32, C.c_int32, C.POINTER(C.c_s
 _sig("naspipe_default_costs", C.c_int, [_SP, _i32p, _i32p])
 _sig("naspipe_partition", C.c_int, [_SP, C.c_int32, _i32p])
 _sig("naspipe_init_params", C.c_int, [_SP, C.c_int32, C.c_int32, C.POINTER(C.c_float), C.c_size_t])
+_sig("naspipe_init_frozen", C.c_int, [_SP, C.c_int32, C.POINTER(C.c_float), C.c_size_t])
 _sig("naspipe_plan_create", C.c_int, [_SP, C.c_int32, _i32p, C.c_int64, C.POINTER(C.c_void_p)])
 _sig("naspipe_plan_trace", C.c_int, [C.c_void_p, _i64p, C.c_size_t, C.POINTER(C.c_size_t)])
 _sig("naspipe_plan_makespan", C.c_int, [C.c_void_p, _i64p])
@@ -80,7 +84,7 @@ EXPORTED_SYMBOLS = [
     "naspipe_create", "naspipe_create_rank", "naspipe_submit", "naspipe_drain", "naspipe_get_params",
     "naspipe_set_params", "naspipe_get_losses", "naspipe_get_trace", "naspipe_get_stats",
     "naspipe_get_residency_trace", "naspipe_destroy", "naspipe_param_count", "naspipe_default_costs",
-    "naspipe_partition", "naspipe_init_params", "naspipe_plan_create", "naspipe_plan_trace",
+    "naspipe_partition", "naspipe_init_params", "naspipe_init_frozen", "naspipe_plan_create", "naspipe_plan_trace",
     "naspipe_plan_makespan", "naspipe_plan_deps", "naspipe_plan_residency", "naspipe_plan_destroy",
     "naspipe_plan_comm_schedule", "naspipe_plan_idle",
     "naspipe_nccl_unique_id", "naspipe_last_error", "naspipe_abi_version"]
@@ -115,7 +119,8 @@ class Spec:
         s.width = cfg.get("width", 0)
         s.d_model, s.seq_len = cfg.get("d_model", 0), cfg.get("seq_len", 0)
         self._keep = []
-        for name in ("choice_heads", "choice_ffn", "stage_of_block", "cost_fwd", "cost_bwd"):
+        for name in ("choice_heads", "choice_ffn", "stage_of_block", "cost_fwd", "cost_bwd", "stage_repeats",
+                     "stage_channels", "choice_kernel", "choice_xception"):
             if cfg.get(name) is not None:
                 arr, ptr = _i32(np.asarray(cfg[name]).ravel())
                 self._keep.append(arr)
@@ -129,6 +134,9 @@ class Spec:
         s.bwd_policy = cfg.get("bwd_policy", 0)
         s.link_latency = cfg.get("link_latency", 0)
         s.flags = cfg.get("flags", 0)
+        s.image_hw, s.num_classes = cfg.get("image_hw", 0), cfg.get("num_classes", 0)
+        s.stem_channels, s.head_channels = cfg.get("stem_channels", 0), cfg.get("head_channels", 0)
+        s.n_cnn_stages = len(cfg.get("stage_repeats", []))
         self.struct = s
         self.cfg = cfg
 
@@ -180,7 +188,8 @@ def _ptr_of(x, keep):
     if hasattr(x, "data_ptr"):          # torch tensor (pinned host or device)
         keep.append(x)
         return x.data_ptr()
-    a = np.ascontiguousarray(x, dtype=np.float32)
+    x = np.asarray(x)
+    a = np.ascontiguousarray(x, dtype=np.int32 if np.issubdtype(x.dtype, np.integer) else np.float32)
     keep.append(a)
     return a.ctypes.data
 
@@ -274,6 +283,12 @@ def naspipe_init_params(spec: Spec, block: int, choice: int) -> np.ndarray:
     n = naspipe_param_count(spec, block, choice)
     out = np.empty(n, dtype=np.float32)
     _check(lib.naspipe_init_params(spec.ptr, block, choice, out.ctypes.data_as(C.POINTER(C.c_float)), n))
+    return out
+
+
+def naspipe_init_frozen(spec: Spec, part: int, n: int) -> np.ndarray:
+    out = np.empty(n, dtype=np.float32)
+    _check(lib.naspipe_init_frozen(spec.ptr, part, out.ctypes.data_as(C.POINTER(C.c_float)), n))
     return out
 
 

@@ -81,6 +81,17 @@ int naspipe_init_params(const naspipe_supernet_spec* spec, int32_t block, int32_
   });
 }
 
+int naspipe_init_frozen(const naspipe_supernet_spec* spec, int32_t part, float* dst, size_t n_floats) {
+  return guarded([&] {
+    Spec s(spec);
+    NP_REQUIRE(s.family() == NASPIPE_SPOS_CNN && part >= 0 && part <= 2, NASPIPE_EINVAL,
+               "frozen part %d (SPOS only: 0 stem, 1 head, 2 fc)", part);
+    NP_REQUIRE(dst && n_floats == s.frozen_count(part), NASPIPE_EINVAL, "n_floats %zu != %zu", n_floats,
+               s.frozen_count(part));
+    s.init_frozen(part, dst);
+  });
+}
+
 int naspipe_plan_create(const naspipe_supernet_spec* spec, int32_t n_stages, const int32_t* choices,
                         int64_t n_subnets, naspipe_plan_t** out) {
   return guarded([&] {

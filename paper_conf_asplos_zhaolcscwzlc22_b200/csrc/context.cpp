@@ -26,7 +26,7 @@ CandidateStore::CandidateStore(const Spec& spec, const Planner& planner, int K, 
       cd.j = (int)j;
       cd.c = c;
       cd.n32 = spec.param_count(blocks[j], c);
-      cd.n16 = fam->shadow_elems(c);
+      cd.n16 = fam->shadow_elems(j, c);
       uids.push_back(uid_of(blocks[j], c));
     }
   CU(cudaSetDevice(dev));

@@ -101,4 +101,67 @@ int naspipe_debug_ln_bwd(const float* dy, const float* x, const float* mean, con
   });
 }
 
+
+int naspipe_debug_dw(const void* x, const float* w, void* z, const void* dz, const void* add, void* dx,
+                     float* dwsum, int B, int H, int C, int k, int S, void* stream) {
+  return dguard([&] {
+    cudaStream_t s = (cudaStream_t)stream;
+    if (x && z) dw_fwd(s, (const bf16*)x, w, (bf16*)z, B, H, C, k, S);
+    if (dz && dx) dw_dgrad(s, (const bf16*)dz, w, (const bf16*)add, (bf16*)dx, B, H, C, k, S);
+    if (dz && x && dwsum) {
+      const int Ho = (H - 1) / S + 1, nblk = dw_wgrad_blocks(B * Ho * Ho);
+      float* part = nullptr;
+      NP_REQUIRE(cudaMalloc(&part, (size_t)nblk * C * k * k * 4) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
+      dw_wgrad(s, (const bf16*)dz, (const bf16*)x, part, B, H, C, k, S);
+      cudaMemsetAsync(dwsum, 0, (size_t)C * k * k * 4, s);
+      sgd_from_partials(s, dwsum, part, nblk, C * k * k, -1.0f);  // 0 - (-1) * sum = sum
+      cudaStreamSynchronize(s);
+      cudaFree(part);
+    }
+  });
+}
+
+int naspipe_debug_bn_fwd(const void* z, int P, int C, const float* g, const float* b, int relu, void* y, int ldy,
+                         float* mean, float* rstd, void* stream) {
+  return dguard([&] {
+    cudaStream_t s = (cudaStream_t)stream;
+    const int nblk = bn_part_blocks(P);
+    float* part = nullptr;
+    NP_REQUIRE(cudaMalloc(&part, (size_t)nblk * 2 * C * 4) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
+    bn_stats(s, (const bf16*)z, P, C, part);
+    bn_finalize(s, part, nblk, C, P, mean, rstd);
+    bn_apply(s, (const bf16*)z, P, C, mean, rstd, g, b, relu, (bf16*)y, ldy);
+    cudaStreamSynchronize(s);
+    cudaFree(part);
+  });
+}
+
+int naspipe_debug_bn_bwd(const void* dy, int lddy, const void* z, int P, int C, const float* mean,
+                         const float* rstd, float* g, float* b, int relu, void* dz, float* sums, float* old, float lr,
+                         int update, void* stream) {
+  return dguard([&] {
+    cudaStream_t s = (cudaStream_t)stream;
+    const int nblk = bn_part_blocks(P);
+    float* part = nullptr;
+    NP_REQUIRE(cudaMalloc(&part, (size_t)nblk * 2 * C * 4) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
+    bn_bwd_reduce(s, (const bf16*)dy, lddy, (const bf16*)z, P, C, mean, rstd, g, b, relu, part);
+    bn_bwd_finalize(s, part, nblk, C, sums, old, g, b, lr, update);
+    bn_bwd_apply(s, (const bf16*)dy, lddy, (const bf16*)z, P, C, mean, rstd, old, sums, relu, (bf16*)dz);
+    cudaStreamSynchronize(s);
+    cudaFree(part);
+  });
+}
+
+int naspipe_debug_chan_split(const void* x, int P, int Ch, void* out, int ldo, void* xm, void* stream) {
+  return dguard([&] { chan_split((cudaStream_t)stream, (const bf16*)x, P, Ch, (bf16*)out, ldo, (bf16*)xm); });
+}
+
+int naspipe_debug_chan_merge(const void* dproj, int ldp, const void* dm, int P, int Ch, void* dx, void* stream) {
+  return dguard([&] { chan_merge((cudaStream_t)stream, (const bf16*)dproj, ldp, (const bf16*)dm, P, Ch, (bf16*)dx); });
+}
+
+int naspipe_debug_stem(const float* x, const float* w, void* z, int B, int H, int C0, void* stream) {
+  return dguard([&] { spos_stem_conv((cudaStream_t)stream, x, w, (bf16*)z, B, H, C0); });
+}
+
 }  // extern "C"

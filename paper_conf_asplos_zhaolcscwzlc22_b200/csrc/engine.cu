@@ -97,6 +97,7 @@ std::unique_ptr<Engine> Engine::create_local(const Spec& spec, int D) {
   CU(cudaGetDevice(&cur));
   std::unique_ptr<Engine> e(new Engine(spec, D));
   e->st_.resize(D);
+  e->stage_sizes();
   for (int K = 0; K < D; ++K) e->setup_stage(K, (cur + K) % ndev, true);
   e->link_local_buffers();
   CU(cudaSetDevice(cur));
@@ -110,6 +111,7 @@ std::unique_ptr<Engine> Engine::create_rank(const Spec& spec, int D, int rank, i
   std::unique_ptr<Engine> e(new Engine(spec, D));
   e->rank_ = rank;
   e->st_.resize(D);
+  e->stage_sizes();
   for (int K = 0; K < D; ++K) {
     e->st_[K].K = K;
     e->st_[K].dev = device;
@@ -146,6 +148,16 @@ std::unique_ptr<Engine> Engine::create_rank(const Spec& spec, int D, int rank, i
   return e;
 }
 
+// Boundary tensor sizes of every stage (also of the non-local ones: a rank posts receives
+// sized by its neighbours' outputs).
+void Engine::stage_sizes() {
+  for (int K = 0; K < D_; ++K) {
+    const auto& bl = planner_.blocks_of(K);
+    st_[K].in_bytes = K == 0 ? spec_.input_bytes() : spec_.act_bytes(bl.front());
+    st_[K].out_bytes = spec_.act_bytes(bl.back() + 1);
+  }
+}
+
 void Engine::setup_stage(int K, int dev, bool local) {
   StageRt& st = st_[K];
   st.K = K;
@@ -159,22 +171,20 @@ void Engine::setup_stage(int K, int dev, bool local) {
   st.fam->timer = &timer_;
   st.store = std::make_unique<CandidateStore>(spec_, planner_, K, dev, st.fam.get(), st.arena.get(),
                                               spec_.raw.hbm_weight_budget_bytes);
-  const size_t n = spec_.batch_elems();
   st.in.assign(W_, nullptr);
   st.gout.assign(W_, nullptr);
   st.out.resize(W_);
   st.gin.assign(W_, nullptr);
   for (int s = 0; s < W_; ++s) {
-    st.out[s] = st.arena->alloc<float>(n);
-    if (K > 0) st.gin[s] = st.arena->alloc<float>(n);
-    if (K == 0) st.in[s] = st.arena->alloc<float>(n);
-    if (K == D_ - 1) st.gout[s] = st.arena->alloc<float>(n);
+    st.out[s] = st.arena->alloc<uint8_t>(st.out_bytes);
+    if (K > 0) st.gin[s] = st.arena->alloc<uint8_t>(st.in_bytes);
+    if (K == 0) st.in[s] = st.arena->alloc<uint8_t>(st.in_bytes);
+    if (K == D_ - 1) st.gout[s] = st.arena->alloc<uint8_t>(st.out_bytes);
   }
   if (K == D_ - 1) {
     st.target.resize(W_);
-    for (auto& p : st.target) p = st.arena->alloc<float>(n);
+    for (auto& p : st.target) p = st.arena->alloc<uint8_t>(spec_.target_bytes());
     st.loss = st.arena->alloc<float>(loss_cap_);
-    st.mse_part = st.arena->alloc<float>(mse_blocks(n));
     CU(cudaMemsetAsync(st.loss, 0, loss_cap_ * sizeof(float), st.comp));
   }
   for (auto* v : {&st.ev_f, &st.ev_b, &st.ev_in, &st.ev_tgt}) {
@@ -187,7 +197,6 @@ void Engine::setup_stage(int K, int dev, bool local) {
 // Same-device neighbours share boundary buffers (zero copy); otherwise each side owns a
 // receive buffer filled by a peer copy (single process) or NCCL (multi-process).
 void Engine::link_local_buffers() {
-  const size_t n = spec_.batch_elems();
   for (int K = 0; K < D_; ++K) {
     StageRt& st = st_[K];
     if (!st.local) continue;
@@ -195,11 +204,11 @@ void Engine::link_local_buffers() {
     for (int s = 0; s < W_; ++s) {
       if (K > 0) {
         const StageRt& p = st_[K - 1];
-        st.in[s] = (p.local && p.dev == st.dev) ? p.out[s] : st.arena->alloc<float>(n);
+        st.in[s] = (p.local && p.dev == st.dev) ? p.out[s] : st.arena->alloc<uint8_t>(st.in_bytes);
       }
       if (K < D_ - 1) {
         const StageRt& q = st_[K + 1];
-        st.gout[s] = (q.local && q.dev == st.dev) ? q.gin[s] : st.arena->alloc<float>(n);
+        st.gout[s] = (q.local && q.dev == st.dev) ? q.gin[s] : st.arena->alloc<uint8_t>(st.out_bytes);
       }
     }
   }
@@ -336,22 +345,21 @@ void Engine::issue(const Task& t) {
     // multi-process: post receives for the neighbours' tasks in their plan order (the sends
     // follow the same rules inside issue_forward / issue_backward; see comm_ops)
     StageRt& me = st_[rank_];
-    const size_t n = spec_.batch_elems();
     CommStep ops[2];
     const int nops = comm_ops(t, rank_, D_, ops);
     for (int k = 0; k < nops; ++k) {
       if (ops[k].op == RECV_ACT) {
         CU(cudaSetDevice(me.dev));
         CU(cudaStreamWaitEvent(tx_->s_act_in, me.ev_b[slot], 0));  // slot free (B(y-W) done)
-        NC(nccl().Recv(me.in[slot], n, ncclFloat32, 0, tx_->act_in, tx_->s_act_in));
+        NC(nccl().Recv(me.in[slot], me.in_bytes, ncclUint8, 0, tx_->act_in, tx_->s_act_in));
         CU(cudaEventRecord(tx_->ev_act_rx[slot], tx_->s_act_in));
-        p2p_bytes_ += 4.0 * n;
+        p2p_bytes_ += (double)me.in_bytes;
       } else if (ops[k].op == RECV_GRAD) {
         CU(cudaSetDevice(me.dev));
         CU(cudaStreamWaitEvent(tx_->s_grad_in, me.ev_b[slot], 0));
-        NC(nccl().Recv(me.gout[slot], n, ncclFloat32, 0, tx_->grad_in, tx_->s_grad_in));
+        NC(nccl().Recv(me.gout[slot], me.out_bytes, ncclUint8, 0, tx_->grad_in, tx_->s_grad_in));
         CU(cudaEventRecord(tx_->ev_grad_rx[slot], tx_->s_grad_in));
-        p2p_bytes_ += 4.0 * n;
+        p2p_bytes_ += (double)me.out_bytes;
       }
     }
   }
@@ -367,48 +375,49 @@ void Engine::issue(const Task& t) {
 
 void Engine::issue_forward(StageRt& st, int64_t y, int slot) {
   const int K = st.K;
-  const size_t n = spec_.batch_elems();
   const naspipe_batch& bt = batches_[y].b;
   const bool null_k = (spec_.raw.flags & NASPIPE_FLAG_NULL_KERNELS) != 0;
-  const float* xin = nullptr;
+  const void* xin = nullptr;
   if (K == 0) {
+    const size_t nb = spec_.input_bytes();
     if (bt.where == NASPIPE_BATCH_HOST) {
       CU(cudaStreamWaitEvent(st.copy, st.ev_b[slot], 0));
-      CU(cudaMemcpyAsync(st.in[slot], bt.input, n * 4, cudaMemcpyHostToDevice, st.copy));
+      CU(cudaMemcpyAsync(st.in[slot], bt.input, nb, cudaMemcpyHostToDevice, st.copy));
       CU(cudaEventRecord(st.ev_in[slot], st.copy));
       CU(cudaStreamWaitEvent(st.comp, st.ev_in[slot], 0));
-      h2d_bytes_ += 4.0 * n;
+      h2d_bytes_ += (double)nb;
       xin = st.in[slot];
     } else if (bt.where == NASPIPE_BATCH_DEVICE) {
-      xin = static_cast<const float*>(bt.input);
+      xin = bt.input;
     } else {
-      if (!null_k) { synth_fill(st.comp, st.in[slot], n, bt.synth_seed * 2 + 0); ++engine_launches_; }
+      if (!null_k) { synth_fill(st.comp, static_cast<float*>(st.in[slot]), nb / 4, bt.synth_seed * 2 + 0); ++engine_launches_; }
       xin = st.in[slot];
     }
   } else if (rank_ < 0) {
     StageRt& p = st_[K - 1];
     CU(cudaStreamWaitEvent(st.comp, p.ev_f[slot], 0));
     if (p.dev != st.dev) {
-      CU(cudaMemcpyPeerAsync(st.in[slot], st.dev, p.out[slot], p.dev, n * 4, st.comp));
-      p2p_bytes_ += 4.0 * n;
+      CU(cudaMemcpyPeerAsync(st.in[slot], st.dev, p.out[slot], p.dev, st.in_bytes, st.comp));
+      p2p_bytes_ += (double)st.in_bytes;
     }
     xin = st.in[slot];
   } else {
     CU(cudaStreamWaitEvent(st.comp, tx_->ev_act_rx[slot], 0));
     xin = st.in[slot];
   }
-  const float* tgt = nullptr;
+  const void* tgt = nullptr;
   if (K == D_ - 1) {
+    const size_t tb = spec_.target_bytes();
     if (bt.where == NASPIPE_BATCH_HOST) {
       CU(cudaStreamWaitEvent(st.copy, st.ev_f[slot], 0));  // previous user's loss done
-      CU(cudaMemcpyAsync(st.target[slot], bt.target, n * 4, cudaMemcpyHostToDevice, st.copy));
+      CU(cudaMemcpyAsync(st.target[slot], bt.target, tb, cudaMemcpyHostToDevice, st.copy));
       CU(cudaEventRecord(st.ev_tgt[slot], st.copy));
-      h2d_bytes_ += 4.0 * n;
+      h2d_bytes_ += (double)tb;
       tgt = st.target[slot];
     } else if (bt.where == NASPIPE_BATCH_DEVICE) {
-      tgt = static_cast<const float*>(bt.target);
+      tgt = bt.target;
     } else {
-      if (!null_k) { synth_fill(st.comp, st.target[slot], n, bt.synth_seed * 2 + 1); ++engine_launches_; }
+      if (!null_k) { st.fam->synth_target(st.target[slot], bt.synth_seed * 2 + 1, st.comp); ++engine_launches_; }
       tgt = st.target[slot];
     }
   }
@@ -418,12 +427,12 @@ void Engine::issue_forward(StageRt& st, int64_t y, int slot) {
   if (!null_k) st.fam->forward(slot, planner_.choice_row(y), xin, st.out[slot], st.comp);
   if (K == D_ - 1) {
     if (bt.where == NASPIPE_BATCH_HOST) CU(cudaStreamWaitEvent(st.comp, st.ev_tgt[slot], 0));
-    if (!null_k) { mse_loss(st.comp, st.out[slot], tgt, st.gout[slot], st.mse_part, st.loss + y, n); engine_launches_ += 2; }
+    if (!null_k) st.fam->loss(slot, st.out[slot], tgt, st.gout[slot], st.loss + y, st.comp);
   }
   CU(cudaEventRecord(st.ev_f[slot], st.comp));
   if (rank_ >= 0 && tx_ && K < D_ - 1) {
     CU(cudaStreamWaitEvent(tx_->s_act_out, st.ev_f[slot], 0));
-    NC(nccl().Send(st.out[slot], n, ncclFloat32, 1, tx_->act_out, tx_->s_act_out));
+    NC(nccl().Send(st.out[slot], st.out_bytes, ncclUint8, 1, tx_->act_out, tx_->s_act_out));
     CU(cudaEventRecord(tx_->ev_act_tx[slot], tx_->s_act_out));
   }
   cuda_check("forward");
@@ -431,27 +440,26 @@ void Engine::issue_forward(StageRt& st, int64_t y, int slot) {
 
 void Engine::issue_backward(StageRt& st, int64_t y, int slot) {
   const int K = st.K;
-  const size_t n = spec_.batch_elems();
   const bool null_k = (spec_.raw.flags & NASPIPE_FLAG_NULL_KERNELS) != 0;
   if (K < D_ - 1) {
     if (rank_ < 0) {
       StageRt& q = st_[K + 1];
       CU(cudaStreamWaitEvent(st.comp, q.ev_b[slot], 0));
       if (q.dev != st.dev) {
-        CU(cudaMemcpyPeerAsync(st.gout[slot], st.dev, q.gin[slot], q.dev, n * 4, st.comp));
-        p2p_bytes_ += 4.0 * n;
+        CU(cudaMemcpyPeerAsync(st.gout[slot], st.dev, q.gin[slot], q.dev, st.out_bytes, st.comp));
+        p2p_bytes_ += (double)st.out_bytes;
       }
     } else {
       CU(cudaStreamWaitEvent(st.comp, tx_->ev_grad_rx[slot], 0));
     }
   }
   if (rank_ >= 0 && tx_ && K > 0) CU(cudaStreamWaitEvent(st.comp, tx_->ev_grad_tx[slot], 0));
-  float* dx = K > 0 ? st.gin[slot] : nullptr;
+  void* dx = K > 0 ? st.gin[slot] : nullptr;
   if (!null_k) st.fam->backward(slot, planner_.choice_row(y), st.gout[slot], dx, st.comp);
   CU(cudaEventRecord(st.ev_b[slot], st.comp));
   if (rank_ >= 0 && tx_ && K > 0) {
     CU(cudaStreamWaitEvent(tx_->s_grad_out, st.ev_b[slot], 0));
-    NC(nccl().Send(st.gin[slot], n, ncclFloat32, 0, tx_->grad_out, tx_->s_grad_out));
+    NC(nccl().Send(st.gin[slot], st.in_bytes, ncclUint8, 0, tx_->grad_out, tx_->s_grad_out));
     CU(cudaEventRecord(tx_->ev_grad_tx[slot], tx_->s_grad_out));
   }
   cuda_check("backward");

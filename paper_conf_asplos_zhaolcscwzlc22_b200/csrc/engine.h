@@ -26,11 +26,11 @@ struct StageRt {
   std::unique_ptr<Family> fam;
   std::unique_ptr<CandidateStore> store;  // candidate parameters (resident or context-switched)
   size_t pushed = 0;                      // stage tasks fed to the store
-  // boundary buffers per slot (device, on dev)
-  std::vector<float*> in, out, gin, gout, target;
+  // boundary buffers per slot (device, on dev); opaque bytes (Spec::act_bytes)
+  size_t in_bytes = 0, out_bytes = 0;  // stage input (batch input at K = 0) / output
+  std::vector<void*> in, out, gin, gout, target;
   std::vector<cudaEvent_t> ev_f, ev_b, ev_in, ev_tgt;
   float* loss = nullptr;  // [loss_cap] on the last stage
-  float* mse_part = nullptr;
 };
 
 struct BatchRec {
@@ -58,6 +58,7 @@ class Engine {
 
  private:
   Engine(const Spec& spec, int D);
+  void stage_sizes();
   void setup_stage(int K, int dev, bool local);
   void link_local_buffers();
   void feed_stores();

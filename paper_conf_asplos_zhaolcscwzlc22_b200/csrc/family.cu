@@ -56,6 +56,17 @@ void KernelTimer::collect() {
   }
   used = 0;
 }
+void Family::loss(int, const void* out, const void* target, void* dy, float* loss_dst, cudaStream_t s) {
+  const size_t n = spec_base_->batch_elems();
+  mse_loss(s, static_cast<const float*>(out), static_cast<const float*>(target), static_cast<float*>(dy), mse_part_,
+           loss_dst, n);
+  counters.launches += 2;
+}
+
+void Family::synth_target(void* dst, uint64_t seed, cudaStream_t s) {
+  synth_fill(s, static_cast<float*>(dst), spec_base_->batch_elems(), seed);
+}
+
 KernelTimer::~KernelTimer() {
   for (auto& p : pairs) {
     cudaEventDestroy(p.first);
@@ -81,30 +92,32 @@ class MlpFamily : public Family {
     for (auto& p : act_) p = A.alloc<float>(act);
     g_[0] = A.alloc<float>(act);
     g_[1] = A.alloc<float>(act);
+    spec_base_ = &spec;
+    mse_part_ = A.alloc<float>(mse_blocks(spec.batch_elems()));
   }
   void bind(int j, int c, float* w32, bf16*) override { params_[(size_t)j * spec_.n() + c] = w32; }
-  size_t shadow_elems(int) const override { return 0; }
+  size_t shadow_elems(int, int) const override { return 0; }
   float* master(int j, int c) override { return params_[(size_t)j * spec_.n() + c]; }
   void refresh_shadow(int, int, cudaStream_t) override {}
 
-  void forward(int slot, const int32_t* ch, const float* x_in, float* x_out, cudaStream_t s) override {
+  void forward(int slot, const int32_t* ch, const void* x_in, void* x_out, cudaStream_t s) override {
     const int nb = (int)blocks_.size();
-    const float* x = x_in;
+    const float* x = static_cast<const float*>(x_in);
     for (int j = 0; j < nb; ++j) {
       float* P = master(j, ch[blocks_[j]]);
-      float* y = (j == nb - 1) ? x_out : act_[(size_t)slot * nb + j + 1];
+      float* y = (j == nb - 1) ? static_cast<float*>(x_out) : act_[(size_t)slot * nb + j + 1];
       xin_[(size_t)slot * nb + j] = x;
       mlp_fwd(s, x, P, P + (size_t)d_ * d_, y, h_[(size_t)slot * nb + j], B_, d_);
       counters.launches++;
       x = y;
     }
   }
-  void backward(int slot, const int32_t* ch, const float* dy, float* dx, cudaStream_t s) override {
+  void backward(int slot, const int32_t* ch, const void* dy, void* dx, cudaStream_t s) override {
     const int nb = (int)blocks_.size();
-    const float* g = dy;
+    const float* g = static_cast<const float*>(dy);
     for (int j = nb - 1; j >= 0; --j) {
       float* P = master(j, ch[blocks_[j]]);
-      float* out = (j == 0) ? dx : g_[j & 1];
+      float* out = (j == 0) ? static_cast<float*>(dx) : g_[j & 1];
       mlp_bwd_sgd(s, xin_[(size_t)slot * nb + j], h_[(size_t)slot * nb + j], g, out, P, P + (size_t)d_ * d_, lr_,
                   B_, d_);
       counters.launches++;
@@ -194,6 +207,8 @@ class TfFamily : public Family {
     }
     p_g1_ = A.alloc<float>((size_t)lnb_ * d_);
     p_b1_ = A.alloc<float>((size_t)lnb_ * d_);
+    spec_base_ = &spec;
+    mse_part_ = A.alloc<float>(mse_blocks(spec.batch_elems()));
     cudaStreamCreateWithFlags(&side_, cudaStreamNonBlocking);
     for (auto* e : {&ev_dz_, &ev_da2_, &ev_do_, &ev_da_, &ev_done_[0], &ev_done_[1], &ev_join_})
       cudaEventCreateWithFlags(e, cudaEventDisableTiming);
@@ -209,7 +224,7 @@ class TfFamily : public Family {
     w32_[(size_t)j * spec_.n() + c] = w32;
     w16_[(size_t)j * spec_.n() + c] = w16;
   }
-  size_t shadow_elems(int c) const override { return 4 * (size_t)d_ * d_ + 2 * (size_t)d_ * spec_.ffn[c]; }
+  size_t shadow_elems(int, int c) const override { return 4 * (size_t)d_ * d_ + 2 * (size_t)d_ * spec_.ffn[c]; }
   float* master(int j, int c) override { return w32_[(size_t)j * spec_.n() + c]; }
 
   void refresh_shadow(int j, int c, cudaStream_t s) override {
@@ -223,14 +238,14 @@ class TfFamily : public Family {
     f32_to_bf16(s, p + o.W2, w + 4 * d * d + f * d, d * f);
   }
 
-  void forward(int slot, const int32_t* ch, const float* x_in, float* x_out, cudaStream_t s) override {
+  void forward(int slot, const int32_t* ch, const void* x_in, void* x_out, cudaStream_t s) override {
     const int nb = (int)blocks_.size();
-    const float* x = x_in;
+    const float* x = static_cast<const float*>(x_in);
     for (int j = 0; j < nb; ++j) {
       const int c = ch[blocks_[j]];
       TfSlot& t = slots_[(size_t)slot * nb + j];
       t.xin = x;
-      float* y = (j == nb - 1) ? x_out : slots_[(size_t)slot * nb + j + 1].act;
+      float* y = (j == nb - 1) ? static_cast<float*>(x_out) : slots_[(size_t)slot * nb + j + 1].act;
       block_fwd(j, c, t, y, s);
       x = y;
     }
@@ -242,8 +257,10 @@ class TfFamily : public Family {
   // that read the pre-update weight is done (reading A4), filling the SMs the dgrad chain
   // leaves idle.  Buffers the side stream reads are double-buffered by block parity; the
   // stage stream joins the side stream before the task ends.
-  void backward(int slot, const int32_t* ch, const float* dy, float* dx, cudaStream_t s) override {
+  void backward(int slot, const int32_t* ch, const void* dy_v, void* dx_v, cudaStream_t s) override {
     const int nb = (int)blocks_.size();
+    const float* dy = static_cast<const float*>(dy_v);
+    float* dx = static_cast<float*>(dx_v);
     const float* g = dy;
     int db2_nblk = 0;
     for (int j = nb - 1; j >= 0; --j) {
@@ -405,6 +422,7 @@ class TfFamily : public Family {
 std::unique_ptr<Family> make_family(const Spec& spec, const std::vector<int>& blocks, int W, DevArena& arena,
                                     cudaStream_t s) {
   if (spec.family() == NASPIPE_MLP) return std::make_unique<MlpFamily>(spec, blocks, W, arena, s);
+  if (spec.family() == NASPIPE_SPOS_CNN) return make_spos_family(spec, blocks, W, arena);
   return std::make_unique<TfFamily>(spec, blocks, W, arena, s);
 }
 

@@ -47,25 +47,38 @@ struct FamilyCounters {
 class Family {
  public:
   virtual ~Family() = default;
-  // blocks: the stage's blocks (global ids), W slots
-  virtual void forward(int slot, const int32_t* choice_of_block, const float* x_in, float* x_out,
+  // blocks: the stage's blocks (global ids), W slots.  Boundary tensors are opaque here:
+  // fp32 [B, sample] for MLP/TRANSFORMER, bf16 NHWC for SPOS (the stage-0 input is the
+  // batch input itself, see Spec::act_bytes / input_bytes).
+  virtual void forward(int slot, const int32_t* choice_of_block, const void* x_in, void* x_out,
                        cudaStream_t s) = 0;
   // dy: grad w.r.t. the stage output; dx: grad w.r.t. the stage input (nullptr: not needed)
-  virtual void backward(int slot, const int32_t* choice_of_block, const float* dy, float* dx,
+  virtual void backward(int slot, const int32_t* choice_of_block, const void* dy, void* dx,
                         cudaStream_t s) = 0;
+  // Last stage only: loss of the stage output against the target -> *loss_dst (device) and
+  // the seed gradient dy (same layout as the output).  MSE (reading A18) unless overridden.
+  virtual void loss(int slot, const void* out, const void* target, void* dy, float* loss_dst,
+                    cudaStream_t s);
+  // synthetic target (perf runs): N(0,1)-like fp32 by default, labels for SPOS
+  virtual void synth_target(void* dst, uint64_t seed, cudaStream_t s);
   // Candidate (local block j, choice c) parameters live in buffers the engine owns (resident
   // for the whole run, or loaded/evicted by the context switch); bind() points the family at
   // them (nullptr = not resident).  master() is the packed fp32 vector, the bf16 shadow holds
-  // the GEMM operands (shadow_elems(c) elements; 0 for fp32 families).
+  // the GEMM operands (shadow_elems(j, c) elements; 0 for fp32 families).
   virtual void bind(int local_block, int c, float* w32, bf16* w16) = 0;
-  virtual size_t shadow_elems(int c) const = 0;
+  virtual size_t shadow_elems(int local_block, int c) const = 0;
   virtual float* master(int local_block, int c) = 0;
   virtual void refresh_shadow(int local_block, int c, cudaStream_t s) = 0;  // bf16 <- fp32
   FamilyCounters counters;
   KernelTimer* timer = nullptr;
+
+ protected:
+  const Spec* spec_base_ = nullptr;
+  float* mse_part_ = nullptr;  // MSE workspace (last stage)
 };
 
 std::unique_ptr<Family> make_family(const Spec& spec, const std::vector<int>& blocks, int W, DevArena& arena,
                                     cudaStream_t s);
+std::unique_ptr<Family> make_spos_family(const Spec& spec, const std::vector<int>& blocks, int W, DevArena& arena);
 
 }  // namespace naspipe

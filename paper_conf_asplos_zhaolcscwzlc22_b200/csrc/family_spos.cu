@@ -1,0 +1,413 @@
+// SPOS CNN family (configs[1]): ShuffleNetV2-style choice blocks {Shuffle 3/5/7, Xception}
+// (SURVEY §8c "C2 SPOS candidate"; oracle/spos.py), frozen stem on the first stage and frozen
+// head + cross-entropy on the last stage (reading A2).
+//
+// Layout: NHWC bf16 activations; a block's output is stored in logical channel order
+// concat(proj, main) (P:L579 SPOS blocks); the stride-1 channel split (even channels pass
+// through, odd channels feed the main branch) is one kernel that writes the pass-through half
+// straight into the block output and the main-branch input contiguously.  Every conv -> BN
+// [-> ReLU] unit keeps z (bf16) and its batch mean / rstd in the slot's stash for the
+// backward; 1x1 convs run on the tcgen05 GEMM (forward: z = x W^T; dgrad: dx = dz W; wgrad
+// with the fused SGD WRITE: W -= lr dz^T x, deterministic split-K over the pixels), depthwise
+// convs and BatchNorm on CUDA cores (spos.cu).
+#include <algorithm>
+#include <cstring>
+
+#include "family.h"
+
+namespace naspipe {
+
+namespace {
+
+struct UnitRec {  // forward stash of one unit of (slot, block)
+  const bf16* x;  // unit input
+  bf16* z;        // conv output
+  float *mean, *rstd;
+};
+
+class SposFamily : public Family {
+ public:
+  SposFamily(const Spec& spec, const std::vector<int>& blocks, int W, DevArena& A)
+      : spec_(spec), blocks_(blocks), W_(W), B_(spec.B()), lr_(spec.raw.lr) {
+    const int nb = (int)blocks.size(), n = spec.n();
+    first_ = blocks.front() == 0;
+    last_ = blocks.back() == spec.m() - 1;
+    w32_.assign((size_t)nb * n, nullptr);
+    w16_.assign((size_t)nb * n, nullptr);
+    plans_.resize((size_t)nb * n);
+    dims_.resize(nb);
+    size_t stash_max = 0, stats_max = 0, dz_max = 0, g_max = 0, blk_max = 0, part_max = 0, dwp_max = 0, C_max = 0;
+    ws_elems_ = 0;
+    for (int j = 0; j < nb; ++j) {
+      const int b = blocks[j];
+      const SposDims d = spec.spos_dims(b);
+      dims_[j] = d;
+      blk_max = std::max({blk_max, spec.act_bytes(b) / 2, spec.act_bytes(b + 1) / 2});
+      for (int c = 0; c < n; ++c) {
+        auto& L = plans_[(size_t)j * n + c];
+        L = spec.spos_convs(b, c);
+        size_t need = d.stride == 1 ? P(d.H_in) * (d.C_out / 2) : 0, st = 0;
+        for (size_t i = 0; i < L.size(); ++i) {
+          const SposConv& u = L[i];
+          const size_t po = P(u.H_out), pi = P(u.H_in);
+          need += po * u.cout * (last_of_branch(L, i) ? 1 : 2);
+          st += 2 * (size_t)u.cout;
+          dz_max = std::max(dz_max, po * u.cout);
+          g_max = std::max({g_max, pi * u.cin, po * u.cout});
+          part_max = std::max(part_max, (size_t)bn_part_blocks((int)po) * 2 * u.cout);
+          C_max = std::max(C_max, (size_t)u.cout);
+          if (u.dw)
+            dwp_max = std::max(dwp_max, (size_t)dw_wgrad_blocks((int)po) * u.cout * u.k * u.k);
+          else
+            ws_elems_ = std::max(ws_elems_, (size_t)gemm_splitk_factor(u.cout, u.cin, (int)po) * u.cout * u.cin);
+        }
+        stash_max = std::max(stash_max, need);
+        stats_max = std::max(stats_max, st);
+      }
+    }
+    const int hw0 = spec.spos_stem_hw(), hwl = spec.spos_last_hw(), C0 = spec.raw.stem_channels,
+              Cl = spec.chans.back(), Ch = spec.raw.head_channels, ncls = spec.raw.num_classes;
+    if (last_) {
+      const size_t PL = P(hwl);
+      part_max = std::max(part_max, (size_t)bn_part_blocks((int)PL) * 2 * Ch);
+      C_max = std::max(C_max, (size_t)Ch);
+    }
+    if (first_) {
+      part_max = std::max(part_max, (size_t)bn_part_blocks((int)P(hw0)) * 2 * C0);
+      C_max = std::max(C_max, (size_t)C0);
+    }
+    stash_.resize((size_t)W * nb);
+    stats_.resize((size_t)W * nb);
+    act_.assign((size_t)W * nb, nullptr);
+    recs_.resize((size_t)W * nb);
+    xin_.assign((size_t)W * nb, nullptr);
+    for (int sl = 0; sl < W; ++sl)
+      for (int j = 0; j < nb; ++j) {
+        const size_t k = (size_t)sl * nb + j;
+        stash_[k] = A.alloc<bf16>(stash_max);
+        stats_[k] = A.alloc<float>(stats_max);
+        if (j < nb - 1) act_[k] = A.alloc<bf16>(spec.act_bytes(blocks[j] + 1) / 2);
+      }
+    dz_ = A.alloc<bf16>(dz_max);
+    g_[0] = A.alloc<bf16>(g_max);
+    g_[1] = A.alloc<bf16>(g_max);
+    gb_[0] = A.alloc<bf16>(blk_max);
+    gb_[1] = A.alloc<bf16>(blk_max);
+    gfirst_ = A.alloc<bf16>(g_max);
+    part_ = A.alloc<float>(part_max);
+    dwpart_ = A.alloc<float>(std::max<size_t>(dwp_max, 1));
+    ws_ = A.alloc<float>(std::max<size_t>(ws_elems_, 4));
+    sums_ = A.alloc<float>(2 * C_max);
+    old_ = A.alloc<float>(2 * C_max);
+    if (first_) {
+      std::vector<float> h(spec.frozen_count(0));
+      spec.init_frozen(0, h.data());
+      w_stem_ = A.alloc<float>(h.size());
+      cudaMemcpy(w_stem_, h.data(), h.size() * 4, cudaMemcpyHostToDevice);
+      stem_z_ = A.alloc<bf16>(P(hw0) * C0);
+      stem_mean_ = A.alloc<float>(C0);
+      stem_rstd_ = A.alloc<float>(C0);
+      stem_y_.resize(W);
+      for (auto& p : stem_y_) p = A.alloc<bf16>(P(hw0) * C0);
+      std::vector<float> ones(C0, 1.0f), zeros(C0, 0.0f);
+      ones_s_ = A.alloc<float>(C0);
+      zeros_s_ = A.alloc<float>(C0);
+      cudaMemcpy(ones_s_, ones.data(), C0 * 4, cudaMemcpyHostToDevice);
+      cudaMemcpy(zeros_s_, zeros.data(), C0 * 4, cudaMemcpyHostToDevice);
+    }
+    if (last_) {
+      std::vector<float> h(spec.frozen_count(1));
+      spec.init_frozen(1, h.data());
+      std::vector<bf16> h16(h.size());
+      for (size_t i = 0; i < h.size(); ++i) h16[i] = __float2bfloat16_rn(h[i]);
+      wh16_ = A.alloc<bf16>(h.size());
+      cudaMemcpy(wh16_, h16.data(), h16.size() * 2, cudaMemcpyHostToDevice);
+      std::vector<float> f(spec.frozen_count(2));
+      spec.init_frozen(2, f.data());
+      wf_ = A.alloc<float>(f.size());
+      cudaMemcpy(wf_, f.data(), f.size() * 4, cudaMemcpyHostToDevice);
+      std::vector<float> ones(Ch, 1.0f), zeros(Ch, 0.0f);
+      ones_ = A.alloc<float>(Ch);
+      zeros_ = A.alloc<float>(Ch);
+      cudaMemcpy(ones_, ones.data(), Ch * 4, cudaMemcpyHostToDevice);
+      cudaMemcpy(zeros_, zeros.data(), Ch * 4, cudaMemcpyHostToDevice);
+      const size_t PL = P(hwl);
+      zh_ = A.alloc<bf16>(PL * Ch);
+      rh_ = A.alloc<bf16>(PL * Ch);
+      dzh_ = A.alloc<bf16>(PL * Ch);
+      hmean_ = A.alloc<float>(Ch);
+      hrstd_ = A.alloc<float>(Ch);
+      gap_ = A.alloc<float>((size_t)B_ * Ch);
+      dgap_ = A.alloc<float>((size_t)B_ * Ch);
+      dlogits_ = A.alloc<float>((size_t)B_ * ncls);
+      loss_per_ = A.alloc<float>(B_);
+    }
+    (void)Cl;
+  }
+
+  void bind(int j, int c, float* w32, bf16* w16) override {
+    w32_[(size_t)j * spec_.n() + c] = w32;
+    w16_[(size_t)j * spec_.n() + c] = w16;
+  }
+  size_t shadow_elems(int j, int c) const override { return spec_.spos_shadow_elems(blocks_[j], c); }
+  float* master(int j, int c) override { return w32_[(size_t)j * spec_.n() + c]; }
+  void refresh_shadow(int j, int c, cudaStream_t s) override {
+    float* p = master(j, c);
+    bf16* w = w16_[(size_t)j * spec_.n() + c];
+    for (const SposConv& u : plans_[(size_t)j * spec_.n() + c])
+      if (!u.dw) f32_to_bf16(s, p + u.off_w, w + u.off_w16, (size_t)u.cout * u.cin);
+  }
+
+  void forward(int slot, const int32_t* ch, const void* x_in, void* x_out, cudaStream_t s) override {
+    const int nb = (int)blocks_.size();
+    const bf16* x = static_cast<const bf16*>(x_in);
+    if (first_) {  // frozen stem: conv3x3 s2 -> BN(1, 0) batch statistics -> ReLU
+      const int H = spec_.raw.image_hw, C0 = spec_.raw.stem_channels;
+      const int Po = (int)P(H / 2);
+      spos_stem_conv(s, static_cast<const float*>(x_in), w_stem_, stem_z_, B_, H, C0);
+      bn_stats(s, stem_z_, Po, C0, part_);
+      bn_finalize(s, part_, bn_part_blocks(Po), C0, Po, stem_mean_, stem_rstd_);
+      bn_apply(s, stem_z_, Po, C0, stem_mean_, stem_rstd_, ones_s_, zeros_s_, 1, stem_y_[slot], C0);
+      counters.launches += 4;
+      x = stem_y_[slot];
+    }
+    for (int j = 0; j < nb; ++j) {
+      const int c = ch[blocks_[j]];
+      const size_t k = (size_t)slot * nb + j;
+      bf16* out = (j == nb - 1) ? static_cast<bf16*>(x_out) : act_[k];
+      xin_[k] = x;
+      block_fwd(j, c, k, x, out, s);
+      x = out;
+    }
+  }
+
+  void backward(int slot, const int32_t* ch, const void* dy, void* dx, cudaStream_t s) override {
+    const int nb = (int)blocks_.size();
+    const bf16* g = static_cast<const bf16*>(dy);
+    for (int j = nb - 1; j >= 0; --j) {
+      const int c = ch[blocks_[j]];
+      const size_t k = (size_t)slot * nb + j;
+      const bool need_dx = j > 0 || dx != nullptr;
+      bf16* out = (j == 0) ? static_cast<bf16*>(dx) : gb_[j & 1];
+      block_bwd(j, c, k, g, out, need_dx, s);
+      g = out;
+    }
+  }
+
+  // Frozen head: pw Clast->Ch (tcgen05) -> BN(1,0) -> ReLU -> GAP -> FC (fp32) -> mean CE,
+  // then its backward down to dL/d(stage output) (no parameter is updated, reading A2).
+  void loss(int, const void* out, const void* target, void* dy, float* loss_dst, cudaStream_t s) override {
+    const int hw = spec_.spos_last_hw(), HW = hw * hw, Cl = spec_.chans.back(), Ch = spec_.raw.head_channels,
+              ncls = spec_.raw.num_classes;
+    const int PL = (int)P(hw), nblk = bn_part_blocks(PL);
+    GemmEpiParams e;
+    e.out = zh_;
+    gemm(s, PL, Ch, Cl, static_cast<const bf16*>(out), false, Cl, wh16_, false, Cl, EPI_BF16, e);
+    bn_stats(s, zh_, PL, Ch, part_);
+    bn_finalize(s, part_, nblk, Ch, PL, hmean_, hrstd_);
+    bn_apply(s, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, 1, rh_, Ch);
+    gap_pool(s, rh_, B_, HW, Ch, gap_);
+    fc_ce(s, gap_, wf_, static_cast<const int*>(target), B_, Ch, ncls, dlogits_, loss_per_);
+    ce_mean(s, loss_per_, B_, loss_dst);
+    fc_dgap(s, dlogits_, wf_, B_, Ch, ncls, dgap_);
+    head_bcast(s, dgap_, B_, HW, Ch, rh_);  // dr overwrites r (the mask is recomputed from z)
+    bn_bwd_reduce(s, rh_, Ch, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, 1, part_);
+    bn_bwd_finalize(s, part_, nblk, Ch, sums_, old_, ones_, zeros_, 0.f, 0);
+    bn_bwd_apply(s, rh_, Ch, zh_, PL, Ch, hmean_, hrstd_, old_, sums_, 1, dzh_);
+    e = GemmEpiParams();
+    e.out = dy;
+    gemm(s, PL, Cl, Ch, dzh_, false, Ch, wh16_, true, Cl, EPI_BF16, e);
+    counters.launches += 12;
+  }
+
+  void synth_target(void* dst, uint64_t seed, cudaStream_t s) override {
+    synth_labels(s, static_cast<int*>(dst), B_, spec_.raw.num_classes, seed);
+  }
+
+ private:
+  size_t P(int hw) const { return (size_t)B_ * hw * hw; }
+  static bool last_of_branch(const std::vector<SposConv>& L, size_t i) {
+    return i + 1 == L.size() || L[i + 1].branch != L[i].branch;
+  }
+  void gemm(cudaStream_t s, int M, int N, int K, const bf16* A, bool amn, int lda, const bf16* B, bool bmn, int ldb,
+            int epi, const GemmEpiParams& ep, bool split_ok = false) {
+    if (timer) timer->begin(s);
+    GemmEpiParams e = ep;
+    if (split_ok) {
+      e.ws = ws_;
+      e.ws_elems = ws_elems_;
+    }
+    gemm_bf16_tc(s, M, N, K, A, amn, lda, B, bmn, ldb, epi, e);
+    if (timer) timer->end(s, 2.0 * M * N * K);
+    counters.launches += (epi == EPI_SGD && gemm_splitk_factor(M, N, K) > 1) ? 2 : 1;
+  }
+
+  void block_fwd(int j, int c, size_t k, const bf16* x, bf16* out, cudaStream_t s) {
+    const SposDims& d = dims_[j];
+    const auto& L = plans_[(size_t)j * spec_.n() + c];
+    float* Pm = master(j, c);
+    const bf16* W16 = w16_[(size_t)j * spec_.n() + c];
+    bf16* cv = stash_[k];
+    float* st = stats_[k];
+    auto& recs = recs_[k];
+    recs.clear();
+    const bf16* main_in = x;
+    int main_col = d.inp;  // column of the main branch in the block output
+    if (d.stride == 1) {
+      bf16* xm = cv;
+      cv += P(d.H_in) * (d.C_out / 2);
+      chan_split(s, x, (int)P(d.H_in), d.C_out / 2, out, d.C_out, xm);
+      counters.launches++;
+      main_in = xm;
+      main_col = d.C_out / 2;
+    }
+    const bf16* h = nullptr;
+    for (size_t i = 0; i < L.size(); ++i) {
+      const SposConv& u = L[i];
+      if (i == 0 || L[i - 1].branch != u.branch) h = (u.branch == 0) ? x : main_in;
+      const int Po = (int)P(u.H_out);
+      UnitRec r{h, cv, st, st + u.cout};
+      cv += (size_t)Po * u.cout;
+      st += 2 * u.cout;
+      if (u.dw) {
+        dw_fwd(s, h, Pm + u.off_w, r.z, B_, u.H_in, u.cin, u.k, u.stride);
+        counters.launches++;
+      } else {
+        GemmEpiParams e;
+        e.out = r.z;
+        gemm(s, Po, u.cout, u.cin, h, false, u.cin, W16 + u.off_w16, false, u.cin, EPI_BF16, e);
+      }
+      bn_stats(s, r.z, Po, u.cout, part_);
+      bn_finalize(s, part_, bn_part_blocks(Po), u.cout, Po, r.mean, r.rstd);
+      bf16* y;
+      int ldy;
+      if (last_of_branch(L, i)) {
+        y = out + (u.branch == 0 ? 0 : main_col);
+        ldy = d.C_out;
+      } else {
+        y = cv;
+        cv += (size_t)Po * u.cout;
+        ldy = u.cout;
+      }
+      bn_apply(s, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, u.relu, y, ldy);
+      counters.launches += 3;
+      recs.push_back(r);
+      h = y;
+    }
+  }
+
+  // One unit's BN backward (+ the WRITE of its gamma/beta), leaves dz in dz_.
+  void unit_bn_bwd(const SposConv& u, const UnitRec& r, float* Pm, const bf16* dy, int lddy, cudaStream_t s) {
+    const int Po = (int)P(u.H_out);
+    bn_bwd_reduce(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, u.relu, part_);
+    bn_bwd_finalize(s, part_, bn_part_blocks(Po), u.cout, sums_, old_, Pm + u.off_g, Pm + u.off_b, lr_, 1);
+    bn_bwd_apply(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, old_, sums_, u.relu, dz_);
+    counters.launches += 3;
+  }
+
+  // conv backward of one unit from dz_: dgrad into dst (+ add) with the pre-update weights
+  // (skipped if dst == nullptr), then the weight gradient with the SGD WRITE.
+  void unit_conv_bwd(const SposConv& u, const UnitRec& r, float* Pm, bf16* W16, bf16* dst, const bf16* add,
+                     cudaStream_t s) {
+    const int Po = (int)P(u.H_out);
+    if (u.dw) {
+      if (dst) {
+        dw_dgrad(s, dz_, Pm + u.off_w, add, dst, B_, u.H_in, u.cin, u.k, u.stride);
+        counters.launches++;
+      }
+      dw_wgrad(s, dz_, r.x, dwpart_, B_, u.H_in, u.cin, u.k, u.stride);
+      sgd_from_partials(s, Pm + u.off_w, dwpart_, dw_wgrad_blocks(Po), u.cout * u.k * u.k, lr_);
+      counters.launches += 2;
+    } else {
+      NP_REQUIRE(add == nullptr, NASPIPE_EINTERNAL, "pw dgrad with an addend");
+      if (dst) {
+        GemmEpiParams e;
+        e.out = dst;
+        gemm(s, Po, u.cin, u.cout, dz_, false, u.cout, W16 + u.off_w16, true, u.cin, EPI_BF16, e);
+      }
+      GemmEpiParams e;
+      e.w32 = Pm + u.off_w;
+      e.w16 = W16 + u.off_w16;
+      e.lr = lr_;
+      gemm(s, u.cout, u.cin, Po, dz_, true, u.cout, r.x, true, u.cin, EPI_SGD, e, true);
+    }
+  }
+
+  void block_bwd(int j, int c, size_t k, const bf16* dyb, bf16* dxb, bool need_dx, cudaStream_t s) {
+    const SposDims& d = dims_[j];
+    const auto& L = plans_[(size_t)j * spec_.n() + c];
+    float* Pm = master(j, c);
+    bf16* W16 = w16_[(size_t)j * spec_.n() + c];
+    const auto& recs = recs_[k];
+    const int main_col = d.stride == 1 ? d.C_out / 2 : d.inp;
+    size_t m0 = 0;  // first main-branch unit
+    while (m0 < L.size() && L[m0].branch == 0) ++m0;
+    // ---- main branch, last unit first
+    const bf16* h = dyb + main_col;
+    int ldh = d.C_out;
+    int pp = 0;
+    for (size_t i = L.size(); i-- > m0;) {
+      const SposConv& u = L[i];
+      unit_bn_bwd(u, recs[i], Pm, h, ldh, s);
+      bf16* dst;
+      if (i > m0) dst = g_[pp ^= 1];
+      else dst = need_dx ? (d.stride == 1 ? g_[pp ^ 1] : gfirst_) : nullptr;
+      unit_conv_bwd(u, recs[i], Pm, W16, dst, nullptr, s);
+      h = dst;
+      ldh = u.cin;
+    }
+    if (d.stride == 1) {
+      if (need_dx) {
+        chan_merge(s, dyb, d.C_out, h, (int)P(d.H_in), d.C_out / 2, dxb);
+        counters.launches++;
+      }
+      return;
+    }
+    // ---- stride 2: proj branch (dw s2 -> BN -> pw -> BN -> ReLU); its input gradient adds
+    // the main branch's (both branches read the block input)
+    const bf16* hp = dyb;
+    int ldp = d.C_out;
+    for (size_t i = m0; i-- > 0;) {
+      const SposConv& u = L[i];
+      unit_bn_bwd(u, recs[i], Pm, hp, ldp, s);
+      bf16* dst = i > 0 ? g_[pp ^= 1] : (need_dx ? dxb : nullptr);
+      unit_conv_bwd(u, recs[i], Pm, W16, dst, (i == 0 && need_dx) ? gfirst_ : nullptr, s);
+      hp = dst;
+      ldp = u.cin;
+    }
+  }
+
+  const Spec& spec_;
+  std::vector<int> blocks_;
+  int W_, B_;
+  float lr_;
+  bool first_ = false, last_ = false;
+  std::vector<float*> w32_;
+  std::vector<bf16*> w16_;
+  std::vector<std::vector<SposConv>> plans_;
+  std::vector<SposDims> dims_;
+  std::vector<bf16*> stash_, act_;
+  std::vector<float*> stats_;
+  std::vector<std::vector<UnitRec>> recs_;
+  std::vector<const bf16*> xin_;
+  bf16 *dz_, *g_[2], *gb_[2], *gfirst_;
+  float *part_, *dwpart_, *ws_, *sums_, *old_;
+  size_t ws_elems_ = 0;
+  // stem
+  float* w_stem_ = nullptr;
+  bf16* stem_z_ = nullptr;
+  float *stem_mean_ = nullptr, *stem_rstd_ = nullptr, *ones_s_ = nullptr, *zeros_s_ = nullptr;
+  std::vector<bf16*> stem_y_;
+  // head
+  bf16 *wh16_ = nullptr, *zh_ = nullptr, *rh_ = nullptr, *dzh_ = nullptr;
+  float *wf_ = nullptr, *ones_ = nullptr, *zeros_ = nullptr, *hmean_ = nullptr, *hrstd_ = nullptr, *gap_ = nullptr,
+        *dgap_ = nullptr, *dlogits_ = nullptr, *loss_per_ = nullptr;
+};
+
+}  // namespace
+
+std::unique_ptr<Family> make_spos_family(const Spec& spec, const std::vector<int>& blocks, int W, DevArena& arena) {
+  return std::make_unique<SposFamily>(spec, blocks, W, arena);
+}
+
+}  // namespace naspipe

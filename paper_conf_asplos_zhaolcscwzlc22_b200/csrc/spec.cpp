@@ -30,8 +30,8 @@ Spec::Spec(const naspipe_supernet_spec* s) {
   NP_REQUIRE(s->abi_version == NASPIPE_ABI_VERSION, NASPIPE_EINVAL, "abi_version %d != %d",
              s->abi_version, NASPIPE_ABI_VERSION);
   raw = *s;
-  NP_REQUIRE(raw.family == NASPIPE_MLP || raw.family == NASPIPE_TRANSFORMER, NASPIPE_EINVAL,
-             "unsupported family %d", raw.family);
+  NP_REQUIRE(raw.family == NASPIPE_MLP || raw.family == NASPIPE_TRANSFORMER || raw.family == NASPIPE_SPOS_CNN,
+             NASPIPE_EINVAL, "unsupported family %d", raw.family);
   NP_REQUIRE(raw.n_blocks >= 1 && raw.n_blocks <= 4096, NASPIPE_EINVAL, "n_blocks %d", raw.n_blocks);
   NP_REQUIRE(raw.n_choices >= 1 && raw.n_choices <= 4096, NASPIPE_EINVAL, "n_choices %d",
              raw.n_choices);
@@ -44,7 +44,7 @@ Spec::Spec(const naspipe_supernet_spec* s) {
   if (raw.family == NASPIPE_MLP) {
     NP_REQUIRE(raw.width >= 1 && raw.width <= 1024, NASPIPE_EINVAL, "width %d", raw.width);
     NP_REQUIRE(raw.compute_dtype == NASPIPE_FP32, NASPIPE_EINVAL, "MLP computes in fp32");
-  } else {
+  } else if (raw.family == NASPIPE_TRANSFORMER) {
     NP_REQUIRE(raw.compute_dtype == NASPIPE_BF16, NASPIPE_EINVAL, "transformer computes in bf16");
     NP_REQUIRE(raw.d_model >= 16 && raw.d_model % 16 == 0, NASPIPE_EINVAL,
                "d_model %d must be a positive multiple of 16", raw.d_model);
@@ -61,6 +61,34 @@ Spec::Spec(const naspipe_supernet_spec* s) {
       NP_REQUIRE(ffn[c] >= 16 && ffn[c] % 16 == 0, NASPIPE_EINVAL, "ffn[%d]=%d must be a multiple of 16",
                  c, ffn[c]);
     }
+  } else {
+    NP_REQUIRE(raw.compute_dtype == NASPIPE_BF16, NASPIPE_EINVAL, "SPOS CNN computes in bf16");
+    NP_REQUIRE(raw.n_cnn_stages >= 1 && raw.n_cnn_stages <= 8 && raw.stage_repeats && raw.stage_channels &&
+                   raw.choice_kernel && raw.choice_xception,
+               NASPIPE_EINVAL, "SPOS: n_cnn_stages / stage_repeats / stage_channels / choice_* missing");
+    reps.assign(raw.stage_repeats, raw.stage_repeats + raw.n_cnn_stages);
+    chans.assign(raw.stage_channels, raw.stage_channels + raw.n_cnn_stages);
+    kern.assign(raw.choice_kernel, raw.choice_kernel + n);
+    xcep.assign(raw.choice_xception, raw.choice_xception + n);
+    int total = 0, prev = raw.stem_channels;
+    NP_REQUIRE(raw.stem_channels >= 16 && raw.stem_channels % 16 == 0, NASPIPE_EINVAL, "stem_channels %d (%%16)",
+               raw.stem_channels);
+    for (int i = 0; i < raw.n_cnn_stages; ++i) {
+      NP_REQUIRE(reps[i] >= 1, NASPIPE_EINVAL, "stage_repeats[%d]=%d", i, reps[i]);
+      NP_REQUIRE(chans[i] % 32 == 0 && chans[i] > prev && (chans[i] - prev) % 16 == 0, NASPIPE_EINVAL,
+                 "stage_channels[%d]=%d must be %%32, > previous (%d), difference %%16", i, chans[i], prev);
+      total += reps[i];
+      prev = chans[i];
+    }
+    NP_REQUIRE(total == m, NASPIPE_EINVAL, "sum(stage_repeats)=%d != n_blocks=%d", total, m);
+    NP_REQUIRE(raw.image_hw >= 32 && raw.image_hw % (2 << raw.n_cnn_stages) == 0, NASPIPE_EINVAL,
+               "image_hw %d must be a multiple of 2^(1+n_cnn_stages)", raw.image_hw);
+    NP_REQUIRE(raw.num_classes >= 2 && raw.head_channels >= 16 && raw.head_channels % 16 == 0, NASPIPE_EINVAL,
+               "num_classes %d / head_channels %d (%%16)", raw.num_classes, raw.head_channels);
+    for (int c = 0; c < n; ++c)
+      NP_REQUIRE((kern[c] == 3 || kern[c] == 5 || kern[c] == 7) && (xcep[c] == 0 || (xcep[c] == 1 && kern[c] == 3)),
+                 NASPIPE_EINVAL, "choice %d: kernel %d xception %d (k in {3,5,7}; Xception uses k=3)", c, kern[c],
+                 xcep[c]);
   }
   if (raw.stage_of_block) {
     stage_of_block.assign(raw.stage_of_block, raw.stage_of_block + m);
@@ -75,26 +103,134 @@ Spec::Spec(const naspipe_supernet_spec* s) {
       NP_REQUIRE(cost_fwd[i] >= 0 && cost_bwd[i] >= 0, NASPIPE_EINVAL, "negative cost");
     has_costs = true;
   }
-  raw.choice_heads = heads.empty() ? nullptr : heads.data();
-  raw.choice_ffn = ffn.empty() ? nullptr : ffn.data();
-  raw.stage_of_block = has_partition ? stage_of_block.data() : nullptr;
-  raw.cost_fwd = has_costs ? cost_fwd.data() : nullptr;
-  raw.cost_bwd = has_costs ? cost_bwd.data() : nullptr;
+  repoint();
 }
 
 Spec::Spec(const Spec& o)
     : raw(o.raw), heads(o.heads), ffn(o.ffn), stage_of_block(o.stage_of_block),
-      cost_fwd(o.cost_fwd), cost_bwd(o.cost_bwd), has_partition(o.has_partition),
-      has_costs(o.has_costs) {
+      cost_fwd(o.cost_fwd), cost_bwd(o.cost_bwd), reps(o.reps), chans(o.chans), kern(o.kern),
+      xcep(o.xcep), has_partition(o.has_partition), has_costs(o.has_costs) {
+  repoint();
+}
+
+void Spec::repoint() {
   raw.choice_heads = heads.empty() ? nullptr : heads.data();
   raw.choice_ffn = ffn.empty() ? nullptr : ffn.data();
   raw.stage_of_block = has_partition ? stage_of_block.data() : nullptr;
   raw.cost_fwd = has_costs ? cost_fwd.data() : nullptr;
   raw.cost_bwd = has_costs ? cost_bwd.data() : nullptr;
+  raw.stage_repeats = reps.empty() ? nullptr : reps.data();
+  raw.stage_channels = chans.empty() ? nullptr : chans.data();
+  raw.choice_kernel = kern.empty() ? nullptr : kern.data();
+  raw.choice_xception = xcep.empty() ? nullptr : xcep.data();
 }
 
 size_t Spec::sample_elems() const {
+  if (family() == NASPIPE_SPOS_CNN) return (size_t)raw.image_hw * raw.image_hw * 3;
   return family() == NASPIPE_MLP ? (size_t)raw.width : (size_t)raw.seq_len * raw.d_model;
+}
+
+size_t Spec::input_bytes() const { return 4 * batch_elems(); }
+size_t Spec::target_bytes() const {
+  return family() == NASPIPE_SPOS_CNN ? 4 * (size_t)B() : 4 * batch_elems();
+}
+size_t Spec::act_bytes(int b) const {
+  if (family() != NASPIPE_SPOS_CNN) return 4 * batch_elems();
+  if (b < m()) {
+    const SposDims d = spos_dims(b);
+    return 2 * (size_t)B() * d.H_in * d.H_in * d.C_in;
+  }
+  const int hw = spos_last_hw();
+  return 2 * (size_t)B() * hw * hw * chans.back();
+}
+
+// oracle/spos.py block_dims: the stem halves image_hw; the first block of every CNN stage
+// has stride 2 (inp = C_prev, mid = C/2, out = C - C_prev), the others stride 1 with the
+// channel split (inp = mid = out = C/2).
+SposDims Spec::spos_dims(int b) const {
+  NP_REQUIRE(family() == NASPIPE_SPOS_CNN && b >= 0 && b < m(), NASPIPE_EINVAL, "spos_dims(%d)", b);
+  int c_prev = raw.stem_channels, H = raw.image_hw / 2, k = 0;
+  for (size_t st = 0; st < reps.size(); ++st) {
+    const int co = chans[st];
+    for (int i = 0; i < reps[st]; ++i, ++k) {
+      if (k == b) {
+        if (i == 0) return {2, c_prev, co / 2, co - c_prev, c_prev, co, H, H / 2};
+        return {1, co / 2, co / 2, co / 2, co, co, H, H};
+      }
+      if (i == 0) H /= 2;
+    }
+    c_prev = co;
+  }
+  return {};
+}
+
+int Spec::spos_last_hw() const { return raw.image_hw >> (1 + (int)reps.size()); }
+
+std::vector<SposConv> Spec::spos_convs(int b, int c) const {
+  const SposDims d = spos_dims(b);
+  const int k = kern[c];
+  std::vector<SposConv> L;
+  // (branch, dw, cin, cout, k, stride, relu, H_in, H_out)
+  auto add = [&](int br, int dw, int ci, int co, int kk, int s, int relu, int hin) {
+    SposConv u{};
+    u.branch = br; u.dw = dw; u.cin = ci; u.cout = co; u.k = kk; u.stride = s; u.relu = relu;
+    u.H_in = hin; u.H_out = hin / s;
+    L.push_back(u);
+  };
+  const int H = d.H_in, s = d.stride, Ho = d.H_out;
+  if (s == 2) {
+    add(0, 1, d.inp, d.inp, k, 2, 0, H);
+    add(0, 0, d.inp, d.inp, 1, 1, 1, Ho);
+  }
+  if (!xcep[c]) {
+    add(1, 0, d.inp, d.mid, 1, 1, 1, H);
+    add(1, 1, d.mid, d.mid, k, s, 0, H);
+    add(1, 0, d.mid, d.outm, 1, 1, 1, Ho);
+  } else {
+    add(1, 1, d.inp, d.inp, 3, s, 0, H);
+    add(1, 0, d.inp, d.mid, 1, 1, 1, Ho);
+    add(1, 1, d.mid, d.mid, 3, 1, 0, Ho);
+    add(1, 0, d.mid, d.mid, 1, 1, 1, Ho);
+    add(1, 1, d.mid, d.mid, 3, 1, 0, Ho);
+    add(1, 0, d.mid, d.outm, 1, 1, 1, Ho);
+  }
+  size_t off = 0, off16 = 0;
+  for (auto& u : L) {
+    u.off_w = off;
+    const size_t nw = u.dw ? (size_t)u.cout * u.k * u.k : (size_t)u.cout * u.cin;
+    off += nw;
+    u.off_g = off;
+    off += u.cout;
+    u.off_b = off;
+    off += u.cout;
+    u.off_w16 = off16;
+    if (!u.dw) off16 += nw;
+  }
+  return L;
+}
+
+size_t Spec::spos_shadow_elems(int b, int c) const {
+  size_t t = 0;
+  for (auto& u : spos_convs(b, c))
+    if (!u.dw) t += (size_t)u.cout * u.cin;
+  return t;
+}
+
+size_t Spec::frozen_count(int part) const {
+  if (part == 0) return (size_t)raw.stem_channels * 27;
+  if (part == 1) return (size_t)raw.head_channels * chans.back();
+  return (size_t)raw.num_classes * raw.head_channels;
+}
+
+void Spec::init_frozen(int part, float* dst) const {
+  const int fan = part == 0 ? 27 : part == 1 ? chans.back() : raw.head_channels;
+  const uint64_t uid = (uint64_t)m() * (uint64_t)n() + (uint64_t)part;
+  const float bound = 1.0f / std::sqrt((float)fan);
+  const size_t cnt = frozen_count(part);
+  for (size_t i = 0; i < cnt; ++i) {
+    const uint64_t z = splitmix64(raw.init_seed ^ (uid * 0x9E3779B97F4A7C15ull + i));
+    dst[i] = bound * (2.0f * ((float)(z >> 40) * 5.9604644775390625e-08f) - 1.0f);
+  }
 }
 
 int Spec::rows() const { return family() == NASPIPE_MLP ? raw.batch : raw.batch * raw.seq_len; }
@@ -115,8 +251,15 @@ TfOffsets Spec::tf_offsets(int c) const {
 }
 
 std::vector<Segment> Spec::segments(int b, int c) const {
-  (void)b;
   std::vector<Segment> s;
+  if (family() == NASPIPE_SPOS_CNN) {
+    for (auto& u : spos_convs(b, c)) {
+      s.push_back({u.off_w, u.off_g - u.off_w, 0, u.dw ? u.k * u.k : u.cin});
+      s.push_back({u.off_g, (size_t)u.cout, 1, 0});
+      s.push_back({u.off_b, (size_t)u.cout, 2, 0});
+    }
+    return s;
+  }
   if (family() == NASPIPE_MLP) {
     const size_t d = raw.width;
     s.push_back({0, d * d, 0, (int)d});
@@ -174,6 +317,14 @@ void Spec::default_costs(int32_t* cf, int32_t* cb) const {
         const double d = raw.width, T = raw.batch;
         flops = 2.0 * T * d * d;
         bytes = 4.0 * (3.0 * T * d + d * d + d);
+      } else if (family() == NASPIPE_SPOS_CNN) {
+        // per conv -> BN unit: conv reads x, writes z; BN stats read z; apply reads z, writes y
+        flops = bytes = 0;
+        for (auto& u : spos_convs(b, c)) {
+          const double Pin = (double)B() * u.H_in * u.H_in, Pout = (double)B() * u.H_out * u.H_out;
+          flops += u.dw ? 2.0 * Pout * u.cout * u.k * u.k : 2.0 * Pout * u.cin * u.cout;
+          bytes += 2.0 * (Pin * u.cin + 4.0 * Pout * u.cout);
+        }
       } else {
         const double d = raw.d_model, f = ffn[c], T = (double)raw.batch * raw.seq_len,
                      S = raw.seq_len;

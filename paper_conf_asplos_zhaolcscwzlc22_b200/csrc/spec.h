@@ -22,13 +22,30 @@ struct TfOffsets {
   size_t Wqkv, bqkv, Wo, bo, ln1g, ln1b, W1, b1, W2, b2, ln2g, ln2b, total;
 };
 
+// SPOS block geometry (SURVEY §8c "C2 SPOS candidate"; oracle/spos.py block_dims).
+struct SposDims {
+  int stride, inp, mid, outm, C_in, C_out, H_in, H_out;
+};
+// One conv -> BN [-> ReLU] unit of a SPOS candidate, in packing order.
+struct SposConv {
+  int branch;   // 0 = proj (stride-2 blocks), 1 = main
+  int dw;       // 1 = depthwise k x k, 0 = pointwise
+  int cin, cout, k, stride;
+  int relu;     // ReLU after the BN
+  int H_in, H_out;
+  size_t off_w, off_g, off_b;  // offsets in the packed fp32 vector
+  size_t off_w16;              // pw: offset of the bf16 GEMM operand in the shadow
+};
+
 struct Spec {
   naspipe_supernet_spec raw{};  // scalar fields; pointer fields re-pointed into vectors below
   std::vector<int32_t> heads, ffn, stage_of_block, cost_fwd, cost_bwd;
+  std::vector<int32_t> reps, chans, kern, xcep;  // SPOS
   bool has_partition = false, has_costs = false;
 
   explicit Spec(const naspipe_supernet_spec* s);
   Spec(const Spec& o);
+  void repoint();  // raw's pointer fields -> the owned vectors
 
   int family() const { return raw.family; }
   int m() const { return raw.n_blocks; }
@@ -40,6 +57,22 @@ struct Spec {
   // elements of one sample of input / output (the residual stream width per batch row)
   size_t sample_elems() const;
   size_t batch_elems() const { return (size_t)B() * sample_elems(); }
+  // Boundary tensors: bytes of the activation entering block b (b == m: the last block's
+  // output), of the batch input and of the target.  MLP/TRANSFORMER: fp32 [B, sample];
+  // SPOS: bf16 NHWC activations, fp32 NHWC image, int32 labels.
+  size_t act_bytes(int b) const;
+  size_t input_bytes() const;
+  size_t target_bytes() const;
+  // SPOS geometry
+  SposDims spos_dims(int b) const;
+  std::vector<SposConv> spos_convs(int b, int c) const;
+  size_t spos_shadow_elems(int b, int c) const;
+  int spos_stem_hw() const { return raw.image_hw / 2; }
+  int spos_last_hw() const;
+  // frozen SPOS parameters (reading A2): part 0 = stem [C0,3,3,3], 1 = head [Ch, Clast],
+  // 2 = fc [classes, Ch]; counter hash with uid m*n + part
+  size_t frozen_count(int part) const;
+  void init_frozen(int part, float* dst) const;
   int rows() const;  // GEMM rows T: B (MLP) or B*S (transformer)
   int d() const { return family() == NASPIPE_MLP ? raw.width : raw.d_model; }
 

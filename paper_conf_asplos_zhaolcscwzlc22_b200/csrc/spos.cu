@@ -1,0 +1,750 @@
+// SPOS CNN kernels (configs[1]): NHWC bf16 activations, fp32 BatchNorm statistics and
+// masters, CUDA cores for everything that is not a dense contraction (the 1x1 convs and the
+// frozen head's 1x1 conv run on the tcgen05 GEMM, gemm.cu).
+//
+// Block internals follow SURVEY §8c "C2 SPOS candidate" (readings A16, A27):
+// every conv is bias-free and followed by training-mode BatchNorm (batch statistics over
+// N*H*W, biased variance, eps 1e-5).  Per conv -> BN [-> ReLU] unit the forward is
+//   conv -> z (bf16);  bn_stats(z) -> per-row-block partial (sum, sum of squares);
+//   bn_finalize -> mean, rstd;  bn_apply -> y = relu?(g * ((z - mean) * rstd) + b) (bf16)
+// and the backward (dy = grad of y; s1 = sum dy', s2 = sum dy' * xh over the batch, dy' = dy
+// masked by the ReLU):
+//   bn_bwd_reduce -> partials of s1, s2;  bn_bwd_finalize -> s1, s2, and the WRITE of g, b
+//   (dg = s2, db = s1; the pre-update g, b are kept for the input gradient);
+//   bn_bwd_apply -> dz = rstd * g * (dy' - s1/P - xh * s2/P)  (bf16).
+// Every reduction has a fixed order (per-thread sequential, then a fixed cross-thread order,
+// then a fixed order over row blocks), never floating-point atomics: bitwise reproducible.
+#include <algorithm>
+
+#include "common.h"
+#include "kernels.h"
+#include "launch.h"
+#include "ptx.cuh"
+
+namespace naspipe {
+namespace {
+
+constexpr int TPB = 256;          // threads per block of the row-block kernels
+constexpr int BN_ROWS = 256;      // rows (pixels) per BN partial
+constexpr int DW_ROWS = 1024;     // output pixels per depthwise weight-gradient partial
+constexpr float BN_EPS = 1e-5f;
+
+inline void check_launch(const char* what) {
+  cudaError_t e = cudaGetLastError();
+  NP_REQUIRE(e == cudaSuccess, NASPIPE_ECUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+inline int grid_for(size_t items, int per_block = TPB) {
+  const size_t g = (items + per_block - 1) / per_block;
+  return (int)std::min<size_t>(std::max<size_t>(g, 1), 148 * 16);
+}
+
+__device__ __forceinline__ void load8(const bf16* p, float (&v)[8]) {
+  const uint4 q = *reinterpret_cast<const uint4*>(p);
+  const uint32_t w[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    v[2 * i] = __uint_as_float(w[i] << 16);
+    v[2 * i + 1] = __uint_as_float(w[i] & 0xffff0000u);
+  }
+}
+__device__ __forceinline__ void store8(bf16* p, const float (&v)[8]) {
+  uint4 q;
+  q.x = ptx::pack_bf16(v[0], v[1]);
+  q.y = ptx::pack_bf16(v[2], v[3]);
+  q.z = ptx::pack_bf16(v[4], v[5]);
+  q.w = ptx::pack_bf16(v[6], v[7]);
+  *reinterpret_cast<uint4*>(p) = q;
+}
+__device__ __forceinline__ void load8f(const float* p, float (&v)[8]) {
+  const float4 a = reinterpret_cast<const float4*>(p)[0], b = reinterpret_cast<const float4*>(p)[1];
+  v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w; v[4] = b.x; v[5] = b.y; v[6] = b.z; v[7] = b.w;
+}
+
+// BN output (also recomputed in the backward for the ReLU mask: same expression, same
+// rounding, explicit fma so no contraction choice can differ between the two kernels)
+__device__ __forceinline__ float bn_y(float z, float mu, float rs, float g, float b) {
+  return __fmaf_rn(g, __fmul_rn(__fsub_rn(z, mu), rs), b);
+}
+
+// ---------------------------------------------------------------- frozen stem (conv3x3 s2)
+// x fp32 NHWC [B,H,H,3], w fp32 [C0][3][3][3] ([out, kh, kw, in]), pad 1 -> z bf16 [B,H/2,H/2,C0]
+__global__ void stem_conv_kernel(const float* __restrict__ x, const float* __restrict__ w, bf16* __restrict__ z,
+                                 int B, int H, int C0) {
+  extern __shared__ float ws[];
+  ptx::pdl_wait();
+  for (int i = threadIdx.x; i < C0 * 27; i += blockDim.x) ws[i] = w[i];
+  __syncthreads();
+  const int Ho = H / 2;
+  const size_t P = (size_t)B * Ho * Ho;
+  for (size_t p = blockIdx.x * (size_t)blockDim.x + threadIdx.x; p < P; p += (size_t)gridDim.x * blockDim.x) {
+    const int b = (int)(p / ((size_t)Ho * Ho));
+    const int rem = (int)(p % ((size_t)Ho * Ho));
+    const int oh = rem / Ho, ow = rem % Ho;
+    float in[27];
+#pragma unroll
+    for (int u = 0; u < 3; ++u)
+#pragma unroll
+      for (int v = 0; v < 3; ++v) {
+        const int ih = 2 * oh + u - 1, iw = 2 * ow + v - 1;
+        const bool ok = ih >= 0 && ih < H && iw >= 0 && iw < H;
+        const float* src = x + (((size_t)b * H + (ok ? ih : 0)) * H + (ok ? iw : 0)) * 3;
+#pragma unroll
+        for (int ci = 0; ci < 3; ++ci) in[(u * 3 + v) * 3 + ci] = ok ? src[ci] : 0.f;
+      }
+    for (int c0 = 0; c0 < C0; c0 += 8) {
+      float acc[8];
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        float a = 0.f;
+        const float* wc = ws + (c0 + i) * 27;
+#pragma unroll
+        for (int t = 0; t < 27; ++t) a = __fmaf_rn(in[t], wc[t], a);
+        acc[i] = a;
+      }
+      store8(z + p * C0 + c0, acc);
+    }
+  }
+}
+
+// ---------------------------------------------------------------- BatchNorm forward
+// Thread (r, g): rows r, r + RP, ... of the block, channels [8g, 8g+8).  RP = TPB / G.
+__global__ void bn_stats_kernel(const bf16* __restrict__ z, int P, int C, float* __restrict__ part) {
+  extern __shared__ float red[];  // [RP][2C]
+  ptx::pdl_wait();
+  const int G = C / 8, RP = TPB / G;
+  const int r = threadIdx.x / G, g = threadIdx.x % G;
+  const int row0 = blockIdx.x * BN_ROWS, row1 = min(P, row0 + BN_ROWS);
+  if (r < RP) {
+    float s[8] = {}, q[8] = {};
+    for (int row = row0 + r; row < row1; row += RP) {
+      float v[8];
+      load8(z + (size_t)row * C + 8 * g, v);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        s[i] += v[i];
+        q[i] = __fmaf_rn(v[i], v[i], q[i]);
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      red[r * 2 * C + 8 * g + i] = s[i];
+      red[r * 2 * C + C + 8 * g + i] = q[i];
+    }
+  }
+  __syncthreads();
+  for (int e = threadIdx.x; e < 2 * C; e += TPB) {
+    float a = 0.f;
+    for (int k = 0; k < RP; ++k) a += red[k * 2 * C + e];
+    part[(size_t)blockIdx.x * 2 * C + e] = a;
+  }
+}
+
+// mean = sum / P, var = sumsq / P - mean^2 (biased), combined over row blocks in order in fp64
+__global__ void bn_finalize_kernel(const float* __restrict__ part, int nblk, int C, int P, float* __restrict__ mean,
+                                   float* __restrict__ rstd) {
+  ptx::pdl_wait();
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= C) return;
+  double s = 0.0, q = 0.0;
+  for (int k = 0; k < nblk; ++k) {
+    s += (double)part[(size_t)k * 2 * C + c];
+    q += (double)part[(size_t)k * 2 * C + C + c];
+  }
+  const double mu = s / P;
+  const double var = fmax(q / P - mu * mu, 0.0);
+  mean[c] = (float)mu;
+  rstd[c] = (float)(1.0 / sqrt(var + (double)BN_EPS));
+}
+
+__global__ void bn_apply_kernel(const bf16* __restrict__ z, int P, int C, const float* __restrict__ mean,
+                                const float* __restrict__ rstd, const float* __restrict__ gam,
+                                const float* __restrict__ bet, int relu, bf16* __restrict__ y, int ldy) {
+  ptx::pdl_wait();
+  const int G = C / 8;
+  const size_t items = (size_t)P * G;
+  for (size_t it = blockIdx.x * (size_t)blockDim.x + threadIdx.x; it < items; it += (size_t)gridDim.x * blockDim.x) {
+    const size_t p = it / G;
+    const int c = (int)(it % G) * 8;
+    float v[8], mu[8], rs[8], g8[8], b8[8];
+    load8(z + p * C + c, v);
+    load8f(mean + c, mu);
+    load8f(rstd + c, rs);
+    load8f(gam + c, g8);
+    load8f(bet + c, b8);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const float o = bn_y(v[i], mu[i], rs[i], g8[i], b8[i]);
+      v[i] = relu ? fmaxf(o, 0.f) : o;
+    }
+    store8(y + p * ldy + c, v);
+  }
+}
+
+// ---------------------------------------------------------------- BatchNorm backward
+__device__ __forceinline__ void bn_bwd_item(const bf16* dy, const bf16* z, const float (&mu)[8], const float (&rs)[8],
+                                            const float (&g8)[8], const float (&b8)[8], int relu, float (&d)[8],
+                                            float (&xh)[8]) {
+  float zz[8];
+  load8(dy, d);
+  load8(z, zz);
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    xh[i] = __fmul_rn(__fsub_rn(zz[i], mu[i]), rs[i]);
+    if (relu && !(bn_y(zz[i], mu[i], rs[i], g8[i], b8[i]) > 0.f)) d[i] = 0.f;
+  }
+}
+
+__global__ void bn_bwd_reduce_kernel(const bf16* __restrict__ dy, int lddy, const bf16* __restrict__ z, int P, int C,
+                                     const float* __restrict__ mean, const float* __restrict__ rstd,
+                                     const float* __restrict__ gam, const float* __restrict__ bet, int relu,
+                                     float* __restrict__ part) {
+  extern __shared__ float red[];  // [RP][2C]
+  ptx::pdl_wait();
+  const int G = C / 8, RP = TPB / G;
+  const int r = threadIdx.x / G, g = threadIdx.x % G;
+  const int row0 = blockIdx.x * BN_ROWS, row1 = min(P, row0 + BN_ROWS);
+  if (r < RP) {
+    float mu[8], rs[8], g8[8], b8[8];
+    load8f(mean + 8 * g, mu);
+    load8f(rstd + 8 * g, rs);
+    load8f(gam + 8 * g, g8);
+    load8f(bet + 8 * g, b8);
+    float s1[8] = {}, s2[8] = {};
+    for (int row = row0 + r; row < row1; row += RP) {
+      float d[8], xh[8];
+      bn_bwd_item(dy + (size_t)row * lddy + 8 * g, z + (size_t)row * C + 8 * g, mu, rs, g8, b8, relu, d, xh);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        s1[i] += d[i];
+        s2[i] = __fmaf_rn(d[i], xh[i], s2[i]);
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      red[r * 2 * C + 8 * g + i] = s1[i];
+      red[r * 2 * C + C + 8 * g + i] = s2[i];
+    }
+  }
+  __syncthreads();
+  for (int e = threadIdx.x; e < 2 * C; e += TPB) {
+    float a = 0.f;
+    for (int k = 0; k < RP; ++k) a += red[k * 2 * C + e];
+    part[(size_t)blockIdx.x * 2 * C + e] = a;
+  }
+}
+
+// sums[0][c] = s1 = dbeta, sums[1][c] = s2 = dgamma (fixed order over row blocks, fp64);
+// old[0] = gamma, old[1] = beta before the update; the WRITE gamma -= lr s2, beta -= lr s1.
+__global__ void bn_bwd_finalize_kernel(const float* __restrict__ part, int nblk, int C, float* __restrict__ sums,
+                                       float* __restrict__ old, float* __restrict__ gam, float* __restrict__ bet,
+                                       float lr, int update) {
+  ptx::pdl_wait();
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= C) return;
+  double s1 = 0.0, s2 = 0.0;
+  for (int k = 0; k < nblk; ++k) {
+    s1 += (double)part[(size_t)k * 2 * C + c];
+    s2 += (double)part[(size_t)k * 2 * C + C + c];
+  }
+  const float f1 = (float)s1, f2 = (float)s2;
+  sums[c] = f1;
+  sums[C + c] = f2;
+  const float g = gam[c], b = bet[c];
+  old[c] = g;
+  old[C + c] = b;
+  if (update) {
+    gam[c] = g - lr * f2;
+    bet[c] = b - lr * f1;
+  }
+}
+
+__global__ void bn_bwd_apply_kernel(const bf16* __restrict__ dy, int lddy, const bf16* __restrict__ z, int P, int C,
+                                    const float* __restrict__ mean, const float* __restrict__ rstd,
+                                    const float* __restrict__ old, const float* __restrict__ sums, int relu,
+                                    bf16* __restrict__ dz) {
+  ptx::pdl_wait();
+  const int G = C / 8;
+  const float invP = 1.0f / (float)P;
+  const size_t items = (size_t)P * G;
+  for (size_t it = blockIdx.x * (size_t)blockDim.x + threadIdx.x; it < items; it += (size_t)gridDim.x * blockDim.x) {
+    const size_t p = it / G;
+    const int c = (int)(it % G) * 8;
+    float mu[8], rs[8], g8[8], b8[8], m1[8], m2[8], d[8], xh[8];
+    load8f(mean + c, mu);
+    load8f(rstd + c, rs);
+    load8f(old + c, g8);
+    load8f(old + C + c, b8);
+    load8f(sums + c, m1);
+    load8f(sums + C + c, m2);
+    bn_bwd_item(dy + p * lddy + c, z + p * C + c, mu, rs, g8, b8, relu, d, xh);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const float t = d[i] - m1[i] * invP - xh[i] * (m2[i] * invP);
+      d[i] = rs[i] * g8[i] * t;
+    }
+    store8(dz + p * C + c, d);
+  }
+}
+
+// ---------------------------------------------------------------- depthwise conv (pad K/2)
+// weights fp32 [C][K][K]; staged in shared memory as [K*K][C]
+template <int K>
+__device__ __forceinline__ void stage_dw_weights(float* ws, const float* w, int C) {
+  for (int i = threadIdx.x; i < C * K * K; i += blockDim.x) {
+    const int c = i / (K * K), t = i % (K * K);
+    ws[t * C + c] = w[i];
+  }
+  __syncthreads();
+}
+
+template <int K>
+__global__ void dw_fwd_kernel(const bf16* __restrict__ x, const float* __restrict__ w, bf16* __restrict__ z, int B,
+                              int H, int C, int S) {
+  extern __shared__ float ws[];
+  ptx::pdl_wait();
+  stage_dw_weights<K>(ws, w, C);
+  constexpr int PAD = K / 2;
+  const int Ho = (H + 2 * PAD - K) / S + 1;
+  const int G = C / 8;
+  const size_t items = (size_t)B * Ho * Ho * G;
+  for (size_t it = blockIdx.x * (size_t)blockDim.x + threadIdx.x; it < items; it += (size_t)gridDim.x * blockDim.x) {
+    const int c = (int)(it % G) * 8;
+    const size_t p = it / G;
+    const int ow = (int)(p % Ho);
+    const int oh = (int)((p / Ho) % Ho);
+    const int b = (int)(p / ((size_t)Ho * Ho));
+    float acc[8] = {};
+#pragma unroll
+    for (int u = 0; u < K; ++u) {
+      const int ih = oh * S + u - PAD;
+      if (ih < 0 || ih >= H) continue;
+      const bf16* row = x + (((size_t)b * H + ih) * H) * C + c;
+#pragma unroll
+      for (int v = 0; v < K; ++v) {
+        const int iw = ow * S + v - PAD;
+        if (iw < 0 || iw >= H) continue;
+        float xv[8], wv[8];
+        load8(row + (size_t)iw * C, xv);
+        const float* wt = ws + (u * K + v) * C + c;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) wv[i] = wt[i];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) acc[i] = __fmaf_rn(xv[i], wv[i], acc[i]);
+      }
+    }
+    store8(z + p * C + c, acc);
+  }
+}
+
+// dx[b,ih,iw,c] = sum_{u,v} dz[b,oh,ow,c] w[c,u,v] with oh*S + u - PAD = ih (+ add[b,ih,iw,c])
+template <int K>
+__global__ void dw_dgrad_kernel(const bf16* __restrict__ dz, const float* __restrict__ w, const bf16* __restrict__ add,
+                                bf16* __restrict__ dx, int B, int H, int C, int S) {
+  extern __shared__ float ws[];
+  ptx::pdl_wait();
+  stage_dw_weights<K>(ws, w, C);
+  constexpr int PAD = K / 2;
+  const int Ho = (H + 2 * PAD - K) / S + 1;
+  const int G = C / 8;
+  const size_t items = (size_t)B * H * H * G;
+  for (size_t it = blockIdx.x * (size_t)blockDim.x + threadIdx.x; it < items; it += (size_t)gridDim.x * blockDim.x) {
+    const int c = (int)(it % G) * 8;
+    const size_t p = it / G;
+    const int iw = (int)(p % H);
+    const int ih = (int)((p / H) % H);
+    const int b = (int)(p / ((size_t)H * H));
+    float acc[8] = {};
+#pragma unroll
+    for (int u = 0; u < K; ++u) {
+      const int t = ih + PAD - u;
+      if (t < 0 || t % S) continue;
+      const int oh = t / S;
+      if (oh >= Ho) continue;
+#pragma unroll
+      for (int v = 0; v < K; ++v) {
+        const int q = iw + PAD - v;
+        if (q < 0 || q % S) continue;
+        const int ow = q / S;
+        if (ow >= Ho) continue;
+        float dv[8];
+        load8(dz + (((size_t)b * Ho + oh) * Ho + ow) * C + c, dv);
+        const float* wt = ws + (u * K + v) * C + c;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) acc[i] = __fmaf_rn(dv[i], wt[i], acc[i]);
+      }
+    }
+    if (add) {
+      float a[8];
+      load8(add + p * C + c, a);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) acc[i] += a[i];
+    }
+    store8(dx + p * C + c, acc);
+  }
+}
+
+// Weight gradient partials: block (blk, u) sums over output pixels [blk*DW_ROWS, ...) the
+// products dz[b,oh,ow,c] * x[b, oh*S+u-PAD, ow*S+v-PAD, c] for every c, v.
+// part[blk][c][u][v] (the [C][K][K] layout of the weight).
+template <int K>
+__global__ void dw_wgrad_kernel(const bf16* __restrict__ dz, const bf16* __restrict__ x, float* __restrict__ part,
+                                int B, int H, int C, int S) {
+  extern __shared__ float red[];  // [RP][C][K]
+  ptx::pdl_wait();
+  constexpr int PAD = K / 2;
+  const int Ho = (H + 2 * PAD - K) / S + 1;
+  const int G = C / 8, RP = TPB / G;
+  const int r = threadIdx.x / G, g = threadIdx.x % G;
+  const int u = blockIdx.y;
+  const int P = B * Ho * Ho;
+  const int q0 = blockIdx.x * DW_ROWS, q1 = min(P, q0 + DW_ROWS);
+  if (r < RP) {
+    float acc[K][8] = {};
+    for (int q = q0 + r; q < q1; q += RP) {
+      const int ow = q % Ho, oh = (q / Ho) % Ho, b = q / (Ho * Ho);
+      const int ih = oh * S + u - PAD;
+      if (ih < 0 || ih >= H) continue;
+      float dv[8];
+      load8(dz + (size_t)q * C + 8 * g, dv);
+      const bf16* row = x + (((size_t)b * H + ih) * H) * C + 8 * g;
+#pragma unroll
+      for (int v = 0; v < K; ++v) {
+        const int iw = ow * S + v - PAD;
+        if (iw < 0 || iw >= H) continue;
+        float xv[8];
+        load8(row + (size_t)iw * C, xv);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) acc[v][i] = __fmaf_rn(dv[i], xv[i], acc[v][i]);
+      }
+    }
+#pragma unroll
+    for (int v = 0; v < K; ++v)
+#pragma unroll
+      for (int i = 0; i < 8; ++i) red[((size_t)r * C + 8 * g + i) * K + v] = acc[v][i];
+  }
+  __syncthreads();
+  for (int e = threadIdx.x; e < C * K; e += TPB) {
+    float a = 0.f;
+    for (int k = 0; k < RP; ++k) a += red[(size_t)k * C * K + e];
+    const int c = e / K, v = e % K;
+    part[(size_t)blockIdx.x * C * K * K + (size_t)c * K * K + u * K + v] = a;
+  }
+}
+
+// ---------------------------------------------------------------- channel split / merge
+// stride-1 block input x [P, 2Ch]: out[:, i] = x[:, 2i] (passed through, ld ldo), xm[:, i] = x[:, 2i+1]
+__global__ void chan_split_kernel(const bf16* __restrict__ x, int P, int Ch, bf16* __restrict__ out, int ldo,
+                                  bf16* __restrict__ xm) {
+  ptx::pdl_wait();
+  const int G = Ch / 8;
+  const size_t items = (size_t)P * G;
+  for (size_t it = blockIdx.x * (size_t)blockDim.x + threadIdx.x; it < items; it += (size_t)gridDim.x * blockDim.x) {
+    const size_t p = it / G;
+    const int g = (int)(it % G);
+    float a[8], b[8], ev[8], od[8];
+    load8(x + p * 2 * Ch + 16 * g, a);
+    load8(x + p * 2 * Ch + 16 * g + 8, b);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      ev[i] = a[2 * i];
+      od[i] = a[2 * i + 1];
+      ev[4 + i] = b[2 * i];
+      od[4 + i] = b[2 * i + 1];
+    }
+    store8(out + p * ldo + 8 * g, ev);
+    store8(xm + p * Ch + 8 * g, od);
+  }
+}
+
+// dx[:, 2i] = dproj[:, i] (ld ldp), dx[:, 2i+1] = dm[:, i]
+__global__ void chan_merge_kernel(const bf16* __restrict__ dproj, int ldp, const bf16* __restrict__ dm, int P, int Ch,
+                                  bf16* __restrict__ dx) {
+  ptx::pdl_wait();
+  const int G = Ch / 8;
+  const size_t items = (size_t)P * G;
+  for (size_t it = blockIdx.x * (size_t)blockDim.x + threadIdx.x; it < items; it += (size_t)gridDim.x * blockDim.x) {
+    const size_t p = it / G;
+    const int g = (int)(it % G);
+    float a[8], b[8], lo[8], hi[8];
+    load8(dproj + p * ldp + 8 * g, a);
+    load8(dm + p * Ch + 8 * g, b);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      lo[2 * i] = a[i];
+      lo[2 * i + 1] = b[i];
+      hi[2 * i] = a[4 + i];
+      hi[2 * i + 1] = b[4 + i];
+    }
+    store8(dx + p * 2 * Ch + 16 * g, lo);
+    store8(dx + p * 2 * Ch + 16 * g + 8, hi);
+  }
+}
+
+// ---------------------------------------------------------------- frozen head
+// gap[b, c] = (sum_{hw} r[b, hw, c]) / HW, in hw order
+__global__ void gap_kernel(const bf16* __restrict__ r, int B, int HW, int C, float* __restrict__ gap) {
+  ptx::pdl_wait();
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= B * C) return;
+  const int b = i / C, c = i % C;
+  float s = 0.f;
+  for (int k = 0; k < HW; ++k) s += __bfloat162float(r[((size_t)b * HW + k) * C + c]);
+  gap[i] = s / (float)HW;
+}
+
+__device__ __forceinline__ float warp_sum(float v) {
+#pragma unroll
+  for (int s = 16; s >= 1; s >>= 1) v += __shfl_xor_sync(0xffffffffu, v, s);
+  return v;
+}
+__device__ __forceinline__ float warp_max(float v) {
+#pragma unroll
+  for (int s = 16; s >= 1; s >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, s));
+  return v;
+}
+
+// One block per sample: logits = W_fc gap[b] (fp32), softmax cross-entropy, dlogits / B.
+__global__ void fc_ce_kernel(const float* __restrict__ gap, const float* __restrict__ wf, const int* __restrict__ labels,
+                             int B, int C, int ncls, float* __restrict__ dlogits, float* __restrict__ loss_per) {
+  extern __shared__ float lg[];  // [ncls]
+  __shared__ float red[TPB / 32];
+  __shared__ float bc;
+  ptx::pdl_wait();
+  const int b = blockIdx.x, warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = TPB / 32;
+  const float* gb = gap + (size_t)b * C;
+  for (int j = warp; j < ncls; j += nw) {
+    const float* wr = wf + (size_t)j * C;
+    float a = 0.f;
+    for (int c = lane; c < C; c += 32) a = __fmaf_rn(gb[c], wr[c], a);
+    a = warp_sum(a);
+    if (lane == 0) lg[j] = a;
+  }
+  __syncthreads();
+  float mx = -INFINITY;
+  for (int j = threadIdx.x; j < ncls; j += TPB) mx = fmaxf(mx, lg[j]);
+  mx = warp_max(mx);
+  if (lane == 0) red[warp] = mx;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    float m = red[0];
+    for (int k = 1; k < nw; ++k) m = fmaxf(m, red[k]);
+    bc = m;
+  }
+  __syncthreads();
+  mx = bc;
+  float se = 0.f;
+  for (int j = threadIdx.x; j < ncls; j += TPB) se += expf(lg[j] - mx);
+  se = warp_sum(se);
+  __syncthreads();
+  if (lane == 0) red[warp] = se;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    float s = 0.f;
+    for (int k = 0; k < nw; ++k) s += red[k];
+    bc = mx + logf(s);
+  }
+  __syncthreads();
+  const float lse = bc;
+  const int lab = labels[b];
+  const bool ok = lab >= 0 && lab < ncls;
+  for (int j = threadIdx.x; j < ncls; j += TPB)
+    dlogits[(size_t)b * ncls + j] = (expf(lg[j] - lse) - (j == lab ? 1.f : 0.f)) / (float)B;
+  if (threadIdx.x == 0) loss_per[b] = ok ? lse - lg[lab] : __int_as_float(0x7fc00000);  // NaN flags a bad label
+}
+
+__global__ void ce_mean_kernel(const float* __restrict__ loss_per, int B, float* __restrict__ loss) {
+  ptx::pdl_wait();
+  if (threadIdx.x == 0 && blockIdx.x == 0) {
+    float s = 0.f;
+    for (int b = 0; b < B; ++b) s += loss_per[b];
+    *loss = s / (float)B;
+  }
+}
+
+// dgap[b, c] = sum_j dlogits[b, j] W_fc[j, c]
+__global__ void fc_dgap_kernel(const float* __restrict__ dlogits, const float* __restrict__ wf, int B, int C, int ncls,
+                               float* __restrict__ dgap) {
+  ptx::pdl_wait();
+  const int b = blockIdx.y, c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= C) return;
+  const float* dl = dlogits + (size_t)b * ncls;
+  float a = 0.f;
+  for (int j = 0; j < ncls; ++j) a = __fmaf_rn(dl[j], wf[(size_t)j * C + c], a);
+  dgap[(size_t)b * C + c] = a;
+}
+
+// dr[b, hw, c] = dgap[b, c] / HW
+__global__ void head_bcast_kernel(const float* __restrict__ dgap, int B, int HW, int C, bf16* __restrict__ dr) {
+  ptx::pdl_wait();
+  const int G = C / 8;
+  const size_t items = (size_t)B * HW * G;
+  for (size_t it = blockIdx.x * (size_t)blockDim.x + threadIdx.x; it < items; it += (size_t)gridDim.x * blockDim.x) {
+    const size_t p = it / G;
+    const int c = (int)(it % G) * 8;
+    const int b = (int)(p / HW);
+    float v[8];
+    load8f(dgap + (size_t)b * C + c, v);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) v[i] = v[i] / (float)HW;
+    store8(dr + p * C + c, v);
+  }
+}
+
+__global__ void synth_labels_kernel(int* __restrict__ labels, int B, int ncls, uint64_t seed) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= B) return;
+  uint64_t z = seed * 0x9E3779B97F4A7C15ull + (uint64_t)i + 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  z ^= z >> 31;
+  labels[i] = (int)(z % (uint64_t)ncls);
+}
+
+template <typename Kern>
+void set_smem(Kern k, size_t bytes) {
+  if (bytes > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+}
+
+}  // namespace
+
+// ================================================================ host launchers
+int bn_part_blocks(int P) { return (P + BN_ROWS - 1) / BN_ROWS; }
+int dw_wgrad_blocks(int P_out) { return (P_out + DW_ROWS - 1) / DW_ROWS; }
+
+void spos_stem_conv(cudaStream_t s, const float* x, const float* w, bf16* z, int B, int H, int C0) {
+  NP_REQUIRE(C0 % 8 == 0 && H % 2 == 0, NASPIPE_EINVAL, "stem C0=%d H=%d", C0, H);
+  const size_t P = (size_t)B * (H / 2) * (H / 2);
+  launch_pdl(stem_conv_kernel, dim3(grid_for(P)), dim3(TPB), C0 * 27 * sizeof(float), s, x, w, z, B, H, C0);
+  check_launch("stem_conv");
+}
+
+void bn_stats(cudaStream_t s, const bf16* z, int P, int C, float* part) {
+  NP_REQUIRE(C % 8 == 0 && C / 8 <= TPB, NASPIPE_EINVAL, "bn_stats C=%d", C);
+  const size_t sm = (size_t)(TPB / (C / 8)) * 2 * C * sizeof(float);
+  set_smem(bn_stats_kernel, sm);
+  launch_pdl(bn_stats_kernel, dim3(bn_part_blocks(P)), dim3(TPB), sm, s, z, P, C, part);
+  check_launch("bn_stats");
+}
+
+void bn_finalize(cudaStream_t s, const float* part, int nblk, int C, int P, float* mean, float* rstd) {
+  launch_pdl(bn_finalize_kernel, dim3((C + 127) / 128), dim3(128), 0, s, part, nblk, C, P, mean, rstd);
+  check_launch("bn_finalize");
+}
+
+void bn_apply(cudaStream_t s, const bf16* z, int P, int C, const float* mean, const float* rstd, const float* g,
+              const float* b, int relu, bf16* y, int ldy) {
+  launch_pdl(bn_apply_kernel, dim3(grid_for((size_t)P * (C / 8))), dim3(TPB), 0, s, z, P, C, mean, rstd, g, b, relu,
+             y, ldy);
+  check_launch("bn_apply");
+}
+
+void bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
+                   const float* rstd, const float* g, const float* b, int relu, float* part) {
+  NP_REQUIRE(C % 8 == 0 && C / 8 <= TPB, NASPIPE_EINVAL, "bn_bwd C=%d", C);
+  const size_t sm = (size_t)(TPB / (C / 8)) * 2 * C * sizeof(float);
+  set_smem(bn_bwd_reduce_kernel, sm);
+  launch_pdl(bn_bwd_reduce_kernel, dim3(bn_part_blocks(P)), dim3(TPB), sm, s, dy, lddy, z, P, C, mean, rstd, g, b,
+             relu, part);
+  check_launch("bn_bwd_reduce");
+}
+
+void bn_bwd_finalize(cudaStream_t s, const float* part, int nblk, int C, float* sums, float* old, float* g, float* b,
+                     float lr, int update) {
+  launch_pdl(bn_bwd_finalize_kernel, dim3((C + 127) / 128), dim3(128), 0, s, part, nblk, C, sums, old, g, b, lr,
+             update);
+  check_launch("bn_bwd_finalize");
+}
+
+void bn_bwd_apply(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
+                  const float* rstd, const float* old, const float* sums, int relu, bf16* dz) {
+  launch_pdl(bn_bwd_apply_kernel, dim3(grid_for((size_t)P * (C / 8))), dim3(TPB), 0, s, dy, lddy, z, P, C, mean, rstd,
+             old, sums, relu, dz);
+  check_launch("bn_bwd_apply");
+}
+
+#define DW_DISPATCH(K, EXPR) \
+  switch (K) {               \
+    case 3: { constexpr int KK = 3; EXPR; break; } \
+    case 5: { constexpr int KK = 5; EXPR; break; } \
+    case 7: { constexpr int KK = 7; EXPR; break; } \
+    default: NP_REQUIRE(false, NASPIPE_EINVAL, "depthwise kernel %d", K); \
+  }
+
+void dw_fwd(cudaStream_t s, const bf16* x, const float* w, bf16* z, int B, int H, int C, int k, int S) {
+  const int Ho = (H - 1) / S + 1;
+  const size_t items = (size_t)B * Ho * Ho * (C / 8);
+  const size_t sm = (size_t)C * k * k * sizeof(float);
+  DW_DISPATCH(k, {
+    set_smem(dw_fwd_kernel<KK>, sm);
+    launch_pdl(dw_fwd_kernel<KK>, dim3(grid_for(items)), dim3(TPB), sm, s, x, w, z, B, H, C, S);
+  });
+  check_launch("dw_fwd");
+}
+
+void dw_dgrad(cudaStream_t s, const bf16* dz, const float* w, const bf16* add, bf16* dx, int B, int H, int C, int k,
+              int S) {
+  const size_t items = (size_t)B * H * H * (C / 8);
+  const size_t sm = (size_t)C * k * k * sizeof(float);
+  DW_DISPATCH(k, {
+    set_smem(dw_dgrad_kernel<KK>, sm);
+    launch_pdl(dw_dgrad_kernel<KK>, dim3(grid_for(items)), dim3(TPB), sm, s, dz, w, add, dx, B, H, C, S);
+  });
+  check_launch("dw_dgrad");
+}
+
+void dw_wgrad(cudaStream_t s, const bf16* dz, const bf16* x, float* part, int B, int H, int C, int k, int S) {
+  NP_REQUIRE(C % 8 == 0 && C / 8 <= TPB, NASPIPE_EINVAL, "dw_wgrad C=%d", C);
+  const int Ho = (H - 1) / S + 1;
+  const int nblk = dw_wgrad_blocks(B * Ho * Ho);
+  const size_t sm = (size_t)(TPB / (C / 8)) * C * k * sizeof(float);
+  DW_DISPATCH(k, {
+    set_smem(dw_wgrad_kernel<KK>, sm);
+    launch_pdl(dw_wgrad_kernel<KK>, dim3(nblk, KK), dim3(TPB), sm, s, dz, x, part, B, H, C, S);
+  });
+  check_launch("dw_wgrad");
+}
+
+void chan_split(cudaStream_t s, const bf16* x, int P, int Ch, bf16* out, int ldo, bf16* xm) {
+  launch_pdl(chan_split_kernel, dim3(grid_for((size_t)P * (Ch / 8))), dim3(TPB), 0, s, x, P, Ch, out, ldo, xm);
+  check_launch("chan_split");
+}
+
+void chan_merge(cudaStream_t s, const bf16* dproj, int ldp, const bf16* dm, int P, int Ch, bf16* dx) {
+  launch_pdl(chan_merge_kernel, dim3(grid_for((size_t)P * (Ch / 8))), dim3(TPB), 0, s, dproj, ldp, dm, P, Ch, dx);
+  check_launch("chan_merge");
+}
+
+void gap_pool(cudaStream_t s, const bf16* r, int B, int HW, int C, float* gap) {
+  launch_pdl(gap_kernel, dim3((B * C + TPB - 1) / TPB), dim3(TPB), 0, s, r, B, HW, C, gap);
+  check_launch("gap");
+}
+
+void fc_ce(cudaStream_t s, const float* gap, const float* wf, const int* labels, int B, int C, int ncls,
+           float* dlogits, float* loss_per) {
+  const size_t sm = (size_t)ncls * sizeof(float);
+  set_smem(fc_ce_kernel, sm);
+  launch_pdl(fc_ce_kernel, dim3(B), dim3(TPB), sm, s, gap, wf, labels, B, C, ncls, dlogits, loss_per);
+  check_launch("fc_ce");
+}
+
+void ce_mean(cudaStream_t s, const float* loss_per, int B, float* loss) {
+  launch_pdl(ce_mean_kernel, dim3(1), dim3(32), 0, s, loss_per, B, loss);
+  check_launch("ce_mean");
+}
+
+void fc_dgap(cudaStream_t s, const float* dlogits, const float* wf, int B, int C, int ncls, float* dgap) {
+  launch_pdl(fc_dgap_kernel, dim3((C + 127) / 128, B), dim3(128), 0, s, dlogits, wf, B, C, ncls, dgap);
+  check_launch("fc_dgap");
+}
+
+void head_bcast(cudaStream_t s, const float* dgap, int B, int HW, int C, bf16* dr) {
+  launch_pdl(head_bcast_kernel, dim3(grid_for((size_t)B * HW * (C / 8))), dim3(TPB), 0, s, dgap, B, HW, C, dr);
+  check_launch("head_bcast");
+}
+
+void synth_labels(cudaStream_t s, int* labels, int B, int ncls, uint64_t seed) {
+  synth_labels_kernel<<<(B + 127) / 128, 128, 0, s>>>(labels, B, ncls, seed);
+  check_launch("synth_labels");
+}
+
+}  // namespace naspipe

@@ -1,0 +1,209 @@
+"""SPOS CNN kernel unit tests on the GPU (SURVEY §4 tier T2) through include/naspipe_debug.h.
+
+Reference: float64 NumPy written here from the textbook definitions (depthwise conv with
+zero padding k//2, training-mode BatchNorm, its backward, the channel split of a stride-1
+ShuffleNetV2 block), evaluated on the SAME bf16-rounded inputs the kernel reads.  Bars:
+bf16 outputs within 2^-8 normwise and >= 99 % of elements within 1 bf16 ulp of the
+rounded reference; fp32 outputs (statistics, weight-gradient sums) normwise <= 1e-5;
+exact copies (split / merge) bitwise; every kernel bitwise reproducible across two runs.
+Shapes include the full configs[1] block-0 geometry (P = 200704 pixels) and ragged BN row
+blocks (P not a multiple of 256).
+"""
+import ctypes as C
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+npipe = pytest.importorskip("paper_conf_asplos_zhaolcscwzlc22_b200")
+L = npipe.lib
+_vp, _i = C.c_void_p, C.c_int
+L.naspipe_debug_dw.argtypes = [_vp] * 7 + [_i] * 5 + [_vp]
+L.naspipe_debug_bn_fwd.argtypes = [_vp, _i, _i, _vp, _vp, _i, _vp, _i, _vp, _vp, _vp]
+L.naspipe_debug_bn_bwd.argtypes = [_vp, _i, _vp, _i, _i, _vp, _vp, _vp, _vp, _i, _vp, _vp, _vp, C.c_float, _i, _vp]
+L.naspipe_debug_chan_split.argtypes = [_vp, _i, _i, _vp, _i, _vp, _vp]
+L.naspipe_debug_chan_merge.argtypes = [_vp, _i, _vp, _i, _i, _vp, _vp]
+L.naspipe_debug_stem.argtypes = [_vp, _vp, _vp, _i, _i, _i, _vp]
+
+
+def _ok(rc):
+    assert rc == 0, L.naspipe_last_error().decode()
+
+
+def _p(t):
+    return None if t is None else t.data_ptr()
+
+
+def _f64(t):
+    return t.detach().to(torch.float64).cpu().numpy()
+
+
+def _bf(a):
+    """bf16 device tensor of a (RNE) and its exact float64 value."""
+    t = torch.from_numpy(np.ascontiguousarray(a, dtype=np.float32)).to(torch.bfloat16).cuda()
+    return t, _f64(t)
+
+
+def _check_bf16(got, ref):
+    scale = max(np.max(np.abs(ref)), 1e-30)
+    assert np.max(np.abs(got - ref)) / scale <= 2.0 ** -8
+    r16 = _f64(torch.from_numpy(ref.astype(np.float32)).to(torch.bfloat16))
+    ulp = np.maximum(np.abs(r16), 1e-30) * 2.0 ** -7
+    assert np.mean(np.abs(got - r16) <= ulp + 1e-30) >= 0.99
+
+
+def _dw_ref(x, w, s):
+    B, H, _, Cc = x.shape
+    k = w.shape[1]
+    p = k // 2
+    Ho = (H + 2 * p - k) // s + 1
+    xp = np.pad(x, ((0, 0), (p, p), (p, p), (0, 0)))
+    y = np.zeros((B, Ho, Ho, Cc))
+    for u in range(k):
+        for v in range(k):
+            y += xp[:, u:u + s * (Ho - 1) + 1:s, v:v + s * (Ho - 1) + 1:s, :] * w[:, u, v]
+    return y
+
+
+def _dw_bwd_ref(x, w, s, dz):
+    k = w.shape[1]
+    p = k // 2
+    B, Ho, _, Cc = dz.shape
+    xp = np.pad(x, ((0, 0), (p, p), (p, p), (0, 0)))
+    dxp = np.zeros_like(xp)
+    dw = np.zeros_like(w)
+    for u in range(k):
+        for v in range(k):
+            sl = (slice(None), slice(u, u + s * (Ho - 1) + 1, s), slice(v, v + s * (Ho - 1) + 1, s), slice(None))
+            dxp[sl] += dz * w[:, u, v]
+            dw[:, u, v] = np.sum(dz * xp[sl], axis=(0, 1, 2))
+    H = x.shape[1]
+    return dxp[:, p:p + H, p:p + H, :], dw
+
+
+@pytest.mark.parametrize("B,H,Cc,k,s", [(2, 9, 16, 3, 1), (3, 8, 48, 5, 2), (2, 14, 32, 7, 1), (1, 7, 640, 3, 1),
+                                        (4, 6, 320, 7, 2), (64, 112, 16, 3, 2)])
+def test_depthwise_fwd_dgrad_wgrad(B, H, Cc, k, s):
+    rng = np.random.default_rng(B * 100 + H + Cc + k)
+    xd, x = _bf(rng.standard_normal((B, H, H, Cc)))
+    w = (rng.standard_normal((Cc, k, k)) / k).astype(np.float32)
+    wd = torch.from_numpy(w).cuda()
+    Ho = (H - 1) // s + 1
+    dzd, dz = _bf(rng.standard_normal((B, Ho, Ho, Cc)))
+    addd, add = _bf(rng.standard_normal((B, H, H, Cc)))
+    z = torch.empty((B, Ho, Ho, Cc), dtype=torch.bfloat16, device="cuda")
+    dx = torch.empty((B, H, H, Cc), dtype=torch.bfloat16, device="cuda")
+    dws = torch.empty((Cc, k, k), dtype=torch.float32, device="cuda")
+    outs = []
+    for _ in range(2):
+        _ok(L.naspipe_debug_dw(_p(xd), _p(wd), _p(z), _p(dzd), _p(addd), _p(dx), _p(dws), B, H, Cc, k, s, None))
+        torch.cuda.synchronize()
+        outs.append((z.clone(), dx.clone(), dws.clone()))
+    for a, b in zip(outs[0], outs[1]):
+        assert torch.equal(a, b)
+    if B * H * H > 100000:   # full-size block 0: check the reductions on a sample of channels
+        ch = [0, 7, 15]
+        x, dz, add, w64 = x[..., ch], dz[..., ch], add[..., ch], w[ch].astype(np.float64)
+        got_z, got_dx, got_dw = _f64(z)[..., ch], _f64(dx)[..., ch], _f64(dws)[ch]
+    else:
+        w64 = w.astype(np.float64)
+        got_z, got_dx, got_dw = _f64(z), _f64(dx), _f64(dws)
+    _check_bf16(got_z, _dw_ref(x, w64, s))
+    rdx, rdw = _dw_bwd_ref(x, w64, s, dz)
+    _check_bf16(got_dx, rdx + add)
+    assert np.max(np.abs(got_dw - rdw)) / np.max(np.abs(rdw)) <= 1e-5
+
+
+def _bn_ref(z, g, b, relu):
+    mu = z.mean(axis=0)
+    var = ((z - mu) ** 2).mean(axis=0)
+    rstd = 1.0 / np.sqrt(var + 1e-5)
+    xh = (z - mu) * rstd
+    y = g * xh + b
+    return (np.maximum(y, 0) if relu else y), mu, rstd, xh
+
+
+@pytest.mark.parametrize("P,Cc,relu", [(16, 64, 1), (4096, 16, 0), (1000, 48, 1), (3136, 1024, 1), (50176, 160, 1),
+                                       (200704, 32, 0)])
+def test_batchnorm_fwd_bwd(P, Cc, relu):
+    rng = np.random.default_rng(P + Cc)
+    zd, z = _bf(rng.standard_normal((P, Cc)) * rng.uniform(0.5, 2.0, Cc) + rng.uniform(-1, 1, Cc))
+    g = rng.uniform(0.5, 1.5, Cc).astype(np.float32)
+    b = rng.uniform(-0.3, 0.3, Cc).astype(np.float32)
+    gd, bd = torch.from_numpy(g).cuda(), torch.from_numpy(b).cuda()
+    ld = Cc + 16   # the output is a column slice of a wider tensor (block-output concat)
+    y = torch.zeros((P, ld), dtype=torch.bfloat16, device="cuda")
+    mean = torch.empty(Cc, device="cuda")
+    rstd = torch.empty(Cc, device="cuda")
+    _ok(L.naspipe_debug_bn_fwd(_p(zd), P, Cc, _p(gd), _p(bd), relu, _p(y[:, 8:]), ld, _p(mean), _p(rstd), None))
+    torch.cuda.synchronize()
+    ry, mu, rs, xh = _bn_ref(z, g.astype(np.float64), b.astype(np.float64), relu)
+    assert np.max(np.abs(_f64(mean) - mu)) <= 1e-5 * max(1.0, np.max(np.abs(mu)))
+    assert np.max(np.abs(_f64(rstd) / rs - 1)) <= 1e-5
+    yy = _f64(y)
+    _check_bf16(yy[:, 8:8 + Cc], ry)
+    assert not yy[:, :8].any() and not yy[:, 8 + Cc:].any()
+    # backward with a strided incoming gradient
+    dyfull_d, dyfull = _bf(rng.standard_normal((P, ld)))
+    dy = dyfull[:, 8:8 + Cc]
+    dz = torch.empty((P, Cc), dtype=torch.bfloat16, device="cuda")
+    sums = torch.empty(2 * Cc, device="cuda")
+    old = torch.empty(2 * Cc, device="cuda")
+    lr = 0.01
+    g2, b2 = gd.clone(), bd.clone()
+    _ok(L.naspipe_debug_bn_bwd(_p(dyfull_d[:, 8:]), ld, _p(zd), P, Cc, _p(mean), _p(rstd), _p(g2), _p(b2), relu,
+                               _p(dz), _p(sums), _p(old), lr, 1, None))
+    torch.cuda.synchronize()
+    # reference with the kernel's own statistics (the statistics were checked above)
+    mu32, rs32 = _f64(mean), _f64(rstd)
+    xh = (z - mu32) * rs32
+    yv = g.astype(np.float64) * xh + b
+    d = dy * (yv > 0) if relu else dy
+    s1, s2 = d.sum(axis=0), (d * xh).sum(axis=0)
+    rdz = rs32 * g * (d - s1 / P - xh * s2 / P)
+    s = _f64(sums)
+    assert np.max(np.abs(s[:Cc] - s1)) <= 1e-5 * np.max(np.abs(s1)) + 1e-6 * np.sqrt(P)
+    assert np.max(np.abs(s[Cc:] - s2)) <= 1e-5 * np.max(np.abs(s2)) + 1e-6 * np.sqrt(P)
+    np.testing.assert_array_equal(_f64(old), np.concatenate([g, b]).astype(np.float64))
+    np.testing.assert_allclose(_f64(g2), g - lr * s[Cc:].astype(np.float32), rtol=1e-6, atol=1e-7)
+    np.testing.assert_allclose(_f64(b2), b - lr * s[:Cc].astype(np.float32), rtol=1e-6, atol=1e-7)
+    _check_bf16(_f64(dz), rdz)
+
+
+@pytest.mark.parametrize("P,Ch", [(7, 16), (3136, 320), (1000, 80)])
+def test_channel_split_merge_exact(P, Ch):
+    rng = np.random.default_rng(P)
+    xd, x = _bf(rng.standard_normal((P, 2 * Ch)))
+    out = torch.zeros((P, 2 * Ch), dtype=torch.bfloat16, device="cuda")
+    xm = torch.empty((P, Ch), dtype=torch.bfloat16, device="cuda")
+    _ok(L.naspipe_debug_chan_split(_p(xd), P, Ch, _p(out), 2 * Ch, _p(xm), None))
+    dmd, dm = _bf(rng.standard_normal((P, Ch)))
+    dx = torch.empty((P, 2 * Ch), dtype=torch.bfloat16, device="cuda")
+    _ok(L.naspipe_debug_chan_merge(_p(xd), 2 * Ch, _p(dmd), P, Ch, _p(dx), None))
+    torch.cuda.synchronize()
+    o = _f64(out)
+    np.testing.assert_array_equal(o[:, :Ch], x[:, 0::2])
+    assert not o[:, Ch:].any()
+    np.testing.assert_array_equal(_f64(xm), x[:, 1::2])
+    r = np.empty((P, 2 * Ch))
+    r[:, 0::2] = x[:, :Ch]
+    r[:, 1::2] = dm
+    np.testing.assert_array_equal(_f64(dx), r)
+
+
+def test_stem_conv():
+    rng = np.random.default_rng(3)
+    B, H, C0 = 2, 32, 16
+    x = rng.standard_normal((B, H, H, 3)).astype(np.float32)
+    w = (rng.standard_normal((C0, 3, 3, 3)) / 5).astype(np.float32)
+    z = torch.empty((B, H // 2, H // 2, C0), dtype=torch.bfloat16, device="cuda")
+    xd, wd = torch.from_numpy(x).cuda(), torch.from_numpy(w).cuda()   # keep both alive during the launch
+    _ok(L.naspipe_debug_stem(_p(xd), _p(wd), _p(z), B, H, C0, None))
+    torch.cuda.synchronize()
+    xp = np.pad(x.astype(np.float64), ((0, 0), (1, 1), (1, 1), (0, 0)))
+    ref = np.zeros((B, H // 2, H // 2, C0))
+    for u in range(3):
+        for v in range(3):
+            ref += xp[:, u:u + H - 1:2, v:v + H - 1:2, :] @ w[:, u, v, :].T.astype(np.float64)
+    _check_bf16(_f64(z), ref)
