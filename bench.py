@@ -108,11 +108,22 @@ class ClockSampler:
 
 # ------------------------------------------------------------------------------ CPU oracle
 def oracle_block_sample(cfg, n_blocks_sample):
-    """Time the fp64 oracle on `n_blocks_sample` full-size blocks (fwd + bwd + SGD) of
-    subnet 0.  Returns (seconds, sample description)."""
+    """Time the fp64 oracle on a bounded sample of one subnet's step (fwd + bwd + SGD).
+    MLP / transformer: `n_blocks_sample` full-size blocks of subnet 0.  SPOS: the whole
+    subnet (stem, 20 blocks, head) on `n_blocks_sample` of the batch's images (its BatchNorm
+    statistics then cover that sub-batch; the arithmetic per image is the same).
+    Returns seconds."""
     from oracle import train, transformer, mlp   # noqa: F401  (test infrastructure, timing only)
     ch = synth.sample_choices(1, cfg["n_blocks"], cfg["n_choices"])[0]
     x, t = synth.make_batch(cfg, 0)
+    if cfg["family"] == "spos":
+        sub = dict(cfg, batch=n_blocks_sample)
+        theta = {(b, int(c)): train.unpack(cfg, b, int(c), v) for (b, c), v in
+                 ((k, v) for k, v in train.initial_theta(cfg).items()) if int(ch[b]) == c}
+        t0 = time.perf_counter()
+        loss, grads = train.subnet_step(sub, theta, ch, x[:n_blocks_sample], t[:n_blocks_sample])
+        train.sgd_apply(theta, grads, cfg["lr"])
+        return time.perf_counter() - t0
     theta = {}
     for b in range(n_blocks_sample):
         c = int(ch[b])
@@ -125,6 +136,15 @@ def oracle_block_sample(cfg, n_blocks_sample):
     return time.perf_counter() - t0
 
 
+def sample_size(cfg):
+    """(sample units, units per subnet, description) of the bounded oracle sample."""
+    if cfg["family"] == "spos":
+        return 4, cfg["batch"], "images"
+    if cfg["family"] == "transformer":
+        return (2 if cfg["d_model"] <= 1024 else 1), cfg["n_blocks"], "blocks"
+    return cfg["n_blocks"], cfg["n_blocks"], "blocks"
+
+
 def cpu_threads():
     try:
         from threadpoolctl import threadpool_info
@@ -133,28 +153,30 @@ def cpu_threads():
         return os.cpu_count()
 
 
-def cpu_baseline(cfg, n_blocks_sample):
-    secs = oracle_block_sample(cfg, n_blocks_sample)
-    per_subnet = secs * cfg["n_blocks"] / n_blocks_sample
+def cpu_baseline(cfg):
+    ns, per, unit = sample_size(cfg)
+    secs = oracle_block_sample(cfg, ns)
+    per_subnet = secs * per / ns
     return {"value": cfg["batch"] / per_subnet, "unit": "samples/s", "cores": cpu_threads(), "kind": "oracle",
-            "sample": f"fp64 NumPy oracle, {n_blocks_sample} of {cfg['n_blocks']} blocks of subnet 0 "
-                      f"(fwd+bwd+SGD, full B={cfg['batch']}, shape of {cfg.get('d_model', cfg.get('width'))}), "
-                      f"{secs:.2f} s, scaled x{cfg['n_blocks'] / n_blocks_sample:g} to one subnet"}
+            "sample": f"fp64 NumPy oracle, {ns} of {per} {unit} of subnet 0 (fwd+bwd+SGD), "
+                      f"{secs:.2f} s, scaled x{per / ns:g} to one subnet of B={cfg['batch']}"}
 
 
 def run_reference(args, cfg, rank, world):
     """--impl reference: the oracle as it stands, on host cores, rank 0 only."""
     if rank != 0:
         return
-    nb = 1 if cfg["family"] == "transformer" else cfg["n_blocks"]
+    ns, per, unit = sample_size(cfg)
+    if cfg["family"] == "transformer":
+        ns = 1
     for _ in range(args.warmup):
-        oracle_block_sample(cfg, nb)
-    ts = [oracle_block_sample(cfg, nb) for _ in range(args.steps)]
-    per_subnet = float(np.mean(ts)) * cfg["n_blocks"] / nb
+        oracle_block_sample(cfg, ns)
+    ts = [oracle_block_sample(cfg, ns) for _ in range(args.steps)]
+    per_subnet = float(np.mean(ts)) * per / ns
     value = cfg["batch"] / per_subnet
     cores = cpu_threads()
-    sample = (f"each step = {nb} full-size block(s) fwd+bwd+SGD of subnet 0 in the fp64 oracle, "
-              f"scaled x{cfg['n_blocks'] / nb:g} to one subnet")
+    sample = (f"each step = {ns} of {per} {unit} of subnet 0, fwd+bwd+SGD in the fp64 oracle, "
+              f"scaled x{per / ns:g} to one subnet")
     print(json.dumps({
         "impl": "reference", "metric": "supernet samples/sec", "value": value, "unit": "samples/s",
         "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * per_subnet,
@@ -166,7 +188,7 @@ def run_reference(args, cfg, rank, world):
 
 def workload_config(args, cfg, world):
     names = {"transformer": "configs[2] transformer", "large_transformer": "configs[3] large_transformer",
-             "toy": "configs[0] toy"}
+             "toy": "configs[0] toy", "spos": "configs[1] SPOS CNN"}
     c = {"workload": names.get(args.workload, args.workload) if not args.n_choices
          else f"configs[4] sweep n={args.n_choices}",
          "n_blocks": cfg["n_blocks"], "n_choices": cfg["n_choices"], "batch": cfg["batch"],
@@ -174,6 +196,10 @@ def workload_config(args, cfg, world):
          "l2": "working set > L2 (active weights + activations per step >> 126 MB)"}
     if cfg["family"] == "transformer":
         c.update(seq_len=cfg["seq_len"], d_model=cfg["d_model"], heads=cfg["choice_heads"], ffn=cfg["choice_ffn"])
+    if cfg["family"] == "spos":
+        c.update(image_hw=cfg["image_hw"], stage_repeats=cfg["stage_repeats"], stage_channels=cfg["stage_channels"],
+                 choice_kernel=cfg["choice_kernel"], choice_xception=cfg["choice_xception"],
+                 num_classes=cfg["num_classes"])
     return c
 
 
@@ -288,9 +314,9 @@ def main():
         e1.record()
         torch.cuda.synchronize()
         ms2 = max_over_ranks(e0.elapsed_time(e1))
-        per = x.numel() * 4
         e2e = {"value": args.steps * B / (ms2 / 1000), "unit": "samples/s",
-               "h2d_bytes_per_step": 2 * per, "d2h_bytes_per_step": 4}
+               "h2d_bytes_per_step": x.numel() * x.element_size() + t.numel() * t.element_size(),
+               "d2h_bytes_per_step": 4}
     losses = npipe.naspipe_get_losses(h, y) if rank == world - 1 else None
     npipe.naspipe_destroy(h)
 
@@ -298,11 +324,10 @@ def main():
         return
     cpu = None
     if world == 1 and not args.no_cpu:
-        nb = (2 if cfg["d_model"] <= 1024 else 1) if cfg["family"] == "transformer" else cfg["n_blocks"]
-        cpu = cpu_baseline(cfg, nb)
+        cpu = cpu_baseline(cfg)
     out = {"metric": "supernet samples/sec", "value": value, "unit": "samples/s", "n_gpus": world,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
-           "scaling": "strong", "vs_baseline": None, "dtype": "bf16" if cfg["family"] == "transformer" else "f32",
+           "scaling": "strong", "vs_baseline": None, "dtype": "f32" if cfg["family"] == "mlp" else "bf16",
            "data": "synthetic (N(0,1) inputs/targets, counter-hash init, uniform per-block choices)",
            "config": workload_config(args, cfg, world), "clocks": clk.summary(), "e2e": e2e,
            "gpu_launches": int(launches), "roofline": roofline, "cpu_baseline": cpu,

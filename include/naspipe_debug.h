@@ -31,22 +31,27 @@ int naspipe_debug_ln_bwd(const float* dy, const float* x, const float* mean, con
                          const float* resid, float* dx, void* dx16, float* dgamma, float* dbeta, float* colsum,
                          int T, int d, void* stream);
 
-/* SPOS CNN kernels (spos.cu).  bf16 NHWC tensors [P = B*H*W rows][C].
- * depthwise k x k, stride S, pad k/2, w fp32 [C][k][k]: z = dw(x) if x && z; dx = dw'(dz)
- * (+ add) if dz && dx; dwsum[C*k*k] = full weight gradient sum(dz * x) if dz && x && dwsum. */
+/* SPOS CNN kernels (spos.cu).  NHWC tensors [P = B*H*W rows][C]; forward tensors are
+ * bf16x2 (hi plane followed by the lo plane; value = hi + lo), gradients plain bf16.
+ * depthwise k x k, stride S, pad k/2, w fp32 [C][k][k]: z = dw(x) (x2 -> x2) if x && z;
+ * dx = dw'(dz) (+ add) if dz && dx; dwsum[C*k*k] = sum(dz * x_hi) if dz && x && dwsum. */
 int naspipe_debug_dw(const void* x, const float* w, void* z, const void* dz, const void* add, void* dx,
                      float* dwsum, int B, int H, int C, int k, int S, void* stream);
-/* BatchNorm forward: mean/rstd of z over P rows (biased variance, eps 1e-5), then
- * y[p*ldy + c] = relu?(g (z - mean) rstd + b). */
+/* BatchNorm forward: mean/rstd of z (x2) over P rows (biased variance, eps 1e-5), then
+ * y[p*ldy + c] = relu?(g (z - mean) rstd + b) (x2, lo plane yplane elements after hi). */
 int naspipe_debug_bn_fwd(const void* z, int P, int C, const float* g, const float* b, int relu, void* y, int ldy,
-                         float* mean, float* rstd, void* stream);
+                         size_t yplane, float* mean, float* rstd, void* stream);
 /* BatchNorm backward: sums[2][C] = (sum dy', sum dy' xh), old[2][C] = (g, b) before the
  * SGD step g -= lr*sums[1], b -= lr*sums[0] (if update), dz = rstd g (dy' - s1/P - xh s2/P). */
 int naspipe_debug_bn_bwd(const void* dy, int lddy, const void* z, int P, int C, const float* mean,
                          const float* rstd, float* g, float* b, int relu, void* dz, float* sums, float* old, float lr,
                          int update, void* stream);
-/* stride-1 channel split / merge and the frozen stem conv (x fp32 [B,H,H,3] -> z bf16) */
-int naspipe_debug_chan_split(const void* x, int P, int Ch, void* out, int ldo, void* xm, void* stream);
+/* stride-1 channel split (x2) / merge (bf16) and the frozen stem conv (x fp32 [B,H,H,3] ->
+ * z x2); 3-pass bf16x2 GEMM out = A B^T (K-major hi/lo planes) -> x2 planes [M][N]. */
+int naspipe_debug_chan_split(const void* x, int P, int Ch, void* out, int ldo, size_t oplane, void* xm,
+                             void* stream);
+int naspipe_debug_gemm_x2(int M, int N, int K, const void* A_hi, const void* A_lo, int lda, const void* B_hi,
+                          const void* B_lo, int ldb, void* out_hi, void* out_lo, void* stream);
 int naspipe_debug_chan_merge(const void* dproj, int ldp, const void* dm, int P, int Ch, void* dx, void* stream);
 int naspipe_debug_stem(const float* x, const float* w, void* z, int B, int H, int C0, void* stream);
 

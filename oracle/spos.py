@@ -24,16 +24,18 @@ ShuffleNetV2 search space — reading SURVEY §8c "C2 SPOS candidate" (DESIGN.md
   order, each conv weight followed by its BN gamma, beta.  pw weights [out, in]; dw weights
   [C, k, k]; the stem weight [out, kh, kw, in].
 
-Storage precision (reading A28).  Every function takes an optional ``q``: the
-rounding applied where a stored tensor is written.  ``q = None`` (default) is the plain fp64
-definition.  ``q = to_bf16`` rounds exactly the tensors the bf16 path stores (conv outputs
-z, BN/ReLU outputs y, 1x1-conv weight operands, the head's operands, and the gradients dz,
-dx between units and blocks) with round-to-nearest-even, and computes everything else in
-fp64.  Reason: the ReLU masks are decisions taken from floating point; the task fixes that
-both sides take such decisions in the same precision, and without it a 2^-9 perturbation
-of the activations flips ~0.2 % of the masks, which moves the fp64 weight update of this
-family by ~20 % (tools/diag_spos.py; A28) -- no bf16 implementation can meet
-1e-3 against the plain definition.
+Storage precision (reading A28).  Every function takes an optional ``st``, the
+rounding applied where a tensor is stored (a ``Storage``): ``st.f`` for forward tensors
+(conv outputs z, BN/ReLU outputs y), ``st.w`` for the 1x1-conv weight operand of the
+forward, ``st.b`` for backward tensors (dz, dx, the head's dr), ``st.op`` for the operands
+the backward contractions read (x in the weight gradients, W in the 1x1 input gradients).
+``PLAIN`` (default) is the fp64 definition.  ``BF16`` rounds all of them to bfloat16;
+``BF16X2`` is the CUDA path's storage (forward tensors and weights as hi + lo bfloat16
+pairs, 16-bit mantissa; backward tensors and operands bfloat16).  These modes exist to
+measure the numerical noise floor of a storage format: BatchNorm + ReLU make the result
+chaotic under rounding (one flipped ReLU mask cascades), and with BF16 storage the weight
+update of configs[1] decorrelates from the fp64 one (A15 2.7e-3 after one step, update
+error > 100 %), which is why the path stores the forward in bf16x2.
 """
 import numpy as np
 
@@ -55,6 +57,24 @@ def to_bf16(x):
 
 def _id(x):
     return x
+
+
+def to_bf16x2(x):
+    """hi + lo with hi = bf16(x), lo = bf16(x - hi) (from the fp32 value)."""
+    a = np.asarray(x, dtype=np.float32).astype(np.float64)
+    hi = to_bf16(a)
+    return hi + to_bf16(a - hi)
+
+
+class Storage:
+    def __init__(self, f=_id, w=_id, b=_id, op=_id):
+        self.f, self.w, self.b, self.op = f, w, b, op
+
+
+PLAIN = Storage()
+BF16 = Storage(to_bf16, to_bf16, to_bf16, to_bf16)
+BF16X2 = Storage(to_bf16x2, to_bf16x2, to_bf16, to_bf16)
+STORAGE = {None: PLAIN, "fp64": PLAIN, "bf16": BF16, "bf16x2": BF16X2}
 
 
 # ------------------------------------------------------------------ shapes / layout
@@ -175,30 +195,31 @@ def bn_bwd(dy, g, cache):
 
 
 # ------------------------------------------------------------------ conv -> BN [-> ReLU] unit
-def _unit_fwd(p, name, kind, s, relu, x, q=_id):
+def _unit_fwd(p, name, kind, s, relu, x, st=PLAIN):
     w = p[name]
-    z = q(dw_fwd(x, w, s) if kind == "dw" else x @ q(w).T)
+    z = st.f(dw_fwd(x, w, s) if kind == "dw" else x @ st.w(w).T)
     y, cb = bn_fwd(z, p[name + "_g"], p[name + "_b"])
     if relu:
         y = np.maximum(y, 0.0)
-    y = q(y)
+    y = st.f(y)
     return y, (x, cb, y if relu else None)
 
 
-def _unit_bwd(p, name, kind, s, dy, tape, grads, q=_id, add=None):
+def _unit_bwd(p, name, kind, s, dy, tape, grads, st=PLAIN, add=None):
     """dx of the unit (+ add, the other branch's gradient of the same input, before the
     storage rounding), accumulating the parameter gradients into grads."""
     x, cb, yr = tape
     if yr is not None:
         dy = dy * (yr > 0)
     dz, grads[name + "_g"], grads[name + "_b"] = bn_bwd(dy, p[name + "_g"], cb)
-    dz = q(dz)
+    dz = st.b(dz)
     if kind == "dw":
-        dx, grads[name] = dw_bwd(x, p[name], s, dz)
+        dx, _ = dw_bwd(x, p[name], s, dz)
+        _, grads[name] = dw_bwd(st.op(x), p[name], s, dz)
     else:
-        grads[name] = np.einsum("bhwo,bhwi->oi", dz, x)
-        dx = dz @ q(p[name])
-    return q(dx if add is None else dx + add)
+        grads[name] = np.einsum("bhwo,bhwi->oi", dz, st.op(x))
+        dx = dz @ st.op(p[name])
+    return st.b(dx if add is None else dx + add)
 
 
 def _chain(cfg, b, c, which):
@@ -211,7 +232,7 @@ def _chain(cfg, b, c, which):
     return out
 
 
-def block_fwd(cfg, b, c, p, x, q=_id):
+def block_fwd(cfg, b, c, p, x, st=PLAIN):
     s = block_dims(cfg, b)[0]
     main_key = "x" if cfg["choice_xception"][c] else "m"
     if s == 1:
@@ -220,20 +241,20 @@ def block_fwd(cfg, b, c, p, x, q=_id):
         xp = xm = x
     tapes = {"p": [], main_key: []}
     h = xm
-    for name, kind, st, relu in _chain(cfg, b, c, main_key):
-        h, t = _unit_fwd(p, name, kind, st, relu, h, q)
+    for name, kind, stride, relu in _chain(cfg, b, c, main_key):
+        h, t = _unit_fwd(p, name, kind, stride, relu, h, st)
         tapes[main_key].append(t)
     main = h
     if s == 2:
         h = xp
-        for name, kind, st, relu in _chain(cfg, b, c, "p"):
-            h, t = _unit_fwd(p, name, kind, st, relu, h, q)
+        for name, kind, stride, relu in _chain(cfg, b, c, "p"):
+            h, t = _unit_fwd(p, name, kind, stride, relu, h, st)
             tapes["p"].append(t)
         xp = h
     return np.concatenate([xp, main], axis=-1), tapes
 
 
-def block_bwd(cfg, b, c, p, tapes, dy, q=_id):
+def block_bwd(cfg, b, c, p, tapes, dy, st=PLAIN):
     s, inp = block_dims(cfg, b)[:2]
     main_key = "x" if cfg["choice_xception"][c] else "m"
     cp = inp if s == 2 else dy.shape[-1] // 2
@@ -241,8 +262,8 @@ def block_bwd(cfg, b, c, p, tapes, dy, q=_id):
     grads = {}
     h = d_main
     chain = _chain(cfg, b, c, main_key)
-    for (name, kind, st, relu), t in zip(reversed(chain), reversed(tapes[main_key])):
-        h = _unit_bwd(p, name, kind, st, h, t, grads, q)
+    for (name, kind, stride, relu), t in zip(reversed(chain), reversed(tapes[main_key])):
+        h = _unit_bwd(p, name, kind, stride, h, t, grads, st)
     if s == 1:
         dx = np.zeros(d_proj.shape[:-1] + (2 * cp,))
         dx[..., 0::2] = d_proj
@@ -250,27 +271,27 @@ def block_bwd(cfg, b, c, p, tapes, dy, q=_id):
         return dx, grads
     g = d_proj
     pchain = list(zip(reversed(_chain(cfg, b, c, "p")), reversed(tapes["p"])))
-    for i, ((name, kind, st, relu), t) in enumerate(pchain):
+    for i, ((name, kind, stride, relu), t) in enumerate(pchain):
         last = i == len(pchain) - 1     # the proj branch's first unit: add the main branch's dx
-        g = _unit_bwd(p, name, kind, st, g, t, grads, q, add=h if last else None)
+        g = _unit_bwd(p, name, kind, stride, g, t, grads, st, add=h if last else None)
     return g, grads
 
 
 # ------------------------------------------------------------------ frozen stem / head
-def stem_fwd(fz, x, q=_id):
-    z = q(conv_fwd(x, fz["stem"]["w"], 2))
+def stem_fwd(fz, x, st=PLAIN):
+    z = st.f(conv_fwd(x, fz["stem"]["w"], 2))
     C = z.shape[-1]
     y, _ = bn_fwd(z, np.ones(C), np.zeros(C))
-    return q(np.maximum(y, 0.0))
+    return st.f(np.maximum(y, 0.0))
 
 
-def head_loss(fz, x, labels, q=_id):
+def head_loss(fz, x, labels, st=PLAIN):
     """Returns (loss, dL/dx) through pw -> BN -> ReLU -> GAP -> FC -> mean CE (frozen)."""
-    wh, wf = q(fz["head"]["w"]), fz["fc"]["w"]
-    z = q(x @ wh.T)
+    wh, wf = fz["head"]["w"], fz["fc"]["w"]
+    z = st.f(x @ st.w(wh).T)
     C = z.shape[-1]
     y, cb = bn_fwd(z, np.ones(C), np.zeros(C))
-    r = q(np.maximum(y, 0.0))
+    r = st.f(np.maximum(y, 0.0))
     gap = r.mean(axis=(1, 2))
     logits = gap @ wf.T
     mx = logits.max(axis=1, keepdims=True)
@@ -282,7 +303,7 @@ def head_loss(fz, x, labels, q=_id):
     dlog[np.arange(B), labels] -= 1.0
     dlog /= B
     dgap = dlog @ wf
-    dr = q(np.broadcast_to(dgap[:, None, None, :] / (r.shape[1] * r.shape[2]), r.shape))
+    dr = st.b(np.broadcast_to(dgap[:, None, None, :] / (r.shape[1] * r.shape[2]), r.shape))
     dy = dr * (r > 0)
     dz, _, _ = bn_bwd(dy, np.ones(C), cb)
-    return loss, q(q(dz) @ wh)
+    return loss, st.b(st.b(dz) @ st.op(wh))

@@ -84,9 +84,9 @@ def frozen_theta(cfg):
 
 
 def _spos_step(cfg, theta, choice, x, labels):
-    """SPOS step; cfg["storage"] == "bf16" selects the kernel-precision storage rounding of
-    reading A28 (spos.to_bf16 at every stored tensor), default plain fp64."""
-    q = spos.to_bf16 if cfg.get("storage") == "bf16" else spos._id
+    """SPOS step; cfg["storage"] in (None, "fp64", "bf16", "bf16x2") selects the storage
+    rounding of reading A28 (spos.Storage); default plain fp64."""
+    q = spos.STORAGE[cfg.get("storage")]
     fz = frozen_theta(cfg)
     h = spos.stem_fwd(fz, np.asarray(x, dtype=np.float64), q)
     tapes = []

@@ -122,7 +122,7 @@ int naspipe_debug_dw(const void* x, const float* w, void* z, const void* dz, con
 }
 
 int naspipe_debug_bn_fwd(const void* z, int P, int C, const float* g, const float* b, int relu, void* y, int ldy,
-                         float* mean, float* rstd, void* stream) {
+                         size_t yplane, float* mean, float* rstd, void* stream) {
   return dguard([&] {
     cudaStream_t s = (cudaStream_t)stream;
     const int nblk = bn_part_blocks(P);
@@ -130,7 +130,7 @@ int naspipe_debug_bn_fwd(const void* z, int P, int C, const float* g, const floa
     NP_REQUIRE(cudaMalloc(&part, (size_t)nblk * 2 * C * 4) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
     bn_stats(s, (const bf16*)z, P, C, part);
     bn_finalize(s, part, nblk, C, P, mean, rstd);
-    bn_apply(s, (const bf16*)z, P, C, mean, rstd, g, b, relu, (bf16*)y, ldy);
+    bn_apply(s, (const bf16*)z, P, C, mean, rstd, g, b, relu, (bf16*)y, ldy, yplane);
     cudaStreamSynchronize(s);
     cudaFree(part);
   });
@@ -152,8 +152,20 @@ int naspipe_debug_bn_bwd(const void* dy, int lddy, const void* z, int P, int C, 
   });
 }
 
-int naspipe_debug_chan_split(const void* x, int P, int Ch, void* out, int ldo, void* xm, void* stream) {
-  return dguard([&] { chan_split((cudaStream_t)stream, (const bf16*)x, P, Ch, (bf16*)out, ldo, (bf16*)xm); });
+int naspipe_debug_chan_split(const void* x, int P, int Ch, void* out, int ldo, size_t oplane, void* xm,
+                             void* stream) {
+  return dguard([&] { chan_split((cudaStream_t)stream, (const bf16*)x, P, Ch, (bf16*)out, ldo, oplane, (bf16*)xm); });
+}
+
+int naspipe_debug_gemm_x2(int M, int N, int K, const void* A_hi, const void* A_lo, int lda, const void* B_hi,
+                          const void* B_lo, int ldb, void* out_hi, void* out_lo, void* stream) {
+  return dguard([&] {
+    GemmEpiParams ep;
+    ep.out = out_hi;
+    ep.out2 = static_cast<bf16*>(out_lo);
+    gemm_bf16x2_tc((cudaStream_t)stream, M, N, K, (const bf16*)A_hi, (const bf16*)A_lo, lda, (const bf16*)B_hi,
+                   (const bf16*)B_lo, ldb, EPI_X2, ep);
+  });
 }
 
 int naspipe_debug_chan_merge(const void* dproj, int ldp, const void* dm, int P, int Ch, void* dx, void* stream) {

@@ -155,6 +155,8 @@ void Engine::stage_sizes() {
     const auto& bl = planner_.blocks_of(K);
     st_[K].in_bytes = K == 0 ? spec_.input_bytes() : spec_.act_bytes(bl.front());
     st_[K].out_bytes = spec_.act_bytes(bl.back() + 1);
+    st_[K].in_gbytes = spec_.grad_bytes(bl.front());
+    st_[K].out_gbytes = spec_.grad_bytes(bl.back() + 1);
   }
 }
 
@@ -177,9 +179,9 @@ void Engine::setup_stage(int K, int dev, bool local) {
   st.gin.assign(W_, nullptr);
   for (int s = 0; s < W_; ++s) {
     st.out[s] = st.arena->alloc<uint8_t>(st.out_bytes);
-    if (K > 0) st.gin[s] = st.arena->alloc<uint8_t>(st.in_bytes);
+    if (K > 0) st.gin[s] = st.arena->alloc<uint8_t>(st.in_gbytes);
     if (K == 0) st.in[s] = st.arena->alloc<uint8_t>(st.in_bytes);
-    if (K == D_ - 1) st.gout[s] = st.arena->alloc<uint8_t>(st.out_bytes);
+    if (K == D_ - 1) st.gout[s] = st.arena->alloc<uint8_t>(st.out_gbytes);
   }
   if (K == D_ - 1) {
     st.target.resize(W_);
@@ -208,7 +210,7 @@ void Engine::link_local_buffers() {
       }
       if (K < D_ - 1) {
         const StageRt& q = st_[K + 1];
-        st.gout[s] = (q.local && q.dev == st.dev) ? q.gin[s] : st.arena->alloc<uint8_t>(st.out_bytes);
+        st.gout[s] = (q.local && q.dev == st.dev) ? q.gin[s] : st.arena->alloc<uint8_t>(st.out_gbytes);
       }
     }
   }
@@ -357,9 +359,9 @@ void Engine::issue(const Task& t) {
       } else if (ops[k].op == RECV_GRAD) {
         CU(cudaSetDevice(me.dev));
         CU(cudaStreamWaitEvent(tx_->s_grad_in, me.ev_b[slot], 0));
-        NC(nccl().Recv(me.gout[slot], me.out_bytes, ncclUint8, 0, tx_->grad_in, tx_->s_grad_in));
+        NC(nccl().Recv(me.gout[slot], me.out_gbytes, ncclUint8, 0, tx_->grad_in, tx_->s_grad_in));
         CU(cudaEventRecord(tx_->ev_grad_rx[slot], tx_->s_grad_in));
-        p2p_bytes_ += (double)me.out_bytes;
+        p2p_bytes_ += (double)me.out_gbytes;
       }
     }
   }
@@ -446,8 +448,8 @@ void Engine::issue_backward(StageRt& st, int64_t y, int slot) {
       StageRt& q = st_[K + 1];
       CU(cudaStreamWaitEvent(st.comp, q.ev_b[slot], 0));
       if (q.dev != st.dev) {
-        CU(cudaMemcpyPeerAsync(st.gout[slot], st.dev, q.gin[slot], q.dev, st.out_bytes, st.comp));
-        p2p_bytes_ += (double)st.out_bytes;
+        CU(cudaMemcpyPeerAsync(st.gout[slot], st.dev, q.gin[slot], q.dev, st.out_gbytes, st.comp));
+        p2p_bytes_ += (double)st.out_gbytes;
       }
     } else {
       CU(cudaStreamWaitEvent(st.comp, tx_->ev_grad_rx[slot], 0));
@@ -459,7 +461,7 @@ void Engine::issue_backward(StageRt& st, int64_t y, int slot) {
   CU(cudaEventRecord(st.ev_b[slot], st.comp));
   if (rank_ >= 0 && tx_ && K > 0) {
     CU(cudaStreamWaitEvent(tx_->s_grad_out, st.ev_b[slot], 0));
-    NC(nccl().Send(st.gin[slot], st.in_bytes, ncclUint8, 0, tx_->grad_out, tx_->s_grad_out));
+    NC(nccl().Send(st.gin[slot], st.in_gbytes, ncclUint8, 0, tx_->grad_out, tx_->s_grad_out));
     CU(cudaEventRecord(tx_->ev_grad_tx[slot], tx_->s_grad_out));
   }
   cuda_check("backward");

@@ -27,7 +27,8 @@ struct StageRt {
   std::unique_ptr<CandidateStore> store;  // candidate parameters (resident or context-switched)
   size_t pushed = 0;                      // stage tasks fed to the store
   // boundary buffers per slot (device, on dev); opaque bytes (Spec::act_bytes)
-  size_t in_bytes = 0, out_bytes = 0;  // stage input (batch input at K = 0) / output
+  size_t in_bytes = 0, out_bytes = 0;    // stage input (batch input at K = 0) / output
+  size_t in_gbytes = 0, out_gbytes = 0;  // gradients w.r.t. them
   std::vector<void*> in, out, gin, gout, target;
   std::vector<cudaEvent_t> ev_f, ev_b, ev_in, ev_tgt;
   float* loss = nullptr;  // [loss_cap] on the last stage

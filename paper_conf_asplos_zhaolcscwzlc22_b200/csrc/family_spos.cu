@@ -2,14 +2,16 @@
 // (SURVEY §8c "C2 SPOS candidate"; oracle/spos.py), frozen stem on the first stage and frozen
 // head + cross-entropy on the last stage (reading A2).
 //
-// Layout: NHWC bf16 activations; a block's output is stored in logical channel order
+// Layout: NHWC activations, forward tensors bf16x2 (hi plane + lo plane, 16-bit mantissa;
+// DESIGN.md A28), gradients bf16; a block's output is stored in logical channel order
 // concat(proj, main) (P:L579 SPOS blocks); the stride-1 channel split (even channels pass
 // through, odd channels feed the main branch) is one kernel that writes the pass-through half
 // straight into the block output and the main-branch input contiguously.  Every conv -> BN
 // [-> ReLU] unit keeps z (bf16) and its batch mean / rstd in the slot's stash for the
-// backward; 1x1 convs run on the tcgen05 GEMM (forward: z = x W^T; dgrad: dx = dz W; wgrad
-// with the fused SGD WRITE: W -= lr dz^T x, deterministic split-K over the pixels), depthwise
-// convs and BatchNorm on CUDA cores (spos.cu).
+// backward; 1x1 convs run on the tcgen05 GEMM (forward: z = x W^T as the 3-pass bf16x2
+// product; dgrad: dx = dz W_hi; wgrad with the fused SGD WRITE: W -= lr dz^T x_hi,
+// deterministic split-K over the pixels, refreshing W's hi/lo planes), depthwise convs and
+// BatchNorm on CUDA cores (spos.cu).
 #include <algorithm>
 #include <cstring>
 
@@ -20,8 +22,8 @@ namespace naspipe {
 namespace {
 
 struct UnitRec {  // forward stash of one unit of (slot, block)
-  const bf16* x;  // unit input
-  bf16* z;        // conv output
+  const bf16* x;  // unit input (hi plane; bf16x2)
+  bf16* z;        // conv output (bf16x2, contiguous)
   float *mean, *rstd;
 };
 
@@ -42,15 +44,16 @@ class SposFamily : public Family {
       const int b = blocks[j];
       const SposDims d = spec.spos_dims(b);
       dims_[j] = d;
-      blk_max = std::max({blk_max, spec.act_bytes(b) / 2, spec.act_bytes(b + 1) / 2});
+      blk_max = std::max({blk_max, spec.grad_bytes(b) / 2, spec.grad_bytes(b + 1) / 2});
       for (int c = 0; c < n; ++c) {
         auto& L = plans_[(size_t)j * n + c];
         L = spec.spos_convs(b, c);
-        size_t need = d.stride == 1 ? P(d.H_in) * (d.C_out / 2) : 0, st = 0;
+        // forward stash in bf16 elements: x2 tensors take two planes
+        size_t need = d.stride == 1 ? 2 * P(d.H_in) * (d.C_out / 2) : 0, st = 0;
         for (size_t i = 0; i < L.size(); ++i) {
           const SposConv& u = L[i];
           const size_t po = P(u.H_out), pi = P(u.H_in);
-          need += po * u.cout * (last_of_branch(L, i) ? 1 : 2);
+          need += 2 * po * u.cout * (last_of_branch(L, i) ? 1 : 2);
           st += 2 * (size_t)u.cout;
           dz_max = std::max(dz_max, po * u.cout);
           g_max = std::max({g_max, pi * u.cin, po * u.cout});
@@ -104,11 +107,11 @@ class SposFamily : public Family {
       spec.init_frozen(0, h.data());
       w_stem_ = A.alloc<float>(h.size());
       cudaMemcpy(w_stem_, h.data(), h.size() * 4, cudaMemcpyHostToDevice);
-      stem_z_ = A.alloc<bf16>(P(hw0) * C0);
+      stem_z_ = A.alloc<bf16>(2 * P(hw0) * C0);
       stem_mean_ = A.alloc<float>(C0);
       stem_rstd_ = A.alloc<float>(C0);
       stem_y_.resize(W);
-      for (auto& p : stem_y_) p = A.alloc<bf16>(P(hw0) * C0);
+      for (auto& p : stem_y_) p = A.alloc<bf16>(2 * P(hw0) * C0);
       std::vector<float> ones(C0, 1.0f), zeros(C0, 0.0f);
       ones_s_ = A.alloc<float>(C0);
       zeros_s_ = A.alloc<float>(C0);
@@ -118,9 +121,12 @@ class SposFamily : public Family {
     if (last_) {
       std::vector<float> h(spec.frozen_count(1));
       spec.init_frozen(1, h.data());
-      std::vector<bf16> h16(h.size());
-      for (size_t i = 0; i < h.size(); ++i) h16[i] = __float2bfloat16_rn(h[i]);
-      wh16_ = A.alloc<bf16>(h.size());
+      std::vector<bf16> h16(2 * h.size());  // hi plane, lo plane
+      for (size_t i = 0; i < h.size(); ++i) {
+        h16[i] = __float2bfloat16_rn(h[i]);
+        h16[h.size() + i] = __float2bfloat16_rn(h[i] - __bfloat162float(h16[i]));
+      }
+      wh16_ = A.alloc<bf16>(h16.size());
       cudaMemcpy(wh16_, h16.data(), h16.size() * 2, cudaMemcpyHostToDevice);
       std::vector<float> f(spec.frozen_count(2));
       spec.init_frozen(2, f.data());
@@ -132,8 +138,8 @@ class SposFamily : public Family {
       cudaMemcpy(ones_, ones.data(), Ch * 4, cudaMemcpyHostToDevice);
       cudaMemcpy(zeros_, zeros.data(), Ch * 4, cudaMemcpyHostToDevice);
       const size_t PL = P(hwl);
-      zh_ = A.alloc<bf16>(PL * Ch);
-      rh_ = A.alloc<bf16>(PL * Ch);
+      zh_ = A.alloc<bf16>(2 * PL * Ch);
+      rh_ = A.alloc<bf16>(2 * PL * Ch);
       dzh_ = A.alloc<bf16>(PL * Ch);
       hmean_ = A.alloc<float>(Ch);
       hrstd_ = A.alloc<float>(Ch);
@@ -154,8 +160,9 @@ class SposFamily : public Family {
   void refresh_shadow(int j, int c, cudaStream_t s) override {
     float* p = master(j, c);
     bf16* w = w16_[(size_t)j * spec_.n() + c];
+    const size_t half = shadow_elems(j, c) / 2;
     for (const SposConv& u : plans_[(size_t)j * spec_.n() + c])
-      if (!u.dw) f32_to_bf16(s, p + u.off_w, w + u.off_w16, (size_t)u.cout * u.cin);
+      if (!u.dw) f32_to_bf16x2(s, p + u.off_w, w + u.off_w16, w + half + u.off_w16, (size_t)u.cout * u.cin);
   }
 
   void forward(int slot, const int32_t* ch, const void* x_in, void* x_out, cudaStream_t s) override {
@@ -167,7 +174,7 @@ class SposFamily : public Family {
       spos_stem_conv(s, static_cast<const float*>(x_in), w_stem_, stem_z_, B_, H, C0);
       bn_stats(s, stem_z_, Po, C0, part_);
       bn_finalize(s, part_, bn_part_blocks(Po), C0, Po, stem_mean_, stem_rstd_);
-      bn_apply(s, stem_z_, Po, C0, stem_mean_, stem_rstd_, ones_s_, zeros_s_, 1, stem_y_[slot], C0);
+      bn_apply(s, stem_z_, Po, C0, stem_mean_, stem_rstd_, ones_s_, zeros_s_, 1, stem_y_[slot], C0, (size_t)Po * C0);
       counters.launches += 4;
       x = stem_y_[slot];
     }
@@ -202,10 +209,12 @@ class SposFamily : public Family {
     const int PL = (int)P(hw), nblk = bn_part_blocks(PL);
     GemmEpiParams e;
     e.out = zh_;
-    gemm(s, PL, Ch, Cl, static_cast<const bf16*>(out), false, Cl, wh16_, false, Cl, EPI_BF16, e);
+    e.out2 = zh_ + (size_t)PL * Ch;
+    const bf16* xo = static_cast<const bf16*>(out);
+    gemm_x2(s, PL, Ch, Cl, xo, xo + (size_t)PL * Cl, Cl, wh16_, wh16_ + (size_t)Ch * Cl, Cl, e);
     bn_stats(s, zh_, PL, Ch, part_);
     bn_finalize(s, part_, nblk, Ch, PL, hmean_, hrstd_);
-    bn_apply(s, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, 1, rh_, Ch);
+    bn_apply(s, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, 1, rh_, Ch, (size_t)PL * Ch);
     gap_pool(s, rh_, B_, HW, Ch, gap_);
     fc_ce(s, gap_, wf_, static_cast<const int*>(target), B_, Ch, ncls, dlogits_, loss_per_);
     ce_mean(s, loss_per_, B_, loss_dst);
@@ -229,6 +238,15 @@ class SposFamily : public Family {
   static bool last_of_branch(const std::vector<SposConv>& L, size_t i) {
     return i + 1 == L.size() || L[i + 1].branch != L[i].branch;
   }
+  // forward 1x1 conv: 3-pass bf16x2 product into z's hi/lo planes
+  void gemm_x2(cudaStream_t s, int M, int N, int K, const bf16* Ahi, const bf16* Alo, int lda, const bf16* Bhi,
+               const bf16* Blo, int ldb, const GemmEpiParams& ep) {
+    if (timer) timer->begin(s);
+    gemm_bf16x2_tc(s, M, N, K, Ahi, Alo, lda, Bhi, Blo, ldb, EPI_X2, ep);
+    if (timer) timer->end(s, 6.0 * M * N * K);
+    counters.launches++;
+  }
+
   void gemm(cudaStream_t s, int M, int N, int K, const bf16* A, bool amn, int lda, const bf16* B, bool bmn, int ldb,
             int epi, const GemmEpiParams& ep, bool split_ok = false) {
     if (timer) timer->begin(s);
@@ -251,23 +269,32 @@ class SposFamily : public Family {
     float* st = stats_[k];
     auto& recs = recs_[k];
     recs.clear();
+    const size_t half = shadow_elems(j, c) / 2;  // lo planes of the 1x1 weights
+    const size_t oplane = P(d.H_out) * d.C_out;   // planes of the block output
     const bf16* main_in = x;
+    size_t main_plane = P(d.H_in) * d.C_in, x_plane = main_plane;
     int main_col = d.inp;  // column of the main branch in the block output
     if (d.stride == 1) {
       bf16* xm = cv;
-      cv += P(d.H_in) * (d.C_out / 2);
-      chan_split(s, x, (int)P(d.H_in), d.C_out / 2, out, d.C_out, xm);
+      main_plane = P(d.H_in) * (d.C_out / 2);
+      cv += 2 * main_plane;
+      chan_split(s, x, (int)P(d.H_in), d.C_out / 2, out, d.C_out, oplane, xm);
       counters.launches++;
       main_in = xm;
       main_col = d.C_out / 2;
     }
     const bf16* h = nullptr;
+    size_t hplane = 0;
     for (size_t i = 0; i < L.size(); ++i) {
       const SposConv& u = L[i];
-      if (i == 0 || L[i - 1].branch != u.branch) h = (u.branch == 0) ? x : main_in;
+      if (i == 0 || L[i - 1].branch != u.branch) {
+        h = (u.branch == 0) ? x : main_in;
+        hplane = (u.branch == 0) ? x_plane : main_plane;
+      }
       const int Po = (int)P(u.H_out);
+      const size_t zplane = (size_t)Po * u.cout;
       UnitRec r{h, cv, st, st + u.cout};
-      cv += (size_t)Po * u.cout;
+      cv += 2 * zplane;
       st += 2 * u.cout;
       if (u.dw) {
         dw_fwd(s, h, Pm + u.off_w, r.z, B_, u.H_in, u.cin, u.k, u.stride);
@@ -275,21 +302,26 @@ class SposFamily : public Family {
       } else {
         GemmEpiParams e;
         e.out = r.z;
-        gemm(s, Po, u.cout, u.cin, h, false, u.cin, W16 + u.off_w16, false, u.cin, EPI_BF16, e);
+        e.out2 = r.z + zplane;
+        gemm_x2(s, Po, u.cout, u.cin, h, h + hplane, u.cin, W16 + u.off_w16, W16 + half + u.off_w16, u.cin, e);
       }
       bn_stats(s, r.z, Po, u.cout, part_);
       bn_finalize(s, part_, bn_part_blocks(Po), u.cout, Po, r.mean, r.rstd);
       bf16* y;
       int ldy;
+      size_t yplane;
       if (last_of_branch(L, i)) {
         y = out + (u.branch == 0 ? 0 : main_col);
         ldy = d.C_out;
+        yplane = oplane;
       } else {
         y = cv;
-        cv += (size_t)Po * u.cout;
+        yplane = zplane;
+        cv += 2 * zplane;
         ldy = u.cout;
       }
-      bn_apply(s, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, u.relu, y, ldy);
+      bn_apply(s, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, u.relu, y, ldy, yplane);
+      hplane = yplane;
       counters.launches += 3;
       recs.push_back(r);
       h = y;
@@ -307,8 +339,8 @@ class SposFamily : public Family {
 
   // conv backward of one unit from dz_: dgrad into dst (+ add) with the pre-update weights
   // (skipped if dst == nullptr), then the weight gradient with the SGD WRITE.
-  void unit_conv_bwd(const SposConv& u, const UnitRec& r, float* Pm, bf16* W16, bf16* dst, const bf16* add,
-                     cudaStream_t s) {
+  void unit_conv_bwd(const SposConv& u, const UnitRec& r, float* Pm, bf16* W16, size_t half, bf16* dst,
+                     const bf16* add, cudaStream_t s) {
     const int Po = (int)P(u.H_out);
     if (u.dw) {
       if (dst) {
@@ -328,6 +360,7 @@ class SposFamily : public Family {
       GemmEpiParams e;
       e.w32 = Pm + u.off_w;
       e.w16 = W16 + u.off_w16;
+      e.w16lo = W16 + half + u.off_w16;
       e.lr = lr_;
       gemm(s, u.cout, u.cin, Po, dz_, true, u.cout, r.x, true, u.cin, EPI_SGD, e, true);
     }
@@ -338,6 +371,7 @@ class SposFamily : public Family {
     const auto& L = plans_[(size_t)j * spec_.n() + c];
     float* Pm = master(j, c);
     bf16* W16 = w16_[(size_t)j * spec_.n() + c];
+    const size_t half = shadow_elems(j, c) / 2;
     const auto& recs = recs_[k];
     const int main_col = d.stride == 1 ? d.C_out / 2 : d.inp;
     size_t m0 = 0;  // first main-branch unit
@@ -352,7 +386,7 @@ class SposFamily : public Family {
       bf16* dst;
       if (i > m0) dst = g_[pp ^= 1];
       else dst = need_dx ? (d.stride == 1 ? g_[pp ^ 1] : gfirst_) : nullptr;
-      unit_conv_bwd(u, recs[i], Pm, W16, dst, nullptr, s);
+      unit_conv_bwd(u, recs[i], Pm, W16, half, dst, nullptr, s);
       h = dst;
       ldh = u.cin;
     }
@@ -371,7 +405,7 @@ class SposFamily : public Family {
       const SposConv& u = L[i];
       unit_bn_bwd(u, recs[i], Pm, hp, ldp, s);
       bf16* dst = i > 0 ? g_[pp ^= 1] : (need_dx ? dxb : nullptr);
-      unit_conv_bwd(u, recs[i], Pm, W16, dst, (i == 0 && need_dx) ? gfirst_ : nullptr, s);
+      unit_conv_bwd(u, recs[i], Pm, W16, half, dst, (i == 0 && need_dx) ? gfirst_ : nullptr, s);
       hp = dst;
       ldp = u.cin;
     }

@@ -27,16 +27,25 @@ namespace naspipe {
 namespace {
 
 constexpr int BM = 128;
-constexpr int BN = 256;
-constexpr int BK = 64;  // 64 bf16 = 128 B = one swizzle row
-constexpr int STAGES = 4;
-constexpr int A_BYTES = BM * BK * 2;               // 16 KB
-constexpr int B_BYTES = BN * BK * 2;               // 32 KB
-constexpr int STAGE_BYTES = A_BYTES + B_BYTES;     // 48 KB
-constexpr int BAR_OFF = STAGES * STAGE_BYTES;
-constexpr int SMEM_TOTAL = BAR_OFF + (2 * STAGES + 4) * 8 + 16 + 1024;  // + alignment slack
+constexpr int BN = 256;  // tile N of the plain (1-pass) GEMM
+constexpr int BK = 64;   // 64 bf16 = 128 B = one swizzle row
+constexpr int A_BYTES = BM * BK * 2;  // 16 KB
 constexpr int THREADS = 320;  // 2 control warps + 8 epilogue warps
 constexpr int EPI_PARTIAL = 100;  // internal: fp32 partial tile of one K slice
+
+// Tile configuration: N tile TN; SPLIT = 3-pass bf16x2 product (A_hi B_hi + A_hi B_lo +
+// A_lo B_hi, fp32 accumulation: ~16-bit-mantissa operands, used by the SPOS forward 1x1
+// convs, A28).  The ring holds as many stages as fit in ~200 KB.
+template <int TN, bool SPLIT>
+struct TileCfg {
+  static constexpr int B_BYTES = TN * BK * 2;
+  static constexpr int OPS = SPLIT ? 2 : 1;
+  static constexpr int STAGE_BYTES = OPS * (A_BYTES + B_BYTES);
+  static constexpr int STAGES = (200 * 1024) / STAGE_BYTES > 6 ? 6 : (200 * 1024) / STAGE_BYTES;
+  static constexpr int BAR_OFF = STAGES * STAGE_BYTES;
+  static constexpr int SMEM_TOTAL = BAR_OFF + (2 * STAGES + 4) * 8 + 16 + 1024;  // + alignment slack
+  static constexpr int TMEM_COLS = 2 * TN <= 128 ? 128 : (2 * TN <= 256 ? 256 : 512);
+};
 
 __device__ __forceinline__ float gelu_tanh(float z) {
   const float c = 0.7978845608028654f;
@@ -117,6 +126,12 @@ __device__ __forceinline__ void epilogue16(float (&v)[16], const Pre16& pre, siz
   }
   if constexpr (EPI == EPI_F32 || EPI == EPI_BIAS_RESID_F32) {
     store16_f32(reinterpret_cast<float*>(ep.out) + off, v);
+  } else if constexpr (EPI == EPI_X2) {
+    float lo[16];
+#pragma unroll
+    for (int i = 0; i < 16; ++i) lo[i] = v[i] - __bfloat162float(__float2bfloat16_rn(v[i]));
+    store16_bf16(reinterpret_cast<bf16*>(ep.out) + off, v);
+    store16_bf16(ep.out2 + off, lo);
   } else if constexpr (EPI == EPI_SGD) {
     float w[16];
 #pragma unroll
@@ -128,6 +143,11 @@ __device__ __forceinline__ void epilogue16(float (&v)[16], const Pre16& pre, siz
       w[4 * i] = x.x; w[4 * i + 1] = x.y; w[4 * i + 2] = x.z; w[4 * i + 3] = x.w;
     }
     store16_bf16(ep.w16 + off, w);
+    if (ep.w16lo) {
+#pragma unroll
+      for (int i = 0; i < 16; ++i) w[i] -= __bfloat162float(__float2bfloat16_rn(w[i]));
+      store16_bf16(ep.w16lo + off, w);
+    }
   } else {
     store16_bf16(reinterpret_cast<bf16*>(ep.out) + off, v);
     if constexpr (EPI == EPI_BIAS_GELU) {
@@ -149,10 +169,16 @@ struct TileSpace {
   }
 };
 
-template <bool A_MN, bool B_MN, int EPI>
+template <bool A_MN, bool B_MN, int EPI, int TN, bool SPLIT>
 __global__ void __launch_bounds__(THREADS, 1)
-    gemm_tc_kernel(const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb, int M, int N,
+    gemm_tc_kernel(const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb,
+                   const __grid_constant__ CUtensorMap ta2, const __grid_constant__ CUtensorMap tb2, int M, int N,
                    TileSpace ts, GemmEpiParams ep) {
+  using Cf = TileCfg<TN, SPLIT>;
+  constexpr int STAGES = Cf::STAGES, STAGE_BYTES = Cf::STAGE_BYTES, BAR_OFF = Cf::BAR_OFF;
+  constexpr int B_BYTES = Cf::B_BYTES;
+  constexpr int OPB = A_BYTES + B_BYTES;  // bytes of one (A, B) operand pair in a stage
+  static_assert(!SPLIT || (!A_MN && !B_MN), "the 3-pass GEMM takes K-major operands");
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + BAR_OFF);
@@ -167,6 +193,10 @@ __global__ void __launch_bounds__(THREADS, 1)
   if (threadIdx.x == 0) {
     ptx::tma_prefetch(&ta);
     ptx::tma_prefetch(&tb);
+    if (SPLIT) {
+      ptx::tma_prefetch(&ta2);
+      ptx::tma_prefetch(&tb2);
+    }
     for (int s = 0; s < STAGES; ++s) {
       ptx::mbar_init(&full[s], 1);
       ptx::mbar_init(&empty[s], 1);
@@ -177,7 +207,7 @@ __global__ void __launch_bounds__(THREADS, 1)
     }
     ptx::fence_mbar_init();
   }
-  if (warp == 1) ptx::tmem_alloc<512>(tmem_holder);
+  if (warp == 1) ptx::tmem_alloc<Cf::TMEM_COLS>(tmem_holder);
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
@@ -190,7 +220,7 @@ __global__ void __launch_bounds__(THREADS, 1)
       for (int t = blockIdx.x; t < n_tiles; t += gridDim.x) {
         int tm, tn, ks;
         ts.decode(t, tm, tn, ks);
-        const int m0 = tm * BM, n0 = tn * BN;
+        const int m0 = tm * BM, n0 = tn * TN;
         const int kb0 = ks * ts.nk_per_split, kb1 = min(ts.nk, kb0 + ts.nk_per_split);
         for (int kb = kb0; kb < kb1; ++kb) {
           ptx::mbar_wait(&empty[s], ph ^ 1);
@@ -208,7 +238,11 @@ __global__ void __launch_bounds__(THREADS, 1)
             ptx::tma_load_2d(sb, &tb, &full[s], k0, n0);
           } else {
 #pragma unroll
-            for (int j = 0; j < BN / 64; ++j) ptx::tma_load_2d(sb + j * 8192, &tb, &full[s], n0 + 64 * j, k0);
+            for (int j = 0; j < TN / 64; ++j) ptx::tma_load_2d(sb + j * 8192, &tb, &full[s], n0 + 64 * j, k0);
+          }
+          if (SPLIT) {  // lo planes of both operands behind the hi pair
+            ptx::tma_load_2d(sa + OPB, &ta2, &full[s], k0, m0);
+            ptx::tma_load_2d(sb + OPB, &tb2, &full[s], k0, n0);
           }
           if (++s == STAGES) { s = 0; ph ^= 1; }
         }
@@ -217,7 +251,7 @@ __global__ void __launch_bounds__(THREADS, 1)
     ptx::pdl_trigger();
   } else if (warp == 1) {
     if (lane == 0) {  // ---------------- MMA issuer
-      constexpr uint32_t idesc = ptx::umma_idesc_bf16(BM, BN, A_MN ? 1 : 0, B_MN ? 1 : 0);
+      constexpr uint32_t idesc = ptx::umma_idesc_bf16(BM, TN, A_MN ? 1 : 0, B_MN ? 1 : 0);
       int s = 0, ph = 0, it = 0;
       for (int t = blockIdx.x; t < n_tiles; t += gridDim.x, ++it) {
         int tm, tn, ks;
@@ -226,7 +260,7 @@ __global__ void __launch_bounds__(THREADS, 1)
         const int acc = it & 1;
         ptx::mbar_wait(&tempty[acc], ((it >> 1) & 1) ^ 1);  // epilogue drained this buffer
         ptx::tc_fence_after();
-        const uint32_t d = tmem + acc * BN;
+        const uint32_t d = tmem + acc * TN;
         for (int kb = kb0; kb < kb1; ++kb) {
           ptx::mbar_wait(&full[s], ph);
           ptx::tc_fence_after();
@@ -242,6 +276,10 @@ __global__ void __launch_bounds__(THREADS, 1)
             const uint64_t bd = B_MN ? ptx::umma_desc_sw128(sb + k * 2048, 8192, 1024)
                                      : ptx::umma_desc_sw128(sb + k * 32, 16, 1024);
             ptx::umma_bf16(d, ad, bd, idesc, (kb > kb0 || k > 0) ? 1u : 0u);
+            if (SPLIT) {  // + A_hi B_lo + A_lo B_hi
+              ptx::umma_bf16(d, ad, ptx::umma_desc_sw128(sb + OPB + k * 32, 16, 1024), idesc, 1u);
+              ptx::umma_bf16(d, ptx::umma_desc_sw128(sa + OPB + k * 32, 16, 1024), bd, idesc, 1u);
+            }
           }
           ptx::umma_commit(&empty[s]);  // frees the smem stage when these MMAs complete
           if (++s == STAGES) { s = 0; ph ^= 1; }
@@ -253,7 +291,7 @@ __global__ void __launch_bounds__(THREADS, 1)
   } else {
     // ---------------- epilogue warps 2..9: TMEM lane quarter (warp % 4), column half
     const int lane_base = 32 * (warp & 3);
-    const int cbeg = ((warp - 2) >> 2) * (BN / 2);
+    const int cbeg = ((warp - 2) >> 2) * (TN / 2);
     int it = 0;
     for (int t = blockIdx.x; t < n_tiles; t += gridDim.x, ++it) {
       int tm, tn, ks;
@@ -264,10 +302,10 @@ __global__ void __launch_bounds__(THREADS, 1)
       if (t + (int)gridDim.x >= n_tiles) ptx::pdl_trigger();  // last tile: let the next kernel launch
       const int row = tm * BM + lane_base + lane;
       const bool row_ok = row < M;
-      const uint32_t taddr = tmem + ((uint32_t)lane_base << 16) + acc * BN;
+      const uint32_t taddr = tmem + ((uint32_t)lane_base << 16) + acc * TN;
 #pragma unroll 1
-      for (int c0 = cbeg; c0 < cbeg + BN / 2; c0 += 32) {
-        const int col = tn * BN + c0;
+      for (int c0 = cbeg; c0 < cbeg + TN / 2; c0 += 32) {
+        const int col = tn * TN + c0;
         if (col >= N) break;               // warp-uniform
         const bool two = col + 16 < N;     // N % 16 == 0: the chunk is 16 or 32 columns
         const size_t off = (size_t)row * N + col;
@@ -298,7 +336,7 @@ __global__ void __launch_bounds__(THREADS, 1)
   __syncthreads();
   if (warp == 1) {
     ptx::tc_fence_after();
-    ptx::tmem_dealloc<512>(tmem);
+    ptx::tmem_dealloc<Cf::TMEM_COLS>(tmem);
   }
 }
 
@@ -323,6 +361,12 @@ __global__ void splitk_reduce_kernel(int M, int N, int splits, GemmEpiParams ep)
       o.x = ptx::pack_bf16(w.x, w.y);
       o.y = ptx::pack_bf16(w.z, w.w);
       reinterpret_cast<uint2*>(ep.w16)[i] = o;
+      if (ep.w16lo) {
+        auto lo = [](float v) { return v - __bfloat162float(__float2bfloat16_rn(v)); };
+        o.x = ptx::pack_bf16(lo(w.x), lo(w.y));
+        o.y = ptx::pack_bf16(lo(w.z), lo(w.w));
+        reinterpret_cast<uint2*>(ep.w16lo)[i] = o;
+      }
     }
   }
 }
@@ -376,20 +420,21 @@ int num_sms() {
   return n;
 }
 
-template <bool A_MN, bool B_MN, int EPI>
+template <bool A_MN, bool B_MN, int EPI, int TN = BN, bool SPLIT = false>
 void launch(cudaStream_t s, int M, int N, const TileSpace& ts, const CUtensorMap& ta, const CUtensorMap& tb,
-            const GemmEpiParams& ep) {
-  auto kern = gemm_tc_kernel<A_MN, B_MN, EPI>;
+            const GemmEpiParams& ep, const CUtensorMap* ta2 = nullptr, const CUtensorMap* tb2 = nullptr) {
+  auto kern = gemm_tc_kernel<A_MN, B_MN, EPI, TN, SPLIT>;
+  constexpr int SMEM = TileCfg<TN, SPLIT>::SMEM_TOTAL;
   static uint32_t configured = 0;  // per instantiation, per device bit
   int dev = 0;
   cudaGetDevice(&dev);
   if (!(configured & (1u << dev))) {
-    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_TOTAL);
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
     configured |= 1u << dev;
   }
   const int tiles = ts.MT * ts.NT * ts.splits;
   const int grid = std::min(tiles, num_sms());
-  launch_pdl(kern, dim3(grid), dim3(THREADS), SMEM_TOTAL, s, ta, tb, M, N, ts, ep);
+  launch_pdl(kern, dim3(grid), dim3(THREADS), SMEM, s, ta, tb, ta2 ? *ta2 : ta, tb2 ? *tb2 : tb, M, N, ts, ep);
   g_gemm_launches.fetch_add(1, std::memory_order_relaxed);
 }
 
@@ -425,7 +470,7 @@ int gemm_splitk_factor(int M, int N, int K) {
     return rounds * ((nk + s - 1) / s) + red_us / 0.3;
   };
   int best = 1;
-  for (int s = 2; s <= 4; s *= 2)
+  for (int s = 2; s <= 256; s *= 2)
     if (nk / s >= 8 && cost(s) < 0.9 * cost(best)) best = s;
   return best;
 }
@@ -459,6 +504,36 @@ void gemm_bf16_tc(cudaStream_t s, int M, int N, int K, const bf16* A, bool a_mn,
     if (epi == EPI_F32) launch_pdl(splitk_reduce_kernel<EPI_F32>, dim3(blocks), dim3(256), 0, s, M, N, ts.splits, ep);
     else launch_pdl(splitk_reduce_kernel<EPI_SGD>, dim3(blocks), dim3(256), 0, s, M, N, ts.splits, ep);
   }
+}
+
+void gemm_bf16x2_tc(cudaStream_t s, int M, int N, int K, const bf16* A_hi, const bf16* A_lo, int lda,
+                    const bf16* B_hi, const bf16* B_lo, int ldb, int epi, const GemmEpiParams& ep) {
+  NP_REQUIRE(M > 0 && N > 0 && K > 0 && N % 16 == 0, NASPIPE_EINVAL, "gemm x2 dims M=%d N=%d K=%d (N%%16)", M, N, K);
+  NP_REQUIRE(epi == EPI_X2 || epi == EPI_BF16 || epi == EPI_F32, NASPIPE_EINVAL, "gemm x2 epilogue %d", epi);
+  const int tn = N <= 64 ? 64 : (N <= 128 ? 128 : 256);
+  const CUtensorMap ta = make_map(A_hi, (uint64_t)K, (uint64_t)M, (uint64_t)lda, BM);
+  const CUtensorMap ta2 = make_map(A_lo, (uint64_t)K, (uint64_t)M, (uint64_t)lda, BM);
+  const CUtensorMap tb = make_map(B_hi, (uint64_t)K, (uint64_t)N, (uint64_t)ldb, tn);
+  const CUtensorMap tb2 = make_map(B_lo, (uint64_t)K, (uint64_t)N, (uint64_t)ldb, tn);
+  TileSpace ts;
+  ts.MT = (M + BM - 1) / BM;
+  ts.NT = (N + tn - 1) / tn;
+  ts.nk = (K + BK - 1) / BK;
+  ts.splits = 1;
+  ts.nk_per_split = ts.nk;
+  GemmEpiParams e = ep;
+  e.ws_stride = (size_t)M * N;
+#define X2_CASE(TNV)                                                                       \
+  if (tn == TNV) {                                                                         \
+    if (epi == EPI_X2) launch<false, false, EPI_X2, TNV, true>(s, M, N, ts, ta, tb, e, &ta2, &tb2);   \
+    else if (epi == EPI_BF16) launch<false, false, EPI_BF16, TNV, true>(s, M, N, ts, ta, tb, e, &ta2, &tb2); \
+    else launch<false, false, EPI_F32, TNV, true>(s, M, N, ts, ta, tb, e, &ta2, &tb2);    \
+    return;                                                                                \
+  }
+  X2_CASE(64)
+  X2_CASE(128)
+  X2_CASE(256)
+#undef X2_CASE
 }
 
 }  // namespace naspipe

@@ -25,6 +25,8 @@ enum GemmEpi {
   EPI_BIAS_GELU = 4,      // z = acc + bias[n]; out16 = bf16(z); out2 = bf16(gelu_tanh(z))
   EPI_DGELU = 5,          // out16 = bf16(acc * gelu_tanh'(aux16[m,n]))
   EPI_SGD = 6,            // w32[m,n] -= lr * acc; w16[m,n] = bf16(w32[m,n])   (the WRITE)
+                          //   (+ w16lo[m,n] = bf16(w32 - w16) when w16lo != nullptr)
+  EPI_X2 = 7,             // out16 = hi = bf16(acc), out2 = lo = bf16(acc - hi)  (bf16x2 planes)
 };
 struct GemmEpiParams {
   const float* bias = nullptr;
@@ -34,6 +36,7 @@ struct GemmEpiParams {
   bf16* out2 = nullptr;
   float* w32 = nullptr;
   bf16* w16 = nullptr;
+  bf16* w16lo = nullptr;
   float lr = 0.f;
   // optional fp32 workspace enabling deterministic split-K for EPI_F32 / EPI_SGD
   float* ws = nullptr;
@@ -44,6 +47,11 @@ struct GemmEpiParams {
 int gemm_splitk_factor(int M, int N, int K);
 void gemm_bf16_tc(cudaStream_t s, int M, int N, int K, const bf16* A, bool a_mn, int lda, const bf16* B,
                   bool b_mn, int ldb, int epi, const GemmEpiParams& ep);
+// 3-pass bf16x2 GEMM (K-major A and B given as hi/lo planes): C = A_hi B_hi + A_hi B_lo +
+// A_lo B_hi (the A_lo B_lo term, < 2^-16 relative, is dropped); epilogues EPI_X2 / EPI_BF16 /
+// EPI_F32.  Tile N adapts to N (64 / 128 / 256).
+void gemm_bf16x2_tc(cudaStream_t s, int M, int N, int K, const bf16* A_hi, const bf16* A_lo, int lda,
+                    const bf16* B_hi, const bf16* B_lo, int ldb, int epi, const GemmEpiParams& ep);
 // number of tcgen05 GEMM launches so far in this process (stats)
 uint64_t gemm_launch_count();
 
@@ -106,16 +114,20 @@ void mlp_bwd_sgd(cudaStream_t s, const float* x, const float* h, const float* dy
                  float* b, float lr, int B, int d);
 
 // ------------------------------------------------------------------ SPOS CNN (spos.cu)
-// NHWC bf16 activations [P = B*H*W rows, C channels]; C % 8 == 0 everywhere.
-// frozen stem: x fp32 [B,H,H,3], w fp32 [C0][3][3][3], stride 2, pad 1 -> z bf16 [B,H/2,H/2,C0]
+// NHWC activations [P = B*H*W rows, C channels]; C % 8 == 0 everywhere.  Forward tensors
+// are bf16x2 (hi plane, lo plane `plane` elements later; contiguous tensors: plane = P*C),
+// backward tensors plain bf16 (A28).
+// w16 hi/lo planes of an fp32 vector
+void f32_to_bf16x2(cudaStream_t s, const float* w32, bf16* hi, bf16* lo, size_t n);
+// frozen stem: x fp32 [B,H,H,3], w fp32 [C0][3][3][3], stride 2, pad 1 -> z x2 [B,H/2,H/2,C0]
 void spos_stem_conv(cudaStream_t s, const float* x, const float* w, bf16* z, int B, int H, int C0);
 // BatchNorm (training mode, biased variance, eps 1e-5).  part: [bn_part_blocks(P)][2][C]
 int bn_part_blocks(int P);
 void bn_stats(cudaStream_t s, const bf16* z, int P, int C, float* part);
 void bn_finalize(cudaStream_t s, const float* part, int nblk, int C, int P, float* mean, float* rstd);
-// y[p*ldy + c] = relu?(g (z - mean) rstd + b)
+// y[p*ldy + c] = relu?(g (z - mean) rstd + b); z x2 (plane P*C), y x2 (planes yplane apart)
 void bn_apply(cudaStream_t s, const bf16* z, int P, int C, const float* mean, const float* rstd, const float* g,
-              const float* b, int relu, bf16* y, int ldy);
+              const float* b, int relu, bf16* y, int ldy, size_t yplane);
 void bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
                    const float* rstd, const float* g, const float* b, int relu, float* part);
 // sums [2][C] = (sum dy', sum dy' xh); old [2][C] = pre-update (g, b); update: SGD of g, b
@@ -123,15 +135,17 @@ void bn_bwd_finalize(cudaStream_t s, const float* part, int nblk, int C, float* 
                      float lr, int update);
 void bn_bwd_apply(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
                   const float* rstd, const float* old, const float* sums, int relu, bf16* dz);
-// depthwise k x k (k in {3,5,7}), stride S, pad k/2; w fp32 [C][k][k]; H = input height = width
+// depthwise k x k (k in {3,5,7}), stride S, pad k/2; w fp32 [C][k][k]; H = input height = width.
+// dw_fwd: x2 -> x2; dw_dgrad: bf16 (+ bf16 add); dw_wgrad reads the hi plane of x.
 void dw_fwd(cudaStream_t s, const bf16* x, const float* w, bf16* z, int B, int H, int C, int k, int S);
 void dw_dgrad(cudaStream_t s, const bf16* dz, const float* w, const bf16* add, bf16* dx, int B, int H, int C, int k,
               int S);
 int dw_wgrad_blocks(int P_out);
 // part [dw_wgrad_blocks(B*Ho*Ho)][C][k][k]
 void dw_wgrad(cudaStream_t s, const bf16* dz, const bf16* x, float* part, int B, int H, int C, int k, int S);
-// channel split of a stride-1 block input [P, 2Ch]: out[:, i] = x[:, 2i] (ld ldo), xm[:, i] = x[:, 2i+1]
-void chan_split(cudaStream_t s, const bf16* x, int P, int Ch, bf16* out, int ldo, bf16* xm);
+// channel split of a stride-1 block input [P, 2Ch] (x2): out[:, i] = x[:, 2i] (ld ldo, planes
+// oplane apart), xm[:, i] = x[:, 2i+1]; merge is its (plain bf16) backward
+void chan_split(cudaStream_t s, const bf16* x, int P, int Ch, bf16* out, int ldo, size_t oplane, bf16* xm);
 void chan_merge(cudaStream_t s, const bf16* dproj, int ldp, const bf16* dm, int P, int Ch, bf16* dx);
 // frozen head pieces
 void gap_pool(cudaStream_t s, const bf16* r, int B, int HW, int C, float* gap);

@@ -134,7 +134,7 @@ size_t Spec::input_bytes() const { return 4 * batch_elems(); }
 size_t Spec::target_bytes() const {
   return family() == NASPIPE_SPOS_CNN ? 4 * (size_t)B() : 4 * batch_elems();
 }
-size_t Spec::act_bytes(int b) const {
+size_t Spec::grad_bytes(int b) const {
   if (family() != NASPIPE_SPOS_CNN) return 4 * batch_elems();
   if (b < m()) {
     const SposDims d = spos_dims(b);
@@ -142,6 +142,9 @@ size_t Spec::act_bytes(int b) const {
   }
   const int hw = spos_last_hw();
   return 2 * (size_t)B() * hw * hw * chans.back();
+}
+size_t Spec::act_bytes(int b) const {
+  return family() == NASPIPE_SPOS_CNN ? 2 * grad_bytes(b) : grad_bytes(b);
 }
 
 // oracle/spos.py block_dims: the stem halves image_hw; the first block of every CNN stage
@@ -209,11 +212,12 @@ std::vector<SposConv> Spec::spos_convs(int b, int c) const {
   return L;
 }
 
+// bf16x2 shadow: hi planes of every 1x1 weight, then the lo planes (same offsets + half)
 size_t Spec::spos_shadow_elems(int b, int c) const {
   size_t t = 0;
   for (auto& u : spos_convs(b, c))
     if (!u.dw) t += (size_t)u.cout * u.cin;
-  return t;
+  return 2 * t;
 }
 
 size_t Spec::frozen_count(int part) const {

@@ -59,8 +59,10 @@ struct Spec {
   size_t batch_elems() const { return (size_t)B() * sample_elems(); }
   // Boundary tensors: bytes of the activation entering block b (b == m: the last block's
   // output), of the batch input and of the target.  MLP/TRANSFORMER: fp32 [B, sample];
-  // SPOS: bf16 NHWC activations, fp32 NHWC image, int32 labels.
+  // SPOS: bf16x2 NHWC activations (hi + lo planes, A28), fp32 NHWC image, int32
+  // labels.
   size_t act_bytes(int b) const;
+  size_t grad_bytes(int b) const;  // gradient w.r.t. that activation (SPOS: plain bf16)
   size_t input_bytes() const;
   size_t target_bytes() const;
   // SPOS geometry

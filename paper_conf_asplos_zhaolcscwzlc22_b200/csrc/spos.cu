@@ -1,6 +1,12 @@
-// SPOS CNN kernels (configs[1]): NHWC bf16 activations, fp32 BatchNorm statistics and
-// masters, CUDA cores for everything that is not a dense contraction (the 1x1 convs and the
-// frozen head's 1x1 conv run on the tcgen05 GEMM, gemm.cu).
+// SPOS CNN kernels (configs[1]): NHWC activations, fp32 BatchNorm statistics and masters,
+// CUDA cores for everything that is not a dense contraction (the 1x1 convs and the frozen
+// head's 1x1 conv run on the tcgen05 GEMM, gemm.cu).
+//
+// Storage (A28): forward tensors (conv outputs z, BN/ReLU outputs y, block
+// outputs) are bf16x2 -- two bf16 planes, hi = bf16(v) and lo = bf16(v - hi), lo plane at
+// `plane` elements after hi -- i.e. a 16-bit mantissa, because BatchNorm + ReLU turn any
+// 2^-9 perturbation of the forward activations into ReLU-mask flips that decorrelate the
+// weight gradient; backward tensors (dy, dz, dx) are plain bf16.
 //
 // Block internals follow SURVEY §8c "C2 SPOS candidate" (readings A16, A27):
 // every conv is bias-free and followed by training-mode BatchNorm (batch statistics over
@@ -55,6 +61,21 @@ __device__ __forceinline__ void store8(bf16* p, const float (&v)[8]) {
   q.w = ptx::pack_bf16(v[6], v[7]);
   *reinterpret_cast<uint4*>(p) = q;
 }
+// bf16x2: v = hi + lo (exact in fp32); store: hi = RNE(v), lo = RNE(v - hi)
+__device__ __forceinline__ void load8x2(const bf16* p, size_t plane, float (&v)[8]) {
+  float lo[8];
+  load8(p, v);
+  load8(p + plane, lo);
+#pragma unroll
+  for (int i = 0; i < 8; ++i) v[i] += lo[i];
+}
+__device__ __forceinline__ void store8x2(bf16* p, size_t plane, const float (&v)[8]) {
+  float lo[8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) lo[i] = v[i] - __bfloat162float(__float2bfloat16_rn(v[i]));
+  store8(p, v);
+  store8(p + plane, lo);
+}
 __device__ __forceinline__ void load8f(const float* p, float (&v)[8]) {
   const float4 a = reinterpret_cast<const float4*>(p)[0], b = reinterpret_cast<const float4*>(p)[1];
   v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w; v[4] = b.x; v[5] = b.y; v[6] = b.z; v[7] = b.w;
@@ -101,7 +122,7 @@ __global__ void stem_conv_kernel(const float* __restrict__ x, const float* __res
         for (int t = 0; t < 27; ++t) a = __fmaf_rn(in[t], wc[t], a);
         acc[i] = a;
       }
-      store8(z + p * C0 + c0, acc);
+      store8x2(z + p * C0 + c0, P * C0, acc);
     }
   }
 }
@@ -118,7 +139,7 @@ __global__ void bn_stats_kernel(const bf16* __restrict__ z, int P, int C, float*
     float s[8] = {}, q[8] = {};
     for (int row = row0 + r; row < row1; row += RP) {
       float v[8];
-      load8(z + (size_t)row * C + 8 * g, v);
+      load8x2(z + (size_t)row * C + 8 * g, (size_t)P * C, v);
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
         s[i] += v[i];
@@ -158,7 +179,8 @@ __global__ void bn_finalize_kernel(const float* __restrict__ part, int nblk, int
 
 __global__ void bn_apply_kernel(const bf16* __restrict__ z, int P, int C, const float* __restrict__ mean,
                                 const float* __restrict__ rstd, const float* __restrict__ gam,
-                                const float* __restrict__ bet, int relu, bf16* __restrict__ y, int ldy) {
+                                const float* __restrict__ bet, int relu, bf16* __restrict__ y, int ldy,
+                                size_t yplane) {
   ptx::pdl_wait();
   const int G = C / 8;
   const size_t items = (size_t)P * G;
@@ -166,7 +188,7 @@ __global__ void bn_apply_kernel(const bf16* __restrict__ z, int P, int C, const 
     const size_t p = it / G;
     const int c = (int)(it % G) * 8;
     float v[8], mu[8], rs[8], g8[8], b8[8];
-    load8(z + p * C + c, v);
+    load8x2(z + p * C + c, (size_t)P * C, v);
     load8f(mean + c, mu);
     load8f(rstd + c, rs);
     load8f(gam + c, g8);
@@ -176,17 +198,17 @@ __global__ void bn_apply_kernel(const bf16* __restrict__ z, int P, int C, const 
       const float o = bn_y(v[i], mu[i], rs[i], g8[i], b8[i]);
       v[i] = relu ? fmaxf(o, 0.f) : o;
     }
-    store8(y + p * ldy + c, v);
+    store8x2(y + p * ldy + c, yplane, v);
   }
 }
 
 // ---------------------------------------------------------------- BatchNorm backward
-__device__ __forceinline__ void bn_bwd_item(const bf16* dy, const bf16* z, const float (&mu)[8], const float (&rs)[8],
-                                            const float (&g8)[8], const float (&b8)[8], int relu, float (&d)[8],
-                                            float (&xh)[8]) {
+__device__ __forceinline__ void bn_bwd_item(const bf16* dy, const bf16* z, size_t zplane, const float (&mu)[8],
+                                            const float (&rs)[8], const float (&g8)[8], const float (&b8)[8],
+                                            int relu, float (&d)[8], float (&xh)[8]) {
   float zz[8];
   load8(dy, d);
-  load8(z, zz);
+  load8x2(z, zplane, zz);
 #pragma unroll
   for (int i = 0; i < 8; ++i) {
     xh[i] = __fmul_rn(__fsub_rn(zz[i], mu[i]), rs[i]);
@@ -212,7 +234,8 @@ __global__ void bn_bwd_reduce_kernel(const bf16* __restrict__ dy, int lddy, cons
     float s1[8] = {}, s2[8] = {};
     for (int row = row0 + r; row < row1; row += RP) {
       float d[8], xh[8];
-      bn_bwd_item(dy + (size_t)row * lddy + 8 * g, z + (size_t)row * C + 8 * g, mu, rs, g8, b8, relu, d, xh);
+      bn_bwd_item(dy + (size_t)row * lddy + 8 * g, z + (size_t)row * C + 8 * g, (size_t)P * C, mu, rs, g8, b8, relu,
+                  d, xh);
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
         s1[i] += d[i];
@@ -276,7 +299,7 @@ __global__ void bn_bwd_apply_kernel(const bf16* __restrict__ dy, int lddy, const
     load8f(old + C + c, b8);
     load8f(sums + c, m1);
     load8f(sums + C + c, m2);
-    bn_bwd_item(dy + p * lddy + c, z + p * C + c, mu, rs, g8, b8, relu, d, xh);
+    bn_bwd_item(dy + p * lddy + c, z + p * C + c, (size_t)P * C, mu, rs, g8, b8, relu, d, xh);
 #pragma unroll
     for (int i = 0; i < 8; ++i) {
       const float t = d[i] - m1[i] * invP - xh[i] * (m2[i] * invP);
@@ -314,6 +337,7 @@ __global__ void dw_fwd_kernel(const bf16* __restrict__ x, const float* __restric
     const int oh = (int)((p / Ho) % Ho);
     const int b = (int)(p / ((size_t)Ho * Ho));
     float acc[8] = {};
+    const size_t xplane = (size_t)B * H * H * C;
 #pragma unroll
     for (int u = 0; u < K; ++u) {
       const int ih = oh * S + u - PAD;
@@ -324,7 +348,7 @@ __global__ void dw_fwd_kernel(const bf16* __restrict__ x, const float* __restric
         const int iw = ow * S + v - PAD;
         if (iw < 0 || iw >= H) continue;
         float xv[8], wv[8];
-        load8(row + (size_t)iw * C, xv);
+        load8x2(row + (size_t)iw * C, xplane, xv);
         const float* wt = ws + (u * K + v) * C + c;
 #pragma unroll
         for (int i = 0; i < 8; ++i) wv[i] = wt[i];
@@ -332,7 +356,7 @@ __global__ void dw_fwd_kernel(const bf16* __restrict__ x, const float* __restric
         for (int i = 0; i < 8; ++i) acc[i] = __fmaf_rn(xv[i], wv[i], acc[i]);
       }
     }
-    store8(z + p * C + c, acc);
+    store8x2(z + p * C + c, items / G * C, acc);
   }
 }
 
@@ -433,26 +457,31 @@ __global__ void dw_wgrad_kernel(const bf16* __restrict__ dz, const bf16* __restr
 
 // ---------------------------------------------------------------- channel split / merge
 // stride-1 block input x [P, 2Ch]: out[:, i] = x[:, 2i] (passed through, ld ldo), xm[:, i] = x[:, 2i+1]
+// (all three bf16x2; x and xm planes P*2Ch and P*Ch apart, out's planes oplane apart)
 __global__ void chan_split_kernel(const bf16* __restrict__ x, int P, int Ch, bf16* __restrict__ out, int ldo,
-                                  bf16* __restrict__ xm) {
+                                  size_t oplane, bf16* __restrict__ xm) {
   ptx::pdl_wait();
   const int G = Ch / 8;
   const size_t items = (size_t)P * G;
   for (size_t it = blockIdx.x * (size_t)blockDim.x + threadIdx.x; it < items; it += (size_t)gridDim.x * blockDim.x) {
     const size_t p = it / G;
     const int g = (int)(it % G);
-    float a[8], b[8], ev[8], od[8];
-    load8(x + p * 2 * Ch + 16 * g, a);
-    load8(x + p * 2 * Ch + 16 * g + 8, b);
+    const size_t xplane = (size_t)P * 2 * Ch, mplane = (size_t)P * Ch;
 #pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      ev[i] = a[2 * i];
-      od[i] = a[2 * i + 1];
-      ev[4 + i] = b[2 * i];
-      od[4 + i] = b[2 * i + 1];
+    for (int pl = 0; pl < 2; ++pl) {  // the hi and lo planes move unchanged (exact copies)
+      float a[8], b[8], ev[8], od[8];
+      load8(x + pl * xplane + p * 2 * Ch + 16 * g, a);
+      load8(x + pl * xplane + p * 2 * Ch + 16 * g + 8, b);
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        ev[i] = a[2 * i];
+        od[i] = a[2 * i + 1];
+        ev[4 + i] = b[2 * i];
+        od[4 + i] = b[2 * i + 1];
+      }
+      store8(out + pl * oplane + p * ldo + 8 * g, ev);
+      store8(xm + pl * mplane + p * Ch + 8 * g, od);
     }
-    store8(out + p * ldo + 8 * g, ev);
-    store8(xm + p * Ch + 8 * g, od);
   }
 }
 
@@ -488,7 +517,11 @@ __global__ void gap_kernel(const bf16* __restrict__ r, int B, int HW, int C, flo
   if (i >= B * C) return;
   const int b = i / C, c = i % C;
   float s = 0.f;
-  for (int k = 0; k < HW; ++k) s += __bfloat162float(r[((size_t)b * HW + k) * C + c]);
+  const size_t plane = (size_t)B * HW * C;
+  for (int k = 0; k < HW; ++k) {
+    const size_t o = ((size_t)b * HW + k) * C + c;
+    s += __bfloat162float(r[o]) + __bfloat162float(r[o + plane]);
+  }
   gap[i] = s / (float)HW;
 }
 
@@ -605,9 +638,24 @@ void set_smem(Kern k, size_t bytes) {
   if (bytes > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
 }
 
+__global__ void f2x2_kernel(const float* __restrict__ a, bf16* __restrict__ hi, bf16* __restrict__ lo, size_t n) {
+  ptx::pdl_wait();
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+    const float v = a[i];
+    const bf16 h = __float2bfloat16_rn(v);
+    hi[i] = h;
+    lo[i] = __float2bfloat16_rn(v - __bfloat162float(h));
+  }
+}
+
 }  // namespace
 
 // ================================================================ host launchers
+void f32_to_bf16x2(cudaStream_t s, const float* w32, bf16* hi, bf16* lo, size_t n) {
+  launch_pdl(f2x2_kernel, dim3(grid_for(n)), dim3(TPB), 0, s, w32, hi, lo, n);
+  check_launch("f32_to_bf16x2");
+}
+
 int bn_part_blocks(int P) { return (P + BN_ROWS - 1) / BN_ROWS; }
 int dw_wgrad_blocks(int P_out) { return (P_out + DW_ROWS - 1) / DW_ROWS; }
 
@@ -632,9 +680,9 @@ void bn_finalize(cudaStream_t s, const float* part, int nblk, int C, int P, floa
 }
 
 void bn_apply(cudaStream_t s, const bf16* z, int P, int C, const float* mean, const float* rstd, const float* g,
-              const float* b, int relu, bf16* y, int ldy) {
+              const float* b, int relu, bf16* y, int ldy, size_t yplane) {
   launch_pdl(bn_apply_kernel, dim3(grid_for((size_t)P * (C / 8))), dim3(TPB), 0, s, z, P, C, mean, rstd, g, b, relu,
-             y, ldy);
+             y, ldy, yplane);
   check_launch("bn_apply");
 }
 
@@ -704,8 +752,9 @@ void dw_wgrad(cudaStream_t s, const bf16* dz, const bf16* x, float* part, int B,
   check_launch("dw_wgrad");
 }
 
-void chan_split(cudaStream_t s, const bf16* x, int P, int Ch, bf16* out, int ldo, bf16* xm) {
-  launch_pdl(chan_split_kernel, dim3(grid_for((size_t)P * (Ch / 8))), dim3(TPB), 0, s, x, P, Ch, out, ldo, xm);
+void chan_split(cudaStream_t s, const bf16* x, int P, int Ch, bf16* out, int ldo, size_t oplane, bf16* xm) {
+  launch_pdl(chan_split_kernel, dim3(grid_for((size_t)P * (Ch / 8))), dim3(TPB), 0, s, x, P, Ch, out, ldo, oplane,
+             xm);
   check_launch("chan_split");
 }
 

@@ -4,11 +4,12 @@
 Bars (BASELINE.json north_star; A15, A28, A29):
 * parameters: A15 metric <= 1e-3 after 1 and 8 steps, <= 1e-2 after 100 steps, against the
   plain fp64 oracle;
-* the bf16 noise floor (A28): the same oracle with its stored tensors rounded to bf16
-  (storage="bf16") is a second, equally valid bf16 computation; BatchNorm + ReLU make the
-  result chaotic under bf16 rounding (any 1-ulp difference cascades), so the GPU is required
-  to be as close to the fp64 definition as that computation is: per-candidate normwise
-  update error <= 2 x the emulation's + 0.05, and A15 <= 2 x the emulation's + 1e-4;
+* the storage noise floor (A28): the same oracle with its stored tensors rounded the way
+  the path stores them (storage="bf16x2": forward hi+lo bf16 pairs, backward bf16) is a
+  second, equally valid computation; BatchNorm + ReLU make the result chaotic under
+  rounding (one flipped ReLU mask cascades), so the GPU is required to be as close to the
+  fp64 definition as that computation is: per-candidate normwise update error <= 2 x the
+  emulation's + 0.05, and A15 <= 2 x the emulation's + 1e-4;
 * losses rtol 1e-2; schedule trace equal to the oracle's CSP plan;
 * bitwise identical across two runs and across D = 1, 2, 4 stages (Table 3).
 tiny_spos covers every candidate kind (Shuffle k = 3/5/7, Xception; stride 1 and 2),
@@ -44,12 +45,12 @@ def _run(name, choices, D=2, **kw):
     batches = [synth.make_batch(cfg, y) for y in range(len(choices))]
     theta0 = train.initial_theta(cfg)
     ref, ref_loss = train.train_sequential(cfg, theta0, choices, batches)
-    emu, _ = train.train_sequential(dict(cfg, storage="bf16"), theta0, choices, batches)
+    emu, _ = train.train_sequential(dict(cfg, storage="bf16x2"), theta0, choices, batches)
     params, losses, trace, stats = run_engine(cfg, choices, batches, D=D, **kw)
     gpu = _errors(params, ref, theta0)
     floor = _errors(emu, ref, theta0)
     print(f"{name} N={len(choices)} D={D}: gpu A15={gpu[0]:.2e} upd={gpu[1]:.2e}; "
-          f"bf16-storage oracle A15={floor[0]:.2e} upd={floor[1]:.2e}")
+          f"bf16x2-storage oracle A15={floor[0]:.2e} upd={floor[1]:.2e}")
     return cfg, gpu, floor, losses, ref_loss, trace, stats
 
 
@@ -103,5 +104,5 @@ def test_spos_full_size_one_step():
     a15, upd = _errors(params, ref, theta0)
     print(f"full-size A15={a15:.3e} upd={upd:.3e} loss {losses[0]:.6f} vs {ref_loss[0]:.6f}")
     assert a15 <= 1e-3, a15
-    assert upd <= 0.5, upd
+    assert upd <= 0.3, upd   # bf16x2-storage oracle at this size: A15 1.5e-4, update 0.10
     np.testing.assert_allclose(losses, ref_loss, rtol=1e-2)

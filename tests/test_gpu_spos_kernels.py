@@ -2,10 +2,11 @@
 
 Reference: float64 NumPy written here from the textbook definitions (depthwise conv with
 zero padding k//2, training-mode BatchNorm, its backward, the channel split of a stride-1
-ShuffleNetV2 block), evaluated on the SAME bf16-rounded inputs the kernel reads.  Bars:
-bf16 outputs within 2^-8 normwise and >= 99 % of elements within 1 bf16 ulp of the
-rounded reference; fp32 outputs (statistics, weight-gradient sums) normwise <= 1e-5;
-exact copies (split / merge) bitwise; every kernel bitwise reproducible across two runs.
+ShuffleNetV2 block), evaluated on the SAME rounded inputs the kernel reads.  Forward
+tensors are bf16x2 (hi + lo planes, A28), gradients bf16.  Bars: bf16 outputs
+within 2^-8 normwise and >= 99 % of elements within 1 bf16 ulp of the rounded reference;
+bf16x2 and fp32 outputs (statistics, weight-gradient sums) normwise <= 1e-5; exact copies
+(split / merge) bitwise; every kernel bitwise reproducible across two runs.
 Shapes include the full configs[1] block-0 geometry (P = 200704 pixels) and ragged BN row
 blocks (P not a multiple of 256).
 """
@@ -20,9 +21,10 @@ npipe = pytest.importorskip("paper_conf_asplos_zhaolcscwzlc22_b200")
 L = npipe.lib
 _vp, _i = C.c_void_p, C.c_int
 L.naspipe_debug_dw.argtypes = [_vp] * 7 + [_i] * 5 + [_vp]
-L.naspipe_debug_bn_fwd.argtypes = [_vp, _i, _i, _vp, _vp, _i, _vp, _i, _vp, _vp, _vp]
+L.naspipe_debug_bn_fwd.argtypes = [_vp, _i, _i, _vp, _vp, _i, _vp, _i, C.c_size_t, _vp, _vp, _vp]
 L.naspipe_debug_bn_bwd.argtypes = [_vp, _i, _vp, _i, _i, _vp, _vp, _vp, _vp, _i, _vp, _vp, _vp, C.c_float, _i, _vp]
-L.naspipe_debug_chan_split.argtypes = [_vp, _i, _i, _vp, _i, _vp, _vp]
+L.naspipe_debug_chan_split.argtypes = [_vp, _i, _i, _vp, _i, C.c_size_t, _vp, _vp]
+L.naspipe_debug_gemm_x2.argtypes = [_i, _i, _i, _vp, _vp, _i, _vp, _vp, _i, _vp, _vp, _vp]
 L.naspipe_debug_chan_merge.argtypes = [_vp, _i, _vp, _i, _i, _vp, _vp]
 L.naspipe_debug_stem.argtypes = [_vp, _vp, _vp, _i, _i, _i, _vp]
 
@@ -43,6 +45,24 @@ def _bf(a):
     """bf16 device tensor of a (RNE) and its exact float64 value."""
     t = torch.from_numpy(np.ascontiguousarray(a, dtype=np.float32)).to(torch.bfloat16).cuda()
     return t, _f64(t)
+
+
+def _x2(a):
+    """bf16x2 device tensor [2, *shape] (hi plane, lo plane) of a and its exact value."""
+    a = np.asarray(a, dtype=np.float32)
+    hi = torch.from_numpy(a).to(torch.bfloat16)
+    lo = (torch.from_numpy(a) - hi.float()).to(torch.bfloat16)
+    t = torch.stack([hi, lo]).cuda()
+    return t, _f64(t[0]) + _f64(t[1])
+
+
+def _v2(t):
+    """value of a bf16x2 tensor [2, ...]"""
+    return _f64(t[0]) + _f64(t[1])
+
+
+def _check_x2(got, ref, tol=1e-5):
+    assert np.max(np.abs(got - ref)) / max(np.max(np.abs(ref)), 1e-30) <= tol
 
 
 def _check_bf16(got, ref):
@@ -86,13 +106,14 @@ def _dw_bwd_ref(x, w, s, dz):
                                         (4, 6, 320, 7, 2), (64, 112, 16, 3, 2)])
 def test_depthwise_fwd_dgrad_wgrad(B, H, Cc, k, s):
     rng = np.random.default_rng(B * 100 + H + Cc + k)
-    xd, x = _bf(rng.standard_normal((B, H, H, Cc)))
+    xd, x = _x2(rng.standard_normal((B, H, H, Cc)))
+    x_hi = _f64(xd[0])
     w = (rng.standard_normal((Cc, k, k)) / k).astype(np.float32)
     wd = torch.from_numpy(w).cuda()
     Ho = (H - 1) // s + 1
     dzd, dz = _bf(rng.standard_normal((B, Ho, Ho, Cc)))
     addd, add = _bf(rng.standard_normal((B, H, H, Cc)))
-    z = torch.empty((B, Ho, Ho, Cc), dtype=torch.bfloat16, device="cuda")
+    z = torch.empty((2, B, Ho, Ho, Cc), dtype=torch.bfloat16, device="cuda")
     dx = torch.empty((B, H, H, Cc), dtype=torch.bfloat16, device="cuda")
     dws = torch.empty((Cc, k, k), dtype=torch.float32, device="cuda")
     outs = []
@@ -104,13 +125,14 @@ def test_depthwise_fwd_dgrad_wgrad(B, H, Cc, k, s):
         assert torch.equal(a, b)
     if B * H * H > 100000:   # full-size block 0: check the reductions on a sample of channels
         ch = [0, 7, 15]
-        x, dz, add, w64 = x[..., ch], dz[..., ch], add[..., ch], w[ch].astype(np.float64)
-        got_z, got_dx, got_dw = _f64(z)[..., ch], _f64(dx)[..., ch], _f64(dws)[ch]
+        x, x_hi, dz, add, w64 = x[..., ch], x_hi[..., ch], dz[..., ch], add[..., ch], w[ch].astype(np.float64)
+        got_z, got_dx, got_dw = _v2(z)[..., ch], _f64(dx)[..., ch], _f64(dws)[ch]
     else:
         w64 = w.astype(np.float64)
-        got_z, got_dx, got_dw = _f64(z), _f64(dx), _f64(dws)
-    _check_bf16(got_z, _dw_ref(x, w64, s))
-    rdx, rdw = _dw_bwd_ref(x, w64, s, dz)
+        got_z, got_dx, got_dw = _v2(z), _f64(dx), _f64(dws)
+    _check_x2(got_z, _dw_ref(x, w64, s))
+    rdx, _ = _dw_bwd_ref(x, w64, s, dz)
+    _, rdw = _dw_bwd_ref(x_hi, w64, s, dz)     # the weight gradient reads the hi plane
     _check_bf16(got_dx, rdx + add)
     assert np.max(np.abs(got_dw - rdw)) / np.max(np.abs(rdw)) <= 1e-5
 
@@ -128,21 +150,22 @@ def _bn_ref(z, g, b, relu):
                                        (200704, 32, 0)])
 def test_batchnorm_fwd_bwd(P, Cc, relu):
     rng = np.random.default_rng(P + Cc)
-    zd, z = _bf(rng.standard_normal((P, Cc)) * rng.uniform(0.5, 2.0, Cc) + rng.uniform(-1, 1, Cc))
+    zd, z = _x2(rng.standard_normal((P, Cc)) * rng.uniform(0.5, 2.0, Cc) + rng.uniform(-1, 1, Cc))
     g = rng.uniform(0.5, 1.5, Cc).astype(np.float32)
     b = rng.uniform(-0.3, 0.3, Cc).astype(np.float32)
     gd, bd = torch.from_numpy(g).cuda(), torch.from_numpy(b).cuda()
     ld = Cc + 16   # the output is a column slice of a wider tensor (block-output concat)
-    y = torch.zeros((P, ld), dtype=torch.bfloat16, device="cuda")
+    y = torch.zeros((2, P, ld), dtype=torch.bfloat16, device="cuda")
     mean = torch.empty(Cc, device="cuda")
     rstd = torch.empty(Cc, device="cuda")
-    _ok(L.naspipe_debug_bn_fwd(_p(zd), P, Cc, _p(gd), _p(bd), relu, _p(y[:, 8:]), ld, _p(mean), _p(rstd), None))
+    _ok(L.naspipe_debug_bn_fwd(_p(zd), P, Cc, _p(gd), _p(bd), relu, _p(y[0, :, 8:]), ld, P * ld, _p(mean), _p(rstd),
+                               None))
     torch.cuda.synchronize()
     ry, mu, rs, xh = _bn_ref(z, g.astype(np.float64), b.astype(np.float64), relu)
     assert np.max(np.abs(_f64(mean) - mu)) <= 1e-5 * max(1.0, np.max(np.abs(mu)))
     assert np.max(np.abs(_f64(rstd) / rs - 1)) <= 1e-5
-    yy = _f64(y)
-    _check_bf16(yy[:, 8:8 + Cc], ry)
+    yy = _v2(y)
+    _check_x2(yy[:, 8:8 + Cc], ry)
     assert not yy[:, :8].any() and not yy[:, 8 + Cc:].any()
     # backward with a strided incoming gradient
     dyfull_d, dyfull = _bf(rng.standard_normal((P, ld)))
@@ -174,20 +197,23 @@ def test_batchnorm_fwd_bwd(P, Cc, relu):
 @pytest.mark.parametrize("P,Ch", [(7, 16), (3136, 320), (1000, 80)])
 def test_channel_split_merge_exact(P, Ch):
     rng = np.random.default_rng(P)
-    xd, x = _bf(rng.standard_normal((P, 2 * Ch)))
-    out = torch.zeros((P, 2 * Ch), dtype=torch.bfloat16, device="cuda")
-    xm = torch.empty((P, Ch), dtype=torch.bfloat16, device="cuda")
-    _ok(L.naspipe_debug_chan_split(_p(xd), P, Ch, _p(out), 2 * Ch, _p(xm), None))
+    xd, _ = _x2(rng.standard_normal((P, 2 * Ch)))
+    out = torch.zeros((2, P, 2 * Ch), dtype=torch.bfloat16, device="cuda")
+    xm = torch.empty((2, P, Ch), dtype=torch.bfloat16, device="cuda")
+    _ok(L.naspipe_debug_chan_split(_p(xd), P, Ch, _p(out), 2 * Ch, P * 2 * Ch, _p(xm), None))
+    gd, g = _bf(rng.standard_normal((P, 2 * Ch)))
     dmd, dm = _bf(rng.standard_normal((P, Ch)))
     dx = torch.empty((P, 2 * Ch), dtype=torch.bfloat16, device="cuda")
-    _ok(L.naspipe_debug_chan_merge(_p(xd), 2 * Ch, _p(dmd), P, Ch, _p(dx), None))
+    _ok(L.naspipe_debug_chan_merge(_p(gd), 2 * Ch, _p(dmd), P, Ch, _p(dx), None))
     torch.cuda.synchronize()
-    o = _f64(out)
-    np.testing.assert_array_equal(o[:, :Ch], x[:, 0::2])
-    assert not o[:, Ch:].any()
-    np.testing.assert_array_equal(_f64(xm), x[:, 1::2])
+    for pl in range(2):   # both planes are exact copies
+        x = _f64(xd[pl])
+        o = _f64(out[pl])
+        np.testing.assert_array_equal(o[:, :Ch], x[:, 0::2])
+        assert not o[:, Ch:].any()
+        np.testing.assert_array_equal(_f64(xm[pl]), x[:, 1::2])
     r = np.empty((P, 2 * Ch))
-    r[:, 0::2] = x[:, :Ch]
+    r[:, 0::2] = g[:, :Ch]
     r[:, 1::2] = dm
     np.testing.assert_array_equal(_f64(dx), r)
 
@@ -197,7 +223,7 @@ def test_stem_conv():
     B, H, C0 = 2, 32, 16
     x = rng.standard_normal((B, H, H, 3)).astype(np.float32)
     w = (rng.standard_normal((C0, 3, 3, 3)) / 5).astype(np.float32)
-    z = torch.empty((B, H // 2, H // 2, C0), dtype=torch.bfloat16, device="cuda")
+    z = torch.empty((2, B, H // 2, H // 2, C0), dtype=torch.bfloat16, device="cuda")
     xd, wd = torch.from_numpy(x).cuda(), torch.from_numpy(w).cuda()   # keep both alive during the launch
     _ok(L.naspipe_debug_stem(_p(xd), _p(wd), _p(z), B, H, C0, None))
     torch.cuda.synchronize()
@@ -206,4 +232,21 @@ def test_stem_conv():
     for u in range(3):
         for v in range(3):
             ref += xp[:, u:u + H - 1:2, v:v + H - 1:2, :] @ w[:, u, v, :].T.astype(np.float64)
-    _check_bf16(_f64(z), ref)
+    _check_x2(_v2(z), ref)
+
+
+@pytest.mark.parametrize("M,N,K", [(128, 64, 64), (200, 48, 16), (3136, 1024, 640), (1000, 320, 160), (512, 144, 96)])
+def test_gemm_bf16x2_three_pass(M, N, K):
+    """z = x W^T on bf16x2 planes: error of the dropped lo*lo term and fp32 accumulation only."""
+    rng = np.random.default_rng(M + N + K)
+    ad, a = _x2(np.maximum(rng.standard_normal((M, K)), 0))
+    bd, b = _x2(rng.standard_normal((N, K)) / np.sqrt(K))
+    out = torch.empty((2, M, N), dtype=torch.bfloat16, device="cuda")
+    res = []
+    for _ in range(2):
+        _ok(L.naspipe_debug_gemm_x2(M, N, K, _p(ad[0]), _p(ad[1]), K, _p(bd[0]), _p(bd[1]), K, _p(out[0]),
+                                    _p(out[1]), None))
+        torch.cuda.synchronize()
+        res.append(out.clone())
+    assert torch.equal(res[0], res[1])
+    _check_x2(_v2(out), a @ b.T)

@@ -141,3 +141,31 @@ def test_tiny_spos_training_updates_only_active():
     for k in th:
         changed = not np.array_equal(th[k], th0[k].astype(np.float64))
         assert changed == (k in used), k
+
+
+def test_storage_rounding_pins():
+    """spos.to_bf16 is round-to-nearest-even to bfloat16 (ties, carries, sign, against torch's
+    independent conversion); to_bf16x2 keeps 16 mantissa bits; PLAIN storage is the identity."""
+    torch = pytest.importorskip("torch")
+    assert spos.to_bf16(1 + 2.0 ** -8) == 1.0                     # tie -> even (down)
+    assert spos.to_bf16(1 + 3 * 2.0 ** -8) == 1 + 2.0 ** -6       # tie -> even (up)
+    assert spos.to_bf16(-(1 + 2.0 ** -7 + 2.0 ** -9)) == -(1 + 2.0 ** -7)
+    assert spos.to_bf16(2.0 - 2.0 ** -9) == 2.0                   # carry into the exponent
+    x = np.random.default_rng(0).standard_normal(10000) * 10.0 ** np.random.default_rng(1).integers(-20, 20, 10000)
+    ref = torch.from_numpy(x.astype(np.float32)).to(torch.bfloat16).to(torch.float64).numpy()
+    np.testing.assert_array_equal(spos.to_bf16(x), ref)
+    x2 = spos.to_bf16x2(x)
+    assert np.all(np.abs(x2 - x.astype(np.float32)) <= 2.0 ** -16 * np.abs(x))
+    assert spos.PLAIN.f(x) is x and spos.STORAGE[None] is spos.PLAIN
+
+
+def test_storage_modes_only_round():
+    """The storage modes change the result only by rounding: one tiny_spos step in BF16X2
+    storage stays within 1e-3 of the plain loss and differs from it (the rounding is applied)."""
+    cfg = synth.get_config("tiny_spos")
+    ch = synth.sample_choices(1, cfg["n_blocks"], cfg["n_choices"])
+    b = [synth.make_batch(cfg, 0)]
+    th0 = train.initial_theta(cfg)
+    _, l0 = train.train_sequential(cfg, th0, ch, b)
+    _, l1 = train.train_sequential(dict(cfg, storage="bf16x2"), th0, ch, b)
+    assert l0[0] != l1[0] and abs(l1[0] - l0[0]) <= 1e-3 * l0[0]
