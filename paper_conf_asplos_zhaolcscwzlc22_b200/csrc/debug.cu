@@ -109,7 +109,7 @@ int naspipe_debug_dw(const void* x, const float* w, void* z, const void* dz, con
     if (x && z) dw_fwd(s, (const bf16*)x, w, (bf16*)z, B, H, C, k, S);
     if (dz && dx) dw_dgrad(s, (const bf16*)dz, w, (const bf16*)add, (bf16*)dx, B, H, C, k, S);
     if (dz && x && dwsum) {
-      const int Ho = (H - 1) / S + 1, nblk = dw_wgrad_blocks(B * Ho * Ho);
+      const int nblk = dw_wgrad_blocks(B, H, C, k, S);
       float* part = nullptr;
       NP_REQUIRE(cudaMalloc(&part, (size_t)nblk * C * k * k * 4) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
       dw_wgrad(s, (const bf16*)dz, (const bf16*)x, part, B, H, C, k, S);
@@ -125,14 +125,17 @@ int naspipe_debug_bn_fwd(const void* z, int P, int C, const float* g, const floa
                          size_t yplane, float* mean, float* rstd, void* stream) {
   return dguard([&] {
     cudaStream_t s = (cudaStream_t)stream;
-    const int nblk = bn_part_blocks(P);
+    const int nblk = bn_part_blocks(P, C);
     float* part = nullptr;
+    int* ctr = nullptr;
     NP_REQUIRE(cudaMalloc(&part, (size_t)nblk * 2 * C * 4) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
-    bn_stats(s, (const bf16*)z, P, C, part);
-    bn_finalize(s, part, nblk, C, P, mean, rstd);
+    NP_REQUIRE(cudaMalloc(&ctr, 4) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
+    cudaMemsetAsync(ctr, 0, 4, s);
+    bn_stats(s, (const bf16*)z, P, C, part, ctr, mean, rstd);
     bn_apply(s, (const bf16*)z, P, C, mean, rstd, g, b, relu, (bf16*)y, ldy, yplane);
     cudaStreamSynchronize(s);
     cudaFree(part);
+    cudaFree(ctr);
   });
 }
 
@@ -141,14 +144,18 @@ int naspipe_debug_bn_bwd(const void* dy, int lddy, const void* z, int P, int C, 
                          int update, void* stream) {
   return dguard([&] {
     cudaStream_t s = (cudaStream_t)stream;
-    const int nblk = bn_part_blocks(P);
+    const int nblk = bn_part_blocks(P, C);
     float* part = nullptr;
+    int* ctr = nullptr;
     NP_REQUIRE(cudaMalloc(&part, (size_t)nblk * 2 * C * 4) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
-    bn_bwd_reduce(s, (const bf16*)dy, lddy, (const bf16*)z, P, C, mean, rstd, g, b, relu, part);
-    bn_bwd_finalize(s, part, nblk, C, sums, old, g, b, lr, update);
+    NP_REQUIRE(cudaMalloc(&ctr, 4) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
+    cudaMemsetAsync(ctr, 0, 4, s);
+    bn_bwd_reduce(s, (const bf16*)dy, lddy, (const bf16*)z, P, C, mean, rstd, g, b, relu, part, ctr, sums, old, lr,
+                  update);
     bn_bwd_apply(s, (const bf16*)dy, lddy, (const bf16*)z, P, C, mean, rstd, old, sums, relu, (bf16*)dz);
     cudaStreamSynchronize(s);
     cudaFree(part);
+    cudaFree(ctr);
   });
 }
 

@@ -57,10 +57,10 @@ class SposFamily : public Family {
           st += 2 * (size_t)u.cout;
           dz_max = std::max(dz_max, po * u.cout);
           g_max = std::max({g_max, pi * u.cin, po * u.cout});
-          part_max = std::max(part_max, (size_t)bn_part_blocks((int)po) * 2 * u.cout);
+          part_max = std::max(part_max, (size_t)bn_part_blocks((int)po, u.cout) * 2 * u.cout);
           C_max = std::max(C_max, (size_t)u.cout);
           if (u.dw)
-            dwp_max = std::max(dwp_max, (size_t)dw_wgrad_blocks((int)po) * u.cout * u.k * u.k);
+            dwp_max = std::max(dwp_max, (size_t)dw_wgrad_blocks(B_, u.H_in, u.cout, u.k, u.stride) * u.cout * u.k * u.k);
           else
             ws_elems_ = std::max(ws_elems_, (size_t)gemm_splitk_factor(u.cout, u.cin, (int)po) * u.cout * u.cin);
         }
@@ -72,11 +72,11 @@ class SposFamily : public Family {
               Cl = spec.chans.back(), Ch = spec.raw.head_channels, ncls = spec.raw.num_classes;
     if (last_) {
       const size_t PL = P(hwl);
-      part_max = std::max(part_max, (size_t)bn_part_blocks((int)PL) * 2 * Ch);
+      part_max = std::max(part_max, (size_t)bn_part_blocks((int)PL, Ch) * 2 * Ch);
       C_max = std::max(C_max, (size_t)Ch);
     }
     if (first_) {
-      part_max = std::max(part_max, (size_t)bn_part_blocks((int)P(hw0)) * 2 * C0);
+      part_max = std::max(part_max, (size_t)bn_part_blocks((int)P(hw0), C0) * 2 * C0);
       C_max = std::max(C_max, (size_t)C0);
     }
     stash_.resize((size_t)W * nb);
@@ -91,7 +91,13 @@ class SposFamily : public Family {
         stats_[k] = A.alloc<float>(stats_max);
         if (j < nb - 1) act_[k] = A.alloc<bf16>(spec.act_bytes(blocks[j] + 1) / 2);
       }
-    dz_ = A.alloc<bf16>(dz_max);
+    for (auto& d : dz_) d = A.alloc<bf16>(dz_max);
+    cudaStreamCreateWithFlags(&side_, cudaStreamNonBlocking);
+    for (int i = 0; i < kRing; ++i) {
+      cudaEventCreateWithFlags(&ev_dg_[i], cudaEventDisableTiming);
+      cudaEventCreateWithFlags(&ev_wg_[i], cudaEventDisableTiming);
+    }
+    cudaEventCreateWithFlags(&ev_join_, cudaEventDisableTiming);
     g_[0] = A.alloc<bf16>(g_max);
     g_[1] = A.alloc<bf16>(g_max);
     gb_[0] = A.alloc<bf16>(blk_max);
@@ -101,6 +107,9 @@ class SposFamily : public Family {
     dwpart_ = A.alloc<float>(std::max<size_t>(dwp_max, 1));
     ws_ = A.alloc<float>(std::max<size_t>(ws_elems_, 4));
     sums_ = A.alloc<float>(2 * C_max);
+    ctr_ = A.alloc<int>(1);
+    cudaMemset(ctr_, 0, sizeof(int));
+
     old_ = A.alloc<float>(2 * C_max);
     if (first_) {
       std::vector<float> h(spec.frozen_count(0));
@@ -146,6 +155,7 @@ class SposFamily : public Family {
       gap_ = A.alloc<float>((size_t)B_ * Ch);
       dgap_ = A.alloc<float>((size_t)B_ * Ch);
       dlogits_ = A.alloc<float>((size_t)B_ * ncls);
+      logits_ = A.alloc<float>((size_t)B_ * ncls);
       loss_per_ = A.alloc<float>(B_);
     }
     (void)Cl;
@@ -172,8 +182,7 @@ class SposFamily : public Family {
       const int H = spec_.raw.image_hw, C0 = spec_.raw.stem_channels;
       const int Po = (int)P(H / 2);
       spos_stem_conv(s, static_cast<const float*>(x_in), w_stem_, stem_z_, B_, H, C0);
-      bn_stats(s, stem_z_, Po, C0, part_);
-      bn_finalize(s, part_, bn_part_blocks(Po), C0, Po, stem_mean_, stem_rstd_);
+      bn_stats(s, stem_z_, Po, C0, part_, ctr_, stem_mean_, stem_rstd_);
       bn_apply(s, stem_z_, Po, C0, stem_mean_, stem_rstd_, ones_s_, zeros_s_, 1, stem_y_[slot], C0, (size_t)Po * C0);
       counters.launches += 4;
       x = stem_y_[slot];
@@ -199,6 +208,19 @@ class SposFamily : public Family {
       block_bwd(j, c, k, g, out, need_dx, s);
       g = out;
     }
+    // the task ends when its weight updates have landed (the next task may read them)
+    cudaEventRecord(ev_join_, side_);
+    cudaStreamWaitEvent(s, ev_join_, 0);
+  }
+
+  ~SposFamily() override {
+    cudaStreamSynchronize(side_);
+    for (int i = 0; i < kRing; ++i) {
+      cudaEventDestroy(ev_dg_[i]);
+      cudaEventDestroy(ev_wg_[i]);
+    }
+    cudaEventDestroy(ev_join_);
+    cudaStreamDestroy(side_);
   }
 
   // Frozen head: pw Clast->Ch (tcgen05) -> BN(1,0) -> ReLU -> GAP -> FC (fp32) -> mean CE,
@@ -206,22 +228,20 @@ class SposFamily : public Family {
   void loss(int, const void* out, const void* target, void* dy, float* loss_dst, cudaStream_t s) override {
     const int hw = spec_.spos_last_hw(), HW = hw * hw, Cl = spec_.chans.back(), Ch = spec_.raw.head_channels,
               ncls = spec_.raw.num_classes;
-    const int PL = (int)P(hw), nblk = bn_part_blocks(PL);
+    const int PL = (int)P(hw);
     GemmEpiParams e;
     e.out = zh_;
     e.out2 = zh_ + (size_t)PL * Ch;
     const bf16* xo = static_cast<const bf16*>(out);
     gemm_x2(s, PL, Ch, Cl, xo, xo + (size_t)PL * Cl, Cl, wh16_, wh16_ + (size_t)Ch * Cl, Cl, e);
-    bn_stats(s, zh_, PL, Ch, part_);
-    bn_finalize(s, part_, nblk, Ch, PL, hmean_, hrstd_);
+    bn_stats(s, zh_, PL, Ch, part_, ctr_, hmean_, hrstd_);
     bn_apply(s, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, 1, rh_, Ch, (size_t)PL * Ch);
     gap_pool(s, rh_, B_, HW, Ch, gap_);
-    fc_ce(s, gap_, wf_, static_cast<const int*>(target), B_, Ch, ncls, dlogits_, loss_per_);
+    fc_ce(s, gap_, wf_, static_cast<const int*>(target), B_, Ch, ncls, logits_, dlogits_, loss_per_);
     ce_mean(s, loss_per_, B_, loss_dst);
     fc_dgap(s, dlogits_, wf_, B_, Ch, ncls, dgap_);
     head_bcast(s, dgap_, B_, HW, Ch, rh_);  // dr overwrites r (the mask is recomputed from z)
-    bn_bwd_reduce(s, rh_, Ch, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, 1, part_);
-    bn_bwd_finalize(s, part_, nblk, Ch, sums_, old_, ones_, zeros_, 0.f, 0);
+    bn_bwd_reduce(s, rh_, Ch, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, 1, part_, ctr_, sums_, old_, 0.f, 0);
     bn_bwd_apply(s, rh_, Ch, zh_, PL, Ch, hmean_, hrstd_, old_, sums_, 1, dzh_);
     e = GemmEpiParams();
     e.out = dy;
@@ -305,8 +325,7 @@ class SposFamily : public Family {
         e.out2 = r.z + zplane;
         gemm_x2(s, Po, u.cout, u.cin, h, h + hplane, u.cin, W16 + u.off_w16, W16 + half + u.off_w16, u.cin, e);
       }
-      bn_stats(s, r.z, Po, u.cout, part_);
-      bn_finalize(s, part_, bn_part_blocks(Po), u.cout, Po, r.mean, r.rstd);
+      bn_stats(s, r.z, Po, u.cout, part_, ctr_, r.mean, r.rstd);
       bf16* y;
       int ldy;
       size_t yplane;
@@ -328,42 +347,54 @@ class SposFamily : public Family {
     }
   }
 
-  // One unit's BN backward (+ the WRITE of its gamma/beta), leaves dz in dz_.
+  // One unit's BN backward (+ the WRITE of its gamma/beta), leaves dz in the next ring
+  // buffer dz_[ring_] (whose previous reader, a weight-gradient on the side stream, is done).
   void unit_bn_bwd(const SposConv& u, const UnitRec& r, float* Pm, const bf16* dy, int lddy, cudaStream_t s) {
     const int Po = (int)P(u.H_out);
-    bn_bwd_reduce(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, u.relu, part_);
-    bn_bwd_finalize(s, part_, bn_part_blocks(Po), u.cout, sums_, old_, Pm + u.off_g, Pm + u.off_b, lr_, 1);
-    bn_bwd_apply(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, old_, sums_, u.relu, dz_);
+    ring_ = (ring_ + 1) % kRing;
+    if (ring_used_[ring_]) cudaStreamWaitEvent(s, ev_wg_[ring_], 0);
+    bn_bwd_reduce(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, u.relu, part_, ctr_, sums_,
+                  old_, lr_, 1);
+    bn_bwd_apply(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, old_, sums_, u.relu, dz_[ring_]);
     counters.launches += 3;
   }
 
-  // conv backward of one unit from dz_: dgrad into dst (+ add) with the pre-update weights
-  // (skipped if dst == nullptr), then the weight gradient with the SGD WRITE.
+  // conv backward of one unit from dz: the input gradient into dst (+ add) with the
+  // pre-update weights on the stage stream (skipped if dst == nullptr); then, on the side
+  // stream once that has been issued, the weight gradient with the SGD WRITE (reading A4),
+  // overlapping the rest of the input-gradient chain.
   void unit_conv_bwd(const SposConv& u, const UnitRec& r, float* Pm, bf16* W16, size_t half, bf16* dst,
                      const bf16* add, cudaStream_t s) {
     const int Po = (int)P(u.H_out);
-    if (u.dw) {
-      if (dst) {
-        dw_dgrad(s, dz_, Pm + u.off_w, add, dst, B_, u.H_in, u.cin, u.k, u.stride);
+    const bf16* dz = dz_[ring_];
+    if (dst) {
+      if (u.dw) {
+        dw_dgrad(s, dz, Pm + u.off_w, add, dst, B_, u.H_in, u.cin, u.k, u.stride);
         counters.launches++;
-      }
-      dw_wgrad(s, dz_, r.x, dwpart_, B_, u.H_in, u.cin, u.k, u.stride);
-      sgd_from_partials(s, Pm + u.off_w, dwpart_, dw_wgrad_blocks(Po), u.cout * u.k * u.k, lr_);
-      counters.launches += 2;
-    } else {
-      NP_REQUIRE(add == nullptr, NASPIPE_EINTERNAL, "pw dgrad with an addend");
-      if (dst) {
+      } else {
+        NP_REQUIRE(add == nullptr, NASPIPE_EINTERNAL, "pw dgrad with an addend");
         GemmEpiParams e;
         e.out = dst;
-        gemm(s, Po, u.cin, u.cout, dz_, false, u.cout, W16 + u.off_w16, true, u.cin, EPI_BF16, e);
+        gemm(s, Po, u.cin, u.cout, dz, false, u.cout, W16 + u.off_w16, true, u.cin, EPI_BF16, e);
       }
+    }
+    cudaEventRecord(ev_dg_[ring_], s);
+    cudaStreamWaitEvent(side_, ev_dg_[ring_], 0);
+    if (u.dw) {
+      dw_wgrad(side_, dz, r.x, dwpart_, B_, u.H_in, u.cin, u.k, u.stride);
+      sgd_from_partials(side_, Pm + u.off_w, dwpart_, dw_wgrad_blocks(B_, u.H_in, u.cout, u.k, u.stride),
+                        u.cout * u.k * u.k, lr_);
+      counters.launches += 2;
+    } else {
       GemmEpiParams e;
       e.w32 = Pm + u.off_w;
       e.w16 = W16 + u.off_w16;
       e.w16lo = W16 + half + u.off_w16;
       e.lr = lr_;
-      gemm(s, u.cout, u.cin, Po, dz_, true, u.cout, r.x, true, u.cin, EPI_SGD, e, true);
+      gemm(side_, u.cout, u.cin, Po, dz, true, u.cout, r.x, true, u.cin, EPI_SGD, e, true);
     }
+    cudaEventRecord(ev_wg_[ring_], side_);
+    ring_used_[ring_] = true;
   }
 
   void block_bwd(int j, int c, size_t k, const bf16* dyb, bf16* dxb, bool need_dx, cudaStream_t s) {
@@ -424,8 +455,14 @@ class SposFamily : public Family {
   std::vector<float*> stats_;
   std::vector<std::vector<UnitRec>> recs_;
   std::vector<const bf16*> xin_;
-  bf16 *dz_, *g_[2], *gb_[2], *gfirst_;
+  static constexpr int kRing = 3;  // dz buffers shared by the stage stream and the side stream
+  bf16 *dz_[kRing], *g_[2], *gb_[2], *gfirst_;
+  int ring_ = 0;
+  bool ring_used_[kRing] = {false, false, false};
+  cudaStream_t side_ = nullptr;  // weight gradients + SGD of the backward
+  cudaEvent_t ev_dg_[kRing], ev_wg_[kRing], ev_join_;
   float *part_, *dwpart_, *ws_, *sums_, *old_;
+  int* ctr_;  // last-CTA ticket of the BN reductions (stage stream)
   size_t ws_elems_ = 0;
   // stem
   float* w_stem_ = nullptr;
@@ -435,7 +472,7 @@ class SposFamily : public Family {
   // head
   bf16 *wh16_ = nullptr, *zh_ = nullptr, *rh_ = nullptr, *dzh_ = nullptr;
   float *wf_ = nullptr, *ones_ = nullptr, *zeros_ = nullptr, *hmean_ = nullptr, *hrstd_ = nullptr, *gap_ = nullptr,
-        *dgap_ = nullptr, *dlogits_ = nullptr, *loss_per_ = nullptr;
+        *dgap_ = nullptr, *dlogits_ = nullptr, *logits_ = nullptr, *loss_per_ = nullptr;
 };
 
 }  // namespace

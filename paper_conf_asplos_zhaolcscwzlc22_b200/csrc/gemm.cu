@@ -341,16 +341,32 @@ __global__ void __launch_bounds__(THREADS, 1)
 }
 
 // Fixed-order sum of the split-K partial tiles, then the final epilogue (EPI_F32 / EPI_SGD).
+// L lanes (a power of two, L | 32) per float4 of output: lane j sums slices j, j+L, ... in
+// order, the lanes are combined by a fixed xor tree; L = 1 (plain slice order) for <= 4
+// slices, so the transformer's wgrads keep their order.
+__device__ __forceinline__ float4 f4add(float4 a, float4 b) { return make_float4(a.x + b.x, a.y + b.y, a.z + b.z, a.w + b.w); }
 template <int EPI>
-__global__ void splitk_reduce_kernel(int M, int N, int splits, GemmEpiParams ep) {
+__global__ void splitk_reduce_kernel(int M, int N, int splits, int L, GemmEpiParams ep) {
   ptx::pdl_wait();
   const size_t total = (size_t)M * N / 4;
-  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < total; i += (size_t)gridDim.x * blockDim.x) {
-    float4 acc = reinterpret_cast<const float4*>(ep.ws)[i];
-    for (int k = 1; k < splits; ++k) {
-      const float4 p = reinterpret_cast<const float4*>(ep.ws + (size_t)k * ep.ws_stride)[i];
-      acc.x += p.x; acc.y += p.y; acc.z += p.z; acc.w += p.w;
+  const int j = threadIdx.x % L;
+  const size_t per_block = blockDim.x / L;
+  for (size_t i = blockIdx.x * per_block + threadIdx.x / L; i - threadIdx.x / L < total; i += (size_t)gridDim.x * per_block) {
+    const bool ok = i < total;
+    float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (ok) {
+      acc = reinterpret_cast<const float4*>(ep.ws + (size_t)j * ep.ws_stride)[i];
+      for (int k = j + L; k < splits; k += L) acc = f4add(acc, reinterpret_cast<const float4*>(ep.ws + (size_t)k * ep.ws_stride)[i]);
     }
+    for (int o = 1; o < L; o <<= 1) {
+      float4 t;
+      t.x = __shfl_xor_sync(0xffffffffu, acc.x, o);
+      t.y = __shfl_xor_sync(0xffffffffu, acc.y, o);
+      t.z = __shfl_xor_sync(0xffffffffu, acc.z, o);
+      t.w = __shfl_xor_sync(0xffffffffu, acc.w, o);
+      acc = (j & o) ? f4add(t, acc) : f4add(acc, t);  // same operand order on both partners
+    }
+    if (!ok || j != 0) continue;
     if constexpr (EPI == EPI_F32) {
       reinterpret_cast<float4*>(ep.out)[i] = acc;
     } else {
@@ -500,9 +516,13 @@ void gemm_bf16_tc(cudaStream_t s, int M, int N, int K, const bf16* A, bool a_mn,
   else if (a_mn && b_mn) dispatch_epi<true, true>(s, M, N, ts, ta, tb, run_epi, ep);
   else dispatch_epi<true, false>(s, M, N, ts, ta, tb, run_epi, ep);
   if (ts.splits > 1) {
-    const int blocks = std::min<size_t>(((size_t)M * N / 4 + 255) / 256, 4 * (size_t)num_sms());
-    if (epi == EPI_F32) launch_pdl(splitk_reduce_kernel<EPI_F32>, dim3(blocks), dim3(256), 0, s, M, N, ts.splits, ep);
-    else launch_pdl(splitk_reduce_kernel<EPI_SGD>, dim3(blocks), dim3(256), 0, s, M, N, ts.splits, ep);
+    const int L = ts.splits <= 4 ? 1 : std::min(32, ts.splits / 4);
+    const size_t per_block = 256 / L;
+    const int blocks = (int)std::min<size_t>(((size_t)M * N / 4 + per_block - 1) / per_block, 4 * (size_t)num_sms());
+    if (epi == EPI_F32)
+      launch_pdl(splitk_reduce_kernel<EPI_F32>, dim3(blocks), dim3(256), 0, s, M, N, ts.splits, L, ep);
+    else
+      launch_pdl(splitk_reduce_kernel<EPI_SGD>, dim3(blocks), dim3(256), 0, s, M, N, ts.splits, L, ep);
   }
 }
 

@@ -121,18 +121,20 @@ void mlp_bwd_sgd(cudaStream_t s, const float* x, const float* h, const float* dy
 void f32_to_bf16x2(cudaStream_t s, const float* w32, bf16* hi, bf16* lo, size_t n);
 // frozen stem: x fp32 [B,H,H,3], w fp32 [C0][3][3][3], stride 2, pad 1 -> z x2 [B,H/2,H/2,C0]
 void spos_stem_conv(cudaStream_t s, const float* x, const float* w, bf16* z, int B, int H, int C0);
-// BatchNorm (training mode, biased variance, eps 1e-5).  part: [bn_part_blocks(P)][2][C]
-int bn_part_blocks(int P);
-void bn_stats(cudaStream_t s, const bf16* z, int P, int C, float* part);
-void bn_finalize(cudaStream_t s, const float* part, int nblk, int C, int P, float* mean, float* rstd);
+// BatchNorm (training mode, biased variance, eps 1e-5).  part: [bn_part_blocks(P, C)][2][C]
+// workspace (per-row-block partial sums, then a parallel finalize kernel summing them in
+// block order in fp64); ctr: reserved (an int that is 0 between launches).
+int bn_part_blocks(int P, int C);
+// mean, rstd of z (x2) over its P rows
+void bn_stats(cudaStream_t s, const bf16* z, int P, int C, float* part, int* ctr, float* mean, float* rstd);
 // y[p*ldy + c] = relu?(g (z - mean) rstd + b); z x2 (plane P*C), y x2 (planes yplane apart)
 void bn_apply(cudaStream_t s, const bf16* z, int P, int C, const float* mean, const float* rstd, const float* g,
               const float* b, int relu, bf16* y, int ldy, size_t yplane);
+// sums [2][C] = (sum dy', sum dy' xh) (dy' = dy masked by the ReLU); old [2][C] = (g, b)
+// before the update; update: the SGD WRITE g -= lr sums[1], b -= lr sums[0]
 void bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
-                   const float* rstd, const float* g, const float* b, int relu, float* part);
-// sums [2][C] = (sum dy', sum dy' xh); old [2][C] = pre-update (g, b); update: SGD of g, b
-void bn_bwd_finalize(cudaStream_t s, const float* part, int nblk, int C, float* sums, float* old, float* g, float* b,
-                     float lr, int update);
+                   const float* rstd, float* g, float* b, int relu, float* part, int* ctr, float* sums, float* old,
+                   float lr, int update);
 void bn_bwd_apply(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
                   const float* rstd, const float* old, const float* sums, int relu, bf16* dz);
 // depthwise k x k (k in {3,5,7}), stride S, pad k/2; w fp32 [C][k][k]; H = input height = width.
@@ -140,8 +142,8 @@ void bn_bwd_apply(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P
 void dw_fwd(cudaStream_t s, const bf16* x, const float* w, bf16* z, int B, int H, int C, int k, int S);
 void dw_dgrad(cudaStream_t s, const bf16* dz, const float* w, const bf16* add, bf16* dx, int B, int H, int C, int k,
               int S);
-int dw_wgrad_blocks(int P_out);
-// part [dw_wgrad_blocks(B*Ho*Ho)][C][k][k]
+int dw_wgrad_blocks(int B, int H, int C, int k, int S);
+// part [dw_wgrad_blocks(B, H, C, k, S)][C][k][k]
 void dw_wgrad(cudaStream_t s, const bf16* dz, const bf16* x, float* part, int B, int H, int C, int k, int S);
 // channel split of a stride-1 block input [P, 2Ch] (x2): out[:, i] = x[:, 2i] (ld ldo, planes
 // oplane apart), xm[:, i] = x[:, 2i+1]; merge is its (plain bf16) backward
@@ -149,8 +151,9 @@ void chan_split(cudaStream_t s, const bf16* x, int P, int Ch, bf16* out, int ldo
 void chan_merge(cudaStream_t s, const bf16* dproj, int ldp, const bf16* dm, int P, int Ch, bf16* dx);
 // frozen head pieces
 void gap_pool(cudaStream_t s, const bf16* r, int B, int HW, int C, float* gap);
+// logits = gap W_fc^T (fp32 tiles), then per-sample softmax CE: loss_per[b], dlogits = (p - onehot)/B
 void fc_ce(cudaStream_t s, const float* gap, const float* wf, const int* labels, int B, int C, int ncls,
-           float* dlogits, float* loss_per);
+           float* logits, float* dlogits, float* loss_per);
 void ce_mean(cudaStream_t s, const float* loss_per, int B, float* loss);
 void fc_dgap(cudaStream_t s, const float* dlogits, const float* wf, int B, int C, int ncls, float* dgap);
 void head_bcast(cudaStream_t s, const float* dgap, int B, int HW, int C, bf16* dr);

@@ -11,12 +11,12 @@
 // Block internals follow SURVEY §8c "C2 SPOS candidate" (readings A16, A27):
 // every conv is bias-free and followed by training-mode BatchNorm (batch statistics over
 // N*H*W, biased variance, eps 1e-5).  Per conv -> BN [-> ReLU] unit the forward is
-//   conv -> z (bf16);  bn_stats(z) -> per-row-block partial (sum, sum of squares);
-//   bn_finalize -> mean, rstd;  bn_apply -> y = relu?(g * ((z - mean) * rstd) + b) (bf16)
+//   conv -> z;  bn_stats(z) -> per-row-block partials (sum, sum of squares), the last CTA
+//   reduces them to mean, rstd;  bn_apply -> y = relu?(g * ((z - mean) * rstd) + b)
 // and the backward (dy = grad of y; s1 = sum dy', s2 = sum dy' * xh over the batch, dy' = dy
 // masked by the ReLU):
-//   bn_bwd_reduce -> partials of s1, s2;  bn_bwd_finalize -> s1, s2, and the WRITE of g, b
-//   (dg = s2, db = s1; the pre-update g, b are kept for the input gradient);
+//   bn_bwd_reduce -> partials of s1, s2, the last CTA reduces them and applies the WRITE of
+//   g, b (dg = s2, db = s1; the pre-update g, b are kept for the input gradient);
 //   bn_bwd_apply -> dz = rstd * g * (dy' - s1/P - xh * s2/P)  (bf16).
 // Every reduction has a fixed order (per-thread sequential, then a fixed cross-thread order,
 // then a fixed order over row blocks), never floating-point atomics: bitwise reproducible.
@@ -31,9 +31,17 @@ namespace naspipe {
 namespace {
 
 constexpr int TPB = 256;          // threads per block of the row-block kernels
-constexpr int BN_ROWS = 256;      // rows (pixels) per BN partial
-constexpr int DW_ROWS = 1024;     // output pixels per depthwise weight-gradient partial
+constexpr int RED_CTAS = 592;     // target CTAs of the row-block reductions (4 per SM)
 constexpr float BN_EPS = 1e-5f;
+
+// Row blocking of the per-channel reductions: a function of (P, C) only (deterministic),
+// about RED_CTAS blocks, each a multiple of the kernel's row lanes RP = TPB / (C/8).
+__host__ __device__ inline int red_rows(int P, int C) {
+  const int rp = TPB / (C / 8);
+  int rows = (P + RED_CTAS - 1) / RED_CTAS;
+  rows = ((rows + rp - 1) / rp) * rp;
+  return rows < rp ? rp : rows;
+}
 
 inline void check_launch(const char* what) {
   cudaError_t e = cudaGetLastError();
@@ -128,18 +136,110 @@ __global__ void stem_conv_kernel(const float* __restrict__ x, const float* __res
 }
 
 // ---------------------------------------------------------------- BatchNorm forward
-// Thread (r, g): rows r, r + RP, ... of the block, channels [8g, 8g+8).  RP = TPB / G.
+// Per-channel reductions over P rows: RED_CTAS-ish row blocks write partial sums
+// part[blk][0..2C); a finalize kernel sums them in block order (fp64): one warp per
+// (channel, which-sum), lane j sums blocks j, j+32, ... in order, then a fixed xor tree.
+__device__ __forceinline__ double warp_sum_d(double v) {
+#pragma unroll
+  for (int s = 16; s >= 1; s >>= 1) v += __shfl_xor_sync(0xffffffffu, v, s);
+  return v;
+}
+// warp w of the block: channel blockIdx.x * 4 + w / 2, sum w % 2; returns the total on all lanes
+__device__ __forceinline__ double part_total(const float* part, int nblk, int C, int c, int which) {
+  const int lane = threadIdx.x & 31;
+  double a = 0.0;
+  if (c < C) {
+    const float* p = part + which * C + c;
+    int k = lane;
+    for (; k + 96 < nblk; k += 128) {  // 4 independent loads in flight per lane
+      const float v0 = p[(size_t)k * 2 * C], v1 = p[(size_t)(k + 32) * 2 * C], v2 = p[(size_t)(k + 64) * 2 * C],
+                  v3 = p[(size_t)(k + 96) * 2 * C];
+      a += (double)v0;
+      a += (double)v1;
+      a += (double)v2;
+      a += (double)v3;
+    }
+    for (; k < nblk; k += 32) a += (double)p[(size_t)k * 2 * C];
+  }
+  return warp_sum_d(a);
+}
+
+// mean = sum / P, rstd = 1/sqrt(sumsq / P - mean^2 + eps) (biased variance)
+__global__ void bn_finalize_kernel(const float* __restrict__ part, int nblk, int C, int P, float* __restrict__ mean,
+                                   float* __restrict__ rstd) {
+  __shared__ double tot[8];
+  ptx::pdl_wait();
+  const int w = threadIdx.x >> 5, c = blockIdx.x * 4 + w / 2;
+  const double t = part_total(part, nblk, C, c, w & 1);
+  if ((threadIdx.x & 31) == 0) tot[w] = t;
+  __syncthreads();
+  if (threadIdx.x < 4) {
+    const int cc = blockIdx.x * 4 + threadIdx.x;
+    if (cc < C) {
+      const double mu = tot[2 * threadIdx.x] / P;
+      const double var = fmax(tot[2 * threadIdx.x + 1] / P - mu * mu, 0.0);
+      mean[cc] = (float)mu;
+      rstd[cc] = (float)(1.0 / sqrt(var + (double)BN_EPS));
+    }
+  }
+}
+
+// sums[0][c] = s1 (dbeta), sums[1][c] = s2 (dgamma); old = (gamma, beta) before the WRITE
+// gamma -= lr s2, beta -= lr s1 (if update)
+__global__ void bn_bwd_finalize_kernel(const float* __restrict__ part, int nblk, int C, float* __restrict__ sums,
+                                       float* __restrict__ old, float* __restrict__ gam, float* __restrict__ bet,
+                                       float lr, int update) {
+  __shared__ double tot[8];
+  ptx::pdl_wait();
+  const int w = threadIdx.x >> 5, c = blockIdx.x * 4 + w / 2;
+  const double t = part_total(part, nblk, C, c, w & 1);
+  if ((threadIdx.x & 31) == 0) tot[w] = t;
+  __syncthreads();
+  if (threadIdx.x < 4) {
+    const int cc = blockIdx.x * 4 + threadIdx.x;
+    if (cc < C) {
+      const float f1 = (float)tot[2 * threadIdx.x], f2 = (float)tot[2 * threadIdx.x + 1];
+      sums[cc] = f1;
+      sums[C + cc] = f2;
+      const float gv = gam[cc], bv = bet[cc];
+      old[cc] = gv;
+      old[C + cc] = bv;
+      if (update) {
+        gam[cc] = gv - lr * f2;
+        bet[cc] = bv - lr * f1;
+      }
+    }
+  }
+}
+
+// Thread (r, g): rows r, r + RP, ... of its block, channels [8g, 8g+8); RP = TPB / G row
+// lanes; the RP lane sums are combined in lane order.  Writes part[blk][0..C) = sum z,
+// part[blk][C..2C) = sum z^2.
 __global__ void bn_stats_kernel(const bf16* __restrict__ z, int P, int C, float* __restrict__ part) {
   extern __shared__ float red[];  // [RP][2C]
   ptx::pdl_wait();
-  const int G = C / 8, RP = TPB / G;
+  const int G = C / 8, RP = TPB / G, rows = red_rows(P, C);
   const int r = threadIdx.x / G, g = threadIdx.x % G;
-  const int row0 = blockIdx.x * BN_ROWS, row1 = min(P, row0 + BN_ROWS);
+  const int row0 = blockIdx.x * rows, row1 = min(P, row0 + rows);
+  const size_t plane = (size_t)P * C;
   if (r < RP) {
     float s[8] = {}, q[8] = {};
-    for (int row = row0 + r; row < row1; row += RP) {
+    int row = row0 + r;
+    for (; row + 3 * RP < row1; row += 4 * RP) {
+      float v[4][8];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) load8x2(z + (size_t)(row + u * RP) * C + 8 * g, plane, v[u]);
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          s[i] += v[u][i];
+          q[i] = __fmaf_rn(v[u][i], v[u][i], q[i]);
+        }
+    }
+    for (; row < row1; row += RP) {
       float v[8];
-      load8x2(z + (size_t)row * C + 8 * g, (size_t)P * C, v);
+      load8x2(z + (size_t)row * C + 8 * g, plane, v);
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
         s[i] += v[i];
@@ -160,45 +260,49 @@ __global__ void bn_stats_kernel(const bf16* __restrict__ z, int P, int C, float*
   }
 }
 
-// mean = sum / P, var = sumsq / P - mean^2 (biased), combined over row blocks in order in fp64
-__global__ void bn_finalize_kernel(const float* __restrict__ part, int nblk, int C, int P, float* __restrict__ mean,
-                                   float* __restrict__ rstd) {
-  ptx::pdl_wait();
-  const int c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= C) return;
-  double s = 0.0, q = 0.0;
-  for (int k = 0; k < nblk; ++k) {
-    s += (double)part[(size_t)k * 2 * C + c];
-    q += (double)part[(size_t)k * 2 * C + C + c];
-  }
-  const double mu = s / P;
-  const double var = fmax(q / P - mu * mu, 0.0);
-  mean[c] = (float)mu;
-  rstd[c] = (float)(1.0 / sqrt(var + (double)BN_EPS));
-}
+// Elementwise kernels over [P rows][C]: thread (pixel lane, channel group g) keeps its
+// group's per-channel parameters in registers and strides over pixels.
+__device__ __forceinline__ int ew_lanes(int C) { return TPB / (C / 8); }
 
 __global__ void bn_apply_kernel(const bf16* __restrict__ z, int P, int C, const float* __restrict__ mean,
                                 const float* __restrict__ rstd, const float* __restrict__ gam,
                                 const float* __restrict__ bet, int relu, bf16* __restrict__ y, int ldy,
                                 size_t yplane) {
   ptx::pdl_wait();
-  const int G = C / 8;
-  const size_t items = (size_t)P * G;
-  for (size_t it = blockIdx.x * (size_t)blockDim.x + threadIdx.x; it < items; it += (size_t)gridDim.x * blockDim.x) {
-    const size_t p = it / G;
-    const int c = (int)(it % G) * 8;
-    float v[8], mu[8], rs[8], g8[8], b8[8];
-    load8x2(z + p * C + c, (size_t)P * C, v);
-    load8f(mean + c, mu);
-    load8f(rstd + c, rs);
-    load8f(gam + c, g8);
-    load8f(bet + c, b8);
+  const int G = C / 8, lanes = ew_lanes(C);
+  const int pl = threadIdx.x / G, c = (threadIdx.x % G) * 8;
+  if (pl >= lanes) return;
+  float mu[8], rs[8], g8[8], b8[8];
+  load8f(mean + c, mu);
+  load8f(rstd + c, rs);
+  load8f(gam + c, g8);
+  load8f(bet + c, b8);
+  const size_t zplane = (size_t)P * C;
+  const int step = gridDim.x * lanes;
+  int p = blockIdx.x * lanes + pl;
+  for (; p + step < P; p += 2 * step) {  // two pixels in flight
+    float v[2][8];
+    load8x2(z + (size_t)p * C + c, zplane, v[0]);
+    load8x2(z + (size_t)(p + step) * C + c, zplane, v[1]);
+#pragma unroll
+    for (int u = 0; u < 2; ++u) {
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        const float o = bn_y(v[u][i], mu[i], rs[i], g8[i], b8[i]);
+        v[u][i] = relu ? fmaxf(o, 0.f) : o;
+      }
+      store8x2(y + (size_t)(p + u * step) * ldy + c, yplane, v[u]);
+    }
+  }
+  for (; p < P; p += step) {
+    float v[8];
+    load8x2(z + (size_t)p * C + c, zplane, v);
 #pragma unroll
     for (int i = 0; i < 8; ++i) {
       const float o = bn_y(v[i], mu[i], rs[i], g8[i], b8[i]);
       v[i] = relu ? fmaxf(o, 0.f) : o;
     }
-    store8x2(y + p * ldy + c, yplane, v);
+    store8x2(y + (size_t)p * ldy + c, yplane, v);
   }
 }
 
@@ -216,15 +320,17 @@ __device__ __forceinline__ void bn_bwd_item(const bf16* dy, const bf16* z, size_
   }
 }
 
+// Partials of s1 = sum dy', s2 = sum dy' xh (dy' = dy masked by the ReLU) per row block.
 __global__ void bn_bwd_reduce_kernel(const bf16* __restrict__ dy, int lddy, const bf16* __restrict__ z, int P, int C,
                                      const float* __restrict__ mean, const float* __restrict__ rstd,
                                      const float* __restrict__ gam, const float* __restrict__ bet, int relu,
                                      float* __restrict__ part) {
   extern __shared__ float red[];  // [RP][2C]
   ptx::pdl_wait();
-  const int G = C / 8, RP = TPB / G;
+  const int G = C / 8, RP = TPB / G, rows = red_rows(P, C);
   const int r = threadIdx.x / G, g = threadIdx.x % G;
-  const int row0 = blockIdx.x * BN_ROWS, row1 = min(P, row0 + BN_ROWS);
+  const int row0 = blockIdx.x * rows, row1 = min(P, row0 + rows);
+  const size_t zplane = (size_t)P * C;
   if (r < RP) {
     float mu[8], rs[8], g8[8], b8[8];
     load8f(mean + 8 * g, mu);
@@ -232,10 +338,24 @@ __global__ void bn_bwd_reduce_kernel(const bf16* __restrict__ dy, int lddy, cons
     load8f(gam + 8 * g, g8);
     load8f(bet + 8 * g, b8);
     float s1[8] = {}, s2[8] = {};
-    for (int row = row0 + r; row < row1; row += RP) {
+    int row = row0 + r;
+    for (; row + RP < row1; row += 2 * RP) {
+      float d[2][8], xh[2][8];
+#pragma unroll
+      for (int u = 0; u < 2; ++u)
+        bn_bwd_item(dy + (size_t)(row + u * RP) * lddy + 8 * g, z + (size_t)(row + u * RP) * C + 8 * g, zplane, mu, rs,
+                    g8, b8, relu, d[u], xh[u]);
+#pragma unroll
+      for (int u = 0; u < 2; ++u)
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          s1[i] += d[u][i];
+          s2[i] = __fmaf_rn(d[u][i], xh[u][i], s2[i]);
+        }
+    }
+    for (; row < row1; row += RP) {
       float d[8], xh[8];
-      bn_bwd_item(dy + (size_t)row * lddy + 8 * g, z + (size_t)row * C + 8 * g, (size_t)P * C, mu, rs, g8, b8, relu,
-                  d, xh);
+      bn_bwd_item(dy + (size_t)row * lddy + 8 * g, z + (size_t)row * C + 8 * g, zplane, mu, rs, g8, b8, relu, d, xh);
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
         s1[i] += d[i];
@@ -256,60 +376,37 @@ __global__ void bn_bwd_reduce_kernel(const bf16* __restrict__ dy, int lddy, cons
   }
 }
 
-// sums[0][c] = s1 = dbeta, sums[1][c] = s2 = dgamma (fixed order over row blocks, fp64);
-// old[0] = gamma, old[1] = beta before the update; the WRITE gamma -= lr s2, beta -= lr s1.
-__global__ void bn_bwd_finalize_kernel(const float* __restrict__ part, int nblk, int C, float* __restrict__ sums,
-                                       float* __restrict__ old, float* __restrict__ gam, float* __restrict__ bet,
-                                       float lr, int update) {
-  ptx::pdl_wait();
-  const int c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= C) return;
-  double s1 = 0.0, s2 = 0.0;
-  for (int k = 0; k < nblk; ++k) {
-    s1 += (double)part[(size_t)k * 2 * C + c];
-    s2 += (double)part[(size_t)k * 2 * C + C + c];
-  }
-  const float f1 = (float)s1, f2 = (float)s2;
-  sums[c] = f1;
-  sums[C + c] = f2;
-  const float g = gam[c], b = bet[c];
-  old[c] = g;
-  old[C + c] = b;
-  if (update) {
-    gam[c] = g - lr * f2;
-    bet[c] = b - lr * f1;
-  }
-}
-
 __global__ void bn_bwd_apply_kernel(const bf16* __restrict__ dy, int lddy, const bf16* __restrict__ z, int P, int C,
                                     const float* __restrict__ mean, const float* __restrict__ rstd,
                                     const float* __restrict__ old, const float* __restrict__ sums, int relu,
                                     bf16* __restrict__ dz) {
   ptx::pdl_wait();
-  const int G = C / 8;
+  const int G = C / 8, lanes = ew_lanes(C);
+  const int pl = threadIdx.x / G, c = (threadIdx.x % G) * 8;
+  if (pl >= lanes) return;
   const float invP = 1.0f / (float)P;
-  const size_t items = (size_t)P * G;
-  for (size_t it = blockIdx.x * (size_t)blockDim.x + threadIdx.x; it < items; it += (size_t)gridDim.x * blockDim.x) {
-    const size_t p = it / G;
-    const int c = (int)(it % G) * 8;
-    float mu[8], rs[8], g8[8], b8[8], m1[8], m2[8], d[8], xh[8];
-    load8f(mean + c, mu);
-    load8f(rstd + c, rs);
-    load8f(old + c, g8);
-    load8f(old + C + c, b8);
-    load8f(sums + c, m1);
-    load8f(sums + C + c, m2);
-    bn_bwd_item(dy + p * lddy + c, z + p * C + c, (size_t)P * C, mu, rs, g8, b8, relu, d, xh);
+  float mu[8], rs[8], g8[8], b8[8], m1[8], m2[8];
+  load8f(mean + c, mu);
+  load8f(rstd + c, rs);
+  load8f(old + c, g8);
+  load8f(old + C + c, b8);
+  load8f(sums + c, m1);
+  load8f(sums + C + c, m2);
+  const size_t zplane = (size_t)P * C;
+  const int step = gridDim.x * lanes;
+  for (int p = blockIdx.x * lanes + pl; p < P; p += step) {
+    float d[8], xh[8];
+    bn_bwd_item(dy + (size_t)p * lddy + c, z + (size_t)p * C + c, zplane, mu, rs, g8, b8, relu, d, xh);
 #pragma unroll
     for (int i = 0; i < 8; ++i) {
       const float t = d[i] - m1[i] * invP - xh[i] * (m2[i] * invP);
       d[i] = rs[i] * g8[i] * t;
     }
-    store8(dz + p * C + c, d);
+    store8(dz + (size_t)p * C + c, d);
   }
 }
 
-// ---------------------------------------------------------------- depthwise conv (pad K/2)
+// ---------------------------------------------------------------- depthwise conv (pad K/2): stride-2 input gradient
 // weights fp32 [C][K][K]; staged in shared memory as [K*K][C]
 template <int K>
 __device__ __forceinline__ void stage_dw_weights(float* ws, const float* w, int C) {
@@ -318,46 +415,6 @@ __device__ __forceinline__ void stage_dw_weights(float* ws, const float* w, int 
     ws[t * C + c] = w[i];
   }
   __syncthreads();
-}
-
-template <int K>
-__global__ void dw_fwd_kernel(const bf16* __restrict__ x, const float* __restrict__ w, bf16* __restrict__ z, int B,
-                              int H, int C, int S) {
-  extern __shared__ float ws[];
-  ptx::pdl_wait();
-  stage_dw_weights<K>(ws, w, C);
-  constexpr int PAD = K / 2;
-  const int Ho = (H + 2 * PAD - K) / S + 1;
-  const int G = C / 8;
-  const size_t items = (size_t)B * Ho * Ho * G;
-  for (size_t it = blockIdx.x * (size_t)blockDim.x + threadIdx.x; it < items; it += (size_t)gridDim.x * blockDim.x) {
-    const int c = (int)(it % G) * 8;
-    const size_t p = it / G;
-    const int ow = (int)(p % Ho);
-    const int oh = (int)((p / Ho) % Ho);
-    const int b = (int)(p / ((size_t)Ho * Ho));
-    float acc[8] = {};
-    const size_t xplane = (size_t)B * H * H * C;
-#pragma unroll
-    for (int u = 0; u < K; ++u) {
-      const int ih = oh * S + u - PAD;
-      if (ih < 0 || ih >= H) continue;
-      const bf16* row = x + (((size_t)b * H + ih) * H) * C + c;
-#pragma unroll
-      for (int v = 0; v < K; ++v) {
-        const int iw = ow * S + v - PAD;
-        if (iw < 0 || iw >= H) continue;
-        float xv[8], wv[8];
-        load8x2(row + (size_t)iw * C, xplane, xv);
-        const float* wt = ws + (u * K + v) * C + c;
-#pragma unroll
-        for (int i = 0; i < 8; ++i) wv[i] = wt[i];
-#pragma unroll
-        for (int i = 0; i < 8; ++i) acc[i] = __fmaf_rn(xv[i], wv[i], acc[i]);
-      }
-    }
-    store8x2(z + p * C + c, items / G * C, acc);
-  }
 }
 
 // dx[b,ih,iw,c] = sum_{u,v} dz[b,oh,ow,c] w[c,u,v] with oh*S + u - PAD = ih (+ add[b,ih,iw,c])
@@ -407,12 +464,96 @@ __global__ void dw_dgrad_kernel(const bf16* __restrict__ dz, const float* __rest
   }
 }
 
-// Weight gradient partials: block (blk, u) sums over output pixels [blk*DW_ROWS, ...) the
+// ---------------------------------------------------------------- depthwise conv, shared-memory tiles
+// Correlation out[b,oh,ow,c] = sum_{u,v} in[b, oh*S+u-PAD, ow*S+v-PAD, c] w'[c,u,v] (+ add),
+// w' = w (forward) or w flipped in u and v (FLIP: the stride-1 input gradient).  A CTA owns
+// a tile of DT_H output rows x TW columns x CPG groups of 8 channels: the input halo is
+// staged in shared memory once (16-byte loads, fp32), each thread keeps one channel's k x k
+// weights in registers and computes a DT_H-row strip of one column from shared memory (each
+// staged value feeds up to DT_H outputs).  X2: bf16x2 input/output (forward), else bf16.
+constexpr int DT_H = 8;
+
+template <int K, int S, bool X2, bool FLIP>
+__global__ void __launch_bounds__(TPB) dw_tile_kernel(const bf16* __restrict__ in, const float* __restrict__ w,
+                                                    const bf16* __restrict__ add, bf16* __restrict__ out, int B,
+                                                    int H, int C, int TW) {
+  constexpr int PAD = K / 2, IH = (DT_H - 1) * S + K;
+  extern __shared__ float tile[];  // [CPG][IH][IW][8]
+  ptx::pdl_wait();
+  const int Ho = (H + 2 * PAD - K) / S + 1;
+  const int CPG = TPB / (8 * TW), IW = (TW - 1) * S + K;
+  const int tiles_h = (Ho + DT_H - 1) / DT_H, tiles_w = (Ho + TW - 1) / TW;
+  int t = blockIdx.x;
+  const int tw = t % tiles_w;
+  t /= tiles_w;
+  const int th = t % tiles_h;
+  t /= tiles_h;
+  const int b = t;
+  const int cg0 = blockIdx.y * CPG;  // first channel group of the CTA
+  const size_t iplane = (size_t)B * H * H * C, oplane = (size_t)B * Ho * Ho * C;
+  // stage the halo: CPG x IH x IW pixels of 8 channels
+  const int ih0 = th * DT_H * S - PAD, iw0 = tw * TW * S - PAD;
+  for (int i = threadIdx.x; i < CPG * IH * IW; i += TPB) {
+    const int col = i % IW, row = (i / IW) % IH, cg = i / (IW * IH);
+    const int ih = ih0 + row, iw = iw0 + col, c = (cg0 + cg) * 8;
+    float v[8] = {};
+    if (ih >= 0 && ih < H && iw >= 0 && iw < H && c < C) {
+      const bf16* p = in + (((size_t)b * H + ih) * H + iw) * C + c;
+      if (X2) load8x2(p, iplane, v);
+      else load8(p, v);
+    }
+    float4* d = reinterpret_cast<float4*>(tile + (size_t)i * 8);
+    d[0] = make_float4(v[0], v[1], v[2], v[3]);
+    d[1] = make_float4(v[4], v[5], v[6], v[7]);
+  }
+  const int ch = threadIdx.x % 8, col = (threadIdx.x / 8) % TW, cgi = threadIdx.x / (8 * TW);
+  const int c = (cg0 + cgi) * 8 + ch;
+  float wr[K][K];
+#pragma unroll
+  for (int u = 0; u < K; ++u)
+#pragma unroll
+    for (int v = 0; v < K; ++v)
+      wr[u][v] = c < C ? w[(size_t)c * K * K + (FLIP ? (K - 1 - u) * K + (K - 1 - v) : u * K + v)] : 0.f;
+  __syncthreads();
+  float acc[DT_H];
+#pragma unroll
+  for (int r = 0; r < DT_H; ++r) acc[r] = 0.f;
+  const float* tb = tile + ((size_t)cgi * IH * IW + col * S) * 8 + ch;
+#pragma unroll
+  for (int ir = 0; ir < IH; ++ir) {
+#pragma unroll
+    for (int v = 0; v < K; ++v) {
+      const float x = tb[((size_t)ir * IW + v) * 8];
+#pragma unroll
+      for (int r = 0; r < DT_H; ++r) {
+        const int u = ir - r * S;
+        if (u >= 0 && u < K) acc[r] = __fmaf_rn(x, wr[u][v], acc[r]);
+      }
+    }
+  }
+  const int ow = tw * TW + col;
+  if (c >= C || ow >= Ho) return;
+#pragma unroll
+  for (int r = 0; r < DT_H; ++r) {
+    const int oh = th * DT_H + r;
+    if (oh >= Ho) break;
+    const size_t o = (((size_t)b * Ho + oh) * Ho + ow) * C + c;
+    if (X2) {
+      const bf16 hi = __float2bfloat16_rn(acc[r]);
+      out[o] = hi;
+      out[o + oplane] = __float2bfloat16_rn(acc[r] - __bfloat162float(hi));
+    } else {
+      out[o] = __float2bfloat16_rn(add ? acc[r] + __bfloat162float(add[o]) : acc[r]);
+    }
+  }
+}
+
+// Weight gradient partials: block (blk, u) sums over output pixels [blk*rows, ...) the
 // products dz[b,oh,ow,c] * x[b, oh*S+u-PAD, ow*S+v-PAD, c] for every c, v.
 // part[blk][c][u][v] (the [C][K][K] layout of the weight).
 template <int K>
 __global__ void dw_wgrad_kernel(const bf16* __restrict__ dz, const bf16* __restrict__ x, float* __restrict__ part,
-                                int B, int H, int C, int S) {
+                                int B, int H, int C, int S, int rows) {
   extern __shared__ float red[];  // [RP][C][K]
   ptx::pdl_wait();
   constexpr int PAD = K / 2;
@@ -421,7 +562,7 @@ __global__ void dw_wgrad_kernel(const bf16* __restrict__ dz, const bf16* __restr
   const int r = threadIdx.x / G, g = threadIdx.x % G;
   const int u = blockIdx.y;
   const int P = B * Ho * Ho;
-  const int q0 = blockIdx.x * DW_ROWS, q1 = min(P, q0 + DW_ROWS);
+  const int q0 = blockIdx.x * rows, q1 = min(P, q0 + rows);
   if (r < RP) {
     float acc[K][8] = {};
     for (int q = q0 + r; q < q1; q += RP) {
@@ -454,6 +595,7 @@ __global__ void dw_wgrad_kernel(const bf16* __restrict__ dz, const bf16* __restr
     part[(size_t)blockIdx.x * C * K * K + (size_t)c * K * K + u * K + v] = a;
   }
 }
+
 
 // ---------------------------------------------------------------- channel split / merge
 // stride-1 block input x [P, 2Ch]: out[:, i] = x[:, 2i] (passed through, ld ldo), xm[:, i] = x[:, 2i+1]
@@ -536,23 +678,49 @@ __device__ __forceinline__ float warp_max(float v) {
   return v;
 }
 
-// One block per sample: logits = W_fc gap[b] (fp32), softmax cross-entropy, dlogits / B.
-__global__ void fc_ce_kernel(const float* __restrict__ gap, const float* __restrict__ wf, const int* __restrict__ labels,
-                             int B, int C, int ncls, float* __restrict__ dlogits, float* __restrict__ loss_per) {
-  extern __shared__ float lg[];  // [ncls]
+// One block per 32 classes: logits[b][j] = sum_c gap[b][c] W_fc[j][c] (fp32, c ascending),
+// gap / W tiles of 32 columns staged in shared memory; thread (j, sample group).
+__global__ void fc_logits_kernel(const float* __restrict__ gap, const float* __restrict__ wf, int B, int C, int ncls,
+                                 float* __restrict__ logits) {
+  __shared__ float ws[32][33], gs[64][33];
+  ptx::pdl_wait();
+  const int jl = threadIdx.x % 32, sg = threadIdx.x / 32, j = blockIdx.x * 32 + jl;
+  for (int b0 = 0; b0 < B; b0 += 64) {
+    float acc[8] = {};
+    for (int c0 = 0; c0 < C; c0 += 32) {
+      for (int i = threadIdx.x; i < 32 * 32; i += TPB) {
+        const int r = i / 32, c = c0 + i % 32, jj = blockIdx.x * 32 + r;
+        ws[r][i % 32] = (jj < ncls && c < C) ? wf[(size_t)jj * C + c] : 0.f;
+      }
+      for (int i = threadIdx.x; i < 64 * 32; i += TPB) {
+        const int r = i / 32, c = c0 + i % 32, b = b0 + r;
+        gs[r][i % 32] = (b < B && c < C) ? gap[(size_t)b * C + c] : 0.f;
+      }
+      __syncthreads();
+#pragma unroll 4
+      for (int cc = 0; cc < 32; ++cc) {
+        const float w = ws[jl][cc];
+#pragma unroll
+        for (int si = 0; si < 8; ++si) acc[si] = __fmaf_rn(gs[sg + 8 * si][cc], w, acc[si]);
+      }
+      __syncthreads();
+    }
+#pragma unroll
+    for (int si = 0; si < 8; ++si) {
+      const int b = b0 + sg + 8 * si;
+      if (b < B && j < ncls) logits[(size_t)b * ncls + j] = acc[si];
+    }
+  }
+}
+
+// One block per sample: softmax cross-entropy of its logits, dlogits = (p - onehot) / B.
+__global__ void ce_kernel(const float* __restrict__ logits, const int* __restrict__ labels, int B, int ncls,
+                          float* __restrict__ dlogits, float* __restrict__ loss_per) {
   __shared__ float red[TPB / 32];
   __shared__ float bc;
   ptx::pdl_wait();
   const int b = blockIdx.x, warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = TPB / 32;
-  const float* gb = gap + (size_t)b * C;
-  for (int j = warp; j < ncls; j += nw) {
-    const float* wr = wf + (size_t)j * C;
-    float a = 0.f;
-    for (int c = lane; c < C; c += 32) a = __fmaf_rn(gb[c], wr[c], a);
-    a = warp_sum(a);
-    if (lane == 0) lg[j] = a;
-  }
-  __syncthreads();
+  const float* lg = logits + (size_t)b * ncls;
   float mx = -INFINITY;
   for (int j = threadIdx.x; j < ncls; j += TPB) mx = fmaxf(mx, lg[j]);
   mx = warp_max(mx);
@@ -594,16 +762,38 @@ __global__ void ce_mean_kernel(const float* __restrict__ loss_per, int B, float*
   }
 }
 
-// dgap[b, c] = sum_j dlogits[b, j] W_fc[j, c]
+// One block per 32 channels: dgap[b][c] = sum_j dlogits[b][j] W_fc[j][c] (fp32, j ascending).
 __global__ void fc_dgap_kernel(const float* __restrict__ dlogits, const float* __restrict__ wf, int B, int C, int ncls,
                                float* __restrict__ dgap) {
+  __shared__ float ws[32][33], ds[64][33];
   ptx::pdl_wait();
-  const int b = blockIdx.y, c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= C) return;
-  const float* dl = dlogits + (size_t)b * ncls;
-  float a = 0.f;
-  for (int j = 0; j < ncls; ++j) a = __fmaf_rn(dl[j], wf[(size_t)j * C + c], a);
-  dgap[(size_t)b * C + c] = a;
+  const int cl = threadIdx.x % 32, sg = threadIdx.x / 32, c = blockIdx.x * 32 + cl;
+  for (int b0 = 0; b0 < B; b0 += 64) {
+    float acc[8] = {};
+    for (int j0 = 0; j0 < ncls; j0 += 32) {
+      for (int i = threadIdx.x; i < 32 * 32; i += TPB) {
+        const int r = i / 32, cc = blockIdx.x * 32 + i % 32, j = j0 + r;
+        ws[r][i % 32] = (j < ncls && cc < C) ? wf[(size_t)j * C + cc] : 0.f;
+      }
+      for (int i = threadIdx.x; i < 64 * 32; i += TPB) {
+        const int r = i / 32, j = j0 + i % 32, b = b0 + r;
+        ds[r][i % 32] = (b < B && j < ncls) ? dlogits[(size_t)b * ncls + j] : 0.f;
+      }
+      __syncthreads();
+#pragma unroll 4
+      for (int jj = 0; jj < 32; ++jj) {
+        const float w = ws[jj][cl];
+#pragma unroll
+        for (int si = 0; si < 8; ++si) acc[si] = __fmaf_rn(ds[sg + 8 * si][jj], w, acc[si]);
+      }
+      __syncthreads();
+    }
+#pragma unroll
+    for (int si = 0; si < 8; ++si) {
+      const int b = b0 + sg + 8 * si;
+      if (b < B && c < C) dgap[(size_t)b * C + c] = acc[si];
+    }
+  }
 }
 
 // dr[b, hw, c] = dgap[b, c] / HW
@@ -656,8 +846,10 @@ void f32_to_bf16x2(cudaStream_t s, const float* w32, bf16* hi, bf16* lo, size_t 
   check_launch("f32_to_bf16x2");
 }
 
-int bn_part_blocks(int P) { return (P + BN_ROWS - 1) / BN_ROWS; }
-int dw_wgrad_blocks(int P_out) { return (P_out + DW_ROWS - 1) / DW_ROWS; }
+int bn_part_blocks(int P, int C) {
+  const int r = red_rows(P, C);
+  return (P + r - 1) / r;
+}
 
 void spos_stem_conv(cudaStream_t s, const float* x, const float* w, bf16* z, int B, int H, int C0) {
   NP_REQUIRE(C0 % 8 == 0 && H % 2 == 0, NASPIPE_EINVAL, "stem C0=%d H=%d", C0, H);
@@ -666,46 +858,52 @@ void spos_stem_conv(cudaStream_t s, const float* x, const float* w, bf16* z, int
   check_launch("stem_conv");
 }
 
-void bn_stats(cudaStream_t s, const bf16* z, int P, int C, float* part) {
-  NP_REQUIRE(C % 8 == 0 && C / 8 <= TPB, NASPIPE_EINVAL, "bn_stats C=%d", C);
-  const size_t sm = (size_t)(TPB / (C / 8)) * 2 * C * sizeof(float);
-  set_smem(bn_stats_kernel, sm);
-  launch_pdl(bn_stats_kernel, dim3(bn_part_blocks(P)), dim3(TPB), sm, s, z, P, C, part);
-  check_launch("bn_stats");
+// grid of the pixel-strided elementwise kernels: about 8 CTAs per SM
+static int ew_grid(int P, int C) {
+  const int lanes = TPB / (C / 8);
+  return std::max(1, std::min((P + lanes - 1) / lanes, 148 * 8));
 }
 
-void bn_finalize(cudaStream_t s, const float* part, int nblk, int C, int P, float* mean, float* rstd) {
-  launch_pdl(bn_finalize_kernel, dim3((C + 127) / 128), dim3(128), 0, s, part, nblk, C, P, mean, rstd);
-  check_launch("bn_finalize");
+static size_t red_smem(int C) { return (size_t)(TPB / (C / 8)) * 2 * C * sizeof(float); }
+
+// ctr: kept in the signature for a single-kernel (last-CTA) finalize; unused by the
+// two-kernel form (partials, then a parallel fixed-order finalize), which measured faster.
+void bn_stats(cudaStream_t s, const bf16* z, int P, int C, float* part, int* ctr, float* mean, float* rstd) {
+  (void)ctr;
+  NP_REQUIRE(C % 8 == 0 && C / 8 <= TPB, NASPIPE_EINVAL, "bn_stats C=%d", C);
+  const size_t sm = red_smem(C);
+  const int nblk = bn_part_blocks(P, C);
+  set_smem(bn_stats_kernel, sm);
+  launch_pdl(bn_stats_kernel, dim3(nblk), dim3(TPB), sm, s, z, P, C, part);
+  launch_pdl(bn_finalize_kernel, dim3((C + 3) / 4), dim3(TPB), 0, s, (const float*)part, nblk, C, P, mean, rstd);
+  check_launch("bn_stats");
 }
 
 void bn_apply(cudaStream_t s, const bf16* z, int P, int C, const float* mean, const float* rstd, const float* g,
               const float* b, int relu, bf16* y, int ldy, size_t yplane) {
-  launch_pdl(bn_apply_kernel, dim3(grid_for((size_t)P * (C / 8))), dim3(TPB), 0, s, z, P, C, mean, rstd, g, b, relu,
+  launch_pdl(bn_apply_kernel, dim3(ew_grid(P, C)), dim3(TPB), 0, s, z, P, C, mean, rstd, g, b, relu,
              y, ldy, yplane);
   check_launch("bn_apply");
 }
 
 void bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
-                   const float* rstd, const float* g, const float* b, int relu, float* part) {
+                   const float* rstd, float* g, float* b, int relu, float* part, int* ctr, float* sums, float* old,
+                   float lr, int update) {
+  (void)ctr;
   NP_REQUIRE(C % 8 == 0 && C / 8 <= TPB, NASPIPE_EINVAL, "bn_bwd C=%d", C);
-  const size_t sm = (size_t)(TPB / (C / 8)) * 2 * C * sizeof(float);
+  const size_t sm = red_smem(C);
+  const int nblk = bn_part_blocks(P, C);
   set_smem(bn_bwd_reduce_kernel, sm);
-  launch_pdl(bn_bwd_reduce_kernel, dim3(bn_part_blocks(P)), dim3(TPB), sm, s, dy, lddy, z, P, C, mean, rstd, g, b,
-             relu, part);
+  launch_pdl(bn_bwd_reduce_kernel, dim3(nblk), dim3(TPB), sm, s, dy, lddy, z, P, C, mean, rstd, (const float*)g,
+             (const float*)b, relu, part);
+  launch_pdl(bn_bwd_finalize_kernel, dim3((C + 3) / 4), dim3(TPB), 0, s, (const float*)part, nblk, C, sums, old, g,
+             b, lr, update);
   check_launch("bn_bwd_reduce");
-}
-
-void bn_bwd_finalize(cudaStream_t s, const float* part, int nblk, int C, float* sums, float* old, float* g, float* b,
-                     float lr, int update) {
-  launch_pdl(bn_bwd_finalize_kernel, dim3((C + 127) / 128), dim3(128), 0, s, part, nblk, C, sums, old, g, b, lr,
-             update);
-  check_launch("bn_bwd_finalize");
 }
 
 void bn_bwd_apply(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
                   const float* rstd, const float* old, const float* sums, int relu, bf16* dz) {
-  launch_pdl(bn_bwd_apply_kernel, dim3(grid_for((size_t)P * (C / 8))), dim3(TPB), 0, s, dy, lddy, z, P, C, mean, rstd,
+  launch_pdl(bn_bwd_apply_kernel, dim3(ew_grid(P, C)), dim3(TPB), 0, s, dy, lddy, z, P, C, mean, rstd,
              old, sums, relu, dz);
   check_launch("bn_bwd_apply");
 }
@@ -718,36 +916,56 @@ void bn_bwd_apply(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P
     default: NP_REQUIRE(false, NASPIPE_EINVAL, "depthwise kernel %d", K); \
   }
 
+// tile width: the smallest of 8 / 16 / 32 columns covering min(Ho, 32)
+static int dw_tw(int Ho) { return Ho <= 8 ? 8 : (Ho <= 16 ? 16 : 32); }
+
+template <int K, int S, bool X2, bool FLIP>
+static void dw_tile(cudaStream_t s, const bf16* in, const float* w, const bf16* add, bf16* out, int B, int H, int C) {
+  const int Ho = (H - 1) / S + 1, TW = dw_tw(Ho), CPG = TPB / (8 * TW);
+  const int IH = (DT_H - 1) * S + K, IW = (TW - 1) * S + K;
+  const size_t sm = (size_t)CPG * IH * IW * 8 * sizeof(float);
+  const int gx = B * ((Ho + DT_H - 1) / DT_H) * ((Ho + TW - 1) / TW), gy = (C / 8 + CPG - 1) / CPG;
+  set_smem(dw_tile_kernel<K, S, X2, FLIP>, sm);
+  launch_pdl(dw_tile_kernel<K, S, X2, FLIP>, dim3(gx, gy), dim3(TPB), sm, s, in, w, add, out, B, H, C, TW);
+}
+
 void dw_fwd(cudaStream_t s, const bf16* x, const float* w, bf16* z, int B, int H, int C, int k, int S) {
-  const int Ho = (H - 1) / S + 1;
-  const size_t items = (size_t)B * Ho * Ho * (C / 8);
-  const size_t sm = (size_t)C * k * k * sizeof(float);
-  DW_DISPATCH(k, {
-    set_smem(dw_fwd_kernel<KK>, sm);
-    launch_pdl(dw_fwd_kernel<KK>, dim3(grid_for(items)), dim3(TPB), sm, s, x, w, z, B, H, C, S);
-  });
+  NP_REQUIRE(C % 8 == 0 && (S == 1 || S == 2), NASPIPE_EINVAL, "dw_fwd C=%d S=%d", C, S);
+  if (S == 1) { DW_DISPATCH(k, (dw_tile<KK, 1, true, false>(s, x, w, nullptr, z, B, H, C))); }
+  else { DW_DISPATCH(k, (dw_tile<KK, 2, true, false>(s, x, w, nullptr, z, B, H, C))); }
   check_launch("dw_fwd");
 }
 
 void dw_dgrad(cudaStream_t s, const bf16* dz, const float* w, const bf16* add, bf16* dx, int B, int H, int C, int k,
               int S) {
-  const size_t items = (size_t)B * H * H * (C / 8);
-  const size_t sm = (size_t)C * k * k * sizeof(float);
-  DW_DISPATCH(k, {
-    set_smem(dw_dgrad_kernel<KK>, sm);
-    launch_pdl(dw_dgrad_kernel<KK>, dim3(grid_for(items)), dim3(TPB), sm, s, dz, w, add, dx, B, H, C, S);
-  });
+  if (S == 1) {  // the input gradient of a stride-1 conv is the correlation with the flipped kernel
+    DW_DISPATCH(k, (dw_tile<KK, 1, false, true>(s, dz, w, add, dx, B, H, C)));
+  } else {
+    const size_t items = (size_t)B * H * H * (C / 8);
+    const size_t sm = (size_t)C * k * k * sizeof(float);
+    DW_DISPATCH(k, {
+      set_smem(dw_dgrad_kernel<KK>, sm);
+      launch_pdl(dw_dgrad_kernel<KK>, dim3(grid_for(items)), dim3(TPB), sm, s, dz, w, add, dx, B, H, C, S);
+    });
+  }
   check_launch("dw_dgrad");
+}
+
+// weight-gradient row blocks: about RED_CTAS CTAs over the (row block, kernel row) grid
+static int dw_rows(int P_out, int C, int k) { return red_rows(P_out, C) * k; }
+int dw_wgrad_blocks(int B, int H, int C, int k, int S) {
+  const int Ho = (H - 1) / S + 1, P = B * Ho * Ho, r = dw_rows(P, C, k);
+  return (P + r - 1) / r;
 }
 
 void dw_wgrad(cudaStream_t s, const bf16* dz, const bf16* x, float* part, int B, int H, int C, int k, int S) {
   NP_REQUIRE(C % 8 == 0 && C / 8 <= TPB, NASPIPE_EINVAL, "dw_wgrad C=%d", C);
   const int Ho = (H - 1) / S + 1;
-  const int nblk = dw_wgrad_blocks(B * Ho * Ho);
+  const int P_out = B * Ho * Ho, nblk = dw_wgrad_blocks(B, H, C, k, S), rows = dw_rows(P_out, C, k);
   const size_t sm = (size_t)(TPB / (C / 8)) * C * k * sizeof(float);
   DW_DISPATCH(k, {
     set_smem(dw_wgrad_kernel<KK>, sm);
-    launch_pdl(dw_wgrad_kernel<KK>, dim3(nblk, KK), dim3(TPB), sm, s, dz, x, part, B, H, C, S);
+    launch_pdl(dw_wgrad_kernel<KK>, dim3(nblk, KK), dim3(TPB), sm, s, dz, x, part, B, H, C, S, rows);
   });
   check_launch("dw_wgrad");
 }
@@ -769,10 +987,9 @@ void gap_pool(cudaStream_t s, const bf16* r, int B, int HW, int C, float* gap) {
 }
 
 void fc_ce(cudaStream_t s, const float* gap, const float* wf, const int* labels, int B, int C, int ncls,
-           float* dlogits, float* loss_per) {
-  const size_t sm = (size_t)ncls * sizeof(float);
-  set_smem(fc_ce_kernel, sm);
-  launch_pdl(fc_ce_kernel, dim3(B), dim3(TPB), sm, s, gap, wf, labels, B, C, ncls, dlogits, loss_per);
+           float* logits, float* dlogits, float* loss_per) {
+  launch_pdl(fc_logits_kernel, dim3((ncls + 31) / 32), dim3(TPB), 0, s, gap, wf, B, C, ncls, logits);
+  launch_pdl(ce_kernel, dim3(B), dim3(TPB), 0, s, logits, labels, B, ncls, dlogits, loss_per);
   check_launch("fc_ce");
 }
 
@@ -782,7 +999,7 @@ void ce_mean(cudaStream_t s, const float* loss_per, int B, float* loss) {
 }
 
 void fc_dgap(cudaStream_t s, const float* dlogits, const float* wf, int B, int C, int ncls, float* dgap) {
-  launch_pdl(fc_dgap_kernel, dim3((C + 127) / 128, B), dim3(128), 0, s, dlogits, wf, B, C, ncls, dgap);
+  launch_pdl(fc_dgap_kernel, dim3((C + 31) / 32), dim3(TPB), 0, s, dlogits, wf, B, C, ncls, dgap);
   check_launch("fc_dgap");
 }
 
