@@ -15,6 +15,7 @@
 
 #include <algorithm>
 #include <atomic>
+#include <cstdlib>
 #include <mutex>
 
 #include "common.h"
@@ -43,7 +44,8 @@ struct TileCfg {
   static constexpr int STAGE_BYTES = OPS * (A_BYTES + B_BYTES);
   static constexpr int STAGES = (200 * 1024) / STAGE_BYTES > 6 ? 6 : (200 * 1024) / STAGE_BYTES;
   static constexpr int BAR_OFF = STAGES * STAGE_BYTES;
-  static constexpr int SMEM_TOTAL = BAR_OFF + (2 * STAGES + 4) * 8 + 16 + 1024;  // + alignment slack
+  static constexpr int STG_OFF = BAR_OFF + (2 * STAGES + 4) * 8 + 16;
+  static constexpr int SMEM_TOTAL = STG_OFF + 8 * 32 * 20 * 4 + 1024;  // + epilogue staging, alignment slack
   static constexpr int TMEM_COLS = 2 * TN <= 128 ? 128 : (2 * TN <= 256 ? 256 : 512);
 };
 
@@ -72,90 +74,117 @@ __device__ __forceinline__ void store16_f32(float* dst, const float (&v)[16]) {
   for (int i = 0; i < 4; ++i) o4[i] = make_float4(v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
 }
 
-// Operands of the epilogue that live in global memory, loaded BEFORE the TMEM read so that
-// their latency overlaps it (residual / fp32 master / pre-activation).
-struct Pre16 {
-  float4 q[4];
-  uint4 z[2];
-};
-template <int EPI>
-__device__ __forceinline__ void preload16(Pre16& p, size_t off, const GemmEpiParams& ep) {
-  if constexpr (EPI == EPI_BIAS_RESID_F32) {
-#pragma unroll
-    for (int i = 0; i < 4; ++i) p.q[i] = reinterpret_cast<const float4*>(ep.resid + off)[i];
-  }
-  if constexpr (EPI == EPI_SGD) {
-#pragma unroll
-    for (int i = 0; i < 4; ++i) p.q[i] = reinterpret_cast<const float4*>(ep.w32 + off)[i];
-  }
-  if constexpr (EPI == EPI_DGELU) {
-#pragma unroll
-    for (int i = 0; i < 2; ++i) p.z[i] = reinterpret_cast<const uint4*>(ep.aux16 + off)[i];
-  }
+// Epilogue EPI on 4 consecutive output columns (row-major element offset `off`, column
+// `col`): the operands it reads (bias, residual, fp32 master, pre-activation) and the
+// outputs it writes are 16-byte (fp32) / 8-byte (bf16) vectors.
+__device__ __forceinline__ uint2 pack4_bf16(float4 v) {
+  return make_uint2(ptx::pack_bf16(v.x, v.y), ptx::pack_bf16(v.z, v.w));
 }
-
-// Apply epilogue EPI to 16 consecutive accumulator columns (row, col..col+15), N = ld.
+__device__ __forceinline__ float bf_lo(float v) { return v - __bfloat162float(__float2bfloat16_rn(v)); }
+// Per-element operand of the epilogue (residual / fp32 master / pre-activation bits), loaded
+// for all of a lane's rows before any store of the chunk so the loads overlap each other and
+// the TMEM read (the compiler cannot hoist them across stores it cannot disambiguate).
 template <int EPI>
-__device__ __forceinline__ void epilogue16(float (&v)[16], const Pre16& pre, size_t off, int col,
-                                           const GemmEpiParams& ep, int split) {
+__device__ __forceinline__ float4 preload4(size_t off, const GemmEpiParams& ep) {
+  if constexpr (EPI == EPI_BIAS_RESID_F32) return *reinterpret_cast<const float4*>(ep.resid + off);
+  if constexpr (EPI == EPI_SGD) return *reinterpret_cast<const float4*>(ep.w32 + off);
+  if constexpr (EPI == EPI_DGELU) {
+    const uint2 z = *reinterpret_cast<const uint2*>(ep.aux16 + off);
+    return make_float4(__uint_as_float(z.x), __uint_as_float(z.y), 0.f, 0.f);
+  }
+  return make_float4(0.f, 0.f, 0.f, 0.f);
+}
+template <int EPI>
+__device__ __forceinline__ void epilogue4(float4 v, float4 pre, float4 b, size_t off, const GemmEpiParams& ep,
+                                          int split) {
   if constexpr (EPI == EPI_PARTIAL) {
-    store16_f32(ep.ws + (size_t)split * ep.ws_stride + off, v);
+    *reinterpret_cast<float4*>(ep.ws + (size_t)split * ep.ws_stride + off) = v;
     return;
   }
   if constexpr (EPI == EPI_BIAS_BF16 || EPI == EPI_BIAS_RESID_F32 || EPI == EPI_BIAS_GELU) {
-    const float4* b4 = reinterpret_cast<const float4*>(ep.bias + col);
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      const float4 b = b4[i];
-      v[4 * i] += b.x; v[4 * i + 1] += b.y; v[4 * i + 2] += b.z; v[4 * i + 3] += b.w;
-    }
+    v.x += b.x; v.y += b.y; v.z += b.z; v.w += b.w;
   }
   if constexpr (EPI == EPI_BIAS_RESID_F32) {
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      v[4 * i] += pre.q[i].x; v[4 * i + 1] += pre.q[i].y; v[4 * i + 2] += pre.q[i].z; v[4 * i + 3] += pre.q[i].w;
-    }
+    v.x += pre.x; v.y += pre.y; v.z += pre.z; v.w += pre.w;
   }
   if constexpr (EPI == EPI_DGELU) {
-#pragma unroll
-    for (int i = 0; i < 2; ++i) {
-      const bf16* zz = reinterpret_cast<const bf16*>(&pre.z[i]);
-#pragma unroll
-      for (int j = 0; j < 8; ++j) v[8 * i + j] *= gelu_tanh_grad(__bfloat162float(zz[j]));
-    }
+    const uint2 zz = make_uint2(__float_as_uint(pre.x), __float_as_uint(pre.y));
+    const bf16* z = reinterpret_cast<const bf16*>(&zz);
+    v.x *= gelu_tanh_grad(__bfloat162float(z[0]));
+    v.y *= gelu_tanh_grad(__bfloat162float(z[1]));
+    v.z *= gelu_tanh_grad(__bfloat162float(z[2]));
+    v.w *= gelu_tanh_grad(__bfloat162float(z[3]));
   }
   if constexpr (EPI == EPI_F32 || EPI == EPI_BIAS_RESID_F32) {
-    store16_f32(reinterpret_cast<float*>(ep.out) + off, v);
+    *reinterpret_cast<float4*>(reinterpret_cast<float*>(ep.out) + off) = v;
   } else if constexpr (EPI == EPI_X2) {
-    float lo[16];
-#pragma unroll
-    for (int i = 0; i < 16; ++i) lo[i] = v[i] - __bfloat162float(__float2bfloat16_rn(v[i]));
-    store16_bf16(reinterpret_cast<bf16*>(ep.out) + off, v);
-    store16_bf16(ep.out2 + off, lo);
+    *reinterpret_cast<uint2*>(reinterpret_cast<bf16*>(ep.out) + off) = pack4_bf16(v);
+    *reinterpret_cast<uint2*>(ep.out2 + off) = pack4_bf16(make_float4(bf_lo(v.x), bf_lo(v.y), bf_lo(v.z), bf_lo(v.w)));
   } else if constexpr (EPI == EPI_SGD) {
-    float w[16];
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      float4 x = pre.q[i];
-      x.x -= ep.lr * v[4 * i]; x.y -= ep.lr * v[4 * i + 1];
-      x.z -= ep.lr * v[4 * i + 2]; x.w -= ep.lr * v[4 * i + 3];
-      reinterpret_cast<float4*>(ep.w32 + off)[i] = x;
-      w[4 * i] = x.x; w[4 * i + 1] = x.y; w[4 * i + 2] = x.z; w[4 * i + 3] = x.w;
-    }
-    store16_bf16(ep.w16 + off, w);
-    if (ep.w16lo) {
-#pragma unroll
-      for (int i = 0; i < 16; ++i) w[i] -= __bfloat162float(__float2bfloat16_rn(w[i]));
-      store16_bf16(ep.w16lo + off, w);
-    }
+    float4 w = pre;
+    w.x -= ep.lr * v.x; w.y -= ep.lr * v.y; w.z -= ep.lr * v.z; w.w -= ep.lr * v.w;
+    *reinterpret_cast<float4*>(ep.w32 + off) = w;
+    *reinterpret_cast<uint2*>(ep.w16 + off) = pack4_bf16(w);
+    if (ep.w16lo)
+      *reinterpret_cast<uint2*>(ep.w16lo + off) =
+          pack4_bf16(make_float4(bf_lo(w.x), bf_lo(w.y), bf_lo(w.z), bf_lo(w.w)));
   } else {
-    store16_bf16(reinterpret_cast<bf16*>(ep.out) + off, v);
-    if constexpr (EPI == EPI_BIAS_GELU) {
-      float g[16];
-#pragma unroll
-      for (int i = 0; i < 16; ++i) g[i] = gelu_tanh(v[i]);
-      store16_bf16(ep.out2 + off, g);
+    *reinterpret_cast<uint2*>(reinterpret_cast<bf16*>(ep.out) + off) = pack4_bf16(v);
+    if constexpr (EPI == EPI_BIAS_GELU)
+      *reinterpret_cast<uint2*>(ep.out2 + off) =
+          pack4_bf16(make_float4(gelu_tanh(v.x), gelu_tanh(v.y), gelu_tanh(v.z), gelu_tanh(v.w)));
+  }
+}
+
+// One epilogue warp's share of an accumulator tile: rows row0..row0+31 (its TMEM lane
+// quarter, `taddr` = lane base | column base), tile columns [cbeg, cend) at output column
+// n0 + c.  Chunks of EC columns go TMEM -> registers (thread = row) -> the warp's padded
+// staging buffer `stg` [32][EC+4] -> registers (EC/4 lanes per row, float4 each) so that
+// every global load/store of the epilogue is a coalesced row segment of 4*EC (fp32) or
+// 2*EC (bf16) bytes, instead of 32 rows x 16 bytes per instruction.  The padding makes
+// both staging passes bank-conflict free.
+template <int EPI, int EC>
+__device__ __forceinline__ void epilogue_warp(uint32_t taddr, float* stg, int row0, int cbeg, int cend, int n0,
+                                              int M, int N, const GemmEpiParams& ep, int split, int lane) {
+  constexpr int LD = EC + 4, LPR = EC / 4, RPI = 32 / LPR, NIT = 32 / RPI;
+  constexpr bool HAS_PRE = EPI == EPI_BIAS_RESID_F32 || EPI == EPI_SGD || EPI == EPI_DGELU;
+  constexpr bool HAS_BIAS = EPI == EPI_BIAS_BF16 || EPI == EPI_BIAS_RESID_F32 || EPI == EPI_BIAS_GELU;
+  const int cc = (lane % LPR) * 4;
+#pragma unroll 1
+  for (int c0 = cbeg; c0 < cend; c0 += EC) {
+    const int col = n0 + c0;
+    if (col >= N) break;  // warp-uniform
+    const int gcol = col + cc;
+    float4 pre[NIT], b = make_float4(0.f, 0.f, 0.f, 0.f);
+    if constexpr (HAS_BIAS) {
+      if (gcol < N) b = *reinterpret_cast<const float4*>(ep.bias + gcol);
     }
+#pragma unroll
+    for (int it = 0; it < NIT; ++it) {
+      const int grow = row0 + it * RPI + lane / LPR;
+      pre[it] = make_float4(0.f, 0.f, 0.f, 0.f);
+      if constexpr (HAS_PRE) {
+        if (grow < M && gcol < N) pre[it] = preload4<EPI>((size_t)grow * N + gcol, ep);
+      }
+    }
+    uint32_t r[EC];
+    if constexpr (EC == 32) ptx::tmem_ld32(taddr + c0, r);
+    else ptx::tmem_ld16(taddr + c0, r);
+    ptx::tmem_ld_wait();
+#pragma unroll
+    for (int j = 0; j < EC / 4; ++j)
+      *reinterpret_cast<float4*>(stg + lane * LD + 4 * j) =
+          make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]), __uint_as_float(r[4 * j + 2]),
+                      __uint_as_float(r[4 * j + 3]));
+    __syncwarp();
+#pragma unroll
+    for (int it = 0; it < NIT; ++it) {
+      const int rr = it * RPI + lane / LPR;
+      const int grow = row0 + rr;
+      const float4 v = *reinterpret_cast<const float4*>(stg + rr * LD + cc);
+      if (grow < M && gcol < N) epilogue4<EPI>(v, pre[it], b, (size_t)grow * N + gcol, ep, split);
+    }
+    __syncwarp();
   }
 }
 
@@ -186,6 +215,7 @@ __global__ void __launch_bounds__(THREADS, 1)
   uint64_t* tfull = empty + STAGES;  // [2]
   uint64_t* tempty = tfull + 2;      // [2]
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(tempty + 2);
+  float* stg = reinterpret_cast<float*>(smem + Cf::STG_OFF);  // [8 warps][32][20]
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int n_tiles = ts.MT * ts.NT * ts.splits;
@@ -300,34 +330,9 @@ __global__ void __launch_bounds__(THREADS, 1)
       ptx::mbar_wait(&tfull[acc], (it >> 1) & 1);
       ptx::tc_fence_after();
       if (t + (int)gridDim.x >= n_tiles) ptx::pdl_trigger();  // last tile: let the next kernel launch
-      const int row = tm * BM + lane_base + lane;
-      const bool row_ok = row < M;
       const uint32_t taddr = tmem + ((uint32_t)lane_base << 16) + acc * TN;
-#pragma unroll 1
-      for (int c0 = cbeg; c0 < cbeg + TN / 2; c0 += 32) {
-        const int col = tn * TN + c0;
-        if (col >= N) break;               // warp-uniform
-        const bool two = col + 16 < N;     // N % 16 == 0: the chunk is 16 or 32 columns
-        const size_t off = (size_t)row * N + col;
-        Pre16 p0, p1;
-        if (row_ok) {
-          preload16<EPI>(p0, off, ep);
-          if (two) preload16<EPI>(p1, off + 16, ep);
-        }
-        uint32_t r[32];
-        ptx::tmem_ld32(taddr + c0, r);
-        ptx::tmem_ld_wait();
-        if (!row_ok) continue;
-        float v[16];
-#pragma unroll
-        for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
-        epilogue16<EPI>(v, p0, off, col, ep, ks);
-        if (two) {
-#pragma unroll
-          for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[16 + i]);
-          epilogue16<EPI>(v, p1, off + 16, col + 16, ep, ks);
-        }
-      }
+      epilogue_warp<EPI, 16>(taddr, stg + (warp - 2) * 32 * 20, tm * BM + lane_base, cbeg, cbeg + TN / 2, tn * TN, M,
+                             N, ep, ks, lane);
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(&tempty[acc]);
@@ -337,6 +342,154 @@ __global__ void __launch_bounds__(THREADS, 1)
   if (warp == 1) {
     ptx::tc_fence_after();
     ptx::tmem_dealloc<Cf::TMEM_COLS>(tmem);
+  }
+}
+
+// CTA-pair variant (cta_group::2): a 2-CTA cluster on one TPC computes a 256 x 256 output
+// tile.  CTA r loads rows [m0 + 128r, +128) of A and rows [n0 + 128r, +128) of B (the B
+// half), i.e. 32 KB per 64-deep K block instead of the 48 KB a single CTA needs for its
+// 128 x 256 tile: the operand traffic from L2 per flop drops by a third, which is what
+// bounds the 1-CTA kernel on the step's shapes (its tensor pipe idles ~55 % of the active
+// time waiting for TMA; profiles/r1_ncu_full_prof_gemm_tf.csv).  The leader (rank 0) issues
+// the M=256 MMAs reading both CTAs' stages; its commits arrive on the `empty` / `tfull`
+// barriers of both CTAs (multicast); both producers' TMA completions land on the leader's
+// `full` barrier; both CTAs' epilogue warps release the leader's `tempty` barrier.  Each
+// CTA's TMEM holds the accumulator of its own 128 rows, so the epilogue is the 1-CTA one.
+// Same tile-to-K order per output element as the 1-CTA kernel: bitwise reproducible.
+constexpr int PAIR_STAGE_BYTES = A_BYTES + 128 * BK * 2;  // 32 KB per CTA
+constexpr int PAIR_STAGES = 5;
+constexpr int PAIR_BAR_OFF = PAIR_STAGES * PAIR_STAGE_BYTES;
+constexpr int PAIR_STG_OFF = PAIR_BAR_OFF + (2 * PAIR_STAGES + 4) * 8 + 16;
+constexpr int PAIR_SMEM_TOTAL = PAIR_STG_OFF + 8 * 32 * 36 * 4 + 1024;
+
+template <bool A_MN, bool B_MN, int EPI>
+__global__ void __launch_bounds__(THREADS, 1)
+    gemm_pair_kernel(const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb, int M, int N,
+                     TileSpace ts, GemmEpiParams ep) {
+  constexpr int TN = 256, STAGES = PAIR_STAGES, STAGE_BYTES = PAIR_STAGE_BYTES;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + PAIR_BAR_OFF);
+  uint64_t* empty = full + STAGES;
+  uint64_t* tfull = empty + STAGES;  // [2]
+  uint64_t* tempty = tfull + 2;      // [2]
+  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(tempty + 2);
+  float* stg = reinterpret_cast<float*>(smem + PAIR_STG_OFF);  // [8 warps][32][36]
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = ptx::cluster_ctarank();
+  const int pair = blockIdx.x >> 1, n_pairs = gridDim.x >> 1;
+  const int n_tiles = ts.MT * ts.NT * ts.splits;
+
+  if (threadIdx.x == 0) {
+    ptx::tma_prefetch(&ta);
+    ptx::tma_prefetch(&tb);
+    for (int s = 0; s < STAGES; ++s) {
+      ptx::mbar_init(&full[s], 1);
+      ptx::mbar_init(&empty[s], 1);
+    }
+    for (int a = 0; a < 2; ++a) {
+      ptx::mbar_init(&tfull[a], 1);
+      ptx::mbar_init(&tempty[a], 16);  // 8 epilogue warps x 2 CTAs (only the leader's is used)
+    }
+    ptx::fence_mbar_init();
+  }
+  if (warp == 1) ptx::tmem_alloc_pair<512>(tmem_holder);
+  ptx::tc_fence_before();
+  ptx::cluster_sync();  // barriers of both CTAs initialised, TMEM allocated
+  ptx::tc_fence_after();
+  const uint32_t tmem = *tmem_holder;
+  ptx::pdl_wait();
+
+  if (warp == 0) {
+    if (lane == 0) {  // ---------------- TMA producer (both CTAs)
+      int s = 0, ph = 0;
+      for (int t = pair; t < n_tiles; t += n_pairs) {
+        int tm, tn, ks;
+        ts.decode(t, tm, tn, ks);
+        const int m0 = tm * 256 + 128 * (int)rank, n0 = tn * TN + 128 * (int)rank;
+        const int kb0 = ks * ts.nk_per_split, kb1 = min(ts.nk, kb0 + ts.nk_per_split);
+        for (int kb = kb0; kb < kb1; ++kb) {
+          ptx::mbar_wait(&empty[s], ph ^ 1);
+          uint8_t* sa = smem + s * STAGE_BYTES;
+          uint8_t* sb = sa + A_BYTES;
+          const uint32_t fb = ptx::mapa(ptx::smem_u32(&full[s]), 0);
+          if (rank == 0) ptx::mbar_arrive_expect_tx(&full[s], 2 * STAGE_BYTES);
+          const int k0 = kb * BK;
+          if (!A_MN) {
+            ptx::tma_load_2d_pair(sa, &ta, fb, k0, m0);
+          } else {
+            ptx::tma_load_2d_pair(sa, &ta, fb, m0, k0);
+            ptx::tma_load_2d_pair(sa + 8192, &ta, fb, m0 + 64, k0);
+          }
+          if (!B_MN) {
+            ptx::tma_load_2d_pair(sb, &tb, fb, k0, n0);
+          } else {
+            ptx::tma_load_2d_pair(sb, &tb, fb, n0, k0);
+            ptx::tma_load_2d_pair(sb + 8192, &tb, fb, n0 + 64, k0);
+          }
+          if (++s == STAGES) { s = 0; ph ^= 1; }
+        }
+      }
+    }
+    ptx::pdl_trigger();
+  } else if (warp == 1) {
+    if (lane == 0 && rank == 0) {  // ---------------- MMA issuer (leader only)
+      constexpr uint32_t idesc = ptx::umma_idesc_bf16(256, TN, A_MN ? 1 : 0, B_MN ? 1 : 0);
+      int s = 0, ph = 0, it = 0;
+      for (int t = pair; t < n_tiles; t += n_pairs, ++it) {
+        int tm, tn, ks;
+        ts.decode(t, tm, tn, ks);
+        const int kb0 = ks * ts.nk_per_split, kb1 = min(ts.nk, kb0 + ts.nk_per_split);
+        const int acc = it & 1;
+        ptx::mbar_wait_cluster(&tempty[acc], ((it >> 1) & 1) ^ 1);  // both CTAs drained this buffer
+        ptx::tc_fence_after();
+        const uint32_t d = tmem + acc * TN;
+        for (int kb = kb0; kb < kb1; ++kb) {
+          ptx::mbar_wait(&full[s], ph);
+          ptx::tc_fence_after();
+          const uint32_t sa = ptx::smem_u32(smem + s * STAGE_BYTES);
+          const uint32_t sb = sa + A_BYTES;
+#pragma unroll
+          for (int k = 0; k < BK / 16; ++k) {
+            const uint64_t ad = A_MN ? ptx::umma_desc_sw128(sa + k * 2048, 8192, 1024)
+                                     : ptx::umma_desc_sw128(sa + k * 32, 16, 1024);
+            const uint64_t bd = B_MN ? ptx::umma_desc_sw128(sb + k * 2048, 8192, 1024)
+                                     : ptx::umma_desc_sw128(sb + k * 32, 16, 1024);
+            ptx::umma_bf16_pair(d, ad, bd, idesc, (kb > kb0 || k > 0) ? 1u : 0u);
+          }
+          ptx::umma_commit_pair(&empty[s], 0x3);  // frees this stage in both CTAs
+          if (++s == STAGES) { s = 0; ph ^= 1; }
+        }
+        ptx::umma_commit_pair(&tfull[acc], 0x3);  // both CTAs' accumulators ready
+      }
+    }
+    ptx::pdl_trigger();
+  } else {
+    // ---------------- epilogue warps 2..9 of both CTAs: this CTA's 128 rows
+    const int lane_base = 32 * (warp & 3);
+    const int cbeg = ((warp - 2) >> 2) * (TN / 2);
+    int it = 0;
+    for (int t = pair; t < n_tiles; t += n_pairs, ++it) {
+      int tm, tn, ks;
+      ts.decode(t, tm, tn, ks);
+      const int acc = it & 1;
+      ptx::mbar_wait(&tfull[acc], (it >> 1) & 1);
+      ptx::tc_fence_after();
+      if (t + n_pairs >= n_tiles) ptx::pdl_trigger();
+      const uint32_t taddr = tmem + ((uint32_t)lane_base << 16) + acc * TN;
+      epilogue_warp<EPI, 32>(taddr, stg + (warp - 2) * 32 * 36, tm * 256 + 128 * (int)rank + lane_base, cbeg,
+                             cbeg + TN / 2, tn * TN, M, N, ep, ks, lane);
+      ptx::tc_fence_before();
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive_cluster(ptx::mapa(ptx::smem_u32(&tempty[acc]), 0));
+    }
+  }
+  __syncthreads();
+  ptx::cluster_sync();  // no remote arrive / MMA operand read is still in flight
+  if (warp == 1) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc_pair<512>(tmem);
   }
 }
 
@@ -454,6 +607,64 @@ void launch(cudaStream_t s, int M, int N, const TileSpace& ts, const CUtensorMap
   g_gemm_launches.fetch_add(1, std::memory_order_relaxed);
 }
 
+template <bool A_MN, bool B_MN, int EPI>
+void launch_pair(cudaStream_t s, int M, int N, const TileSpace& ts, const CUtensorMap& ta, const CUtensorMap& tb,
+                 const GemmEpiParams& ep) {
+  auto kern = gemm_pair_kernel<A_MN, B_MN, EPI>;
+  static uint32_t configured = 0;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (!(configured & (1u << dev))) {
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, PAIR_SMEM_TOTAL);
+    cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+    configured |= 1u << dev;
+  }
+  const int tiles = ts.MT * ts.NT * ts.splits;
+  const int pairs = std::min(tiles, num_sms() / 2);
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(2 * pairs);
+  cfg.blockDim = dim3(THREADS);
+  cfg.dynamicSmemBytes = PAIR_SMEM_TOTAL;
+  cfg.stream = s;
+  cudaLaunchAttribute at[2];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  at[1].id = cudaLaunchAttributeClusterDimension;
+  at[1].val.clusterDim.x = 2;
+  at[1].val.clusterDim.y = 1;
+  at[1].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 2;
+  const cudaError_t e = cudaLaunchKernelEx(&cfg, kern, ta, tb, M, N, ts, ep);
+  NP_REQUIRE(e == cudaSuccess, NASPIPE_ECUDA, "pair GEMM launch: %s", cudaGetErrorString(e));
+  g_gemm_launches.fetch_add(1, std::memory_order_relaxed);
+}
+
+template <bool A_MN, bool B_MN>
+void dispatch_pair(cudaStream_t s, int M, int N, const TileSpace& ts, const CUtensorMap& ta, const CUtensorMap& tb,
+                   int epi, const GemmEpiParams& ep) {
+  switch (epi) {
+    case EPI_BF16: return launch_pair<A_MN, B_MN, EPI_BF16>(s, M, N, ts, ta, tb, ep);
+    case EPI_F32: return launch_pair<A_MN, B_MN, EPI_F32>(s, M, N, ts, ta, tb, ep);
+    case EPI_BIAS_BF16: return launch_pair<A_MN, B_MN, EPI_BIAS_BF16>(s, M, N, ts, ta, tb, ep);
+    case EPI_BIAS_RESID_F32: return launch_pair<A_MN, B_MN, EPI_BIAS_RESID_F32>(s, M, N, ts, ta, tb, ep);
+    case EPI_BIAS_GELU: return launch_pair<A_MN, B_MN, EPI_BIAS_GELU>(s, M, N, ts, ta, tb, ep);
+    case EPI_DGELU: return launch_pair<A_MN, B_MN, EPI_DGELU>(s, M, N, ts, ta, tb, ep);
+    case EPI_SGD: return launch_pair<A_MN, B_MN, EPI_SGD>(s, M, N, ts, ta, tb, ep);
+    case EPI_PARTIAL: return launch_pair<A_MN, B_MN, EPI_PARTIAL>(s, M, N, ts, ta, tb, ep);
+    default: NP_REQUIRE(false, NASPIPE_EINVAL, "bad epilogue %d", epi);
+  }
+}
+
+bool pair_enabled() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("NASPIPE_GEMM_PAIR");
+    v = (e && e[0] == '0') ? 0 : 1;
+  }
+  return v == 1;
+}
+
 template <bool A_MN, bool B_MN>
 void dispatch_epi(cudaStream_t s, int M, int N, const TileSpace& ts, const CUtensorMap& ta, const CUtensorMap& tb,
                   int epi, const GemmEpiParams& ep) {
@@ -474,10 +685,16 @@ void dispatch_epi(cudaStream_t s, int M, int N, const TileSpace& ts, const CUten
 
 uint64_t gemm_launch_count() { return g_gemm_launches.load(); }
 
+// The CTA-pair kernel serves every GEMM with M, N >= 256 (the transformer's and the SPOS
+// head's); smaller ones (SPOS 1x1 convs with N < 256, the 3-pass product) use 1-CTA tiles.
+bool gemm_uses_pair(int M, int N) { return pair_enabled() && M >= 256 && N >= 256; }
+
 int gemm_splitk_factor(int M, int N, int K) {
-  const int tiles = ((M + BM - 1) / BM) * ((N + BN - 1) / BN);
+  const bool pair = gemm_uses_pair(M, N);
+  const int bm = pair ? 2 * BM : BM;
+  const int tiles = ((M + bm - 1) / bm) * ((N + BN - 1) / BN);
   const int nk = (K + BK - 1) / BK;
-  const int sms = num_sms();
+  const int sms = pair ? num_sms() / 2 : num_sms();
   // cost in k-block rounds (~0.3 us each): rounds * k-blocks per round, plus the fp32
   // round trip of the split-K reduction ((s + 2.5) * M * N * 4 bytes at ~6 TB/s)
   auto cost = [&](int s) {
@@ -495,12 +712,13 @@ void gemm_bf16_tc(cudaStream_t s, int M, int N, int K, const bf16* A, bool a_mn,
                   bool b_mn, int ldb, int epi, const GemmEpiParams& ep_in) {
   NP_REQUIRE(M > 0 && N > 0 && K > 0 && N % 16 == 0, NASPIPE_EINVAL, "gemm dims M=%d N=%d K=%d (N%%16)", M, N, K);
   GemmEpiParams ep = ep_in;
+  const bool pair = gemm_uses_pair(M, N);
   const CUtensorMap ta = a_mn ? make_map(A, (uint64_t)M, (uint64_t)K, (uint64_t)lda, BK)
                               : make_map(A, (uint64_t)K, (uint64_t)M, (uint64_t)lda, BM);
   const CUtensorMap tb = b_mn ? make_map(B, (uint64_t)N, (uint64_t)K, (uint64_t)ldb, BK)
-                              : make_map(B, (uint64_t)K, (uint64_t)N, (uint64_t)ldb, BN);
+                              : make_map(B, (uint64_t)K, (uint64_t)N, (uint64_t)ldb, pair ? BN / 2 : BN);
   TileSpace ts;
-  ts.MT = (M + BM - 1) / BM;
+  ts.MT = (M + (pair ? 2 * BM : BM) - 1) / (pair ? 2 * BM : BM);
   ts.NT = (N + BN - 1) / BN;
   ts.nk = (K + BK - 1) / BK;
   ts.splits = 1;
@@ -511,7 +729,12 @@ void gemm_bf16_tc(cudaStream_t s, int M, int N, int K, const bf16* A, bool a_mn,
   ts.nk_per_split = (ts.nk + ts.splits - 1) / ts.splits;
   const int run_epi = ts.splits > 1 ? EPI_PARTIAL : epi;
   ep.ws_stride = (size_t)M * N;
-  if (!a_mn && !b_mn) dispatch_epi<false, false>(s, M, N, ts, ta, tb, run_epi, ep);
+  if (pair) {
+    if (!a_mn && !b_mn) dispatch_pair<false, false>(s, M, N, ts, ta, tb, run_epi, ep);
+    else if (!a_mn && b_mn) dispatch_pair<false, true>(s, M, N, ts, ta, tb, run_epi, ep);
+    else if (a_mn && b_mn) dispatch_pair<true, true>(s, M, N, ts, ta, tb, run_epi, ep);
+    else dispatch_pair<true, false>(s, M, N, ts, ta, tb, run_epi, ep);
+  } else if (!a_mn && !b_mn) dispatch_epi<false, false>(s, M, N, ts, ta, tb, run_epi, ep);
   else if (!a_mn && b_mn) dispatch_epi<false, true>(s, M, N, ts, ta, tb, run_epi, ep);
   else if (a_mn && b_mn) dispatch_epi<true, true>(s, M, N, ts, ta, tb, run_epi, ep);
   else dispatch_epi<true, false>(s, M, N, ts, ta, tb, run_epi, ep);

@@ -56,7 +56,8 @@ def _gemm(M, N, K, A, a_mn, B, b_mn, epi, **kw):
     torch.cuda.synchronize()
 
 
-SHAPES = [(128, 128, 64), (256, 384, 512), (304, 208, 200), (4096, 1024, 1024), (256, 512, 4096)]  # last: split-K
+SHAPES = [(128, 128, 64), (256, 384, 512), (304, 208, 200), (304, 272, 192), (4096, 1024, 1024),
+          (256, 512, 4096)]  # M, N >= 256: CTA-pair kernel (ragged: 304 x 272); last: split-K
 
 
 @pytest.mark.parametrize("M,N,K", SHAPES)

@@ -16,18 +16,22 @@ L.naspipe_debug_gemm.argtypes = [C.c_int] * 3 + [_vp, C.c_int, C.c_int, _vp, C.c
                                                  _vp, _vp, _vp, _vp, _vp, _vp, _vp, C.c_float, _vp]
 
 
-def bench(fn, reps=20):
+def bench(fn, reps=5, inner=20):
+    """Median over `reps` of the mean time of `inner` back-to-back calls (the host enqueues
+    ahead of the GPU, as in a training step, so host-side launch cost is not timed)."""
     for _ in range(3):
         fn()
     torch.cuda.synchronize()
     ts = []
     for _ in range(reps):
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda._sleep(2_000_000)  # keep the GPU busy while the host enqueues the calls
         a.record()
-        fn()
+        for _ in range(inner):
+            fn()
         b.record()
         torch.cuda.synchronize()
-        ts.append(a.elapsed_time(b))
+        ts.append(a.elapsed_time(b) / inner)
     ts.sort()
     return ts[len(ts) // 2]
 
