@@ -8,11 +8,14 @@ SGD WRITE of every active candidate on every stage) on one synthetic batch.  N =
 whole supernet as one stage on one GPU; N > 1 (torchrun, one process per GPU) runs an
 N-stage CSP pipeline with NCCL send/recv between stages.
 
+Default workload: configs[1] (SPOS CNN supernet, 20 blocks x 4 choices, 224x224, batch 64).
 Printed by rank 0 as ONE JSON line: value = samples/s of the whole job with the inputs
 already resident in HBM (device batches); e2e = the same through the C ABI with pinned HOST
 buffers (H2D of input+target inside the timed region, D2H of the step losses);
-roofline = the tcgen05 GEMM (the dominant kernel) timed by CUDA events on its stream;
-cpu_baseline = the fp64 NumPy oracle on a bounded sample, on this host's cores.
+roofline = the dominant kernel timed by CUDA events on its stream (SPOS: the BatchNorm
+kernels against HBM bandwidth; transformer: the tcgen05 GEMM against bf16 peak);
+cpu_baseline = the fp64 NumPy oracle on a bounded sample, on this host's cores;
+secondary = the configs[2] transformer (the tensor-core path) measured the same way.
 """
 import argparse
 import json
@@ -33,12 +36,13 @@ import synth  # noqa: E402
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=12)
+    ap.add_argument("--steps", type=int, default=40)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--workload", default="transformer")
+    ap.add_argument("--workload", default="spos")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-secondary", action="store_true", help="skip the configs[2] line embedded in the output")
     ap.add_argument("--budget-x", type=float, default=0.0,
                     help="HBM weight budget per stage as a multiple of one subnet's mean stage slice "
                          "(0 = all candidates resident; P:L337 uses ~3)")
@@ -69,7 +73,7 @@ def peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+    """nvidia-smi clocks + throttle reasons sampled every 100 ms during the timed region."""
     Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
          "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
 
@@ -79,7 +83,7 @@ class ClockSampler:
     def __enter__(self):
         try:
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.Q}",
-                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
@@ -139,7 +143,7 @@ def oracle_block_sample(cfg, n_blocks_sample):
 def sample_size(cfg):
     """(sample units, units per subnet, description) of the bounded oracle sample."""
     if cfg["family"] == "spos":
-        return 4, cfg["batch"], "images"
+        return 16, cfg["batch"], "images"
     if cfg["family"] == "transformer":
         return (2 if cfg["d_model"] <= 1024 else 1), cfg["n_blocks"], "blocks"
     return cfg["n_blocks"], cfg["n_blocks"], "blocks"
@@ -169,6 +173,8 @@ def run_reference(args, cfg, rank, world):
     ns, per, unit = sample_size(cfg)
     if cfg["family"] == "transformer":
         ns = 1
+    if cfg["family"] == "spos":
+        ns = 2   # ~1 s of oracle work per step: the default K/W run ends within a few minutes
     for _ in range(args.warmup):
         oracle_block_sample(cfg, ns)
     ts = [oracle_block_sample(cfg, ns) for _ in range(args.steps)]
@@ -184,6 +190,30 @@ def run_reference(args, cfg, rank, world):
         "config": workload_config(args, cfg, world),
         "cpu_baseline": {"kind": "oracle", "cores": cores, "sample": sample, "value": value, "unit": "samples/s"},
         "e2e": {"value": value, "unit": "samples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}))
+
+
+def _traffic(family):
+    """dram bytes per launch of the dominant kernel from the committed ncu --set full summary."""
+    p = os.path.join(ROOT, "profiles", "dominant_traffic.json")
+    if not os.path.exists(p):
+        return None
+    with open(p) as f:
+        d = json.load(f).get(family)
+    return None if d is None else {"dram_bytes_per_launch": d["dram_bytes_per_launch_mean"],
+                                   "source": "profiles/dominant_traffic.json (ncu --set full capture)"}
+
+
+def secondary(args):
+    """configs[2] (transformer, the tensor-core path) measured in a child process, reported
+    beside the headline configs[1] line."""
+    cmd = [sys.executable, os.path.join(ROOT, "bench.py"), "--workload", "transformer", "--steps", str(args.steps),
+           "--warmup", str(args.warmup), "--no-cpu", "--no-e2e", "--no-secondary"]
+    try:
+        out = subprocess.run(cmd, capture_output=True, text=True, timeout=300).stdout.strip().splitlines()
+        d = json.loads(out[-1])
+        return {k: d[k] for k in ("value", "unit", "ms_per_step", "config", "roofline", "clocks", "gpu_launches")}
+    except Exception as e:  # reported, never fatal for the headline line
+        return {"error": repr(e)[:200]}
 
 
 def workload_config(args, cfg, world):
@@ -213,6 +243,11 @@ def main():
     if args.impl == "reference":
         run_reference(args, cfg, rank, world)
         return
+    # the configs[2] line runs in a child process BEFORE this process touches the GPU (a
+    # child started while the parent holds a CUDA context stalled on the box)
+    sec = None
+    if world == 1 and args.workload == "spos" and not args.no_secondary and not args.n_choices:
+        sec = secondary(args)
 
     import torch
     import torch.distributed as dist
@@ -223,14 +258,14 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     D = world
     m, n, B = cfg["n_blocks"], cfg["n_choices"], cfg["batch"]
-    total = args.warmup + 2 * args.steps
+    total = args.warmup + 3 * args.steps
     choices = synth.sample_choices(total, m, n)
     # device-resident input pool (value run) and pinned host pool (e2e run)
     pool = [synth.make_batch(cfg, y) for y in range(4)]
     dev_pool = [(torch.from_numpy(x).cuda(), torch.from_numpy(t).cuda()) for x, t in pool]
     host_pool = [(torch.from_numpy(x).pin_memory(), torch.from_numpy(t).pin_memory()) for x, t in pool]
     budget = stage_budget(cfg, D, args.budget_x, npipe) if args.budget_x > 0 else 0
-    spec = npipe.Spec(cfg, flags=npipe.FLAG_TIMING, hbm_weight_budget_bytes=budget, lookahead=args.lookahead)
+    spec = npipe.Spec(cfg, hbm_weight_budget_bytes=budget, lookahead=args.lookahead)
     if world == 1:
         h = npipe.naspipe_create(spec, 1)
     else:
@@ -262,6 +297,9 @@ def main():
     # ---- timed region 1: inputs resident in HBM
     s0 = npipe.naspipe_get_stats(h)
     barrier()
+    prof = os.environ.get("NASPIPE_PROFILE_RANGE") == "1"   # ncu --profile-from-start off
+    if prof:
+        torch.cuda.profiler.start()
     with ClockSampler(local) as clk:
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         t_wall = time.perf_counter()
@@ -274,32 +312,61 @@ def main():
         e1.record()
         torch.cuda.synchronize()
         t_wall = time.perf_counter() - t_wall
+    if prof:
+        torch.cuda.profiler.stop()
     s1 = npipe.naspipe_get_stats(h)
     # the default-stream events bracket the drain (host waits for every stage stream), so
     # the elapsed time covers all device work of the K steps
     ms = max_over_ranks(e0.elapsed_time(e1))
     value = args.steps * B / (ms / 1000)
 
-    # ---- roofline of the dominant kernel (tcgen05 GEMM), CUDA events on its stream
-    g_flops = s1["dominant_flops"] - s0["dominant_flops"]
-    g_ms = s1["dominant_ms"] - s0["dominant_ms"]
-    g_n = s1["dominant_launches"] - s0["dominant_launches"]
-    pk = peaks()
-    achieved = (g_flops / g_n) / ((g_ms / g_n) / 1000) / 1e12 if g_n else None
-    traffic = None
-    prof = os.path.join(ROOT, "profiles", "gemm_traffic.json")
-    if os.path.exists(prof):
-        with open(prof) as f:
-            traffic = json.load(f).get("dram_bytes_per_launch_by_shape")
-    roofline = {"bound": "tensor", "kernel": "gemm_tc_kernel (tcgen05, all shapes of the step)",
-                "achieved": achieved, "peak": pk["bf16_sustained"], "unit": "TFLOP/s",
-                "frac": achieved / pk["bf16_sustained"] if achieved else None, "traffic": traffic,
-                "peak_source": pk["source"] + " bf16_tflops_sustained (kernel timed inside a long step)",
-                "launches": g_n, "gemm_share_of_step": g_ms / ms if ms else None,
-                "algorithmic_flops_per_step": g_flops / args.steps}
     launches = (s1["kernel_launches"] - s0["kernel_launches"])
 
-    # ---- timed region 2: end to end through the C ABI with pinned host buffers
+    # ---- roofline of the dominant kernel: a second timed region of the same K steps with
+    # CUDA events bracketing each of its launches on its stream (kept out of `value`: the
+    # events cost the kernels' PDL overlap)
+    npipe.naspipe_set_timing(h, True)
+    s2 = npipe.naspipe_get_stats(h)
+    barrier()
+    e0.record()
+    for _ in range(args.steps):
+        x, t = dev_pool[y % 4]
+        npipe.naspipe_submit(h, choices[y], x, t, where=npipe.BATCH_DEVICE)
+        y += 1
+    npipe.naspipe_drain(h)
+    e1.record()
+    torch.cuda.synchronize()
+    ms_timed = max_over_ranks(e0.elapsed_time(e1))
+    s3 = npipe.naspipe_get_stats(h)
+    npipe.naspipe_set_timing(h, False)
+    g_flops = s3["dominant_flops"] - s2["dominant_flops"]
+    g_ms = s3["dominant_ms"] - s2["dominant_ms"]
+    g_n = s3["dominant_launches"] - s2["dominant_launches"]
+    ms_r = ms_timed
+    pk = peaks()
+    if cfg["family"] == "spos":
+        # SPOS: the BatchNorm kernels are the step's dominant family (HBM-bound); work = their
+        # algorithmic bytes, one timed unit = one BN call (stats/apply/bwd)
+        achieved = (g_flops / g_n) / ((g_ms / g_n) / 1000) / 1e9 if g_n else None
+        traffic = _traffic("spos")
+        roofline = {"bound": "hbm", "kernel": "BatchNorm kernels (bn_stats+finalize, bn_apply, "
+                                              "bn_bwd_reduce+finalize, bn_bwd_apply), all units of the step",
+                    "achieved": achieved, "peak": pk["hbm"], "unit": "GB/s",
+                    "frac": achieved / pk["hbm"] if achieved else None, "traffic": traffic,
+                    "peak_source": pk["source"] + " hbm_gbs (copy bandwidth)",
+                    "launches": g_n, "share_of_timed_step": g_ms / ms_r if ms_r else None,
+                    "algorithmic_bytes_per_step": g_flops / args.steps}
+    else:
+        achieved = (g_flops / g_n) / ((g_ms / g_n) / 1000) / 1e12 if g_n else None
+        traffic = _traffic("transformer")
+        roofline = {"bound": "tensor", "kernel": "tcgen05 GEMM (gemm_pair_kernel / gemm_tc_kernel, all shapes)",
+                    "achieved": achieved, "peak": pk["bf16_sustained"], "unit": "TFLOP/s",
+                    "frac": achieved / pk["bf16_sustained"] if achieved else None, "traffic": traffic,
+                    "peak_source": pk["source"] + " bf16_tflops_sustained (kernel timed inside a long step)",
+                    "launches": g_n, "share_of_timed_step": g_ms / ms_r if ms_r else None,
+                    "algorithmic_flops_per_step": g_flops / args.steps}
+
+    # ---- timed region 3: end to end through the C ABI with pinned host buffers
     e2e = None
     if not args.no_e2e:
         barrier()
@@ -338,6 +405,8 @@ def main():
                               "h2d_GBps": (s1["h2d_bytes"] - s0["h2d_bytes"]) / (ms / 1000) / 1e9,
                               "d2h_GBps": (s1["d2h_bytes"] - s0["d2h_bytes"]) / (ms / 1000) / 1e9} if budget else None,
            "loss_finite": bool(losses is None or np.all(np.isfinite(losses)))}
+    if sec is not None:
+        out["secondary"] = {"configs[2] transformer": sec}
     print(json.dumps(out))
 
 

@@ -200,6 +200,12 @@ int naspipe_get_trace(naspipe_t* h, int64_t* dst, size_t cap_tasks, size_t* n_ta
  * [11] writebacks, [12] version checks passed, [13..15] reserved. */
 int naspipe_get_stats(naspipe_t* h, double* dst16);
 
+/* Turn the dominant-kernel CUDA-event timing (stats [6..8]) on or off for the work submitted
+ * from now on (bench.py measures throughput with it off and the roofline with it on: the
+ * events between kernels cost PDL overlap).  Only between a drain and the next submit:
+ * ESTATE otherwise.  The initial state is the spec's NASPIPE_FLAG_TIMING. */
+int naspipe_set_timing(naspipe_t* h, int on);
+
 /* Residency trace: 4 int64 per event (stage, task index, op 0=LOAD/1=EVICT, uid=b*n+c). */
 int naspipe_get_residency_trace(naspipe_t* h, int64_t* dst, size_t cap, size_t* n);
 

@@ -62,6 +62,7 @@ _sig("naspipe_set_params", C.c_int, [C.c_void_p, C.c_int32, C.c_int32, C.POINTER
 _sig("naspipe_get_losses", C.c_int, [C.c_void_p, C.POINTER(C.c_float), C.c_int64])
 _sig("naspipe_get_trace", C.c_int, [C.c_void_p, _i64p, C.c_size_t, C.POINTER(C.c_size_t)])
 _sig("naspipe_get_stats", C.c_int, [C.c_void_p, C.POINTER(C.c_double)])
+_sig("naspipe_set_timing", C.c_int, [C.c_void_p, C.c_int])
 _sig("naspipe_get_residency_trace", C.c_int, [C.c_void_p, _i64p, C.c_size_t, C.POINTER(C.c_size_t)])
 _sig("naspipe_destroy", None, [C.c_void_p])
 _sig("naspipe_param_count", C.c_int, [_SP, C.c_int32, C.c_int32, C.POINTER(C.c_size_t)])
@@ -82,7 +83,7 @@ _sig("naspipe_nccl_unique_id", C.c_int, [C.c_void_p])
 
 EXPORTED_SYMBOLS = [
     "naspipe_create", "naspipe_create_rank", "naspipe_submit", "naspipe_drain", "naspipe_get_params",
-    "naspipe_set_params", "naspipe_get_losses", "naspipe_get_trace", "naspipe_get_stats",
+    "naspipe_set_params", "naspipe_get_losses", "naspipe_get_trace", "naspipe_get_stats", "naspipe_set_timing",
     "naspipe_get_residency_trace", "naspipe_destroy", "naspipe_param_count", "naspipe_default_costs",
     "naspipe_partition", "naspipe_init_params", "naspipe_init_frozen", "naspipe_plan_create", "naspipe_plan_trace",
     "naspipe_plan_makespan", "naspipe_plan_deps", "naspipe_plan_residency", "naspipe_plan_destroy",
@@ -263,6 +264,10 @@ def naspipe_get_stats(h: Handle) -> dict:
     out = (C.c_double * 16)()
     _check(lib.naspipe_get_stats(h.ptr, out))
     return dict(zip(STATS_FIELDS, list(out)))
+
+
+def naspipe_set_timing(h: Handle, on: bool) -> None:
+    _check(lib.naspipe_set_timing(h.ptr, 1 if on else 0))
 
 
 def naspipe_default_costs(spec: Spec):

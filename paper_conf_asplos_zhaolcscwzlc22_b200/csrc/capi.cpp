@@ -281,6 +281,8 @@ int naspipe_get_trace(naspipe_t* h, int64_t* dst, size_t cap_tasks, size_t* n_ta
 
 int naspipe_get_stats(naspipe_t* h, double* dst16) { return ENGINE_CALL(h, e.get_stats(dst16)); }
 
+int naspipe_set_timing(naspipe_t* h, int on) { return ENGINE_CALL(h, e.set_timing(on != 0)); }
+
 int naspipe_get_residency_trace(naspipe_t* h, int64_t* dst, size_t cap, size_t* n) {
   return ENGINE_CALL(h, e.get_residency_trace(dst, cap, n));
 }

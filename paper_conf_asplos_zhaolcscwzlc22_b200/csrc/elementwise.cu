@@ -54,14 +54,6 @@ __global__ void colsum_bf16_kernel(const bf16* __restrict__ X, float* __restrict
   o[1] = make_float4(acc[4], acc[5], acc[6], acc[7]);
 }
 
-__global__ void sgd_partials_kernel(float* __restrict__ p, const float* __restrict__ part, int nblk, int n, float lr) {
-  const int i = blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= n) return;
-  float g = 0.f;
-  for (int j = 0; j < nblk; ++j) g += part[(size_t)j * n + i];
-  p[i] -= lr * g;
-}
-
 // 32 columns x 8 row-groups per block; group g sums partials [g*G, (g+1)*G) in order, the 8
 // group sums are added in group order.
 __global__ void sgd_multi_kernel(SgdJobs jobs) {
@@ -196,9 +188,14 @@ void colsum_bf16(cudaStream_t s, const bf16* X, float* part, int T, int N) {
   check_launch("colsum");
 }
 
+// p -= lr * (fixed-order sum of the nblk partial rows): 8 row groups per column, summed in
+// group order (sgd_multi_kernel), so long partial lists do not serialise on one thread.
 void sgd_from_partials(cudaStream_t s, float* p, const float* part, int nblk, int n, float lr) {
-  sgd_partials_kernel<<<(n + 255) / 256, 256, 0, s>>>(p, part, nblk, n, lr);
-  check_launch("sgd_from_partials");
+  SgdJobs j{};
+  j.lr = lr;
+  j.job[0] = {p, part, nblk, n};
+  j.count = 1;
+  sgd_multi(s, j);
 }
 
 void sgd_multi(cudaStream_t s, const SgdJobs& jobs) {

@@ -513,6 +513,11 @@ void Engine::get_trace(int64_t* dst, size_t cap, size_t* n) {
   }
 }
 
+void Engine::set_timing(bool on) {
+  NP_REQUIRE(drained_ || planner_.n_subnets() == 0, NASPIPE_ESTATE, "set_timing with work in flight");
+  timer_.on = on;
+}
+
 void Engine::get_stats(double* o) {
   NP_REQUIRE(o, NASPIPE_EINVAL, "dst NULL");
   std::fill(o, o + 16, 0.0);

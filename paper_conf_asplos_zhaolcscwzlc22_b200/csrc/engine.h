@@ -51,6 +51,7 @@ class Engine {
   void get_losses(float* dst, int64_t n);
   void get_trace(int64_t* dst, size_t cap, size_t* n);
   void get_stats(double* dst16);
+  void set_timing(bool on);
   void get_residency_trace(int64_t* dst, size_t cap, size_t* n);
   void shutdown();
 

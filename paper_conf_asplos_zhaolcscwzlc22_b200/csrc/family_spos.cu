@@ -182,8 +182,8 @@ class SposFamily : public Family {
       const int H = spec_.raw.image_hw, C0 = spec_.raw.stem_channels;
       const int Po = (int)P(H / 2);
       spos_stem_conv(s, static_cast<const float*>(x_in), w_stem_, stem_z_, B_, H, C0);
-      bn_stats(s, stem_z_, Po, C0, part_, ctr_, stem_mean_, stem_rstd_);
-      bn_apply(s, stem_z_, Po, C0, stem_mean_, stem_rstd_, ones_s_, zeros_s_, 1, stem_y_[slot], C0, (size_t)Po * C0);
+      t_bn_stats(s, stem_z_, Po, C0, stem_mean_, stem_rstd_);
+      t_bn_apply(s, stem_z_, Po, C0, stem_mean_, stem_rstd_, ones_s_, zeros_s_, 1, stem_y_[slot], C0, (size_t)Po * C0);
       counters.launches += 4;
       x = stem_y_[slot];
     }
@@ -234,15 +234,15 @@ class SposFamily : public Family {
     e.out2 = zh_ + (size_t)PL * Ch;
     const bf16* xo = static_cast<const bf16*>(out);
     gemm_x2(s, PL, Ch, Cl, xo, xo + (size_t)PL * Cl, Cl, wh16_, wh16_ + (size_t)Ch * Cl, Cl, e);
-    bn_stats(s, zh_, PL, Ch, part_, ctr_, hmean_, hrstd_);
-    bn_apply(s, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, 1, rh_, Ch, (size_t)PL * Ch);
+    t_bn_stats(s, zh_, PL, Ch, hmean_, hrstd_);
+    t_bn_apply(s, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, 1, rh_, Ch, (size_t)PL * Ch);
     gap_pool(s, rh_, B_, HW, Ch, gap_);
     fc_ce(s, gap_, wf_, static_cast<const int*>(target), B_, Ch, ncls, logits_, dlogits_, loss_per_);
     ce_mean(s, loss_per_, B_, loss_dst);
     fc_dgap(s, dlogits_, wf_, B_, Ch, ncls, dgap_);
     head_bcast(s, dgap_, B_, HW, Ch, rh_);  // dr overwrites r (the mask is recomputed from z)
-    bn_bwd_reduce(s, rh_, Ch, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, 1, part_, ctr_, sums_, old_, 0.f, 0);
-    bn_bwd_apply(s, rh_, Ch, zh_, PL, Ch, hmean_, hrstd_, old_, sums_, 1, dzh_);
+    t_bn_bwd_reduce(s, rh_, Ch, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, 1, 0.f, 0);
+    t_bn_bwd_apply(s, rh_, Ch, zh_, PL, Ch, hmean_, hrstd_, 1, dzh_);
     e = GemmEpiParams();
     e.out = dy;
     gemm(s, PL, Cl, Ch, dzh_, false, Ch, wh16_, true, Cl, EPI_BF16, e);
@@ -261,23 +261,46 @@ class SposFamily : public Family {
   // forward 1x1 conv: 3-pass bf16x2 product into z's hi/lo planes
   void gemm_x2(cudaStream_t s, int M, int N, int K, const bf16* Ahi, const bf16* Alo, int lda, const bf16* Bhi,
                const bf16* Blo, int ldb, const GemmEpiParams& ep) {
-    if (timer) timer->begin(s);
     gemm_bf16x2_tc(s, M, N, K, Ahi, Alo, lda, Bhi, Blo, ldb, EPI_X2, ep);
-    if (timer) timer->end(s, 6.0 * M * N * K);
     counters.launches++;
   }
 
   void gemm(cudaStream_t s, int M, int N, int K, const bf16* A, bool amn, int lda, const bf16* B, bool bmn, int ldb,
             int epi, const GemmEpiParams& ep, bool split_ok = false) {
-    if (timer) timer->begin(s);
     GemmEpiParams e = ep;
     if (split_ok) {
       e.ws = ws_;
       e.ws_elems = ws_elems_;
     }
     gemm_bf16_tc(s, M, N, K, A, amn, lda, B, bmn, ldb, epi, e);
-    if (timer) timer->end(s, 2.0 * M * N * K);
     counters.launches += (epi == EPI_SGD && gemm_splitk_factor(M, N, K) > 1) ? 2 : 1;
+  }
+
+  // BatchNorm kernels, the step's dominant kernel family (bench.py roofline):
+  // with FLAG_TIMING each call is bracketed by CUDA events on its stream and credited with
+  // its algorithmic HBM bytes (bf16x2 forward tensors 4 B/element, bf16 gradients 2 B).
+  void t_bn_stats(cudaStream_t s, const bf16* z, int Pp, int C, float* mean, float* rstd) {
+    if (timer) timer->begin(s);
+    bn_stats(s, z, Pp, C, part_, ctr_, mean, rstd);
+    if (timer) timer->end(s, 4.0 * Pp * C);
+  }
+  void t_bn_apply(cudaStream_t s, const bf16* z, int Pp, int C, const float* mean, const float* rstd, const float* g,
+                  const float* b, int relu, bf16* y, int ldy, size_t yplane) {
+    if (timer) timer->begin(s);
+    bn_apply(s, z, Pp, C, mean, rstd, g, b, relu, y, ldy, yplane);
+    if (timer) timer->end(s, 8.0 * Pp * C);
+  }
+  void t_bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int Pp, int C, const float* mean,
+                       const float* rstd, float* g, float* b, int relu, float lr, int update) {
+    if (timer) timer->begin(s);
+    bn_bwd_reduce(s, dy, lddy, z, Pp, C, mean, rstd, g, b, relu, part_, ctr_, sums_, old_, lr, update);
+    if (timer) timer->end(s, 6.0 * Pp * C);
+  }
+  void t_bn_bwd_apply(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int Pp, int C, const float* mean,
+                      const float* rstd, int relu, bf16* dz) {
+    if (timer) timer->begin(s);
+    bn_bwd_apply(s, dy, lddy, z, Pp, C, mean, rstd, old_, sums_, relu, dz);
+    if (timer) timer->end(s, 8.0 * Pp * C);
   }
 
   void block_fwd(int j, int c, size_t k, const bf16* x, bf16* out, cudaStream_t s) {
@@ -325,7 +348,7 @@ class SposFamily : public Family {
         e.out2 = r.z + zplane;
         gemm_x2(s, Po, u.cout, u.cin, h, h + hplane, u.cin, W16 + u.off_w16, W16 + half + u.off_w16, u.cin, e);
       }
-      bn_stats(s, r.z, Po, u.cout, part_, ctr_, r.mean, r.rstd);
+      t_bn_stats(s, r.z, Po, u.cout, r.mean, r.rstd);
       bf16* y;
       int ldy;
       size_t yplane;
@@ -339,7 +362,7 @@ class SposFamily : public Family {
         cv += 2 * zplane;
         ldy = u.cout;
       }
-      bn_apply(s, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, u.relu, y, ldy, yplane);
+      t_bn_apply(s, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, u.relu, y, ldy, yplane);
       hplane = yplane;
       counters.launches += 3;
       recs.push_back(r);
@@ -353,9 +376,8 @@ class SposFamily : public Family {
     const int Po = (int)P(u.H_out);
     ring_ = (ring_ + 1) % kRing;
     if (ring_used_[ring_]) cudaStreamWaitEvent(s, ev_wg_[ring_], 0);
-    bn_bwd_reduce(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, u.relu, part_, ctr_, sums_,
-                  old_, lr_, 1);
-    bn_bwd_apply(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, old_, sums_, u.relu, dz_[ring_]);
+    t_bn_bwd_reduce(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, u.relu, lr_, 1);
+    t_bn_bwd_apply(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, u.relu, dz_[ring_]);
     counters.launches += 3;
   }
 

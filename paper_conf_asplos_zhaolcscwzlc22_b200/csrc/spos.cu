@@ -21,6 +21,7 @@
 // Every reduction has a fixed order (per-thread sequential, then a fixed cross-thread order,
 // then a fixed order over row blocks), never floating-point atomics: bitwise reproducible.
 #include <algorithm>
+#include <cstdlib>
 
 #include "common.h"
 #include "kernels.h"
@@ -31,14 +32,24 @@ namespace naspipe {
 namespace {
 
 constexpr int TPB = 256;          // threads per block of the row-block kernels
-constexpr int RED_CTAS = 592;     // target CTAs of the row-block reductions (4 per SM)
+// target CTAs of the row-block reductions: fewer, longer row blocks keep the partial count
+// (and so the fixed-order finalize) short; NASPIPE_RED_CTAS overrides it for tuning.
+static int red_ctas() {
+  static int v = 0;
+  if (!v) {
+    const char* e = getenv("NASPIPE_RED_CTAS");
+    v = e ? std::max(16, atoi(e)) : 296;
+  }
+  return v;
+}
 constexpr float BN_EPS = 1e-5f;
 
 // Row blocking of the per-channel reductions: a function of (P, C) only (deterministic),
 // about RED_CTAS blocks, each a multiple of the kernel's row lanes RP = TPB / (C/8).
-__host__ __device__ inline int red_rows(int P, int C) {
+inline int red_rows(int P, int C) {
   const int rp = TPB / (C / 8);
-  int rows = (P + RED_CTAS - 1) / RED_CTAS;
+  const int target = red_ctas();
+  int rows = (P + target - 1) / target;
   rows = ((rows + rp - 1) / rp) * rp;
   return rows < rp ? rp : rows;
 }
@@ -215,10 +226,10 @@ __global__ void bn_bwd_finalize_kernel(const float* __restrict__ part, int nblk,
 // Thread (r, g): rows r, r + RP, ... of its block, channels [8g, 8g+8); RP = TPB / G row
 // lanes; the RP lane sums are combined in lane order.  Writes part[blk][0..C) = sum z,
 // part[blk][C..2C) = sum z^2.
-__global__ void bn_stats_kernel(const bf16* __restrict__ z, int P, int C, float* __restrict__ part) {
+__global__ void bn_stats_kernel(const bf16* __restrict__ z, int P, int C, int rows, float* __restrict__ part) {
   extern __shared__ float red[];  // [RP][2C]
   ptx::pdl_wait();
-  const int G = C / 8, RP = TPB / G, rows = red_rows(P, C);
+  const int G = C / 8, RP = TPB / G;
   const int r = threadIdx.x / G, g = threadIdx.x % G;
   const int row0 = blockIdx.x * rows, row1 = min(P, row0 + rows);
   const size_t plane = (size_t)P * C;
@@ -324,10 +335,10 @@ __device__ __forceinline__ void bn_bwd_item(const bf16* dy, const bf16* z, size_
 __global__ void bn_bwd_reduce_kernel(const bf16* __restrict__ dy, int lddy, const bf16* __restrict__ z, int P, int C,
                                      const float* __restrict__ mean, const float* __restrict__ rstd,
                                      const float* __restrict__ gam, const float* __restrict__ bet, int relu,
-                                     float* __restrict__ part) {
+                                     int rows, float* __restrict__ part) {
   extern __shared__ float red[];  // [RP][2C]
   ptx::pdl_wait();
-  const int G = C / 8, RP = TPB / G, rows = red_rows(P, C);
+  const int G = C / 8, RP = TPB / G;
   const int r = threadIdx.x / G, g = threadIdx.x % G;
   const int row0 = blockIdx.x * rows, row1 = min(P, row0 + rows);
   const size_t zplane = (size_t)P * C;
@@ -680,37 +691,30 @@ __device__ __forceinline__ float warp_max(float v) {
 
 // One block per 32 classes: logits[b][j] = sum_c gap[b][c] W_fc[j][c] (fp32, c ascending),
 // gap / W tiles of 32 columns staged in shared memory; thread (j, sample group).
+// logits[b, j] = sum_c gap[b, c] wf[j, c]: CTA = 8 samples x 32 classes (grid 32 x B/8 on
+// configs[1]), c in chunks of 32 through shared memory; each output is one sequential fp32
+// FMA chain over c = 0..C-1 (fixed order, bitwise reproducible).
 __global__ void fc_logits_kernel(const float* __restrict__ gap, const float* __restrict__ wf, int B, int C, int ncls,
                                  float* __restrict__ logits) {
-  __shared__ float ws[32][33], gs[64][33];
+  __shared__ float ws[32][33], gs[8][33];
   ptx::pdl_wait();
-  const int jl = threadIdx.x % 32, sg = threadIdx.x / 32, j = blockIdx.x * 32 + jl;
-  for (int b0 = 0; b0 < B; b0 += 64) {
-    float acc[8] = {};
-    for (int c0 = 0; c0 < C; c0 += 32) {
-      for (int i = threadIdx.x; i < 32 * 32; i += TPB) {
-        const int r = i / 32, c = c0 + i % 32, jj = blockIdx.x * 32 + r;
-        ws[r][i % 32] = (jj < ncls && c < C) ? wf[(size_t)jj * C + c] : 0.f;
-      }
-      for (int i = threadIdx.x; i < 64 * 32; i += TPB) {
-        const int r = i / 32, c = c0 + i % 32, b = b0 + r;
-        gs[r][i % 32] = (b < B && c < C) ? gap[(size_t)b * C + c] : 0.f;
-      }
-      __syncthreads();
-#pragma unroll 4
-      for (int cc = 0; cc < 32; ++cc) {
-        const float w = ws[jl][cc];
-#pragma unroll
-        for (int si = 0; si < 8; ++si) acc[si] = __fmaf_rn(gs[sg + 8 * si][cc], w, acc[si]);
-      }
-      __syncthreads();
+  const int jl = threadIdx.x % 32, bl = threadIdx.x / 32, j = blockIdx.x * 32 + jl, b = blockIdx.y * 8 + bl;
+  float acc = 0.f;
+  for (int c0 = 0; c0 < C; c0 += 32) {
+    for (int i = threadIdx.x; i < 32 * 32; i += TPB) {
+      const int r = i / 32, c = c0 + i % 32, jj = blockIdx.x * 32 + r;
+      ws[r][i % 32] = (jj < ncls && c < C) ? wf[(size_t)jj * C + c] : 0.f;
     }
-#pragma unroll
-    for (int si = 0; si < 8; ++si) {
-      const int b = b0 + sg + 8 * si;
-      if (b < B && j < ncls) logits[(size_t)b * ncls + j] = acc[si];
+    {
+      const int r = threadIdx.x / 32, c = c0 + threadIdx.x % 32, bb = blockIdx.y * 8 + r;
+      gs[r][threadIdx.x % 32] = (bb < B && c < C) ? gap[(size_t)bb * C + c] : 0.f;
     }
+    __syncthreads();
+#pragma unroll 8
+    for (int cc = 0; cc < 32; ++cc) acc = __fmaf_rn(gs[bl][cc], ws[jl][cc], acc);
+    __syncthreads();
   }
+  if (b < B && j < ncls) logits[(size_t)b * ncls + j] = acc;
 }
 
 // One block per sample: softmax cross-entropy of its logits, dlogits = (p - onehot) / B.
@@ -763,37 +767,29 @@ __global__ void ce_mean_kernel(const float* __restrict__ loss_per, int B, float*
 }
 
 // One block per 32 channels: dgap[b][c] = sum_j dlogits[b][j] W_fc[j][c] (fp32, j ascending).
+// dgap[b, c] = sum_j dlogits[b, j] wf[j, c]: CTA = 8 samples x 32 channels (grid C/32 x B/8),
+// j in chunks of 32 through shared memory; one sequential FMA chain over j per output.
 __global__ void fc_dgap_kernel(const float* __restrict__ dlogits, const float* __restrict__ wf, int B, int C, int ncls,
                                float* __restrict__ dgap) {
-  __shared__ float ws[32][33], ds[64][33];
+  __shared__ float ws[32][33], ds[8][33];
   ptx::pdl_wait();
-  const int cl = threadIdx.x % 32, sg = threadIdx.x / 32, c = blockIdx.x * 32 + cl;
-  for (int b0 = 0; b0 < B; b0 += 64) {
-    float acc[8] = {};
-    for (int j0 = 0; j0 < ncls; j0 += 32) {
-      for (int i = threadIdx.x; i < 32 * 32; i += TPB) {
-        const int r = i / 32, cc = blockIdx.x * 32 + i % 32, j = j0 + r;
-        ws[r][i % 32] = (j < ncls && cc < C) ? wf[(size_t)j * C + cc] : 0.f;
-      }
-      for (int i = threadIdx.x; i < 64 * 32; i += TPB) {
-        const int r = i / 32, j = j0 + i % 32, b = b0 + r;
-        ds[r][i % 32] = (b < B && j < ncls) ? dlogits[(size_t)b * ncls + j] : 0.f;
-      }
-      __syncthreads();
-#pragma unroll 4
-      for (int jj = 0; jj < 32; ++jj) {
-        const float w = ws[jj][cl];
-#pragma unroll
-        for (int si = 0; si < 8; ++si) acc[si] = __fmaf_rn(ds[sg + 8 * si][jj], w, acc[si]);
-      }
-      __syncthreads();
+  const int cl = threadIdx.x % 32, bl = threadIdx.x / 32, c = blockIdx.x * 32 + cl, b = blockIdx.y * 8 + bl;
+  float acc = 0.f;
+  for (int j0 = 0; j0 < ncls; j0 += 32) {
+    for (int i = threadIdx.x; i < 32 * 32; i += TPB) {
+      const int r = i / 32, cc = blockIdx.x * 32 + i % 32, j = j0 + r;
+      ws[r][i % 32] = (j < ncls && cc < C) ? wf[(size_t)j * C + cc] : 0.f;
     }
-#pragma unroll
-    for (int si = 0; si < 8; ++si) {
-      const int b = b0 + sg + 8 * si;
-      if (b < B && c < C) dgap[(size_t)b * C + c] = acc[si];
+    {
+      const int r = threadIdx.x / 32, j = j0 + threadIdx.x % 32, bb = blockIdx.y * 8 + r;
+      ds[r][threadIdx.x % 32] = (bb < B && j < ncls) ? dlogits[(size_t)bb * ncls + j] : 0.f;
     }
+    __syncthreads();
+#pragma unroll 8
+    for (int jj = 0; jj < 32; ++jj) acc = __fmaf_rn(ds[bl][jj], ws[jj][cl], acc);
+    __syncthreads();
   }
+  if (b < B && c < C) dgap[(size_t)b * C + c] = acc;
 }
 
 // dr[b, hw, c] = dgap[b, c] / HW
@@ -874,7 +870,7 @@ void bn_stats(cudaStream_t s, const bf16* z, int P, int C, float* part, int* ctr
   const size_t sm = red_smem(C);
   const int nblk = bn_part_blocks(P, C);
   set_smem(bn_stats_kernel, sm);
-  launch_pdl(bn_stats_kernel, dim3(nblk), dim3(TPB), sm, s, z, P, C, part);
+  launch_pdl(bn_stats_kernel, dim3(nblk), dim3(TPB), sm, s, z, P, C, red_rows(P, C), part);
   launch_pdl(bn_finalize_kernel, dim3((C + 3) / 4), dim3(TPB), 0, s, (const float*)part, nblk, C, P, mean, rstd);
   check_launch("bn_stats");
 }
@@ -895,7 +891,7 @@ void bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int 
   const int nblk = bn_part_blocks(P, C);
   set_smem(bn_bwd_reduce_kernel, sm);
   launch_pdl(bn_bwd_reduce_kernel, dim3(nblk), dim3(TPB), sm, s, dy, lddy, z, P, C, mean, rstd, (const float*)g,
-             (const float*)b, relu, part);
+             (const float*)b, relu, red_rows(P, C), part);
   launch_pdl(bn_bwd_finalize_kernel, dim3((C + 3) / 4), dim3(TPB), 0, s, (const float*)part, nblk, C, sums, old, g,
              b, lr, update);
   check_launch("bn_bwd_reduce");
@@ -988,7 +984,7 @@ void gap_pool(cudaStream_t s, const bf16* r, int B, int HW, int C, float* gap) {
 
 void fc_ce(cudaStream_t s, const float* gap, const float* wf, const int* labels, int B, int C, int ncls,
            float* logits, float* dlogits, float* loss_per) {
-  launch_pdl(fc_logits_kernel, dim3((ncls + 31) / 32), dim3(TPB), 0, s, gap, wf, B, C, ncls, logits);
+  launch_pdl(fc_logits_kernel, dim3((ncls + 31) / 32, (B + 7) / 8), dim3(TPB), 0, s, gap, wf, B, C, ncls, logits);
   launch_pdl(ce_kernel, dim3(B), dim3(TPB), 0, s, logits, labels, B, ncls, dlogits, loss_per);
   check_launch("fc_ce");
 }
@@ -999,7 +995,7 @@ void ce_mean(cudaStream_t s, const float* loss_per, int B, float* loss) {
 }
 
 void fc_dgap(cudaStream_t s, const float* dlogits, const float* wf, int B, int C, int ncls, float* dgap) {
-  launch_pdl(fc_dgap_kernel, dim3((C + 31) / 32), dim3(TPB), 0, s, dlogits, wf, B, C, ncls, dgap);
+  launch_pdl(fc_dgap_kernel, dim3((C + 31) / 32, (B + 7) / 8), dim3(TPB), 0, s, dlogits, wf, B, C, ncls, dgap);
   check_launch("fc_dgap");
 }
 
