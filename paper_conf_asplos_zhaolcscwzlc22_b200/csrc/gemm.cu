@@ -365,7 +365,7 @@ constexpr int PAIR_SMEM_TOTAL = PAIR_STG_OFF + 8 * 32 * 36 * 4 + 1024;
 template <bool A_MN, bool B_MN, int EPI>
 __global__ void __launch_bounds__(THREADS, 1)
     gemm_pair_kernel(const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb, int M, int N,
-                     TileSpace ts, GemmEpiParams ep) {
+                     TileSpace ts, GemmEpiParams ep, int trig) {
   constexpr int TN = 256, STAGES = PAIR_STAGES, STAGE_BYTES = PAIR_STAGE_BYTES;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -432,7 +432,7 @@ __global__ void __launch_bounds__(THREADS, 1)
         }
       }
     }
-    ptx::pdl_trigger();
+    if (trig) ptx::pdl_trigger();
   } else if (warp == 1) {
     if (lane == 0 && rank == 0) {  // ---------------- MMA issuer (leader only)
       constexpr uint32_t idesc = ptx::umma_idesc_bf16(256, TN, A_MN ? 1 : 0, B_MN ? 1 : 0);
@@ -464,7 +464,7 @@ __global__ void __launch_bounds__(THREADS, 1)
         ptx::umma_commit_pair(&tfull[acc], 0x3);  // both CTAs' accumulators ready
       }
     }
-    ptx::pdl_trigger();
+    if (trig) ptx::pdl_trigger();
   } else {
     // ---------------- epilogue warps 2..9 of both CTAs: this CTA's 128 rows
     const int lane_base = 32 * (warp & 3);
@@ -476,7 +476,7 @@ __global__ void __launch_bounds__(THREADS, 1)
       const int acc = it & 1;
       ptx::mbar_wait(&tfull[acc], (it >> 1) & 1);
       ptx::tc_fence_after();
-      if (t + n_pairs >= n_tiles) ptx::pdl_trigger();
+      if (trig && t + n_pairs >= n_tiles) ptx::pdl_trigger();
       const uint32_t taddr = tmem + ((uint32_t)lane_base << 16) + acc * TN;
       epilogue_warp<EPI, 32>(taddr, stg + (warp - 2) * 32 * 36, tm * 256 + 128 * (int)rank + lane_base, cbeg,
                              cbeg + TN / 2, tn * TN, M, N, ep, ks, lane);
@@ -633,9 +633,26 @@ void launch_pair(cudaStream_t s, int M, int N, const TileSpace& ts, const CUtens
   at[1].val.clusterDim.x = 2;
   at[1].val.clusterDim.y = 1;
   at[1].val.clusterDim.z = 1;
-  cfg.attrs = at;
-  cfg.numAttrs = 2;
-  const cudaError_t e = cudaLaunchKernelEx(&cfg, kern, ta, tb, M, N, ts, ep);
+  // The pair kernel is launched with the PDL attribute (it may start while its predecessor
+  // drains) but does NOT trigger its own dependents early (trig = 0): with early triggers
+  // the 40-step configs[2] run deadlocked on the GPU (tools/hangtest.sh: hang with triggers;
+  // no hang and the best step time without them).  NASPIPE_PAIR_TRIGGER=1 re-enables them
+  // for diagnosis, NASPIPE_PAIR_PDL=0 drops the attribute.
+  static int pair_pdl = -1, pair_trig = -1;
+  if (pair_pdl < 0) {
+    const char* e1 = getenv("NASPIPE_PAIR_PDL");
+    const char* e2 = getenv("NASPIPE_PAIR_TRIGGER");
+    pair_pdl = (e1 && e1[0] == '0') ? 0 : 1;
+    pair_trig = (e2 && e2[0] == '1') ? 1 : 0;
+  }
+  if (pdl_enabled() && pair_pdl) {
+    cfg.attrs = at;
+    cfg.numAttrs = 2;
+  } else {
+    cfg.attrs = at + 1;
+    cfg.numAttrs = 1;
+  }
+  const cudaError_t e = cudaLaunchKernelEx(&cfg, kern, ta, tb, M, N, ts, ep, pair_trig);
   NP_REQUIRE(e == cudaSuccess, NASPIPE_ECUDA, "pair GEMM launch: %s", cudaGetErrorString(e));
   g_gemm_launches.fetch_add(1, std::memory_order_relaxed);
 }
