@@ -43,7 +43,7 @@ extern "C" {
 #pragma GCC visibility push(default) /* the library builds with -fvisibility=hidden */
 #endif
 
-#define NASPIPE_ABI_VERSION 2
+#define NASPIPE_ABI_VERSION 3
 
 typedef enum {
   NASPIPE_OK = 0,
@@ -57,6 +57,24 @@ typedef enum {
 } naspipe_status;
 
 typedef enum { NASPIPE_MLP = 0, NASPIPE_TRANSFORMER = 1, NASPIPE_SPOS_CNN = 2 } naspipe_family;
+
+/* spec.sync_policy: how stages admit queued forwards (Fig.1).
+ *   CSP      causal synchronous parallel (Def.2): admit the lowest-id queued forward
+ *            whose dependencies are finished on the stage (Alg.1/Alg.2) — the method.
+ *   INORDER  "NASPipe w/o scheduler" (Fig.6 ablation): queued forwards are taken
+ *            strictly in id order; a blocked head blocks the stage.  Numerics = CSP.
+ *   ASP      asynchronous (PipeDream-style): dependencies ignored; a forward
+ *            reads the weights current on its stage, a backward's input gradient uses the
+ *            weights current at its start (no weight stashing).  Executable; results
+ *            depend on the stage count (Table 3).
+ *   BSP      bulk synchronous (GPipe / Retiarii): bulks of `bulk_size`
+ *            consecutive subnets; within a bulk dependencies are ignored, forwards run
+ *            before backwards on every stage, and the next bulk starts after the flush
+ *            (every subnet of the bulk finished on every stage).  Its numerics (the bulk's
+ *            gradients summed at the bulk's start weights) need gradient accumulation, which
+ *            the executor does not implement: BSP is a planning policy only
+ *            (naspipe_plan_*; naspipe_create rejects it with EINVAL). */
+typedef enum { NASPIPE_SYNC_CSP = 0, NASPIPE_SYNC_INORDER = 1, NASPIPE_SYNC_ASP = 2, NASPIPE_SYNC_BSP = 3 } naspipe_sync;
 typedef enum { NASPIPE_FP32 = 0, NASPIPE_BF16 = 1 } naspipe_dtype; /* compute dtype; masters fp32 */
 
 /* spec.flags */
@@ -135,6 +153,9 @@ typedef struct {
   const int32_t* stage_channels;
   const int32_t* choice_kernel;
   const int32_t* choice_xception;
+  /* ABI 3: synchronisation policy (naspipe_sync; 0 = CSP) and BSP bulk size (0 = 4 * n_stages) */
+  int32_t sync_policy;
+  int32_t bulk_size;
 } naspipe_supernet_spec;
 
 /* naspipe_batch.where */

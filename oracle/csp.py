@@ -112,7 +112,7 @@ def task_costs(choices, stage_of_block, cost_f, cost_b, D):
 
 
 def simulate_csp(choices, stage_of_block, D, W, cf, cb, lam=0, policy=0, ignore_deps=False,
-                 admit=None):
+                 admit=None, sync="csp", bulk=0):
     """O2.  Returns dict(trace=[(t, K, kind, y)], makespan, order=[[(kind, y)] per stage],
     stall=[ticks per stage], bubble=[ticks per stage]).  An idle stage is *stalled* while a
     queued forward is blocked by a dependency and in a *bubble* while nothing is queued
@@ -122,9 +122,19 @@ def simulate_csp(choices, stage_of_block, D, W, cf, cb, lam=0, policy=0, ignore_
     policy 0: strict backward-first (A5).  policy 1: after a backward, try one forward
     first (Alg.1's alternation).  ``ignore_deps`` gives the no-dependency upper bound used
     in the sweep report (not CSP).  ``admit(K, inF_K, fin_K) -> y or None`` replaces the
-    dependency-table admission rule (used to cross-check against Algorithm 2 verbatim)."""
+    dependency-table admission rule (used to cross-check against Algorithm 2 verbatim).
+
+    ``sync`` (include/naspipe.h naspipe_sync) changes only the admission:
+    "csp" the method; "inorder" NASPipe w/o scheduler (Fig.6): only the lowest-id
+    queued forward may start, a blocked head blocks the stage; "asp" (PipeDream-style,
+    P:L123) dependencies ignored; "bsp" (GPipe/Retiarii): dependencies ignored inside
+    bulks of ``bulk`` consecutive subnets (0 = 4 D), a stage runs any queued forward before
+    a backward, and stage 0 admits bulk k only once every subnet of bulk k-1 finished on
+    stage 0 (the flush: a subnet's stage-0 backward is its last task)."""
     N = len(choices)
-    dep_sets = [[set() if ignore_deps else deps(choices, stage_of_block, y, K)
+    G = bulk if bulk > 0 else 4 * D
+    no_deps = ignore_deps or sync in ("asp", "bsp")
+    dep_sets = [[set() if no_deps else deps(choices, stage_of_block, y, K)
                  for y in range(N)] for K in range(D)]
     fin = [set() for _ in range(D)]
     inF = [set() for _ in range(D)]
@@ -165,20 +175,26 @@ def simulate_csp(choices, stage_of_block, D, W, cf, cb, lam=0, policy=0, ignore_
             return dict(trace=trace, makespan=t, order=order, stall=stall, bubble=bubble)
         # (2) stage-0 source under the window
         wm0 = min([y for y in range(N) if y not in fin[0]], default=N)
+        hi = (wm0 // G + 1) * G if sync == "bsp" else wm0 + W
         for y in range(N):
-            if y < wm0 + W and y not in started0:
+            if y < hi and y not in started0:
                 inF[0].add(y)
         # (3) decisions on idle stages
         for K in range(D):
             if busy[K] is not None:
                 continue
-            if admit is None:
+            if admit is not None:
+                first = admit(K, set(inF[K]), set(fin[K]))
+            elif sync == "inorder":
+                head = min(inF[K]) if inF[K] else None
+                first = head if head is not None and dep_sets[K][head] <= fin[K] else None
+            else:
                 admissible = sorted(y for y in inF[K] if dep_sets[K][y] <= fin[K])
                 first = admissible[0] if admissible else None
-            else:
-                first = admit(K, set(inF[K]), set(fin[K]))
             choose = None
-            if policy == 1 and last_kind[K] == 1 and first is not None:
+            if sync == "bsp" and first is not None:
+                choose = (0, first)
+            elif policy == 1 and last_kind[K] == 1 and first is not None:
                 choose = (0, first)
             elif inB[K]:
                 choose = (1, min(inB[K]))

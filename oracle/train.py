@@ -160,3 +160,68 @@ def initial_theta(cfg):
             segs = [(int(np.prod(s)), kind, fan) for _, s, kind, fan in candidate_layout(cfg, b, c)]
             theta[(b, c)] = init_packed(cfg["init_seed"], b * n + c, segs)
     return theta
+
+
+# --------------------------------------------------------------------------------------
+# Other synchronisation policies (include/naspipe.h naspipe_sync)
+# --------------------------------------------------------------------------------------
+def train_bsp(cfg, theta0, choices, batches, bulk):
+    """BSP (GPipe / Retiarii bulk update): subnets in bulks of ``bulk``
+    consecutive ids; every subnet of a bulk computes its gradient at the bulk's start
+    parameters, the bulk's gradients are summed in id order and applied at the flush.
+    bulk = 1 is the sequential result (O1)."""
+    theta = {k: unpack(cfg, k[0], k[1], v) for k, v in theta0.items()}
+    N = len(choices)
+    losses = np.zeros(N)
+    for y0 in range(0, N, bulk):
+        total = {}
+        for y in range(y0, min(N, y0 + bulk)):
+            x, t = batches[y]
+            loss, grads = subnet_step(cfg, theta, choices[y], x, t)
+            losses[y] = loss
+            for key, g in grads.items():
+                if key not in total:
+                    total[key] = {name: np.array(v, dtype=np.float64) for name, v in g.items()}
+                else:
+                    for name in g:
+                        total[key][name] = total[key][name] + g[name]
+        sgd_apply(theta, total, cfg["lr"])
+    return {k: pack(cfg, k[0], k[1], v) for k, v in theta.items()}, losses
+
+
+def train_replay(cfg, theta0, choices, batches, stage_of_block, trace):
+    """Execute a stage-level task trace [(t, K, kind, y)] in its order (MLP / transformer):
+    F(y, K) runs stage K's blocks forward with the parameters current at that point, the
+    last stage computes the loss and its seed gradient; B(y, K) back-propagates through
+    stage K's blocks in reverse with the parameters current at its start (every input
+    gradient of the task uses pre-update weights, reading A4), then applies SGD to stage K's
+    candidates.  For a CSP trace this is the sequential result (O1); for an ASP trace it
+    defines what the asynchronous pipeline computes (stale reads, no weight stashing)."""
+    assert cfg["family"] in ("mlp", "transformer")
+    theta = {k: unpack(cfg, k[0], k[1], v) for k, v in theta0.items()}
+    D = int(max(stage_of_block)) + 1
+    blocks = [[b for b in range(len(stage_of_block)) if stage_of_block[b] == K] for K in range(D)]
+    act = {}    # (y, K) -> stage input
+    tapes = {}  # (y, b) -> block tape
+    grad = {}   # (y, K) -> gradient w.r.t. the stage output
+    losses = np.zeros(len(choices))
+    for (_, K, kind, y) in trace:
+        ch = choices[y]
+        if kind == 0:
+            h = np.asarray(batches[y][0], dtype=np.float64) if K == 0 else act[(y, K)]
+            for b in blocks[K]:
+                h, tapes[(y, b)] = _block_fwd(cfg, theta[(b, int(ch[b]))], h, int(ch[b]))
+            if K < D - 1:
+                act[(y, K + 1)] = h
+            else:
+                losses[y], grad[(y, K)] = mse_loss(h, np.asarray(batches[y][1], dtype=np.float64))
+        else:
+            dy = grad.pop((y, K))
+            grads = {}
+            for b in reversed(blocks[K]):
+                key = (b, int(ch[b]))
+                dy, grads[key] = _block_bwd(cfg, theta[key], tapes.pop((y, b)), dy)
+            if K > 0:
+                grad[(y, K - 1)] = dy
+            sgd_apply(theta, grads, cfg["lr"])
+    return {k: pack(cfg, k[0], k[1], v) for k, v in theta.items()}, losses

@@ -10,7 +10,8 @@ if not os.path.exists(LIB_PATH):
                       "`python -m paper_conf_asplos_zhaolcscwzlc22_b200.build` (no CPU fallback exists)")
 lib = C.CDLL(LIB_PATH)
 
-ABI_VERSION = 2
+ABI_VERSION = 3
+SYNC = {"csp": 0, "inorder": 1, "asp": 2, "bsp": 3}  # naspipe_sync (include/naspipe.h)
 FAMILY = {"mlp": 0, "transformer": 1, "spos": 2}
 DTYPE = {"fp32": 0, "bf16": 1}
 BATCH_HOST, BATCH_DEVICE, BATCH_SYNTHETIC = 0, 1, 2
@@ -35,7 +36,8 @@ class _SpecStruct(C.Structure):
                 ("link_latency", C.c_int32), ("flags", C.c_int32),
                 ("image_hw", C.c_int32), ("num_classes", C.c_int32), ("stem_channels", C.c_int32),
                 ("head_channels", C.c_int32), ("n_cnn_stages", C.c_int32), ("stage_repeats", _i32p),
-                ("stage_channels", _i32p), ("choice_kernel", _i32p), ("choice_xception", _i32p)]
+                ("stage_channels", _i32p), ("choice_kernel", _i32p), ("choice_xception", _i32p),
+                ("sync_policy", C.c_int32), ("bulk_size", C.c_int32)]
 
 
 class _BatchStruct(C.Structure):
@@ -138,6 +140,8 @@ class Spec:
         s.image_hw, s.num_classes = cfg.get("image_hw", 0), cfg.get("num_classes", 0)
         s.stem_channels, s.head_channels = cfg.get("stem_channels", 0), cfg.get("head_channels", 0)
         s.n_cnn_stages = len(cfg.get("stage_repeats", []))
+        s.sync_policy = SYNC[cfg.get("sync", "csp")]
+        s.bulk_size = cfg.get("bulk_size", 0)
         self.struct = s
         self.cfg = cfg
 

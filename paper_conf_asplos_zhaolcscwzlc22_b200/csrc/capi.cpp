@@ -225,8 +225,11 @@ struct naspipe_handle {
 int naspipe_create(const naspipe_supernet_spec* spec, int32_t n_stages, naspipe_t** out) {
   return guarded([&] {
     NP_REQUIRE(out, NASPIPE_EINVAL, "out NULL");
+    const Spec sp(spec);
+    NP_REQUIRE(sp.raw.sync_policy != NASPIPE_SYNC_BSP, NASPIPE_EINVAL,
+               "BSP is a planning policy only (its bulk update needs gradient accumulation): use naspipe_plan_*");
     auto h = std::make_unique<naspipe_handle>();
-    h->eng = Engine::create_local(Spec(spec), n_stages);
+    h->eng = Engine::create_local(sp, n_stages);
     *out = h.release();
   });
 }
@@ -235,8 +238,11 @@ int naspipe_create_rank(const naspipe_supernet_spec* spec, int32_t n_stages, int
                         int32_t device, const void* nccl_ids, naspipe_t** out) {
   return guarded([&] {
     NP_REQUIRE(out, NASPIPE_EINVAL, "out NULL");
+    const Spec sp(spec);
+    NP_REQUIRE(sp.raw.sync_policy != NASPIPE_SYNC_BSP, NASPIPE_EINVAL,
+               "BSP is a planning policy only (its bulk update needs gradient accumulation): use naspipe_plan_*");
     auto h = std::make_unique<naspipe_handle>();
-    h->eng = Engine::create_rank(Spec(spec), n_stages, stage_rank, device, nccl_ids);
+    h->eng = Engine::create_rank(sp, n_stages, stage_rank, device, nccl_ids);
     *out = h.release();
   });
 }

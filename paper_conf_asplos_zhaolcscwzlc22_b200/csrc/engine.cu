@@ -85,6 +85,8 @@ struct Transport {
 
 // ------------------------------------------------------------------------------ construction
 Engine::Engine(const Spec& spec, int D) : spec_(spec), D_(D), W_(spec.window(D)), planner_(spec_, D) {
+  NP_REQUIRE(spec_.raw.sync_policy != NASPIPE_SYNC_BSP, NASPIPE_EINVAL,
+             "BSP is a planning policy only (its bulk update needs gradient accumulation): use naspipe_plan_*");
   version_.assign((size_t)spec_.m() * spec_.n(), 0);
   timer_.on = (spec_.raw.flags & NASPIPE_FLAG_TIMING) != 0;
 }
@@ -366,7 +368,8 @@ void Engine::issue(const Task& t) {
     }
   }
   if (!st.local) return;
-  if (spec_.raw.flags & NASPIPE_FLAG_VERSION_CHECK) version_check(t);
+  // the version invariant is CSP's (and INORDER's); ASP reads whatever version is current
+  if ((spec_.raw.flags & NASPIPE_FLAG_VERSION_CHECK) && spec_.raw.sync_policy != NASPIPE_SYNC_ASP) version_check(t);
   if (spec_.raw.flags & NASPIPE_FLAG_TRACE) trace_.push_back(t);
   CU(cudaSetDevice(st.dev));
   st.store->before_task(t, st.comp, st.copy);  // context switch: LOAD/EVICT, wait for this task's candidates

@@ -9,7 +9,7 @@ namespace naspipe {
 
 Planner::Planner(const Spec& spec, int D)
     : D_(D), m_(spec.m()), n_(spec.n()), W_(spec.window(D)), policy_(spec.raw.bwd_policy),
-      lambda_(spec.raw.link_latency) {
+      lambda_(spec.raw.link_latency), sync_(spec.raw.sync_policy), G_(spec.bulk(D)) {
   sob_ = spec.partition(D);
   blocks_.assign(D, {});
   for (int b = 0; b < m_; ++b) blocks_[sob_[b]].push_back(b);
@@ -71,6 +71,7 @@ int64_t Planner::cost(int K, int64_t y, int kind) const {
 }
 
 bool Planner::admissible(int K, int64_t y) const {
+  if (sync_ == NASPIPE_SYNC_ASP || sync_ == NASPIPE_SYNC_BSP) return true;  // dependencies ignored
   for (int b : blocks_[K]) {
     const int64_t d = dep(y, b);
     if (d >= 0 && !fin_[K][d]) return false;
@@ -117,10 +118,11 @@ void Planner::advance() {
       makespan_ = t_;
       return;
     }
-    // (2) stage-0 source under the window: y < wm0 + W (reading A7)
+    // (2) stage-0 source under the window: y < wm0 + W (reading A7); BSP: the current bulk,
+    // which opens once every subnet of the previous bulk finished on stage 0 (the flush)
     const int64_t N = n_subnets();
     const int64_t wm0 = fin_wm_[0];
-    const int64_t hi = wm0 + W_;
+    const int64_t hi = sync_ == NASPIPE_SYNC_BSP ? (wm0 / G_ + 1) * G_ : wm0 + W_;
     if (!finalized_ && N < hi) return;  // streaming rule: wait for more subnets
     const int64_t lim = std::min(hi, N);
     for (; src_next_ < lim; ++src_next_) inF_[0].insert(src_next_);
@@ -128,9 +130,16 @@ void Planner::advance() {
     for (int K = 0; K < D_; ++K) {
       if (busy_[K].on) continue;
       int64_t first = -1;
-      for (int64_t y : inF_[K])
-        if (admissible(K, y)) { first = y; break; }  // ascending id (reading A6)
-      if (policy_ == 1 && last_kind_[K] == 1 && first >= 0) {
+      if (sync_ == NASPIPE_SYNC_INORDER) {             // w/o scheduler: only the head may go
+        if (!inF_[K].empty() && admissible(K, *inF_[K].begin())) first = *inF_[K].begin();
+      } else {
+        for (int64_t y : inF_[K])
+          if (admissible(K, y)) { first = y; break; }  // ascending id (reading A6)
+      }
+      if (sync_ == NASPIPE_SYNC_BSP && first >= 0) {  // GPipe: a bulk's forwards before its backwards
+        inF_[K].erase(first);
+        start(K, 0, first);
+      } else if (policy_ == 1 && last_kind_[K] == 1 && first >= 0) {
         inF_[K].erase(first);
         start(K, 0, first);
       } else if (!inB_[K].empty()) {                  // backward first, lowest id (A5)

@@ -62,7 +62,7 @@ class Planner {
   bool admissible(int K, int64_t y) const;
   void start(int K, int kind, int64_t y);
 
-  int D_, m_, n_, W_, policy_, lambda_;
+  int D_, m_, n_, W_, policy_, lambda_, sync_, G_;
   std::vector<int32_t> sob_;
   std::vector<std::vector<int>> blocks_;
   std::vector<int32_t> cf_tab_, cb_tab_;  // [m*n]

@@ -40,6 +40,8 @@ Spec::Spec(const naspipe_supernet_spec* s) {
   NP_REQUIRE(raw.window >= 0 && raw.lookahead >= 0 && raw.bwd_policy >= 0 && raw.bwd_policy <= 1 &&
                  raw.link_latency >= 0 && raw.hbm_weight_budget_bytes >= 0,
              NASPIPE_EINVAL, "bad window/lookahead/policy/latency/budget");
+  NP_REQUIRE(raw.sync_policy >= NASPIPE_SYNC_CSP && raw.sync_policy <= NASPIPE_SYNC_BSP && raw.bulk_size >= 0,
+             NASPIPE_EINVAL, "bad sync_policy %d / bulk_size %d", raw.sync_policy, raw.bulk_size);
   const int n = raw.n_choices, m = raw.n_blocks;
   if (raw.family == NASPIPE_MLP) {
     NP_REQUIRE(raw.width >= 1 && raw.width <= 1024, NASPIPE_EINVAL, "width %d", raw.width);

@@ -52,6 +52,7 @@ struct Spec {
   int n() const { return raw.n_choices; }
   int B() const { return raw.batch; }
   int window(int D) const { return raw.window > 0 ? raw.window : 4 * D; }
+  int bulk(int D) const { return raw.bulk_size > 0 ? raw.bulk_size : 4 * D; }
   int lookahead() const { return raw.lookahead > 0 ? raw.lookahead : 2; }
   int64_t residency_horizon() const { return raw.residency_horizon == 0 ? 64 : raw.residency_horizon; }
   // elements of one sample of input / output (the residual stream width per batch row)

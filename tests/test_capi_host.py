@@ -22,7 +22,7 @@ def test_exports_every_declared_symbol():
     for name in sorted(declared):
         assert hasattr(npipe.lib, name), name
     assert declared == set(npipe.EXPORTED_SYMBOLS)
-    assert npipe.naspipe_abi_version() == 2
+    assert npipe.naspipe_abi_version() == 3
 
 
 @pytest.mark.parametrize("name", ["toy", "tiny_transformer", "transformer"])
@@ -190,3 +190,28 @@ def test_default_costs_and_partition_of_real_configs():
         assert sob[0] == 0 and sob[-1] == D - 1 and np.all(np.diff(sob) >= 0)
         if name == "toy":
             assert list(sob) == [0, 0, 1, 1]
+
+
+@pytest.mark.parametrize("sync", ["inorder", "asp", "bsp"])
+@pytest.mark.parametrize("seed", range(12))
+def test_sync_policies_match_oracle_bit_exact(sync, seed):
+    """the C++ planner's INORDER / ASP / BSP schedules equal the oracle's."""
+    cfg, ch, D = _random_case(100 + seed)
+    cfg = dict(cfg, sync=sync, bulk_size=int(np.random.default_rng(seed).integers(0, 6)))
+    spec = npipe.Spec(cfg)
+    sob = npipe.naspipe_partition(spec, D)
+    plan = npipe.naspipe_plan(spec, D, ch)
+    tf, tb = csp.task_costs(ch, sob, cfg["cost_fwd"], cfg["cost_bwd"], D)
+    ref = csp.simulate_csp(ch, sob, D, cfg["window"], tf, tb, lam=cfg["link_latency"], policy=cfg["bwd_policy"],
+                           sync=sync, bulk=cfg["bulk_size"])
+    assert [tuple(int(v) for v in row) for row in plan.trace()] == [tuple(r) for r in ref["trace"]]
+    assert plan.makespan() == ref["makespan"]
+    st, bu = plan.idle(D)
+    assert list(st) == ref["stall"] and list(bu) == ref["bubble"]
+
+
+def test_bsp_is_plan_only():
+    cfg = dict(synth.get_config("toy"), sync="bsp")
+    with pytest.raises(npipe.NaspipeError) as e:
+        npipe.naspipe_create(npipe.Spec(cfg), 1)
+    assert e.value.code == -1

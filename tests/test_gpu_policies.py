@@ -1,0 +1,74 @@
+"""Synchronisation policies on the GPU (include/naspipe.h naspipe_sync).
+
+* ASP (dependencies ignored, PipeDream-style): the executed schedule equals the
+  oracle's ASP plan, and the parameters equal the oracle replaying that plan stage by stage
+  (oracle/train.py train_replay: stale reads, no weight stashing) — same bars as the CSP
+  parity tests.  Its result depends on the stage count while CSP's does not: the
+  reproducibility contrast of Table 3, here on B200.
+* INORDER ("NASPipe w/o scheduler", Fig.6): a different, still causal schedule with
+  bitwise the CSP numerics.
+"""
+import numpy as np
+import pytest
+
+import synth
+from oracle import csp, train
+
+from test_gpu_parity import FLAGS, param_errors, run_engine
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+npipe = pytest.importorskip("paper_conf_asplos_zhaolcscwzlc22_b200")
+
+
+def _workload(name, N, sync):
+    cfg = synth.get_config(name, sync=sync)
+    choices = synth.sample_choices(N, cfg["n_blocks"], cfg["n_choices"])
+    batches = [synth.make_batch(cfg, y) for y in range(N)]
+    return cfg, choices, batches
+
+
+def _oracle_plan(cfg, choices, D, sync):
+    spec = npipe.Spec(cfg)
+    sob = npipe.naspipe_partition(spec, D)
+    cf, cb = npipe.naspipe_default_costs(spec)
+    tf, tb = csp.task_costs(choices, sob, cf, cb, D)
+    return sob, csp.simulate_csp(choices, sob, D, 4 * D, tf, tb, sync=sync)["trace"]
+
+
+@pytest.mark.parametrize("name,N,D,tol_upd,rtol", [("toy", 24, 2, 1e-5, 1e-5), ("toy", 24, 4, 1e-5, 1e-5),
+                                                   ("tiny_transformer", 8, 2, 1e-1, 1e-2)])
+def test_asp_matches_oracle_replay(name, N, D, tol_upd, rtol):
+    cfg, choices, batches = _workload(name, N, "asp")
+    sob, tr = _oracle_plan(cfg, choices, D, "asp")
+    params, losses, trace, _ = run_engine(cfg, choices, batches, D)
+    assert [tuple(int(v) for v in r) for r in trace] == [tuple(r) for r in tr]
+    theta0 = train.initial_theta(cfg)
+    ref, ref_loss = train.train_replay(cfg, theta0, choices, batches, sob, tr)
+    err, derr = param_errors(cfg, params, ref, theta0)
+    assert err <= 1e-3 and derr <= tol_upd, (err, derr)
+    np.testing.assert_allclose(losses, ref_loss, rtol=rtol)
+
+
+def test_table3_reproducibility_contrast():
+    """CSP: bitwise identical parameters at D = 1, 2, 4.  ASP: the stage count changes them."""
+    N = 24
+    res = {}
+    for sync in ("csp", "asp"):
+        cfg, choices, batches = _workload("toy", N, sync)
+        res[sync] = [run_engine(cfg, choices, batches, D)[0] for D in (1, 2, 4)]
+    for p in res["csp"][1:]:
+        assert all(np.array_equal(p[k].view(np.uint32), res["csp"][0][k].view(np.uint32)) for k in p)
+    a2, a4 = res["asp"][1], res["asp"][2]
+    assert any(not np.array_equal(a2[k], a4[k]) for k in a2)
+
+
+def test_inorder_has_csp_numerics():
+    cfg, choices, batches = _workload("toy", 24, "inorder")
+    sob, tr = _oracle_plan(cfg, choices, 4, "inorder")
+    p_in, l_in, trace, _ = run_engine(cfg, choices, batches, 4)
+    assert [tuple(int(v) for v in r) for r in trace] == [tuple(r) for r in tr]
+    cfg_c = synth.get_config("toy")
+    p_csp, l_csp, _, _ = run_engine(cfg_c, choices, batches, 4)
+    assert all(np.array_equal(p_in[k].view(np.uint32), p_csp[k].view(np.uint32)) for k in p_in)
+    assert np.array_equal(l_in.view(np.uint32), l_csp.view(np.uint32))

@@ -202,3 +202,51 @@ def test_dep_table_small():
     ch = np.array([[0, 1], [0, 0], [1, 1], [0, 1]])
     np.testing.assert_array_equal(csp.dep_table(ch), [[-1, -1], [0, -1], [-1, 0], [1, 2]])
     np.testing.assert_array_equal(csp.expected_versions(ch), [[0, 0], [1, 0], [0, 1], [2, 2]])
+
+
+# ------------------------------------------------------------------ other sync policies (§8f(1))
+def _unit(choices, D, m):
+    sob = np.repeat(np.arange(D), m // D)
+    ones = np.ones((m, int(np.max(choices)) + 1), dtype=np.int64)
+    return sob, csp.task_costs(choices, sob, ones, 2 * ones, D)
+
+
+def test_bsp_hand_example():
+    """D=2, bulk 2, cf=1, cb=2: both forwards before the backwards on each stage, then the
+    flush (derived tick by tick: stage 0 F0@0 F1@1 B0@5 B1@7, stage 1 F0@1 F1@2 B0@3 B1@5)."""
+    ch = np.array([[0, 0], [0, 0]])
+    sob, (tf, tb) = _unit(ch, 2, 2)
+    r = csp.simulate_csp(ch, sob, 2, 8, tf, tb, sync="bsp", bulk=2)
+    s0 = [("F" if k == 0 else "B") + f"{y}@{t}" for t, K, k, y in r["trace"] if K == 0]
+    s1 = [("F" if k == 0 else "B") + f"{y}@{t}" for t, K, k, y in r["trace"] if K == 1]
+    assert s0 == ["F0@0", "F1@1", "B0@5", "B1@7"] and s1 == ["F0@1", "F1@2", "B0@3", "B1@5"]
+    assert r["makespan"] == 9
+    # bulk 1: one subnet at a time, fully serial: N * D * (cf + cb), 2 blocks per stage
+    ch4 = synth.sample_choices(4, 4, 3)
+    sob, (tf, tb) = _unit(ch4, 2, 4)
+    r1 = csp.simulate_csp(ch4, sob, 2, 8, tf, tb, sync="bsp", bulk=1)
+    assert r1["makespan"] == 4 * 2 * (2 + 4) and csp.check_trace(r1["trace"], ch4, sob, 2) == []
+
+
+def test_inorder_is_causal_and_never_overtakes():
+    """NASPipe w/o scheduler (Fig.6): forwards start in id order on every stage and the trace
+    is still causally valid (so its numerics are the sequential result)."""
+    for seed in range(8):
+        ch = synth.sample_choices(24, 8, 2, seed)
+        sob, (tf, tb) = _unit(ch, 4, 8)
+        r = csp.simulate_csp(ch, sob, 4, 16, tf, tb, sync="inorder")
+        assert csp.check_trace(r["trace"], ch, sob, 4) == []
+        for K in range(4):
+            fw = [y for k, y in r["order"][K] if k == 0]
+            assert fw == sorted(fw)
+
+
+def test_asp_is_the_no_dependency_schedule():
+    ch = synth.sample_choices(20, 8, 2, 3)
+    sob, (tf, tb) = _unit(ch, 4, 8)
+    a = csp.simulate_csp(ch, sob, 4, 16, tf, tb, sync="asp")
+    b = csp.simulate_csp(ch, sob, 4, 16, tf, tb, ignore_deps=True)
+    assert a["trace"] == b["trace"]
+    # with conflicts it violates the Table 4 access pattern (CSP never does)
+    assert csp.check_trace(a["trace"], ch, sob, 4) != []
+    assert csp.check_trace(csp.simulate_csp(ch, sob, 4, 16, tf, tb)["trace"], ch, sob, 4) == []

@@ -98,3 +98,73 @@ def test_causally_invalid_swap_changes_result():
     order[y - 1], order[y] = order[y], order[y - 1]
     th, _ = train.train_sequential(cfg, theta0, choices, batches, order=order)
     assert any(not np.array_equal(th[k], ref[k]) for k in ref)
+
+
+# ------------------------------------------------------------------ other sync policies
+def test_bsp_bulk_is_gd_on_the_summed_gradient():
+    """BSP (GPipe bulk update): a bulk of two subnets with the same candidates, from
+    zero weights (every block the identity), updates by -lr (G0^T X0 + G1^T X1) — both
+    gradients at the bulk's start weights — where sequential training would not."""
+    cfg, choices, batches = _toy(N=2)
+    choices = np.array([choices[0], choices[0]])
+    d, B, lr = cfg["width"], cfg["batch"], cfg["lr"]
+    theta0 = {k: np.zeros_like(v) for k, v in train.initial_theta(cfg).items()}
+    theta, losses = train.train_bsp(cfg, theta0, choices, batches, bulk=2)
+    W_expect = np.zeros((d, d))
+    b_expect = np.zeros(d)
+    for y in range(2):
+        X, T = (a.astype(np.float64) for a in batches[y])
+        assert losses[y] == np.mean((X - T) ** 2)
+        G = 2.0 / (B * d) * (X - T)
+        W_expect -= lr * (G.T @ X)
+        b_expect -= lr * G.sum(axis=0)
+    for b in range(cfg["n_blocks"]):
+        v = theta[(b, int(choices[0][b]))]
+        np.testing.assert_allclose(v[: d * d].reshape(d, d), W_expect, rtol=1e-12, atol=1e-15)
+        np.testing.assert_allclose(v[d * d:], b_expect, rtol=1e-12, atol=1e-15)
+    seq, _ = train.train_sequential(cfg, theta0, choices, batches)
+    assert any(not np.array_equal(seq[k], theta[k]) for k in seq)
+
+
+def test_bsp_bulk_one_is_sequential():
+    cfg, choices, batches = _toy(N=6)
+    th0 = train.initial_theta(cfg)
+    a, la = train.train_bsp(cfg, th0, choices, batches, bulk=1)
+    b, lb = train.train_sequential(cfg, th0, choices, batches)
+    assert all(np.array_equal(a[k], b[k]) for k in a) and np.array_equal(la, lb)
+
+
+def _replay_case(name, N, D, sync):
+    from oracle import csp
+    cfg = synth.get_config(name)
+    choices = synth.sample_choices(N, cfg["n_blocks"], cfg["n_choices"])
+    batches = [synth.make_batch(cfg, y) for y in range(N)]
+    sob = np.repeat(np.arange(D), cfg["n_blocks"] // D)
+    ones = np.ones((cfg["n_blocks"], cfg["n_choices"]), dtype=np.int64)
+    tf, tb = csp.task_costs(choices, sob, ones, 2 * ones, D)
+    tr = csp.simulate_csp(choices, sob, D, 4 * D, tf, tb, sync=sync)["trace"]
+    return cfg, choices, batches, sob, tr
+
+
+def test_replay_of_csp_trace_is_sequential():
+    """Executing a CSP schedule stage by stage is bitwise the sequential result."""
+    for name, N, D in (("toy", 12, 2), ("toy", 12, 4), ("tiny_transformer", 4, 2)):
+        cfg, choices, batches, sob, tr = _replay_case(name, N, D, "csp")
+        th0 = train.initial_theta(cfg)
+        a, la = train.train_replay(cfg, th0, choices, batches, sob, tr)
+        b, lb = train.train_sequential(cfg, th0, choices, batches)
+        assert all(np.array_equal(a[k], b[k]) for k in a), (name, D)
+        assert np.array_equal(la, lb)
+
+
+def test_replay_of_asp_trace_breaks_causality():
+    """ASP (dependencies ignored): at one stage it is sequential; on a pipeline, subnets read
+    weights their predecessors have not written yet, so the result changes (Table 3)."""
+    cfg, choices, batches, sob, tr = _replay_case("toy", 12, 1, "asp")
+    th0 = train.initial_theta(cfg)
+    a, _ = train.train_replay(cfg, th0, choices, batches, np.zeros(cfg["n_blocks"], dtype=int), tr)
+    b, _ = train.train_sequential(cfg, th0, choices, batches)
+    assert all(np.array_equal(a[k], b[k]) for k in a)
+    cfg, choices, batches, sob, tr = _replay_case("toy", 12, 2, "asp")
+    c, _ = train.train_replay(cfg, th0, choices, batches, sob, tr)
+    assert any(not np.array_equal(c[k], b[k]) for k in c)
