@@ -174,19 +174,24 @@ __global__ void __launch_bounds__(256) attn_fwd_kernel(const bf16* __restrict__ 
   }
 }
 
+// Backward.  HD <= 64 keeps ONE S x S bf16 buffer (P, then dS) so that two CTAs fit per SM
+// (108 KB of shared memory instead of 143 KB; the configs[2] h=16 blocks launch B*h = 512
+// CTAs): P is written, dV = P^T dO is formed, then dS (kept in registers) replaces it and
+// dK = dS^T Q follows.  HD > 64 keeps both buffers (one CTA per SM either way).
 template <int HD>
-__global__ void __launch_bounds__(256) attn_bwd_kernel(const bf16* __restrict__ qkv, const bf16* __restrict__ o,
+__global__ void __launch_bounds__(256, (HD <= 64 ? 2 : 1)) attn_bwd_kernel(const bf16* __restrict__ qkv, const bf16* __restrict__ o,
                                                        const float* __restrict__ lse, const bf16* __restrict__ dout,
                                                        bf16* __restrict__ dqkv, int S, int d, int h) {
   using C = AttnCfg<HD>;
+  constexpr bool ONEBUF = HD <= 64;
   extern __shared__ __align__(16) uint8_t sm[];
   bf16* Qs = reinterpret_cast<bf16*>(sm);
   bf16* Ks = Qs + SMAX * C::LDH;
   bf16* Vs = Ks + SMAX * C::LDH;
   bf16* dOs = Vs + SMAX * C::LDH;
   bf16* Ps = dOs + SMAX * C::LDH;
-  bf16* dSs = Ps + SMAX * C::LDS;
-  float* Di = reinterpret_cast<float*>(dSs + SMAX * C::LDS);
+  bf16* dSs = ONEBUF ? Ps : Ps + SMAX * C::LDS;
+  float* Di = reinterpret_cast<float*>(Ps + (ONEBUF ? 1 : 2) * SMAX * C::LDS);
   const int bh = blockIdx.x, b = bh / h, hh = bh % h;
   const size_t ld = 3 * (size_t)d;
   const bf16* base = qkv + (size_t)b * S * ld + hh * HD;
@@ -229,6 +234,7 @@ __global__ void __launch_bounds__(256) attn_bwd_kernel(const bf16* __restrict__ 
   const float scale_log2 = 1.4426950408889634f * scale;
   const int r0 = warp * 16;
   const bool active = r0 < S;
+  float dp[SMAX / 8][4];  // dS rows of this warp (kept for the one-buffer path)
   if (active) {
     float sacc[SMAX / 8][4];
     scores<HD>(Qs, Ks, r0, S, sacc);
@@ -242,7 +248,6 @@ __global__ void __launch_bounds__(256) attn_bwd_kernel(const bf16* __restrict__ 
       sacc[nb][3] = exp2f(sacc[nb][3] * scale_log2 - l1);
     }
     // dP = dO V^T
-    float dp[SMAX / 8][4];
     scores<HD>(dOs, Vs, r0, S, dp);
     const float d0 = Di[r0 + g], d1 = Di[r0 + g + 8];
 #pragma unroll
@@ -256,8 +261,10 @@ __global__ void __launch_bounds__(256) attn_bwd_kernel(const bf16* __restrict__ 
         dp[nb][3] = sacc[nb][3] * (dp[nb][3] - d1);
         *reinterpret_cast<uint32_t*>(Ps + (r0 + g) * C::LDS + col) = ptx::pack_bf16(sacc[nb][0], sacc[nb][1]);
         *reinterpret_cast<uint32_t*>(Ps + (r0 + g + 8) * C::LDS + col) = ptx::pack_bf16(sacc[nb][2], sacc[nb][3]);
-        *reinterpret_cast<uint32_t*>(dSs + (r0 + g) * C::LDS + col) = ptx::pack_bf16(dp[nb][0], dp[nb][1]);
-        *reinterpret_cast<uint32_t*>(dSs + (r0 + g + 8) * C::LDS + col) = ptx::pack_bf16(dp[nb][2], dp[nb][3]);
+        if (!ONEBUF) {
+          *reinterpret_cast<uint32_t*>(dSs + (r0 + g) * C::LDS + col) = ptx::pack_bf16(dp[nb][0], dp[nb][1]);
+          *reinterpret_cast<uint32_t*>(dSs + (r0 + g + 8) * C::LDS + col) = ptx::pack_bf16(dp[nb][2], dp[nb][3]);
+        }
       }
     }
     // dQ = dS K * scale
@@ -290,6 +297,73 @@ __global__ void __launch_bounds__(256) attn_bwd_kernel(const bf16* __restrict__ 
     }
   }
   __syncthreads();
+  bf16* k0p = dqkv + ((size_t)b * S + r0 + g) * ld + d + hh * HD;
+  bf16* k1p = k0p + 8 * ld;
+  bf16* v0p = k0p + d;
+  bf16* v1p = k1p + d;
+  if (ONEBUF) {
+    // dV = P^T dO (this warp: key rows r0..r0+15), then dS replaces P and dK = dS^T Q * scale
+    if (active) {
+      float dv[HD / 8][4];
+#pragma unroll
+      for (int nb = 0; nb < HD / 8; ++nb) dv[nb][0] = dv[nb][1] = dv[nb][2] = dv[nb][3] = 0.f;
+#pragma unroll
+      for (int kk = 0; kk < SMAX / 16; ++kk) {
+        if (kk * 16 < S) {
+          uint32_t ap[4];
+          lds_a_t(Ps, C::LDS, r0, kk * 16, ap);
+#pragma unroll
+          for (int np = 0; np < HD / 16; ++np) {
+            uint32_t bo[4];
+            lds_b_kn(dOs, C::LDH, kk * 16, np * 16, bo);
+            ptx::mma_bf16_16816(dv[2 * np], ap, bo[0], bo[1]);
+            ptx::mma_bf16_16816(dv[2 * np + 1], ap, bo[2], bo[3]);
+          }
+        }
+      }
+#pragma unroll
+      for (int nb = 0; nb < HD / 8; ++nb) {
+        *reinterpret_cast<uint32_t*>(v0p + nb * 8 + 2 * t) = ptx::pack_bf16(dv[nb][0], dv[nb][1]);
+        *reinterpret_cast<uint32_t*>(v1p + nb * 8 + 2 * t) = ptx::pack_bf16(dv[nb][2], dv[nb][3]);
+      }
+    }
+    __syncthreads();  // every warp has read P
+    if (active) {
+#pragma unroll
+      for (int nb = 0; nb < SMAX / 8; ++nb) {
+        if (nb * 8 < S) {
+          const int col = nb * 8 + 2 * t;
+          *reinterpret_cast<uint32_t*>(dSs + (r0 + g) * C::LDS + col) = ptx::pack_bf16(dp[nb][0], dp[nb][1]);
+          *reinterpret_cast<uint32_t*>(dSs + (r0 + g + 8) * C::LDS + col) = ptx::pack_bf16(dp[nb][2], dp[nb][3]);
+        }
+      }
+    }
+    __syncthreads();
+    if (!active) return;
+    float dk[HD / 8][4];
+#pragma unroll
+    for (int nb = 0; nb < HD / 8; ++nb) dk[nb][0] = dk[nb][1] = dk[nb][2] = dk[nb][3] = 0.f;
+#pragma unroll
+    for (int kk = 0; kk < SMAX / 16; ++kk) {
+      if (kk * 16 < S) {
+        uint32_t as[4];
+        lds_a_t(dSs, C::LDS, r0, kk * 16, as);
+#pragma unroll
+        for (int np = 0; np < HD / 16; ++np) {
+          uint32_t bq[4];
+          lds_b_kn(Qs, C::LDH, kk * 16, np * 16, bq);
+          ptx::mma_bf16_16816(dk[2 * np], as, bq[0], bq[1]);
+          ptx::mma_bf16_16816(dk[2 * np + 1], as, bq[2], bq[3]);
+        }
+      }
+    }
+#pragma unroll
+    for (int nb = 0; nb < HD / 8; ++nb) {
+      *reinterpret_cast<uint32_t*>(k0p + nb * 8 + 2 * t) = ptx::pack_bf16(dk[nb][0] * scale, dk[nb][1] * scale);
+      *reinterpret_cast<uint32_t*>(k1p + nb * 8 + 2 * t) = ptx::pack_bf16(dk[nb][2] * scale, dk[nb][3] * scale);
+    }
+    return;
+  }
   if (!active) return;
   // dK = dS^T Q * scale ; dV = P^T dO   (this warp: key rows r0..r0+15)
   float dk[HD / 8][4], dv[HD / 8][4];
@@ -316,10 +390,6 @@ __global__ void __launch_bounds__(256) attn_bwd_kernel(const bf16* __restrict__ 
       }
     }
   }
-  bf16* k0p = dqkv + ((size_t)b * S + r0 + g) * ld + d + hh * HD;
-  bf16* k1p = k0p + 8 * ld;
-  bf16* v0p = k0p + d;
-  bf16* v1p = k1p + d;
 #pragma unroll
   for (int nb = 0; nb < HD / 8; ++nb) {
     *reinterpret_cast<uint32_t*>(k0p + nb * 8 + 2 * t) = ptx::pack_bf16(dk[nb][0] * scale, dk[nb][1] * scale);
@@ -338,7 +408,7 @@ void fwd_launch(cudaStream_t s, const bf16* qkv, bf16* o, float* lse, int B, int
 template <int HD>
 void bwd_launch(cudaStream_t s, const bf16* qkv, const bf16* o, const float* lse, const bf16* dout, bf16* dqkv,
                 int B, int S, int d, int h) {
-  const int smem = 4 * SMAX * AttnCfg<HD>::LDH * 2 + 2 * SMAX * AttnCfg<HD>::LDS * 2 + SMAX * 4;
+  const int smem = 4 * SMAX * AttnCfg<HD>::LDH * 2 + (HD <= 64 ? 1 : 2) * SMAX * AttnCfg<HD>::LDS * 2 + SMAX * 4;
   cudaFuncSetAttribute(attn_bwd_kernel<HD>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   launch_pdl(attn_bwd_kernel<HD>, dim3(B * h), dim3(256), smem, s, qkv, o, lse, dout, dqkv, S, d, h);
 }

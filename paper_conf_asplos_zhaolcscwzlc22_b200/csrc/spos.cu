@@ -559,51 +559,82 @@ __global__ void __launch_bounds__(TPB) dw_tile_kernel(const bf16* __restrict__ i
   }
 }
 
-// Weight gradient partials: block (blk, u) sums over output pixels [blk*rows, ...) the
-// products dz[b,oh,ow,c] * x[b, oh*S+u-PAD, ow*S+v-PAD, c] for every c, v.
-// part[blk][c][u][v] (the [C][K][K] layout of the weight).
-template <int K>
-__global__ void dw_wgrad_kernel(const bf16* __restrict__ dz, const bf16* __restrict__ x, float* __restrict__ part,
-                                int B, int H, int C, int S, int rows) {
-  extern __shared__ float red[];  // [RP][C][K]
+// Weight gradient partials, tiled like the forward (dw_tile_kernel): CTA (tile column tw,
+// part p; channel-group block blockIdx.y) loops over the (image, DT_H-row strip) tiles
+// q = p, p + NP, ... < B * tiles_h; per tile it stages the input halo in shared memory and
+// thread (ch, col, cg) — output column tw*TW + col, channel c — holds its DT_H values of dz
+// in registers and accumulates all K x K taps, reading each staged input once per tile
+// (K*K FMAs per DT_H*K*K / (IH*K) reads instead of one load per FMA).  The TW column sums
+// are then added in column order; part[tw + tiles_w * p][c][u][v] (the weight's layout),
+// later summed over the partial blocks in a fixed order.  Bitwise reproducible.
+template <int K, int S>
+__global__ void __launch_bounds__(TPB) dw_wgrad_kernel(const bf16* __restrict__ dz, const bf16* __restrict__ x,
+                                                       float* __restrict__ part, int B, int H, int C, int TW,
+                                                       int NP) {
+  constexpr int PAD = K / 2, IH = (DT_H - 1) * S + K, K2 = K * K;
+  extern __shared__ float tile[];  // [CPG][IH][IW][8]; later [TPB][K2] for the column sums
   ptx::pdl_wait();
-  constexpr int PAD = K / 2;
   const int Ho = (H + 2 * PAD - K) / S + 1;
-  const int G = C / 8, RP = TPB / G;
-  const int r = threadIdx.x / G, g = threadIdx.x % G;
-  const int u = blockIdx.y;
-  const int P = B * Ho * Ho;
-  const int q0 = blockIdx.x * rows, q1 = min(P, q0 + rows);
-  if (r < RP) {
-    float acc[K][8] = {};
-    for (int q = q0 + r; q < q1; q += RP) {
-      const int ow = q % Ho, oh = (q / Ho) % Ho, b = q / (Ho * Ho);
-      const int ih = oh * S + u - PAD;
-      if (ih < 0 || ih >= H) continue;
-      float dv[8];
-      load8(dz + (size_t)q * C + 8 * g, dv);
-      const bf16* row = x + (((size_t)b * H + ih) * H) * C + 8 * g;
+  const int CPG = TPB / (8 * TW), IW = (TW - 1) * S + K;
+  const int tiles_h = (Ho + DT_H - 1) / DT_H, tiles_w = (Ho + TW - 1) / TW;
+  const int tw = blockIdx.x % tiles_w, p = blockIdx.x / tiles_w;
+  const int cg0 = blockIdx.y * CPG;
+  const int ch = threadIdx.x % 8, col = (threadIdx.x / 8) % TW, cgi = threadIdx.x / (8 * TW);
+  const int c = (cg0 + cgi) * 8 + ch, ow = tw * TW + col;
+  float acc[K][K];
+#pragma unroll
+  for (int u = 0; u < K; ++u)
+#pragma unroll
+    for (int v = 0; v < K; ++v) acc[u][v] = 0.f;
+  for (int q = p; q < B * tiles_h; q += NP) {
+    const int b = q / tiles_h, th = q % tiles_h;
+    const int ih0 = th * DT_H * S - PAD, iw0 = tw * TW * S - PAD;
+    __syncthreads();  // the previous tile has been consumed
+    for (int i = threadIdx.x; i < CPG * IH * IW; i += TPB) {
+      const int cl = i % IW, row = (i / IW) % IH, cg = i / (IW * IH);
+      const int ih = ih0 + row, iw = iw0 + cl, cc = (cg0 + cg) * 8;
+      float v[8] = {};
+      if (ih >= 0 && ih < H && iw >= 0 && iw < H && cc < C) load8(x + (((size_t)b * H + ih) * H + iw) * C + cc, v);
+      float4* d = reinterpret_cast<float4*>(tile + (size_t)i * 8);
+      d[0] = make_float4(v[0], v[1], v[2], v[3]);
+      d[1] = make_float4(v[4], v[5], v[6], v[7]);
+    }
+    float g[DT_H];
+#pragma unroll
+    for (int r = 0; r < DT_H; ++r) {
+      const int oh = th * DT_H + r;
+      g[r] = (c < C && ow < Ho && oh < Ho) ? __bfloat162float(dz[(((size_t)b * Ho + oh) * Ho + ow) * C + c]) : 0.f;
+    }
+    __syncthreads();
+    const float* tb = tile + ((size_t)cgi * IH * IW + col * S) * 8 + ch;
+#pragma unroll
+    for (int ir = 0; ir < IH; ++ir) {
 #pragma unroll
       for (int v = 0; v < K; ++v) {
-        const int iw = ow * S + v - PAD;
-        if (iw < 0 || iw >= H) continue;
-        float xv[8];
-        load8(row + (size_t)iw * C, xv);
+        const float xv = tb[((size_t)ir * IW + v) * 8];
 #pragma unroll
-        for (int i = 0; i < 8; ++i) acc[v][i] = __fmaf_rn(dv[i], xv[i], acc[v][i]);
+        for (int r = 0; r < DT_H; ++r) {
+          const int u = ir - r * S;
+          if (u >= 0 && u < K) acc[u][v] = __fmaf_rn(g[r], xv, acc[u][v]);
+        }
       }
     }
-#pragma unroll
-    for (int v = 0; v < K; ++v)
-#pragma unroll
-      for (int i = 0; i < 8; ++i) red[((size_t)r * C + 8 * g + i) * K + v] = acc[v][i];
   }
   __syncthreads();
-  for (int e = threadIdx.x; e < C * K; e += TPB) {
-    float a = 0.f;
-    for (int k = 0; k < RP; ++k) a += red[(size_t)k * C * K + e];
-    const int c = e / K, v = e % K;
-    part[(size_t)blockIdx.x * C * K * K + (size_t)c * K * K + u * K + v] = a;
+  float* red = tile;  // [TPB][K2]
+#pragma unroll
+  for (int u = 0; u < K; ++u)
+#pragma unroll
+    for (int v = 0; v < K; ++v) red[(size_t)threadIdx.x * K2 + u * K + v] = acc[u][v];
+  __syncthreads();
+  const size_t pbase = (size_t)blockIdx.x * C * K2;
+  for (int e = threadIdx.x; e < CPG * 8 * K2; e += TPB) {
+    const int tap = e % K2, cc = e / K2, cgl = cc / 8, chl = cc % 8;
+    const int cglob = (cg0 + cgl) * 8 + chl;
+    if (cglob >= C) continue;
+    float sum = 0.f;
+    for (int cl = 0; cl < TW; ++cl) sum += red[(size_t)((cgl * TW + cl) * 8 + chl) * K2 + tap];
+    part[pbase + (size_t)cglob * K2 + tap] = sum;
   }
 }
 
@@ -692,26 +723,30 @@ __device__ __forceinline__ float warp_max(float v) {
 // One block per 32 classes: logits[b][j] = sum_c gap[b][c] W_fc[j][c] (fp32, c ascending),
 // gap / W tiles of 32 columns staged in shared memory; thread (j, sample group).
 // logits[b, j] = sum_c gap[b, c] wf[j, c]: CTA = 8 samples x 32 classes (grid 32 x B/8 on
-// configs[1]), c in chunks of 32 through shared memory; each output is one sequential fp32
-// FMA chain over c = 0..C-1 (fixed order, bitwise reproducible).
+// configs[1]); c in chunks of FC_KC through shared memory (a few long coalesced load phases
+// instead of many short latency-bound ones); each output is one sequential fp32 FMA chain
+// over c = 0..C-1 (fixed order, bitwise reproducible).
+constexpr int FC_KC = 256;
 __global__ void fc_logits_kernel(const float* __restrict__ gap, const float* __restrict__ wf, int B, int C, int ncls,
                                  float* __restrict__ logits) {
-  __shared__ float ws[32][33], gs[8][33];
+  extern __shared__ float fsm[];
+  float* ws = fsm;                     // [32][FC_KC + 1]
+  float* gs = fsm + 32 * (FC_KC + 1);  // [8][FC_KC]
   ptx::pdl_wait();
   const int jl = threadIdx.x % 32, bl = threadIdx.x / 32, j = blockIdx.x * 32 + jl, b = blockIdx.y * 8 + bl;
   float acc = 0.f;
-  for (int c0 = 0; c0 < C; c0 += 32) {
-    for (int i = threadIdx.x; i < 32 * 32; i += TPB) {
-      const int r = i / 32, c = c0 + i % 32, jj = blockIdx.x * 32 + r;
-      ws[r][i % 32] = (jj < ncls && c < C) ? wf[(size_t)jj * C + c] : 0.f;
+  for (int c0 = 0; c0 < C; c0 += FC_KC) {
+    for (int i = threadIdx.x; i < 32 * FC_KC; i += TPB) {
+      const int r = i / FC_KC, c = c0 + i % FC_KC, jj = blockIdx.x * 32 + r;
+      ws[r * (FC_KC + 1) + i % FC_KC] = (jj < ncls && c < C) ? wf[(size_t)jj * C + c] : 0.f;
     }
-    {
-      const int r = threadIdx.x / 32, c = c0 + threadIdx.x % 32, bb = blockIdx.y * 8 + r;
-      gs[r][threadIdx.x % 32] = (bb < B && c < C) ? gap[(size_t)bb * C + c] : 0.f;
+    for (int i = threadIdx.x; i < 8 * FC_KC; i += TPB) {
+      const int r = i / FC_KC, c = c0 + i % FC_KC, bb = blockIdx.y * 8 + r;
+      gs[i] = (bb < B && c < C) ? gap[(size_t)bb * C + c] : 0.f;
     }
     __syncthreads();
 #pragma unroll 8
-    for (int cc = 0; cc < 32; ++cc) acc = __fmaf_rn(gs[bl][cc], ws[jl][cc], acc);
+    for (int cc = 0; cc < FC_KC; ++cc) acc = __fmaf_rn(gs[bl * FC_KC + cc], ws[jl * (FC_KC + 1) + cc], acc);
     __syncthreads();
   }
   if (b < B && j < ncls) logits[(size_t)b * ncls + j] = acc;
@@ -768,25 +803,27 @@ __global__ void ce_mean_kernel(const float* __restrict__ loss_per, int B, float*
 
 // One block per 32 channels: dgap[b][c] = sum_j dlogits[b][j] W_fc[j][c] (fp32, j ascending).
 // dgap[b, c] = sum_j dlogits[b, j] wf[j, c]: CTA = 8 samples x 32 channels (grid C/32 x B/8),
-// j in chunks of 32 through shared memory; one sequential FMA chain over j per output.
+// j in chunks of FC_KC through shared memory; one sequential FMA chain over j per output.
 __global__ void fc_dgap_kernel(const float* __restrict__ dlogits, const float* __restrict__ wf, int B, int C, int ncls,
                                float* __restrict__ dgap) {
-  __shared__ float ws[32][33], ds[8][33];
+  extern __shared__ float fsm[];
+  float* ws = fsm;                // [FC_KC][32]
+  float* ds = fsm + FC_KC * 32;   // [8][FC_KC]
   ptx::pdl_wait();
   const int cl = threadIdx.x % 32, bl = threadIdx.x / 32, c = blockIdx.x * 32 + cl, b = blockIdx.y * 8 + bl;
   float acc = 0.f;
-  for (int j0 = 0; j0 < ncls; j0 += 32) {
-    for (int i = threadIdx.x; i < 32 * 32; i += TPB) {
+  for (int j0 = 0; j0 < ncls; j0 += FC_KC) {
+    for (int i = threadIdx.x; i < FC_KC * 32; i += TPB) {
       const int r = i / 32, cc = blockIdx.x * 32 + i % 32, j = j0 + r;
-      ws[r][i % 32] = (j < ncls && cc < C) ? wf[(size_t)j * C + cc] : 0.f;
+      ws[i] = (j < ncls && cc < C) ? wf[(size_t)j * C + cc] : 0.f;
     }
-    {
-      const int r = threadIdx.x / 32, j = j0 + threadIdx.x % 32, bb = blockIdx.y * 8 + r;
-      ds[r][threadIdx.x % 32] = (bb < B && j < ncls) ? dlogits[(size_t)bb * ncls + j] : 0.f;
+    for (int i = threadIdx.x; i < 8 * FC_KC; i += TPB) {
+      const int r = i / FC_KC, j = j0 + i % FC_KC, bb = blockIdx.y * 8 + r;
+      ds[i] = (bb < B && j < ncls) ? dlogits[(size_t)bb * ncls + j] : 0.f;
     }
     __syncthreads();
 #pragma unroll 8
-    for (int jj = 0; jj < 32; ++jj) acc = __fmaf_rn(ds[bl][jj], ws[jj][cl], acc);
+    for (int jj = 0; jj < FC_KC; ++jj) acc = __fmaf_rn(ds[bl * FC_KC + jj], ws[jj * 32 + cl], acc);
     __syncthreads();
   }
   if (b < B && c < C) dgap[(size_t)b * C + c] = acc;
@@ -947,22 +984,46 @@ void dw_dgrad(cudaStream_t s, const bf16* dz, const float* w, const bf16* add, b
   check_launch("dw_dgrad");
 }
 
-// weight-gradient row blocks: about RED_CTAS CTAs over the (row block, kernel row) grid
-static int dw_rows(int P_out, int C, int k) { return red_rows(P_out, C) * k; }
+// weight-gradient grid: tiles_w tile columns x NP parts x channel-group blocks, about
+// red_ctas() CTAs; partial blocks = tiles_w * NP (a function of the shape only).
+static void dw_wgrad_grid(int B, int H, int C, int k, int S, int& TW, int& NP, int& gy, int& tiles_w) {
+  const int Ho = (H - 1) / S + 1;
+  TW = dw_tw(Ho);
+  const int CPG = TPB / (8 * TW);
+  tiles_w = (Ho + TW - 1) / TW;
+  gy = (C / 8 + CPG - 1) / CPG;
+  const int tiles = B * ((Ho + DT_H - 1) / DT_H);
+  NP = std::max(1, std::min(tiles, red_ctas() / std::max(1, tiles_w * gy)));
+  (void)k;
+}
 int dw_wgrad_blocks(int B, int H, int C, int k, int S) {
-  const int Ho = (H - 1) / S + 1, P = B * Ho * Ho, r = dw_rows(P, C, k);
-  return (P + r - 1) / r;
+  int TW, NP, gy, tw;
+  dw_wgrad_grid(B, H, C, k, S, TW, NP, gy, tw);
+  return tw * NP;
 }
 
 void dw_wgrad(cudaStream_t s, const bf16* dz, const bf16* x, float* part, int B, int H, int C, int k, int S) {
   NP_REQUIRE(C % 8 == 0 && C / 8 <= TPB, NASPIPE_EINVAL, "dw_wgrad C=%d", C);
-  const int Ho = (H - 1) / S + 1;
-  const int P_out = B * Ho * Ho, nblk = dw_wgrad_blocks(B, H, C, k, S), rows = dw_rows(P_out, C, k);
-  const size_t sm = (size_t)(TPB / (C / 8)) * C * k * sizeof(float);
-  DW_DISPATCH(k, {
-    set_smem(dw_wgrad_kernel<KK>, sm);
-    launch_pdl(dw_wgrad_kernel<KK>, dim3(nblk, KK), dim3(TPB), sm, s, dz, x, part, B, H, C, S, rows);
-  });
+  NP_REQUIRE(S == 1 || S == 2, NASPIPE_EINVAL, "dw_wgrad stride %d", S);
+  int TW, NP, gy, tiles_w;
+  dw_wgrad_grid(B, H, C, k, S, TW, NP, gy, tiles_w);
+  const int CPG = TPB / (8 * TW);
+  auto smem = [&](int K) {
+    const int IH = (DT_H - 1) * S + K, IW = (TW - 1) * S + K;
+    return std::max((size_t)CPG * IH * IW * 8, (size_t)TPB * K * K) * sizeof(float);
+  };
+  const dim3 grid(tiles_w * NP, gy);
+#define DW_WG(KK, SS)                                                                                  \
+  {                                                                                                    \
+    set_smem(dw_wgrad_kernel<KK, SS>, smem(KK));                                                       \
+    launch_pdl(dw_wgrad_kernel<KK, SS>, grid, dim3(TPB), smem(KK), s, dz, x, part, B, H, C, TW, NP);    \
+  }
+  if (S == 1) {
+    DW_DISPATCH(k, DW_WG(KK, 1));
+  } else {
+    DW_DISPATCH(k, DW_WG(KK, 2));
+  }
+#undef DW_WG
   check_launch("dw_wgrad");
 }
 
@@ -984,7 +1045,9 @@ void gap_pool(cudaStream_t s, const bf16* r, int B, int HW, int C, float* gap) {
 
 void fc_ce(cudaStream_t s, const float* gap, const float* wf, const int* labels, int B, int C, int ncls,
            float* logits, float* dlogits, float* loss_per) {
-  launch_pdl(fc_logits_kernel, dim3((ncls + 31) / 32, (B + 7) / 8), dim3(TPB), 0, s, gap, wf, B, C, ncls, logits);
+  const size_t sm = (32 * (FC_KC + 1) + 8 * FC_KC) * sizeof(float);
+  set_smem(fc_logits_kernel, sm);
+  launch_pdl(fc_logits_kernel, dim3((ncls + 31) / 32, (B + 7) / 8), dim3(TPB), sm, s, gap, wf, B, C, ncls, logits);
   launch_pdl(ce_kernel, dim3(B), dim3(TPB), 0, s, logits, labels, B, ncls, dlogits, loss_per);
   check_launch("fc_ce");
 }
@@ -995,7 +1058,9 @@ void ce_mean(cudaStream_t s, const float* loss_per, int B, float* loss) {
 }
 
 void fc_dgap(cudaStream_t s, const float* dlogits, const float* wf, int B, int C, int ncls, float* dgap) {
-  launch_pdl(fc_dgap_kernel, dim3((C + 31) / 32, (B + 7) / 8), dim3(TPB), 0, s, dlogits, wf, B, C, ncls, dgap);
+  const size_t sm = (FC_KC * 32 + 8 * FC_KC) * sizeof(float);
+  set_smem(fc_dgap_kernel, sm);
+  launch_pdl(fc_dgap_kernel, dim3((C + 31) / 32, (B + 7) / 8), dim3(TPB), sm, s, dlogits, wf, B, C, ncls, dgap);
   check_launch("fc_dgap");
 }
 
