@@ -43,6 +43,7 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-secondary", action="store_true", help="skip the configs[2] line embedded in the output")
+    ap.add_argument("--no-repro", action="store_true", help="skip the bit-reproducibility digests")
     ap.add_argument("--budget-x", type=float, default=0.0,
                     help="HBM weight budget per stage as a multiple of one subnet's mean stage slice "
                          "(0 = all candidates resident; P:L337 uses ~3)")
@@ -211,9 +212,39 @@ def secondary(args):
     try:
         out = subprocess.run(cmd, capture_output=True, text=True, timeout=300).stdout.strip().splitlines()
         d = json.loads(out[-1])
-        return {k: d[k] for k in ("value", "unit", "ms_per_step", "config", "roofline", "clocks", "gpu_launches")}
+        return {k: d.get(k) for k in ("value", "unit", "ms_per_step", "config", "roofline", "clocks", "gpu_launches",
+                                      "bit_repro")}
     except Exception as e:  # reported, never fatal for the headline line
         return {"error": repr(e)[:200]}
+
+
+def bit_repro(cfg, npipe, dev_pool, n_sub=8, stage_counts=(1, 1, 2, 4)):
+    """BJ's "bit-repro check" (Def.1, Table 3): train the same n_sub subnets
+    on the same device batches with fresh handles — twice at D=1, then at D=2 and D=4 (all
+    stages on this GPU; the stage boundaries then sit in the middle of the supernet) — and
+    hash every trained candidate's fp32 master plus the losses with SHA-256.  All digests must
+    be equal."""
+    import hashlib
+    m, n = cfg["n_blocks"], cfg["n_choices"]
+    choices = synth.sample_choices(n_sub, m, n)
+    used = sorted({(b, int(choices[y][b])) for y in range(n_sub) for b in range(m)})
+    digests = []
+    for D in stage_counts:
+        if D > m:
+            continue
+        h = npipe.naspipe_create(npipe.Spec(cfg), D)
+        for y in range(n_sub):
+            x, t = dev_pool[y % len(dev_pool)]
+            npipe.naspipe_submit(h, choices[y], x, t, where=npipe.BATCH_DEVICE)
+        npipe.naspipe_drain(h)
+        sha = hashlib.sha256()
+        for b, c in used:
+            sha.update(np.ascontiguousarray(npipe.naspipe_get_params(h, b, c), dtype=np.float32).tobytes())
+        sha.update(np.ascontiguousarray(npipe.naspipe_get_losses(h, n_sub), dtype=np.float32).tobytes())
+        npipe.naspipe_destroy(h)
+        digests.append({"stages": D, "sha256": sha.hexdigest()})
+    return {"subnets": n_sub, "candidates_hashed": len(used), "runs": digests,
+            "bitwise_equal": len({d["sha256"] for d in digests}) == 1}
 
 
 def workload_config(args, cfg, world):
@@ -386,6 +417,9 @@ def main():
                "d2h_bytes_per_step": 4}
     losses = npipe.naspipe_get_losses(h, y) if rank == world - 1 else None
     npipe.naspipe_destroy(h)
+    repro = None
+    if world == 1 and not args.no_repro and not args.budget_x:
+        repro = bit_repro(cfg, npipe, dev_pool)
 
     if rank != 0:
         return
@@ -404,7 +438,7 @@ def main():
                               "writebacks": s1["writebacks"] - s0["writebacks"],
                               "h2d_GBps": (s1["h2d_bytes"] - s0["h2d_bytes"]) / (ms / 1000) / 1e9,
                               "d2h_GBps": (s1["d2h_bytes"] - s0["d2h_bytes"]) / (ms / 1000) / 1e9} if budget else None,
-           "loss_finite": bool(losses is None or np.all(np.isfinite(losses)))}
+           "loss_finite": bool(losses is None or np.all(np.isfinite(losses))), "bit_repro": repro}
     if sec is not None:
         out["secondary"] = {"configs[2] transformer": sec}
     print(json.dumps(out))

@@ -742,8 +742,13 @@ void gemm_bf16_tc(cudaStream_t s, int M, int N, int K, const bf16* A, bool a_mn,
   if ((epi == EPI_SGD || epi == EPI_F32) && ep.ws != nullptr) {
     ts.splits = gemm_splitk_factor(M, N, K);
     if ((size_t)ts.splits * M * N > ep.ws_elems || (M * (size_t)N) % 4 != 0) ts.splits = 1;
+    static const bool no_split = getenv("NASPIPE_NO_SPLITK") != nullptr;  // diagnostics
+    if (no_split) ts.splits = 1;
   }
   ts.nk_per_split = (ts.nk + ts.splits - 1) / ts.splits;
+  // effective split count: every split owns >= 1 k-block (with ceil-sized splits the last
+  // ones could otherwise be empty and leave their workspace slice unwritten)
+  ts.splits = (ts.nk + ts.nk_per_split - 1) / ts.nk_per_split;
   const int run_epi = ts.splits > 1 ? EPI_PARTIAL : epi;
   ep.ws_stride = (size_t)M * N;
   if (pair) {
@@ -756,7 +761,8 @@ void gemm_bf16_tc(cudaStream_t s, int M, int N, int K, const bf16* A, bool a_mn,
   else if (a_mn && b_mn) dispatch_epi<true, true>(s, M, N, ts, ta, tb, run_epi, ep);
   else dispatch_epi<true, false>(s, M, N, ts, ta, tb, run_epi, ep);
   if (ts.splits > 1) {
-    const int L = ts.splits <= 4 ? 1 : std::min(32, ts.splits / 4);
+    int L = 1;  // lanes per output vector: a power of two (xor tree), <= splits / 4
+    while (2 * L <= 32 && 2 * L <= ts.splits / 4) L *= 2;
     const size_t per_block = 256 / L;
     const int blocks = (int)std::min<size_t>(((size_t)M * N / 4 + per_block - 1) / per_block, 4 * (size_t)num_sms());
     if (epi == EPI_F32)

@@ -112,6 +112,29 @@ def test_gemm_epilogues(M, N, K):
     assert _normwise(_f64(dz), C0 * gp) <= 2 ** -7
 
 
+@pytest.mark.parametrize("M,N,K", [(32, 32, 64 * 56 * 56), (80, 80, 64 * 28 * 28 + 64)])
+def test_gemm_splitk_ragged_k(M, N, K):
+    """Split-K with a k-block count the split factor does not divide (the SPOS weight
+    gradients: K = B*H*W pixels).  Every split must own >= 1 k-block: an empty split would
+    leave its workspace slice stale (here: filled with another GEMM's partials first), and
+    the result would depend on what ran before it."""
+    rng = np.random.default_rng(K)
+    junk = rng.standard_normal((512, 4096)).astype(np.float32)
+    jd = _dev(junk, torch.bfloat16)
+    _gemm(512, 512, 4096, jd, False, jd, False, 1, out=torch.empty((512, 512), device="cuda"))  # dirty workspace
+    A = rng.standard_normal((M, K)).astype(np.float32)
+    B = rng.standard_normal((N, K)).astype(np.float32)
+    Ad, Bd = _dev(A.T, torch.bfloat16), _dev(B.T, torch.bfloat16)   # MN-major, as the wgrad reads them
+    out = torch.empty((M, N), device="cuda", dtype=torch.float32)
+    _gemm(M, N, K, Ad, True, Bd, True, 1, out=out)
+    ref = _bf16_round(A) @ _bf16_round(B).T
+    assert _normwise(_f64(out), ref) <= 1e-5 * np.sqrt(K / 1024)
+    _gemm(512, 512, 4096, jd, False, jd, False, 1, out=torch.empty((512, 512), device="cuda"))
+    out2 = torch.empty_like(out)
+    _gemm(M, N, K, Ad, True, Bd, True, 1, out=out2)
+    assert torch.equal(out, out2), "split-K result depends on the workspace's previous contents"
+
+
 def test_gemm_sgd_epilogue():
     rng = np.random.default_rng(9)
     T, N, K = 4096, 1024, 768         # dW[N,K] = dY^T X : MN-major operands, K = T

@@ -106,3 +106,18 @@ def test_spos_full_size_one_step():
     assert a15 <= 1e-3, a15
     assert upd <= 0.3, upd   # bf16x2-storage oracle at this size: A15 1.5e-4, update 0.10
     np.testing.assert_allclose(losses, ref_loss, rtol=1e-2)
+
+
+def test_spos_full_size_bitwise_across_runs_and_stage_counts():
+    """configs[1] at full size: 3 subnets, twice at D = 1 and once at D = 2 and 4 (stages on
+    this GPU): parameters and losses bitwise equal (Def.1, Table 3).  At
+    this size the weight gradients take the split-K path with ragged k-block counts."""
+    cfg = synth.get_config("spos")
+    choices = synth.sample_choices(3, cfg["n_blocks"], cfg["n_choices"])
+    batches = [synth.make_batch(cfg, y) for y in range(3)]
+    base, base_loss, _, _ = run_engine(cfg, choices, batches, D=1)
+    for D in (1, 2, 4):
+        p, l, _, _ = run_engine(cfg, choices, batches, D=D, where=npipe.BATCH_DEVICE)
+        assert np.array_equal(l.view(np.uint32), base_loss.view(np.uint32)), D
+        for k in base:
+            assert np.array_equal(p[k].view(np.uint32), base[k].view(np.uint32)), (D, k)
