@@ -121,3 +121,4 @@ def test_spos_full_size_bitwise_across_runs_and_stage_counts():
         assert np.array_equal(l.view(np.uint32), base_loss.view(np.uint32)), D
         for k in base:
             assert np.array_equal(p[k].view(np.uint32), base[k].view(np.uint32)), (D, k)
+
