@@ -241,6 +241,26 @@ int naspipe_param_count(const naspipe_supernet_spec* spec, int32_t block, int32_
 int naspipe_default_costs(const naspipe_supernet_spec* spec, int32_t* cost_fwd, int32_t* cost_bwd);
 /* Stage of each block for n_stages (the spec's or the balanced partition). */
 int naspipe_partition(const naspipe_supernet_spec* spec, int32_t n_stages, int32_t* stage_of_block);
+/* Per-subnet balanced partitions with layer mirroring ("a D-partition
+ * ... of a subnet's sequential list of layers, with each partition having roughly the same
+ * execution time"; "Layer Mirroring ... the new parameters are actively pushed to all
+ * the other mirrored ones"; reading A31).  PLANNING ONLY (the executor runs the
+ * supernet partition of naspipe_partition).
+ *   Subnet y's stage of block b = the balanced partition (A12's DP and tie rule) of y's own
+ *   per-block costs cost_fwd + cost_bwd of (b, c_y[b]); stage_of_block [N*m] receives it.
+ *   Schedule: the O2 event model (spec window, link_latency, strict backward-first, lowest id)
+ *   with CSP read across stages: F(y, K) starts at t only if for each of y's blocks b on K
+ *   the previous user x of (b, c_y[b]) finished B(x, stage_x(b)) (its WRITE) by t, plus
+ *   mirror_latency ticks (>= 0) when stage_x(b) != K.
+ *   trace: 4 int64 per task start (tick, stage, kind 0=F/1=B, y), *n_tasks = 2*N*n_stages
+ *   (entries beyond cap_tasks are not written); stall/bubble [n_stages] or NULL.
+ *   Errors: EINVAL for a choice out of range, n_stages outside 1..m, a sync_policy other
+ *   than CSP or bwd_policy != 0, mirror_latency < 0, NULL n_tasks/makespan. */
+int naspipe_plan_mirrored(const naspipe_supernet_spec* spec, int32_t n_stages, const int32_t* choices,
+                          int64_t n_subnets, int32_t mirror_latency, int32_t* stage_of_block, int64_t* trace,
+                          size_t cap_tasks, size_t* n_tasks, int64_t* makespan, int64_t* stall,
+                          int64_t* bubble);
+
 /* Initial packed parameters of one candidate (same generator the engine uses). */
 int naspipe_init_params(const naspipe_supernet_spec* spec, int32_t block, int32_t choice,
                         float* dst, size_t n_floats);

@@ -274,3 +274,175 @@ def expected_versions(choices):
         for b in range(m):
             v[y, b] = sum(1 for x in range(y) if choices[x][b] == choices[y][b])
     return v
+
+
+# --------------------------------------------------------------------------------------
+# per-subnet balanced partitions with layer mirroring
+# --------------------------------------------------------------------------------------
+def subnet_partitions(choices, cost_f, cost_b, D):
+    """"The partition is a D-partition ... of a subnet's sequential list of layers,
+    with each partition having roughly the same execution time": subnet y's stage of block
+    b from balanced_partition over y's own per-block costs cf(b, c_y[b]) + cb(b, c_y[b])
+    (same tie rule as A12).  Returns int32 [N][m]."""
+    return np.array([balanced_partition([int(cost_f[b][c[b]]) + int(cost_b[b][c[b]]) for b in range(len(c))], D)
+                     for c in choices], dtype=np.int32)
+
+
+def simulate_csp_mirrored(choices, sob, D, W, cost_f, cost_b, lam=0, lam_w=0):
+    """O2 with a stage assignment per subnet (reading A31).  sob[y][b] = stage of block b in
+    subnet y; a candidate used by subnets on different stages is mirrored.
+
+    Task costs: cf[K][y] = max(1, sum of cost_f[b][c_y[b]] over y's blocks on K) (cb alike).
+    Dependency (Def.2): F(y, K) may start at t only if, for every block b of y on K
+    with an earlier user x = dep[y][b] of candidate (b, c_y[b]), x's WRITE of it — the end of
+    B(x, sob[x][b]) — happened at or before t, plus lam_w ticks when sob[x][b] != K (the
+    updated parameters are pushed to the mirror).  Everything else is O2: strict
+    backward-first, lowest id first, the stage-0 window W, deliveries after lam ticks.
+    With sob[y] equal for all y and lam_w = 0 this is simulate_csp.
+    Returns dict(trace, makespan, order, stall, bubble)."""
+    N, m = len(choices), len(choices[0])
+    sob = np.asarray(sob)
+    dep = dep_table(choices)
+    cf = np.zeros((D, N), dtype=np.int64)
+    cb = np.zeros((D, N), dtype=np.int64)
+    for y in range(N):
+        for K in range(D):
+            bl = [b for b in range(m) if sob[y][b] == K]
+            cf[K, y] = max(1, sum(int(cost_f[b][choices[y][b]]) for b in bl))
+            cb[K, y] = max(1, sum(int(cost_b[b][choices[y][b]]) for b in bl))
+    bend = {}                      # (x, K) -> end time of B(x, K)
+    inF = [set() for _ in range(D)]
+    inB = [set() for _ in range(D)]
+    fin0 = set()
+    started0 = set()
+    busy = [None] * D
+    deliveries = []
+    trace, order = [], [[] for _ in range(D)]
+    stall, bubble = [0] * D, [0] * D
+    t = 0
+
+    def ready_at(y, K):
+        """Earliest time F(y, K)'s dependencies allow (None while some WRITE is pending)."""
+        r = 0
+        for b in range(m):
+            if sob[y][b] != K or dep[y, b] < 0:
+                continue
+            x = int(dep[y, b])
+            Kx = int(sob[x][b])
+            if (x, Kx) not in bend or bend[(x, Kx)] > t:
+                return None
+            r = max(r, bend[(x, Kx)] + (lam_w if Kx != K else 0))
+        return r
+
+    while True:
+        for K in range(D):
+            if busy[K] is not None and busy[K][0] == t:
+                _, kind, y = busy[K]
+                busy[K] = None
+                if kind == 0:
+                    if K < D - 1:
+                        deliveries.append((t + lam, 0, K + 1, y))
+                    else:
+                        inB[K].add(y)
+                else:
+                    if K > 0:
+                        deliveries.append((t + lam, 1, K - 1, y))
+                    else:
+                        fin0.add(y)
+        keep = []
+        for dv in deliveries:
+            if dv[0] <= t:
+                (inF if dv[1] == 0 else inB)[dv[2]].add(dv[3])
+            else:
+                keep.append(dv)
+        deliveries = keep
+        if len(fin0) == N:
+            return dict(trace=trace, makespan=t, order=order, stall=stall, bubble=bubble)
+        wm0 = min([y for y in range(N) if y not in fin0], default=N)
+        for y in range(N):
+            if y < wm0 + W and y not in started0:
+                inF[0].add(y)
+        wake = []                  # future times at which a mirror push completes
+        for K in range(D):
+            if busy[K] is not None:
+                continue
+            choose = None
+            if inB[K]:
+                choose = (1, min(inB[K]))
+            else:
+                for y in sorted(inF[K]):
+                    r = ready_at(y, K)
+                    if r is None:
+                        continue
+                    if r <= t:
+                        choose = (0, y)
+                        break
+                    wake.append(r)
+            if choose is None:
+                continue
+            kind, y = choose
+            if kind == 0:
+                inF[K].discard(y)
+                if K == 0:
+                    started0.add(y)
+                busy[K] = (t + int(cf[K][y]), 0, y)
+            else:
+                inB[K].discard(y)
+                busy[K] = (t + int(cb[K][y]), 1, y)
+                bend[(y, K)] = t + int(cb[K][y])
+            trace.append((t, K, kind, y))
+            order[K].append((kind, y))
+        nxt = [b[0] for b in busy if b is not None] + [dv[0] for dv in deliveries] + [w for w in wake if w > t]
+        assert nxt, "mirrored CSP simulation stalled (no pending event)"
+        dt = min(nxt) - t
+        for K in range(D):
+            if busy[K] is None:
+                if inF[K]:
+                    stall[K] += dt
+                else:
+                    bubble[K] += dt
+        t = min(nxt)
+
+
+def check_trace_mirrored(trace, choices, sob, D, cost_b, lam_w=0):
+    """Validity of a mirrored trace: every task once; F(y,K) after F(y,K-1), B(y,K) after
+    B(y,K+1), F before B on a stage; and for every candidate l, in start-time order, its
+    users' accesses read F(x1) B(x1) F(x2) B(x2) ... with x1 < x2 < ... (Table 4 pattern,
+    P:L435) where each F(x_{i+1}) starts no earlier than B(x_i)'s end (+ lam_w across
+    stages).  Returns a list of violations."""
+    errs = []
+    N, m = len(choices), len(choices[0])
+    sob = np.asarray(sob)
+    pos = {}
+    for idx, (t, K, kind, y) in enumerate(trace):
+        if (kind, y, K) in pos:
+            errs.append(f"task twice {(kind, y, K)}")
+        pos[(kind, y, K)] = (t, idx)
+    for y in range(N):
+        for K in range(D):
+            if (0, y, K) not in pos or (1, y, K) not in pos:
+                errs.append(f"missing task y={y} K={K}")
+                continue
+            if pos[(0, y, K)] >= pos[(1, y, K)]:
+                errs.append(f"B before F y={y} K={K}")
+            if K > 0 and pos[(0, y, K)] <= pos[(0, y, K - 1)]:
+                errs.append(f"F({y},{K}) not after F({y},{K-1})")
+            if K < D - 1 and pos[(1, y, K)] <= pos[(1, y, K + 1)]:
+                errs.append(f"B({y},{K}) not after B({y},{K+1})")
+    acc = {}
+    for (t, K, kind, y) in trace:
+        for b in range(m):
+            if sob[y][b] == K:
+                acc.setdefault((b, int(choices[y][b])), []).append((t, kind, y, K))
+    for l, seq in acc.items():
+        users = sorted({y for _, _, y, _ in seq})
+        if [(k, y) for _, k, y, _ in seq] != [(k, y) for y in users for k in (0, 1)]:
+            errs.append(f"candidate {l} access order {[(k, y) for _, k, y, _ in seq]}")
+            continue
+        for i in range(1, len(users)):
+            tb, Kb = next((t, K) for t, k, y, K in seq if k == 1 and y == users[i - 1])
+            cbx = sum(int(cost_b[b][choices[users[i - 1]][b]]) for b in range(m) if sob[users[i - 1]][b] == Kb)
+            tf, Kf = next((t, K) for t, k, y, K in seq if k == 0 and y == users[i])
+            if tf < tb + max(1, cbx) + (lam_w if Kf != Kb else 0):
+                errs.append(f"candidate {l}: F({users[i]}) at {tf} before the WRITE of {users[i - 1]} landed")
+    return errs

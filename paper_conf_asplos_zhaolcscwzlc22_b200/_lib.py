@@ -70,6 +70,8 @@ _sig("naspipe_destroy", None, [C.c_void_p])
 _sig("naspipe_param_count", C.c_int, [_SP, C.c_int32, C.c_int32, C.POINTER(C.c_size_t)])
 _sig("naspipe_default_costs", C.c_int, [_SP, _i32p, _i32p])
 _sig("naspipe_partition", C.c_int, [_SP, C.c_int32, _i32p])
+_sig("naspipe_plan_mirrored", C.c_int, [_SP, C.c_int32, _i32p, C.c_int64, C.c_int32, _i32p, _i64p, C.c_size_t,
+                                        C.POINTER(C.c_size_t), _i64p, _i64p, _i64p])
 _sig("naspipe_init_params", C.c_int, [_SP, C.c_int32, C.c_int32, C.POINTER(C.c_float), C.c_size_t])
 _sig("naspipe_init_frozen", C.c_int, [_SP, C.c_int32, C.POINTER(C.c_float), C.c_size_t])
 _sig("naspipe_plan_create", C.c_int, [_SP, C.c_int32, _i32p, C.c_int64, C.POINTER(C.c_void_p)])
@@ -89,7 +91,7 @@ EXPORTED_SYMBOLS = [
     "naspipe_get_residency_trace", "naspipe_destroy", "naspipe_param_count", "naspipe_default_costs",
     "naspipe_partition", "naspipe_init_params", "naspipe_init_frozen", "naspipe_plan_create", "naspipe_plan_trace",
     "naspipe_plan_makespan", "naspipe_plan_deps", "naspipe_plan_residency", "naspipe_plan_destroy",
-    "naspipe_plan_comm_schedule", "naspipe_plan_idle",
+    "naspipe_plan_comm_schedule", "naspipe_plan_idle", "naspipe_plan_mirrored",
     "naspipe_nccl_unique_id", "naspipe_last_error", "naspipe_abi_version"]
 
 
@@ -286,6 +288,24 @@ def naspipe_partition(spec: Spec, n_stages: int) -> np.ndarray:
     out = np.zeros(spec.struct.n_blocks, dtype=np.int32)
     _check(lib.naspipe_partition(spec.ptr, n_stages, out.ctypes.data_as(_i32p)))
     return out
+
+
+def naspipe_plan_mirrored(spec: Spec, n_stages: int, choices, mirror_latency: int = 0) -> dict:
+    """Per-subnet balanced partitions with layer mirroring (planning only; include/naspipe.h):
+    dict(stage_of_block [N][m], trace [T][4] (tick, stage, kind, y), makespan, stall [D], bubble [D])."""
+    ch, chp = _i32(choices)
+    N = ch.shape[0] if ch.ndim == 2 else 0
+    m = spec.struct.n_blocks
+    sob = np.zeros((N, m), dtype=np.int32)
+    cap = 2 * N * n_stages
+    tr = np.zeros((max(cap, 1), 4), dtype=np.int64)
+    nt, ms = C.c_size_t(0), C.c_int64(0)
+    stall = np.zeros(n_stages, dtype=np.int64)
+    bubble = np.zeros(n_stages, dtype=np.int64)
+    _check(lib.naspipe_plan_mirrored(spec.ptr, n_stages, chp, N, int(mirror_latency),
+                                     sob.ctypes.data_as(_i32p), tr.ctypes.data_as(_i64p), cap, C.byref(nt),
+                                     C.byref(ms), stall.ctypes.data_as(_i64p), bubble.ctypes.data_as(_i64p)))
+    return dict(stage_of_block=sob, trace=tr[: nt.value], makespan=ms.value, stall=stall, bubble=bubble)
 
 
 def naspipe_init_params(spec: Spec, block: int, choice: int) -> np.ndarray:

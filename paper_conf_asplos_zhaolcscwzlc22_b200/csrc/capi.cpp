@@ -5,6 +5,7 @@
 #include <memory>
 
 #include "engine.h"
+#include "mirror.h"
 #include "planner.h"
 
 using namespace naspipe;
@@ -66,6 +67,29 @@ int naspipe_partition(const naspipe_supernet_spec* spec, int32_t n_stages, int32
     NP_REQUIRE(stage_of_block, NASPIPE_EINVAL, "NULL output");
     auto sob = s.partition(n_stages);
     std::memcpy(stage_of_block, sob.data(), sob.size() * sizeof(int32_t));
+  });
+}
+
+int naspipe_plan_mirrored(const naspipe_supernet_spec* spec, int32_t n_stages, const int32_t* choices,
+                          int64_t n_subnets, int32_t mirror_latency, int32_t* stage_of_block, int64_t* trace,
+                          size_t cap_tasks, size_t* n_tasks, int64_t* makespan, int64_t* stall, int64_t* bubble) {
+  return guarded([&] {
+    Spec s(spec);
+    NP_REQUIRE(n_tasks && makespan, NASPIPE_EINVAL, "NULL output");
+    const MirrorPlan P = plan_mirrored(s, n_stages, choices, n_subnets, mirror_latency);
+    if (stage_of_block) std::memcpy(stage_of_block, P.sob.data(), P.sob.size() * sizeof(int32_t));
+    *n_tasks = P.trace.size();
+    for (size_t i = 0; i < P.trace.size() && i < cap_tasks && trace; ++i) {
+      trace[4 * i] = P.trace[i].t;
+      trace[4 * i + 1] = P.trace[i].K;
+      trace[4 * i + 2] = P.trace[i].kind;
+      trace[4 * i + 3] = P.trace[i].y;
+    }
+    *makespan = P.makespan;
+    for (int K = 0; K < n_stages; ++K) {
+      if (stall) stall[K] = P.stall[K];
+      if (bubble) bubble[K] = P.bubble[K];
+    }
   });
 }
 

@@ -49,8 +49,22 @@ CandidateStore::CandidateStore(const Spec& spec, const Planner& planner, int K, 
       CU(cudaEventCreateWithFlags(&cands_[u].ready, cudaEventDisableTiming));
       CU(cudaEventCreateWithFlags(&cands_[u].last_use, cudaEventDisableTiming));
       CU(cudaEventCreateWithFlags(&cands_[u].wb_done, cudaEventDisableTiming));
+      CU(cudaEventCreateWithFlags(&cands_[u].h2d_done, cudaEventDisableTiming));
     }
     CU(cudaStreamCreateWithFlags(&evict_, cudaStreamNonBlocking));
+    CU(cudaStreamCreateWithFlags(&shadow_, cudaStreamNonBlocking));
+    CU(cudaStreamCreateWithFlags(&wb_, cudaStreamNonBlocking));
+    // write-back staging ring: an evicted dirty candidate is copied device-to-device into a
+    // staging slot (HBM speed) and its memory freed at once; the D2H from the slot runs on
+    // wb_.  A load that reuses the freed memory therefore waits only for the D2D copy, not for
+    // the PCIe write-back, so both PCIe directions stream concurrently.
+    size_t max_n32 = 0;
+    for (int u : uids) max_n32 = std::max(max_n32, cands_[u].n32);
+    for (int i = 0; i < kStage; ++i) {
+      CU(cudaMalloc(reinterpret_cast<void**>(&stage_[i]), max_n32 * 4));
+      CU(cudaEventCreateWithFlags(&stage_free_[i], cudaEventDisableTiming));
+      CU(cudaEventCreateWithFlags(&staged_[i], cudaEventDisableTiming));
+    }
     // keep freed blocks in the stream-ordered pool: loads reuse evicted memory
     cudaMemPool_t pool;
     CU(cudaDeviceGetDefaultMemPool(&pool, dev));
@@ -104,7 +118,8 @@ CandidateStore::CandidateStore(const Spec& spec, const Planner& planner, int K, 
 
 CandidateStore::~CandidateStore() {
   cudaSetDevice(dev_);
-  if (evict_) cudaStreamSynchronize(evict_);  // write-backs into the stash have landed
+  if (evict_) cudaStreamSynchronize(evict_);
+  if (wb_) cudaStreamSynchronize(wb_);  // write-backs into the stash have landed
   for (auto& cd : cands_) {
     if (cd.stash) cudaFreeHost(cd.stash);
     if (managed() && cd.w32) cudaFree(cd.w32);
@@ -112,10 +127,24 @@ CandidateStore::~CandidateStore() {
     if (cd.ready) cudaEventDestroy(cd.ready);
     if (cd.last_use) cudaEventDestroy(cd.last_use);
     if (cd.wb_done) cudaEventDestroy(cd.wb_done);
+    if (cd.h2d_done) cudaEventDestroy(cd.h2d_done);
   }
   if (evict_) {
     cudaStreamSynchronize(evict_);
     cudaStreamDestroy(evict_);
+  }
+  if (shadow_) {
+    cudaStreamSynchronize(shadow_);
+    cudaStreamDestroy(shadow_);
+  }
+  if (wb_) {
+    cudaStreamSynchronize(wb_);
+    cudaStreamDestroy(wb_);
+  }
+  for (int i = 0; i < kStage; ++i) {
+    if (stage_[i]) cudaFree(stage_[i]);
+    if (stage_free_[i]) cudaEventDestroy(stage_free_[i]);
+    if (staged_[i]) cudaEventDestroy(staged_[i]);
   }
 }
 
@@ -140,8 +169,12 @@ void CandidateStore::load(Cand& cd, cudaStream_t copy) {
   if (cd.n16) CU(cudaMallocAsync(reinterpret_cast<void**>(&cd.w16), cd.n16 * 2, copy));
   CU(cudaMemcpyAsync(cd.w32, cd.stash, cd.n32 * 4, cudaMemcpyHostToDevice, copy));
   fam_->bind(cd.j, cd.c, cd.w32, cd.w16);
-  fam_->refresh_shadow(cd.j, cd.c, copy);
-  CU(cudaEventRecord(cd.ready, copy));
+  // the bf16 shadow is a kernel: on its own stream, so the copy stream's next H2D does not
+  // queue behind it while the compute stream holds the SMs
+  CU(cudaEventRecord(cd.h2d_done, copy));
+  CU(cudaStreamWaitEvent(shadow_, cd.h2d_done, 0));
+  fam_->refresh_shadow(cd.j, cd.c, shadow_);
+  CU(cudaEventRecord(cd.ready, shadow_));
   h2d_bytes += 4.0 * cd.n32;
   ++loads;
 }
@@ -150,11 +183,20 @@ void CandidateStore::evict(Cand& cd, bool writeback, cudaStream_t) {
   CU(cudaStreamWaitEvent(evict_, cd.last_use, 0));  // the last task reading/updating it is done
   CU(cudaStreamWaitEvent(evict_, cd.ready, 0));     // (and its load finished)
   if (writeback) {
-    CU(cudaMemcpyAsync(cd.stash, cd.w32, cd.n32 * 4, cudaMemcpyDeviceToHost, evict_));
+    const int k = stage_next_++ % kStage;
+    if (stage_used_[k]) CU(cudaStreamWaitEvent(evict_, stage_free_[k], 0));  // slot's previous D2H done
+    CU(cudaMemcpyAsync(stage_[k], cd.w32, cd.n32 * 4, cudaMemcpyDeviceToDevice, evict_));
+    CU(cudaEventRecord(staged_[k], evict_));
+    CU(cudaStreamWaitEvent(wb_, staged_[k], 0));
+    CU(cudaMemcpyAsync(cd.stash, stage_[k], cd.n32 * 4, cudaMemcpyDeviceToHost, wb_));
+    CU(cudaEventRecord(stage_free_[k], wb_));
+    CU(cudaEventRecord(cd.wb_done, wb_));
+    stage_used_[k] = true;
     d2h_bytes += 4.0 * cd.n32;
     ++writebacks;
+  } else {
+    CU(cudaEventRecord(cd.wb_done, evict_));
   }
-  CU(cudaEventRecord(cd.wb_done, evict_));
   CU(cudaFreeAsync(cd.w32, evict_));
   if (cd.w16) CU(cudaFreeAsync(cd.w16, evict_));
   cd.w32 = nullptr;
@@ -191,6 +233,8 @@ void CandidateStore::after_task(const Task& t, cudaStream_t comp) {
 
 void CandidateStore::sync() {
   if (evict_) CU(cudaStreamSynchronize(evict_));
+  if (wb_) CU(cudaStreamSynchronize(wb_));
+  if (shadow_) CU(cudaStreamSynchronize(shadow_));
 }
 
 void CandidateStore::get(int b, int c, float* dst) {

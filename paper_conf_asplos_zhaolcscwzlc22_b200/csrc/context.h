@@ -6,8 +6,9 @@
 // the supernet's operators all reside in CPU storage"); before each task the Belady plan
 // (BeladyResidency: farthest next use within the horizon, depth-L prefetch that fits the
 // budget) issues EVICTs (D2H write-back only if updated since load) and LOADs (H2D + bf16
-// shadow refresh) on the stage's copy stream (write-backs on their own stream, so both PCIe
-// directions run concurrently); the compute stream waits only for the
+// shadow refresh) on the stage's copy stream; an eviction copies a dirty candidate into a
+// device staging slot and frees it at once, the D2H from the slot and the shadow kernels run
+// on their own streams, so both PCIe directions stay busy; the compute stream waits only for the
 // candidates of the task it is about to run, so prefetches for later tasks overlap compute.
 // Numerics are unaffected by residency: a candidate's bytes are the same wherever it lives.
 #pragma once
@@ -53,7 +54,7 @@ class CandidateStore {
     float* stash = nullptr;  // pinned host fp32 master (managed mode)
     float* w32 = nullptr;    // device, when resident
     bf16* w16 = nullptr;
-    cudaEvent_t ready = nullptr, last_use = nullptr, wb_done = nullptr;
+    cudaEvent_t ready = nullptr, last_use = nullptr, wb_done = nullptr, h2d_done = nullptr;
   };
   int uid_of(int b, int c) const { return b * n_ + c; }
   std::vector<int64_t> task_uids(const Task& t) const;
@@ -66,7 +67,14 @@ class CandidateStore {
   Family* fam_;
   int64_t budget_;
   std::vector<Cand> cands_;  // indexed by uid (only this stage's blocks are populated)
-  cudaStream_t evict_ = nullptr;  // D2H write-backs + frees, concurrent with the H2D loads
+  cudaStream_t evict_ = nullptr;   // evictions: D2D into a staging slot, then the free
+  cudaStream_t shadow_ = nullptr;  // bf16 shadow refresh of loaded candidates (a kernel)
+  cudaStream_t wb_ = nullptr;      // D2H of staged write-backs
+  static constexpr int kStage = 2;  // write-back staging slots (max candidate fp32 bytes each)
+  float* stage_[kStage] = {nullptr, nullptr};
+  cudaEvent_t stage_free_[kStage] = {nullptr, nullptr}, staged_[kStage] = {nullptr, nullptr};
+  bool stage_used_[kStage] = {false, false};
+  uint64_t stage_next_ = 0;
   std::unique_ptr<BeladyResidency> belady_;
 };
 

@@ -361,20 +361,14 @@ void Spec::validate_stages(int D) const {
                NASPIPE_EINVAL, "stage_of_block must be contiguous and non-decreasing");
 }
 
-// Balanced contiguous partition: minimise the max stage weight, weight(b) = sum_c (cf+cb);
-// ties -> lexicographically smallest split points (reading A12).  Exact integer DP.
-std::vector<int32_t> Spec::partition(int D) const {
-  validate_stages(D);
-  if (has_partition) return stage_of_block;
-  std::vector<int32_t> cf, cb;
-  costs(cf, cb);
-  const int M = m();
+// Balanced contiguous partition of per-block weights w into D non-empty stages: minimise the
+// max stage weight; ties -> lexicographically smallest split points (reading A12).  Exact
+// integer DP.
+std::vector<int32_t> balanced_partition(const std::vector<int64_t>& w, int D) {
+  const int M = (int)w.size();
+  NP_REQUIRE(D >= 1 && D <= M, NASPIPE_EINVAL, "partition of %d blocks into %d stages", M, D);
   std::vector<int64_t> pre(M + 1, 0);
-  for (int b = 0; b < M; ++b) {
-    int64_t w = 0;
-    for (int c = 0; c < n(); ++c) w += (int64_t)cf[b * n() + c] + cb[b * n() + c];
-    pre[b + 1] = pre[b] + w;
-  }
+  for (int b = 0; b < M; ++b) pre[b + 1] = pre[b] + w[b];
   auto seg = [&](int i, int e) { return pre[e] - pre[i]; };
   const int64_t INF = std::numeric_limits<int64_t>::max();
   // g[k][i]: min over splits of blocks [i, M) into k non-empty stages of the max weight
@@ -397,6 +391,18 @@ std::vector<int32_t> Spec::partition(int D) const {
   }
   for (int b = start; b < M; ++b) sob[b] = D - 1;
   return sob;
+}
+
+// The supernet partition: the spec's, else balanced over weight(b) = sum_c (cf + cb).
+std::vector<int32_t> Spec::partition(int D) const {
+  validate_stages(D);
+  if (has_partition) return stage_of_block;
+  std::vector<int32_t> cf, cb;
+  costs(cf, cb);
+  std::vector<int64_t> w(m(), 0);
+  for (int b = 0; b < m(); ++b)
+    for (int c = 0; c < n(); ++c) w[b] += (int64_t)cf[b * n() + c] + cb[b * n() + c];
+  return balanced_partition(w, D);
 }
 
 }  // namespace naspipe

@@ -9,6 +9,10 @@
 
 namespace naspipe {
 
+// contiguous partition of per-block weights into D stages minimising the max stage weight,
+// ties -> lexicographically smallest split points (reading A12)
+std::vector<int32_t> balanced_partition(const std::vector<int64_t>& w, int D);
+
 // One tensor of a candidate's packed parameter vector.
 struct Segment {
   size_t offset, size;

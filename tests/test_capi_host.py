@@ -1,6 +1,7 @@
 """Host-side C ABI tests (no GPU): the library loads and exports every declared symbol; the
 C++ planner, dependency table, partition, residency planner and initialiser agree
 bit-exactly with the oracle (SURVEY §4 tier T1)."""
+import json
 import os
 import re
 
@@ -215,3 +216,42 @@ def test_bsp_is_plan_only():
     with pytest.raises(npipe.NaspipeError) as e:
         npipe.naspipe_create(npipe.Spec(cfg), 1)
     assert e.value.code == -1
+
+
+def test_mirrored_plan_matches_oracle_bit_exact():
+    """naspipe_plan_mirrored (C++) vs oracle.csp.simulate_csp_mirrored: partitions, every
+    task start, makespan and idle ticks, on the worked example and random cases."""
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "mirror_worked_example.json")))
+    base = synth.get_config("toy")
+    cfg = dict(base, n_blocks=3, n_choices=2, cost_fwd=np.array(g["cost_f"]), cost_bwd=np.array(g["cost_b"]), window=4)
+    for key, lw in (("lam_w_0", 0), ("lam_w_3", 3)):
+        r = npipe.naspipe_plan_mirrored(npipe.Spec(cfg), 2, g["choices"], lw)
+        assert r["stage_of_block"].tolist() == g["stage_of_block"]
+        assert r["trace"].tolist() == g[key]["trace"] and r["makespan"] == g[key]["makespan"]
+    rng = np.random.default_rng(5)
+    for _ in range(40):
+        m, n = int(rng.integers(2, 8)), int(rng.integers(1, 5))
+        D, N = int(rng.integers(1, min(m, 4) + 1)), int(rng.integers(1, 16))
+        W, lam, lw = int(rng.integers(1, 6)), int(rng.integers(0, 3)), int(rng.integers(0, 4))
+        ch = rng.integers(0, n, (N, m))
+        cf, cb = rng.integers(0, 5, (m, n)), rng.integers(0, 9, (m, n))
+        spec = npipe.Spec(dict(base, n_blocks=m, n_choices=n, cost_fwd=cf, cost_bwd=cb, window=W, link_latency=lam))
+        r = npipe.naspipe_plan_mirrored(spec, D, ch, lw)
+        sob = csp.subnet_partitions(ch.tolist(), cf, cb, D)
+        o = csp.simulate_csp_mirrored(ch.tolist(), sob, D, W, cf, cb, lam=lam, lam_w=lw)
+        assert np.array_equal(r["stage_of_block"], sob)
+        assert [tuple(t) for t in r["trace"].tolist()] == [tuple(t) for t in o["trace"]]
+        assert r["makespan"] == o["makespan"]
+        assert r["stall"].tolist() == list(o["stall"]) and r["bubble"].tolist() == list(o["bubble"])
+
+
+def test_mirrored_plan_rejects_other_policies():
+    cfg = synth.get_config("toy")
+    ch = synth.sample_choices(3, cfg["n_blocks"], cfg["n_choices"])
+    for over in (dict(sync="asp"), dict(bwd_policy=1)):
+        with pytest.raises(npipe.NaspipeError):
+            npipe.naspipe_plan_mirrored(npipe.Spec(cfg, **over), 2, ch)
+    with pytest.raises(npipe.NaspipeError):
+        npipe.naspipe_plan_mirrored(npipe.Spec(cfg), 2, ch, -1)
+    with pytest.raises(npipe.NaspipeError):
+        npipe.naspipe_plan_mirrored(npipe.Spec(cfg), 2, np.full_like(ch, cfg["n_choices"]))

@@ -250,3 +250,79 @@ def test_asp_is_the_no_dependency_schedule():
     # with conflicts it violates the Table 4 access pattern (CSP never does)
     assert csp.check_trace(a["trace"], ch, sob, 4) != []
     assert csp.check_trace(csp.simulate_csp(ch, sob, 4, 16, tf, tb)["trace"], ch, sob, 4) == []
+
+
+# ---------------------------------------------------------------------- §8f(2) mirroring
+def _mirror_golden():
+    with open(os.path.join(os.path.dirname(__file__), "golden", "mirror_worked_example.json")) as f:
+        return json.load(f)
+
+
+def test_mirrored_worked_example():
+    g = _mirror_golden()
+    sob = csp.subnet_partitions(g["choices"], g["cost_f"], g["cost_b"], g["D"])
+    assert sob.tolist() == g["stage_of_block"]
+    for key, lw in (("lam_w_0", 0), ("lam_w_3", 3)):
+        r = csp.simulate_csp_mirrored(g["choices"], sob, g["D"], g["W"], g["cost_f"], g["cost_b"], lam_w=lw)
+        assert [list(t) for t in r["trace"]] == g[key]["trace"], key
+        assert r["makespan"] == g[key]["makespan"], key
+        assert csp.check_trace_mirrored(r["trace"], g["choices"], sob, g["D"], g["cost_b"], lam_w=lw) == []
+    r = csp.simulate_csp_mirrored(g["choices"], sob, g["D"], g["W"], g["cost_f"], g["cost_b"])
+    assert r["stall"] == g["lam_w_0"]["stall"] and r["bubble"] == g["lam_w_0"]["bubble"]
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_mirrored_reduces_to_o2_on_a_common_partition(seed):
+    """Every subnet on the supernet partition, no mirror latency: exactly simulate_csp."""
+    rng = np.random.default_rng(100 + seed)
+    m, n, D, N, W, lam = 6, 3, 3, 14, 3, seed % 2
+    ch = rng.integers(0, n, (N, m)).tolist()
+    cf, cb = rng.integers(0, 5, (m, n)), rng.integers(1, 9, (m, n))
+    sob = csp.balanced_partition(csp.block_partition_cost(cf, cb), D)
+    a = csp.simulate_csp(ch, sob, D, W, *csp.task_costs(ch, sob, cf, cb, D), lam=lam)
+    b = csp.simulate_csp_mirrored(ch, [sob] * N, D, W, cf, cb, lam=lam)
+    for k in ("trace", "makespan", "stall", "bubble"):
+        assert a[k] == b[k], k
+
+
+@pytest.mark.parametrize("D", [2, 3])
+def test_mirrored_single_choice_is_sequential(D):
+    """n = 1: every subnet shares every candidate (and so has the same partition): the
+    schedule is strictly sequential, makespan = N * (sum of the subnet's task costs)."""
+    m, N = 5, 6
+    cf = np.array([[1], [3], [2], [4], [1]])
+    cb = 2 * cf
+    ch = [[0] * m for _ in range(N)]
+    sob = csp.subnet_partitions(ch, cf, cb, D)
+    r = csp.simulate_csp_mirrored(ch, sob, D, 4, cf, cb)
+    per = sum(max(1, int(sum(cf[b][0] for b in range(m) if sob[0][b] == K))) +
+              max(1, int(sum(cb[b][0] for b in range(m) if sob[0][b] == K))) for K in range(D))
+    assert r["makespan"] == N * per
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_mirrored_traces_are_csp_valid_and_idle_adds_up(seed):
+    rng = np.random.default_rng(200 + seed)
+    m, n, D, N = int(rng.integers(3, 8)), int(rng.integers(2, 5)), int(rng.integers(2, 4)), 16
+    ch = rng.integers(0, n, (N, m)).tolist()
+    cf, cb = rng.integers(0, 6, (m, n)), rng.integers(0, 12, (m, n))
+    sob = csp.subnet_partitions(ch, cf, cb, D)
+    for lw in (0, 2):
+        r = csp.simulate_csp_mirrored(ch, sob, D, 4, cf, cb, lam_w=lw)
+        assert csp.check_trace_mirrored(r["trace"], ch, sob, D, cb, lam_w=lw) == []
+        for K in range(D):
+            busy = 0
+            for (t, KK, kind, y) in r["trace"]:
+                if KK == K:
+                    bl = [b for b in range(m) if sob[y][b] == K]
+                    busy += max(1, int(sum((cf if kind == 0 else cb)[b][ch[y][b]] for b in bl)))
+            assert busy + r["stall"][K] + r["bubble"][K] == r["makespan"]
+
+
+def test_mirrored_checker_rejects_early_read():
+    g = _mirror_golden()
+    sob = np.array(g["stage_of_block"])
+    bad = [list(t) for t in g["lam_w_0"]["trace"]]
+    bad[5] = [17, 1, 0, 1]   # F(1, stage 1) one tick before the WRITE of (1,0) lands
+    assert csp.check_trace_mirrored(bad, g["choices"], sob, g["D"], g["cost_b"])
+    assert csp.check_trace_mirrored(g["lam_w_0"]["trace"], g["choices"], sob, g["D"], g["cost_b"], lam_w=3)
