@@ -70,10 +70,11 @@ typedef enum { NASPIPE_MLP = 0, NASPIPE_TRANSFORMER = 1, NASPIPE_SPOS_CNN = 2 } 
  *   BSP      bulk synchronous (GPipe / Retiarii): bulks of `bulk_size`
  *            consecutive subnets; within a bulk dependencies are ignored, forwards run
  *            before backwards on every stage, and the next bulk starts after the flush
- *            (every subnet of the bulk finished on every stage).  Its numerics (the bulk's
- *            gradients summed at the bulk's start weights) need gradient accumulation, which
- *            the executor does not implement: BSP is a planning policy only
- *            (naspipe_plan_*; naspipe_create rejects it with EINVAL). */
+ *            (every subnet of the bulk finished on every stage).  Numerics: every task of a
+ *            bulk reads the bulk-start weights, the SGD WRITEs accumulate into a per-
+ *            candidate fp32 copy, copied back into the masters at the flush (= the bulk's
+ *            gradients, summed, applied once).  Executable with every candidate resident
+ *            (naspipe_create: EINVAL with hbm_weight_budget_bytes > 0). */
 typedef enum { NASPIPE_SYNC_CSP = 0, NASPIPE_SYNC_INORDER = 1, NASPIPE_SYNC_ASP = 2, NASPIPE_SYNC_BSP = 3 } naspipe_sync;
 typedef enum { NASPIPE_FP32 = 0, NASPIPE_BF16 = 1 } naspipe_dtype; /* compute dtype; masters fp32 */
 

@@ -250,8 +250,8 @@ int naspipe_create(const naspipe_supernet_spec* spec, int32_t n_stages, naspipe_
   return guarded([&] {
     NP_REQUIRE(out, NASPIPE_EINVAL, "out NULL");
     const Spec sp(spec);
-    NP_REQUIRE(sp.raw.sync_policy != NASPIPE_SYNC_BSP, NASPIPE_EINVAL,
-               "BSP is a planning policy only (its bulk update needs gradient accumulation): use naspipe_plan_*");
+    NP_REQUIRE(sp.raw.sync_policy != NASPIPE_SYNC_BSP || sp.raw.hbm_weight_budget_bytes == 0, NASPIPE_EINVAL,
+               "BSP runs with every candidate resident (hbm_weight_budget_bytes = 0)");
     auto h = std::make_unique<naspipe_handle>();
     h->eng = Engine::create_local(sp, n_stages);
     *out = h.release();
@@ -263,8 +263,8 @@ int naspipe_create_rank(const naspipe_supernet_spec* spec, int32_t n_stages, int
   return guarded([&] {
     NP_REQUIRE(out, NASPIPE_EINVAL, "out NULL");
     const Spec sp(spec);
-    NP_REQUIRE(sp.raw.sync_policy != NASPIPE_SYNC_BSP, NASPIPE_EINVAL,
-               "BSP is a planning policy only (its bulk update needs gradient accumulation): use naspipe_plan_*");
+    NP_REQUIRE(sp.raw.sync_policy != NASPIPE_SYNC_BSP || sp.raw.hbm_weight_budget_bytes == 0, NASPIPE_EINVAL,
+               "BSP runs with every candidate resident (hbm_weight_budget_bytes = 0)");
     auto h = std::make_unique<naspipe_handle>();
     h->eng = Engine::create_rank(sp, n_stages, stage_rank, device, nccl_ids);
     *out = h.release();

@@ -226,7 +226,30 @@ void CandidateStore::before_task(const Task& t, cudaStream_t comp, cudaStream_t 
   }
 }
 
+void CandidateStore::enable_bsp(DevArena* arena) {
+  NP_REQUIRE(!managed(), NASPIPE_EINVAL, "BSP needs every candidate resident");
+  CU(cudaSetDevice(dev_));
+  for (auto& cd : cands_) {
+    if (cd.j < 0) continue;
+    cd.acc = arena->alloc<float>(cd.n32);
+    CU(cudaMemcpy(cd.acc, cd.w32, cd.n32 * 4, cudaMemcpyDeviceToDevice));
+    fam_->bind_update(cd.j, cd.c, cd.acc);
+  }
+  bsp_ = true;
+}
+
+void CandidateStore::bsp_flush(cudaStream_t s) {
+  for (auto& cd : cands_) {
+    if (!cd.dirty) continue;
+    CU(cudaMemcpyAsync(cd.w32, cd.acc, cd.n32 * 4, cudaMemcpyDeviceToDevice, s));
+    fam_->refresh_shadow(cd.j, cd.c, s);
+    cd.dirty = false;
+  }
+}
+
 void CandidateStore::after_task(const Task& t, cudaStream_t comp) {
+  if (bsp_ && t.kind == 1)
+    for (int64_t u : task_uids(t)) cands_[u].dirty = true;
   if (!managed()) return;
   for (int64_t u : task_uids(t)) CU(cudaEventRecord(cands_[u].last_use, comp));
 }
@@ -248,6 +271,7 @@ void CandidateStore::set(int b, int c, const float* src, cudaStream_t s) {
   Cand& cd = cands_[uid_of(b, c)];
   CU(cudaSetDevice(dev_));
   if (cd.stash) std::memcpy(cd.stash, src, cd.n32 * 4);
+  if (cd.acc) CU(cudaMemcpy(cd.acc, src, cd.n32 * 4, cudaMemcpyHostToDevice));
   if (cd.w32) {
     CU(cudaMemcpy(cd.w32, src, cd.n32 * 4, cudaMemcpyHostToDevice));
     fam_->refresh_shadow(cd.j, cd.c, s);

@@ -39,6 +39,13 @@ class CandidateStore {
   void after_task(const Task& t, cudaStream_t comp);
 
   void sync();  // wait for outstanding write-backs
+
+  // BSP (reading A30; all candidates resident): an fp32 accumulator per candidate takes the
+  // SGD WRITEs of a bulk (Family::bind_update) while the bulk reads the masters; after_task
+  // marks a backward's candidates dirty, bsp_flush copies the dirty accumulators into the
+  // masters and refreshes their bf16 shadows on stream s.
+  void enable_bsp(DevArena* arena);
+  void bsp_flush(cudaStream_t s);
   // read-out (streams idle)
   void get(int b, int c, float* dst);
   void set(int b, int c, const float* src, cudaStream_t s);
@@ -55,6 +62,8 @@ class CandidateStore {
     float* w32 = nullptr;    // device, when resident
     bf16* w16 = nullptr;
     cudaEvent_t ready = nullptr, last_use = nullptr, wb_done = nullptr, h2d_done = nullptr;
+    float* acc = nullptr;  // BSP accumulator
+    bool dirty = false;
   };
   int uid_of(int b, int c) const { return b * n_ + c; }
   std::vector<int64_t> task_uids(const Task& t) const;
@@ -76,6 +85,7 @@ class CandidateStore {
   bool stage_used_[kStage] = {false, false};
   uint64_t stage_next_ = 0;
   std::unique_ptr<BeladyResidency> belady_;
+  bool bsp_ = false;
 };
 
 }  // namespace naspipe

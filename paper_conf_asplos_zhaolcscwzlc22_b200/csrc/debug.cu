@@ -150,7 +150,7 @@ int naspipe_debug_bn_bwd(const void* dy, int lddy, const void* z, int P, int C, 
     NP_REQUIRE(cudaMalloc(&part, (size_t)nblk * 2 * C * 4) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
     NP_REQUIRE(cudaMalloc(&ctr, 4) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
     cudaMemsetAsync(ctr, 0, 4, s);
-    bn_bwd_reduce(s, (const bf16*)dy, lddy, (const bf16*)z, P, C, mean, rstd, g, b, relu, part, ctr, sums, old, lr,
+    bn_bwd_reduce(s, (const bf16*)dy, lddy, (const bf16*)z, P, C, mean, rstd, g, b, g, b, relu, part, ctr, sums, old, lr,
                   update);
     bn_bwd_apply(s, (const bf16*)dy, lddy, (const bf16*)z, P, C, mean, rstd, old, sums, relu, (bf16*)dz);
     cudaStreamSynchronize(s);

@@ -146,9 +146,10 @@ __global__ void mlp_fwd_kernel(const float* __restrict__ x, const float* __restr
 }
 
 // dz = dy (1 - h^2); dx = dy + dz W (pre-update); W -= lr dz^T x; b -= lr sum_r dz
+// W, b: the weights this subnet read (input gradient); Wu, bu: the SGD WRITE targets (== W, b
+// in place; the bulk accumulator copy under BSP, reading A30)
 __global__ void mlp_bwd_kernel(const float* __restrict__ x, const float* __restrict__ h, const float* __restrict__ dy,
-                               float* __restrict__ dx, float* __restrict__ W, float* __restrict__ b, float lr, int B,
-                               int d) {
+                               float* __restrict__ dx, const float* W, float* Wu, float* bu, float lr, int B, int d) {
   extern __shared__ float dz[];
   for (int idx = threadIdx.x; idx < B * d; idx += blockDim.x) {
     const float hv = h[idx];
@@ -168,12 +169,12 @@ __global__ void mlp_bwd_kernel(const float* __restrict__ x, const float* __restr
     const int j = idx / d, k = idx % d;
     float g = 0.f;
     for (int r = 0; r < B; ++r) g = fmaf(dz[r * d + j], x[r * d + k], g);
-    W[idx] -= lr * g;
+    Wu[idx] -= lr * g;
   }
   for (int j = threadIdx.x; j < d; j += blockDim.x) {
     float g = 0.f;
     for (int r = 0; r < B; ++r) g += dz[r * d + j];
-    b[j] -= lr * g;
+    bu[j] -= lr * g;
   }
 }
 
@@ -232,13 +233,13 @@ void mlp_fwd(cudaStream_t s, const float* x, const float* W, const float* b, flo
   check_launch("mlp_fwd");
 }
 
-void mlp_bwd_sgd(cudaStream_t s, const float* x, const float* h, const float* dy, float* dx, float* W, float* b,
-                 float lr, int B, int d) {
+void mlp_bwd_sgd(cudaStream_t s, const float* x, const float* h, const float* dy, float* dx, const float* W, float* Wu,
+                 float* bu, float lr, int B, int d) {
   const size_t smem = (size_t)B * d * sizeof(float);
   NP_REQUIRE(smem <= 200 * 1024, NASPIPE_EINVAL, "MLP batch*width too large for one CTA");
   if (smem > 48 * 1024)
     cudaFuncSetAttribute(mlp_bwd_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  mlp_bwd_kernel<<<1, 512, smem, s>>>(x, h, dy, dx, W, b, lr, B, d);
+  mlp_bwd_kernel<<<1, 512, smem, s>>>(x, h, dy, dx, W, Wu, bu, lr, B, d);
   check_launch("mlp_bwd_sgd");
 }
 

@@ -85,8 +85,8 @@ struct Transport {
 
 // ------------------------------------------------------------------------------ construction
 Engine::Engine(const Spec& spec, int D) : spec_(spec), D_(D), W_(spec.window(D)), planner_(spec_, D) {
-  NP_REQUIRE(spec_.raw.sync_policy != NASPIPE_SYNC_BSP, NASPIPE_EINVAL,
-             "BSP is a planning policy only (its bulk update needs gradient accumulation): use naspipe_plan_*");
+  NP_REQUIRE(spec_.raw.sync_policy != NASPIPE_SYNC_BSP || spec_.raw.hbm_weight_budget_bytes == 0, NASPIPE_EINVAL,
+             "BSP runs with every candidate resident (hbm_weight_budget_bytes = 0)");
   version_.assign((size_t)spec_.m() * spec_.n(), 0);
   timer_.on = (spec_.raw.flags & NASPIPE_FLAG_TIMING) != 0;
 }
@@ -175,6 +175,7 @@ void Engine::setup_stage(int K, int dev, bool local) {
   st.fam->timer = &timer_;
   st.store = std::make_unique<CandidateStore>(spec_, planner_, K, dev, st.fam.get(), st.arena.get(),
                                               spec_.raw.hbm_weight_budget_bytes);
+  if (spec_.raw.sync_policy == NASPIPE_SYNC_BSP) st.store->enable_bsp(st.arena.get());
   st.in.assign(W_, nullptr);
   st.gout.assign(W_, nullptr);
   st.out.resize(W_);
@@ -297,6 +298,7 @@ void Engine::drain() {
   for (auto& st : st_) {
     if (!st.local) continue;
     CU(cudaSetDevice(st.dev));
+    if (spec_.raw.sync_policy == NASPIPE_SYNC_BSP) st.store->bsp_flush(st.comp);  // the last bulk's flush
     CU(cudaStreamSynchronize(st.copy));
     CU(cudaStreamSynchronize(st.comp));
     st.store->sync();
@@ -369,9 +371,19 @@ void Engine::issue(const Task& t) {
   }
   if (!st.local) return;
   // the version invariant is CSP's (and INORDER's); ASP reads whatever version is current
-  if ((spec_.raw.flags & NASPIPE_FLAG_VERSION_CHECK) && spec_.raw.sync_policy != NASPIPE_SYNC_ASP) version_check(t);
+  if ((spec_.raw.flags & NASPIPE_FLAG_VERSION_CHECK) && spec_.raw.sync_policy != NASPIPE_SYNC_ASP &&
+      spec_.raw.sync_policy != NASPIPE_SYNC_BSP)
+    version_check(t);
   if (spec_.raw.flags & NASPIPE_FLAG_TRACE) trace_.push_back(t);
   CU(cudaSetDevice(st.dev));
+  if (spec_.raw.sync_policy == NASPIPE_SYNC_BSP) {
+    // BSP flush (reading A30): the first task of a new bulk on this stage runs after every
+    // task of the previous bulk (the plan's flush; same stream), so the accumulated WRITEs
+    // become the masters the new bulk reads
+    const int64_t bulk = t.y / spec_.bulk(D_);
+    if (bulk != st.bulk) st.store->bsp_flush(st.comp);
+    st.bulk = bulk;
+  }
   st.store->before_task(t, st.comp, st.copy);  // context switch: LOAD/EVICT, wait for this task's candidates
   if (t.kind == 0) issue_forward(st, t.y, slot);
   else issue_backward(st, t.y, slot);

@@ -21,6 +21,7 @@ int nccl_unique_id(void* out128);
 struct StageRt {
   int K = 0, dev = 0;
   bool local = false;
+  int64_t bulk = 0;  // BSP: bulk of the last task issued on this stage
   cudaStream_t comp = nullptr, copy = nullptr;
   std::unique_ptr<DevArena> arena;
   std::unique_ptr<Family> fam;

@@ -93,6 +93,7 @@ class MlpFamily : public Family {
     g_[0] = A.alloc<float>(act);
     g_[1] = A.alloc<float>(act);
     spec_base_ = &spec;
+    n_choices_ = spec.n();
     mse_part_ = A.alloc<float>(mse_blocks(spec.batch_elems()));
   }
   void bind(int j, int c, float* w32, bf16*) override { params_[(size_t)j * spec_.n() + c] = w32; }
@@ -117,8 +118,9 @@ class MlpFamily : public Family {
     const float* g = static_cast<const float*>(dy);
     for (int j = nb - 1; j >= 0; --j) {
       float* P = master(j, ch[blocks_[j]]);
+      float* U = upd(j, ch[blocks_[j]]);  // SGD WRITE target (P in place; the BSP accumulator)
       float* out = (j == 0) ? static_cast<float*>(dx) : g_[j & 1];
-      mlp_bwd_sgd(s, xin_[(size_t)slot * nb + j], h_[(size_t)slot * nb + j], g, out, P, P + (size_t)d_ * d_, lr_,
+      mlp_bwd_sgd(s, xin_[(size_t)slot * nb + j], h_[(size_t)slot * nb + j], g, out, P, U, U + (size_t)d_ * d_, lr_,
                   B_, d_);
       counters.launches++;
       g = out;
@@ -208,6 +210,7 @@ class TfFamily : public Family {
     p_g1_ = A.alloc<float>((size_t)lnb_ * d_);
     p_b1_ = A.alloc<float>((size_t)lnb_ * d_);
     spec_base_ = &spec;
+    n_choices_ = spec.n();
     mse_part_ = A.alloc<float>(mse_blocks(spec.batch_elems()));
     cudaStreamCreateWithFlags(&side_, cudaStreamNonBlocking);
     for (auto* e : {&ev_dz_, &ev_da2_, &ev_do_, &ev_da_, &ev_done_[0], &ev_done_[1], &ev_join_})
@@ -338,10 +341,12 @@ class TfFamily : public Family {
     float* P = master(j, c);
     bf16* W = w16_[(size_t)j * spec_.n() + c];
     bf16 *Wqkv = W, *Wo = W + 3 * (size_t)d * d, *W1 = W + 4 * (size_t)d * d, *W2 = W1 + (size_t)f * d;
+    float* U = upd(j, c);  // SGD WRITE target (P in place; the BSP accumulator, no shadow refresh)
+    const bool inplace = in_place(j, c);
     auto sgd_ep = [&](float* w32, bf16* w16) {
       GemmEpiParams e;
       e.w32 = w32;
-      e.w16 = w16;
+      e.w16 = inplace ? w16 : nullptr;
       e.lr = lr_;
       return e;
     };
@@ -352,14 +357,14 @@ class TfFamily : public Family {
     gemm(s, T, f, d, dy16_[p], false, d, W2, true, f, EPI_DGELU, e);        // dz = (dy W2) * gelu'(z)
     cudaEventRecord(ev_dz_, s);
     cudaStreamWaitEvent(side_, ev_dz_, 0);
-    gemm(side_, d, f, T, dy16_[p], true, d, t.g, true, f, EPI_SGD, sgd_ep(P + o.W2, W2), true);  // W2 -= lr dy^T g
+    gemm(side_, d, f, T, dy16_[p], true, d, t.g, true, f, EPI_SGD, sgd_ep(U + o.W2, W2), true);  // W2 -= lr dy^T g
     colsum_bf16(side_, dz_[p], p_db1_[p], T, f);
     e = GemmEpiParams();
     e.out = da_;
     gemm(s, T, d, f, dz_[p], false, f, W1, true, d, EPI_F32, e);             // da2 = dz W1
     cudaEventRecord(ev_da2_, s);
     cudaStreamWaitEvent(side_, ev_da2_, 0);
-    gemm(side_, f, d, T, dz_[p], true, f, t.a2, true, d, EPI_SGD, sgd_ep(P + o.W1, W1), true);  // W1 -= lr dz^T a2
+    gemm(side_, f, d, T, dz_[p], true, f, t.a2, true, d, EPI_SGD, sgd_ep(U + o.W1, W1), true);  // W1 -= lr dz^T a2
     ln_bwd(s, da_, t.x1, t.mean2, t.rstd2, P + o.ln2g, dy, dx1_, dx1_16_[p], p_g2_[p], p_b2_[p], p_dbo_[p], T, d);
     // ---- attention half
     e = GemmEpiParams();
@@ -367,7 +372,7 @@ class TfFamily : public Family {
     gemm(s, T, d, d, dx1_16_[p], false, d, Wo, true, d, EPI_BF16, e);        // do = dx1 Wo
     cudaEventRecord(ev_do_, s);
     cudaStreamWaitEvent(side_, ev_do_, 0);
-    gemm(side_, d, d, T, dx1_16_[p], true, d, t.o, true, d, EPI_SGD, sgd_ep(P + o.Wo, Wo), true);  // Wo -= lr dx1^T o
+    gemm(side_, d, d, T, dx1_16_[p], true, d, t.o, true, d, EPI_SGD, sgd_ep(U + o.Wo, Wo), true);  // Wo -= lr dx1^T o
     attn_bwd(s, t.qkv, t.o, t.lse, do16_, dqkv_[p], B_, S_, d, h);
     e = GemmEpiParams();
     e.out = da_;
@@ -375,16 +380,16 @@ class TfFamily : public Family {
     cudaEventRecord(ev_da_, s);
     cudaStreamWaitEvent(side_, ev_da_, 0);
     colsum_bf16(side_, dqkv_[p], p_dbqkv_[p], T, 3 * d);
-    gemm(side_, 3 * d, d, T, dqkv_[p], true, 3 * d, t.a, true, d, EPI_SGD, sgd_ep(P + o.Wqkv, Wqkv), true);
+    gemm(side_, 3 * d, d, T, dqkv_[p], true, 3 * d, t.a, true, d, EPI_SGD, sgd_ep(U + o.Wqkv, Wqkv), true);
     // bias / LN2 updates (all their partials are complete)
     SgdJobs j1{};
     j1.lr = lr_;
-    j1.job[0] = {P + o.b2, p_db2_[p], db2_nblk, d};
-    j1.job[1] = {P + o.b1, p_db1_[p], csb_, f};
-    j1.job[2] = {P + o.bo, p_dbo_[p], lnb_, d};
-    j1.job[3] = {P + o.bqkv, p_dbqkv_[p], csb_, 3 * d};
-    j1.job[4] = {P + o.ln2g, p_g2_[p], lnb_, d};
-    j1.job[5] = {P + o.ln2b, p_b2_[p], lnb_, d};
+    j1.job[0] = {U + o.b2, p_db2_[p], db2_nblk, d};
+    j1.job[1] = {U + o.b1, p_db1_[p], csb_, f};
+    j1.job[2] = {U + o.bo, p_dbo_[p], lnb_, d};
+    j1.job[3] = {U + o.bqkv, p_dbqkv_[p], csb_, 3 * d};
+    j1.job[4] = {U + o.ln2g, p_g2_[p], lnb_, d};
+    j1.job[5] = {U + o.ln2b, p_b2_[p], lnb_, d};
     j1.count = 6;
     sgd_multi(side_, j1);
     cudaEventRecord(ev_done_[p], side_);
@@ -395,8 +400,8 @@ class TfFamily : public Family {
            want_next ? p_db2_[p ^ 1] : nullptr, T, d);
     SgdJobs j2{};
     j2.lr = lr_;
-    j2.job[0] = {P + o.ln1g, p_g1_, lnb_, d};
-    j2.job[1] = {P + o.ln1b, p_b1_, lnb_, d};
+    j2.job[0] = {U + o.ln1g, p_g1_, lnb_, d};
+    j2.job[1] = {U + o.ln1b, p_b1_, lnb_, d};
     j2.count = 2;
     sgd_multi(s, j2);
     counters.launches += 7;

@@ -69,11 +69,30 @@ class Family {
   virtual size_t shadow_elems(int local_block, int c) const = 0;
   virtual float* master(int local_block, int c) = 0;
   virtual void refresh_shadow(int local_block, int c, cudaStream_t s) = 0;  // bf16 <- fp32
+  // BSP (reading A30): inside a bulk every forward and input gradient reads the bulk-start
+  // weights (master + shadow) while the SGD WRITEs accumulate into a separate fp32 copy
+  // bound here (nullptr = update in place, every other policy); the engine copies it back
+  // into the master (and refreshes the shadow) at the bulk's flush.
+  void bind_update(int local_block, int c, float* acc) {
+    const size_t k = (size_t)local_block * n_choices_ + c;
+    if (upd_.size() <= k) upd_.resize(k + 1, nullptr);
+    upd_[k] = acc;
+  }
+  float* upd(int local_block, int c) {
+    const size_t k = (size_t)local_block * n_choices_ + c;
+    return (k < upd_.size() && upd_[k]) ? upd_[k] : master(local_block, c);
+  }
+  bool in_place(int local_block, int c) const {
+    const size_t k = (size_t)local_block * n_choices_ + c;
+    return k >= upd_.size() || upd_[k] == nullptr;
+  }
   FamilyCounters counters;
   KernelTimer* timer = nullptr;
 
  protected:
   const Spec* spec_base_ = nullptr;
+  int n_choices_ = 1;            // set by the families (bind_update's key)
+  std::vector<float*> upd_;      // BSP accumulators, [local_block * n + c]
   float* mse_part_ = nullptr;  // MSE workspace (last stage)
 };
 

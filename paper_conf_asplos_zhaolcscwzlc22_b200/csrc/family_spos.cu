@@ -31,6 +31,8 @@ class SposFamily : public Family {
  public:
   SposFamily(const Spec& spec, const std::vector<int>& blocks, int W, DevArena& A)
       : spec_(spec), blocks_(blocks), W_(W), B_(spec.B()), lr_(spec.raw.lr) {
+    spec_base_ = &spec;
+    n_choices_ = spec.n();
     const int nb = (int)blocks.size(), n = spec.n();
     first_ = blocks.front() == 0;
     last_ = blocks.back() == spec.m() - 1;
@@ -241,7 +243,7 @@ class SposFamily : public Family {
     ce_mean(s, loss_per_, B_, loss_dst);
     fc_dgap(s, dlogits_, wf_, B_, Ch, ncls, dgap_);
     head_bcast(s, dgap_, B_, HW, Ch, rh_);  // dr overwrites r (the mask is recomputed from z)
-    t_bn_bwd_reduce(s, rh_, Ch, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, 1, 0.f, 0);
+    t_bn_bwd_reduce(s, rh_, Ch, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, ones_, zeros_, 1, 0.f, 0);
     t_bn_bwd_apply(s, rh_, Ch, zh_, PL, Ch, hmean_, hrstd_, 1, dzh_);
     e = GemmEpiParams();
     e.out = dy;
@@ -291,9 +293,10 @@ class SposFamily : public Family {
     if (timer) timer->end(s, 8.0 * Pp * C);
   }
   void t_bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int Pp, int C, const float* mean,
-                       const float* rstd, float* g, float* b, int relu, float lr, int update) {
+                       const float* rstd, const float* g, const float* b, float* gu, float* bu, int relu, float lr,
+                       int update) {
     if (timer) timer->begin(s);
-    bn_bwd_reduce(s, dy, lddy, z, Pp, C, mean, rstd, g, b, relu, part_, ctr_, sums_, old_, lr, update);
+    bn_bwd_reduce(s, dy, lddy, z, Pp, C, mean, rstd, g, b, gu, bu, relu, part_, ctr_, sums_, old_, lr, update);
     if (timer) timer->end(s, 6.0 * Pp * C);
   }
   void t_bn_bwd_apply(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int Pp, int C, const float* mean,
@@ -372,11 +375,12 @@ class SposFamily : public Family {
 
   // One unit's BN backward (+ the WRITE of its gamma/beta), leaves dz in the next ring
   // buffer dz_[ring_] (whose previous reader, a weight-gradient on the side stream, is done).
-  void unit_bn_bwd(const SposConv& u, const UnitRec& r, float* Pm, const bf16* dy, int lddy, cudaStream_t s) {
+  void unit_bn_bwd(const SposConv& u, const UnitRec& r, float* Pm, float* Um, const bf16* dy, int lddy, cudaStream_t s) {
     const int Po = (int)P(u.H_out);
     ring_ = (ring_ + 1) % kRing;
     if (ring_used_[ring_]) cudaStreamWaitEvent(s, ev_wg_[ring_], 0);
-    t_bn_bwd_reduce(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, u.relu, lr_, 1);
+    t_bn_bwd_reduce(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, Um + u.off_g,
+                    Um + u.off_b, u.relu, lr_, 1);
     t_bn_bwd_apply(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, u.relu, dz_[ring_]);
     counters.launches += 3;
   }
@@ -385,8 +389,8 @@ class SposFamily : public Family {
   // pre-update weights on the stage stream (skipped if dst == nullptr); then, on the side
   // stream once that has been issued, the weight gradient with the SGD WRITE (reading A4),
   // overlapping the rest of the input-gradient chain.
-  void unit_conv_bwd(const SposConv& u, const UnitRec& r, float* Pm, bf16* W16, size_t half, bf16* dst,
-                     const bf16* add, cudaStream_t s) {
+  void unit_conv_bwd(const SposConv& u, const UnitRec& r, float* Pm, float* Um, bool inplace, bf16* W16, size_t half,
+                     bf16* dst, const bf16* add, cudaStream_t s) {
     const int Po = (int)P(u.H_out);
     const bf16* dz = dz_[ring_];
     if (dst) {
@@ -404,14 +408,14 @@ class SposFamily : public Family {
     cudaStreamWaitEvent(side_, ev_dg_[ring_], 0);
     if (u.dw) {
       dw_wgrad(side_, dz, r.x, dwpart_, B_, u.H_in, u.cin, u.k, u.stride);
-      sgd_from_partials(side_, Pm + u.off_w, dwpart_, dw_wgrad_blocks(B_, u.H_in, u.cout, u.k, u.stride),
+      sgd_from_partials(side_, Um + u.off_w, dwpart_, dw_wgrad_blocks(B_, u.H_in, u.cout, u.k, u.stride),
                         u.cout * u.k * u.k, lr_);
       counters.launches += 2;
     } else {
       GemmEpiParams e;
-      e.w32 = Pm + u.off_w;
-      e.w16 = W16 + u.off_w16;
-      e.w16lo = W16 + half + u.off_w16;
+      e.w32 = Um + u.off_w;  // the BSP accumulator has no shadow (refreshed at the flush)
+      e.w16 = inplace ? W16 + u.off_w16 : nullptr;
+      e.w16lo = inplace ? W16 + half + u.off_w16 : nullptr;
       e.lr = lr_;
       gemm(side_, u.cout, u.cin, Po, dz, true, u.cout, r.x, true, u.cin, EPI_SGD, e, true);
     }
@@ -423,6 +427,8 @@ class SposFamily : public Family {
     const SposDims& d = dims_[j];
     const auto& L = plans_[(size_t)j * spec_.n() + c];
     float* Pm = master(j, c);
+    float* Um = upd(j, c);
+    const bool inplace = in_place(j, c);
     bf16* W16 = w16_[(size_t)j * spec_.n() + c];
     const size_t half = shadow_elems(j, c) / 2;
     const auto& recs = recs_[k];
@@ -435,11 +441,11 @@ class SposFamily : public Family {
     int pp = 0;
     for (size_t i = L.size(); i-- > m0;) {
       const SposConv& u = L[i];
-      unit_bn_bwd(u, recs[i], Pm, h, ldh, s);
+      unit_bn_bwd(u, recs[i], Pm, Um, h, ldh, s);
       bf16* dst;
       if (i > m0) dst = g_[pp ^= 1];
       else dst = need_dx ? (d.stride == 1 ? g_[pp ^ 1] : gfirst_) : nullptr;
-      unit_conv_bwd(u, recs[i], Pm, W16, half, dst, nullptr, s);
+      unit_conv_bwd(u, recs[i], Pm, Um, inplace, W16, half, dst, nullptr, s);
       h = dst;
       ldh = u.cin;
     }
@@ -456,9 +462,9 @@ class SposFamily : public Family {
     int ldp = d.C_out;
     for (size_t i = m0; i-- > 0;) {
       const SposConv& u = L[i];
-      unit_bn_bwd(u, recs[i], Pm, hp, ldp, s);
+      unit_bn_bwd(u, recs[i], Pm, Um, hp, ldp, s);
       bf16* dst = i > 0 ? g_[pp ^= 1] : (need_dx ? dxb : nullptr);
-      unit_conv_bwd(u, recs[i], Pm, W16, half, dst, (i == 0 && need_dx) ? gfirst_ : nullptr, s);
+      unit_conv_bwd(u, recs[i], Pm, Um, inplace, W16, half, dst, (i == 0 && need_dx) ? gfirst_ : nullptr, s);
       hp = dst;
       ldp = u.cin;
     }

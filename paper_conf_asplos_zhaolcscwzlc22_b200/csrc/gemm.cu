@@ -124,7 +124,7 @@ __device__ __forceinline__ void epilogue4(float4 v, float4 pre, float4 b, size_t
     float4 w = pre;
     w.x -= ep.lr * v.x; w.y -= ep.lr * v.y; w.z -= ep.lr * v.z; w.w -= ep.lr * v.w;
     *reinterpret_cast<float4*>(ep.w32 + off) = w;
-    *reinterpret_cast<uint2*>(ep.w16 + off) = pack4_bf16(w);
+    if (ep.w16) *reinterpret_cast<uint2*>(ep.w16 + off) = pack4_bf16(w);  // no shadow: BSP accumulator
     if (ep.w16lo)
       *reinterpret_cast<uint2*>(ep.w16lo + off) =
           pack4_bf16(make_float4(bf_lo(w.x), bf_lo(w.y), bf_lo(w.z), bf_lo(w.w)));
@@ -526,6 +526,7 @@ __global__ void splitk_reduce_kernel(int M, int N, int splits, int L, GemmEpiPar
       float4 w = reinterpret_cast<float4*>(ep.w32)[i];
       w.x -= ep.lr * acc.x; w.y -= ep.lr * acc.y; w.z -= ep.lr * acc.z; w.w -= ep.lr * acc.w;
       reinterpret_cast<float4*>(ep.w32)[i] = w;
+      if (!ep.w16) continue;  // no shadow: BSP accumulator
       uint2 o;
       o.x = ptx::pack_bf16(w.x, w.y);
       o.y = ptx::pack_bf16(w.z, w.w);

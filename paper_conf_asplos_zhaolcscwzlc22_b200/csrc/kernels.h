@@ -109,9 +109,10 @@ void synth_fill(cudaStream_t s, float* x, size_t n, uint64_t seed);
 // ------------------------------------------------------------------ MLP family (fp32)
 // y = x + tanh(x W^T + b), x [B, d]; saves h = tanh(.) for backward
 void mlp_fwd(cudaStream_t s, const float* x, const float* W, const float* b, float* y, float* h, int B, int d);
-// dz = dy (1 - h^2); dx = dy + dz W (pre-update W); then W -= lr dz^T x, b -= lr sum dz
-void mlp_bwd_sgd(cudaStream_t s, const float* x, const float* h, const float* dy, float* dx, float* W,
-                 float* b, float lr, int B, int d);
+// dz = dy (1 - h^2); dx = dy + dz W (the W this subnet read); then the WRITE
+// Wu -= lr dz^T x, bu -= lr sum dz (Wu, bu = W, b in place; the BSP accumulator, reading A30)
+void mlp_bwd_sgd(cudaStream_t s, const float* x, const float* h, const float* dy, float* dx, const float* W, float* Wu,
+                 float* bu, float lr, int B, int d);
 
 // ------------------------------------------------------------------ SPOS CNN (spos.cu)
 // NHWC activations [P = B*H*W rows, C channels]; C % 8 == 0 everywhere.  Forward tensors
@@ -131,10 +132,11 @@ void bn_stats(cudaStream_t s, const bf16* z, int P, int C, float* part, int* ctr
 void bn_apply(cudaStream_t s, const bf16* z, int P, int C, const float* mean, const float* rstd, const float* g,
               const float* b, int relu, bf16* y, int ldy, size_t yplane);
 // sums [2][C] = (sum dy', sum dy' xh) (dy' = dy masked by the ReLU); old [2][C] = (g, b)
-// before the update; update: the SGD WRITE g -= lr sums[1], b -= lr sums[0]
+// as read by the forward; update: the SGD WRITE gu -= lr sums[1], bu -= lr sums[0] (gu, bu
+// = g, b in place; the bulk accumulator under BSP, reading A30)
 void bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
-                   const float* rstd, float* g, float* b, int relu, float* part, int* ctr, float* sums, float* old,
-                   float lr, int update);
+                   const float* rstd, const float* g, const float* b, float* gu, float* bu, int relu, float* part,
+                   int* ctr, float* sums, float* old, float lr, int update);
 void bn_bwd_apply(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
                   const float* rstd, const float* old, const float* sums, int relu, bf16* dz);
 // depthwise k x k (k in {3,5,7}), stride S, pad k/2; w fp32 [C][k][k]; H = input height = width.

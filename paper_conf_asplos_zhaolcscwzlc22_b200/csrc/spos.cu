@@ -198,8 +198,8 @@ __global__ void bn_finalize_kernel(const float* __restrict__ part, int nblk, int
 // sums[0][c] = s1 (dbeta), sums[1][c] = s2 (dgamma); old = (gamma, beta) before the WRITE
 // gamma -= lr s2, beta -= lr s1 (if update)
 __global__ void bn_bwd_finalize_kernel(const float* __restrict__ part, int nblk, int C, float* __restrict__ sums,
-                                       float* __restrict__ old, float* __restrict__ gam, float* __restrict__ bet,
-                                       float lr, int update) {
+                                       float* __restrict__ old, const float* gam, const float* bet, float* gamu,
+                                       float* betu, float lr, int update) {
   __shared__ double tot[8];
   ptx::pdl_wait();
   const int w = threadIdx.x >> 5, c = blockIdx.x * 4 + w / 2;
@@ -215,9 +215,9 @@ __global__ void bn_bwd_finalize_kernel(const float* __restrict__ part, int nblk,
       const float gv = gam[cc], bv = bet[cc];
       old[cc] = gv;
       old[C + cc] = bv;
-      if (update) {
-        gam[cc] = gv - lr * f2;
-        bet[cc] = bv - lr * f1;
+      if (update) {  // the WRITE; gamu/betu = gam/bet in place, the bulk accumulator under BSP
+        gamu[cc] = (gamu == gam ? gv : gamu[cc]) - lr * f2;
+        betu[cc] = (betu == bet ? bv : betu[cc]) - lr * f1;
       }
     }
   }
@@ -920,8 +920,8 @@ void bn_apply(cudaStream_t s, const bf16* z, int P, int C, const float* mean, co
 }
 
 void bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
-                   const float* rstd, float* g, float* b, int relu, float* part, int* ctr, float* sums, float* old,
-                   float lr, int update) {
+                   const float* rstd, const float* g, const float* b, float* gu, float* bu, int relu, float* part,
+                   int* ctr, float* sums, float* old, float lr, int update) {
   (void)ctr;
   NP_REQUIRE(C % 8 == 0 && C / 8 <= TPB, NASPIPE_EINVAL, "bn_bwd C=%d", C);
   const size_t sm = red_smem(C);
@@ -930,7 +930,7 @@ void bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int 
   launch_pdl(bn_bwd_reduce_kernel, dim3(nblk), dim3(TPB), sm, s, dy, lddy, z, P, C, mean, rstd, (const float*)g,
              (const float*)b, relu, red_rows(P, C), part);
   launch_pdl(bn_bwd_finalize_kernel, dim3((C + 3) / 4), dim3(TPB), 0, s, (const float*)part, nblk, C, sums, old, g,
-             b, lr, update);
+             b, gu, bu, lr, update);
   check_launch("bn_bwd_reduce");
 }
 

@@ -211,8 +211,10 @@ def test_sync_policies_match_oracle_bit_exact(sync, seed):
     assert list(st) == ref["stall"] and list(bu) == ref["bubble"]
 
 
-def test_bsp_is_plan_only():
-    cfg = dict(synth.get_config("toy"), sync="bsp")
+def test_bsp_needs_resident_candidates():
+    """BSP executes with every candidate resident (its accumulators live beside the
+    masters); with a context-switch budget create fails with EINVAL before touching CUDA."""
+    cfg = dict(synth.get_config("toy"), sync="bsp", hbm_weight_budget_bytes=1 << 20)
     with pytest.raises(npipe.NaspipeError) as e:
         npipe.naspipe_create(npipe.Spec(cfg), 1)
     assert e.value.code == -1

@@ -7,6 +7,11 @@
   reproducibility contrast of Table 3, here on B200.
 * INORDER ("NASPipe w/o scheduler", Fig.6): a different, still causal schedule with
   bitwise the CSP numerics.
+* BSP (GPipe / Retiarii bulks; reading A30): the executed schedule is the
+  planner's BSP plan; the parameters equal oracle/train.py train_bsp (each bulk's gradients
+  at the bulk-start weights, summed, applied at the flush) within the CSP parity bars;
+  bulk = 1 is bitwise the CSP result; a fixed bulk size gives bitwise the same result at
+  D = 1, 2, 4 (the bulk, not the stage count, defines the arithmetic).
 """
 import numpy as np
 import pytest
@@ -72,3 +77,52 @@ def test_inorder_has_csp_numerics():
     p_csp, l_csp, _, _ = run_engine(cfg_c, choices, batches, 4)
     assert all(np.array_equal(p_in[k].view(np.uint32), p_csp[k].view(np.uint32)) for k in p_in)
     assert np.array_equal(l_in.view(np.uint32), l_csp.view(np.uint32))
+
+
+def _run_bsp(name, N, D, bulk, where=None):
+    cfg = synth.get_config(name, sync="bsp", bulk_size=bulk, window=4 * D)
+    choices = synth.sample_choices(N, cfg["n_blocks"], cfg["n_choices"])
+    batches = [synth.make_batch(cfg, y) for y in range(N)]
+    kw = {} if where is None else dict(where=where)
+    return cfg, choices, batches, run_engine(cfg, choices, batches, D, **kw)
+
+
+@pytest.mark.parametrize("name,N,D,bulk,tol_upd,rtol", [("toy", 24, 2, 4, 1e-5, 1e-5), ("toy", 24, 4, 6, 1e-5, 1e-5),
+                                                        ("tiny_transformer", 8, 2, 4, 1e-1, 1e-2)])
+def test_bsp_matches_oracle(name, N, D, bulk, tol_upd, rtol):
+    cfg, choices, batches, (params, losses, trace, _) = _run_bsp(name, N, D, bulk)
+    sob = npipe.naspipe_partition(npipe.Spec(cfg), D)
+    cf, cb = npipe.naspipe_default_costs(npipe.Spec(cfg))
+    tf, tb = csp.task_costs(choices, sob, cf, cb, D)
+    plan = csp.simulate_csp(choices, sob, D, 4 * D, tf, tb, sync="bsp", bulk=bulk)["trace"]
+    assert [tuple(int(v) for v in r) for r in trace] == [tuple(r) for r in plan]
+    theta0 = train.initial_theta(cfg)
+    ref, ref_loss = train.train_bsp(cfg, theta0, choices, batches, bulk)
+    err, derr = param_errors(cfg, params, ref, theta0)
+    assert err <= 1e-3 and derr <= tol_upd, (err, derr)
+    np.testing.assert_allclose(losses, ref_loss, rtol=rtol)
+
+
+@pytest.mark.parametrize("name,N", [("toy", 12), ("tiny_transformer", 6), ("tiny_spos", 6)])
+def test_bsp_bulk1_is_bitwise_csp(name, N):
+    """bulk = 1: the accumulator path (WRITE into the copy, flush before the next subnet)
+    computes exactly the in-place update: bitwise the CSP parameters and losses."""
+    cfg, choices, batches, (p_bsp, l_bsp, _, _) = _run_bsp(name, N, 2, 1)
+    ccfg = synth.get_config(name)
+    p_csp, l_csp, _, _ = run_engine(ccfg, choices, batches, 2)
+    assert np.array_equal(l_bsp.view(np.uint32), l_csp.view(np.uint32))
+    for k in p_csp:
+        assert np.array_equal(p_bsp[k].view(np.uint32), p_csp[k].view(np.uint32)), k
+
+
+@pytest.mark.parametrize("name,N", [("toy", 24), ("tiny_spos", 8)])
+def test_bsp_fixed_bulk_is_bitwise_across_stage_counts(name, N):
+    base = None
+    for D in (1, 2, 4):
+        _, _, _, (p, l, _, _) = _run_bsp(name, N, D, 4)
+        if base is None:
+            base = (p, l)
+            continue
+        assert np.array_equal(l.view(np.uint32), base[1].view(np.uint32)), D
+        for k in p:
+            assert np.array_equal(p[k].view(np.uint32), base[0][k].view(np.uint32)), (D, k)
