@@ -9,6 +9,7 @@
 #include <cstring>
 
 #include "engine.h"
+#include "launch.h"
 
 namespace naspipe {
 
@@ -89,6 +90,10 @@ Engine::Engine(const Spec& spec, int D) : spec_(spec), D_(D), W_(spec.window(D))
              "BSP runs with every candidate resident (hbm_weight_budget_bytes = 0)");
   version_.assign((size_t)spec_.m() * spec_.n(), 0);
   timer_.on = (spec_.raw.flags & NASPIPE_FLAG_TIMING) != 0;
+  if (spec_.raw.hbm_weight_budget_bytes > 0) {  // context switching: no PDL (launch.h)
+    pdl_suppressors().fetch_add(1);
+    suppress_pdl_ = true;
+  }
 }
 
 std::unique_ptr<Engine> Engine::create_local(const Spec& spec, int D) {
@@ -219,7 +224,10 @@ void Engine::link_local_buffers() {
   }
 }
 
-Engine::~Engine() { shutdown(); }
+Engine::~Engine() {
+  shutdown();
+  if (suppress_pdl_) pdl_suppressors().fetch_sub(1);
+}
 
 void Engine::shutdown() {
   for (auto& st : st_) {

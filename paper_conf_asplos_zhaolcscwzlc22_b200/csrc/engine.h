@@ -60,6 +60,7 @@ class Engine {
   void set_sticky(int code, const std::string& msg);
 
  private:
+  bool suppress_pdl_ = false;  // this engine context-switches: PDL off while it lives
   Engine(const Spec& spec, int D);
   void stage_sizes();
   void setup_stage(int K, int dev, bool local);

@@ -16,6 +16,7 @@ import paper_conf_asplos_zhaolcscwzlc22_b200 as npipe  # noqa: E402
 ap = argparse.ArgumentParser()
 ap.add_argument("--budget-x", type=float, default=3.0)
 ap.add_argument("--subnets", type=int, default=6)
+ap.add_argument("--no-drain", action="store_true", help="submit all subnets, drain once at the end")
 a = ap.parse_args()
 cfg = synth.get_config("large_transformer")
 t0 = time.time()
@@ -28,8 +29,15 @@ xd, td = torch.from_numpy(x).cuda(), torch.from_numpy(t).cuda()
 for y in range(a.subnets):
     t1 = time.time()
     npipe.naspipe_submit(h, choices[y], xd, td, where=npipe.BATCH_DEVICE)
+    if a.no_drain:
+        print(f"submitted {y} in {1e3 * (time.time() - t1):.1f} ms", flush=True)
+        continue
     npipe.naspipe_drain(h)
     s = npipe.naspipe_get_stats(h)
     print(f"subnet {y}: {1e3 * (time.time() - t1):.1f} ms  loads {s['res_loads']:.0f} evicts {s['res_evicts']:.0f} "
           f"h2d {s['h2d_bytes'] / 1e9:.1f} GB d2h {s['d2h_bytes'] / 1e9:.1f} GB", flush=True)
+if a.no_drain:
+    t1 = time.time()
+    npipe.naspipe_drain(h)
+    print(f"drain {1e3 * (time.time() - t1):.1f} ms", flush=True)
 npipe.naspipe_destroy(h)
