@@ -83,6 +83,12 @@ typedef enum { NASPIPE_FP32 = 0, NASPIPE_BF16 = 1 } naspipe_dtype; /* compute dt
 #define NASPIPE_FLAG_VERSION_CHECK 2 /* assert candidate versions at every task start        */
 #define NASPIPE_FLAG_NULL_KERNELS 4  /* run planner/transport only; kernels become no-ops     */
 #define NASPIPE_FLAG_TIMING 8        /* CUDA-event timing of the dominant kernel (GEMM)      */
+/* Activation recomputation ("NASPIPE adopts activation recomputing techniques";
+ * reading A13): the forward keeps only each block's input; the backward recomputes the
+ * block's forward before its gradient.  The kernels are deterministic and CSP/BSP never
+ * update a candidate between F(y) and B(y), so results are bitwise those without it.
+ * TRANSFORMER family only, not with ASP (EINVAL otherwise). */
+#define NASPIPE_FLAG_RECOMPUTE 16
 
 /*
  * Supernet specification.  naspipe_create deep-copies it and every array it points to.

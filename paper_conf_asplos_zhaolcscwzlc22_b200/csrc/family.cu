@@ -157,24 +157,35 @@ class TfFamily : public Family {
     w32_.assign((size_t)nb * n, nullptr);
     w16_.assign((size_t)nb * n, nullptr);
     const size_t Td = (size_t)T_ * d_;
+    recompute_ = (spec.raw.flags & NASPIPE_FLAG_RECOMPUTE) != 0;
+    auto alloc_acts = [&](TfSlot& t) {
+      t.a = A.alloc<bf16>(Td);
+      t.qkv = A.alloc<bf16>(3 * Td);
+      t.o = A.alloc<bf16>(Td);
+      t.a2 = A.alloc<bf16>(Td);
+      t.z = A.alloc<bf16>((size_t)T_ * fmax_);
+      t.g = A.alloc<bf16>((size_t)T_ * fmax_);
+      t.mean1 = A.alloc<float>(T_);
+      t.rstd1 = A.alloc<float>(T_);
+      t.mean2 = A.alloc<float>(T_);
+      t.rstd2 = A.alloc<float>(T_);
+      t.lse = A.alloc<float>((size_t)B_ * hmax_ * S_);
+      t.x1 = A.alloc<float>(Td);
+    };
+    // activation stash per (slot, block); with recomputation (reading A13) only the
+    // block inputs are kept and two scratch sets (by block parity) hold a block's activations
+    // while it is recomputed and back-propagated
     slots_.resize((size_t)W * nb);
     for (int sl = 0; sl < W; ++sl)
       for (int j = 0; j < nb; ++j) {
         TfSlot& t = slots_[(size_t)sl * nb + j];
         t.act = (j > 0) ? A.alloc<float>(Td) : nullptr;
-        t.a = A.alloc<bf16>(Td);
-        t.qkv = A.alloc<bf16>(3 * Td);
-        t.o = A.alloc<bf16>(Td);
-        t.a2 = A.alloc<bf16>(Td);
-        t.z = A.alloc<bf16>((size_t)T_ * fmax_);
-        t.g = A.alloc<bf16>((size_t)T_ * fmax_);
-        t.mean1 = A.alloc<float>(T_);
-        t.rstd1 = A.alloc<float>(T_);
-        t.mean2 = A.alloc<float>(T_);
-        t.rstd2 = A.alloc<float>(T_);
-        t.lse = A.alloc<float>((size_t)B_ * hmax_ * S_);
-        t.x1 = A.alloc<float>(Td);
+        if (!recompute_) alloc_acts(t);
       }
+    if (recompute_) {
+      for (auto& t : rs_) alloc_acts(t);
+      ry_ = A.alloc<float>(Td);
+    }
     // backward workspace (tasks on a stage are serialised on its stream).  Buffers the side
     // stream reads are double buffered by block parity (see backward()).
     for (int p = 0; p < 2; ++p) {
@@ -249,7 +260,13 @@ class TfFamily : public Family {
       TfSlot& t = slots_[(size_t)slot * nb + j];
       t.xin = x;
       float* y = (j == nb - 1) ? static_cast<float*>(x_out) : slots_[(size_t)slot * nb + j + 1].act;
-      block_fwd(j, c, t, y, s);
+      if (recompute_) {  // activations into the scratch set; only the block input is kept
+        TfSlot tt = rs_[j & 1];
+        tt.xin = x;
+        block_fwd(j, c, tt, y, s);
+      } else {
+        block_fwd(j, c, t, y, s);
+      }
       x = y;
     }
   }
@@ -278,7 +295,19 @@ class TfFamily : public Family {
       // stage 0 needs no input gradient, but LN1's backward still runs (dgamma/dbeta):
       // its dx goes to a scratch buffer (gb_[0] is free: block 1 wrote gb_[1])
       float* out = (j == 0) ? (dx ? dx : gb_[0]) : gb_[j & 1];
-      block_bwd(j, c, t, g, out, /*want_next=*/j > 0, db2_nblk, p, s);
+      if (recompute_) {
+        // recompute block j's forward from its kept input into scratch set p (bitwise the
+        // forward's activations: same kernels, same input, same weights — CSP/BSP do not
+        // update a candidate between F(y) and B(y)); the side stream's last reads of set p
+        // (block j+2's weight gradients) end with ev_done_[p]
+        TfSlot tt = rs_[p];
+        tt.xin = t.xin;
+        cudaStreamWaitEvent(s, ev_done_[p], 0);
+        block_fwd(j, c, tt, ry_, s);
+        block_bwd(j, c, tt, g, out, /*want_next=*/j > 0, db2_nblk, p, s);
+      } else {
+        block_bwd(j, c, t, g, out, /*want_next=*/j > 0, db2_nblk, p, s);
+      }
       db2_nblk = lnb_;
       g = out;
     }
@@ -414,6 +443,9 @@ class TfFamily : public Family {
   std::vector<float*> w32_;
   std::vector<bf16*> w16_;
   std::vector<TfSlot> slots_;
+  bool recompute_ = false;
+  TfSlot rs_[2];          // recomputation scratch activations, by block parity
+  float* ry_ = nullptr;   // recomputed block output (discarded)
   bf16 *dy16_[2], *dz_[2], *dx1_16_[2], *dqkv_[2], *do16_;
   float *da_, *dx1_, *gb_[2], *ws_ = nullptr;
   size_t ws_elems_ = 0;

@@ -42,6 +42,9 @@ Spec::Spec(const naspipe_supernet_spec* s) {
              NASPIPE_EINVAL, "bad window/lookahead/policy/latency/budget");
   NP_REQUIRE(raw.sync_policy >= NASPIPE_SYNC_CSP && raw.sync_policy <= NASPIPE_SYNC_BSP && raw.bulk_size >= 0,
              NASPIPE_EINVAL, "bad sync_policy %d / bulk_size %d", raw.sync_policy, raw.bulk_size);
+  NP_REQUIRE(!(raw.flags & NASPIPE_FLAG_RECOMPUTE) ||
+                 (raw.family == NASPIPE_TRANSFORMER && raw.sync_policy != NASPIPE_SYNC_ASP),
+             NASPIPE_EINVAL, "activation recomputation: transformer family, not under ASP (reading A13)");
   const int n = raw.n_choices, m = raw.n_blocks;
   if (raw.family == NASPIPE_MLP) {
     NP_REQUIRE(raw.width >= 1 && raw.width <= 1024, NASPIPE_EINVAL, "width %d", raw.width);

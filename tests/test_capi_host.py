@@ -257,3 +257,13 @@ def test_mirrored_plan_rejects_other_policies():
         npipe.naspipe_plan_mirrored(npipe.Spec(cfg), 2, ch, -1)
     with pytest.raises(npipe.NaspipeError):
         npipe.naspipe_plan_mirrored(npipe.Spec(cfg), 2, np.full_like(ch, cfg["n_choices"]))
+
+
+def test_recompute_flag_validation():
+    """NASPIPE_FLAG_RECOMPUTE: transformer family only, never with ASP (EINVAL)."""
+    ok = synth.get_config("tiny_transformer")
+    npipe.naspipe_partition(npipe.Spec(ok, flags=npipe.FLAG_RECOMPUTE), 2)
+    for cfg in (synth.get_config("toy"), synth.get_config("tiny_spos"), synth.get_config("tiny_transformer", sync="asp")):
+        with pytest.raises(npipe.NaspipeError) as e:
+            npipe.naspipe_partition(npipe.Spec(cfg, flags=npipe.FLAG_RECOMPUTE), 2)
+        assert e.value.code == -1
