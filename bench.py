@@ -44,6 +44,8 @@ def parse():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-secondary", action="store_true", help="skip the configs[2] line embedded in the output")
     ap.add_argument("--no-repro", action="store_true", help="skip the bit-reproducibility digests")
+    ap.add_argument("--recompute", action="store_true",
+                    help="activation recomputation (transformer family; P:L282, reading A13)")
     ap.add_argument("--budget-x", type=float, default=0.0,
                     help="HBM weight budget per stage as a multiple of one subnet's mean stage slice "
                          "(0 = all candidates resident; P:L337 uses ~3)")
@@ -254,6 +256,7 @@ def workload_config(args, cfg, world):
          else f"configs[4] sweep n={args.n_choices}",
          "n_blocks": cfg["n_blocks"], "n_choices": cfg["n_choices"], "batch": cfg["batch"],
          "stages": world, "parallelism": f"pp{world}" if world > 1 else "single stage",
+         "activation_recompute": bool(getattr(args, "recompute", False)),
          "l2": "working set > L2 (active weights + activations per step >> 126 MB)"}
     if cfg["family"] == "transformer":
         c.update(seq_len=cfg["seq_len"], d_model=cfg["d_model"], heads=cfg["choice_heads"], ffn=cfg["choice_ffn"])
@@ -296,7 +299,8 @@ def main():
     dev_pool = [(torch.from_numpy(x).cuda(), torch.from_numpy(t).cuda()) for x, t in pool]
     host_pool = [(torch.from_numpy(x).pin_memory(), torch.from_numpy(t).pin_memory()) for x, t in pool]
     budget = stage_budget(cfg, D, args.budget_x, npipe) if args.budget_x > 0 else 0
-    spec = npipe.Spec(cfg, hbm_weight_budget_bytes=budget, lookahead=args.lookahead)
+    spec = npipe.Spec(cfg, hbm_weight_budget_bytes=budget, lookahead=args.lookahead,
+                      flags=npipe.FLAG_RECOMPUTE if args.recompute else 0)
     if world == 1:
         h = npipe.naspipe_create(spec, 1)
     else:
