@@ -202,8 +202,13 @@ def _traffic(family):
         return None
     with open(p) as f:
         d = json.load(f).get(family)
-    return None if d is None else {"dram_bytes_per_launch": d["dram_bytes_per_launch_mean"],
-                                   "source": "profiles/dominant_traffic.json (ncu --set full capture)"}
+    if d is None:
+        return None
+    out = {"dram_bytes_per_launch": d["dram_bytes_per_launch_mean"],
+           "source": "profiles/dominant_traffic.json (ncu --set full capture)"}
+    if "tensor_pipe_pct_mean" in d:   # sm__pipe_tensor_cycles_active, time-weighted over the captured GEMMs
+        out["tensor_pipe_pct"] = d["tensor_pipe_pct_mean"]
+    return out
 
 
 def secondary(args):
