@@ -683,9 +683,30 @@ bool pair_enabled() {
   return v == 1;
 }
 
+// N tile of the 1-CTA kernel: narrow outputs (the SPOS 1x1-conv input gradients and weight
+// gradients, N = C_in <= 320) get 64- or 128-wide tiles instead of wasting 3/4 or 1/2 of a
+// 256-wide tile's MMA and TMEM work on zero columns (epilogues without per-column operands).
+bool small_n_epi(int epi) { return epi == EPI_BF16 || epi == EPI_F32 || epi == EPI_SGD || epi == EPI_PARTIAL; }
+int tile_n(int N, int epi) { return !small_n_epi(epi) ? BN : (N <= 64 ? 64 : (N <= 128 ? 128 : BN)); }
+
+template <bool A_MN, bool B_MN, int TN>
+void dispatch_narrow(cudaStream_t s, int M, int N, const TileSpace& ts, const CUtensorMap& ta, const CUtensorMap& tb,
+                     int epi, const GemmEpiParams& ep) {
+  switch (epi) {
+    case EPI_BF16: return launch<A_MN, B_MN, EPI_BF16, TN>(s, M, N, ts, ta, tb, ep);
+    case EPI_F32: return launch<A_MN, B_MN, EPI_F32, TN>(s, M, N, ts, ta, tb, ep);
+    case EPI_SGD: return launch<A_MN, B_MN, EPI_SGD, TN>(s, M, N, ts, ta, tb, ep);
+    case EPI_PARTIAL: return launch<A_MN, B_MN, EPI_PARTIAL, TN>(s, M, N, ts, ta, tb, ep);
+    default: NP_REQUIRE(false, NASPIPE_EINVAL, "narrow-tile epilogue %d", epi);
+  }
+}
+
 template <bool A_MN, bool B_MN>
 void dispatch_epi(cudaStream_t s, int M, int N, const TileSpace& ts, const CUtensorMap& ta, const CUtensorMap& tb,
                   int epi, const GemmEpiParams& ep) {
+  const int tn = tile_n(N, epi);
+  if (tn == 64) return dispatch_narrow<A_MN, B_MN, 64>(s, M, N, ts, ta, tb, epi, ep);
+  if (tn == 128) return dispatch_narrow<A_MN, B_MN, 128>(s, M, N, ts, ta, tb, epi, ep);
   switch (epi) {
     case EPI_BF16: return launch<A_MN, B_MN, EPI_BF16>(s, M, N, ts, ta, tb, ep);
     case EPI_F32: return launch<A_MN, B_MN, EPI_F32>(s, M, N, ts, ta, tb, ep);
@@ -710,7 +731,8 @@ bool gemm_uses_pair(int M, int N) { return pair_enabled() && M >= 256 && N >= 25
 int gemm_splitk_factor(int M, int N, int K) {
   const bool pair = gemm_uses_pair(M, N);
   const int bm = pair ? 2 * BM : BM;
-  const int tiles = ((M + bm - 1) / bm) * ((N + BN - 1) / BN);
+  const int bn = pair ? BN : tile_n(N, EPI_PARTIAL);  // split-K runs the partial epilogue
+  const int tiles = ((M + bm - 1) / bm) * ((N + bn - 1) / bn);
   const int nk = (K + BK - 1) / BK;
   const int sms = pair ? num_sms() / 2 : num_sms();
   // cost in k-block rounds (~0.3 us each): rounds * k-blocks per round, plus the fp32
@@ -731,21 +753,23 @@ void gemm_bf16_tc(cudaStream_t s, int M, int N, int K, const bf16* A, bool a_mn,
   NP_REQUIRE(M > 0 && N > 0 && K > 0 && N % 16 == 0, NASPIPE_EINVAL, "gemm dims M=%d N=%d K=%d (N%%16)", M, N, K);
   GemmEpiParams ep = ep_in;
   const bool pair = gemm_uses_pair(M, N);
+  int splits = 1;
+  if ((epi == EPI_SGD || epi == EPI_F32) && ep.ws != nullptr) {
+    splits = gemm_splitk_factor(M, N, K);
+    if ((size_t)splits * M * N > ep.ws_elems || (M * (size_t)N) % 4 != 0) splits = 1;
+    static const bool no_split = getenv("NASPIPE_NO_SPLITK") != nullptr;  // diagnostics
+    if (no_split) splits = 1;
+  }
+  const int tn = pair ? BN : tile_n(N, splits > 1 ? EPI_PARTIAL : epi);
   const CUtensorMap ta = a_mn ? make_map(A, (uint64_t)M, (uint64_t)K, (uint64_t)lda, BK)
                               : make_map(A, (uint64_t)K, (uint64_t)M, (uint64_t)lda, BM);
   const CUtensorMap tb = b_mn ? make_map(B, (uint64_t)N, (uint64_t)K, (uint64_t)ldb, BK)
-                              : make_map(B, (uint64_t)K, (uint64_t)N, (uint64_t)ldb, pair ? BN / 2 : BN);
+                              : make_map(B, (uint64_t)K, (uint64_t)N, (uint64_t)ldb, pair ? BN / 2 : tn);
   TileSpace ts;
   ts.MT = (M + (pair ? 2 * BM : BM) - 1) / (pair ? 2 * BM : BM);
-  ts.NT = (N + BN - 1) / BN;
+  ts.NT = (N + tn - 1) / tn;
   ts.nk = (K + BK - 1) / BK;
-  ts.splits = 1;
-  if ((epi == EPI_SGD || epi == EPI_F32) && ep.ws != nullptr) {
-    ts.splits = gemm_splitk_factor(M, N, K);
-    if ((size_t)ts.splits * M * N > ep.ws_elems || (M * (size_t)N) % 4 != 0) ts.splits = 1;
-    static const bool no_split = getenv("NASPIPE_NO_SPLITK") != nullptr;  // diagnostics
-    if (no_split) ts.splits = 1;
-  }
+  ts.splits = splits;
   ts.nk_per_split = (ts.nk + ts.splits - 1) / ts.splits;
   // effective split count: every split owns >= 1 k-block (with ceil-sized splits the last
   // ones could otherwise be empty and leave their workspace slice unwritten)

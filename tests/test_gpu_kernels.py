@@ -57,7 +57,8 @@ def _gemm(M, N, K, A, a_mn, B, b_mn, epi, **kw):
 
 
 SHAPES = [(128, 128, 64), (256, 384, 512), (304, 208, 200), (304, 272, 192), (4096, 1024, 1024),
-          (256, 512, 4096)]  # M, N >= 256: CTA-pair kernel (ragged: 304 x 272); last: split-K
+          (256, 512, 4096),   # M, N >= 256: CTA-pair kernel (ragged: 304 x 272); split-K
+          (1000, 32, 640), (520, 80, 96), (4096, 160, 200), (96, 64, 20000)]  # 64 / 128-wide N tiles; split-K
 
 
 @pytest.mark.parametrize("M,N,K", SHAPES)
