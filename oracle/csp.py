@@ -112,7 +112,7 @@ def task_costs(choices, stage_of_block, cost_f, cost_b, D):
 
 
 def simulate_csp(choices, stage_of_block, D, W, cf, cb, lam=0, policy=0, ignore_deps=False,
-                 admit=None, sync="csp", bulk=0):
+                 admit=None, sync="csp", bulk=0, observe=None):
     """O2.  Returns dict(trace=[(t, K, kind, y)], makespan, order=[[(kind, y)] per stage],
     stall=[ticks per stage], bubble=[ticks per stage]).  An idle stage is *stalled* while a
     queued forward is blocked by a dependency and in a *bubble* while nothing is queued
@@ -130,7 +130,10 @@ def simulate_csp(choices, stage_of_block, D, W, cf, cb, lam=0, policy=0, ignore_
     P:L123) dependencies ignored; "bsp" (GPipe/Retiarii): dependencies ignored inside
     bulks of ``bulk`` consecutive subnets (0 = 4 D), a stage runs any queued forward before
     a backward, and stage 0 admits bulk k only once every subnet of bulk k-1 finished on
-    stage 0 (the flush: a subnet's stage-0 backward is its last task)."""
+    stage 0 (the flush: a subnet's stage-0 backward is its last task).
+
+    ``observe(t, K, kind, y, queued, finished)``, if given, sees every task start with the
+    stage's queued forwards and finished set just before it (an observer: no effect)."""
     N = len(choices)
     G = bulk if bulk > 0 else 4 * D
     no_deps = ignore_deps or sync in ("asp", "bsp")
@@ -203,6 +206,8 @@ def simulate_csp(choices, stage_of_block, D, W, cf, cb, lam=0, policy=0, ignore_
             if choose is None:
                 continue
             kind, y = choose
+            if observe is not None:
+                observe(t, K, kind, y, sorted(inF[K]), set(fin[K]))
             if kind == 0:
                 inF[K].discard(y)
                 if K == 0:
@@ -446,3 +451,37 @@ def check_trace_mirrored(trace, choices, sob, D, cost_b, lam_w=0):
             if tf < tb + max(1, cbx) + (lam_w if Kf != Kb else 0):
                 errs.append(f"candidate {l}: F({users[i]}) at {tf} before the WRITE of {users[i - 1]} landed")
     return errs
+
+
+
+
+# --------------------------------------------------------------------------------------
+# the Alg.3 context predictor, evaluated against the exact plan
+# --------------------------------------------------------------------------------------
+def alg3_backward_predictions(choices, stage_of_block, D, W, cf, cb, lam=0):
+    """Alg.3's backward branch (its lines 4-8): before B(x, K) runs, the stage
+    pre-adds x to a copy of its finished list L_f (reading A10: L' is a copy) and re-runs
+    SCHEDULE (Alg.2, literal_alg2) on its queue L_q to predict the forward it will run next,
+    whose context it prefetches.  Every B(x, K) start of the O2 plan is replayed with the
+    plan's own L_q / L_f at that tick; the prediction is compared with the forward the plan
+    actually starts next on K (None if a backward comes first or nothing follows).  The exact
+    plan lookahead the executor uses (readings A9, A26) is right by construction.
+
+    Returns [(t, K, x, predicted, actual)] in start order."""
+    m = len(choices[0])
+    L_SN = [[(b, int(choices[y][b])) for b in range(m)] for y in range(len(choices))]
+    starts = []
+
+    def observe(t, K, kind, y, queued, finished):
+        starts.append((t, K, kind, y, queued, finished))
+
+    simulate_csp(choices, stage_of_block, D, W, cf, cb, lam=lam, observe=observe)
+    out = []
+    for i, (t, K, kind, y, queued, finished) in enumerate(starts):
+        if kind != 1:
+            continue
+        _, pred = literal_alg2(queued, sorted(finished | {y}), L_SN, K, stage_of_block)
+        nxt = next(((k2, y2) for (_, K2, k2, y2, _, _) in starts[i + 1:] if K2 == K), None)
+        actual = nxt[1] if nxt is not None and nxt[0] == 0 else None
+        out.append((t, K, y, None if pred < 0 else pred, actual))
+    return out

@@ -326,3 +326,31 @@ def test_mirrored_checker_rejects_early_read():
     bad[5] = [17, 1, 0, 1]   # F(1, stage 1) one tick before the WRITE of (1,0) lands
     assert csp.check_trace_mirrored(bad, g["choices"], sob, g["D"], g["cost_b"])
     assert csp.check_trace_mirrored(g["lam_w_0"]["trace"], g["choices"], sob, g["D"], g["cost_b"], lam_w=3)
+
+
+# ---------------------------------------------------------------------- §8f(3) Alg.3
+def test_alg3_predictions_on_the_worked_example():
+    """Alg.3's backward branch replayed on SURVEY §8c's worked example, derived
+    by hand from its stage orders: before B(x,K) the stage pre-finishes x and runs Alg.2 on
+    its queue.  Stage 0: B0@4 sees queue {2,3} -> predicts F2 (next: F2@6), B1@7 -> F3 (F3@9).
+    Stage 1: B0@2 sees {1} (F1 delivered at tick 2) -> F1 (F1@4); B1@5 and B2@8 see an empty
+    queue (F2 / F3 not yet delivered) -> no prediction, although F2@7 / F3@10 follow."""
+    with open(os.path.join(GOLD, "csp_worked_example.json")) as f:
+        g = json.load(f)
+    N, D = len(g["choices"]), g["D"]
+    cf = [[g["cf"]] * N for _ in range(D)]
+    cb = [[g["cb"]] * N for _ in range(D)]
+    got = csp.alg3_backward_predictions(g["choices"], g["stage_of_block"], D, g["W"], cf, cb)
+    assert got == [(2, 1, 0, 1, 1), (4, 0, 0, 2, 2), (5, 1, 1, None, 2), (7, 0, 1, 3, 3), (8, 1, 2, None, 3),
+                   (10, 0, 2, None, None), (11, 1, 3, None, None), (13, 0, 3, None, None)]
+
+
+def test_alg3_predictions_are_never_wrong_when_made_at_d1():
+    """D = 1: after B(x) the stage runs the lowest admissible queued forward, which is
+    exactly Alg.2 on L_f + {x}: every prediction made equals the next forward."""
+    rng = np.random.default_rng(3)
+    ch = rng.integers(0, 3, (20, 5)).tolist()
+    cf, cb = np.ones((1, 20), dtype=np.int64), 2 * np.ones((1, 20), dtype=np.int64)
+    preds = csp.alg3_backward_predictions(ch, [0] * 5, 1, 4, cf, cb)
+    assert len(preds) == 20
+    assert all(p == a for (_, _, _, p, a) in preds if p is not None)
