@@ -44,6 +44,8 @@ def parse():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-secondary", action="store_true", help="skip the configs[2] line embedded in the output")
     ap.add_argument("--no-repro", action="store_true", help="skip the bit-reproducibility digests")
+    ap.add_argument("--sync", default="csp", choices=["csp", "inorder", "asp", "bsp"],
+                    help="synchronisation policy (include/naspipe.h naspipe_sync; SURVEY §8f(1))")
     ap.add_argument("--recompute", action="store_true",
                     help="activation recomputation (transformer family; P:L282, reading A13)")
     ap.add_argument("--budget-x", type=float, default=0.0,
@@ -250,7 +252,7 @@ def bit_repro(cfg, npipe, dev_pool, n_sub=8, stage_counts=(1, 1, 2, 4)):
         sha.update(np.ascontiguousarray(npipe.naspipe_get_losses(h, n_sub), dtype=np.float32).tobytes())
         npipe.naspipe_destroy(h)
         digests.append({"stages": D, "sha256": sha.hexdigest()})
-    return {"subnets": n_sub, "candidates_hashed": len(used), "runs": digests,
+    return {"policy": "csp", "subnets": n_sub, "candidates_hashed": len(used), "runs": digests,
             "bitwise_equal": len({d["sha256"] for d in digests}) == 1}
 
 
@@ -262,6 +264,7 @@ def workload_config(args, cfg, world):
          "n_blocks": cfg["n_blocks"], "n_choices": cfg["n_choices"], "batch": cfg["batch"],
          "stages": world, "parallelism": f"pp{world}" if world > 1 else "single stage",
          "activation_recompute": bool(getattr(args, "recompute", False)),
+         "sync_policy": getattr(args, "sync", "csp"),
          "l2": "working set > L2 (active weights + activations per step >> 126 MB)"}
     if cfg["family"] == "transformer":
         c.update(seq_len=cfg["seq_len"], d_model=cfg["d_model"], heads=cfg["choice_heads"], ffn=cfg["choice_ffn"])
@@ -304,7 +307,7 @@ def main():
     dev_pool = [(torch.from_numpy(x).cuda(), torch.from_numpy(t).cuda()) for x, t in pool]
     host_pool = [(torch.from_numpy(x).pin_memory(), torch.from_numpy(t).pin_memory()) for x, t in pool]
     budget = stage_budget(cfg, D, args.budget_x, npipe) if args.budget_x > 0 else 0
-    spec = npipe.Spec(cfg, hbm_weight_budget_bytes=budget, lookahead=args.lookahead,
+    spec = npipe.Spec(cfg, hbm_weight_budget_bytes=budget, lookahead=args.lookahead, sync=args.sync,
                       flags=npipe.FLAG_RECOMPUTE if args.recompute else 0)
     if world == 1:
         h = npipe.naspipe_create(spec, 1)
