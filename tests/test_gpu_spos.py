@@ -122,3 +122,32 @@ def test_spos_full_size_bitwise_across_runs_and_stage_counts():
         for k in base:
             assert np.array_equal(p[k].view(np.uint32), base[k].view(np.uint32)), (D, k)
 
+
+
+def test_spos_full_size_20_steps_against_oracle_samples():
+    """configs[1] at full size, 20 subnets trained sequentially by the fp64 oracle
+    (tests/golden/spos_fullsize_20steps.npz, written by tools/make_spos_multistep_golden.py
+    from oracle/ only) against the GPU in the bench's launch configuration: A15 over 512
+    sampled entries of every trained candidate (denominator max |theta| over the whole
+    candidate) <= 1e-2 (BJ's multi-step bar), losses rtol 1e-2."""
+    import os
+    path = os.path.join(os.path.dirname(__file__), "golden", "spos_fullsize_20steps.npz")
+    if not os.path.exists(path):
+        pytest.skip("golden not generated")
+    g = np.load(path)
+    cfg = synth.get_config("spos")
+    choices = g["choices"]
+    N = len(choices)
+    batches = [synth.make_batch(cfg, y) for y in range(N)]
+    params, losses, _, _ = run_engine(cfg, choices, batches, D=1, where=npipe.BATCH_DEVICE)
+    worst = 0.0
+    for key in g.files:
+        if not key.startswith("idx_"):
+            continue
+        _, b, c = key.split("_")
+        got = params[(int(b), int(c))].astype(np.float64)[g[key]]
+        ref = g[f"new_{b}_{c}"]
+        worst = max(worst, float(np.max(np.abs(got - ref)) / g[f"maxabs_{b}_{c}"]))
+    print(f"20-step full-size sampled A15 = {worst:.3e}; losses {losses[-3:]} vs {g['losses'][-3:]}")
+    assert worst <= 1e-2, worst
+    np.testing.assert_allclose(losses, g["losses"], rtol=1e-2)
