@@ -891,10 +891,56 @@ void spos_stem_conv(cudaStream_t s, const float* x, const float* w, bf16* z, int
   check_launch("stem_conv");
 }
 
-// grid of the pixel-strided elementwise kernels: about 8 CTAs per SM
-static int ew_grid(int P, int C) {
+// grid of the pixel-strided elementwise kernels: a whole number of waves of the kernel's
+// resident CTAs (occ per SM, from the occupancy calculator), so the grid-stride loop gives
+// every SM the same work -- a fixed 8 CTAs/SM left a 2/3-full third wave for a 3-CTA/SM
+// kernel.  NASPIPE_EW_WAVES (default 1: measured best, 7.15 -> 7.01 ms per configs[1] step) overrides the wave count for tuning.
+static int ew_waves() {
+  static int v = 0;
+  if (!v) {
+    const char* e = getenv("NASPIPE_EW_WAVES");
+    v = e ? std::max(1, atoi(e)) : 1;
+  }
+  return v;
+}
+// NASPIPE_MAX_CTAS_PER_SM (tuning): cap the resident-CTA count used for the grid sizes below
+template <typename Kern>
+static int occupancy(Kern kern, size_t smem) {
+  int n = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, TPB, smem) != cudaSuccess || n < 1) n = 1;
+  static int cap = -1;
+  if (cap < 0) {
+    const char* e = getenv("NASPIPE_MAX_CTAS_PER_SM");
+    cap = e ? std::max(1, atoi(e)) : 0;
+  }
+  return cap ? std::min(n, cap) : n;
+}
+// grid-stride kernels over `items` threads of work: capped at NASPIPE_GS_WAVES (default 1:
+// measured best, 7.01 -> 6.95 ms per configs[1] step) waves of resident CTAs; 0 = grid_for's
+// fixed 16 CTAs/SM
+static int gs_waves() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("NASPIPE_GS_WAVES");
+    v = e ? std::max(0, atoi(e)) : 1;
+  }
+  return v;
+}
+template <typename Kern>
+static int gs_grid(Kern kern, size_t items, size_t smem = 0) {
+  if (!gs_waves()) return grid_for(items);
+  static int occ = 0;  // per kernel instantiation (and its last dynamic smem size)
+  static size_t occ_smem = 0;
+  if (!occ || smem != occ_smem) occ = occupancy(kern, smem), occ_smem = smem;
+  const size_t g = (items + TPB - 1) / TPB;
+  return (int)std::min<size_t>(std::max<size_t>(g, 1), (size_t)148 * occ * gs_waves());
+}
+template <typename Kern>
+static int ew_grid(Kern kern, int P, int C) {
+  static int occ = 0;  // per kernel (one static per instantiation)
+  if (!occ) occ = occupancy(kern, 0);
   const int lanes = TPB / (C / 8);
-  return std::max(1, std::min((P + lanes - 1) / lanes, 148 * 8));
+  return std::max(1, std::min((P + lanes - 1) / lanes, 148 * occ * ew_waves()));
 }
 
 static size_t red_smem(int C) { return (size_t)(TPB / (C / 8)) * 2 * C * sizeof(float); }
@@ -914,7 +960,7 @@ void bn_stats(cudaStream_t s, const bf16* z, int P, int C, float* part, int* ctr
 
 void bn_apply(cudaStream_t s, const bf16* z, int P, int C, const float* mean, const float* rstd, const float* g,
               const float* b, int relu, bf16* y, int ldy, size_t yplane) {
-  launch_pdl(bn_apply_kernel, dim3(ew_grid(P, C)), dim3(TPB), 0, s, z, P, C, mean, rstd, g, b, relu,
+  launch_pdl(bn_apply_kernel, dim3(ew_grid(bn_apply_kernel, P, C)), dim3(TPB), 0, s, z, P, C, mean, rstd, g, b, relu,
              y, ldy, yplane);
   check_launch("bn_apply");
 }
@@ -936,7 +982,7 @@ void bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int 
 
 void bn_bwd_apply(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
                   const float* rstd, const float* old, const float* sums, int relu, bf16* dz) {
-  launch_pdl(bn_bwd_apply_kernel, dim3(ew_grid(P, C)), dim3(TPB), 0, s, dy, lddy, z, P, C, mean, rstd,
+  launch_pdl(bn_bwd_apply_kernel, dim3(ew_grid(bn_bwd_apply_kernel, P, C)), dim3(TPB), 0, s, dy, lddy, z, P, C, mean, rstd,
              old, sums, relu, dz);
   check_launch("bn_bwd_apply");
 }
@@ -978,7 +1024,7 @@ void dw_dgrad(cudaStream_t s, const bf16* dz, const float* w, const bf16* add, b
     const size_t sm = (size_t)C * k * k * sizeof(float);
     DW_DISPATCH(k, {
       set_smem(dw_dgrad_kernel<KK>, sm);
-      launch_pdl(dw_dgrad_kernel<KK>, dim3(grid_for(items)), dim3(TPB), sm, s, dz, w, add, dx, B, H, C, S);
+      launch_pdl(dw_dgrad_kernel<KK>, dim3(gs_grid(dw_dgrad_kernel<KK>, items, sm)), dim3(TPB), sm, s, dz, w, add, dx, B, H, C, S);
     });
   }
   check_launch("dw_dgrad");
@@ -1028,13 +1074,13 @@ void dw_wgrad(cudaStream_t s, const bf16* dz, const bf16* x, float* part, int B,
 }
 
 void chan_split(cudaStream_t s, const bf16* x, int P, int Ch, bf16* out, int ldo, size_t oplane, bf16* xm) {
-  launch_pdl(chan_split_kernel, dim3(grid_for((size_t)P * (Ch / 8))), dim3(TPB), 0, s, x, P, Ch, out, ldo, oplane,
+  launch_pdl(chan_split_kernel, dim3(gs_grid(chan_split_kernel, (size_t)P * (Ch / 8))), dim3(TPB), 0, s, x, P, Ch, out, ldo, oplane,
              xm);
   check_launch("chan_split");
 }
 
 void chan_merge(cudaStream_t s, const bf16* dproj, int ldp, const bf16* dm, int P, int Ch, bf16* dx) {
-  launch_pdl(chan_merge_kernel, dim3(grid_for((size_t)P * (Ch / 8))), dim3(TPB), 0, s, dproj, ldp, dm, P, Ch, dx);
+  launch_pdl(chan_merge_kernel, dim3(gs_grid(chan_merge_kernel, (size_t)P * (Ch / 8))), dim3(TPB), 0, s, dproj, ldp, dm, P, Ch, dx);
   check_launch("chan_merge");
 }
 
