@@ -789,7 +789,12 @@ void gemm_bf16_tc(cudaStream_t s, int M, int N, int K, const bf16* A, bool a_mn,
     int L = 1;  // lanes per output vector: a power of two (xor tree), <= splits / 4
     while (2 * L <= 32 && 2 * L <= ts.splits / 4) L *= 2;
     const size_t per_block = 256 / L;
-    const int blocks = (int)std::min<size_t>(((size_t)M * N / 4 + per_block - 1) / per_block, 4 * (size_t)num_sms());
+    static int per_sm = 0;  // CTAs per SM of the reduce; NASPIPE_SPLITK_CTAS_PER_SM overrides (tuning)
+    if (!per_sm) {
+      const char* e = getenv("NASPIPE_SPLITK_CTAS_PER_SM");
+      per_sm = e ? std::max(1, atoi(e)) : 4;
+    }
+    const int blocks = (int)std::min<size_t>(((size_t)M * N / 4 + per_block - 1) / per_block, (size_t)per_sm * num_sms());
     if (epi == EPI_F32)
       launch_pdl(splitk_reduce_kernel<EPI_F32>, dim3(blocks), dim3(256), 0, s, M, N, ts.splits, L, ep);
     else
