@@ -42,6 +42,16 @@ static int red_ctas() {
   }
   return v;
 }
+// target CTAs of the depthwise weight-gradient partials (NASPIPE_DW_RED_CTAS, default: the
+// BatchNorm target above)
+static int dw_red_ctas() {
+  static int v = 0;
+  if (!v) {
+    const char* e = getenv("NASPIPE_DW_RED_CTAS");
+    v = e ? std::max(16, atoi(e)) : red_ctas();
+  }
+  return v;
+}
 constexpr float BN_EPS = 1e-5f;
 
 // Row blocking of the per-channel reductions: a function of (P, C) only (deterministic),
@@ -1031,7 +1041,7 @@ void dw_dgrad(cudaStream_t s, const bf16* dz, const float* w, const bf16* add, b
 }
 
 // weight-gradient grid: tiles_w tile columns x NP parts x channel-group blocks, about
-// red_ctas() CTAs; partial blocks = tiles_w * NP (a function of the shape only).
+// dw_red_ctas() CTAs; partial blocks = tiles_w * NP (a function of the shape only).
 static void dw_wgrad_grid(int B, int H, int C, int k, int S, int& TW, int& NP, int& gy, int& tiles_w) {
   const int Ho = (H - 1) / S + 1;
   TW = dw_tw(Ho);
@@ -1039,7 +1049,7 @@ static void dw_wgrad_grid(int B, int H, int C, int k, int S, int& TW, int& NP, i
   tiles_w = (Ho + TW - 1) / TW;
   gy = (C / 8 + CPG - 1) / CPG;
   const int tiles = B * ((Ho + DT_H - 1) / DT_H);
-  NP = std::max(1, std::min(tiles, red_ctas() / std::max(1, tiles_w * gy)));
+  NP = std::max(1, std::min(tiles, dw_red_ctas() / std::max(1, tiles_w * gy)));
   (void)k;
 }
 int dw_wgrad_blocks(int B, int H, int C, int k, int S) {
