@@ -2,6 +2,9 @@
 // MSE loss, casts, synthetic data, and the fp32 MLP family (configs[0]).  All reductions
 // use a fixed order (per-thread sequential, fixed shuffle tree, fixed partial order), never
 // floating-point atomics, so every result is bitwise reproducible.
+#include <algorithm>
+#include <cstdlib>
+
 #include "common.h"
 #include "kernels.h"
 #include "launch.h"
@@ -10,7 +13,16 @@
 namespace naspipe {
 namespace {
 
-constexpr int CS_ROWS = 64;    // rows per block in colsum partials
+// rows per block in colsum partials (a function of the process environment only, so the
+// partial count is fixed per run: NASPIPE_CS_ROWS overrides it for tuning)
+static int cs_rows() {
+  static int v = 0;
+  if (!v) {
+    const char* e = getenv("NASPIPE_CS_ROWS");
+    v = e ? std::max(8, atoi(e)) : 16;
+  }
+  return v;
+}
 
 inline void check_launch(const char* what) {
   cudaError_t e = cudaGetLastError();
@@ -32,7 +44,8 @@ template <>
 __device__ __forceinline__ float to_f<bf16>(bf16 v) { return __bfloat162float(v); }
 
 // thread = 8 consecutive bf16 columns (one 16-byte load per row), rows of the block in order
-__global__ void colsum_bf16_kernel(const bf16* __restrict__ X, float* __restrict__ part, int T_rows, int N) {
+__global__ void colsum_bf16_kernel(const bf16* __restrict__ X, float* __restrict__ part, int T_rows, int N,
+                                   int CS_ROWS) {
   ptx::pdl_wait();
   const int c8 = blockIdx.x * blockDim.x + threadIdx.x;
   if (c8 * 8 >= N) return;
@@ -180,12 +193,12 @@ __global__ void mlp_bwd_kernel(const float* __restrict__ x, const float* __restr
 
 }  // namespace
 
-int colsum_blocks(int T) { return (T + CS_ROWS - 1) / CS_ROWS; }
+int colsum_blocks(int T) { return (T + cs_rows() - 1) / cs_rows(); }
 
 void colsum_bf16(cudaStream_t s, const bf16* X, float* part, int T, int N) {
   NP_REQUIRE(N % 8 == 0, NASPIPE_EINVAL, "colsum width %d must be a multiple of 8", N);
   dim3 grid((N / 8 + 127) / 128, colsum_blocks(T));
-  launch_pdl(colsum_bf16_kernel, grid, dim3(128), 0, s, X, part, T, N);
+  launch_pdl(colsum_bf16_kernel, grid, dim3(128), 0, s, X, part, T, N, cs_rows());
   check_launch("colsum");
 }
 
