@@ -8,6 +8,7 @@
 // block's output gradient comes from the block above (ln_bwd) or from the stage boundary
 // (cast_colsum): results do not depend on where stage boundaries sit.
 #include <algorithm>
+#include <cstdlib>
 
 #include "common.h"
 #include "kernels.h"
@@ -17,8 +18,17 @@
 namespace naspipe {
 namespace {
 
-constexpr int LN_ROWS = 16;  // rows per backward block: warp w takes rows w and w + 8
+constexpr int LN_ROWS_MAX = 32;  // rows per backward block (runtime, <= this): warp w takes rows w, w + 8, ...
 constexpr int LN_WARPS = 8;
+// NASPIPE_LN_ROWS (tuning; default 16) -- fixed per process, so partial counts are too
+static int ln_rows() {
+  static int v = 0;
+  if (!v) {
+    const char* e = getenv("NASPIPE_LN_ROWS");
+    v = e ? std::min(LN_ROWS_MAX, std::max(1, atoi(e))) : 16;
+  }
+  return v;
+}
 
 inline void check_launch(const char* what) {
   cudaError_t e = cudaGetLastError();
@@ -92,8 +102,8 @@ __global__ void __launch_bounds__(256) ln_bwd_kernel(const float* __restrict__ d
                                                      const float* __restrict__ g, const float* __restrict__ resid,
                                                      float* __restrict__ dx, bf16* __restrict__ dx16,
                                                      float* __restrict__ pdg, float* __restrict__ pdb,
-                                                     float* __restrict__ pcs, int T, int d) {
-  __shared__ float s_m1[LN_ROWS], s_m2[LN_ROWS], s_mu[LN_ROWS], s_rs[LN_ROWS];
+                                                     float* __restrict__ pcs, int T, int d, int LN_ROWS) {
+  __shared__ float s_m1[LN_ROWS_MAX], s_m2[LN_ROWS_MAX], s_mu[LN_ROWS_MAX], s_rs[LN_ROWS_MAX];
   ptx::pdl_wait();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int n4 = d / 4, r0 = blockIdx.x * LN_ROWS;
@@ -159,7 +169,7 @@ __global__ void __launch_bounds__(256) ln_bwd_kernel(const float* __restrict__ d
 // X16 = bf16(X) and the column partials of X over LN_ROWS-row blocks, rows summed in order
 // (ln_bwd's colsum order)
 __global__ void __launch_bounds__(256) cast_colsum_kernel(const float* __restrict__ X, bf16* __restrict__ X16,
-                                                          float* __restrict__ part, int T, int d) {
+                                                          float* __restrict__ part, int T, int d, int LN_ROWS) {
   ptx::pdl_wait();
   const int n4 = d / 4, r0 = blockIdx.x * LN_ROWS;
   const int nrows = min(LN_ROWS, T - r0);
@@ -187,7 +197,7 @@ int vpl_for(int d) {
 
 }  // namespace
 
-int ln_bwd_blocks(int T) { return (T + LN_ROWS - 1) / LN_ROWS; }
+int ln_bwd_blocks(int T) { return (T + ln_rows() - 1) / ln_rows(); }
 
 void ln_fwd(cudaStream_t s, const float* x, const float* g, const float* b, bf16* y16, float* mean, float* rstd,
             int T, int d) {
@@ -207,13 +217,13 @@ void ln_bwd(cudaStream_t s, const float* dy, const float* x, const float* mean, 
             int d) {
   NP_REQUIRE(d % 4 == 0, NASPIPE_EINVAL, "LayerNorm width %d must be a multiple of 4", d);
   launch_pdl(ln_bwd_kernel, dim3(ln_bwd_blocks(T)), dim3(256), 0, s, dy, x, mean, rstd, g, resid, dx, dx16, part_dg,
-             part_db, part_colsum, T, d);
+             part_db, part_colsum, T, d, ln_rows());
   check_launch("ln_bwd");
 }
 
 void cast_colsum(cudaStream_t s, const float* X, bf16* X16, float* part, int T, int N) {
   NP_REQUIRE(N % 4 == 0, NASPIPE_EINVAL, "cast_colsum width %d must be a multiple of 4", N);
-  launch_pdl(cast_colsum_kernel, dim3(ln_bwd_blocks(T)), dim3(256), 0, s, X, X16, part, T, N);
+  launch_pdl(cast_colsum_kernel, dim3(ln_bwd_blocks(T)), dim3(256), 0, s, X, X16, part, T, N, ln_rows());
   check_launch("cast_colsum");
 }
 
