@@ -201,6 +201,28 @@ int naspipe_create(const naspipe_supernet_spec* spec, int32_t n_stages, naspipe_
 int naspipe_create_rank(const naspipe_supernet_spec* spec, int32_t n_stages, int32_t stage_rank,
                         int32_t device, const void* nccl_ids, naspipe_t** out);
 
+/* Multi-process engine with the PEER-MEMORY transport (the paper's
+ * inter-stage send/recv, re-designed for NVLink/NVSwitch): this process runs stage
+ * `stage_rank` on CUDA device `device` and allocates its receive rings (stage-input
+ * activations and output gradients, `window` slots each) plus a flag page.  The producing
+ * kernels of the neighbouring ranks store boundary tensors straight into these rings over
+ * CUDA IPC mappings (NVLink peer stores; plain HBM stores when two ranks share one GPU) and
+ * publish each slot with a stream memory write; consumers wait on it with a stream memory
+ * wait.  Protocol: create on every rank -> naspipe_peer_export -> exchange the blobs out of
+ * band (e.g. torch.distributed all_gather_object over gloo) -> naspipe_peer_connect with the
+ * blob of rank-1 (NULL on rank 0) and of rank+1 (NULL on the last rank) -> identical
+ * submit / drain sequences on every rank.  ESTATE if submit comes before connect (D > 1);
+ * EINVAL for a blob of the wrong rank, stage count, window or slot size.  The engine owns
+ * the rings; blobs are plain bytes, valid while the exporting engine lives. */
+int naspipe_create_rank_peer(const naspipe_supernet_spec* spec, int32_t n_stages, int32_t stage_rank,
+                             int32_t device, naspipe_t** out);
+/* Write this rank's blob (CUDA IPC handles of its rings and flag page, sizes, rank) into dst;
+ * *n = its size (dst NULL: size query only).  EINVAL if cap < size or not a peer engine. */
+int naspipe_peer_export(naspipe_t* h, void* dst, size_t cap, size_t* n);
+/* Map the neighbours' rings (see naspipe_create_rank_peer).  Once per engine. */
+int naspipe_peer_connect(naspipe_t* h, const void* prev_blob, size_t prev_n, const void* next_blob,
+                         size_t next_n);
+
 /* Submit the next subnet in chronological order.  subnet_choice_vec [m] with entries in
  * [0, n).  Assigns and returns its sequence id (0, 1, 2, ...).  Plans as far as the
  * streaming rule allows and issues the planned tasks asynchronously. */

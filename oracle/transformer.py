@@ -75,11 +75,11 @@ def _merge(t):
 def attn_fwd(q, k, v, h):
     qh, kh, vh = _heads(q, h), _heads(k, h), _heads(v, h)
     scale = 1.0 / np.sqrt(qh.shape[-1])
-    s = np.einsum("bhqe,bhke->bhqk", qh, kh) * scale
+    s = (qh @ kh.swapaxes(-1, -2)) * scale              # [B,h,S,S] = q k^T
     s = s - s.max(axis=-1, keepdims=True)
     p = np.exp(s)
     p = p / p.sum(axis=-1, keepdims=True)
-    o = np.einsum("bhqk,bhke->bhqe", p, vh)
+    o = p @ vh
     return _merge(o), (qh, kh, vh, p, scale)
 
 
@@ -87,11 +87,11 @@ def attn_bwd(do, cache):
     qh, kh, vh, p, scale = cache
     h = qh.shape[1]
     doh = _heads(do, h)
-    dv = np.einsum("bhqk,bhqe->bhke", p, doh)
-    dp = np.einsum("bhqe,bhke->bhqk", doh, vh)
+    dv = p.swapaxes(-1, -2) @ doh
+    dp = doh @ vh.swapaxes(-1, -2)
     ds = p * (dp - (dp * p).sum(axis=-1, keepdims=True))
-    dq = np.einsum("bhqk,bhke->bhqe", ds, kh) * scale
-    dk = np.einsum("bhqk,bhqe->bhke", ds, qh) * scale
+    dq = (ds @ kh) * scale
+    dk = (ds.swapaxes(-1, -2) @ qh) * scale
     return _merge(dq), _merge(dk), _merge(dv)
 
 

@@ -84,6 +84,9 @@ _sig("naspipe_plan_idle", C.c_int, [C.c_void_p, _i64p, _i64p])
 _sig("naspipe_plan_comm_schedule", C.c_int, [C.c_void_p, C.c_int32, _i64p, C.c_size_t, C.POINTER(C.c_size_t)])
 _sig("naspipe_plan_destroy", None, [C.c_void_p])
 _sig("naspipe_nccl_unique_id", C.c_int, [C.c_void_p])
+_sig("naspipe_create_rank_peer", C.c_int, [_SP, C.c_int32, C.c_int32, C.c_int32, C.POINTER(C.c_void_p)])
+_sig("naspipe_peer_export", C.c_int, [C.c_void_p, C.c_void_p, C.c_size_t, C.POINTER(C.c_size_t)])
+_sig("naspipe_peer_connect", C.c_int, [C.c_void_p, C.c_void_p, C.c_size_t, C.c_void_p, C.c_size_t])
 
 EXPORTED_SYMBOLS = [
     "naspipe_create", "naspipe_create_rank", "naspipe_submit", "naspipe_drain", "naspipe_get_params",
@@ -92,7 +95,8 @@ EXPORTED_SYMBOLS = [
     "naspipe_partition", "naspipe_init_params", "naspipe_init_frozen", "naspipe_plan_create", "naspipe_plan_trace",
     "naspipe_plan_makespan", "naspipe_plan_deps", "naspipe_plan_residency", "naspipe_plan_destroy",
     "naspipe_plan_comm_schedule", "naspipe_plan_idle", "naspipe_plan_mirrored",
-    "naspipe_nccl_unique_id", "naspipe_last_error", "naspipe_abi_version"]
+    "naspipe_nccl_unique_id", "naspipe_last_error", "naspipe_abi_version",
+    "naspipe_create_rank_peer", "naspipe_peer_export", "naspipe_peer_connect"]
 
 
 class NaspipeError(RuntimeError):
@@ -179,6 +183,27 @@ def naspipe_create_rank(spec: Spec, n_stages: int, stage_rank: int, device: int,
     buf = C.create_string_buffer(bytes(nccl_ids), max(1, len(nccl_ids)))
     _check(lib.naspipe_create_rank(spec.ptr, n_stages, stage_rank, device, buf, C.byref(h)))
     return Handle(h, spec)
+
+
+def naspipe_create_rank_peer(spec: Spec, n_stages: int, stage_rank: int, device: int) -> Handle:
+    h = C.c_void_p()
+    _check(lib.naspipe_create_rank_peer(spec.ptr, n_stages, stage_rank, device, C.byref(h)))
+    return Handle(h, spec)
+
+
+def naspipe_peer_export(h: Handle) -> bytes:
+    n = C.c_size_t()
+    _check(lib.naspipe_peer_export(h.ptr, None, 0, C.byref(n)))
+    buf = C.create_string_buffer(n.value)
+    _check(lib.naspipe_peer_export(h.ptr, buf, n.value, C.byref(n)))
+    return buf.raw
+
+
+def naspipe_peer_connect(h: Handle, prev_blob, next_blob) -> None:
+    pb = C.create_string_buffer(bytes(prev_blob), len(prev_blob)) if prev_blob else None
+    nb = C.create_string_buffer(bytes(next_blob), len(next_blob)) if next_blob else None
+    _check(lib.naspipe_peer_connect(h.ptr, pb, len(prev_blob) if prev_blob else 0, nb,
+                                    len(next_blob) if next_blob else 0))
 
 
 def naspipe_nccl_unique_id() -> bytes:

@@ -271,6 +271,19 @@ int naspipe_create_rank(const naspipe_supernet_spec* spec, int32_t n_stages, int
   });
 }
 
+int naspipe_create_rank_peer(const naspipe_supernet_spec* spec, int32_t n_stages, int32_t stage_rank,
+                             int32_t device, naspipe_t** out) {
+  return guarded([&] {
+    NP_REQUIRE(out, NASPIPE_EINVAL, "out NULL");
+    const Spec sp(spec);
+    NP_REQUIRE(sp.raw.sync_policy != NASPIPE_SYNC_BSP || sp.raw.hbm_weight_budget_bytes == 0, NASPIPE_EINVAL,
+               "BSP runs with every candidate resident (hbm_weight_budget_bytes = 0)");
+    auto h = std::make_unique<naspipe_handle>();
+    h->eng = Engine::create_rank_peer(sp, n_stages, stage_rank, device);
+    *out = h.release();
+  });
+}
+
 #define ENGINE_CALL(h, body)                                         \
   guarded([&] {                                                       \
     NP_REQUIRE((h) != nullptr, NASPIPE_EINVAL, "handle NULL");       \
@@ -294,6 +307,14 @@ int naspipe_submit(naspipe_t* h, const int32_t* choice, const naspipe_batch* bat
 }
 
 int naspipe_drain(naspipe_t* h) { return ENGINE_CALL(h, e.drain()); }
+
+int naspipe_peer_export(naspipe_t* h, void* dst, size_t cap, size_t* n) {
+  return ENGINE_CALL(h, e.peer_export(dst, cap, n));
+}
+
+int naspipe_peer_connect(naspipe_t* h, const void* prev_blob, size_t prev_n, const void* next_blob, size_t next_n) {
+  return ENGINE_CALL(h, e.peer_connect(prev_blob, prev_n, next_blob, next_n));
+}
 
 int naspipe_get_params(naspipe_t* h, int32_t block, int32_t choice, float* dst, size_t n_floats) {
   return ENGINE_CALL(h, e.get_params(block, choice, dst, n_floats));

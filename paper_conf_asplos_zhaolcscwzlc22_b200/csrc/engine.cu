@@ -5,6 +5,8 @@
 #include <dlfcn.h>
 #include <nccl.h>
 
+#include <unistd.h>
+
 #include <algorithm>
 #include <cstring>
 
@@ -85,15 +87,26 @@ struct Transport {
 };
 
 // ------------------------------------------------------------------------------ construction
-Engine::Engine(const Spec& spec, int D) : spec_(spec), D_(D), W_(spec.window(D)), planner_(spec_, D) {
+// Slots: every in-flight subnet lies in [wm0, wm0 + W) under CSP / INORDER / ASP (reading A7);
+// under BSP the planner releases a whole bulk regardless of W (the bulk opens after the
+// previous one finished on stage 0, i.e. everywhere), so in-flight ids lie in one bulk and the
+// ring needs max(W, G) slots — with W slots, F(y + W) would overwrite y's stash before B(y).
+static int slot_count(const Spec& s, int D) {
+  return s.raw.sync_policy == NASPIPE_SYNC_BSP ? std::max(s.window(D), s.bulk(D)) : s.window(D);
+}
+
+Engine::Engine(const Spec& spec, int D) : spec_(spec), D_(D), W_(slot_count(spec, D)), planner_(spec_, D) {
   NP_REQUIRE(spec_.raw.sync_policy != NASPIPE_SYNC_BSP || spec_.raw.hbm_weight_budget_bytes == 0, NASPIPE_EINVAL,
              "BSP runs with every candidate resident (hbm_weight_budget_bytes = 0)");
   version_.assign((size_t)spec_.m() * spec_.n(), 0);
   timer_.on = (spec_.raw.flags & NASPIPE_FLAG_TIMING) != 0;
-  if (spec_.raw.hbm_weight_budget_bytes > 0) {  // context switching: no PDL (launch.h)
-    pdl_suppressors().fetch_add(1);
-    suppress_pdl_ = true;
-  }
+  if (spec_.raw.hbm_weight_budget_bytes > 0) suppress_pdl();  // context switching: no PDL (launch.h)
+}
+
+void Engine::suppress_pdl() {
+  if (suppress_pdl_) return;
+  pdl_suppressors().fetch_add(1);
+  suppress_pdl_ = true;
 }
 
 std::unique_ptr<Engine> Engine::create_local(const Spec& spec, int D) {
@@ -117,6 +130,10 @@ std::unique_ptr<Engine> Engine::create_rank(const Spec& spec, int D, int rank, i
   NP_REQUIRE(D == 1 || ids != nullptr, NASPIPE_EINVAL, "nccl_ids NULL");
   std::unique_ptr<Engine> e(new Engine(spec, D));
   e->rank_ = rank;
+  // Multi-process: the compute stream waits on transport streams (NCCL) between kernels;
+  // that cross-stream pattern deadlocked with PDL under context switching (launch.h), so
+  // rank engines launch without PDL until a reproduction clears it.
+  if (D > 1) e->suppress_pdl();
   e->st_.resize(D);
   e->stage_sizes();
   for (int K = 0; K < D; ++K) {
@@ -155,6 +172,116 @@ std::unique_ptr<Engine> Engine::create_rank(const Spec& spec, int D, int rank, i
   return e;
 }
 
+// ------------------------------------------------------------------------------ peer transport
+std::unique_ptr<Engine> Engine::create_rank_peer(const Spec& spec, int D, int rank, int device) {
+  spec.validate_stages(D);
+  NP_REQUIRE(rank >= 0 && rank < D, NASPIPE_EINVAL, "stage_rank %d not in [0,%d)", rank, D);
+  std::unique_ptr<Engine> e(new Engine(spec, D));
+  e->rank_ = rank;
+  // the compute stream waits on stream memory operations between kernels: no PDL across
+  // them (a programmatic launch must never overtake a wait on a peer's flag)
+  if (D > 1) e->suppress_pdl();
+  e->peer_ = std::make_unique<PeerLink>();
+  e->peer_->dev = device;
+  e->st_.resize(D);
+  e->stage_sizes();
+  for (int K = 0; K < D; ++K) {
+    e->st_[K].K = K;
+    e->st_[K].dev = device;
+  }
+  e->setup_stage(rank, device, true);
+  StageRt& st = e->st_[rank];
+  PeerLink& pl = *e->peer_;
+  const int W = e->W_;
+  CU(cudaSetDevice(device));
+  // receive rings and the flag page: plain cudaMalloc allocations (IPC-exportable)
+  if (rank > 0) {
+    CU(cudaMalloc(&pl.in_ring, (size_t)W * st.in_bytes));
+    for (int s = 0; s < W; ++s) st.in[s] = static_cast<uint8_t*>(pl.in_ring) + (size_t)s * st.in_bytes;
+  }
+  if (rank < D - 1) {
+    CU(cudaMalloc(&pl.gout_ring, (size_t)W * st.out_gbytes));
+    for (int s = 0; s < W; ++s) st.gout[s] = static_cast<uint8_t*>(pl.gout_ring) + (size_t)s * st.out_gbytes;
+  }
+  CU(cudaMalloc(reinterpret_cast<void**>(&pl.flags), 2 * (size_t)W * sizeof(uint32_t)));
+  CU(cudaMemset(pl.flags, 0, 2 * (size_t)W * sizeof(uint32_t)));
+  CU(cudaDeviceSynchronize());
+  return e;
+}
+
+void Engine::peer_export(void* dst, size_t cap, size_t* n) {
+  NP_REQUIRE(peer_, NASPIPE_EINVAL, "not a peer-transport engine (naspipe_create_rank_peer)");
+  NP_REQUIRE(n, NASPIPE_EINVAL, "n NULL");
+  *n = sizeof(PeerBlob);
+  if (!dst) return;
+  NP_REQUIRE(cap >= sizeof(PeerBlob), NASPIPE_EINVAL, "blob capacity %zu < %zu", cap, sizeof(PeerBlob));
+  PeerBlob b;
+  std::memset(&b, 0, sizeof b);
+  b.magic = PEER_BLOB_MAGIC;
+  b.version = PEER_BLOB_VERSION;
+  b.rank = rank_;
+  b.device = peer_->dev;
+  b.D = D_;
+  b.W = W_;
+  b.pid = (int32_t)getpid();
+  const StageRt& st = st_[rank_];
+  CU(cudaSetDevice(peer_->dev));
+  if (peer_->in_ring) {
+    b.in_slot_bytes = st.in_bytes;
+    CU(cudaIpcGetMemHandle(&b.in_ring, peer_->in_ring));
+  }
+  if (peer_->gout_ring) {
+    b.gout_slot_bytes = st.out_gbytes;
+    CU(cudaIpcGetMemHandle(&b.gout_ring, peer_->gout_ring));
+  }
+  CU(cudaIpcGetMemHandle(&b.flags, peer_->flags));
+  std::memcpy(dst, &b, sizeof b);
+}
+
+void Engine::peer_connect(const void* prev, size_t prev_n, const void* next, size_t next_n) {
+  NP_REQUIRE(peer_, NASPIPE_EINVAL, "not a peer-transport engine (naspipe_create_rank_peer)");
+  NP_REQUIRE(!peer_->connected, NASPIPE_ESTATE, "peer transport already connected");
+  NP_REQUIRE((rank_ > 0) == (prev != nullptr) && (rank_ < D_ - 1) == (next != nullptr), NASPIPE_EINVAL,
+             "rank %d of %d needs %s", rank_, D_,
+             rank_ == 0 ? "no prev blob" : rank_ == D_ - 1 ? "no next blob" : "both neighbour blobs");
+  PeerLink& pl = *peer_;
+  StageRt& st = st_[rank_];
+  CU(cudaSetDevice(pl.dev));
+  auto open = [&](const cudaIpcMemHandle_t& h) {
+    void* p = nullptr;
+    CU(cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess));
+    pl.opened.push_back(p);
+    return p;
+  };
+  auto check = [&](const void* blob, size_t n, int want_rank) {
+    NP_REQUIRE(n >= sizeof(PeerBlob), NASPIPE_EINVAL, "peer blob of %zu bytes", n);
+    PeerBlob b;
+    std::memcpy(&b, blob, sizeof b);
+    NP_REQUIRE(b.magic == PEER_BLOB_MAGIC && b.version == PEER_BLOB_VERSION, NASPIPE_EINVAL, "not a peer blob");
+    NP_REQUIRE(b.rank == want_rank && b.D == D_ && b.W == W_, NASPIPE_EINVAL,
+               "peer blob of rank %d (D %d, W %d), expected rank %d (D %d, W %d)", b.rank, b.D, b.W, want_rank, D_,
+               W_);
+    return b;
+  };
+  if (rank_ < D_ - 1) {
+    const PeerBlob b = check(next, next_n, rank_ + 1);
+    NP_REQUIRE(b.in_slot_bytes == st.out_bytes, NASPIPE_EINVAL, "activation slot %llu bytes, stage output %zu",
+               (unsigned long long)b.in_slot_bytes, st.out_bytes);
+    pl.next_in = open(b.in_ring);
+    pl.next_flags = static_cast<uint32_t*>(open(b.flags));
+    for (int s = 0; s < W_; ++s) st.out[s] = static_cast<uint8_t*>(pl.next_in) + (size_t)s * st.out_bytes;
+  }
+  if (rank_ > 0) {
+    const PeerBlob b = check(prev, prev_n, rank_ - 1);
+    NP_REQUIRE(b.gout_slot_bytes == st.in_gbytes, NASPIPE_EINVAL, "gradient slot %llu bytes, stage input grad %zu",
+               (unsigned long long)b.gout_slot_bytes, st.in_gbytes);
+    pl.prev_gout = open(b.gout_ring);
+    pl.prev_flags = static_cast<uint32_t*>(open(b.flags));
+    for (int s = 0; s < W_; ++s) st.gin[s] = static_cast<uint8_t*>(pl.prev_gout) + (size_t)s * st.in_gbytes;
+  }
+  pl.connected = true;
+}
+
 // Boundary tensor sizes of every stage (also of the non-local ones: a rank posts receives
 // sized by its neighbours' outputs).
 void Engine::stage_sizes() {
@@ -185,9 +312,10 @@ void Engine::setup_stage(int K, int dev, bool local) {
   st.gout.assign(W_, nullptr);
   st.out.resize(W_);
   st.gin.assign(W_, nullptr);
+  const bool peer = peer_ != nullptr;  // peer transport: out / gin live in the neighbours' rings
   for (int s = 0; s < W_; ++s) {
-    st.out[s] = st.arena->alloc<uint8_t>(st.out_bytes);
-    if (K > 0) st.gin[s] = st.arena->alloc<uint8_t>(st.in_gbytes);
+    if (!peer || K == D_ - 1) st.out[s] = st.arena->alloc<uint8_t>(st.out_bytes);
+    if (K > 0 && !peer) st.gin[s] = st.arena->alloc<uint8_t>(st.in_gbytes);
     if (K == 0) st.in[s] = st.arena->alloc<uint8_t>(st.in_bytes);
     if (K == D_ - 1) st.gout[s] = st.arena->alloc<uint8_t>(st.out_gbytes);
   }
@@ -240,6 +368,7 @@ void Engine::shutdown() {
     for (cudaStream_t s : {tx_->s_act_in, tx_->s_act_out, tx_->s_grad_in, tx_->s_grad_out}) cudaStreamSynchronize(s);
   }
   tx_.reset();
+  peer_.reset();
   for (auto& st : st_) {
     if (!st.local || !st.comp) continue;
     cudaSetDevice(st.dev);
@@ -272,6 +401,7 @@ void Engine::cuda_check(const char* what) {
 // ------------------------------------------------------------------------------ submit / issue
 int64_t Engine::submit(const int32_t* choice, const naspipe_batch* batch) {
   NP_REQUIRE(choice && batch, NASPIPE_EINVAL, "choice/batch NULL");
+  NP_REQUIRE(!peer_ || peer_->connected || D_ == 1, NASPIPE_ESTATE, "peer transport not connected (naspipe_peer_connect)");
   NP_REQUIRE(batch->where >= NASPIPE_BATCH_HOST && batch->where <= NASPIPE_BATCH_SYNTHETIC, NASPIPE_EINVAL,
              "batch.where %d", batch->where);
   NP_REQUIRE(batch->where == NASPIPE_BATCH_SYNTHETIC || (batch->input && batch->target), NASPIPE_EINVAL,
@@ -426,6 +556,9 @@ void Engine::issue_forward(StageRt& st, int64_t y, int slot) {
       p2p_bytes_ += (double)st.in_bytes;
     }
     xin = st.in[slot];
+  } else if (peer_) {
+    stream_wait_geq(st.comp, peer_->flags + slot, (uint32_t)(y + 1));  // F(y, K-1) wrote in[slot]
+    xin = st.in[slot];
   } else {
     CU(cudaStreamWaitEvent(st.comp, tx_->ev_act_rx[slot], 0));
     xin = st.in[slot];
@@ -455,6 +588,10 @@ void Engine::issue_forward(StageRt& st, int64_t y, int slot) {
     if (!null_k) st.fam->loss(slot, st.out[slot], tgt, st.gout[slot], st.loss + y, st.comp);
   }
   CU(cudaEventRecord(st.ev_f[slot], st.comp));
+  if (peer_ && K < D_ - 1) {  // the forward wrote rank K+1's in[slot]: publish it
+    stream_write(st.comp, peer_->next_flags + slot, (uint32_t)(y + 1));
+    p2p_bytes_ += (double)st.out_bytes;
+  }
   if (rank_ >= 0 && tx_ && K < D_ - 1) {
     CU(cudaStreamWaitEvent(tx_->s_act_out, st.ev_f[slot], 0));
     NC(nccl().Send(st.out[slot], st.out_bytes, ncclUint8, 1, tx_->act_out, tx_->s_act_out));
@@ -474,6 +611,8 @@ void Engine::issue_backward(StageRt& st, int64_t y, int slot) {
         CU(cudaMemcpyPeerAsync(st.gout[slot], st.dev, q.gin[slot], q.dev, st.out_gbytes, st.comp));
         p2p_bytes_ += (double)st.out_gbytes;
       }
+    } else if (peer_) {
+      stream_wait_geq(st.comp, peer_->flags + W_ + slot, (uint32_t)(y + 1));  // B(y, K+1) wrote gout[slot]
     } else {
       CU(cudaStreamWaitEvent(st.comp, tx_->ev_grad_rx[slot], 0));
     }
@@ -482,6 +621,10 @@ void Engine::issue_backward(StageRt& st, int64_t y, int slot) {
   void* dx = K > 0 ? st.gin[slot] : nullptr;
   if (!null_k) st.fam->backward(slot, planner_.choice_row(y), st.gout[slot], dx, st.comp);
   CU(cudaEventRecord(st.ev_b[slot], st.comp));
+  if (peer_ && K > 0) {  // the backward wrote rank K-1's gout[slot]: publish it
+    stream_write(st.comp, peer_->prev_flags + W_ + slot, (uint32_t)(y + 1));
+    p2p_bytes_ += (double)st.in_gbytes;
+  }
   if (rank_ >= 0 && tx_ && K > 0) {
     CU(cudaStreamWaitEvent(tx_->s_grad_out, st.ev_b[slot], 0));
     NC(nccl().Send(st.gin[slot], st.in_gbytes, ncclUint8, 0, tx_->grad_out, tx_->s_grad_out));

@@ -11,6 +11,7 @@
 
 #include "context.h"
 #include "family.h"
+#include "peer.h"
 #include "planner.h"
 
 namespace naspipe {
@@ -43,6 +44,11 @@ class Engine {
  public:
   static std::unique_ptr<Engine> create_local(const Spec& spec, int D);
   static std::unique_ptr<Engine> create_rank(const Spec& spec, int D, int rank, int device, const void* nccl_ids);
+  // one process per GPU, peer-memory transport (peer.h): create, export the blob, exchange
+  // blobs out of band, connect to the neighbours' blobs, then submit as usual
+  static std::unique_ptr<Engine> create_rank_peer(const Spec& spec, int D, int rank, int device);
+  void peer_export(void* dst, size_t cap, size_t* n);
+  void peer_connect(const void* prev, size_t prev_n, const void* next, size_t next_n);
   ~Engine();
 
   int64_t submit(const int32_t* choice, const naspipe_batch* batch);
@@ -60,7 +66,8 @@ class Engine {
   void set_sticky(int code, const std::string& msg);
 
  private:
-  bool suppress_pdl_ = false;  // this engine context-switches: PDL off while it lives
+  bool suppress_pdl_ = false;  // context switching or multi-process: PDL off while it lives
+  void suppress_pdl();
   Engine(const Spec& spec, int D);
   void stage_sizes();
   void setup_stage(int K, int dev, bool local);
@@ -78,7 +85,8 @@ class Engine {
   int rank_ = -1;  // -1: single process, all stages local
   Planner planner_;
   std::vector<StageRt> st_;
-  std::unique_ptr<Transport> tx_;
+  std::unique_ptr<Transport> tx_;   // NCCL channels (create_rank)
+  std::unique_ptr<PeerLink> peer_;  // peer-memory transport (create_rank_peer)
   std::vector<BatchRec> batches_;
   std::vector<int32_t> stage_choice_;  // scratch
   size_t issued_ = 0;

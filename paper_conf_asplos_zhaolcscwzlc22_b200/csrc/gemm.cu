@@ -237,12 +237,15 @@ __global__ void __launch_bounds__(THREADS, 1)
     }
     ptx::fence_mbar_init();
   }
+  // PDL: wait for the predecessor grid BEFORE taking TMEM.  An early-launched CTA that held
+  // TMEM columns while it waited could sit on an SM beside a predecessor CTA that still owns
+  // its accumulators; after the wait no earlier kernel of the stream is running.
+  ptx::pdl_wait();  // predecessors' outputs (A, B, residual, ...) are visible from here
   if (warp == 1) ptx::tmem_alloc<Cf::TMEM_COLS>(tmem_holder);
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_holder;
-  ptx::pdl_wait();  // predecessors' outputs (A, B, residual, ...) are visible from here
 
   if (warp == 0) {
     if (lane == 0) {  // ---------------- TMA producer
@@ -394,12 +397,12 @@ __global__ void __launch_bounds__(THREADS, 1)
     }
     ptx::fence_mbar_init();
   }
+  ptx::pdl_wait();  // before taking TMEM (see gemm_tc_kernel)
   if (warp == 1) ptx::tmem_alloc_pair<512>(tmem_holder);
   ptx::tc_fence_before();
   ptx::cluster_sync();  // barriers of both CTAs initialised, TMEM allocated
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_holder;
-  ptx::pdl_wait();
 
   if (warp == 0) {
     if (lane == 0) {  // ---------------- TMA producer (both CTAs)

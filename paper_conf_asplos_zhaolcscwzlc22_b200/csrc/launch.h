@@ -22,14 +22,15 @@ inline std::atomic<int>& pdl_suppressors() {
   return n;
 }
 
-// NASPIPE_NO_PDL=1 launches without the PDL attribute (diagnostics).
+// NASPIPE_NO_PDL=1 launches without the PDL attribute; NASPIPE_FORCE_PDL=1 keeps it even
+// while a suppressing engine lives (diagnostics: the deadlock reproductions).
 inline bool pdl_enabled() {
-  static int v = -1;
-  if (v < 0) {
+  static const int v = [] {
     const char* e = getenv("NASPIPE_NO_PDL");
-    v = (e && e[0] == '1') ? 0 : 1;
-  }
-  return v == 1 && pdl_suppressors().load(std::memory_order_relaxed) == 0;
+    const char* f = getenv("NASPIPE_FORCE_PDL");
+    return (e && e[0] == '1') ? 0 : (f && f[0] == '1') ? 2 : 1;
+  }();
+  return v == 2 || (v == 1 && pdl_suppressors().load(std::memory_order_relaxed) == 0);
 }
 
 template <typename... KArgs, typename... Args>

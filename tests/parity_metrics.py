@@ -1,0 +1,141 @@
+"""Parity metrics of the GPU path against the oracle (reading A15, round 2).
+
+BASELINE.json north_star: parameters "within 1e-3 max relative error after 1 step and within
+1e-2 after 100 steps".  Reading A15 (round 2): the relative error is taken PER TENSOR of the
+packed layout (Wqkv, bqkv, ..., ln2_b; each SPOS conv weight and its BN gamma / beta):
+
+    a15(tensor) = max_i |gpu_i - ref_i| / max_i |ref_i|
+
+over every tensor whose initial value is not identically zero (LayerNorm / BatchNorm beta
+start at 0, so their "relative error" would be the relative error of the update itself).
+The per-candidate number of round 1 (denominator max over the whole packed vector, which LN /
+BN gamma = 1 pins near 1) is kept as a printout only.
+
+Update bar (the parameters after a few steps are dominated by theta_0, so the update is where
+an arithmetic mistake shows):  upd(tensor) = ||dg - dr||_2 / ||dr||_2 with dg = gpu - theta_0,
+dr = ref - theta_0, per tensor, bars per tensor class (fp32 MLP 1e-5;
+bf16 paths: weight matrices and biases 2e-2, LN/BN gamma and beta 5e-2).
+
+Structurally static tensors: the exact gradient of a BatchNorm shift beta is identically zero
+when the BN output reaches the next BatchNorm through a linear map only (SPOS depthwise
+units: dw -> BN -> pw -> BN; the second BN removes any per-channel constant), so their
+reference update is fp64 round-off and a relative bar is meaningless.  They get an absolute
+bar instead: max |dg| <= STATIC_ABS x the largest |dr| of the candidate.
+"""
+import numpy as np
+
+from oracle import train
+
+STATIC_ABS = 1e-3
+
+
+def structurally_static(cfg, name):
+    return cfg["family"] == "spos" and "_dw" in name and name.endswith("_b")
+
+
+def tensor_class(name, shape, kind):
+    if kind == "ones":
+        return "norm_g"
+    if kind == "zeros":
+        return "norm_b"
+    return "matrix" if len(shape) >= 2 else "bias"
+
+
+def per_tensor(cfg, got, ref, theta0):
+    """Records for every tensor of every candidate in ref.  got/ref/theta0: {(b,c): packed}."""
+    recs = []
+    for (b, c), r in ref.items():
+        g = np.asarray(got[(b, c)], dtype=np.float64)
+        r = np.asarray(r, dtype=np.float64)
+        t0 = np.asarray(theta0[(b, c)], dtype=np.float64)
+        cand_a15 = float(np.max(np.abs(g - r)) / np.max(np.abs(r)))
+        cand_dmax = float(np.max(np.abs(r - t0)))
+        off = 0
+        for name, shape, kind, _ in train.candidate_layout(cfg, b, c):
+            n = int(np.prod(shape))
+            gs, rs, ts = g[off:off + n], r[off:off + n], t0[off:off + n]
+            off += n
+            dr, dg = rs - ts, gs - ts
+            rec = {"key": (b, c), "name": name, "cls": tensor_class(name, shape, kind),
+                   "cand_a15": cand_a15, "a15": None, "upd": None, "static": None}
+            if kind != "zeros":
+                rec["a15"] = float(np.max(np.abs(gs - rs)) / np.max(np.abs(rs)))
+            if structurally_static(cfg, name):
+                rec["static"] = float(np.max(np.abs(dg)) / cand_dmax) if cand_dmax > 0 else 0.0
+            elif np.any(dr != 0):
+                rec["upd"] = float(np.linalg.norm(dg - dr) / np.linalg.norm(dr))
+            else:
+                assert np.array_equal(gs, ts), ((b, c), name, "untouched tensor changed")
+            recs.append(rec)
+    return recs
+
+
+def summary(recs):
+    s = {"a15": 0.0, "a15_cand": 0.0, "upd": {}, "static": 0.0, "worst_a15": None, "worst_upd": {}}
+    for r in recs:
+        s["a15_cand"] = max(s["a15_cand"], r["cand_a15"])
+        if r["a15"] is not None and r["a15"] >= s["a15"]:
+            s["a15"], s["worst_a15"] = r["a15"], (r["key"], r["name"])
+        if r["upd"] is not None and r["upd"] >= s["upd"].get(r["cls"], -1.0):
+            s["upd"][r["cls"]] = r["upd"]
+            s["worst_upd"][r["cls"]] = (r["key"], r["name"])
+        if r["static"] is not None:
+            s["static"] = max(s["static"], r["static"])
+    return s
+
+
+def fmt(s):
+    u = " ".join(f"{k}={v:.2e}@{s['worst_upd'][k][0]}{s['worst_upd'][k][1]}" for k, v in sorted(s["upd"].items()))
+    return (f"A15/tensor={s['a15']:.2e} (worst {s['worst_a15']}) A15/candidate={s['a15_cand']:.2e} "
+            f"upd[{u}] static={s['static']:.2e}")
+
+
+UPD_FP32 = {"matrix": 1e-5, "bias": 1e-5, "norm_g": 1e-5, "norm_b": 1e-5}
+UPD_BF16 = {"matrix": 2e-2, "bias": 2e-2, "norm_g": 5e-2, "norm_b": 5e-2}
+
+
+def check(s, a15, upd=None):
+    """Assert the per-tensor A15 bar and (optionally) the per-class update bars."""
+    assert s["a15"] <= a15, fmt(s)
+    if upd is not None:
+        for cls, v in s["upd"].items():
+            assert v <= upd[cls], (cls, fmt(s))
+        assert s["static"] <= STATIC_ABS, fmt(s)
+
+
+def errors(cfg, got, ref, theta0):
+    return summary(per_tensor(cfg, got, ref, theta0))
+
+
+def sampled_errors(cfg, gold, step, got_of):
+    """Per-tensor metrics against a sampled multi-step golden (tools/make_multistep_golden.py).
+    got_of(b, c) -> the GPU's packed vector of candidate (b, c).  The golden stores, per tensor,
+    sampled indices, theta_0 and theta_k at them, and the whole-tensor max |theta_k| (the A15
+    denominator).  A15 as in per_tensor (non-zero-init tensors); upd = normwise update error
+    over the samples, per tensor."""
+    recs = []
+    pre = f"s{step}_"
+    cands = sorted({tuple(int(v) for v in k[len(pre):].split("_", 2)[:2]) for k in gold.files
+                    if k.startswith(pre) and not k.startswith((pre + "max_", pre + "dmax_"))})
+    for (b, c) in cands:
+        g = np.asarray(got_of(b, c), dtype=np.float64)
+        off = 0
+        for name, shape, kind, _ in train.candidate_layout(cfg, b, c):
+            n = int(np.prod(shape))
+            tag = f"{b}_{c}_{name}"
+            gs = g[off:off + n][gold[f"idx_{tag}"]]
+            off += n
+            rs, t0 = gold[pre + tag], gold[f"init_{tag}"]
+            rec = {"key": (b, c), "name": name, "cls": tensor_class(name, shape, kind), "cand_a15": 0.0,
+                   "a15": None, "upd": None, "static": None}
+            if kind != "zeros":
+                rec["a15"] = float(np.max(np.abs(gs - rs)) / gold[f"{pre}max_{tag}"])
+            dr, dg = rs - t0, gs - t0
+            if structurally_static(cfg, name):
+                rec["static"] = float(np.max(np.abs(dg)) / max(float(gold[f"{pre}dmax_{k}"]) for k in
+                                                              [f"{b}_{c}_{nm}" for nm, _, _, _ in
+                                                               train.candidate_layout(cfg, b, c)]))
+            elif np.any(dr != 0):
+                rec["upd"] = float(np.linalg.norm(dg - dr) / np.linalg.norm(dr))
+            recs.append(rec)
+    return summary(recs)

@@ -2,10 +2,10 @@
 through the C ABI (naspipe_create / submit / drain / get_params).
 
 Bars (BASELINE.json north_star, reading A15):
-* parameters: max over candidates of max|gpu - ref| / max|ref| <= 1e-3 after 1 step,
-  <= 1e-2 after 100 steps;  diagnostic on the update Delta = theta_t - theta_0 (the params
-  alone are dominated by theta_0), normwise per tensor: <= 1e-5 (fp32 MLP), <= 1e-1 (bf16
-  transformer; derivation in DESIGN.md "Tolerances");
+* parameters: per tensor max|gpu - ref| / max|ref| <= 1e-3 after 1 step, <= 1e-2 after 100
+  steps (tests/parity_metrics.py); the update Delta = theta_t - theta_0 (the params alone are
+  dominated by theta_0), normwise per tensor: <= 1e-5 (fp32 MLP); bf16: matrices and biases
+  <= 2e-2, LN gamma/beta <= 5e-2 (derivation in DESIGN.md "Tolerances");
 * schedule decisions bit-exact: the executed task trace equals the oracle CSP schedule;
 * two GPU runs bitwise identical; runs at different stage counts D bitwise identical
   (Table 3, artifact P:L557-561) — all stages of a run share one GPU here.
@@ -15,6 +15,8 @@ import pytest
 
 import synth
 from oracle import csp, train
+
+import parity_metrics as pm
 
 torch = pytest.importorskip("torch")
 pytestmark = pytest.mark.gpu
@@ -50,28 +52,10 @@ def run_engine(cfg, choices, batches, D, where=npipe.BATCH_HOST, flags=FLAGS, th
 
 
 def param_errors(cfg, got, ref, theta0):
-    """(A15 metric, update diagnostic).
-
-    A15: max over candidates of max_i |gpu_i - ref_i| / max_i |ref_i| over the
-    candidate's packed parameter vector (the unit naspipe_get_params returns).
-    Diagnostic: max over tensors of the normwise relative error of the update
-    ||(gpu - theta0) - (ref - theta0)||_2 / ||ref - theta0||_2 (untouched tensors must be
-    bitwise unchanged)."""
-    worst, worst_delta = 0.0, 0.0
-    for (b, c), r in ref.items():
-        g = got[(b, c)].astype(np.float64)
-        worst = max(worst, np.max(np.abs(g - r)) / np.max(np.abs(r)))
-        off = 0
-        for name, shape, _, _ in train.candidate_layout(cfg, b, c):
-            n = int(np.prod(shape))
-            gs, rs, t0 = g[off:off + n], r[off:off + n], theta0[(b, c)][off:off + n].astype(np.float64)
-            off += n
-            dr = rs - t0
-            if np.any(dr != 0):
-                worst_delta = max(worst_delta, np.linalg.norm((gs - t0) - dr) / np.linalg.norm(dr))
-            else:
-                assert np.array_equal(gs, t0), (b, c, name)
-    return worst, worst_delta
+    """Per-tensor A15 and update metrics (tests/parity_metrics.py, A15); printed."""
+    sm = pm.errors(cfg, got, ref, theta0)
+    print(cfg.get("family"), pm.fmt(sm))
+    return sm
 
 
 def _workload(name, N, **over):
@@ -102,8 +86,7 @@ def test_toy_mlp_parity(N, tol):
     cfg, choices, batches = _workload("toy", N)
     theta0, ref, ref_loss = _oracle(cfg, choices, batches)
     params, losses, trace, stats = run_engine(cfg, choices, batches, D=2)
-    err, derr = param_errors(cfg, params, ref, theta0)
-    assert err <= tol and derr <= 1e-5, (err, derr)
+    pm.check(param_errors(cfg, params, ref, theta0), tol, pm.UPD_FP32)
     np.testing.assert_allclose(losses, ref_loss, rtol=1e-5)
     _check_trace(cfg, choices, 2, trace)
     assert stats["version_checks"] == 2 * N * cfg["n_blocks"]
@@ -125,8 +108,8 @@ def test_tiny_transformer_parity(N, tol):
     cfg, choices, batches = _workload("tiny_transformer", N)
     theta0, ref, ref_loss = _oracle(cfg, choices, batches)
     params, losses, trace, _ = run_engine(cfg, choices, batches, D=2)
-    err, derr = param_errors(cfg, params, ref, theta0)
-    assert err <= tol and derr <= 1e-1, (err, derr)
+    sm = param_errors(cfg, params, ref, theta0)
+    pm.check(sm, tol, pm.UPD_BF16 if N <= 8 else None)
     np.testing.assert_allclose(losses, ref_loss, rtol=1e-2)
     _check_trace(cfg, choices, 2, trace)
 
@@ -163,42 +146,52 @@ def test_null_kernels_and_errors():
     npipe.naspipe_destroy(h)
 
 
-def test_transformer_full_size_sampled():
-    """configs[2] at BASELINE.json's full size (24 blocks, d = 1024, S = 128, B = 32, bf16) in
-    the bench's launch configuration (one stage, DEVICE batch), one subnet, against sampled
-    outputs of the fp64 oracle (tests/golden/transformer_fullsize_step1.npz, written by
-    tools/make_fullsize_golden.py, which calls only oracle/).  Bars: loss rtol 1e-2; A15
-    (max |gpu - ref| / max |ref| per candidate, over the sampled entries with the stored
-    full-vector max |ref|) <= 1e-3; update diagnostic on the sampled entries of every tensor
-    <= 1e-1 (DESIGN.md "Tolerances")."""
-    import os
-    gold = np.load(os.path.join(os.path.dirname(__file__), "golden", "transformer_fullsize_step1.npz"))
-    cfg = synth.get_config("transformer")
-    ch = synth.sample_choices(1, cfg["n_blocks"], cfg["n_choices"])[0]
-    assert np.array_equal(ch, gold["choices"])
-    x, t = synth.make_batch(cfg, 0)
+def run_fullsize(name, gold, steps):
+    """The first `steps` subnets of a BASELINE.json config at full size, in the bench's launch
+    configuration (one stage, DEVICE batches).  Returns (params getter, losses)."""
+    cfg = synth.get_config(name)
+    ch = gold["choices"][:steps]
+    assert np.array_equal(ch, synth.sample_choices(steps, cfg["n_blocks"], cfg["n_choices"]))
     h = npipe.naspipe_create(npipe.Spec(cfg, flags=npipe.FLAG_VERSION_CHECK), 1)
-    xd, td = torch.from_numpy(x).cuda(), torch.from_numpy(t).cuda()
-    npipe.naspipe_submit(h, ch, xd, td, where=npipe.BATCH_DEVICE)
+    keep = []
+    for y in range(steps):
+        x, t = synth.make_batch(cfg, y)
+        xd, td = torch.from_numpy(x).cuda(), torch.from_numpy(t).cuda()
+        keep += [xd, td]
+        npipe.naspipe_submit(h, ch[y], xd, td, where=npipe.BATCH_DEVICE)
     npipe.naspipe_drain(h)
-    loss = npipe.naspipe_get_losses(h, 1)[0]
-    a15 = upd = 0.0
-    for b in range(cfg["n_blocks"]):
-        c = int(ch[b])
-        g = npipe.naspipe_get_params(h, b, c).astype(np.float64)
-        off = 0
-        for name, shape, _, _ in train.candidate_layout(cfg, b, c):
-            k = int(np.prod(shape))
-            idx = gold[f"idx_{b}_{name}"]
-            seg = g[off:off + k][idx]
-            off += k
-            a15 = max(a15, np.max(np.abs(seg - gold[f"new_{b}_{name}"])) / gold[f"maxabs_{b}"])
-            dref = gold[f"dsamp_{b}_{name}"]
-            dgpu = seg - (gold[f"new_{b}_{name}"] - dref)
-            if np.linalg.norm(dref) > 0:
-                upd = max(upd, np.linalg.norm(dgpu - dref) / np.linalg.norm(dref))
+    losses = npipe.naspipe_get_losses(h, steps)
+    params = {}
+
+    def got_of(b, c):
+        if (b, c) not in params:
+            params[(b, c)] = npipe.naspipe_get_params(h, b, c)
+        return params[(b, c)]
+    return cfg, h, got_of, losses
+
+
+def load_gold(name):
+    import os
+    path = os.path.join(os.path.dirname(__file__), "golden", name)
+    if not os.path.exists(path):
+        pytest.skip(f"{name} not generated (tools/make_multistep_golden.py)")
+    return np.load(path)
+
+
+@pytest.mark.parametrize("steps,tol", [(1, 1e-3), (100, 1e-2)])
+def test_transformer_full_size_against_oracle_samples(steps, tol):
+    """configs[2] at BASELINE.json's full size (24 blocks x 4 choices, d = 1024, S = 128, B = 32,
+    bf16) in the bench's launch configuration, the first `steps` subnets, against sampled
+    outputs of the fp64 oracle's sequential training (tests/golden/transformer_fullsize_100steps.npz,
+    written by tools/make_multistep_golden.py, which calls only oracle/).  Bars (north_star):
+    per-tensor A15 <= 1e-3 after 1 step and <= 1e-2 after 100; after 1 step the update bars of
+    tests/parity_metrics.py over the sampled entries; losses rtol 1e-2."""
+    gold = load_gold("transformer_fullsize_100steps.npz")
+    if f"s{steps}_max_0_{int(gold['choices'][0][0])}_Wqkv" not in gold.files:
+        pytest.skip(f"checkpoint {steps} not in the golden yet")
+    cfg, h, got_of, losses = run_fullsize("transformer", gold, steps)
+    sm = pm.sampled_errors(cfg, gold, steps, got_of)
     npipe.naspipe_destroy(h)
-    print(f"configs[2] full size: A15(sampled)={a15:.3e} update={upd:.3e} loss {loss:.6f} vs {float(gold['loss']):.6f}")
-    assert abs(loss - gold["loss"]) <= 1e-2 * abs(gold["loss"])
-    assert a15 <= 1e-3, a15
-    assert upd <= 1e-1, upd
+    print(f"configs[2] full size, {steps} steps: {pm.fmt(sm)}; losses {losses[-2:]} vs {gold['losses'][steps - 2:steps]}")
+    pm.check(sm, tol, pm.UPD_BF16 if steps == 1 else None)
+    np.testing.assert_allclose(losses, gold["losses"][:steps], rtol=1e-2)
