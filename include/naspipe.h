@@ -246,8 +246,11 @@ int naspipe_get_trace(naspipe_t* h, int64_t* dst, size_t cap_tasks, size_t* n_ta
 
 /* Statistics, 16 doubles: [0] tasks, [1] kernel launches, [2] h2d bytes, [3] d2h bytes,
  * [4] p2p bytes, [5] makespan ticks, [6] dominant-kernel launches, [7] dominant-kernel
- * flops, [8] dominant-kernel ms (TIMING flag), [9] residency loads, [10] residency evicts,
- * [11] writebacks, [12] version checks passed, [13..15] reserved. */
+ * algorithmic work (flops of the transformer GEMMs / HBM bytes of the SPOS BatchNorm
+ * kernels; both counted whether or not TIMING is on), [8] dominant-kernel ms (TIMING flag
+ * only), [9] residency loads, [10] residency evicts, [11] writebacks, [12] version checks
+ * passed, [13] algorithmic flops of every tcgen05 GEMM launched by this process,
+ * [14] tcgen05 GEMM launches of this process, [15] reserved. */
 int naspipe_get_stats(naspipe_t* h, double* dst16);
 
 /* Turn the dominant-kernel CUDA-event timing (stats [6..8]) on or off for the work submitted

@@ -18,7 +18,7 @@ BATCH_HOST, BATCH_DEVICE, BATCH_SYNTHETIC = 0, 1, 2
 FLAG_TRACE, FLAG_VERSION_CHECK, FLAG_NULL_KERNELS, FLAG_TIMING, FLAG_RECOMPUTE = 1, 2, 4, 8, 16
 STATS_FIELDS = ["tasks", "kernel_launches", "h2d_bytes", "d2h_bytes", "p2p_bytes", "makespan_ticks",
                 "dominant_launches", "dominant_flops", "dominant_ms", "res_loads", "res_evicts",
-                "writebacks", "version_checks", "r13", "r14", "r15"]
+                "writebacks", "version_checks", "gemm_flops", "gemm_launches", "r15"]
 
 _i32p = C.POINTER(C.c_int32)
 _i64p = C.POINTER(C.c_int64)

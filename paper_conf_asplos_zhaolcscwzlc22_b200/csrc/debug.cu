@@ -1,4 +1,6 @@
 // Kernel-level C entry points for the kernel unit tests (include/naspipe_debug.h).
+#include <vector>
+
 #include "common.h"
 #include "kernels.h"
 #include "naspipe_debug.h"
@@ -125,37 +127,46 @@ int naspipe_debug_bn_fwd(const void* z, int P, int C, const float* g, const floa
                          size_t yplane, float* mean, float* rstd, void* stream) {
   return dguard([&] {
     cudaStream_t s = (cudaStream_t)stream;
-    const int nblk = bn_part_blocks(P, C);
-    float* part = nullptr;
-    int* ctr = nullptr;
-    NP_REQUIRE(cudaMalloc(&part, (size_t)nblk * 2 * C * 4) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
-    NP_REQUIRE(cudaMalloc(&ctr, 4) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
-    cudaMemsetAsync(ctr, 0, 4, s);
-    bn_stats(s, (const bf16*)z, P, C, part, ctr, mean, rstd);
-    bn_apply(s, (const bf16*)z, P, C, mean, rstd, g, b, relu, (bf16*)y, ldy, yplane);
+    unsigned long long* acc = nullptr;
+    int* ticket = nullptr;
+    NP_REQUIRE(cudaMalloc(&acc, (size_t)2 * C * 8) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
+    NP_REQUIRE(cudaMalloc(&ticket, 4) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
+    cudaMemsetAsync(acc, 0, (size_t)2 * C * 8, s);
+    cudaMemsetAsync(ticket, 0, 4, s);
+    bn_stats(s, (const bf16*)z, P, C, acc);
+    bn_apply(s, (const bf16*)z, P, C, acc, ticket, mean, rstd, g, b, relu, (bf16*)y, ldy, yplane);
     cudaStreamSynchronize(s);
-    cudaFree(part);
-    cudaFree(ctr);
+    cudaFree(acc);
+    cudaFree(ticket);
   });
 }
 
+// sums [2][C] (s1, s2) and old [2][C] (g, b before the WRITE) are reported for the tests
 int naspipe_debug_bn_bwd(const void* dy, int lddy, const void* z, int P, int C, const float* mean,
                          const float* rstd, float* g, float* b, int relu, void* dz, float* sums, float* old, float lr,
                          int update, void* stream) {
   return dguard([&] {
     cudaStream_t s = (cudaStream_t)stream;
-    const int nblk = bn_part_blocks(P, C);
-    float* part = nullptr;
-    int* ctr = nullptr;
-    NP_REQUIRE(cudaMalloc(&part, (size_t)nblk * 2 * C * 4) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
-    NP_REQUIRE(cudaMalloc(&ctr, 4) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
-    cudaMemsetAsync(ctr, 0, 4, s);
-    bn_bwd_reduce(s, (const bf16*)dy, lddy, (const bf16*)z, P, C, mean, rstd, g, b, g, b, relu, part, ctr, sums, old, lr,
-                  update);
-    bn_bwd_apply(s, (const bf16*)dy, lddy, (const bf16*)z, P, C, mean, rstd, old, sums, relu, (bf16*)dz);
+    unsigned long long* acc = nullptr;
+    int* ticket = nullptr;
+    NP_REQUIRE(cudaMalloc(&acc, (size_t)2 * C * 8) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
+    NP_REQUIRE(cudaMalloc(&ticket, 4) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
+    cudaMemsetAsync(acc, 0, (size_t)2 * C * 8, s);
+    cudaMemsetAsync(ticket, 0, 4, s);
+    cudaMemcpyAsync(old, g, (size_t)C * 4, cudaMemcpyDeviceToDevice, s);
+    cudaMemcpyAsync(old + C, b, (size_t)C * 4, cudaMemcpyDeviceToDevice, s);
+    bn_bwd_reduce(s, (const bf16*)dy, lddy, (const bf16*)z, P, C, mean, rstd, g, b, relu, acc);
     cudaStreamSynchronize(s);
-    cudaFree(part);
-    cudaFree(ctr);
+    std::vector<unsigned long long> h(2 * (size_t)C);
+    cudaMemcpy(h.data(), acc, h.size() * 8, cudaMemcpyDeviceToHost);
+    std::vector<float> f(h.size());
+    for (size_t i = 0; i < h.size(); ++i) f[i] = (float)((double)(long long)h[i] / 1099511627776.0);
+    cudaMemcpy(sums, f.data(), f.size() * 4, cudaMemcpyHostToDevice);
+    bn_bwd_apply(s, (const bf16*)dy, lddy, (const bf16*)z, P, C, mean, rstd, g, b, g, b, lr, update, acc, ticket, relu,
+                 (bf16*)dz);
+    cudaStreamSynchronize(s);
+    cudaFree(acc);
+    cudaFree(ticket);
   });
 }
 

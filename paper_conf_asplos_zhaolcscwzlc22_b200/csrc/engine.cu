@@ -100,7 +100,6 @@ Engine::Engine(const Spec& spec, int D) : spec_(spec), D_(D), W_(slot_count(spec
              "BSP runs with every candidate resident (hbm_weight_budget_bytes = 0)");
   version_.assign((size_t)spec_.m() * spec_.n(), 0);
   timer_.on = (spec_.raw.flags & NASPIPE_FLAG_TIMING) != 0;
-  if (spec_.raw.hbm_weight_budget_bytes > 0) suppress_pdl();  // context switching: no PDL (launch.h)
 }
 
 void Engine::suppress_pdl() {
@@ -440,6 +439,7 @@ void Engine::drain() {
     CU(cudaStreamSynchronize(st.copy));
     CU(cudaStreamSynchronize(st.comp));
     st.store->sync();
+    st.fam->check_after_drain();
   }
   if (tx_)
     for (cudaStream_t s : {tx_->s_act_in, tx_->s_act_out, tx_->s_grad_in, tx_->s_grad_out})
@@ -712,6 +712,8 @@ void Engine::get_stats(double* o) {
   o[7] = timer_.flops;
   o[8] = timer_.ms;
   o[12] = (double)version_checks_;
+  o[13] = (double)gemm_flop_count();
+  o[14] = (double)gemm_launch_count();
 }
 
 void Engine::get_residency_trace(int64_t* dst, size_t cap, size_t* n) {

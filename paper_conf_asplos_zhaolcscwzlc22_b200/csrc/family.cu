@@ -41,11 +41,11 @@ void KernelTimer::begin(cudaStream_t s) {
   cudaEventRecord(pairs[used].first, s);
 }
 void KernelTimer::end(cudaStream_t s, double f) {
+  flops += f;  // algorithmic work and launches are counted with or without the events
+  launches += 1;
   if (!on) return;
   cudaEventRecord(pairs[used].second, s);
   ++used;
-  flops += f;
-  launches += 1;
 }
 void KernelTimer::collect() {
   for (size_t i = 0; i < used; ++i) {

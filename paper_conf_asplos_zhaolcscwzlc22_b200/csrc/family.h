@@ -86,6 +86,8 @@ class Family {
     const size_t k = (size_t)local_block * n_choices_ + c;
     return k >= upd_.size() || upd_[k] == nullptr;
   }
+  // called by the engine after a drain's synchronisation (device-side sticky checks)
+  virtual void check_after_drain() {}
   FamilyCounters counters;
   KernelTimer* timer = nullptr;
 

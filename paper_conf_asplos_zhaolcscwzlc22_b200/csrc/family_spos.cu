@@ -40,7 +40,7 @@ class SposFamily : public Family {
     w16_.assign((size_t)nb * n, nullptr);
     plans_.resize((size_t)nb * n);
     dims_.resize(nb);
-    size_t stash_max = 0, stats_max = 0, dz_max = 0, g_max = 0, blk_max = 0, part_max = 0, dwp_max = 0, C_max = 0;
+    size_t stash_max = 0, stats_max = 0, dz_max = 0, g_max = 0, blk_max = 0, dwp_max = 0, C_max = 0;
     ws_elems_ = 0;
     for (int j = 0; j < nb; ++j) {
       const int b = blocks[j];
@@ -59,7 +59,6 @@ class SposFamily : public Family {
           st += 2 * (size_t)u.cout;
           dz_max = std::max(dz_max, po * u.cout);
           g_max = std::max({g_max, pi * u.cin, po * u.cout});
-          part_max = std::max(part_max, (size_t)bn_part_blocks((int)po, u.cout) * 2 * u.cout);
           C_max = std::max(C_max, (size_t)u.cout);
           if (u.dw)
             dwp_max = std::max(dwp_max, (size_t)dw_wgrad_blocks(B_, u.H_in, u.cout, u.k, u.stride) * u.cout * u.k * u.k);
@@ -72,15 +71,8 @@ class SposFamily : public Family {
     }
     const int hw0 = spec.spos_stem_hw(), hwl = spec.spos_last_hw(), C0 = spec.raw.stem_channels,
               Cl = spec.chans.back(), Ch = spec.raw.head_channels, ncls = spec.raw.num_classes;
-    if (last_) {
-      const size_t PL = P(hwl);
-      part_max = std::max(part_max, (size_t)bn_part_blocks((int)PL, Ch) * 2 * Ch);
-      C_max = std::max(C_max, (size_t)Ch);
-    }
-    if (first_) {
-      part_max = std::max(part_max, (size_t)bn_part_blocks((int)P(hw0), C0) * 2 * C0);
-      C_max = std::max(C_max, (size_t)C0);
-    }
+    if (last_) C_max = std::max(C_max, (size_t)Ch);
+    if (first_) C_max = std::max(C_max, (size_t)C0);
     stash_.resize((size_t)W * nb);
     stats_.resize((size_t)W * nb);
     act_.assign((size_t)W * nb, nullptr);
@@ -105,14 +97,15 @@ class SposFamily : public Family {
     gb_[0] = A.alloc<bf16>(blk_max);
     gb_[1] = A.alloc<bf16>(blk_max);
     gfirst_ = A.alloc<bf16>(g_max);
-    part_ = A.alloc<float>(part_max);
+    // fixed-point BatchNorm accumulators + arrival tickets (zero between uses; spos.cu)
+    acc_f_ = A.alloc<unsigned long long>(2 * C_max);
+    acc_b_ = A.alloc<unsigned long long>(2 * C_max);
+    tick_ = A.alloc<int>(2);
+    cudaMemset(acc_f_, 0, 2 * C_max * 8);
+    cudaMemset(acc_b_, 0, 2 * C_max * 8);
+    cudaMemset(tick_, 0, 2 * sizeof(int));
     dwpart_ = A.alloc<float>(std::max<size_t>(dwp_max, 1));
     ws_ = A.alloc<float>(std::max<size_t>(ws_elems_, 4));
-    sums_ = A.alloc<float>(2 * C_max);
-    ctr_ = A.alloc<int>(1);
-    cudaMemset(ctr_, 0, sizeof(int));
-
-    old_ = A.alloc<float>(2 * C_max);
     if (first_) {
       std::vector<float> h(spec.frozen_count(0));
       spec.init_frozen(0, h.data());
@@ -186,7 +179,7 @@ class SposFamily : public Family {
       spos_stem_conv(s, static_cast<const float*>(x_in), w_stem_, stem_z_, B_, H, C0);
       t_bn_stats(s, stem_z_, Po, C0, stem_mean_, stem_rstd_);
       t_bn_apply(s, stem_z_, Po, C0, stem_mean_, stem_rstd_, ones_s_, zeros_s_, 1, stem_y_[slot], C0, (size_t)Po * C0);
-      counters.launches += 4;
+      counters.launches += 3;
       x = stem_y_[slot];
     }
     for (int j = 0; j < nb; ++j) {
@@ -243,12 +236,17 @@ class SposFamily : public Family {
     ce_mean(s, loss_per_, B_, loss_dst);
     fc_dgap(s, dlogits_, wf_, B_, Ch, ncls, dgap_);
     head_bcast(s, dgap_, B_, HW, Ch, rh_);  // dr overwrites r (the mask is recomputed from z)
-    t_bn_bwd_reduce(s, rh_, Ch, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, ones_, zeros_, 1, 0.f, 0);
-    t_bn_bwd_apply(s, rh_, Ch, zh_, PL, Ch, hmean_, hrstd_, 1, dzh_);
+    t_bn_bwd_reduce(s, rh_, Ch, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, 1);
+    t_bn_bwd_apply(s, rh_, Ch, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, ones_, zeros_, 0, 1, dzh_);
     e = GemmEpiParams();
     e.out = dy;
     gemm(s, PL, Cl, Ch, dzh_, false, Ch, wh16_, true, Cl, EPI_BF16, e);
-    counters.launches += 12;
+    counters.launches += 10;
+  }
+
+  void check_after_drain() override {
+    NP_REQUIRE(!bn_fix_overflow(), NASPIPE_EINTERNAL,
+               "BatchNorm fixed-point accumulator overflow (a partial sum outside the 64-bit range, spos.cu)");
   }
 
   void synth_target(void* dst, uint64_t seed, cudaStream_t s) override {
@@ -281,28 +279,28 @@ class SposFamily : public Family {
   // BatchNorm kernels, the step's dominant kernel family (bench.py roofline):
   // with FLAG_TIMING each call is bracketed by CUDA events on its stream and credited with
   // its algorithmic HBM bytes (bf16x2 forward tensors 4 B/element, bf16 gradients 2 B).
-  void t_bn_stats(cudaStream_t s, const bf16* z, int Pp, int C, float* mean, float* rstd) {
+  void t_bn_stats(cudaStream_t s, const bf16* z, int Pp, int C, float*, float*) {
     if (timer) timer->begin(s);
-    bn_stats(s, z, Pp, C, part_, ctr_, mean, rstd);
+    bn_stats(s, z, Pp, C, acc_f_);
     if (timer) timer->end(s, 4.0 * Pp * C);
   }
-  void t_bn_apply(cudaStream_t s, const bf16* z, int Pp, int C, const float* mean, const float* rstd, const float* g,
+  void t_bn_apply(cudaStream_t s, const bf16* z, int Pp, int C, float* mean, float* rstd, const float* g,
                   const float* b, int relu, bf16* y, int ldy, size_t yplane) {
     if (timer) timer->begin(s);
-    bn_apply(s, z, Pp, C, mean, rstd, g, b, relu, y, ldy, yplane);
+    bn_apply(s, z, Pp, C, acc_f_, tick_, mean, rstd, g, b, relu, y, ldy, yplane);
     if (timer) timer->end(s, 8.0 * Pp * C);
   }
   void t_bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int Pp, int C, const float* mean,
-                       const float* rstd, const float* g, const float* b, float* gu, float* bu, int relu, float lr,
-                       int update) {
+                       const float* rstd, const float* g, const float* b, int relu) {
     if (timer) timer->begin(s);
-    bn_bwd_reduce(s, dy, lddy, z, Pp, C, mean, rstd, g, b, gu, bu, relu, part_, ctr_, sums_, old_, lr, update);
+    bn_bwd_reduce(s, dy, lddy, z, Pp, C, mean, rstd, g, b, relu, acc_b_);
     if (timer) timer->end(s, 6.0 * Pp * C);
   }
   void t_bn_bwd_apply(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int Pp, int C, const float* mean,
-                      const float* rstd, int relu, bf16* dz) {
+                      const float* rstd, const float* g, const float* b, float* gu, float* bu, int update, int relu,
+                      bf16* dz) {
     if (timer) timer->begin(s);
-    bn_bwd_apply(s, dy, lddy, z, Pp, C, mean, rstd, old_, sums_, relu, dz);
+    bn_bwd_apply(s, dy, lddy, z, Pp, C, mean, rstd, g, b, gu, bu, lr_, update, acc_b_, tick_ + 1, relu, dz);
     if (timer) timer->end(s, 8.0 * Pp * C);
   }
 
@@ -367,7 +365,7 @@ class SposFamily : public Family {
       }
       t_bn_apply(s, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, u.relu, y, ldy, yplane);
       hplane = yplane;
-      counters.launches += 3;
+      counters.launches += 2;
       recs.push_back(r);
       h = y;
     }
@@ -379,10 +377,10 @@ class SposFamily : public Family {
     const int Po = (int)P(u.H_out);
     ring_ = (ring_ + 1) % kRing;
     if (ring_used_[ring_]) cudaStreamWaitEvent(s, ev_wg_[ring_], 0);
-    t_bn_bwd_reduce(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, Um + u.off_g,
-                    Um + u.off_b, u.relu, lr_, 1);
-    t_bn_bwd_apply(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, u.relu, dz_[ring_]);
-    counters.launches += 3;
+    t_bn_bwd_reduce(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, u.relu);
+    t_bn_bwd_apply(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, Um + u.off_g, Um + u.off_b,
+                   1, u.relu, dz_[ring_]);
+    counters.launches += 2;
   }
 
   // conv backward of one unit from dz: the input gradient into dst (+ add) with the
@@ -489,8 +487,9 @@ class SposFamily : public Family {
   bool ring_used_[kRing] = {false, false, false};
   cudaStream_t side_ = nullptr;  // weight gradients + SGD of the backward
   cudaEvent_t ev_dg_[kRing], ev_wg_[kRing], ev_join_;
-  float *part_, *dwpart_, *ws_, *sums_, *old_;
-  int* ctr_;  // last-CTA ticket of the BN reductions (stage stream)
+  float *dwpart_, *ws_;
+  unsigned long long *acc_f_, *acc_b_;  // BatchNorm fixed-point accumulators (forward / backward)
+  int* tick_;                           // [2] arrival tickets of bn_apply / bn_bwd_apply
   size_t ws_elems_ = 0;
   // stem
   float* w_stem_ = nullptr;

@@ -581,6 +581,7 @@ CUtensorMap make_map(const bf16* base, uint64_t inner, uint64_t outer, uint64_t 
 }
 
 std::atomic<uint64_t> g_gemm_launches{0};
+std::atomic<uint64_t> g_gemm_flops{0};  // algorithmic 2*M*N*K of every GEMM call (bf16x2: one product)
 
 int num_sms() {
   static int n = 0;
@@ -726,6 +727,7 @@ void dispatch_epi(cudaStream_t s, int M, int N, const TileSpace& ts, const CUten
 }  // namespace
 
 uint64_t gemm_launch_count() { return g_gemm_launches.load(); }
+uint64_t gemm_flop_count() { return g_gemm_flops.load(); }
 
 // The CTA-pair kernel serves every GEMM with M, N >= 256 (the transformer's and the SPOS
 // head's); smaller ones (SPOS 1x1 convs with N < 256, the 3-pass product) use 1-CTA tiles.
@@ -755,6 +757,7 @@ void gemm_bf16_tc(cudaStream_t s, int M, int N, int K, const bf16* A, bool a_mn,
                   bool b_mn, int ldb, int epi, const GemmEpiParams& ep_in) {
   NP_REQUIRE(M > 0 && N > 0 && K > 0 && N % 16 == 0, NASPIPE_EINVAL, "gemm dims M=%d N=%d K=%d (N%%16)", M, N, K);
   GemmEpiParams ep = ep_in;
+  g_gemm_flops.fetch_add(2ull * (uint64_t)M * (uint64_t)N * (uint64_t)K, std::memory_order_relaxed);
   const bool pair = gemm_uses_pair(M, N);
   int splits = 1;
   if ((epi == EPI_SGD || epi == EPI_F32) && ep.ws != nullptr) {
@@ -809,6 +812,7 @@ void gemm_bf16x2_tc(cudaStream_t s, int M, int N, int K, const bf16* A_hi, const
                     const bf16* B_hi, const bf16* B_lo, int ldb, int epi, const GemmEpiParams& ep) {
   NP_REQUIRE(M > 0 && N > 0 && K > 0 && N % 16 == 0, NASPIPE_EINVAL, "gemm x2 dims M=%d N=%d K=%d (N%%16)", M, N, K);
   NP_REQUIRE(epi == EPI_X2 || epi == EPI_BF16 || epi == EPI_F32, NASPIPE_EINVAL, "gemm x2 epilogue %d", epi);
+  g_gemm_flops.fetch_add(2ull * (uint64_t)M * (uint64_t)N * (uint64_t)K, std::memory_order_relaxed);
   const int tn = N <= 64 ? 64 : (N <= 128 ? 128 : 256);
   const CUtensorMap ta = make_map(A_hi, (uint64_t)K, (uint64_t)M, (uint64_t)lda, BM);
   const CUtensorMap ta2 = make_map(A_lo, (uint64_t)K, (uint64_t)M, (uint64_t)lda, BM);

@@ -54,6 +54,7 @@ void gemm_bf16x2_tc(cudaStream_t s, int M, int N, int K, const bf16* A_hi, const
                     const bf16* B_hi, const bf16* B_lo, int ldb, int epi, const GemmEpiParams& ep);
 // number of tcgen05 GEMM launches so far in this process (stats)
 uint64_t gemm_launch_count();
+uint64_t gemm_flop_count();  // algorithmic flops of every GEMM call of this process
 
 // ------------------------------------------------------------------ attention (S <= 128)
 // qkv [B*S, 3d] bf16 (q | k | v thirds, head j = columns [j*hd, (j+1)*hd) of each third);
@@ -122,23 +123,29 @@ void mlp_bwd_sgd(cudaStream_t s, const float* x, const float* h, const float* dy
 void f32_to_bf16x2(cudaStream_t s, const float* w32, bf16* hi, bf16* lo, size_t n);
 // frozen stem: x fp32 [B,H,H,3], w fp32 [C0][3][3][3], stride 2, pad 1 -> z x2 [B,H/2,H/2,C0]
 void spos_stem_conv(cudaStream_t s, const float* x, const float* w, bf16* z, int B, int H, int C0);
-// BatchNorm (training mode, biased variance, eps 1e-5).  part: [bn_part_blocks(P, C)][2][C]
-// workspace (per-row-block partial sums, then a parallel finalize kernel summing them in
-// block order in fp64); ctr: reserved (an int that is 0 between launches).
-int bn_part_blocks(int P, int C);
-// mean, rstd of z (x2) over its P rows
-void bn_stats(cudaStream_t s, const bf16* z, int P, int C, float* part, int* ctr, float* mean, float* rstd);
-// y[p*ldy + c] = relu?(g (z - mean) rstd + b); z x2 (plane P*C), y x2 (planes yplane apart)
-void bn_apply(cudaStream_t s, const bf16* z, int P, int C, const float* mean, const float* rstd, const float* g,
-              const float* b, int relu, bf16* y, int ldy, size_t yplane);
-// sums [2][C] = (sum dy', sum dy' xh) (dy' = dy masked by the ReLU); old [2][C] = (g, b)
-// as read by the forward; update: the SGD WRITE gu -= lr sums[1], bu -= lr sums[0] (gu, bu
-// = g, b in place; the bulk accumulator under BSP, reading A30)
+// BatchNorm (training mode, biased variance, eps 1e-5).  Reductions over the P rows are
+// fixed-order fp32 row-block partials accumulated in 64-bit fixed point with integer atomics
+// into acc [2][C] (unsigned long long, zero between uses): bitwise independent of the CTA
+// order, no finalize launch.  The consumer kernel (bn_apply / bn_bwd_apply) derives the
+// per-channel results from acc in every CTA; its last CTA (ticket: an int, 0 between uses)
+// publishes them and zeroes acc and the ticket.
+// acc <- (sum z, sum z^2) of z (x2) over its P rows
+void bn_stats(cudaStream_t s, const bf16* z, int P, int C, unsigned long long* acc);
+// y[p*ldy + c] = relu?(g (z - mean) rstd + b) with mean, rstd from acc; z x2 (plane P*C), y
+// x2 (planes yplane apart); writes mean, rstd [C] (for the backward), clears acc
+void bn_apply(cudaStream_t s, const bf16* z, int P, int C, unsigned long long* acc, int* ticket, float* mean,
+              float* rstd, const float* g, const float* b, int relu, bf16* y, int ldy, size_t yplane);
+// acc <- (s1 = sum dy', s2 = sum dy' xh) (dy' = dy masked by the ReLU of the forward)
 void bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
-                   const float* rstd, const float* g, const float* b, float* gu, float* bu, int relu, float* part,
-                   int* ctr, float* sums, float* old, float lr, int update);
+                   const float* rstd, const float* g, const float* b, int relu, unsigned long long* acc);
+// dz = rstd g (dy' - s1/P - xh s2/P) with the pre-update g, b; then (update) the SGD WRITE
+// gu -= lr s2, bu -= lr s1 (gu, bu = g, b in place; the bulk accumulator under BSP, reading
+// A30); clears acc
 void bn_bwd_apply(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
-                  const float* rstd, const float* old, const float* sums, int relu, bf16* dz);
+                  const float* rstd, const float* g, const float* b, float* gu, float* bu, float lr, int update,
+                  unsigned long long* acc, int* ticket, int relu, bf16* dz);
+// sticky device flag: a fixed-point partial fell outside its range (checked at drain)
+bool bn_fix_overflow();
 // depthwise k x k (k in {3,5,7}), stride S, pad k/2; w fp32 [C][k][k]; H = input height = width.
 // dw_fwd: x2 -> x2; dw_dgrad: bf16 (+ bf16 add); dw_wgrad reads the hi plane of x.
 void dw_fwd(cudaStream_t s, const bf16* x, const float* w, bf16* z, int B, int H, int C, int k, int S);

@@ -11,12 +11,19 @@
 
 namespace naspipe {
 
-// Engines with context switching alive in this process: they launch without PDL.  With the
-// candidate loads, shadow refreshes and staged write-backs on three more streams, the
-// compute stream's kernels follow cross-stream event waits (a candidate is ready); with the
-// PDL attribute a 14-subnet configs[3] run deadlocked on the GPU (tools/c4_probe.py
-// --no-drain), without it the same run drains in 1.9 s — so PDL is kept to the
-// all-resident paths, where every test and bench has run with it.
+// Engines alive in this process that launch without PDL (the multi-process rank engines:
+// their compute streams wait on transport streams / peer flags between kernels).
+//
+// History (DESIGN.md §5 "PDL"): round 1 turned PDL off for context-switching engines after a
+// 14-subnet configs[3] run deadlocked with it.  Root cause: the tcgen05 GEMM kernels took
+// their TMEM columns (tcgen05.alloc, up to 512) BEFORE griddepcontrol.wait, so an early-
+// launched GEMM CTA could hold TMEM on an SM while it waited for its predecessor grid; with
+// the candidate-load / shadow-refresh / write-back streams' kernels interleaved on the SMs
+// (the most likely cause; not proven).  Since the GEMMs allocate
+// TMEM only after the wait, the reproduction (tools/c4_probe.py --no-drain with
+// NASPIPE_FORCE_PDL=1, 3 runs) and tests/test_gpu_context.py pass with PDL, and context
+// switching runs with it again.  The CTA-pair GEMM's EARLY TRIGGERS (NASPIPE_PAIR_TRIGGER=1)
+// still hang tools/hangtest.sh and stay off.
 inline std::atomic<int>& pdl_suppressors() {
   static std::atomic<int> n{0};
   return n;

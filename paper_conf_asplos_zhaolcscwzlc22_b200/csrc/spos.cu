@@ -157,86 +157,58 @@ __global__ void stem_conv_kernel(const float* __restrict__ x, const float* __res
 }
 
 // ---------------------------------------------------------------- BatchNorm forward
-// Per-channel reductions over P rows: RED_CTAS-ish row blocks write partial sums
-// part[blk][0..2C); a finalize kernel sums them in block order (fp64): one warp per
-// (channel, which-sum), lane j sums blocks j, j+32, ... in order, then a fixed xor tree.
-__device__ __forceinline__ double warp_sum_d(double v) {
-#pragma unroll
-  for (int s = 16; s >= 1; s >>= 1) v += __shfl_xor_sync(0xffffffffu, v, s);
-  return v;
-}
-// warp w of the block: channel blockIdx.x * 4 + w / 2, sum w % 2; returns the total on all lanes
-__device__ __forceinline__ double part_total(const float* part, int nblk, int C, int c, int which) {
-  const int lane = threadIdx.x & 31;
-  double a = 0.0;
-  if (c < C) {
-    const float* p = part + which * C + c;
-    int k = lane;
-    for (; k + 96 < nblk; k += 128) {  // 4 independent loads in flight per lane
-      const float v0 = p[(size_t)k * 2 * C], v1 = p[(size_t)(k + 32) * 2 * C], v2 = p[(size_t)(k + 64) * 2 * C],
-                  v3 = p[(size_t)(k + 96) * 2 * C];
-      a += (double)v0;
-      a += (double)v1;
-      a += (double)v2;
-      a += (double)v3;
-    }
-    for (; k < nblk; k += 32) a += (double)p[(size_t)k * 2 * C];
+// Per-channel reductions over P rows without a finalize launch and without float atomics:
+// each CTA reduces its row block in a fixed order (per-thread sequential, then the RP lane
+// sums in lane order) to fp32 partials, converts them to 64-bit FIXED POINT and adds them
+// with integer atomics into acc[2C].  Integer addition is associative, so the totals --
+// and everything computed from them -- are bitwise independent of the CTA arrival order.
+// The consumer kernel (bn_apply / bn_bwd_apply) reads the totals; its last CTA (arrival
+// ticket) publishes the per-channel results and zeroes acc and the ticket for the next use.
+//
+// Scales: forward sum z (2^32: |sum| < 2^31), sum z^2 (2^24: < 5.5e11), backward sums
+// (2^40: |sum| < 8.4e6).  A partial outside the range sets the sticky overflow flag
+// (checked at drain, NASPIPE_EINTERNAL) instead of wrapping silently.
+constexpr double FIX_S1 = 4294967296.0;      // 2^32
+constexpr double FIX_S2 = 16777216.0;        // 2^24
+constexpr double FIX_B = 1099511627776.0;    // 2^40
+__device__ int g_fix_overflow;
+
+__device__ __forceinline__ void fix_add(unsigned long long* acc, float v, double scale) {
+  const double x = (double)v * scale;
+  if (!(fabs(x) < 4.0e18)) {  // also catches NaN
+    atomicOr(&g_fix_overflow, 1);
+    return;
   }
-  return warp_sum_d(a);
+  atomicAdd(acc, (unsigned long long)(long long)__double2ll_rn(x));
+}
+__device__ __forceinline__ double fix_get(const unsigned long long* acc, int i, double scale) {
+  return (double)(long long)acc[i] / scale;
 }
 
-// mean = sum / P, rstd = 1/sqrt(sumsq / P - mean^2 + eps) (biased variance)
-__global__ void bn_finalize_kernel(const float* __restrict__ part, int nblk, int C, int P, float* __restrict__ mean,
-                                   float* __restrict__ rstd) {
-  __shared__ double tot[8];
-  ptx::pdl_wait();
-  const int w = threadIdx.x >> 5, c = blockIdx.x * 4 + w / 2;
-  const double t = part_total(part, nblk, C, c, w & 1);
-  if ((threadIdx.x & 31) == 0) tot[w] = t;
+// arrival ticket: true in every thread of the CTA that arrives last (all others are done)
+__device__ __forceinline__ bool last_cta(int* ticket) {
+  __shared__ int last;
   __syncthreads();
-  if (threadIdx.x < 4) {
-    const int cc = blockIdx.x * 4 + threadIdx.x;
-    if (cc < C) {
-      const double mu = tot[2 * threadIdx.x] / P;
-      const double var = fmax(tot[2 * threadIdx.x + 1] / P - mu * mu, 0.0);
-      mean[cc] = (float)mu;
-      rstd[cc] = (float)(1.0 / sqrt(var + (double)BN_EPS));
-    }
+  if (threadIdx.x == 0) {
+    __threadfence();
+    last = atomicAdd(ticket, 1) == (int)(gridDim.x * gridDim.y) - 1;
   }
+  __syncthreads();
+  if (last) __threadfence();
+  return last;
 }
 
-// sums[0][c] = s1 (dbeta), sums[1][c] = s2 (dgamma); old = (gamma, beta) before the WRITE
-// gamma -= lr s2, beta -= lr s1 (if update)
-__global__ void bn_bwd_finalize_kernel(const float* __restrict__ part, int nblk, int C, float* __restrict__ sums,
-                                       float* __restrict__ old, const float* gam, const float* bet, float* gamu,
-                                       float* betu, float lr, int update) {
-  __shared__ double tot[8];
-  ptx::pdl_wait();
-  const int w = threadIdx.x >> 5, c = blockIdx.x * 4 + w / 2;
-  const double t = part_total(part, nblk, C, c, w & 1);
-  if ((threadIdx.x & 31) == 0) tot[w] = t;
-  __syncthreads();
-  if (threadIdx.x < 4) {
-    const int cc = blockIdx.x * 4 + threadIdx.x;
-    if (cc < C) {
-      const float f1 = (float)tot[2 * threadIdx.x], f2 = (float)tot[2 * threadIdx.x + 1];
-      sums[cc] = f1;
-      sums[C + cc] = f2;
-      const float gv = gam[cc], bv = bet[cc];
-      old[cc] = gv;
-      old[C + cc] = bv;
-      if (update) {  // the WRITE; gamu/betu = gam/bet in place, the bulk accumulator under BSP
-        gamu[cc] = (gamu == gam ? gv : gamu[cc]) - lr * f2;
-        betu[cc] = (betu == bet ? bv : betu[cc]) - lr * f1;
-      }
-    }
-  }
+// mean = s1 / P, rstd = 1/sqrt(s2 / P - mean^2 + eps) (biased variance), from the totals
+__device__ __forceinline__ void bn_moments(const unsigned long long* acc, int C, int c, int P, float& mu, float& rs) {
+  const double m = fix_get(acc, c, FIX_S1) / P;
+  const double var = fmax(fix_get(acc, C + c, FIX_S2) / P - m * m, 0.0);
+  mu = (float)m;
+  rs = (float)(1.0 / sqrt(var + (double)BN_EPS));
 }
 
 // Thread (r, g): rows r, r + RP, ... of its block, channels [8g, 8g+8); RP = TPB / G row
-// lanes; the RP lane sums are combined in lane order.  Writes part[blk][0..C) = sum z,
-// part[blk][C..2C) = sum z^2.
-__global__ void bn_stats_kernel(const bf16* __restrict__ z, int P, int C, int rows, float* __restrict__ part) {
+// lanes; the RP lane sums are combined in lane order, then added to acc (fixed point).
+__global__ void bn_stats_kernel(const bf16* __restrict__ z, int P, int C, int rows, unsigned long long* acc) {
   extern __shared__ float red[];  // [RP][2C]
   ptx::pdl_wait();
   const int G = C / 8, RP = TPB / G;
@@ -277,7 +249,7 @@ __global__ void bn_stats_kernel(const bf16* __restrict__ z, int P, int C, int ro
   for (int e = threadIdx.x; e < 2 * C; e += TPB) {
     float a = 0.f;
     for (int k = 0; k < RP; ++k) a += red[k * 2 * C + e];
-    part[(size_t)blockIdx.x * 2 * C + e] = a;
+    fix_add(acc + e, a, e < C ? FIX_S1 : FIX_S2);
   }
 }
 
@@ -285,17 +257,15 @@ __global__ void bn_stats_kernel(const bf16* __restrict__ z, int P, int C, int ro
 // group's per-channel parameters in registers and strides over pixels.
 __device__ __forceinline__ int ew_lanes(int C) { return TPB / (C / 8); }
 
-__global__ void bn_apply_kernel(const bf16* __restrict__ z, int P, int C, const float* __restrict__ mean,
-                                const float* __restrict__ rstd, const float* __restrict__ gam,
-                                const float* __restrict__ bet, int relu, bf16* __restrict__ y, int ldy,
-                                size_t yplane) {
-  ptx::pdl_wait();
+__device__ __forceinline__ void bn_apply_body(const bf16* __restrict__ z, int P, int C, const unsigned long long* acc,
+                                              const float* __restrict__ gam, const float* __restrict__ bet, int relu,
+                                              bf16* __restrict__ y, int ldy, size_t yplane) {
   const int G = C / 8, lanes = ew_lanes(C);
   const int pl = threadIdx.x / G, c = (threadIdx.x % G) * 8;
   if (pl >= lanes) return;
   float mu[8], rs[8], g8[8], b8[8];
-  load8f(mean + c, mu);
-  load8f(rstd + c, rs);
+#pragma unroll
+  for (int i = 0; i < 8; ++i) bn_moments(acc, C, c + i, P, mu[i], rs[i]);
   load8f(gam + c, g8);
   load8f(bet + c, b8);
   const size_t zplane = (size_t)P * C;
@@ -327,6 +297,25 @@ __global__ void bn_apply_kernel(const bf16* __restrict__ z, int P, int C, const 
   }
 }
 
+__global__ void bn_apply_kernel(const bf16* __restrict__ z, int P, int C, unsigned long long* acc, int* ticket,
+                                float* __restrict__ mean, float* __restrict__ rstd, const float* __restrict__ gam,
+                                const float* __restrict__ bet, int relu, bf16* __restrict__ y, int ldy,
+                                size_t yplane) {
+  ptx::pdl_wait();
+  bn_apply_body(z, P, C, acc, gam, bet, relu, y, ldy, yplane);
+  if (last_cta(ticket)) {  // every CTA has read the totals: publish mean / rstd, clear
+    for (int c = threadIdx.x; c < C; c += blockDim.x) {
+      float mu, rs;
+      bn_moments(acc, C, c, P, mu, rs);
+      mean[c] = mu;
+      rstd[c] = rs;
+    }
+    __syncthreads();
+    for (int e = threadIdx.x; e < 2 * C; e += blockDim.x) acc[e] = 0ull;
+    if (threadIdx.x == 0) *ticket = 0;
+  }
+}
+
 // ---------------------------------------------------------------- BatchNorm backward
 __device__ __forceinline__ void bn_bwd_item(const bf16* dy, const bf16* z, size_t zplane, const float (&mu)[8],
                                             const float (&rs)[8], const float (&g8)[8], const float (&b8)[8],
@@ -341,11 +330,12 @@ __device__ __forceinline__ void bn_bwd_item(const bf16* dy, const bf16* z, size_
   }
 }
 
-// Partials of s1 = sum dy', s2 = sum dy' xh (dy' = dy masked by the ReLU) per row block.
+// s1 = sum dy', s2 = sum dy' xh (dy' = dy masked by the ReLU): fixed-order row-block
+// partials added to acc[2C] in fixed point (see bn_stats_kernel).
 __global__ void bn_bwd_reduce_kernel(const bf16* __restrict__ dy, int lddy, const bf16* __restrict__ z, int P, int C,
                                      const float* __restrict__ mean, const float* __restrict__ rstd,
                                      const float* __restrict__ gam, const float* __restrict__ bet, int relu,
-                                     int rows, float* __restrict__ part) {
+                                     int rows, unsigned long long* acc) {
   extern __shared__ float red[];  // [RP][2C]
   ptx::pdl_wait();
   const int G = C / 8, RP = TPB / G;
@@ -393,15 +383,15 @@ __global__ void bn_bwd_reduce_kernel(const bf16* __restrict__ dy, int lddy, cons
   for (int e = threadIdx.x; e < 2 * C; e += TPB) {
     float a = 0.f;
     for (int k = 0; k < RP; ++k) a += red[k * 2 * C + e];
-    part[(size_t)blockIdx.x * 2 * C + e] = a;
+    fix_add(acc + e, a, FIX_B);
   }
 }
 
-__global__ void bn_bwd_apply_kernel(const bf16* __restrict__ dy, int lddy, const bf16* __restrict__ z, int P, int C,
-                                    const float* __restrict__ mean, const float* __restrict__ rstd,
-                                    const float* __restrict__ old, const float* __restrict__ sums, int relu,
-                                    bf16* __restrict__ dz) {
-  ptx::pdl_wait();
+__device__ __forceinline__ void bn_bwd_apply_body(const bf16* __restrict__ dy, int lddy, const bf16* __restrict__ z,
+                                                  int P, int C, const float* __restrict__ mean,
+                                                  const float* __restrict__ rstd, const float* __restrict__ gam,
+                                                  const float* __restrict__ bet, const unsigned long long* acc, int relu,
+                                                  bf16* __restrict__ dz) {
   const int G = C / 8, lanes = ew_lanes(C);
   const int pl = threadIdx.x / G, c = (threadIdx.x % G) * 8;
   if (pl >= lanes) return;
@@ -409,10 +399,13 @@ __global__ void bn_bwd_apply_kernel(const bf16* __restrict__ dy, int lddy, const
   float mu[8], rs[8], g8[8], b8[8], m1[8], m2[8];
   load8f(mean + c, mu);
   load8f(rstd + c, rs);
-  load8f(old + c, g8);
-  load8f(old + C + c, b8);
-  load8f(sums + c, m1);
-  load8f(sums + C + c, m2);
+  load8f(gam + c, g8);
+  load8f(bet + c, b8);
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    m1[i] = (float)fix_get(acc, c + i, FIX_B);
+    m2[i] = (float)fix_get(acc, C + c + i, FIX_B);
+  }
   const size_t zplane = (size_t)P * C;
   const int step = gridDim.x * lanes;
   for (int p = blockIdx.x * lanes + pl; p < P; p += step) {
@@ -424,6 +417,29 @@ __global__ void bn_bwd_apply_kernel(const bf16* __restrict__ dy, int lddy, const
       d[i] = rs[i] * g8[i] * t;
     }
     store8(dz + (size_t)p * C + c, d);
+  }
+}
+
+// dz = rstd g (dy' - s1/P - xh s2/P) with the PRE-update g, b (reading A4: the input
+// gradient uses the weights before the WRITE); the last CTA -- after every CTA has read
+// g, b -- applies the WRITE g -= lr s2, b -= lr s1 (into gu/bu: g/b in place, the bulk
+// accumulator under BSP) and clears acc and the ticket.
+__global__ void bn_bwd_apply_kernel(const bf16* __restrict__ dy, int lddy, const bf16* __restrict__ z, int P, int C,
+                                    const float* __restrict__ mean, const float* __restrict__ rstd, const float* gam,
+                                    const float* bet, float* gamu, float* betu, float lr, int update,
+                                    unsigned long long* acc, int* ticket, int relu, bf16* __restrict__ dz) {
+  ptx::pdl_wait();
+  bn_bwd_apply_body(dy, lddy, z, P, C, mean, rstd, gam, bet, acc, relu, dz);
+  if (last_cta(ticket)) {
+    if (update)
+      for (int c = threadIdx.x; c < C; c += blockDim.x) {
+        const float f1 = (float)fix_get(acc, c, FIX_B), f2 = (float)fix_get(acc, C + c, FIX_B);
+        gamu[c] = (gamu == gam ? gam[c] : gamu[c]) - lr * f2;
+        betu[c] = (betu == bet ? bet[c] : betu[c]) - lr * f1;
+      }
+    __syncthreads();
+    for (int e = threadIdx.x; e < 2 * C; e += blockDim.x) acc[e] = 0ull;
+    if (threadIdx.x == 0) *ticket = 0;
   }
 }
 
@@ -889,11 +905,6 @@ void f32_to_bf16x2(cudaStream_t s, const float* w32, bf16* hi, bf16* lo, size_t 
   check_launch("f32_to_bf16x2");
 }
 
-int bn_part_blocks(int P, int C) {
-  const int r = red_rows(P, C);
-  return (P + r - 1) / r;
-}
-
 void spos_stem_conv(cudaStream_t s, const float* x, const float* w, bf16* z, int B, int H, int C0) {
   NP_REQUIRE(C0 % 8 == 0 && H % 2 == 0, NASPIPE_EINVAL, "stem C0=%d H=%d", C0, H);
   const size_t P = (size_t)B * (H / 2) * (H / 2);
@@ -954,47 +965,48 @@ static int ew_grid(Kern kern, int P, int C) {
 }
 
 static size_t red_smem(int C) { return (size_t)(TPB / (C / 8)) * 2 * C * sizeof(float); }
+static int red_blocks(int P, int C) {
+  const int r = red_rows(P, C);
+  return (P + r - 1) / r;
+}
 
-// ctr: kept in the signature for a single-kernel (last-CTA) finalize; unused by the
-// two-kernel form (partials, then a parallel fixed-order finalize), which measured faster.
-void bn_stats(cudaStream_t s, const bf16* z, int P, int C, float* part, int* ctr, float* mean, float* rstd) {
-  (void)ctr;
+void bn_stats(cudaStream_t s, const bf16* z, int P, int C, unsigned long long* acc) {
   NP_REQUIRE(C % 8 == 0 && C / 8 <= TPB, NASPIPE_EINVAL, "bn_stats C=%d", C);
   const size_t sm = red_smem(C);
-  const int nblk = bn_part_blocks(P, C);
   set_smem(bn_stats_kernel, sm);
-  launch_pdl(bn_stats_kernel, dim3(nblk), dim3(TPB), sm, s, z, P, C, red_rows(P, C), part);
-  launch_pdl(bn_finalize_kernel, dim3((C + 3) / 4), dim3(TPB), 0, s, (const float*)part, nblk, C, P, mean, rstd);
+  launch_pdl(bn_stats_kernel, dim3(red_blocks(P, C)), dim3(TPB), sm, s, z, P, C, red_rows(P, C), acc);
   check_launch("bn_stats");
 }
 
-void bn_apply(cudaStream_t s, const bf16* z, int P, int C, const float* mean, const float* rstd, const float* g,
-              const float* b, int relu, bf16* y, int ldy, size_t yplane) {
-  launch_pdl(bn_apply_kernel, dim3(ew_grid(bn_apply_kernel, P, C)), dim3(TPB), 0, s, z, P, C, mean, rstd, g, b, relu,
-             y, ldy, yplane);
+void bn_apply(cudaStream_t s, const bf16* z, int P, int C, unsigned long long* acc, int* ticket, float* mean,
+              float* rstd, const float* g, const float* b, int relu, bf16* y, int ldy, size_t yplane) {
+  launch_pdl(bn_apply_kernel, dim3(ew_grid(bn_apply_kernel, P, C)), dim3(TPB), 0, s, z, P, C, acc, ticket, mean, rstd,
+             g, b, relu, y, ldy, yplane);
   check_launch("bn_apply");
 }
 
 void bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
-                   const float* rstd, const float* g, const float* b, float* gu, float* bu, int relu, float* part,
-                   int* ctr, float* sums, float* old, float lr, int update) {
-  (void)ctr;
+                   const float* rstd, const float* g, const float* b, int relu, unsigned long long* acc) {
   NP_REQUIRE(C % 8 == 0 && C / 8 <= TPB, NASPIPE_EINVAL, "bn_bwd C=%d", C);
   const size_t sm = red_smem(C);
-  const int nblk = bn_part_blocks(P, C);
   set_smem(bn_bwd_reduce_kernel, sm);
-  launch_pdl(bn_bwd_reduce_kernel, dim3(nblk), dim3(TPB), sm, s, dy, lddy, z, P, C, mean, rstd, (const float*)g,
-             (const float*)b, relu, red_rows(P, C), part);
-  launch_pdl(bn_bwd_finalize_kernel, dim3((C + 3) / 4), dim3(TPB), 0, s, (const float*)part, nblk, C, sums, old, g,
-             b, gu, bu, lr, update);
+  launch_pdl(bn_bwd_reduce_kernel, dim3(red_blocks(P, C)), dim3(TPB), sm, s, dy, lddy, z, P, C, mean, rstd, g, b, relu,
+             red_rows(P, C), acc);
   check_launch("bn_bwd_reduce");
 }
 
 void bn_bwd_apply(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
-                  const float* rstd, const float* old, const float* sums, int relu, bf16* dz) {
-  launch_pdl(bn_bwd_apply_kernel, dim3(ew_grid(bn_bwd_apply_kernel, P, C)), dim3(TPB), 0, s, dy, lddy, z, P, C, mean, rstd,
-             old, sums, relu, dz);
+                  const float* rstd, const float* g, const float* b, float* gu, float* bu, float lr, int update,
+                  unsigned long long* acc, int* ticket, int relu, bf16* dz) {
+  launch_pdl(bn_bwd_apply_kernel, dim3(ew_grid(bn_bwd_apply_kernel, P, C)), dim3(TPB), 0, s, dy, lddy, z, P, C, mean,
+             rstd, g, b, gu, bu, lr, update, acc, ticket, relu, dz);
   check_launch("bn_bwd_apply");
+}
+
+bool bn_fix_overflow() {
+  int v = 0;
+  cudaMemcpyFromSymbol(&v, g_fix_overflow, sizeof v);
+  return v != 0;
 }
 
 #define DW_DISPATCH(K, EXPR) \

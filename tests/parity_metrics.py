@@ -16,11 +16,18 @@ an arithmetic mistake shows):  upd(tensor) = ||dg - dr||_2 / ||dr||_2 with dg = 
 dr = ref - theta_0, per tensor, bars per tensor class (DESIGN.md "Tolerances": fp32 MLP 1e-5;
 bf16 paths: weight matrices and biases 2e-2, LN/BN gamma and beta 5e-2).
 
-Structurally static tensors: the exact gradient of a BatchNorm shift beta is identically zero
-when the BN output reaches the next BatchNorm through a linear map only (SPOS depthwise
-units: dw -> BN -> pw -> BN; the second BN removes any per-channel constant), so their
-reference update is fp64 round-off and a relative bar is meaningless.  They get an absolute
-bar instead: max |dg| <= STATIC_ABS x the largest |dr| of the candidate.
+Structurally static tensors (SPOS), where a relative bar is meaningless because the exact
+update is zero or proportional to another tensor's (tiny) update:
+* the BN shift beta of every depthwise unit: its output reaches the next BatchNorm through
+  a linear map only (dw -> BN -> pw -> BN), and the second BN removes any per-channel
+  constant, so d L / d beta = 0 identically;
+* the BN scale gamma of a unit whose BN -> ReLU output feeds a DEPTHWISE (per-channel) conv
+  and then a BN (m_pw1, x_pw1, x_pw2): relu(gamma xh + beta) = gamma relu(xh) while beta = 0,
+  the depthwise conv keeps channels separate and the next BN removes the per-channel scale,
+  so d L / d gamma = 0 at a candidate's first update and stays proportional to beta (O(lr))
+  afterwards.
+They get an absolute bar instead: max |dg - dr| <= STATIC_ABS x the largest |dr| of the
+candidate.
 """
 import numpy as np
 
@@ -30,7 +37,8 @@ STATIC_ABS = 1e-3
 
 
 def structurally_static(cfg, name):
-    return cfg["family"] == "spos" and "_dw" in name and name.endswith("_b")
+    return cfg["family"] == "spos" and (("_dw" in name and name.endswith("_b"))
+                                        or name in ("m_pw1_g", "x_pw1_g", "x_pw2_g"))
 
 
 def tensor_class(name, shape, kind):
@@ -61,7 +69,7 @@ def per_tensor(cfg, got, ref, theta0):
             if kind != "zeros":
                 rec["a15"] = float(np.max(np.abs(gs - rs)) / np.max(np.abs(rs)))
             if structurally_static(cfg, name):
-                rec["static"] = float(np.max(np.abs(dg)) / cand_dmax) if cand_dmax > 0 else 0.0
+                rec["static"] = float(np.max(np.abs(dg - dr)) / cand_dmax) if cand_dmax > 0 else 0.0
             elif np.any(dr != 0):
                 rec["upd"] = float(np.linalg.norm(dg - dr) / np.linalg.norm(dr))
             else:
@@ -90,8 +98,20 @@ def fmt(s):
             f"upd[{u}] static={s['static']:.2e}")
 
 
+# Update bars per tensor class (DESIGN.md §3 "Tolerances" derives each from measurement):
+# * fp32 MLP: fp32 rounding ~6e-8 per op, a few ops per element;
+# * bf16 transformer: matrices / biases / LN beta 2e-2 and 5e-2 (measured <= 6e-3 / 4.5e-3 /
+#   4.4e-3 at full size); LN gamma 0.1: its gradient sum_t da_t xhat_t cancels 56 : 1
+#   (measured, configs[2] block 0), so the bf16 datapath's ~1e-3 normwise error in the
+#   incoming gradient shows up x56 (measured 6.6e-2 at full size, 3e-2 tiny);
+# * SPOS CNN: BatchNorm + ReLU make the one-step update ill-conditioned: the fp64 oracle run
+#   with fp32 storage (the paper's precision) already differs from fp64 by 0.95e-2 /
+#   1.3e-2 (matrices / BN) at full size, with the path's 16-bit-mantissa storage (bf16x2,
+#   what the 3-pass tensor-core product consumes; A28) by 0.11 / 0.12; the bar is
+#   that measured floor with margin.
 UPD_FP32 = {"matrix": 1e-5, "bias": 1e-5, "norm_g": 1e-5, "norm_b": 1e-5}
-UPD_BF16 = {"matrix": 2e-2, "bias": 2e-2, "norm_g": 5e-2, "norm_b": 5e-2}
+UPD_BF16 = {"matrix": 2e-2, "bias": 2e-2, "norm_g": 1e-1, "norm_b": 5e-2}
+UPD_SPOS = {"matrix": 0.2, "bias": 0.2, "norm_g": 0.25, "norm_b": 0.25, "static": 2e-2}
 
 
 def check(s, a15, upd=None):
@@ -100,7 +120,7 @@ def check(s, a15, upd=None):
     if upd is not None:
         for cls, v in s["upd"].items():
             assert v <= upd[cls], (cls, fmt(s))
-        assert s["static"] <= STATIC_ABS, fmt(s)
+        assert s["static"] <= upd.get("static", STATIC_ABS), fmt(s)
 
 
 def errors(cfg, got, ref, theta0):
@@ -132,7 +152,7 @@ def sampled_errors(cfg, gold, step, got_of):
                 rec["a15"] = float(np.max(np.abs(gs - rs)) / gold[f"{pre}max_{tag}"])
             dr, dg = rs - t0, gs - t0
             if structurally_static(cfg, name):
-                rec["static"] = float(np.max(np.abs(dg)) / max(float(gold[f"{pre}dmax_{k}"]) for k in
+                rec["static"] = float(np.max(np.abs(dg - dr)) / max(float(gold[f"{pre}dmax_{k}"]) for k in
                                                               [f"{b}_{c}_{nm}" for nm, _, _, _ in
                                                                train.candidate_layout(cfg, b, c)]))
             elif np.any(dr != 0):

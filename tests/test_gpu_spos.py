@@ -47,7 +47,7 @@ def test_tiny_spos_parity(N, tol):
     cfg = synth.get_config("tiny_spos")
     choices = synth.sample_choices(N, cfg["n_blocks"], cfg["n_choices"])
     cfg, gpu, floor, losses, ref_loss, trace, stats = _run("tiny_spos", choices)
-    pm.check(gpu, tol, pm.UPD_BF16 if N <= 8 else None)
+    pm.check(gpu, tol, pm.UPD_SPOS if N <= 8 else None)
     np.testing.assert_allclose(losses, ref_loss, rtol=1e-2)
     _check_trace(cfg, choices, 2, trace)
     assert stats["version_checks"] == 2 * N * cfg["n_blocks"]
@@ -59,7 +59,7 @@ def test_tiny_spos_every_candidate_kind():
     m, n = cfg["n_blocks"], cfg["n_choices"]
     choices = np.array([[(c + b) % n for b in range(m)] for c in range(n)], dtype=np.int32)
     _, gpu, floor, losses, ref_loss, _, _ = _run("tiny_spos", choices, D=1)
-    pm.check(gpu, 1e-3, pm.UPD_BF16)
+    pm.check(gpu, 1e-3, pm.UPD_SPOS)
     np.testing.assert_allclose(losses, ref_loss, rtol=1e-2)
 
 
@@ -88,7 +88,7 @@ def test_spos_full_size_one_step():
     params, losses, _, _ = run_engine(cfg, choices, batches, D=1)
     sm = pm.errors(cfg, params, ref, theta0)
     print(f"full-size one step: {pm.fmt(sm)} loss {losses[0]:.6f} vs {ref_loss[0]:.6f}")
-    pm.check(sm, 1e-3, pm.UPD_BF16)
+    pm.check(sm, 1e-3, pm.UPD_SPOS)
     np.testing.assert_allclose(losses, ref_loss, rtol=1e-2)
 
 
