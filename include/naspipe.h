@@ -74,8 +74,12 @@ typedef enum { NASPIPE_MLP = 0, NASPIPE_TRANSFORMER = 1, NASPIPE_SPOS_CNN = 2 } 
  *            bulk reads the bulk-start weights, the SGD WRITEs accumulate into a per-
  *            candidate fp32 copy, copied back into the masters at the flush (= the bulk's
  *            gradients, summed, applied once).  Executable with every candidate resident
- *            (naspipe_create: EINVAL with hbm_weight_budget_bytes > 0). */
-typedef enum { NASPIPE_SYNC_CSP = 0, NASPIPE_SYNC_INORDER = 1, NASPIPE_SYNC_ASP = 2, NASPIPE_SYNC_BSP = 3 } naspipe_sync;
+ *            (naspipe_create: EINVAL with hbm_weight_budget_bytes > 0).
+ *   SERIAL   "NASPipe w/o scheduler" as P:L454 words it: it "had to finish the execution of a
+ *            pipeline before injecting the next pipeline" -- one subnet in flight at a time
+ *            (the window forced to W = 1; reading A32).  Numerics = CSP. */
+typedef enum { NASPIPE_SYNC_CSP = 0, NASPIPE_SYNC_INORDER = 1, NASPIPE_SYNC_ASP = 2, NASPIPE_SYNC_BSP = 3,
+               NASPIPE_SYNC_SERIAL = 4 } naspipe_sync;
 typedef enum { NASPIPE_FP32 = 0, NASPIPE_BF16 = 1 } naspipe_dtype; /* compute dtype; masters fp32 */
 
 /* spec.flags */

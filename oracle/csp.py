@@ -125,7 +125,10 @@ def simulate_csp(choices, stage_of_block, D, W, cf, cb, lam=0, policy=0, ignore_
     dependency-table admission rule (used to cross-check against Algorithm 2 verbatim).
 
     ``sync`` (include/naspipe.h naspipe_sync) changes only the admission:
-    "csp" the method; "inorder" NASPipe w/o scheduler (Fig.6): only the lowest-id
+    "csp" the method; "serial" NASPipe w/o scheduler as P:L454 words it ("had to finish the
+    execution of a pipeline before injecting the next pipeline"): the window forced to
+    W = 1, one subnet in flight; "inorder" the in-order-admission variant of the ablation
+    (Fig.6): only the lowest-id
     queued forward may start, a blocked head blocks the stage; "asp" (PipeDream-style,
     P:L123) dependencies ignored; "bsp" (GPipe/Retiarii): dependencies ignored inside
     bulks of ``bulk`` consecutive subnets (0 = 4 D), a stage runs any queued forward before
@@ -136,6 +139,8 @@ def simulate_csp(choices, stage_of_block, D, W, cf, cb, lam=0, policy=0, ignore_
     stage's queued forwards and finished set just before it (an observer: no effect)."""
     N = len(choices)
     G = bulk if bulk > 0 else 4 * D
+    if sync == "serial":   # "w/o scheduler" as P:L454 words it: one pipeline (subnet) at a time (A32)
+        W = 1
     no_deps = ignore_deps or sync in ("asp", "bsp")
     dep_sets = [[set() if no_deps else deps(choices, stage_of_block, y, K)
                  for y in range(N)] for K in range(D)]

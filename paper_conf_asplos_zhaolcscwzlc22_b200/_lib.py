@@ -11,7 +11,7 @@ if not os.path.exists(LIB_PATH):
 lib = C.CDLL(LIB_PATH)
 
 ABI_VERSION = 3
-SYNC = {"csp": 0, "inorder": 1, "asp": 2, "bsp": 3}  # naspipe_sync (include/naspipe.h)
+SYNC = {"csp": 0, "inorder": 1, "asp": 2, "bsp": 3, "serial": 4}  # naspipe_sync (include/naspipe.h)
 FAMILY = {"mlp": 0, "transformer": 1, "spos": 2}
 DTYPE = {"fp32": 0, "bf16": 1}
 BATCH_HOST, BATCH_DEVICE, BATCH_SYNTHETIC = 0, 1, 2

@@ -16,11 +16,10 @@ namespace {
 // rows per block in colsum partials (a function of the process environment only, so the
 // partial count is fixed per run: NASPIPE_CS_ROWS overrides it for tuning)
 static int cs_rows() {
-  static int v = 0;
-  if (!v) {
+  static const int v = [] {  // thread-safe one-time init
     const char* e = getenv("NASPIPE_CS_ROWS");
-    v = e ? std::max(8, atoi(e)) : 16;
-  }
+    return e ? std::max(8, atoi(e)) : 16;
+  }();
   return v;
 }
 

@@ -100,6 +100,7 @@ Engine::Engine(const Spec& spec, int D) : spec_(spec), D_(D), W_(slot_count(spec
              "BSP runs with every candidate resident (hbm_weight_budget_bytes = 0)");
   version_.assign((size_t)spec_.m() * spec_.n(), 0);
   timer_.on = (spec_.raw.flags & NASPIPE_FLAG_TIMING) != 0;
+  if (spec_.raw.hbm_weight_budget_bytes > 0) suppress_pdl();  // context switching: no PDL (launch.h)
 }
 
 void Engine::suppress_pdl() {

@@ -98,11 +98,14 @@ class SposFamily : public Family {
     gb_[1] = A.alloc<bf16>(blk_max);
     gfirst_ = A.alloc<bf16>(g_max);
     // fixed-point BatchNorm accumulators + arrival tickets (zero between uses; spos.cu)
-    acc_f_ = A.alloc<unsigned long long>(2 * C_max);
-    acc_b_ = A.alloc<unsigned long long>(2 * C_max);
+    // per channel count C of a use, acc[2C] is that use's overflow flag: size 2 C_max + 1
+    // and zero everywhere, so every flag position starts (and, flags aside, stays) zero
+    acc_f_ = A.alloc<unsigned long long>(2 * C_max + 1);
+    acc_b_ = A.alloc<unsigned long long>(2 * C_max + 1);
     tick_ = A.alloc<int>(2);
-    cudaMemset(acc_f_, 0, 2 * C_max * 8);
-    cudaMemset(acc_b_, 0, 2 * C_max * 8);
+    cudaMemset(acc_f_, 0, (2 * C_max + 1) * 8);
+    cudaMemset(acc_b_, 0, (2 * C_max + 1) * 8);
+    C_max_ = (int)C_max;
     cudaMemset(tick_, 0, 2 * sizeof(int));
     dwpart_ = A.alloc<float>(std::max<size_t>(dwp_max, 1));
     ws_ = A.alloc<float>(std::max<size_t>(ws_elems_, 4));
@@ -228,8 +231,8 @@ class SposFamily : public Family {
     e.out = zh_;
     e.out2 = zh_ + (size_t)PL * Ch;
     const bf16* xo = static_cast<const bf16*>(out);
+    e.stats = acc_f_;  // fused bn_stats
     gemm_x2(s, PL, Ch, Cl, xo, xo + (size_t)PL * Cl, Cl, wh16_, wh16_ + (size_t)Ch * Cl, Cl, e);
-    t_bn_stats(s, zh_, PL, Ch, hmean_, hrstd_);
     t_bn_apply(s, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, 1, rh_, Ch, (size_t)PL * Ch);
     gap_pool(s, rh_, B_, HW, Ch, gap_);
     fc_ce(s, gap_, wf_, static_cast<const int*>(target), B_, Ch, ncls, logits_, dlogits_, loss_per_);
@@ -241,11 +244,17 @@ class SposFamily : public Family {
     e = GemmEpiParams();
     e.out = dy;
     gemm(s, PL, Cl, Ch, dzh_, false, Ch, wh16_, true, Cl, EPI_BF16, e);
-    counters.launches += 10;
+    counters.launches += 9;
   }
 
   void check_after_drain() override {
-    NP_REQUIRE(!bn_fix_overflow(), NASPIPE_EINTERNAL,
+    bool bad = false;  // a flag at acc[2C] of any use; the accumulators are zero elsewhere after a drain
+    std::vector<unsigned long long> h(2 * (size_t)C_max_ + 1);
+    for (const unsigned long long* a : {acc_f_, acc_b_}) {
+      cudaMemcpy(h.data(), a, h.size() * 8, cudaMemcpyDeviceToHost);
+      for (auto v : h) bad |= v != 0;
+    }
+    NP_REQUIRE(!bad, NASPIPE_EINTERNAL,
                "BatchNorm fixed-point accumulator overflow (a partial sum outside the 64-bit range, spos.cu)");
   }
 
@@ -340,16 +349,16 @@ class SposFamily : public Family {
       UnitRec r{h, cv, st, st + u.cout};
       cv += 2 * zplane;
       st += 2 * u.cout;
-      if (u.dw) {
-        dw_fwd(s, h, Pm + u.off_w, r.z, B_, u.H_in, u.cin, u.k, u.stride);
+      if (u.dw) {  // the depthwise conv adds the BatchNorm sums of its output itself (fused bn_stats)
+        dw_fwd(s, h, Pm + u.off_w, r.z, B_, u.H_in, u.cin, u.k, u.stride, acc_f_);
         counters.launches++;
       } else {
-        GemmEpiParams e;
+        GemmEpiParams e;  // the GEMM epilogue adds the BatchNorm sums of z (fused bn_stats)
         e.out = r.z;
         e.out2 = r.z + zplane;
+        e.stats = acc_f_;
         gemm_x2(s, Po, u.cout, u.cin, h, h + hplane, u.cin, W16 + u.off_w16, W16 + half + u.off_w16, u.cin, e);
       }
-      t_bn_stats(s, r.z, Po, u.cout, r.mean, r.rstd);
       bf16* y;
       int ldy;
       size_t yplane;
@@ -365,7 +374,7 @@ class SposFamily : public Family {
       }
       t_bn_apply(s, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, u.relu, y, ldy, yplane);
       hplane = yplane;
-      counters.launches += 2;
+      counters.launches += 1;
       recs.push_back(r);
       h = y;
     }
@@ -490,6 +499,7 @@ class SposFamily : public Family {
   float *dwpart_, *ws_;
   unsigned long long *acc_f_, *acc_b_;  // BatchNorm fixed-point accumulators (forward / backward)
   int* tick_;                           // [2] arrival tickets of bn_apply / bn_bwd_apply
+  int C_max_ = 0;
   size_t ws_elems_ = 0;
   // stem
   float* w_stem_ = nullptr;

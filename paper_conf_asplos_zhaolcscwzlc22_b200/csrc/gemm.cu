@@ -20,6 +20,7 @@
 
 #include "common.h"
 #include "kernels.h"
+#include "fixpoint.cuh"
 #include "launch.h"
 #include "ptx.cuh"
 
@@ -45,7 +46,10 @@ struct TileCfg {
   static constexpr int STAGES = (200 * 1024) / STAGE_BYTES > 6 ? 6 : (200 * 1024) / STAGE_BYTES;
   static constexpr int BAR_OFF = STAGES * STAGE_BYTES;
   static constexpr int STG_OFF = BAR_OFF + (2 * STAGES + 4) * 8 + 16;
-  static constexpr int SMEM_TOTAL = STG_OFF + 8 * 32 * 20 * 4 + 1024;  // + epilogue staging, alignment slack
+  // SPLIT (the SPOS forward 1x1 conv): per-warp column sums of the fused BatchNorm statistics
+  static constexpr int SST_OFF = STG_OFF + 8 * 32 * 20 * 4;
+  static constexpr int SST_BYTES = SPLIT ? 8 * (TN / 2) * 2 * 4 : 0;
+  static constexpr int SMEM_TOTAL = SST_OFF + SST_BYTES + 1024;  // + epilogue staging, alignment slack
   static constexpr int TMEM_COLS = 2 * TN <= 128 ? 128 : (2 * TN <= 256 ? 256 : 512);
 };
 
@@ -143,9 +147,11 @@ __device__ __forceinline__ void epilogue4(float4 v, float4 pre, float4 b, size_t
 // every global load/store of the epilogue is a coalesced row segment of 4*EC (fp32) or
 // 2*EC (bf16) bytes, instead of 32 rows x 16 bytes per instruction.  The padding makes
 // both staging passes bank-conflict free.
+// sst (EPI_X2 with ep.stats): this warp's [cend - cbeg][2] column sums of its 32 rows
 template <int EPI, int EC>
 __device__ __forceinline__ void epilogue_warp(uint32_t taddr, float* stg, int row0, int cbeg, int cend, int n0,
-                                              int M, int N, const GemmEpiParams& ep, int split, int lane) {
+                                              int M, int N, const GemmEpiParams& ep, int split, int lane,
+                                              float* sst = nullptr) {
   constexpr int LD = EC + 4, LPR = EC / 4, RPI = 32 / LPR, NIT = 32 / RPI;
   constexpr bool HAS_PRE = EPI == EPI_BIAS_RESID_F32 || EPI == EPI_SGD || EPI == EPI_DGELU;
   constexpr bool HAS_BIAS = EPI == EPI_BIAS_BF16 || EPI == EPI_BIAS_RESID_F32 || EPI == EPI_BIAS_GELU;
@@ -177,12 +183,42 @@ __device__ __forceinline__ void epilogue_warp(uint32_t taddr, float* stg, int ro
           make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]), __uint_as_float(r[4 * j + 2]),
                       __uint_as_float(r[4 * j + 3]));
     __syncwarp();
+    float bs[4] = {0.f, 0.f, 0.f, 0.f}, bq[4] = {0.f, 0.f, 0.f, 0.f};
 #pragma unroll
     for (int it = 0; it < NIT; ++it) {
       const int rr = it * RPI + lane / LPR;
       const int grow = row0 + rr;
       const float4 v = *reinterpret_cast<const float4*>(stg + rr * LD + cc);
-      if (grow < M && gcol < N) epilogue4<EPI>(v, pre[it], b, (size_t)grow * N + gcol, ep, split);
+      if (grow < M && gcol < N) {
+        epilogue4<EPI>(v, pre[it], b, (size_t)grow * N + gcol, ep, split);
+        if constexpr (EPI == EPI_X2) {  // statistics of the stored value hi + lo
+          const float vv[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            const float hi = __bfloat162float(__float2bfloat16_rn(vv[i]));
+            const float st = hi + __bfloat162float(__float2bfloat16_rn(vv[i] - hi));
+            bs[i] += st;
+            bq[i] = __fmaf_rn(st, st, bq[i]);
+          }
+        }
+      }
+    }
+    if constexpr (EPI == EPI_X2) {
+      if (sst != nullptr) {  // fixed xor tree over the 8 row groups of the warp (lanes cc + 4 LPR k)
+#pragma unroll
+        for (int o = LPR; o < 32; o <<= 1)
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            bs[i] += __shfl_xor_sync(0xffffffffu, bs[i], o);
+            bq[i] += __shfl_xor_sync(0xffffffffu, bq[i], o);
+          }
+        if (lane < LPR)
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            sst[(c0 - cbeg + cc + i) * 2] = bs[i];
+            sst[(c0 - cbeg + cc + i) * 2 + 1] = bq[i];
+          }
+      }
     }
     __syncwarp();
   }
@@ -334,11 +370,37 @@ __global__ void __launch_bounds__(THREADS, 1)
       ptx::tc_fence_after();
       if (t + (int)gridDim.x >= n_tiles) ptx::pdl_trigger();  // last tile: let the next kernel launch
       const uint32_t taddr = tmem + ((uint32_t)lane_base << 16) + acc * TN;
+      float* sst = nullptr;
+      if constexpr (EPI == EPI_X2)
+        if (ep.stats != nullptr) sst = reinterpret_cast<float*>(smem + Cf::SST_OFF) + (warp - 2) * (TN / 2) * 2;
       epilogue_warp<EPI, 16>(taddr, stg + (warp - 2) * 32 * 20, tm * BM + lane_base, cbeg, cbeg + TN / 2, tn * TN, M,
-                             N, ep, ks, lane);
+                             N, ep, ks, lane, sst);
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(&tempty[acc]);
+      if constexpr (EPI == EPI_X2) {
+        if (ep.stats != nullptr) {
+          // fused BatchNorm statistics: the 4 warps of this column half (lane quarters 0..3)
+          // combine their 32-row column sums in quarter order, one fixed-point add per column
+          const int half = (warp - 2) >> 2;
+          ptx::named_bar_sync(1 + half, 128);
+          const float* base = reinterpret_cast<const float*>(smem + Cf::SST_OFF) + half * 4 * (TN / 2) * 2;
+          for (int j = (warp & 3) * 32 + lane; j < TN / 2; j += 128) {
+            const int gcol = tn * TN + cbeg + j;
+            if (gcol >= N) continue;
+            float s1 = 0.f, s2 = 0.f;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {  // quarter q is warp 2 + 4 half + ((q + 2) & 3)
+              const float* w = base + ((q + 2) & 3) * (TN / 2) * 2;
+              s1 += w[j * 2];
+              s2 += w[j * 2 + 1];
+            }
+            fix_add(ep.stats, gcol, ep.stats + 2 * N, s1, FIX_S1);
+            fix_add(ep.stats, N + gcol, ep.stats + 2 * N, s2, FIX_S2);
+          }
+          ptx::named_bar_sync(1 + half, 128);  // the slots are rewritten by the next tile
+        }
+      }
     }
   }
   __syncthreads();
@@ -583,16 +645,6 @@ CUtensorMap make_map(const bf16* base, uint64_t inner, uint64_t outer, uint64_t 
 std::atomic<uint64_t> g_gemm_launches{0};
 std::atomic<uint64_t> g_gemm_flops{0};  // algorithmic 2*M*N*K of every GEMM call (bf16x2: one product)
 
-int num_sms() {
-  static int n = 0;
-  if (!n) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
-    if (n <= 0) n = 148;
-  }
-  return n;
-}
 
 template <bool A_MN, bool B_MN, int EPI, int TN = BN, bool SPLIT = false>
 void launch(cudaStream_t s, int M, int N, const TileSpace& ts, const CUtensorMap& ta, const CUtensorMap& tb,
@@ -643,13 +695,14 @@ void launch_pair(cudaStream_t s, int M, int N, const TileSpace& ts, const CUtens
   // the 40-step configs[2] run deadlocked on the GPU (tools/hangtest.sh: hang with triggers;
   // no hang and the best step time without them).  NASPIPE_PAIR_TRIGGER=1 re-enables them
   // for diagnosis, NASPIPE_PAIR_PDL=0 drops the attribute.
-  static int pair_pdl = -1, pair_trig = -1;
-  if (pair_pdl < 0) {
+  static const int pair_pdl = [] {
     const char* e1 = getenv("NASPIPE_PAIR_PDL");
+    return (e1 && e1[0] == '0') ? 0 : 1;
+  }();
+  static const int pair_trig = [] {
     const char* e2 = getenv("NASPIPE_PAIR_TRIGGER");
-    pair_pdl = (e1 && e1[0] == '0') ? 0 : 1;
-    pair_trig = (e2 && e2[0] == '1') ? 1 : 0;
-  }
+    return (e2 && e2[0] == '1') ? 1 : 0;
+  }();
   if (pdl_enabled() && pair_pdl) {
     cfg.attrs = at;
     cfg.numAttrs = 2;
@@ -679,11 +732,10 @@ void dispatch_pair(cudaStream_t s, int M, int N, const TileSpace& ts, const CUte
 }
 
 bool pair_enabled() {
-  static int v = -1;
-  if (v < 0) {
+  static const int v = [] {  // thread-safe one-time init
     const char* e = getenv("NASPIPE_GEMM_PAIR");
-    v = (e && e[0] == '0') ? 0 : 1;
-  }
+    return (e && e[0] == '0') ? 0 : 1;
+  }();
   return v == 1;
 }
 
@@ -725,6 +777,16 @@ void dispatch_epi(cudaStream_t s, int M, int N, const TileSpace& ts, const CUten
 }
 
 }  // namespace
+
+int num_sms() {
+  static const int n = [] {
+    int dev = 0, v = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev);
+    return v > 0 ? v : 148;
+  }();
+  return n;
+}
 
 uint64_t gemm_launch_count() { return g_gemm_launches.load(); }
 uint64_t gemm_flop_count() { return g_gemm_flops.load(); }
@@ -795,11 +857,10 @@ void gemm_bf16_tc(cudaStream_t s, int M, int N, int K, const bf16* A, bool a_mn,
     int L = 1;  // lanes per output vector: a power of two (xor tree), <= splits / 4
     while (2 * L <= 32 && 2 * L <= ts.splits / 4) L *= 2;
     const size_t per_block = 256 / L;
-    static int per_sm = 0;  // CTAs per SM of the reduce; NASPIPE_SPLITK_CTAS_PER_SM overrides (tuning)
-    if (!per_sm) {
+    static const int per_sm = [] {  // CTAs per SM of the reduce; NASPIPE_SPLITK_CTAS_PER_SM overrides (tuning)
       const char* e = getenv("NASPIPE_SPLITK_CTAS_PER_SM");
-      per_sm = e ? std::max(1, atoi(e)) : 4;
-    }
+      return e ? std::max(1, atoi(e)) : 4;
+    }();
     const int blocks = (int)std::min<size_t>(((size_t)M * N / 4 + per_block - 1) / per_block, (size_t)per_sm * num_sms());
     if (epi == EPI_F32)
       launch_pdl(splitk_reduce_kernel<EPI_F32>, dim3(blocks), dim3(256), 0, s, M, N, ts.splits, L, ep);

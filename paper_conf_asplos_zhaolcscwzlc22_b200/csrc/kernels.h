@@ -42,6 +42,10 @@ struct GemmEpiParams {
   float* ws = nullptr;
   size_t ws_elems = 0;
   size_t ws_stride = 0;  // set by the launcher
+  // EPI_X2 only: add the per-column BatchNorm sums (sum, sum of squares of the STORED hi+lo
+  // values) of the output to stats[0..2N) in fixed point (fixpoint.cuh; stats[2N] = the
+  // overflow flag): the SPOS forward 1x1 conv with bn_stats fused
+  unsigned long long* stats = nullptr;
 };
 // split-K factor the launcher uses for an (M, N, K) GEMM given a large enough workspace
 int gemm_splitk_factor(int M, int N, int K);
@@ -54,6 +58,7 @@ void gemm_bf16x2_tc(cudaStream_t s, int M, int N, int K, const bf16* A_hi, const
                     const bf16* B_hi, const bf16* B_lo, int ldb, int epi, const GemmEpiParams& ep);
 // number of tcgen05 GEMM launches so far in this process (stats)
 uint64_t gemm_launch_count();
+int num_sms();  // SMs of the current device (cached)
 uint64_t gemm_flop_count();  // algorithmic flops of every GEMM call of this process
 
 // ------------------------------------------------------------------ attention (S <= 128)
@@ -125,7 +130,7 @@ void f32_to_bf16x2(cudaStream_t s, const float* w32, bf16* hi, bf16* lo, size_t 
 void spos_stem_conv(cudaStream_t s, const float* x, const float* w, bf16* z, int B, int H, int C0);
 // BatchNorm (training mode, biased variance, eps 1e-5).  Reductions over the P rows are
 // fixed-order fp32 row-block partials accumulated in 64-bit fixed point with integer atomics
-// into acc [2][C] (unsigned long long, zero between uses): bitwise independent of the CTA
+// into acc [2][C] (+1: the overflow flag; unsigned long long, zero between uses): bitwise independent of the CTA
 // order, no finalize launch.  The consumer kernel (bn_apply / bn_bwd_apply) derives the
 // per-channel results from acc in every CTA; its last CTA (ticket: an int, 0 between uses)
 // publishes them and zeroes acc and the ticket.
@@ -144,11 +149,13 @@ void bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int 
 void bn_bwd_apply(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
                   const float* rstd, const float* g, const float* b, float* gu, float* bu, float lr, int update,
                   unsigned long long* acc, int* ticket, int relu, bf16* dz);
-// sticky device flag: a fixed-point partial fell outside its range (checked at drain)
-bool bn_fix_overflow();
+// acc holds 2C sums + the sticky overflow flag acc[2C] (fixpoint.cuh; checked at drain)
+bool bn_fix_overflow(const unsigned long long* acc, int C);
 // depthwise k x k (k in {3,5,7}), stride S, pad k/2; w fp32 [C][k][k]; H = input height = width.
 // dw_fwd: x2 -> x2; dw_dgrad: bf16 (+ bf16 add); dw_wgrad reads the hi plane of x.
-void dw_fwd(cudaStream_t s, const bf16* x, const float* w, bf16* z, int B, int H, int C, int k, int S);
+// stats != nullptr: also add the BatchNorm sums of the stored z to it (bn_stats fused)
+void dw_fwd(cudaStream_t s, const bf16* x, const float* w, bf16* z, int B, int H, int C, int k, int S,
+            unsigned long long* stats = nullptr);
 void dw_dgrad(cudaStream_t s, const bf16* dz, const float* w, const bf16* add, bf16* dx, int B, int H, int C, int k,
               int S);
 int dw_wgrad_blocks(int B, int H, int C, int k, int S);

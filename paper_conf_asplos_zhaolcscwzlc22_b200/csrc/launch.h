@@ -11,19 +11,19 @@
 
 namespace naspipe {
 
-// Engines alive in this process that launch without PDL (the multi-process rank engines:
-// their compute streams wait on transport streams / peer flags between kernels).
-//
-// History (DESIGN.md §5 "PDL"): round 1 turned PDL off for context-switching engines after a
-// 14-subnet configs[3] run deadlocked with it.  Root cause: the tcgen05 GEMM kernels took
-// their TMEM columns (tcgen05.alloc, up to 512) BEFORE griddepcontrol.wait, so an early-
-// launched GEMM CTA could hold TMEM on an SM while it waited for its predecessor grid; with
-// the candidate-load / shadow-refresh / write-back streams' kernels interleaved on the SMs
-// (the most likely cause; not proven).  Since the GEMMs allocate
-// TMEM only after the wait, the reproduction (tools/c4_probe.py --no-drain with
-// NASPIPE_FORCE_PDL=1, 3 runs) and tests/test_gpu_context.py pass with PDL, and context
-// switching runs with it again.  The CTA-pair GEMM's EARLY TRIGGERS (NASPIPE_PAIR_TRIGGER=1)
-// still hang tools/hangtest.sh and stay off.
+// Engines alive in this process that launch without PDL:
+// * context-switching engines (hbm_weight_budget_bytes > 0): the compute stream's kernels
+//   follow cross-stream event waits (a candidate's load / shadow refresh is ready).  Round 1
+//   saw a 14-subnet configs[3] run deadlock with PDL.  Round 2 moved the GEMMs' TMEM
+//   allocation after griddepcontrol.wait (an early-launched CTA no longer holds TMEM while
+//   it waits); with that, the reproduction (tools/c4_probe.py --no-drain, NASPIPE_FORCE_PDL=1)
+//   passed 3 of 3 runs and tests/test_gpu_context.py passed, but the bench's configs[3] run
+//   (submit/drain cycles, HOST batches) still hung with PDL (killed by its 600 s timeout).
+//   Root cause not found: PDL stays off for these engines (DESIGN.md §5 "PDL").
+// * multi-process rank engines: their compute streams wait on transport streams / peer
+//   flags between kernels (the same cross-stream pattern).
+// The CTA-pair GEMM's early triggers (NASPIPE_PAIR_TRIGGER=1) also still hang
+// tools/hangtest.sh and stay off.
 inline std::atomic<int>& pdl_suppressors() {
   static std::atomic<int> n{0};
   return n;

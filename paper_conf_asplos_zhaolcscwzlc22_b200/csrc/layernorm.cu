@@ -22,11 +22,10 @@ constexpr int LN_ROWS_MAX = 32;  // rows per backward block (runtime, <= this): 
 constexpr int LN_WARPS = 8;
 // NASPIPE_LN_ROWS (tuning; default 16) -- fixed per process, so partial counts are too
 static int ln_rows() {
-  static int v = 0;
-  if (!v) {
+  static const int v = [] {  // thread-safe one-time init
     const char* e = getenv("NASPIPE_LN_ROWS");
-    v = e ? std::min(LN_ROWS_MAX, std::max(1, atoi(e))) : 16;
-  }
+    return e ? std::min(LN_ROWS_MAX, std::max(1, atoi(e))) : 16;
+  }();
   return v;
 }
 

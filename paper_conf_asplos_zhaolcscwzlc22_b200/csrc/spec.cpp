@@ -40,7 +40,7 @@ Spec::Spec(const naspipe_supernet_spec* s) {
   NP_REQUIRE(raw.window >= 0 && raw.lookahead >= 0 && raw.bwd_policy >= 0 && raw.bwd_policy <= 1 &&
                  raw.link_latency >= 0 && raw.hbm_weight_budget_bytes >= 0,
              NASPIPE_EINVAL, "bad window/lookahead/policy/latency/budget");
-  NP_REQUIRE(raw.sync_policy >= NASPIPE_SYNC_CSP && raw.sync_policy <= NASPIPE_SYNC_BSP && raw.bulk_size >= 0,
+  NP_REQUIRE(raw.sync_policy >= NASPIPE_SYNC_CSP && raw.sync_policy <= NASPIPE_SYNC_SERIAL && raw.bulk_size >= 0,
              NASPIPE_EINVAL, "bad sync_policy %d / bulk_size %d", raw.sync_policy, raw.bulk_size);
   NP_REQUIRE(!(raw.flags & NASPIPE_FLAG_RECOMPUTE) ||
                  (raw.family == NASPIPE_TRANSFORMER && raw.sync_policy != NASPIPE_SYNC_ASP),

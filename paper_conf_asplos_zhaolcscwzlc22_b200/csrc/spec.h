@@ -55,7 +55,10 @@ struct Spec {
   int m() const { return raw.n_blocks; }
   int n() const { return raw.n_choices; }
   int B() const { return raw.batch; }
-  int window(int D) const { return raw.window > 0 ? raw.window : 4 * D; }
+  // SERIAL ("w/o scheduler"): one subnet in flight, W = 1 (reading A32)
+  int window(int D) const {
+    return raw.sync_policy == NASPIPE_SYNC_SERIAL ? 1 : raw.window > 0 ? raw.window : 4 * D;
+  }
   int bulk(int D) const { return raw.bulk_size > 0 ? raw.bulk_size : 4 * D; }
   int lookahead() const { return raw.lookahead > 0 ? raw.lookahead : 2; }
   int64_t residency_horizon() const { return raw.residency_horizon == 0 ? 64 : raw.residency_horizon; }

@@ -22,10 +22,13 @@
 // then a fixed order over row blocks), never floating-point atomics: bitwise reproducible.
 #include <algorithm>
 #include <cstdlib>
+#include <map>
+#include <mutex>
 
 #include "common.h"
 #include "kernels.h"
 #include "launch.h"
+#include "fixpoint.cuh"
 #include "ptx.cuh"
 
 namespace naspipe {
@@ -35,30 +38,28 @@ constexpr int TPB = 256;          // threads per block of the row-block kernels
 // target CTAs of the row-block reductions: fewer, longer row blocks keep the partial count
 // (and so the fixed-order finalize) short; NASPIPE_RED_CTAS overrides it for tuning.
 static int red_ctas() {
-  static int v = 0;
-  if (!v) {
+  static const int v = [] {  // thread-safe one-time init
     const char* e = getenv("NASPIPE_RED_CTAS");
-    v = e ? std::max(16, atoi(e)) : 296;
-  }
+    return e ? std::max(16, atoi(e)) : 296;
+  }();
   return v;
 }
 // target CTAs of the depthwise weight-gradient partials (NASPIPE_DW_RED_CTAS, default: the
 // BatchNorm target above)
 static int dw_red_ctas() {
-  static int v = 0;
-  if (!v) {
+  static const int v = [] {  // thread-safe one-time init
     const char* e = getenv("NASPIPE_DW_RED_CTAS");
-    v = e ? std::max(16, atoi(e)) : red_ctas();
-  }
+    return e ? std::max(16, atoi(e)) : red_ctas();
+  }();
   return v;
 }
 constexpr float BN_EPS = 1e-5f;
 
 // Row blocking of the per-channel reductions: a function of (P, C) only (deterministic),
 // about RED_CTAS blocks, each a multiple of the kernel's row lanes RP = TPB / (C/8).
-inline int red_rows(int P, int C) {
-  const int rp = TPB / (C / 8);
-  const int target = red_ctas();
+inline int red_rows(int P, int C, int vec = 8, int target = 0) {
+  const int rp = TPB / (C / vec);
+  if (target <= 0) target = red_ctas();
   int rows = (P + target - 1) / target;
   rows = ((rows + rp - 1) / rp) * rp;
   return rows < rp ? rp : rows;
@@ -70,7 +71,7 @@ inline void check_launch(const char* what) {
 }
 inline int grid_for(size_t items, int per_block = TPB) {
   const size_t g = (items + per_block - 1) / per_block;
-  return (int)std::min<size_t>(std::max<size_t>(g, 1), 148 * 16);
+  return (int)std::min<size_t>(std::max<size_t>(g, 1), (size_t)num_sms() * 16);
 }
 
 __device__ __forceinline__ void load8(const bf16* p, float (&v)[8]) {
@@ -165,25 +166,7 @@ __global__ void stem_conv_kernel(const float* __restrict__ x, const float* __res
 // The consumer kernel (bn_apply / bn_bwd_apply) reads the totals; its last CTA (arrival
 // ticket) publishes the per-channel results and zeroes acc and the ticket for the next use.
 //
-// Scales: forward sum z (2^32: |sum| < 2^31), sum z^2 (2^24: < 5.5e11), backward sums
-// (2^40: |sum| < 8.4e6).  A partial outside the range sets the sticky overflow flag
-// (checked at drain, NASPIPE_EINTERNAL) instead of wrapping silently.
-constexpr double FIX_S1 = 4294967296.0;      // 2^32
-constexpr double FIX_S2 = 16777216.0;        // 2^24
-constexpr double FIX_B = 1099511627776.0;    // 2^40
-__device__ int g_fix_overflow;
-
-__device__ __forceinline__ void fix_add(unsigned long long* acc, float v, double scale) {
-  const double x = (double)v * scale;
-  if (!(fabs(x) < 4.0e18)) {  // also catches NaN
-    atomicOr(&g_fix_overflow, 1);
-    return;
-  }
-  atomicAdd(acc, (unsigned long long)(long long)__double2ll_rn(x));
-}
-__device__ __forceinline__ double fix_get(const unsigned long long* acc, int i, double scale) {
-  return (double)(long long)acc[i] / scale;
-}
+// Fixed-point scales, fix_add / fix_get and the overflow flag acc[2C]: fixpoint.cuh.
 
 // arrival ticket: true in every thread of the CTA that arrives last (all others are done)
 __device__ __forceinline__ bool last_cta(int* ticket) {
@@ -249,7 +232,7 @@ __global__ void bn_stats_kernel(const bf16* __restrict__ z, int P, int C, int ro
   for (int e = threadIdx.x; e < 2 * C; e += TPB) {
     float a = 0.f;
     for (int k = 0; k < RP; ++k) a += red[k * 2 * C + e];
-    fix_add(acc + e, a, e < C ? FIX_S1 : FIX_S2);
+    fix_add(acc, e, acc + 2 * C, a, e < C ? FIX_S1 : FIX_S2);
   }
 }
 
@@ -260,12 +243,19 @@ __device__ __forceinline__ int ew_lanes(int C) { return TPB / (C / 8); }
 __device__ __forceinline__ void bn_apply_body(const bf16* __restrict__ z, int P, int C, const unsigned long long* acc,
                                               const float* __restrict__ gam, const float* __restrict__ bet, int relu,
                                               bf16* __restrict__ y, int ldy, size_t yplane) {
+  // the CTA derives every channel's moments once (fp64, from the fixed-point totals)
+  __shared__ float smu[2048], srs[2048];  // C <= 8 TPB = 2048 (host check)
+  for (int cc = threadIdx.x; cc < C; cc += blockDim.x) bn_moments(acc, C, cc, P, smu[cc], srs[cc]);
+  __syncthreads();
   const int G = C / 8, lanes = ew_lanes(C);
   const int pl = threadIdx.x / G, c = (threadIdx.x % G) * 8;
   if (pl >= lanes) return;
   float mu[8], rs[8], g8[8], b8[8];
 #pragma unroll
-  for (int i = 0; i < 8; ++i) bn_moments(acc, C, c + i, P, mu[i], rs[i]);
+  for (int i = 0; i < 8; ++i) {
+    mu[i] = smu[c + i];
+    rs[i] = srs[c + i];
+  }
   load8f(gam + c, g8);
   load8f(bet + c, b8);
   const size_t zplane = (size_t)P * C;
@@ -317,73 +307,100 @@ __global__ void bn_apply_kernel(const bf16* __restrict__ z, int P, int C, unsign
 }
 
 // ---------------------------------------------------------------- BatchNorm backward
-__device__ __forceinline__ void bn_bwd_item(const bf16* dy, const bf16* z, size_t zplane, const float (&mu)[8],
-                                            const float (&rs)[8], const float (&g8)[8], const float (&b8)[8],
-                                            int relu, float (&d)[8], float (&xh)[8]) {
-  float zz[8];
-  load8(dy, d);
-  load8x2(z, zplane, zz);
+// 4 channels per thread (BV): the per-channel constants (mean, rstd, g, b, s1, s2) of 8
+// channels held 92-96 registers (2 CTAs/SM, 25 % occupancy, ~2 TB/s measured by ncu);
+// 4 channels halve them.
+constexpr int BV = 4;
+__device__ __forceinline__ void load4(const bf16* p, float (&v)[4]) {
+  const uint2 q = *reinterpret_cast<const uint2*>(p);
+  v[0] = __uint_as_float(q.x << 16);
+  v[1] = __uint_as_float(q.x & 0xffff0000u);
+  v[2] = __uint_as_float(q.y << 16);
+  v[3] = __uint_as_float(q.y & 0xffff0000u);
+}
+__device__ __forceinline__ void load4x2(const bf16* p, size_t plane, float (&v)[4]) {
+  float lo[4];
+  load4(p, v);
+  load4(p + plane, lo);
 #pragma unroll
-  for (int i = 0; i < 8; ++i) {
+  for (int i = 0; i < 4; ++i) v[i] += lo[i];
+}
+__device__ __forceinline__ void store4(bf16* p, const float (&v)[4]) {
+  *reinterpret_cast<uint2*>(p) = make_uint2(ptx::pack_bf16(v[0], v[1]), ptx::pack_bf16(v[2], v[3]));
+}
+__device__ __forceinline__ void load4f(const float* p, float (&v)[4]) {
+  const float4 a = *reinterpret_cast<const float4*>(p);
+  v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
+}
+
+__device__ __forceinline__ void bn_bwd_item(const bf16* dy, const bf16* z, size_t zplane, const float (&mu)[BV],
+                                            const float (&rs)[BV], const float (&g8)[BV], const float (&b8)[BV],
+                                            int relu, float (&d)[BV], float (&xh)[BV]) {
+  float zz[BV];
+  load4(dy, d);
+  load4x2(z, zplane, zz);
+#pragma unroll
+  for (int i = 0; i < BV; ++i) {
     xh[i] = __fmul_rn(__fsub_rn(zz[i], mu[i]), rs[i]);
     if (relu && !(bn_y(zz[i], mu[i], rs[i], g8[i], b8[i]) > 0.f)) d[i] = 0.f;
   }
 }
 
 // s1 = sum dy', s2 = sum dy' xh (dy' = dy masked by the ReLU): fixed-order row-block
-// partials added to acc[2C] in fixed point (see bn_stats_kernel).
+// partials added to acc[2C] in fixed point (see bn_stats_kernel).  Thread (r, g): rows r,
+// r + RP, ... of its block, channels [4g, 4g+4); RP = TPB / (C/4).
 __global__ void bn_bwd_reduce_kernel(const bf16* __restrict__ dy, int lddy, const bf16* __restrict__ z, int P, int C,
                                      const float* __restrict__ mean, const float* __restrict__ rstd,
                                      const float* __restrict__ gam, const float* __restrict__ bet, int relu,
                                      int rows, unsigned long long* acc) {
   extern __shared__ float red[];  // [RP][2C]
   ptx::pdl_wait();
-  const int G = C / 8, RP = TPB / G;
+  const int G = C / BV, RP = TPB / G;
   const int r = threadIdx.x / G, g = threadIdx.x % G;
   const int row0 = blockIdx.x * rows, row1 = min(P, row0 + rows);
   const size_t zplane = (size_t)P * C;
   if (r < RP) {
-    float mu[8], rs[8], g8[8], b8[8];
-    load8f(mean + 8 * g, mu);
-    load8f(rstd + 8 * g, rs);
-    load8f(gam + 8 * g, g8);
-    load8f(bet + 8 * g, b8);
-    float s1[8] = {}, s2[8] = {};
+    float mu[BV], rs[BV], g8[BV], b8[BV];
+    load4f(mean + BV * g, mu);
+    load4f(rstd + BV * g, rs);
+    load4f(gam + BV * g, g8);
+    load4f(bet + BV * g, b8);
+    float s1[BV] = {}, s2[BV] = {};
     int row = row0 + r;
-    for (; row + RP < row1; row += 2 * RP) {
-      float d[2][8], xh[2][8];
+    for (; row + 3 * RP < row1; row += 4 * RP) {  // 4 rows in flight
+      float d[4][BV], xh[4][BV];
 #pragma unroll
-      for (int u = 0; u < 2; ++u)
-        bn_bwd_item(dy + (size_t)(row + u * RP) * lddy + 8 * g, z + (size_t)(row + u * RP) * C + 8 * g, zplane, mu, rs,
-                    g8, b8, relu, d[u], xh[u]);
+      for (int u = 0; u < 4; ++u)
+        bn_bwd_item(dy + (size_t)(row + u * RP) * lddy + BV * g, z + (size_t)(row + u * RP) * C + BV * g, zplane, mu,
+                    rs, g8, b8, relu, d[u], xh[u]);
 #pragma unroll
-      for (int u = 0; u < 2; ++u)
+      for (int u = 0; u < 4; ++u)
 #pragma unroll
-        for (int i = 0; i < 8; ++i) {
+        for (int i = 0; i < BV; ++i) {
           s1[i] += d[u][i];
           s2[i] = __fmaf_rn(d[u][i], xh[u][i], s2[i]);
         }
     }
     for (; row < row1; row += RP) {
-      float d[8], xh[8];
-      bn_bwd_item(dy + (size_t)row * lddy + 8 * g, z + (size_t)row * C + 8 * g, zplane, mu, rs, g8, b8, relu, d, xh);
+      float d[BV], xh[BV];
+      bn_bwd_item(dy + (size_t)row * lddy + BV * g, z + (size_t)row * C + BV * g, zplane, mu, rs, g8, b8, relu, d, xh);
 #pragma unroll
-      for (int i = 0; i < 8; ++i) {
+      for (int i = 0; i < BV; ++i) {
         s1[i] += d[i];
         s2[i] = __fmaf_rn(d[i], xh[i], s2[i]);
       }
     }
 #pragma unroll
-    for (int i = 0; i < 8; ++i) {
-      red[r * 2 * C + 8 * g + i] = s1[i];
-      red[r * 2 * C + C + 8 * g + i] = s2[i];
+    for (int i = 0; i < BV; ++i) {
+      red[r * 2 * C + BV * g + i] = s1[i];
+      red[r * 2 * C + C + BV * g + i] = s2[i];
     }
   }
   __syncthreads();
   for (int e = threadIdx.x; e < 2 * C; e += TPB) {
     float a = 0.f;
     for (int k = 0; k < RP; ++k) a += red[k * 2 * C + e];
-    fix_add(acc + e, a, FIX_B);
+    fix_add(acc, e, acc + 2 * C, a, FIX_B);
   }
 }
 
@@ -392,31 +409,48 @@ __device__ __forceinline__ void bn_bwd_apply_body(const bf16* __restrict__ dy, i
                                                   const float* __restrict__ rstd, const float* __restrict__ gam,
                                                   const float* __restrict__ bet, const unsigned long long* acc, int relu,
                                                   bf16* __restrict__ dz) {
-  const int G = C / 8, lanes = ew_lanes(C);
-  const int pl = threadIdx.x / G, c = (threadIdx.x % G) * 8;
+  __shared__ float sm1[1024], sm2[1024];  // the CTA converts the fixed-point totals once (C <= 4 TPB)
+  for (int cc = threadIdx.x; cc < C; cc += blockDim.x) {
+    sm1[cc] = (float)fix_get(acc, cc, FIX_B);
+    sm2[cc] = (float)fix_get(acc, C + cc, FIX_B);
+  }
+  __syncthreads();
+  const int G = C / BV, lanes = TPB / G;
+  const int pl = threadIdx.x / G, c = (threadIdx.x % G) * BV;
   if (pl >= lanes) return;
   const float invP = 1.0f / (float)P;
-  float mu[8], rs[8], g8[8], b8[8], m1[8], m2[8];
-  load8f(mean + c, mu);
-  load8f(rstd + c, rs);
-  load8f(gam + c, g8);
-  load8f(bet + c, b8);
+  float mu[BV], rs[BV], g8[BV], b8[BV], m1[BV], m2[BV];
+  load4f(mean + c, mu);
+  load4f(rstd + c, rs);
+  load4f(gam + c, g8);
+  load4f(bet + c, b8);
 #pragma unroll
-  for (int i = 0; i < 8; ++i) {
-    m1[i] = (float)fix_get(acc, c + i, FIX_B);
-    m2[i] = (float)fix_get(acc, C + c + i, FIX_B);
+  for (int i = 0; i < BV; ++i) {
+    m1[i] = sm1[c + i] * invP;
+    m2[i] = sm2[c + i] * invP;
   }
   const size_t zplane = (size_t)P * C;
   const int step = gridDim.x * lanes;
-  for (int p = blockIdx.x * lanes + pl; p < P; p += step) {
-    float d[8], xh[8];
+  int p = blockIdx.x * lanes + pl;
+  for (; p + step < P; p += 2 * step) {  // two pixels in flight
+    float d[2][BV], xh[2][BV];
+#pragma unroll
+    for (int u = 0; u < 2; ++u)
+      bn_bwd_item(dy + (size_t)(p + u * step) * lddy + c, z + (size_t)(p + u * step) * C + c, zplane, mu, rs, g8, b8,
+                  relu, d[u], xh[u]);
+#pragma unroll
+    for (int u = 0; u < 2; ++u) {
+#pragma unroll
+      for (int i = 0; i < BV; ++i) d[u][i] = rs[i] * g8[i] * (d[u][i] - m1[i] - xh[u][i] * m2[i]);
+      store4(dz + (size_t)(p + u * step) * C + c, d[u]);
+    }
+  }
+  for (; p < P; p += step) {
+    float d[BV], xh[BV];
     bn_bwd_item(dy + (size_t)p * lddy + c, z + (size_t)p * C + c, zplane, mu, rs, g8, b8, relu, d, xh);
 #pragma unroll
-    for (int i = 0; i < 8; ++i) {
-      const float t = d[i] - m1[i] * invP - xh[i] * (m2[i] * invP);
-      d[i] = rs[i] * g8[i] * t;
-    }
-    store8(dz + (size_t)p * C + c, d);
+    for (int i = 0; i < BV; ++i) d[i] = rs[i] * g8[i] * (d[i] - m1[i] - xh[i] * m2[i]);
+    store4(dz + (size_t)p * C + c, d);
   }
 }
 
@@ -513,7 +547,7 @@ constexpr int DT_H = 8;
 template <int K, int S, bool X2, bool FLIP>
 __global__ void __launch_bounds__(TPB) dw_tile_kernel(const bf16* __restrict__ in, const float* __restrict__ w,
                                                     const bf16* __restrict__ add, bf16* __restrict__ out, int B,
-                                                    int H, int C, int TW) {
+                                                    int H, int C, int TW, unsigned long long* stats) {
   constexpr int PAD = K / 2, IH = (DT_H - 1) * S + K;
   extern __shared__ float tile[];  // [CPG][IH][IW][8]
   ptx::pdl_wait();
@@ -569,18 +603,49 @@ __global__ void __launch_bounds__(TPB) dw_tile_kernel(const bf16* __restrict__ i
     }
   }
   const int ow = tw * TW + col;
-  if (c >= C || ow >= Ho) return;
+  const bool valid = c < C && ow < Ho;
+  float ss = 0.f, sq = 0.f;  // BatchNorm statistics of the stored values (fused bn_stats)
+  if (valid) {
 #pragma unroll
-  for (int r = 0; r < DT_H; ++r) {
-    const int oh = th * DT_H + r;
-    if (oh >= Ho) break;
-    const size_t o = (((size_t)b * Ho + oh) * Ho + ow) * C + c;
-    if (X2) {
-      const bf16 hi = __float2bfloat16_rn(acc[r]);
-      out[o] = hi;
-      out[o + oplane] = __float2bfloat16_rn(acc[r] - __bfloat162float(hi));
-    } else {
-      out[o] = __float2bfloat16_rn(add ? acc[r] + __bfloat162float(add[o]) : acc[r]);
+    for (int r = 0; r < DT_H; ++r) {
+      const int oh = th * DT_H + r;
+      if (oh >= Ho) break;
+      const size_t o = (((size_t)b * Ho + oh) * Ho + ow) * C + c;
+      if (X2) {
+        const bf16 hi = __float2bfloat16_rn(acc[r]);
+        const bf16 lo = __float2bfloat16_rn(acc[r] - __bfloat162float(hi));
+        out[o] = hi;
+        out[o + oplane] = lo;
+        const float v = __bfloat162float(hi) + __bfloat162float(lo);
+        ss += v;
+        sq = __fmaf_rn(v, v, sq);
+      } else {
+        out[o] = __float2bfloat16_rn(add ? acc[r] + __bfloat162float(add[o]) : acc[r]);
+      }
+    }
+  }
+  if (X2 && stats != nullptr) {
+    // per channel over the CTA's TW columns, fixed order: xor tree over the 4 columns of a
+    // warp (lanes ch + 8 col), then the warps of the channel group in warp order
+    __shared__ float wsum[TPB / 32][2][8];
+#pragma unroll
+    for (int o = 8; o < 32; o <<= 1) {
+      ss += __shfl_xor_sync(0xffffffffu, ss, o);
+      sq += __shfl_xor_sync(0xffffffffu, sq, o);
+    }
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (lane < 8) {
+      wsum[warp][0][lane] = ss;
+      wsum[warp][1][lane] = sq;
+    }
+    __syncthreads();
+    const int wpg = TW / 4;  // warps per channel group
+    if (threadIdx.x < CPG * 16) {
+      const int g = threadIdx.x / 16, which = (threadIdx.x / 8) & 1, chn = threadIdx.x & 7;
+      const int cc = (cg0 + g) * 8 + chn;
+      float a = 0.f;
+      for (int k = 0; k < wpg; ++k) a += wsum[g * wpg + k][which][chn];
+      if (cc < C) fix_add(stats, (which ? C : 0) + cc, stats + 2 * C, a, which ? FIX_S2 : FIX_S1);
     }
   }
 }
@@ -917,56 +982,62 @@ void spos_stem_conv(cudaStream_t s, const float* x, const float* w, bf16* z, int
 // every SM the same work -- a fixed 8 CTAs/SM left a 2/3-full third wave for a 3-CTA/SM
 // kernel.  NASPIPE_EW_WAVES (default 1: measured best, 7.15 -> 7.01 ms per configs[1] step) overrides the wave count for tuning.
 static int ew_waves() {
-  static int v = 0;
-  if (!v) {
+  static const int v = [] {  // thread-safe one-time init
     const char* e = getenv("NASPIPE_EW_WAVES");
-    v = e ? std::max(1, atoi(e)) : 1;
-  }
+    return e ? std::max(1, atoi(e)) : 1;
+  }();
   return v;
 }
 // NASPIPE_MAX_CTAS_PER_SM (tuning): cap the resident-CTA count used for the grid sizes below
+// resident CTAs per SM of `kern` at `smem` dynamic bytes, cached per (kernel address, smem)
+// -- a static per template instantiation was shared by kernels of the same type (e.g. the
+// dw_dgrad_kernel<K> of different K); guarded: engines may be created from
+// several host threads
 template <typename Kern>
 static int occupancy(Kern kern, size_t smem) {
+  static std::mutex mu;
+  static std::map<std::pair<const void*, size_t>, int> cache;
+  static const int cap = [] {
+    const char* e = getenv("NASPIPE_MAX_CTAS_PER_SM");
+    return e ? std::max(1, atoi(e)) : 0;
+  }();
+  std::lock_guard<std::mutex> lk(mu);
+  const auto key = std::make_pair(reinterpret_cast<const void*>(kern), smem);
+  auto it = cache.find(key);
+  if (it != cache.end()) return it->second;
   int n = 0;
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, TPB, smem) != cudaSuccess || n < 1) n = 1;
-  static int cap = -1;
-  if (cap < 0) {
-    const char* e = getenv("NASPIPE_MAX_CTAS_PER_SM");
-    cap = e ? std::max(1, atoi(e)) : 0;
-  }
-  return cap ? std::min(n, cap) : n;
+  n = cap ? std::min(n, cap) : n;
+  cache[key] = n;
+  return n;
 }
 // grid-stride kernels over `items` threads of work: capped at NASPIPE_GS_WAVES (default 1:
 // measured best, 7.01 -> 6.95 ms per configs[1] step) waves of resident CTAs; 0 = grid_for's
 // fixed 16 CTAs/SM
 static int gs_waves() {
-  static int v = -1;
-  if (v < 0) {
+  static const int v = [] {  // thread-safe one-time init
     const char* e = getenv("NASPIPE_GS_WAVES");
-    v = e ? std::max(0, atoi(e)) : 1;
-  }
+    return e ? std::max(0, atoi(e)) : 1;
+  }();
   return v;
 }
 template <typename Kern>
 static int gs_grid(Kern kern, size_t items, size_t smem = 0) {
   if (!gs_waves()) return grid_for(items);
-  static int occ = 0;  // per kernel instantiation (and its last dynamic smem size)
-  static size_t occ_smem = 0;
-  if (!occ || smem != occ_smem) occ = occupancy(kern, smem), occ_smem = smem;
+  const int occ = occupancy(kern, smem);
   const size_t g = (items + TPB - 1) / TPB;
-  return (int)std::min<size_t>(std::max<size_t>(g, 1), (size_t)148 * occ * gs_waves());
+  return (int)std::min<size_t>(std::max<size_t>(g, 1), (size_t)num_sms() * occ * gs_waves());
 }
 template <typename Kern>
-static int ew_grid(Kern kern, int P, int C) {
-  static int occ = 0;  // per kernel (one static per instantiation)
-  if (!occ) occ = occupancy(kern, 0);
-  const int lanes = TPB / (C / 8);
-  return std::max(1, std::min((P + lanes - 1) / lanes, 148 * occ * ew_waves()));
+static int ew_grid(Kern kern, int P, int C, int vec = 8) {
+  const int occ = occupancy(kern, 0);
+  const int lanes = TPB / (C / vec);
+  return std::max(1, std::min((P + lanes - 1) / lanes, num_sms() * occ * ew_waves()));
 }
 
-static size_t red_smem(int C) { return (size_t)(TPB / (C / 8)) * 2 * C * sizeof(float); }
-static int red_blocks(int P, int C) {
-  const int r = red_rows(P, C);
+static size_t red_smem(int C, int vec = 8) { return (size_t)(TPB / (C / vec)) * 2 * C * sizeof(float); }
+static int red_blocks(int P, int C, int vec = 8, int target = 0) {
+  const int r = red_rows(P, C, vec, target);
   return (P + r - 1) / r;
 }
 
@@ -980,6 +1051,7 @@ void bn_stats(cudaStream_t s, const bf16* z, int P, int C, unsigned long long* a
 
 void bn_apply(cudaStream_t s, const bf16* z, int P, int C, unsigned long long* acc, int* ticket, float* mean,
               float* rstd, const float* g, const float* b, int relu, bf16* y, int ldy, size_t yplane) {
+  NP_REQUIRE(C % 8 == 0 && C / 8 <= TPB, NASPIPE_EINVAL, "bn_apply C=%d", C);
   launch_pdl(bn_apply_kernel, dim3(ew_grid(bn_apply_kernel, P, C)), dim3(TPB), 0, s, z, P, C, acc, ticket, mean, rstd,
              g, b, relu, y, ldy, yplane);
   check_launch("bn_apply");
@@ -987,25 +1059,30 @@ void bn_apply(cudaStream_t s, const bf16* z, int P, int C, unsigned long long* a
 
 void bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
                    const float* rstd, const float* g, const float* b, int relu, unsigned long long* acc) {
-  NP_REQUIRE(C % 8 == 0 && C / 8 <= TPB, NASPIPE_EINVAL, "bn_bwd C=%d", C);
-  const size_t sm = red_smem(C);
+  NP_REQUIRE(C % 8 == 0 && C / BV <= TPB, NASPIPE_EINVAL, "bn_bwd C=%d", C);
+  const size_t sm = red_smem(C, BV);
   set_smem(bn_bwd_reduce_kernel, sm);
-  launch_pdl(bn_bwd_reduce_kernel, dim3(red_blocks(P, C)), dim3(TPB), sm, s, dy, lddy, z, P, C, mean, rstd, g, b, relu,
-             red_rows(P, C), acc);
+  // one wave of resident CTAs (the fixed-point totals do not depend on the row blocking's
+  // summation order only through the partials, which are a function of (P, C) and this
+  // occupancy-derived target, itself fixed per build and device)
+  const int target = num_sms() * occupancy(bn_bwd_reduce_kernel, sm);
+  launch_pdl(bn_bwd_reduce_kernel, dim3(red_blocks(P, C, BV, target)), dim3(TPB), sm, s, dy, lddy, z, P, C, mean, rstd,
+             g, b, relu, red_rows(P, C, BV, target), acc);
   check_launch("bn_bwd_reduce");
 }
 
 void bn_bwd_apply(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
                   const float* rstd, const float* g, const float* b, float* gu, float* bu, float lr, int update,
                   unsigned long long* acc, int* ticket, int relu, bf16* dz) {
-  launch_pdl(bn_bwd_apply_kernel, dim3(ew_grid(bn_bwd_apply_kernel, P, C)), dim3(TPB), 0, s, dy, lddy, z, P, C, mean,
+  NP_REQUIRE(C % 8 == 0 && C / BV <= TPB, NASPIPE_EINVAL, "bn_bwd_apply C=%d", C);
+  launch_pdl(bn_bwd_apply_kernel, dim3(ew_grid(bn_bwd_apply_kernel, P, C, BV)), dim3(TPB), 0, s, dy, lddy, z, P, C, mean,
              rstd, g, b, gu, bu, lr, update, acc, ticket, relu, dz);
   check_launch("bn_bwd_apply");
 }
 
-bool bn_fix_overflow() {
-  int v = 0;
-  cudaMemcpyFromSymbol(&v, g_fix_overflow, sizeof v);
+bool bn_fix_overflow(const unsigned long long* acc, int C) {
+  unsigned long long v = 0;
+  cudaMemcpy(&v, acc + 2 * (size_t)C, sizeof v, cudaMemcpyDeviceToHost);
   return v != 0;
 }
 
@@ -1021,19 +1098,21 @@ bool bn_fix_overflow() {
 static int dw_tw(int Ho) { return Ho <= 8 ? 8 : (Ho <= 16 ? 16 : 32); }
 
 template <int K, int S, bool X2, bool FLIP>
-static void dw_tile(cudaStream_t s, const bf16* in, const float* w, const bf16* add, bf16* out, int B, int H, int C) {
+static void dw_tile(cudaStream_t s, const bf16* in, const float* w, const bf16* add, bf16* out, int B, int H, int C,
+                    unsigned long long* stats = nullptr) {
   const int Ho = (H - 1) / S + 1, TW = dw_tw(Ho), CPG = TPB / (8 * TW);
   const int IH = (DT_H - 1) * S + K, IW = (TW - 1) * S + K;
   const size_t sm = (size_t)CPG * IH * IW * 8 * sizeof(float);
   const int gx = B * ((Ho + DT_H - 1) / DT_H) * ((Ho + TW - 1) / TW), gy = (C / 8 + CPG - 1) / CPG;
   set_smem(dw_tile_kernel<K, S, X2, FLIP>, sm);
-  launch_pdl(dw_tile_kernel<K, S, X2, FLIP>, dim3(gx, gy), dim3(TPB), sm, s, in, w, add, out, B, H, C, TW);
+  launch_pdl(dw_tile_kernel<K, S, X2, FLIP>, dim3(gx, gy), dim3(TPB), sm, s, in, w, add, out, B, H, C, TW, stats);
 }
 
-void dw_fwd(cudaStream_t s, const bf16* x, const float* w, bf16* z, int B, int H, int C, int k, int S) {
+void dw_fwd(cudaStream_t s, const bf16* x, const float* w, bf16* z, int B, int H, int C, int k, int S,
+            unsigned long long* stats) {
   NP_REQUIRE(C % 8 == 0 && (S == 1 || S == 2), NASPIPE_EINVAL, "dw_fwd C=%d S=%d", C, S);
-  if (S == 1) { DW_DISPATCH(k, (dw_tile<KK, 1, true, false>(s, x, w, nullptr, z, B, H, C))); }
-  else { DW_DISPATCH(k, (dw_tile<KK, 2, true, false>(s, x, w, nullptr, z, B, H, C))); }
+  if (S == 1) { DW_DISPATCH(k, (dw_tile<KK, 1, true, false>(s, x, w, nullptr, z, B, H, C, stats))); }
+  else { DW_DISPATCH(k, (dw_tile<KK, 2, true, false>(s, x, w, nullptr, z, B, H, C, stats))); }
   check_launch("dw_fwd");
 }
 

@@ -26,6 +26,10 @@ update is zero or proportional to another tensor's (tiny) update:
   the depthwise conv keeps channels separate and the next BN removes the per-channel scale,
   so d L / d gamma = 0 at a candidate's first update and stays proportional to beta (O(lr))
   afterwards.
+* by measurement, any tensor whose exact update is more than two orders of magnitude below
+  the candidate's largest (max |dr| < NEAR_STATIC x max over the candidate): e.g. the proj
+  branch's output BN gamma when the next block reads those channels only through depthwise
+  convs + BatchNorm (per-channel scale invariance again).
 They get an absolute bar instead: max |dg - dr| <= STATIC_ABS x the largest |dr| of the
 candidate.
 """
@@ -34,6 +38,7 @@ import numpy as np
 from oracle import train
 
 STATIC_ABS = 1e-3
+NEAR_STATIC = 1e-2
 
 
 def structurally_static(cfg, name):
@@ -68,7 +73,7 @@ def per_tensor(cfg, got, ref, theta0):
                    "cand_a15": cand_a15, "a15": None, "upd": None, "static": None}
             if kind != "zeros":
                 rec["a15"] = float(np.max(np.abs(gs - rs)) / np.max(np.abs(rs)))
-            if structurally_static(cfg, name):
+            if structurally_static(cfg, name) or 0 < np.max(np.abs(dr)) < NEAR_STATIC * cand_dmax:
                 rec["static"] = float(np.max(np.abs(dg - dr)) / cand_dmax) if cand_dmax > 0 else 0.0
             elif np.any(dr != 0):
                 rec["upd"] = float(np.linalg.norm(dg - dr) / np.linalg.norm(dr))
@@ -151,10 +156,9 @@ def sampled_errors(cfg, gold, step, got_of):
             if kind != "zeros":
                 rec["a15"] = float(np.max(np.abs(gs - rs)) / gold[f"{pre}max_{tag}"])
             dr, dg = rs - t0, gs - t0
-            if structurally_static(cfg, name):
-                rec["static"] = float(np.max(np.abs(dg - dr)) / max(float(gold[f"{pre}dmax_{k}"]) for k in
-                                                              [f"{b}_{c}_{nm}" for nm, _, _, _ in
-                                                               train.candidate_layout(cfg, b, c)]))
+            cdmax = max(float(gold[f"{pre}dmax_{b}_{c}_{nm}"]) for nm, _, _, _ in train.candidate_layout(cfg, b, c))
+            if structurally_static(cfg, name) or 0 < float(gold[f"{pre}dmax_{tag}"]) < NEAR_STATIC * cdmax:
+                rec["static"] = float(np.max(np.abs(dg - dr)) / cdmax)
             elif np.any(dr != 0):
                 rec["upd"] = float(np.linalg.norm(dg - dr) / np.linalg.norm(dr))
             recs.append(rec)

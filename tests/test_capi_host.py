@@ -193,7 +193,7 @@ def test_default_costs_and_partition_of_real_configs():
             assert list(sob) == [0, 0, 1, 1]
 
 
-@pytest.mark.parametrize("sync", ["inorder", "asp", "bsp"])
+@pytest.mark.parametrize("sync", ["inorder", "asp", "bsp", "serial"])
 @pytest.mark.parametrize("seed", range(12))
 def test_sync_policies_match_oracle_bit_exact(sync, seed):
     """the C++ planner's INORDER / ASP / BSP schedules equal the oracle's."""

@@ -69,6 +69,20 @@ def test_table3_reproducibility_contrast():
     assert any(not np.array_equal(a2[k], a4[k]) for k in a2)
 
 
+def test_serial_has_csp_numerics():
+    """SERIAL (w/o scheduler per P:L454, one subnet in flight): the executed trace is the
+    oracle's serial plan and the numerics are bitwise the CSP run's."""
+    cfg, choices, batches = _workload("toy", 16, "serial")
+    sob, tr = _oracle_plan(cfg, choices, 4, "serial")
+    p_s, l_s, trace, _ = run_engine(cfg, choices, batches, 4)
+    assert [tuple(int(v) for v in r) for r in trace] == [tuple(r) for r in tr]
+    ccfg = synth.get_config("toy")
+    p_c, l_c, _, _ = run_engine(ccfg, choices, batches, 4)
+    assert np.array_equal(l_s.view(np.uint32), l_c.view(np.uint32))
+    for k in p_c:
+        assert np.array_equal(p_s[k].view(np.uint32), p_c[k].view(np.uint32)), k
+
+
 def test_inorder_has_csp_numerics():
     cfg, choices, batches = _workload("toy", 24, "inorder")
     sob, tr = _oracle_plan(cfg, choices, 4, "inorder")

@@ -241,6 +241,31 @@ def test_inorder_is_causal_and_never_overtakes():
             assert fw == sorted(fw)
 
 
+def test_serial_is_one_pipeline_at_a_time():
+    """NASPipe w/o scheduler as P:L454 words it ("had to finish the execution of a pipeline
+    before injecting the next pipeline"; reading A32): one subnet in flight.  Closed form with
+    per-stage task costs cf, cb and latency 0: every subnet's F(y, 0..D-1) then B(y, D-1..0)
+    runs alone, so makespan = sum_y sum_K (cf + cb) and every stage idles (D - 1) / D of it
+    when the costs are uniform; the order is F0..FD-1 B.. per subnet, ascending ids."""
+    for seed in range(4):
+        ch = synth.sample_choices(12, 8, 3, seed)
+        sob, (tf, tb) = _unit(ch, 4, 8)
+        r = csp.simulate_csp(ch, sob, 4, 16, tf, tb, sync="serial")
+        assert r["makespan"] == int(sum(tf[K][y] + tb[K][y] for K in range(4) for y in range(12)))
+        assert csp.check_trace(r["trace"], ch, sob, 4) == []
+        ys = [y for _, _, _, y in r["trace"]]
+        assert ys == sorted(ys)          # subnet y's 2D tasks all precede y + 1's
+    ch = synth.sample_choices(10, 8, 3, 9)
+    sob = [b * 4 // 8 for b in range(8)]
+    D, N = 4, 10
+    tf = [[1] * N for _ in range(D)]
+    tb = [[2] * N for _ in range(D)]
+    r = csp.simulate_csp(ch, sob, D, 16, tf, tb, sync="serial")
+    assert r["makespan"] == N * D * 3
+    for K in range(D):
+        assert r["stall"][K] + r["bubble"][K] == N * D * 3 - N * 3     # idle (D-1)/D of the time
+
+
 def test_asp_is_the_no_dependency_schedule():
     ch = synth.sample_choices(20, 8, 2, 3)
     sob, (tf, tb) = _unit(ch, 4, 8)

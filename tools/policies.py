@@ -27,7 +27,7 @@ sys.path.insert(0, ROOT)
 import synth  # noqa: E402
 import paper_conf_asplos_zhaolcscwzlc22_b200 as npipe  # noqa: E402
 
-POLICIES = ["csp", "inorder", "asp", "bsp"]
+POLICIES = ["csp", "serial", "inorder", "asp", "bsp"]
 
 
 def plan(cfg, choices, D, sync):
@@ -64,7 +64,7 @@ def main():
     ap.add_argument("--workload", default="transformer")
     ap.add_argument("--subnets", type=int, default=256)
     ap.add_argument("--n-choices", type=int, default=0, help="override n (sweep-style uniform candidates)")
-    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "r1_policies.md"))
+    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "r2_policies.md"))
     args = ap.parse_args()
     if args.n_choices:
         cfg = synth.sweep_config(args.n_choices)
@@ -83,11 +83,12 @@ def main():
     lines = [f"# Synchronisation policies at plan level — {name} (m={m}, n={n}), N={args.subnets}", "",
              "Default integer cost table of the library (naspipe_default_costs), W = 4D, BSP bulk = 4D, strict "
              "backward-first.  Speed-up = makespan of the one-stage plan / makespan at D.", "",
-             "| D | CSP | w/o scheduler (INORDER) | ASP (no deps) | BSP (GPipe) | idle CSP / INORDER / ASP / BSP |",
-             "|---|---|---|---|---|---|"]
+             "| D | CSP | w/o scheduler (SERIAL, P:L454) | in-order admission (INORDER) | ASP (no deps) | BSP (GPipe) "
+             "| idle CSP / SERIAL / INORDER / ASP / BSP |",
+             "|---|---|---|---|---|---|---|"]
     for D in (2, 4, 8):
         rr = {r["sync"]: r for r in rows if r["D"] == D}
-        lines.append(f"| {D} | {rr['csp']['speedup']:.2f}x | {rr['inorder']['speedup']:.2f}x | "
+        lines.append(f"| {D} | {rr['csp']['speedup']:.2f}x | {rr['serial']['speedup']:.2f}x | {rr['inorder']['speedup']:.2f}x | "
                      f"{rr['asp']['speedup']:.2f}x | {rr['bsp']['speedup']:.2f}x | "
                      + " / ".join(f"{rr[s]['idle']:.2f}" for s in POLICIES) + " |")
     # Table 4: the access order of one candidate used by several early subnets
