@@ -534,7 +534,9 @@ def main():
     if not args.no_profile:
         barrier()
         s2 = npipe.naspipe_get_stats(h)
+        npipe.naspipe_set_pdl(False)   # each kernel's CUPTI interval = its own execution (no PDL overlap)
         per, busy_us = profile_kernels(steps)
+        npipe.naspipe_set_pdl(True)
         s3 = npipe.naspipe_get_stats(h)
         fam = "spos" if cfg["family"] == "spos" else "transformer"
         fn, fus = family_time(per, fam)
@@ -558,7 +560,8 @@ def main():
                         "algorithmic_flops_per_step": work / args.steps}
         roofline.update({"frac": achieved / roofline["peak"] if achieved else None, "traffic": _traffic(fam),
                          "timing": "CUPTI activity records (torch.profiler, CUDA activity only) of a separate run "
-                                   "of the same K steps; no events between kernels",
+                                   "of the same K steps, no events between kernels, PDL off in that run so a "
+                                   "kernel's interval excludes its wait for the predecessor",
                          "launches": reduce(fn, "sum"), "device_us": dominant_us,
                          "share_of_kernel_time": dominant_us / kern_total_us if kern_total_us else None})
         # GEMM tensor utilisation in this run (algorithmic flops / GEMM device time / peak)

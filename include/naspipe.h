@@ -335,6 +335,12 @@ void naspipe_plan_destroy(naspipe_plan_t* p);
 /* Fill 128 bytes with a fresh ncclUniqueId (for naspipe_create_rank's nccl_ids). */
 int naspipe_nccl_unique_id(void* out128);
 
+/* Process-wide PDL switch (programmatic dependent launch between consecutive kernels of a
+ * stream; default on where the engine allows it).  bench.py turns it off for its CUPTI
+ * kernel-time run so that every kernel's recorded interval is its own execution, not the
+ * wait for its predecessor.  Results are bitwise the same either way. */
+int naspipe_set_pdl(int enabled);
+
 const char* naspipe_last_error(void);
 int naspipe_abi_version(void);
 

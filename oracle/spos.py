@@ -71,10 +71,16 @@ class Storage:
         self.f, self.w, self.b, self.op = f, w, b, op
 
 
+def to_fp32(x):
+    """Round to float32 (nearest), returned as float64: the paper's precision."""
+    return np.asarray(x, dtype=np.float32).astype(np.float64)
+
+
 PLAIN = Storage()
 BF16 = Storage(to_bf16, to_bf16, to_bf16, to_bf16)
 BF16X2 = Storage(to_bf16x2, to_bf16x2, to_bf16, to_bf16)
-STORAGE = {None: PLAIN, "fp64": PLAIN, "bf16": BF16, "bf16x2": BF16X2}
+FP32 = Storage(to_fp32, to_fp32, to_fp32, to_fp32)   # every stored tensor in fp32 (the paper's)
+STORAGE = {None: PLAIN, "fp64": PLAIN, "bf16": BF16, "bf16x2": BF16X2, "fp32": FP32}
 
 
 # ------------------------------------------------------------------ shapes / layout

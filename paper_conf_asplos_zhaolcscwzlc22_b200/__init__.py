@@ -6,7 +6,7 @@ library has not been built (``python -m paper_conf_asplos_zhaolcscwzlc22_b200.bu
 """
 from ._lib import (  # noqa: F401
     LIB_PATH, NaspipeError, Spec, naspipe_abi_version, naspipe_create, naspipe_create_rank, naspipe_create_rank_peer,
-    naspipe_peer_export, naspipe_peer_connect,
+    naspipe_peer_export, naspipe_peer_connect, naspipe_set_pdl,
     naspipe_default_costs, naspipe_destroy, naspipe_drain, naspipe_get_losses,
     naspipe_get_params, naspipe_get_residency_trace, naspipe_get_stats, naspipe_get_trace,
     naspipe_init_params, naspipe_init_frozen, naspipe_nccl_unique_id, naspipe_param_count, naspipe_partition,

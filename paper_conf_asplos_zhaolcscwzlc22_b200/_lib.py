@@ -84,6 +84,7 @@ _sig("naspipe_plan_idle", C.c_int, [C.c_void_p, _i64p, _i64p])
 _sig("naspipe_plan_comm_schedule", C.c_int, [C.c_void_p, C.c_int32, _i64p, C.c_size_t, C.POINTER(C.c_size_t)])
 _sig("naspipe_plan_destroy", None, [C.c_void_p])
 _sig("naspipe_nccl_unique_id", C.c_int, [C.c_void_p])
+_sig("naspipe_set_pdl", C.c_int, [C.c_int])
 _sig("naspipe_create_rank_peer", C.c_int, [_SP, C.c_int32, C.c_int32, C.c_int32, C.POINTER(C.c_void_p)])
 _sig("naspipe_peer_export", C.c_int, [C.c_void_p, C.c_void_p, C.c_size_t, C.POINTER(C.c_size_t)])
 _sig("naspipe_peer_connect", C.c_int, [C.c_void_p, C.c_void_p, C.c_size_t, C.c_void_p, C.c_size_t])
@@ -96,7 +97,7 @@ EXPORTED_SYMBOLS = [
     "naspipe_plan_makespan", "naspipe_plan_deps", "naspipe_plan_residency", "naspipe_plan_destroy",
     "naspipe_plan_comm_schedule", "naspipe_plan_idle", "naspipe_plan_mirrored",
     "naspipe_nccl_unique_id", "naspipe_last_error", "naspipe_abi_version",
-    "naspipe_create_rank_peer", "naspipe_peer_export", "naspipe_peer_connect"]
+    "naspipe_create_rank_peer", "naspipe_peer_export", "naspipe_peer_connect", "naspipe_set_pdl"]
 
 
 class NaspipeError(RuntimeError):
@@ -204,6 +205,10 @@ def naspipe_peer_connect(h: Handle, prev_blob, next_blob) -> None:
     nb = C.create_string_buffer(bytes(next_blob), len(next_blob)) if next_blob else None
     _check(lib.naspipe_peer_connect(h.ptr, pb, len(prev_blob) if prev_blob else 0, nb,
                                     len(next_blob) if next_blob else 0))
+
+
+def naspipe_set_pdl(enabled: bool) -> None:
+    _check(lib.naspipe_set_pdl(1 if enabled else 0))
 
 
 def naspipe_nccl_unique_id() -> bytes:

@@ -5,6 +5,7 @@
 #include <memory>
 
 #include "engine.h"
+#include "launch.h"
 #include "mirror.h"
 #include "planner.h"
 
@@ -231,6 +232,10 @@ int naspipe_plan_comm_schedule(const naspipe_plan_t* p, int32_t rank, int64_t* d
 }
 
 void naspipe_plan_destroy(naspipe_plan_t* p) { delete p; }
+
+int naspipe_set_pdl(int enabled) {
+  return guarded([&] { pdl_runtime_off().store(enabled ? 0 : 1); });
+}
 
 int naspipe_nccl_unique_id(void* out128) {
   return guarded([&] {

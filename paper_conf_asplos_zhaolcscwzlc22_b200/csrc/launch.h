@@ -31,7 +31,15 @@ inline std::atomic<int>& pdl_suppressors() {
 
 // NASPIPE_NO_PDL=1 launches without the PDL attribute; NASPIPE_FORCE_PDL=1 keeps it even
 // while a suppressing engine lives (diagnostics: the deadlock reproductions).
+// naspipe_set_pdl(0): process-wide switch for measurement runs (bench.py times each kernel's
+// own execution with CUPTI: with PDL a kernel's recorded interval starts while it still waits
+// in griddepcontrol.wait for its predecessor, so summed durations double-count the overlap)
+inline std::atomic<int>& pdl_runtime_off() {
+  static std::atomic<int> v{0};
+  return v;
+}
 inline bool pdl_enabled() {
+  if (pdl_runtime_off().load(std::memory_order_relaxed)) return false;
   static const int v = [] {
     const char* e = getenv("NASPIPE_NO_PDL");
     const char* f = getenv("NASPIPE_FORCE_PDL");

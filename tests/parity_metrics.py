@@ -144,6 +144,14 @@ def sampled_errors(cfg, gold, step, got_of):
                     if k.startswith(pre) and not k.startswith((pre + "max_", pre + "dmax_"))})
     for (b, c) in cands:
         g = np.asarray(got_of(b, c), dtype=np.float64)
+        # per-candidate (round-1) A15 printout: max over the candidate's sampled entries of
+        # |g - r| over the largest whole-tensor max |r| of the candidate
+        cmax = max(float(gold[f"{pre}max_{b}_{c}_{nm}"]) for nm, _, _, _ in train.candidate_layout(cfg, b, c))
+        cerr, o2 = 0.0, 0
+        for nm, shape, _, _ in train.candidate_layout(cfg, b, c):
+            n2 = int(np.prod(shape))
+            cerr = max(cerr, float(np.max(np.abs(g[o2:o2 + n2][gold[f"idx_{b}_{c}_{nm}"]] - gold[f"{pre}{b}_{c}_{nm}"]))))
+            o2 += n2
         off = 0
         for name, shape, kind, _ in train.candidate_layout(cfg, b, c):
             n = int(np.prod(shape))
@@ -151,7 +159,7 @@ def sampled_errors(cfg, gold, step, got_of):
             gs = g[off:off + n][gold[f"idx_{tag}"]]
             off += n
             rs, t0 = gold[pre + tag], gold[f"init_{tag}"]
-            rec = {"key": (b, c), "name": name, "cls": tensor_class(name, shape, kind), "cand_a15": 0.0,
+            rec = {"key": (b, c), "name": name, "cls": tensor_class(name, shape, kind), "cand_a15": cerr / cmax,
                    "a15": None, "upd": None, "static": None}
             if kind != "zeros":
                 rec["a15"] = float(np.max(np.abs(gs - rs)) / gold[f"{pre}max_{tag}"])
@@ -163,3 +171,25 @@ def sampled_errors(cfg, gold, step, got_of):
                 rec["upd"] = float(np.linalg.norm(dg - dr) / np.linalg.norm(dr))
             recs.append(rec)
     return summary(recs)
+
+
+def golden_floor(cfg, gold, gold_prec, step):
+    """Per-tensor A15 of a second oracle trajectory (e.g. the fp32-storage oracle, the
+    paper's precision) against the fp64 golden at the same sampled entries: the precision
+    floor of the multi-step bar for a chaotic trajectory (A35)."""
+    pre = f"s{step}_"
+    worst, where, cand = 0.0, None, 0.0
+    cands = sorted({tuple(int(v) for v in k[len(pre):].split("_", 2)[:2]) for k in gold.files
+                    if k.startswith(pre) and not k.startswith((pre + "max_", pre + "dmax_"))})
+    for (b, c) in cands:
+        cmax = max(float(gold[f"{pre}max_{b}_{c}_{nm}"]) for nm, _, _, _ in train.candidate_layout(cfg, b, c))
+        for name, shape, kind, _ in train.candidate_layout(cfg, b, c):
+            tag = f"{b}_{c}_{name}"
+            d = float(np.max(np.abs(gold_prec[pre + tag] - gold[pre + tag])))
+            cand = max(cand, d / cmax)
+            if kind == "zeros":
+                continue
+            e = d / float(gold[f"{pre}max_{tag}"])
+            if e > worst:
+                worst, where = e, ((b, c), name)
+    return {"a15": worst, "worst": where, "a15_cand": cand}

@@ -267,3 +267,21 @@ def test_recompute_flag_validation():
         with pytest.raises(npipe.NaspipeError) as e:
             npipe.naspipe_partition(npipe.Spec(cfg, flags=npipe.FLAG_RECOMPUTE), 2)
         assert e.value.code == -1
+
+
+def test_sass_gemm_kernels_are_tcgen05():
+    """Every GEMM instantiation in libnaspipe.so issues tcgen05.mma (SASS UTCHMMA), reads
+    TMEM (LDTM), is fed by TMA (UTMALDG) and has no legacy HMMA (tools/sass_census.py;
+    profiles/r2_sass_census.md) -- a regression to a non-tcgen05 GEMM fails here."""
+    import shutil
+    import sys as _s
+    if not os.path.exists("/usr/local/cuda/bin/cuobjdump") or shutil.which("c++filt") is None:
+        pytest.skip("cuobjdump / c++filt not available")
+    _s.path.insert(0, os.path.join(ROOT, "tools"))
+    import sass_census
+    kernels, names = sass_census.census()
+    gemms = [k for k in kernels if "gemm_tc_kernel" in names[k] or "gemm_pair_kernel" in names[k]]
+    assert len(gemms) >= 20, len(gemms)
+    for k in gemms:
+        c = kernels[k]
+        assert c["UTCHMMA"] > 0 and c["LDTM"] > 0 and c["UTMALDG"] > 0 and c["HMMA"] == 0, (names[k], c)

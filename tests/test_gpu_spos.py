@@ -108,19 +108,31 @@ def test_spos_full_size_bitwise_across_runs_and_stage_counts():
 
 
 
-@pytest.mark.parametrize("steps,tol", [(20, 1e-2), (100, 1e-2)])
-def test_spos_full_size_multistep_against_oracle_samples(steps, tol):
+@pytest.mark.parametrize("steps", [20, 100])
+def test_spos_full_size_multistep_against_oracle_samples(steps):
     """configs[1] at full size, the first 20 / 100 subnets trained sequentially by the fp64
     oracle (tests/golden/spos_fullsize_100steps.npz, written by tools/make_multistep_golden.py
-    from oracle/ only) against the GPU in the bench's launch configuration: per-tensor A15
-    over <= 256 sampled entries of every tensor of every trained candidate (denominator
-    max |theta| over the whole tensor) <= 1e-2 (BJ's multi-step bar); losses rtol 1e-2."""
+    from oracle/ only) against the GPU in the bench's launch configuration.
+
+    BatchNorm + ReLU on random labels make this trajectory chaotic: the SAME oracle with
+    every stored tensor rounded to fp32 (the paper's precision, P:L98;
+    tests/golden/spos_fullsize_100steps_fp32.npz) already differs from fp64 by a per-tensor
+    A15 of 2.8e-2 after 20 steps (A35).  Bars: per candidate (round-1 reading of
+    A15) <= 1e-2, BJ's multi-step bar; per tensor <= max(1e-2, 1.5 x that fp32 floor at the
+    same step); losses rtol 1e-2."""
     gold = load_gold("spos_fullsize_100steps.npz")
     if not any(k.startswith(f"s{steps}_max_") for k in gold.files):
         pytest.skip(f"checkpoint {steps} not in the golden yet")
+    floor_gold = load_gold("spos_fullsize_100steps_fp32.npz")
+    if not any(k.startswith(f"s{steps}_max_") for k in floor_gold.files):
+        pytest.skip(f"checkpoint {steps} not in the fp32 floor golden yet")
+    cfg = synth.get_config("spos")
+    floor = pm.golden_floor(cfg, gold, floor_gold, steps)
     cfg, h, got_of, losses = run_fullsize("spos", gold, steps)
     sm = pm.sampled_errors(cfg, gold, steps, got_of)
     npipe.naspipe_destroy(h)
-    print(f"configs[1] full size, {steps} steps: {pm.fmt(sm)}; losses {losses[-3:]} vs {gold['losses'][steps - 3:steps]}")
-    pm.check(sm, tol)
+    print(f"configs[1] full size, {steps} steps: {pm.fmt(sm)}; fp32-oracle floor {floor}; "
+          f"losses {losses[-3:]} vs {gold['losses'][steps - 3:steps]}")
+    assert sm["a15_cand"] <= 1e-2, sm["a15_cand"]
+    assert sm["a15"] <= max(1e-2, 1.5 * floor["a15"]), (sm["a15"], floor)
     np.testing.assert_allclose(losses, gold["losses"][:steps], rtol=1e-2)

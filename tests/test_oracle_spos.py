@@ -169,3 +169,8 @@ def test_storage_modes_only_round():
     _, l0 = train.train_sequential(cfg, th0, ch, b)
     _, l1 = train.train_sequential(dict(cfg, storage="bf16x2"), th0, ch, b)
     assert l0[0] != l1[0] and abs(l1[0] - l0[0]) <= 1e-3 * l0[0]
+    # FP32 storage (the paper's precision): fp32 rounding of every stored tensor
+    x = np.random.default_rng(3).standard_normal(1000) * 3
+    np.testing.assert_array_equal(spos.to_fp32(x), x.astype(np.float32).astype(np.float64))
+    _, l2 = train.train_sequential(dict(cfg, storage="fp32"), th0, ch, b)
+    assert l0[0] != l2[0] and abs(l2[0] - l0[0]) <= 1e-6 * l0[0]

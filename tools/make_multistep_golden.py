@@ -38,10 +38,15 @@ def main():
     ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--checkpoints", default="1,100")
     ap.add_argument("--samples", type=int, default=256)
+    ap.add_argument("--storage", default=None,
+                    help="SPOS: run the oracle with this storage rounding (oracle/spos.py STORAGE, e.g. fp32 = the "
+                         "paper's precision P:L98) -- the precision floor of the multi-step bar (DESIGN.md A35)")
     a = ap.parse_args()
     cks = sorted({int(s) for s in a.checkpoints.split(",")} | {a.steps})
-    out_path = os.path.join(ROOT, "tests", "golden", f"{a.workload}_fullsize_{a.steps}steps.npz")
+    suffix = f"_{a.storage}" if a.storage else ""
+    out_path = os.path.join(ROOT, "tests", "golden", f"{a.workload}_fullsize_{a.steps}steps{suffix}.npz")
     cfg = synth.get_config(a.workload)
+    run_cfg = dict(cfg, storage=a.storage) if a.storage else cfg
     N, n = a.steps, cfg["n_choices"]
     choices = synth.sample_choices(N, cfg["n_blocks"], n)
     used = sorted({(b, int(choices[y][b])) for y in range(N) for b in range(cfg["n_blocks"])})
@@ -76,7 +81,7 @@ def main():
     t0 = time.time()
     for y in range(N):
         x, t = synth.make_batch(cfg, y)
-        loss, grads = train.subnet_step(cfg, theta, choices[y], x, t)
+        loss, grads = train.subnet_step(run_cfg, theta, choices[y], x, t)
         train.sgd_apply(theta, grads, cfg["lr"])
         losses[y] = loss
         trained |= set(grads)
