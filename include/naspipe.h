@@ -93,6 +93,18 @@ typedef enum { NASPIPE_FP32 = 0, NASPIPE_BF16 = 1 } naspipe_dtype; /* compute dt
  * update a candidate between F(y) and B(y), so results are bitwise those without it.
  * TRANSFORMER family only, not with ASP (EINVAL otherwise). */
 #define NASPIPE_FLAG_RECOMPUTE 16
+/* Executed layer mirroring (P:L166 per-subnet balanced partitions, P:L298
+ * "Layer Mirroring ... the new parameters are actively pushed to all the other mirrored
+ * ones"; reading A31): subnet y runs its blocks on the stages of ITS OWN balanced
+ * partition (naspipe_plan_mirrored's schedule, mirror latency = link_latency), every stage
+ * holds a mirror copy of every candidate, and after each backward's SGD WRITE the updated
+ * fp32 master and bf16 shadow are pushed to the other stages' copies on a push stream; a task
+ * that reads a candidate last written on another stage waits for that push.  Numerics are the
+ * sequential result (CSP).  naspipe_create only (single process), CSP with strict
+ * backward-first, every candidate resident, no recompute (EINVAL otherwise).  Tasks are
+ * planned and issued at naspipe_drain (the mirrored plan is computed over the submitted
+ * stream). */
+#define NASPIPE_FLAG_MIRROR 32
 
 /*
  * Supernet specification.  naspipe_create deep-copies it and every array it points to.

@@ -11,6 +11,6 @@ from ._lib import (  # noqa: F401
     naspipe_get_params, naspipe_get_residency_trace, naspipe_get_stats, naspipe_get_trace,
     naspipe_init_params, naspipe_init_frozen, naspipe_nccl_unique_id, naspipe_param_count, naspipe_partition,
     naspipe_plan, naspipe_plan_mirrored, naspipe_set_params, naspipe_set_timing, naspipe_submit, lib, BATCH_HOST, BATCH_DEVICE,
-    BATCH_SYNTHETIC, FLAG_TRACE, FLAG_VERSION_CHECK, FLAG_NULL_KERNELS, FLAG_TIMING, FLAG_RECOMPUTE,
+    BATCH_SYNTHETIC, FLAG_TRACE, FLAG_VERSION_CHECK, FLAG_NULL_KERNELS, FLAG_TIMING, FLAG_RECOMPUTE, FLAG_MIRROR,
     STATS_FIELDS, EXPORTED_SYMBOLS,
 )

@@ -15,7 +15,7 @@ SYNC = {"csp": 0, "inorder": 1, "asp": 2, "bsp": 3, "serial": 4}  # naspipe_sync
 FAMILY = {"mlp": 0, "transformer": 1, "spos": 2}
 DTYPE = {"fp32": 0, "bf16": 1}
 BATCH_HOST, BATCH_DEVICE, BATCH_SYNTHETIC = 0, 1, 2
-FLAG_TRACE, FLAG_VERSION_CHECK, FLAG_NULL_KERNELS, FLAG_TIMING, FLAG_RECOMPUTE = 1, 2, 4, 8, 16
+FLAG_TRACE, FLAG_VERSION_CHECK, FLAG_NULL_KERNELS, FLAG_TIMING, FLAG_RECOMPUTE, FLAG_MIRROR = 1, 2, 4, 8, 16, 32
 STATS_FIELDS = ["tasks", "kernel_launches", "h2d_bytes", "d2h_bytes", "p2p_bytes", "makespan_ticks",
                 "dominant_launches", "dominant_flops", "dominant_ms", "res_loads", "res_evicts",
                 "writebacks", "version_checks", "gemm_flops", "gemm_launches", "r15"]

@@ -15,9 +15,8 @@ namespace naspipe {
   } while (0)
 
 CandidateStore::CandidateStore(const Spec& spec, const Planner& planner, int K, int dev, Family* fam,
-                               DevArena* arena, int64_t budget)
+                               DevArena* arena, int64_t budget, const std::vector<int>& blocks)
     : spec_(spec), planner_(planner), K_(K), dev_(dev), n_(spec.n()), fam_(fam), budget_(budget) {
-  const auto& blocks = planner.blocks_of(K);
   cands_.resize((size_t)spec.m() * n_);
   std::vector<int> uids;
   for (size_t j = 0; j < blocks.size(); ++j)

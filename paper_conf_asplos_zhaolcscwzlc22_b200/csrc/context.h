@@ -24,8 +24,10 @@ namespace naspipe {
 
 class CandidateStore {
  public:
+  // blocks: the blocks this stage holds candidates of (the planner's partition, or every
+  // block under layer mirroring)
   CandidateStore(const Spec& spec, const Planner& planner, int K, int dev, Family* fam, DevArena* arena,
-                 int64_t budget);
+                 int64_t budget, const std::vector<int>& blocks);
   ~CandidateStore();
   bool managed() const { return budget_ > 0; }
 
@@ -46,6 +48,11 @@ class CandidateStore {
   // masters and refreshes their bf16 shadows on stream s.
   void enable_bsp(DevArena* arena);
   void bsp_flush(cudaStream_t s);
+  // device copy of candidate (b, c) (resident mode): fp32 master, bf16 shadow and their sizes
+  float* dev_master(int b, int c) { return cands_[uid_of(b, c)].w32; }
+  bf16* dev_shadow(int b, int c) { return cands_[uid_of(b, c)].w16; }
+  size_t n32(int b, int c) const { return cands_[uid_of(b, c)].n32; }
+  size_t n16(int b, int c) const { return cands_[uid_of(b, c)].n16; }
   // read-out (streams idle)
   void get(int b, int c, float* dst);
   void set(int b, int c, const float* src, cudaStream_t s);

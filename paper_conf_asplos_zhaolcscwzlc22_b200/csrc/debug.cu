@@ -111,14 +111,17 @@ int naspipe_debug_dw(const void* x, const float* w, void* z, const void* dz, con
     if (x && z) dw_fwd(s, (const bf16*)x, w, (bf16*)z, B, H, C, k, S);
     if (dz && dx) dw_dgrad(s, (const bf16*)dz, w, (const bf16*)add, (bf16*)dx, B, H, C, k, S);
     if (dz && x && dwsum) {
-      const int nblk = dw_wgrad_blocks(B, H, C, k, S);
-      float* part = nullptr;
-      NP_REQUIRE(cudaMalloc(&part, (size_t)nblk * C * k * k * 4) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
-      dw_wgrad(s, (const bf16*)dz, (const bf16*)x, part, B, H, C, k, S);
+      unsigned long long* acc = nullptr;
+      int* ticket = nullptr;
+      NP_REQUIRE(cudaMalloc(&acc, ((size_t)C * k * k + 1) * 8) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
+      NP_REQUIRE(cudaMalloc(&ticket, 4) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
+      cudaMemsetAsync(acc, 0, ((size_t)C * k * k + 1) * 8, s);
+      cudaMemsetAsync(ticket, 0, 4, s);
       cudaMemsetAsync(dwsum, 0, (size_t)C * k * k * 4, s);
-      sgd_from_partials(s, dwsum, part, nblk, C * k * k, -1.0f);  // 0 - (-1) * sum = sum
+      dw_wgrad_sgd(s, (const bf16*)dz, (const bf16*)x, acc, ticket, dwsum, -1.0f, B, H, C, k, S);  // 0 + sum
       cudaStreamSynchronize(s);
-      cudaFree(part);
+      cudaFree(acc);
+      cudaFree(ticket);
     }
   });
 }

@@ -12,6 +12,7 @@
 
 #include "engine.h"
 #include "launch.h"
+#include "mirror.h"
 
 namespace naspipe {
 
@@ -115,11 +116,29 @@ std::unique_ptr<Engine> Engine::create_local(const Spec& spec, int D) {
   CU(cudaGetDeviceCount(&ndev));
   NP_REQUIRE(ndev >= 1, NASPIPE_ECUDA, "no CUDA device");
   CU(cudaGetDevice(&cur));
+  const bool mirror = (spec.raw.flags & NASPIPE_FLAG_MIRROR) != 0;
+  NP_REQUIRE(!mirror || (spec.raw.sync_policy == NASPIPE_SYNC_CSP && spec.raw.bwd_policy == 0 &&
+                         spec.raw.hbm_weight_budget_bytes == 0 && !(spec.raw.flags & NASPIPE_FLAG_RECOMPUTE)),
+             NASPIPE_EINVAL, "layer mirroring: CSP, strict backward-first, all candidates resident, no recompute");
   std::unique_ptr<Engine> e(new Engine(spec, D));
+  e->mirror_ = mirror;
   e->st_.resize(D);
   e->stage_sizes();
   for (int K = 0; K < D; ++K) e->setup_stage(K, (cur + K) % ndev, true);
   e->link_local_buffers();
+  if (mirror) {
+    const size_t nc = (size_t)spec.m() * spec.n();
+    e->mwriter_.assign(nc, -1);
+    e->ev_push_.resize(nc);
+    for (auto& ev : e->ev_push_) CU(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+    e->push_.resize(D);
+    e->ev_wrote_.resize(D);
+    for (int K = 0; K < D; ++K) {
+      CU(cudaSetDevice(e->st_[K].dev));
+      CU(cudaStreamCreateWithFlags(&e->push_[K], cudaStreamNonBlocking));
+      CU(cudaEventCreateWithFlags(&e->ev_wrote_[K], cudaEventDisableTiming));
+    }
+  }
   CU(cudaSetDevice(cur));
   return e;
 }
@@ -285,6 +304,20 @@ void Engine::peer_connect(const void* prev, size_t prev_n, const void* next, siz
 // Boundary tensor sizes of every stage (also of the non-local ones: a rank posts receives
 // sized by its neighbours' outputs).
 void Engine::stage_sizes() {
+  if (spec_.raw.flags & NASPIPE_FLAG_MIRROR) {  // a stage boundary may fall at any block boundary
+    size_t a = 0, g = 0;
+    for (int b = 1; b < spec_.m(); ++b) {
+      a = std::max(a, spec_.act_bytes(b));
+      g = std::max(g, spec_.grad_bytes(b));
+    }
+    for (int K = 0; K < D_; ++K) {
+      st_[K].in_bytes = K == 0 ? spec_.input_bytes() : a;
+      st_[K].out_bytes = K == D_ - 1 ? spec_.act_bytes(spec_.m()) : a;
+      st_[K].in_gbytes = K == 0 ? spec_.grad_bytes(0) : g;
+      st_[K].out_gbytes = K == D_ - 1 ? spec_.grad_bytes(spec_.m()) : g;
+    }
+    return;
+  }
   for (int K = 0; K < D_; ++K) {
     const auto& bl = planner_.blocks_of(K);
     st_[K].in_bytes = K == 0 ? spec_.input_bytes() : spec_.act_bytes(bl.front());
@@ -303,10 +336,15 @@ void Engine::setup_stage(int K, int dev, bool local) {
   CU(cudaStreamCreateWithFlags(&st.comp, cudaStreamNonBlocking));
   CU(cudaStreamCreateWithFlags(&st.copy, cudaStreamNonBlocking));
   st.arena = std::make_unique<DevArena>(dev);
-  st.fam = make_family(spec_, planner_.blocks_of(K), W_, *st.arena, st.comp);
+  std::vector<int> blocks = planner_.blocks_of(K);
+  if (spec_.raw.flags & NASPIPE_FLAG_MIRROR) {  // a mirror copy of every block's candidates
+    blocks.resize(spec_.m());
+    for (int b = 0; b < spec_.m(); ++b) blocks[b] = b;
+  }
+  st.fam = make_family(spec_, blocks, W_, *st.arena, st.comp);
   st.fam->timer = &timer_;
   st.store = std::make_unique<CandidateStore>(spec_, planner_, K, dev, st.fam.get(), st.arena.get(),
-                                              spec_.raw.hbm_weight_budget_bytes);
+                                              spec_.raw.hbm_weight_budget_bytes, blocks);
   if (spec_.raw.sync_policy == NASPIPE_SYNC_BSP) st.store->enable_bsp(st.arena.get());
   st.in.assign(W_, nullptr);
   st.gout.assign(W_, nullptr);
@@ -369,6 +407,13 @@ void Engine::shutdown() {
   }
   tx_.reset();
   peer_.reset();
+  for (cudaStream_t s : push_) cudaStreamSynchronize(s);
+  for (cudaStream_t s : push_) cudaStreamDestroy(s);
+  for (cudaEvent_t ev : ev_push_) cudaEventDestroy(ev);
+  for (cudaEvent_t ev : ev_wrote_) cudaEventDestroy(ev);
+  push_.clear();
+  ev_push_.clear();
+  ev_wrote_.clear();
   for (auto& st : st_) {
     if (!st.local || !st.comp) continue;
     cudaSetDevice(st.dev);
@@ -416,6 +461,7 @@ int64_t Engine::submit(const int32_t* choice, const naspipe_batch* batch) {
   }
   const int64_t y = planner_.add_subnet(choice);
   batches_.push_back({*batch});
+  if (mirror_) return y;  // planned and issued at drain (drain_mirrored)
   planner_.advance();
   feed_stores();
   issue_planned();
@@ -423,7 +469,8 @@ int64_t Engine::submit(const int32_t* choice, const naspipe_batch* batch) {
 }
 
 void Engine::drain() {
-  if (!drained_) {
+  if (!drained_ && mirror_) drain_mirrored();
+  if (!drained_ && !mirror_) {
     planner_.finalize();
     planner_.advance();
     NP_REQUIRE(planner_.done(), NASPIPE_EINTERNAL, "planner did not finish");
@@ -445,6 +492,7 @@ void Engine::drain() {
   if (tx_)
     for (cudaStream_t s : {tx_->s_act_in, tx_->s_act_out, tx_->s_grad_in, tx_->s_grad_out})
       CU(cudaStreamSynchronize(s));
+  for (cudaStream_t s : push_) CU(cudaStreamSynchronize(s));
   cuda_check("drain");
   timer_.collect();
   drained_ = true;
@@ -467,6 +515,78 @@ void Engine::issue_planned() {
     const Task& t = tasks[issued_];
     if (st_[t.K].local && !st_[t.K].store->ready()) break;
     issue(tasks[issued_++]);
+  }
+}
+
+// ------------------------------------------------------------------------------ layer mirroring
+// Plan the undrained subnets [mbase_, N) with per-subnet balanced partitions (mirror.cpp,
+// reading A31; mirror latency = link_latency) and issue the plan in its decision order.
+void Engine::drain_mirrored() {
+  const int64_t N = planner_.n_subnets(), n = N - mbase_, m = spec_.m();
+  std::vector<int32_t> ch((size_t)n * m);
+  for (int64_t y = 0; y < n; ++y)
+    for (int b = 0; b < m; ++b) ch[y * m + b] = planner_.choice(mbase_ + y, b);
+  const MirrorPlan P = plan_mirrored(spec_, D_, ch.data(), n, spec_.raw.link_latency);
+  msob_.resize((size_t)N * m);
+  std::copy(P.sob.begin(), P.sob.end(), msob_.begin() + mbase_ * m);
+  for (Task t : P.trace) {
+    t.y += mbase_;
+    t.t += mticks_;
+    issue_mirrored(t);
+  }
+  mticks_ += P.makespan;
+  mbase_ = N;
+  issued_ = 0;
+}
+
+void Engine::issue_mirrored(const Task& t) {
+  const int slot = (int)(t.y % W_);
+  const int m = spec_.m();
+  StageRt& st = st_[t.K];
+  int lo = m, hi = 0;
+  for (int b = 0; b < m; ++b)
+    if (msob_[t.y * m + b] == t.K) lo = std::min(lo, b), hi = std::max(hi, b + 1);
+  NP_REQUIRE(lo < hi, NASPIPE_EINTERNAL, "subnet %lld has no block on stage %d", (long long)t.y, t.K);
+  CU(cudaSetDevice(st.dev));
+  for (int b = lo; b < hi; ++b) {
+    const size_t key = (size_t)b * spec_.n() + planner_.choice(t.y, b);
+    if (spec_.raw.flags & NASPIPE_FLAG_VERSION_CHECK) {
+      NP_REQUIRE(version_[key] == planner_.version(t.y, b), NASPIPE_EINTERNAL,
+                 "version check: subnet %lld stage %d block %d sees version %lld, expected %lld", (long long)t.y,
+                 t.K, b, (long long)version_[key], (long long)planner_.version(t.y, b));
+      ++version_checks_;
+    }
+    if (t.kind == 1) version_[key] += 1;
+    // the READ (forward) / READ + WRITE (backward) of a candidate last written on another
+    // stage waits for the push of that WRITE into this stage's mirror copy
+    if (mwriter_[key] >= 0 && mwriter_[key] != t.K) CU(cudaStreamWaitEvent(st.comp, ev_push_[key], 0));
+  }
+  if (spec_.raw.flags & NASPIPE_FLAG_TRACE) trace_.push_back(t);
+  st.fam->set_range(lo, hi);
+  if (t.kind == 0) issue_forward(st, t.y, slot);
+  else issue_backward(st, t.y, slot);
+  ++issued_;
+  if (t.kind != 1) return;
+  // push the WRITE (fp32 master + bf16 shadow) of every candidate of this task to the other
+  // stages' mirror copies, on this stage's push stream once the backward is done
+  CU(cudaEventRecord(ev_wrote_[t.K], st.comp));
+  CU(cudaStreamWaitEvent(push_[t.K], ev_wrote_[t.K], 0));
+  for (int b = lo; b < hi; ++b) {
+    const int c = planner_.choice(t.y, b);
+    const size_t key = (size_t)b * spec_.n() + c;
+    CandidateStore& src = *st.store;
+    for (int K2 = 0; K2 < D_; ++K2) {
+      if (K2 == t.K) continue;
+      CandidateStore& dst = *st_[K2].store;
+      CU(cudaMemcpyPeerAsync(dst.dev_master(b, c), st_[K2].dev, src.dev_master(b, c), st.dev, src.n32(b, c) * 4,
+                             push_[t.K]));
+      if (src.n16(b, c))
+        CU(cudaMemcpyPeerAsync(dst.dev_shadow(b, c), st_[K2].dev, src.dev_shadow(b, c), st.dev, src.n16(b, c) * 2,
+                               push_[t.K]));
+      p2p_bytes_ += 4.0 * src.n32(b, c) + 2.0 * src.n16(b, c);
+    }
+    CU(cudaEventRecord(ev_push_[key], push_[t.K]));
+    mwriter_[key] = t.K;
   }
 }
 
@@ -641,7 +761,8 @@ void Engine::get_params(int block, int choice, float* dst, size_t n) {
   NP_REQUIRE(dst && n == spec_.param_count(block, choice), NASPIPE_EINVAL, "n_floats %zu != %zu", n,
              spec_.param_count(block, choice));
   NP_REQUIRE(drained_ || planner_.n_subnets() == 0, NASPIPE_ESTATE, "get_params before naspipe_drain");
-  const int K = planner_.stage_of_block()[block];
+  // (mirroring: after a drain every mirror copy holds the last WRITE; read stage 0's)
+  const int K = mirror_ ? 0 : planner_.stage_of_block()[block];
   StageRt& st = st_[K];
   NP_REQUIRE(st.local, NASPIPE_EINVAL, "block %d lives on stage %d, not on this rank", block, K);
   st.store->get(block, choice, dst);
@@ -654,6 +775,10 @@ void Engine::set_params(int block, int choice, const float* src, size_t n) {
   NP_REQUIRE(src && n == spec_.param_count(block, choice), NASPIPE_EINVAL, "n_floats %zu != %zu", n,
              spec_.param_count(block, choice));
   NP_REQUIRE(drained_ || planner_.n_subnets() == 0, NASPIPE_ESTATE, "set_params with work in flight");
+  if (mirror_) {  // every stage's mirror copy
+    for (auto& s2 : st_) s2.store->set(block, choice, src, s2.comp);
+    return;
+  }
   const int K = planner_.stage_of_block()[block];
   StageRt& st = st_[K];
   NP_REQUIRE(st.local, NASPIPE_EINVAL, "block %d lives on stage %d, not on this rank", block, K);
@@ -708,7 +833,7 @@ void Engine::get_stats(double* o) {
   o[10] = evicts;
   o[11] = wbs;
   o[4] = p2p_bytes_;
-  o[5] = (double)planner_.makespan();
+  o[5] = mirror_ ? (double)mticks_ : (double)planner_.makespan();
   o[6] = timer_.launches;
   o[7] = timer_.flops;
   o[8] = timer_.ms;

@@ -76,6 +76,8 @@ class Engine {
   void issue_planned();
   void issue(const Task& t);
   void issue_forward(StageRt& st, int64_t y, int slot);
+  void drain_mirrored();
+  void issue_mirrored(const Task& t);
   void issue_backward(StageRt& st, int64_t y, int slot);
   void version_check(const Task& t);
   void cuda_check(const char* what);
@@ -87,6 +89,14 @@ class Engine {
   std::vector<StageRt> st_;
   std::unique_ptr<Transport> tx_;   // NCCL channels (create_rank)
   std::unique_ptr<PeerLink> peer_;  // peer-memory transport (create_rank_peer)
+  // layer mirroring (NASPIPE_FLAG_MIRROR): per-subnet partitions, mirror copies, pushes
+  bool mirror_ = false;
+  std::vector<int32_t> msob_;          // [N][m] stage of block b for subnet y
+  int64_t mbase_ = 0, mticks_ = 0;     // first subnet of the undrained batch; ticks so far
+  std::vector<int> mwriter_;           // per candidate: stage of its last WRITE (-1: none)
+  std::vector<cudaEvent_t> ev_push_;   // per candidate: its last push to the other stages
+  std::vector<cudaStream_t> push_;     // per stage
+  std::vector<cudaEvent_t> ev_wrote_;  // per stage: the backward whose WRITEs are pushed
   std::vector<BatchRec> batches_;
   std::vector<int32_t> stage_choice_;  // scratch
   size_t issued_ = 0;

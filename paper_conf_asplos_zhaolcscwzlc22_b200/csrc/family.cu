@@ -102,11 +102,11 @@ class MlpFamily : public Family {
   void refresh_shadow(int, int, cudaStream_t) override {}
 
   void forward(int slot, const int32_t* ch, const void* x_in, void* x_out, cudaStream_t s) override {
-    const int nb = (int)blocks_.size();
+    const int nb = (int)blocks_.size(), lo = rlo(), hi = rhi(nb);
     const float* x = static_cast<const float*>(x_in);
-    for (int j = 0; j < nb; ++j) {
+    for (int j = lo; j < hi; ++j) {
       float* P = master(j, ch[blocks_[j]]);
-      float* y = (j == nb - 1) ? static_cast<float*>(x_out) : act_[(size_t)slot * nb + j + 1];
+      float* y = (j == hi - 1) ? static_cast<float*>(x_out) : act_[(size_t)slot * nb + j + 1];
       xin_[(size_t)slot * nb + j] = x;
       mlp_fwd(s, x, P, P + (size_t)d_ * d_, y, h_[(size_t)slot * nb + j], B_, d_);
       counters.launches++;
@@ -114,12 +114,12 @@ class MlpFamily : public Family {
     }
   }
   void backward(int slot, const int32_t* ch, const void* dy, void* dx, cudaStream_t s) override {
-    const int nb = (int)blocks_.size();
+    const int nb = (int)blocks_.size(), lo = rlo(), hi = rhi(nb);
     const float* g = static_cast<const float*>(dy);
-    for (int j = nb - 1; j >= 0; --j) {
+    for (int j = hi - 1; j >= lo; --j) {
       float* P = master(j, ch[blocks_[j]]);
       float* U = upd(j, ch[blocks_[j]]);  // SGD WRITE target (P in place; the BSP accumulator)
-      float* out = (j == 0) ? static_cast<float*>(dx) : g_[j & 1];
+      float* out = (j == lo) ? static_cast<float*>(dx) : g_[j & 1];
       mlp_bwd_sgd(s, xin_[(size_t)slot * nb + j], h_[(size_t)slot * nb + j], g, out, P, U, U + (size_t)d_ * d_, lr_,
                   B_, d_);
       counters.launches++;
@@ -253,13 +253,13 @@ class TfFamily : public Family {
   }
 
   void forward(int slot, const int32_t* ch, const void* x_in, void* x_out, cudaStream_t s) override {
-    const int nb = (int)blocks_.size();
+    const int nb = (int)blocks_.size(), lo = rlo(), hi = rhi(nb);
     const float* x = static_cast<const float*>(x_in);
-    for (int j = 0; j < nb; ++j) {
+    for (int j = lo; j < hi; ++j) {
       const int c = ch[blocks_[j]];
       TfSlot& t = slots_[(size_t)slot * nb + j];
       t.xin = x;
-      float* y = (j == nb - 1) ? static_cast<float*>(x_out) : slots_[(size_t)slot * nb + j + 1].act;
+      float* y = (j == hi - 1) ? static_cast<float*>(x_out) : slots_[(size_t)slot * nb + j + 1].act;
       if (recompute_) {  // activations into the scratch set; only the block input is kept
         TfSlot tt = rs_[j & 1];
         tt.xin = x;
@@ -278,23 +278,23 @@ class TfFamily : public Family {
   // leaves idle.  Buffers the side stream reads are double-buffered by block parity; the
   // stage stream joins the side stream before the task ends.
   void backward(int slot, const int32_t* ch, const void* dy_v, void* dx_v, cudaStream_t s) override {
-    const int nb = (int)blocks_.size();
+    const int nb = (int)blocks_.size(), lo = rlo(), hi = rhi(nb);
     const float* dy = static_cast<const float*>(dy_v);
     float* dx = static_cast<float*>(dx_v);
     const float* g = dy;
     int db2_nblk = 0;
-    for (int j = nb - 1; j >= 0; --j) {
+    for (int j = hi - 1; j >= lo; --j) {
       const int c = ch[blocks_[j]];
       const int p = j & 1;
       TfSlot& t = slots_[(size_t)slot * nb + j];
-      if (j == nb - 1) {  // grad entering the stage: bf16 copy + colsum for b2
+      if (j == hi - 1) {  // grad entering the stage: bf16 copy + colsum for b2
         cast_colsum(s, g, dy16_[p], p_db2_[p], T_, d_);
         counters.launches++;
         db2_nblk = lnb_;
       }
       // stage 0 needs no input gradient, but LN1's backward still runs (dgamma/dbeta):
-      // its dx goes to a scratch buffer (gb_[0] is free: block 1 wrote gb_[1])
-      float* out = (j == 0) ? (dx ? dx : gb_[0]) : gb_[j & 1];
+      // its dx goes to a scratch buffer (gb_[lo & 1] is free: block lo + 1 wrote the other)
+      float* out = (j == lo) ? (dx ? dx : gb_[lo & 1]) : gb_[j & 1];
       if (recompute_) {
         // recompute block j's forward from its kept input into scratch set p (bitwise the
         // forward's activations: same kernels, same input, same weights — CSP/BSP do not
@@ -304,9 +304,9 @@ class TfFamily : public Family {
         tt.xin = t.xin;
         cudaStreamWaitEvent(s, ev_done_[p], 0);
         block_fwd(j, c, tt, ry_, s);
-        block_bwd(j, c, tt, g, out, /*want_next=*/j > 0, db2_nblk, p, s);
+        block_bwd(j, c, tt, g, out, /*want_next=*/j > lo, db2_nblk, p, s);
       } else {
-        block_bwd(j, c, t, g, out, /*want_next=*/j > 0, db2_nblk, p, s);
+        block_bwd(j, c, t, g, out, /*want_next=*/j > lo, db2_nblk, p, s);
       }
       db2_nblk = lnb_;
       g = out;

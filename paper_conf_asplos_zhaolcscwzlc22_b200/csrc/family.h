@@ -86,6 +86,15 @@ class Family {
     const size_t k = (size_t)local_block * n_choices_ + c;
     return k >= upd_.size() || upd_[k] == nullptr;
   }
+  // Layer mirroring (NASPIPE_FLAG_MIRROR, reading A31): a stage's family holds every block and
+  // a task runs the contiguous local range [lo, hi) its subnet's partition assigns to the
+  // stage; the fixed partition runs [0, #blocks).  Set by the engine before forward/backward.
+  void set_range(int lo, int hi) {
+    lo_ = lo;
+    hi_ = hi;
+  }
+  int rlo() const { return lo_; }
+  int rhi(int nb) const { return hi_ < nb ? hi_ : nb; }
   // called by the engine after a drain's synchronisation (device-side sticky checks)
   virtual void check_after_drain() {}
   FamilyCounters counters;
@@ -96,6 +105,7 @@ class Family {
   int n_choices_ = 1;            // set by the families (bind_update's key)
   std::vector<float*> upd_;      // BSP accumulators, [local_block * n + c]
   float* mse_part_ = nullptr;  // MSE workspace (last stage)
+  int lo_ = 0, hi_ = 1 << 30;  // task block range (set_range)
 };
 
 std::unique_ptr<Family> make_family(const Spec& spec, const std::vector<int>& blocks, int W, DevArena& arena,

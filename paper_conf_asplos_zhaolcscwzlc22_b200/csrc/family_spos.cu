@@ -40,7 +40,7 @@ class SposFamily : public Family {
     w16_.assign((size_t)nb * n, nullptr);
     plans_.resize((size_t)nb * n);
     dims_.resize(nb);
-    size_t stash_max = 0, stats_max = 0, dz_max = 0, g_max = 0, blk_max = 0, dwp_max = 0, C_max = 0;
+    size_t stash_max = 0, stats_max = 0, dz_max = 0, g_max = 0, blk_max = 0, dwk_max = 0, C_max = 0;
     ws_elems_ = 0;
     for (int j = 0; j < nb; ++j) {
       const int b = blocks[j];
@@ -60,8 +60,7 @@ class SposFamily : public Family {
           dz_max = std::max(dz_max, po * u.cout);
           g_max = std::max({g_max, pi * u.cin, po * u.cout});
           C_max = std::max(C_max, (size_t)u.cout);
-          if (u.dw)
-            dwp_max = std::max(dwp_max, (size_t)dw_wgrad_blocks(B_, u.H_in, u.cout, u.k, u.stride) * u.cout * u.k * u.k);
+          if (u.dw) dwk_max = std::max(dwk_max, (size_t)u.cout * u.k * u.k);
           else
             ws_elems_ = std::max(ws_elems_, (size_t)gemm_splitk_factor(u.cout, u.cin, (int)po) * u.cout * u.cin);
         }
@@ -102,12 +101,14 @@ class SposFamily : public Family {
     // and zero everywhere, so every flag position starts (and, flags aside, stays) zero
     acc_f_ = A.alloc<unsigned long long>(2 * C_max + 1);
     acc_b_ = A.alloc<unsigned long long>(2 * C_max + 1);
-    tick_ = A.alloc<int>(2);
+    tick_ = A.alloc<int>(3);  // bn_apply, bn_bwd_apply, dw weight gradient (side stream)
     cudaMemset(acc_f_, 0, (2 * C_max + 1) * 8);
     cudaMemset(acc_b_, 0, (2 * C_max + 1) * 8);
     C_max_ = (int)C_max;
-    cudaMemset(tick_, 0, 2 * sizeof(int));
-    dwpart_ = A.alloc<float>(std::max<size_t>(dwp_max, 1));
+    cudaMemset(tick_, 0, 3 * sizeof(int));
+    dwk_max_ = dwk_max;
+    acc_w_ = A.alloc<unsigned long long>(dwk_max + 1);
+    cudaMemset(acc_w_, 0, (dwk_max + 1) * 8);
     ws_ = A.alloc<float>(std::max<size_t>(ws_elems_, 4));
     if (first_) {
       std::vector<float> h(spec.frozen_count(0));
@@ -174,9 +175,9 @@ class SposFamily : public Family {
   }
 
   void forward(int slot, const int32_t* ch, const void* x_in, void* x_out, cudaStream_t s) override {
-    const int nb = (int)blocks_.size();
+    const int nb = (int)blocks_.size(), lo = rlo(), hi = rhi(nb);
     const bf16* x = static_cast<const bf16*>(x_in);
-    if (first_) {  // frozen stem: conv3x3 s2 -> BN(1, 0) batch statistics -> ReLU
+    if (first_ && lo == 0) {  // frozen stem: conv3x3 s2 -> BN(1, 0) batch statistics -> ReLU
       const int H = spec_.raw.image_hw, C0 = spec_.raw.stem_channels;
       const int Po = (int)P(H / 2);
       spos_stem_conv(s, static_cast<const float*>(x_in), w_stem_, stem_z_, B_, H, C0);
@@ -185,10 +186,10 @@ class SposFamily : public Family {
       counters.launches += 3;
       x = stem_y_[slot];
     }
-    for (int j = 0; j < nb; ++j) {
+    for (int j = lo; j < hi; ++j) {
       const int c = ch[blocks_[j]];
       const size_t k = (size_t)slot * nb + j;
-      bf16* out = (j == nb - 1) ? static_cast<bf16*>(x_out) : act_[k];
+      bf16* out = (j == hi - 1) ? static_cast<bf16*>(x_out) : act_[k];
       xin_[k] = x;
       block_fwd(j, c, k, x, out, s);
       x = out;
@@ -196,13 +197,13 @@ class SposFamily : public Family {
   }
 
   void backward(int slot, const int32_t* ch, const void* dy, void* dx, cudaStream_t s) override {
-    const int nb = (int)blocks_.size();
+    const int nb = (int)blocks_.size(), lo = rlo(), hi = rhi(nb);
     const bf16* g = static_cast<const bf16*>(dy);
-    for (int j = nb - 1; j >= 0; --j) {
+    for (int j = hi - 1; j >= lo; --j) {
       const int c = ch[blocks_[j]];
       const size_t k = (size_t)slot * nb + j;
-      const bool need_dx = j > 0 || dx != nullptr;
-      bf16* out = (j == 0) ? static_cast<bf16*>(dx) : gb_[j & 1];
+      const bool need_dx = j > lo || dx != nullptr;
+      bf16* out = (j == lo) ? static_cast<bf16*>(dx) : gb_[j & 1];
       block_bwd(j, c, k, g, out, need_dx, s);
       g = out;
     }
@@ -254,6 +255,9 @@ class SposFamily : public Family {
       cudaMemcpy(h.data(), a, h.size() * 8, cudaMemcpyDeviceToHost);
       for (auto v : h) bad |= v != 0;
     }
+    h.resize(dwk_max_ + 1);
+    cudaMemcpy(h.data(), acc_w_, h.size() * 8, cudaMemcpyDeviceToHost);
+    for (auto v : h) bad |= v != 0;
     NP_REQUIRE(!bad, NASPIPE_EINTERNAL,
                "BatchNorm fixed-point accumulator overflow (a partial sum outside the 64-bit range, spos.cu)");
   }
@@ -414,10 +418,8 @@ class SposFamily : public Family {
     cudaEventRecord(ev_dg_[ring_], s);
     cudaStreamWaitEvent(side_, ev_dg_[ring_], 0);
     if (u.dw) {
-      dw_wgrad(side_, dz, r.x, dwpart_, B_, u.H_in, u.cin, u.k, u.stride);
-      sgd_from_partials(side_, Um + u.off_w, dwpart_, dw_wgrad_blocks(B_, u.H_in, u.cout, u.k, u.stride),
-                        u.cout * u.k * u.k, lr_);
-      counters.launches += 2;
+      dw_wgrad_sgd(side_, dz, r.x, acc_w_, tick_ + 2, Um + u.off_w, lr_, B_, u.H_in, u.cin, u.k, u.stride);
+      counters.launches += 1;
     } else {
       GemmEpiParams e;
       e.w32 = Um + u.off_w;  // the BSP accumulator has no shadow (refreshed at the flush)
@@ -496,8 +498,10 @@ class SposFamily : public Family {
   bool ring_used_[kRing] = {false, false, false};
   cudaStream_t side_ = nullptr;  // weight gradients + SGD of the backward
   cudaEvent_t ev_dg_[kRing], ev_wg_[kRing], ev_join_;
-  float *dwpart_, *ws_;
+  float* ws_;
   unsigned long long *acc_f_, *acc_b_;  // BatchNorm fixed-point accumulators (forward / backward)
+  unsigned long long* acc_w_ = nullptr; // depthwise weight gradient accumulator (side stream)
+  size_t dwk_max_ = 0;
   int* tick_;                           // [2] arrival tickets of bn_apply / bn_bwd_apply
   int C_max_ = 0;
   size_t ws_elems_ = 0;

@@ -159,8 +159,10 @@ void dw_fwd(cudaStream_t s, const bf16* x, const float* w, bf16* z, int B, int H
 void dw_dgrad(cudaStream_t s, const bf16* dz, const float* w, const bf16* add, bf16* dx, int B, int H, int C, int k,
               int S);
 int dw_wgrad_blocks(int B, int H, int C, int k, int S);
-// part [dw_wgrad_blocks(B, H, C, k, S)][C][k][k]
-void dw_wgrad(cudaStream_t s, const bf16* dz, const bf16* x, float* part, int B, int H, int C, int k, int S);
+// weight gradient of a depthwise conv with the SGD WRITE fused: w -= lr * sum over the batch
+// (acc [C*k*k + 1] and ticket zero between uses, fixpoint.cuh; w = master or BSP accumulator)
+void dw_wgrad_sgd(cudaStream_t s, const bf16* dz, const bf16* x, unsigned long long* acc, int* ticket, float* w,
+                  float lr, int B, int H, int C, int k, int S);
 // channel split of a stride-1 block input [P, 2Ch] (x2): out[:, i] = x[:, 2i] (ld ldo, planes
 // oplane apart), xm[:, i] = x[:, 2i+1]; merge is its (plain bf16) backward
 void chan_split(cudaStream_t s, const bf16* x, int P, int Ch, bf16* out, int ldo, size_t oplane, bf16* xm);

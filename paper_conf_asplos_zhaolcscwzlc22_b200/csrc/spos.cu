@@ -656,12 +656,14 @@ __global__ void __launch_bounds__(TPB) dw_tile_kernel(const bf16* __restrict__ i
 // thread (ch, col, cg) — output column tw*TW + col, channel c — holds its DT_H values of dz
 // in registers and accumulates all K x K taps, reading each staged input once per tile
 // (K*K FMAs per DT_H*K*K / (IH*K) reads instead of one load per FMA).  The TW column sums
-// are then added in column order; part[tw + tiles_w * p][c][u][v] (the weight's layout),
-// later summed over the partial blocks in a fixed order.  Bitwise reproducible.
+// are then added in column order and, in 64-bit fixed point, into acc[c][u][v] (the weight's
+// layout; fixpoint.cuh: bitwise independent of the CTA order).  The last CTA (ticket) applies
+// the SGD WRITE w -= lr * total (w = the master, or the bulk accumulator under BSP) and clears
+// acc: one launch instead of partials + a fixed-order summing SGD kernel.
 template <int K, int S>
 __global__ void __launch_bounds__(TPB) dw_wgrad_kernel(const bf16* __restrict__ dz, const bf16* __restrict__ x,
-                                                       float* __restrict__ part, int B, int H, int C, int TW,
-                                                       int NP) {
+                                                       unsigned long long* gacc, int* ticket, float* w, float lr,
+                                                       int B, int H, int C, int TW, int NP) {
   constexpr int PAD = K / 2, IH = (DT_H - 1) * S + K, K2 = K * K;
   extern __shared__ float tile[];  // [CPG][IH][IW][8]; later [TPB][K2] for the column sums
   ptx::pdl_wait();
@@ -718,14 +720,20 @@ __global__ void __launch_bounds__(TPB) dw_wgrad_kernel(const bf16* __restrict__ 
 #pragma unroll
     for (int v = 0; v < K; ++v) red[(size_t)threadIdx.x * K2 + u * K + v] = acc[u][v];
   __syncthreads();
-  const size_t pbase = (size_t)blockIdx.x * C * K2;
   for (int e = threadIdx.x; e < CPG * 8 * K2; e += TPB) {
     const int tap = e % K2, cc = e / K2, cgl = cc / 8, chl = cc % 8;
     const int cglob = (cg0 + cgl) * 8 + chl;
     if (cglob >= C) continue;
     float sum = 0.f;
     for (int cl = 0; cl < TW; ++cl) sum += red[(size_t)((cgl * TW + cl) * 8 + chl) * K2 + tap];
-    part[pbase + (size_t)cglob * K2 + tap] = sum;
+    fix_add(gacc, cglob * K2 + tap, gacc + (size_t)C * K2, sum, FIX_B);
+  }
+  if (last_cta(ticket)) {  // every CTA's partial is in: the WRITE, then clear for the next use
+    for (int i = threadIdx.x; i < C * K2; i += TPB) {
+      w[i] -= lr * (float)fix_get(gacc, i, FIX_B);
+      gacc[i] = 0ull;
+    }
+    if (threadIdx.x == 0) *ticket = 0;
   }
 }
 
@@ -1143,13 +1151,14 @@ static void dw_wgrad_grid(int B, int H, int C, int k, int S, int& TW, int& NP, i
   NP = std::max(1, std::min(tiles, dw_red_ctas() / std::max(1, tiles_w * gy)));
   (void)k;
 }
-int dw_wgrad_blocks(int B, int H, int C, int k, int S) {
+int dw_wgrad_blocks(int B, int H, int C, int k, int S) {  // grid size (diagnostics)
   int TW, NP, gy, tw;
   dw_wgrad_grid(B, H, C, k, S, TW, NP, gy, tw);
   return tw * NP;
 }
 
-void dw_wgrad(cudaStream_t s, const bf16* dz, const bf16* x, float* part, int B, int H, int C, int k, int S) {
+void dw_wgrad_sgd(cudaStream_t s, const bf16* dz, const bf16* x, unsigned long long* acc, int* ticket, float* w,
+                  float lr, int B, int H, int C, int k, int S) {
   NP_REQUIRE(C % 8 == 0 && C / 8 <= TPB, NASPIPE_EINVAL, "dw_wgrad C=%d", C);
   NP_REQUIRE(S == 1 || S == 2, NASPIPE_EINVAL, "dw_wgrad stride %d", S);
   int TW, NP, gy, tiles_w;
@@ -1163,7 +1172,7 @@ void dw_wgrad(cudaStream_t s, const bf16* dz, const bf16* x, float* part, int B,
 #define DW_WG(KK, SS)                                                                                  \
   {                                                                                                    \
     set_smem(dw_wgrad_kernel<KK, SS>, smem(KK));                                                       \
-    launch_pdl(dw_wgrad_kernel<KK, SS>, grid, dim3(TPB), smem(KK), s, dz, x, part, B, H, C, TW, NP);    \
+    launch_pdl(dw_wgrad_kernel<KK, SS>, grid, dim3(TPB), smem(KK), s, dz, x, acc, ticket, w, lr, B, H, C, TW, NP); \
   }
   if (S == 1) {
     DW_DISPATCH(k, DW_WG(KK, 1));
