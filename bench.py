@@ -589,7 +589,7 @@ def main():
                                                      "a lower bound (the conv kernels' bytes are not counted)"),
                      "end_to_end_vs_csp_plan": (plan_ms / ms) if plan_ms else None,
                      "csp_plan_ms": plan_ms, "measured_ms": ms, "busy_ms_per_rank": [b / 1000 for b in busy]}
-        top = sorted(per.items(), key=lambda kv: -kv[1][1])[:8]
+        top = sorted(per.items(), key=lambda kv: -kv[1][1])[:14]
         kernels_top = [{"name": k[:90], "launches": c, "us": round(t, 1)} for k, (c, t) in top]
 
     # ---- timed region 3: end to end through the C ABI with pinned host buffers

@@ -1,4 +1,6 @@
-// Non-causal multi-head attention for S <= 128 (reading A17): one CTA per (batch, head)
+// Non-causal multi-head attention for S <= 128 (reading A17), the mma.sync kernels used for
+// the shapes the tcgen05 kernels (attention_tc.cu: S = 128, head dim 64 / 128) do not cover
+// (NASPIPE_ATTN_MMA_SYNC=1 forces these everywhere): one CTA per (batch, head)
 // holds the whole S x S score tile, so forward and backward need no atomics and are
 // bitwise deterministic.  Tensor-core math via mma.sync m16n8k16 (bf16 in, fp32 acc);
 // each of the 8 warps owns 16 query rows (forward, dQ) and 16 key rows (dK, dV).
@@ -430,6 +432,7 @@ void bwd_launch(cudaStream_t s, const bf16* qkv, const bf16* o, const float* lse
 
 void attn_fwd(cudaStream_t s, const bf16* qkv, bf16* o, float* lse, int B, int S, int d, int h) {
   NP_REQUIRE(S % 16 == 0 && S <= SMAX, NASPIPE_EINVAL, "attention needs S %% 16 == 0 and S <= 128 (S=%d)", S);
+  if (attn_tc_supported(S, d, h)) return attn_fwd_tc(s, qkv, o, lse, B, S, d, h);  // tcgen05 (attention_tc.cu)
   const int hd = d / h;
 #define CALLF(X) fwd_launch<X>(s, qkv, o, lse, B, S, d, h)
   NP_HD_DISPATCH(hd, CALLF)
@@ -441,6 +444,7 @@ void attn_fwd(cudaStream_t s, const bf16* qkv, bf16* o, float* lse, int B, int S
 void attn_bwd(cudaStream_t s, const bf16* qkv, const bf16* o, const float* lse, const bf16* dout, bf16* dqkv,
               int B, int S, int d, int h) {
   NP_REQUIRE(S % 16 == 0 && S <= SMAX, NASPIPE_EINVAL, "attention needs S %% 16 == 0 and S <= 128 (S=%d)", S);
+  if (attn_tc_supported(S, d, h)) return attn_bwd_tc(s, qkv, o, lse, dout, dqkv, B, S, d, h);
   const int hd = d / h;
 #define CALLB(X) bwd_launch<X>(s, qkv, o, lse, dout, dqkv, B, S, d, h)
   NP_HD_DISPATCH(hd, CALLB)

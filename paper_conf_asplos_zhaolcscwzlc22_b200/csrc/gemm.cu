@@ -23,6 +23,7 @@
 #include "fixpoint.cuh"
 #include "launch.h"
 #include "ptx.cuh"
+#include "tma.h"
 
 namespace naspipe {
 
@@ -786,6 +787,10 @@ int num_sms() {
     return v > 0 ? v : 148;
   }();
   return n;
+}
+
+CUtensorMap tma_map_bf16(const bf16* base, uint64_t inner, uint64_t outer, uint64_t ld, uint32_t box_outer) {
+  return make_map(base, inner, outer, ld, box_outer);
 }
 
 uint64_t gemm_launch_count() { return g_gemm_launches.load(); }

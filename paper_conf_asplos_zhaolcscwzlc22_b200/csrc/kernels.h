@@ -64,6 +64,12 @@ uint64_t gemm_flop_count();  // algorithmic flops of every GEMM call of this pro
 // ------------------------------------------------------------------ attention (S <= 128)
 // qkv [B*S, 3d] bf16 (q | k | v thirds, head j = columns [j*hd, (j+1)*hd) of each third);
 // o [B*S, d] bf16; lse [B*h*S] f32 (natural log of the softmax denominator incl. scale).
+// tcgen05 attention (attention_tc.cu) for S = 128 and head dim 64 / 128; attn_fwd / attn_bwd
+// dispatch to it when attn_tc_supported
+bool attn_tc_supported(int S, int d, int h);
+void attn_fwd_tc(cudaStream_t s, const bf16* qkv, bf16* o, float* lse, int B, int S, int d, int h);
+void attn_bwd_tc(cudaStream_t s, const bf16* qkv, const bf16* o, const float* lse, const bf16* dout, bf16* dqkv,
+                 int B, int S, int d, int h);
 void attn_fwd(cudaStream_t s, const bf16* qkv, bf16* o, float* lse, int B, int S, int d, int h);
 // do_ [B*S, d] bf16 -> dqkv [B*S, 3d] bf16
 void attn_bwd(cudaStream_t s, const bf16* qkv, const bf16* o, const float* lse, const bf16* do_,

@@ -62,6 +62,7 @@ inline void launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t sme
   cfg.attrs = at;
   cfg.numAttrs = pdl_enabled() ? 1 : 0;
   const cudaError_t e = cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+  if (e != cudaSuccess) cudaGetLastError();  // consume it: a launch-configuration error is not sticky
   NP_REQUIRE(e == cudaSuccess, NASPIPE_ECUDA, "kernel launch: %s", cudaGetErrorString(e));
 }
 
