@@ -78,19 +78,22 @@ __global__ void __launch_bounds__(128, 1) attn_fwd_tc_kernel(const __grid_consta
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_holder;
-  if (threadIdx.x == 0) {
-    ptx::mbar_arrive_expect_tx(&bar[0], 3 * NCH * TILE);
-    for (int j = 0; j < NCH; ++j) {
-      ptx::tma_load_2d(sQ + j * TILE, &tq, &bar[0], hh * HD + 64 * j, b * AS);
-      ptx::tma_load_2d(sK + j * TILE, &tq, &bar[0], d + hh * HD + 64 * j, b * AS);
-      ptx::tma_load_2d(sV + j * TILE, &tq, &bar[0], 2 * d + hh * HD + 64 * j, b * AS);
+  if (warp == 0) {  // lane 0 issues; lanes 1-31 wait at the __syncwarp, not spinning on an mbarrier
+    if (lane == 0) {
+      ptx::mbar_arrive_expect_tx(&bar[0], 3 * NCH * TILE);
+      for (int j = 0; j < NCH; ++j) {
+        ptx::tma_load_2d(sQ + j * TILE, &tq, &bar[0], hh * HD + 64 * j, b * AS);
+        ptx::tma_load_2d(sK + j * TILE, &tq, &bar[0], d + hh * HD + 64 * j, b * AS);
+        ptx::tma_load_2d(sV + j * TILE, &tq, &bar[0], 2 * d + hh * HD + 64 * j, b * AS);
+      }
+      ptx::mbar_wait(&bar[0], 0);
+      ptx::tc_fence_after();
+      constexpr uint32_t idesc = ptx::umma_idesc_bf16(128, 128, 0, 0);
+  #pragma unroll
+      for (int kk = 0; kk < HD / 16; ++kk) ptx::umma_bf16(tmem, desc_k(sQ, kk), desc_k(sK, kk), idesc, kk > 0);
+      ptx::umma_commit(&bar[1]);
     }
-    ptx::mbar_wait(&bar[0], 0);
-    ptx::tc_fence_after();
-    constexpr uint32_t idesc = ptx::umma_idesc_bf16(128, 128, 0, 0);
-#pragma unroll
-    for (int kk = 0; kk < HD / 16; ++kk) ptx::umma_bf16(tmem, desc_k(sQ, kk), desc_k(sK, kk), idesc, kk > 0);
-    ptx::umma_commit(&bar[1]);
+    __syncwarp();
   }
   ptx::mbar_wait(&bar[1], 0);
   ptx::tc_fence_after();
@@ -126,11 +129,14 @@ __global__ void __launch_bounds__(128, 1) attn_fwd_tc_kernel(const __grid_consta
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
-  if (threadIdx.x == 0) {
-    constexpr uint32_t idesc = ptx::umma_idesc_bf16(128, HD, 0, 1);  // A = P K-major, B = V MN-major
-#pragma unroll
-    for (int kk = 0; kk < AS / 16; ++kk) ptx::umma_bf16(tmem + 128, desc_k(sP, kk), desc_mn(sV, kk), idesc, kk > 0);
-    ptx::umma_commit(&bar[2]);
+  if (warp == 0) {  // lane 0 issues; lanes 1-31 wait at the __syncwarp, not spinning on an mbarrier
+    if (lane == 0) {
+      constexpr uint32_t idesc = ptx::umma_idesc_bf16(128, HD, 0, 1);  // A = P K-major, B = V MN-major
+  #pragma unroll
+      for (int kk = 0; kk < AS / 16; ++kk) ptx::umma_bf16(tmem + 128, desc_k(sP, kk), desc_mn(sV, kk), idesc, kk > 0);
+      ptx::umma_commit(&bar[2]);
+    }
+    __syncwarp();
   }
   ptx::mbar_wait(&bar[2], 0);
   ptx::tc_fence_after();
@@ -177,7 +183,7 @@ __global__ void __launch_bounds__(128, 1) attn_bwd_tc_kernel(const __grid_consta
   uint64_t* bar = reinterpret_cast<uint64_t*>(sdS + 2 * TILE);  // [0] TMA, [1] S + dP, [2] gradients
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bar + 3);
   const int bh = blockIdx.x, b = bh / h, hh = bh % h;
-  const int warp = threadIdx.x >> 5, r = threadIdx.x;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, r = threadIdx.x;
   if (threadIdx.x == 0) {
     ptx::tma_prefetch(&tq);
     ptx::tma_prefetch(&tdo);
@@ -190,23 +196,26 @@ __global__ void __launch_bounds__(128, 1) attn_bwd_tc_kernel(const __grid_consta
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_holder;
-  if (threadIdx.x == 0) {
-    ptx::mbar_arrive_expect_tx(&bar[0], 4 * NCH * TILE);
-    for (int j = 0; j < NCH; ++j) {
-      ptx::tma_load_2d(sQ + j * TILE, &tq, &bar[0], hh * HD + 64 * j, b * AS);
-      ptx::tma_load_2d(sK + j * TILE, &tq, &bar[0], d + hh * HD + 64 * j, b * AS);
-      ptx::tma_load_2d(sV + j * TILE, &tq, &bar[0], 2 * d + hh * HD + 64 * j, b * AS);
-      ptx::tma_load_2d(sdO + j * TILE, &tdo, &bar[0], hh * HD + 64 * j, b * AS);
+  if (warp == 0) {  // lane 0 issues; lanes 1-31 wait at the __syncwarp, not spinning on an mbarrier
+    if (lane == 0) {
+      ptx::mbar_arrive_expect_tx(&bar[0], 4 * NCH * TILE);
+      for (int j = 0; j < NCH; ++j) {
+        ptx::tma_load_2d(sQ + j * TILE, &tq, &bar[0], hh * HD + 64 * j, b * AS);
+        ptx::tma_load_2d(sK + j * TILE, &tq, &bar[0], d + hh * HD + 64 * j, b * AS);
+        ptx::tma_load_2d(sV + j * TILE, &tq, &bar[0], 2 * d + hh * HD + 64 * j, b * AS);
+        ptx::tma_load_2d(sdO + j * TILE, &tdo, &bar[0], hh * HD + 64 * j, b * AS);
+      }
+      ptx::mbar_wait(&bar[0], 0);
+      ptx::tc_fence_after();
+      constexpr uint32_t idesc = ptx::umma_idesc_bf16(128, 128, 0, 0);
+  #pragma unroll
+      for (int kk = 0; kk < HD / 16; ++kk) {
+        ptx::umma_bf16(tmem, desc_k(sQ, kk), desc_k(sK, kk), idesc, kk > 0);         // S = Q K^T
+        ptx::umma_bf16(tmem + 128, desc_k(sdO, kk), desc_k(sV, kk), idesc, kk > 0);  // dP = dO V^T
+      }
+      ptx::umma_commit(&bar[1]);
     }
-    ptx::mbar_wait(&bar[0], 0);
-    ptx::tc_fence_after();
-    constexpr uint32_t idesc = ptx::umma_idesc_bf16(128, 128, 0, 0);
-#pragma unroll
-    for (int kk = 0; kk < HD / 16; ++kk) {
-      ptx::umma_bf16(tmem, desc_k(sQ, kk), desc_k(sK, kk), idesc, kk > 0);         // S = Q K^T
-      ptx::umma_bf16(tmem + 128, desc_k(sdO, kk), desc_k(sV, kk), idesc, kk > 0);  // dP = dO V^T
-    }
-    ptx::umma_commit(&bar[1]);
+    __syncwarp();
   }
   // Di = rowsum(dO o O) (fp32, column order) while the MMAs run
   const bf16* drow = dout + ((size_t)b * AS + r) * d + hh * HD;
@@ -250,16 +259,19 @@ __global__ void __launch_bounds__(128, 1) attn_bwd_tc_kernel(const __grid_consta
   ptx::tc_fence_before();
   __syncthreads();  // every thread has read S and dP: their TMEM columns are reused below
   ptx::tc_fence_after();
-  if (threadIdx.x == 0) {
-    constexpr uint32_t idesc_t = ptx::umma_idesc_bf16(128, HD, 1, 1);  // A, B MN-major
-    constexpr uint32_t idesc_q = ptx::umma_idesc_bf16(128, HD, 0, 1);  // A K-major, B MN-major
-#pragma unroll
-    for (int kk = 0; kk < AS / 16; ++kk) {
-      ptx::umma_bf16(tmem, desc_mn(sP, kk), desc_mn(sdO, kk), idesc_t, kk > 0);        // dV = P^T dO
-      ptx::umma_bf16(tmem + HD, desc_mn(sdS, kk), desc_mn(sQ, kk), idesc_t, kk > 0);   // dK = dS^T Q
-      ptx::umma_bf16(tmem + 256, desc_k(sdS, kk), desc_mn(sK, kk), idesc_q, kk > 0);   // dQ = dS K
+  if (warp == 0) {  // lane 0 issues; lanes 1-31 wait at the __syncwarp, not spinning on an mbarrier
+    if (lane == 0) {
+      constexpr uint32_t idesc_t = ptx::umma_idesc_bf16(128, HD, 1, 1);  // A, B MN-major
+      constexpr uint32_t idesc_q = ptx::umma_idesc_bf16(128, HD, 0, 1);  // A K-major, B MN-major
+  #pragma unroll
+      for (int kk = 0; kk < AS / 16; ++kk) {
+        ptx::umma_bf16(tmem, desc_mn(sP, kk), desc_mn(sdO, kk), idesc_t, kk > 0);        // dV = P^T dO
+        ptx::umma_bf16(tmem + HD, desc_mn(sdS, kk), desc_mn(sQ, kk), idesc_t, kk > 0);   // dK = dS^T Q
+        ptx::umma_bf16(tmem + 256, desc_k(sdS, kk), desc_mn(sK, kk), idesc_q, kk > 0);   // dQ = dS K
+      }
+      ptx::umma_commit(&bar[2]);
     }
-    ptx::umma_commit(&bar[2]);
+    __syncwarp();
   }
   ptx::mbar_wait(&bar[2], 0);
   ptx::tc_fence_after();
@@ -320,7 +332,7 @@ __global__ void __launch_bounds__(128, 2) attn_bwd_tc64_kernel(const __grid_cons
   uint64_t* bar = reinterpret_cast<uint64_t*>(sB + 2 * TILE);  // [0] TMA, [1] S + dP, [2] dV, [3] dK + dQ
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bar + 4);
   const int bh = blockIdx.x, b = bh / h, hh = bh % h;
-  const int warp = threadIdx.x >> 5, r = threadIdx.x;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, r = threadIdx.x;
   if (threadIdx.x == 0) {
     ptx::tma_prefetch(&tq);
     ptx::tma_prefetch(&tdo);
@@ -333,21 +345,24 @@ __global__ void __launch_bounds__(128, 2) attn_bwd_tc64_kernel(const __grid_cons
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_holder;
-  if (threadIdx.x == 0) {
-    ptx::mbar_arrive_expect_tx(&bar[0], 4 * TILE);
-    ptx::tma_load_2d(sQ, &tq, &bar[0], hh * HD, b * AS);
-    ptx::tma_load_2d(sK, &tq, &bar[0], d + hh * HD, b * AS);
-    ptx::tma_load_2d(sV, &tq, &bar[0], 2 * d + hh * HD, b * AS);
-    ptx::tma_load_2d(sdO, &tdo, &bar[0], hh * HD, b * AS);
-    ptx::mbar_wait(&bar[0], 0);
-    ptx::tc_fence_after();
-    constexpr uint32_t idesc = ptx::umma_idesc_bf16(128, 128, 0, 0);
-#pragma unroll
-    for (int kk = 0; kk < HD / 16; ++kk) {
-      ptx::umma_bf16(tmem, desc_k(sQ, kk), desc_k(sK, kk), idesc, kk > 0);         // S = Q K^T
-      ptx::umma_bf16(tmem + 128, desc_k(sdO, kk), desc_k(sV, kk), idesc, kk > 0);  // dP = dO V^T
+  if (warp == 0) {  // lane 0 issues; lanes 1-31 wait at the __syncwarp, not spinning on an mbarrier
+    if (lane == 0) {
+      ptx::mbar_arrive_expect_tx(&bar[0], 4 * TILE);
+      ptx::tma_load_2d(sQ, &tq, &bar[0], hh * HD, b * AS);
+      ptx::tma_load_2d(sK, &tq, &bar[0], d + hh * HD, b * AS);
+      ptx::tma_load_2d(sV, &tq, &bar[0], 2 * d + hh * HD, b * AS);
+      ptx::tma_load_2d(sdO, &tdo, &bar[0], hh * HD, b * AS);
+      ptx::mbar_wait(&bar[0], 0);
+      ptx::tc_fence_after();
+      constexpr uint32_t idesc = ptx::umma_idesc_bf16(128, 128, 0, 0);
+  #pragma unroll
+      for (int kk = 0; kk < HD / 16; ++kk) {
+        ptx::umma_bf16(tmem, desc_k(sQ, kk), desc_k(sK, kk), idesc, kk > 0);         // S = Q K^T
+        ptx::umma_bf16(tmem + 128, desc_k(sdO, kk), desc_k(sV, kk), idesc, kk > 0);  // dP = dO V^T
+      }
+      ptx::umma_commit(&bar[1]);
     }
-    ptx::umma_commit(&bar[1]);
+    __syncwarp();
   }
   const bf16* drow = dout + ((size_t)b * AS + r) * d + hh * HD;
   const bf16* orow = o + ((size_t)b * AS + r) * d + hh * HD;
@@ -393,10 +408,13 @@ __global__ void __launch_bounds__(128, 2) attn_bwd_tc64_kernel(const __grid_cons
   ptx::tc_fence_after();
   constexpr uint32_t idesc_t = ptx::umma_idesc_bf16(128, HD, 1, 1);
   constexpr uint32_t idesc_q = ptx::umma_idesc_bf16(128, HD, 0, 1);
-  if (threadIdx.x == 0) {
-#pragma unroll
-    for (int kk = 0; kk < AS / 16; ++kk) ptx::umma_bf16(tmem, desc_mn(sB, kk), desc_mn(sdO, kk), idesc_t, kk > 0);  // dV
-    ptx::umma_commit(&bar[2]);
+  if (warp == 0) {  // lane 0 issues; lanes 1-31 wait at the __syncwarp, not spinning on an mbarrier
+    if (lane == 0) {
+  #pragma unroll
+      for (int kk = 0; kk < AS / 16; ++kk) ptx::umma_bf16(tmem, desc_mn(sB, kk), desc_mn(sdO, kk), idesc_t, kk > 0);  // dV
+      ptx::umma_commit(&bar[2]);
+    }
+    __syncwarp();
   }
   ptx::mbar_wait(&bar[2], 0);  // dV done: the tensor core no longer reads P
   ptx::tc_fence_after();
@@ -410,13 +428,16 @@ __global__ void __launch_bounds__(128, 2) attn_bwd_tc64_kernel(const __grid_cons
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
-  if (threadIdx.x == 0) {
-#pragma unroll
-    for (int kk = 0; kk < AS / 16; ++kk) {
-      ptx::umma_bf16(tmem + HD, desc_mn(sB, kk), desc_mn(sQ, kk), idesc_t, kk > 0);      // dK = dS^T Q
-      ptx::umma_bf16(tmem + 2 * HD, desc_k(sB, kk), desc_mn(sK, kk), idesc_q, kk > 0);   // dQ = dS K
+  if (warp == 0) {  // lane 0 issues; lanes 1-31 wait at the __syncwarp, not spinning on an mbarrier
+    if (lane == 0) {
+  #pragma unroll
+      for (int kk = 0; kk < AS / 16; ++kk) {
+        ptx::umma_bf16(tmem + HD, desc_mn(sB, kk), desc_mn(sQ, kk), idesc_t, kk > 0);      // dK = dS^T Q
+        ptx::umma_bf16(tmem + 2 * HD, desc_k(sB, kk), desc_mn(sK, kk), idesc_q, kk > 0);   // dQ = dS K
+      }
+      ptx::umma_commit(&bar[3]);
     }
-    ptx::umma_commit(&bar[3]);
+    __syncwarp();
   }
   ptx::mbar_wait(&bar[3], 0);
   ptx::tc_fence_after();
