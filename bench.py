@@ -368,7 +368,8 @@ def algorithmic_work(cfg, st, steps):
 
 def workload_config(args, cfg, world):
     names = {"transformer": "configs[2] transformer", "large_transformer": "configs[3] large_transformer",
-             "toy": "configs[0] toy", "spos": "configs[1] SPOS CNN"}
+             "toy": "configs[0] toy", "spos": "configs[1] SPOS CNN",
+             "cv_c3": "CV.c3 analog (Table 1: 32 blocks x 12 choices, Table 5 ops incl. dilated)"}
     c = {"workload": names.get(args.workload, args.workload) if not args.n_choices
          else f"configs[4] sweep n={args.n_choices}",
          "n_blocks": cfg["n_blocks"], "n_choices": cfg["n_choices"], "batch": cfg["batch"],
@@ -381,6 +382,7 @@ def workload_config(args, cfg, world):
     if cfg["family"] == "spos":
         c.update(image_hw=cfg["image_hw"], stage_repeats=cfg["stage_repeats"], stage_channels=cfg["stage_channels"],
                  choice_kernel=cfg["choice_kernel"], choice_xception=cfg["choice_xception"],
+                 choice_dilation=cfg.get("choice_dilation", [1] * cfg["n_choices"]),
                  num_classes=cfg["num_classes"])
     return c
 
@@ -431,7 +433,8 @@ def main():
     if world == 1 and args.workload == "spos" and not args.no_secondary and not args.n_choices:
         sec = {"configs[2] transformer": secondary(args, "transformer"),
                "configs[3] large_transformer (budget 3x, context switching)":
-                   secondary(args, "large_transformer", ["--budget-x", "3", "--no-repro"], steps=min(args.steps, 12))}
+                   secondary(args, "large_transformer", ["--budget-x", "3", "--no-repro"], steps=min(args.steps, 12)),
+               "CV.c3 analog (32 x 12, dilated candidates)": secondary(args, "cv_c3", ["--no-repro"])}
 
     import torch
     import torch.distributed as dist

@@ -43,7 +43,7 @@ extern "C" {
 #pragma GCC visibility push(default) /* the library builds with -fvisibility=hidden */
 #endif
 
-#define NASPIPE_ABI_VERSION 3
+#define NASPIPE_ABI_VERSION 4
 
 typedef enum {
   NASPIPE_OK = 0,
@@ -138,7 +138,10 @@ typedef enum { NASPIPE_FP32 = 0, NASPIPE_BF16 = 1 } naspipe_dtype; /* compute dt
  *                 strictly increasing, first > stem_channels): the first block of each
  *                 stage has stride 2, inp = C_prev, mid = C/2, out = C - C_prev; the
  *                 others stride 1 with inp = mid = out = C/2 (channel split).
- *   choice_kernel[n] (3, 5 or 7), choice_xception[n] (0 = Shuffle, 1 = Xception k=3)
+ *   choice_kernel[n] (3, 5 or 7): the k of every depthwise conv of choice n;
+ *   choice_xception[n] (0 = Shuffle, 1 = Xception); choice_dilation[n] (ABI 4; 1 or 2,
+ *                 NULL = all 1): dilation of choice n's depthwise convs, pad dilation*(k/2)
+ *                 (Table 5's "Dil Conv 3x3"; A36)
  *   Frozen stem/head/FC weights use the counter hash with uids m*n + {0, 1, 2}, fan_in
  *   27 / C_last / head_channels; they are never updated (reading A2).
  */
@@ -179,6 +182,8 @@ typedef struct {
   /* ABI 3: synchronisation policy (naspipe_sync; 0 = CSP) and BSP bulk size (0 = 4 * n_stages) */
   int32_t sync_policy;
   int32_t bulk_size;
+  /* ABI 4: per-choice depthwise dilation (SPOS_CNN; NULL = 1) */
+  const int32_t* choice_dilation;
 } naspipe_supernet_spec;
 
 /* naspipe_batch.where */

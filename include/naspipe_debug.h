@@ -33,10 +33,10 @@ int naspipe_debug_ln_bwd(const float* dy, const float* x, const float* mean, con
 
 /* SPOS CNN kernels (spos.cu).  NHWC tensors [P = B*H*W rows][C]; forward tensors are
  * bf16x2 (hi plane followed by the lo plane; value = hi + lo), gradients plain bf16.
- * depthwise k x k, stride S, pad k/2, w fp32 [C][k][k]: z = dw(x) (x2 -> x2) if x && z;
+ * depthwise k x k, stride S, dilation dil (1 or 2), pad dil*(k/2), w fp32 [C][k][k]: z = dw(x) (x2 -> x2) if x && z;
  * dx = dw'(dz) (+ add) if dz && dx; dwsum[C*k*k] = sum(dz * x_hi) if dz && x && dwsum. */
 int naspipe_debug_dw(const void* x, const float* w, void* z, const void* dz, const void* add, void* dx,
-                     float* dwsum, int B, int H, int C, int k, int S, void* stream);
+                     float* dwsum, int B, int H, int C, int k, int S, int dil, void* stream);
 /* BatchNorm forward: mean/rstd of z (x2) over P rows (biased variance, eps 1e-5), then
  * y[p*ldy + c] = relu?(g (z - mean) rstd + b) (x2, lo plane yplane elements after hi). */
 int naspipe_debug_bn_fwd(const void* z, int P, int C, const float* g, const float* b, int relu, void* y, int ldy,

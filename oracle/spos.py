@@ -102,8 +102,16 @@ def block_dims(cfg, b):
     raise IndexError(b)
 
 
+def dilation(cfg, c):
+    """Dilation of candidate c's depthwise convs (Table 5's "Dil Conv 3x3"; reading
+    A36): cfg["choice_dilation"][c], default 1."""
+    return int(cfg.get("choice_dilation", [1] * cfg["n_choices"])[c])
+
+
 def convs(cfg, b, c):
-    """Ordered conv list of candidate (b, c): (name, kind 'pw'|'dw', cin, cout, k, stride)."""
+    """Ordered conv list of candidate (b, c): (name, kind 'pw'|'dw', cin, cout, k, stride).
+    Every depthwise conv of the candidate uses its kernel size k = choice_kernel[c] (the
+    Xception choice of the default configs has k = 3) and its dilation (dilation())."""
     s, inp, mid, out, _, _ = block_dims(cfg, b)
     k = cfg["choice_kernel"][c]
     L = []
@@ -112,8 +120,8 @@ def convs(cfg, b, c):
     if not cfg["choice_xception"][c]:
         L += [("m_pw1", "pw", inp, mid, 1, 1), ("m_dw", "dw", mid, mid, k, s), ("m_pw2", "pw", mid, out, 1, 1)]
     else:
-        L += [("x_dw1", "dw", inp, inp, 3, s), ("x_pw1", "pw", inp, mid, 1, 1), ("x_dw2", "dw", mid, mid, 3, 1),
-              ("x_pw2", "pw", mid, mid, 1, 1), ("x_dw3", "dw", mid, mid, 3, 1), ("x_pw3", "pw", mid, out, 1, 1)]
+        L += [("x_dw1", "dw", inp, inp, k, s), ("x_pw1", "pw", inp, mid, 1, 1), ("x_dw2", "dw", mid, mid, k, 1),
+              ("x_pw2", "pw", mid, mid, 1, 1), ("x_dw3", "dw", mid, mid, k, 1), ("x_pw3", "pw", mid, out, 1, 1)]
     return L
 
 
@@ -142,30 +150,31 @@ def pad_hw(x, p):
     return np.pad(x, ((0, 0), (p, p), (p, p), (0, 0)))
 
 
-def dw_fwd(x, w, s):
-    """Depthwise conv, pad k//2: y[b,i,j,c] = sum_{u,v} xpad[b, i*s+u, j*s+v, c] w[c,u,v]."""
+def dw_fwd(x, w, s, dil=1):
+    """Depthwise conv, pad dil*(k//2): y[b,i,j,c] = sum_{u,v} xpad[b, i*s+u*dil, j*s+v*dil, c] w[c,u,v]."""
     k = w.shape[1]
-    p = k // 2
+    p = dil * (k // 2)
     xp = pad_hw(x, p)
     B, H, W, C = x.shape
-    Ho, Wo = (H + 2 * p - k) // s + 1, (W + 2 * p - k) // s + 1
+    Ho, Wo = (H + 2 * p - dil * (k - 1) - 1) // s + 1, (W + 2 * p - dil * (k - 1) - 1) // s + 1
     y = np.zeros((B, Ho, Wo, C))
     for u in range(k):
         for v in range(k):
-            y += xp[:, u:u + s * (Ho - 1) + 1:s, v:v + s * (Wo - 1) + 1:s, :] * w[:, u, v]
+            y += xp[:, u * dil:u * dil + s * (Ho - 1) + 1:s, v * dil:v * dil + s * (Wo - 1) + 1:s, :] * w[:, u, v]
     return y
 
 
-def dw_bwd(x, w, s, dy):
+def dw_bwd(x, w, s, dy, dil=1):
     k = w.shape[1]
-    p = k // 2
+    p = dil * (k // 2)
     xp = pad_hw(x, p)
     B, Ho, Wo, C = dy.shape
     dxp = np.zeros_like(xp)
     dw = np.zeros_like(w)
     for u in range(k):
         for v in range(k):
-            sl = (slice(None), slice(u, u + s * (Ho - 1) + 1, s), slice(v, v + s * (Wo - 1) + 1, s), slice(None))
+            sl = (slice(None), slice(u * dil, u * dil + s * (Ho - 1) + 1, s),
+                  slice(v * dil, v * dil + s * (Wo - 1) + 1, s), slice(None))
             dxp[sl] += dy * w[:, u, v]
             dw[:, u, v] = np.sum(dy * xp[sl], axis=(0, 1, 2))
     return dxp[:, p:p + x.shape[1], p:p + x.shape[2], :], dw
@@ -201,9 +210,9 @@ def bn_bwd(dy, g, cache):
 
 
 # ------------------------------------------------------------------ conv -> BN [-> ReLU] unit
-def _unit_fwd(p, name, kind, s, relu, x, st=PLAIN):
+def _unit_fwd(p, name, kind, s, relu, x, st=PLAIN, dil=1):
     w = p[name]
-    z = st.f(dw_fwd(x, w, s) if kind == "dw" else x @ st.w(w).T)
+    z = st.f(dw_fwd(x, w, s, dil) if kind == "dw" else x @ st.w(w).T)
     y, cb = bn_fwd(z, p[name + "_g"], p[name + "_b"])
     if relu:
         y = np.maximum(y, 0.0)
@@ -211,7 +220,7 @@ def _unit_fwd(p, name, kind, s, relu, x, st=PLAIN):
     return y, (x, cb, y if relu else None)
 
 
-def _unit_bwd(p, name, kind, s, dy, tape, grads, st=PLAIN, add=None):
+def _unit_bwd(p, name, kind, s, dy, tape, grads, st=PLAIN, add=None, dil=1):
     """dx of the unit (+ add, the other branch's gradient of the same input, before the
     storage rounding), accumulating the parameter gradients into grads."""
     x, cb, yr = tape
@@ -220,8 +229,8 @@ def _unit_bwd(p, name, kind, s, dy, tape, grads, st=PLAIN, add=None):
     dz, grads[name + "_g"], grads[name + "_b"] = bn_bwd(dy, p[name + "_g"], cb)
     dz = st.b(dz)
     if kind == "dw":
-        dx, _ = dw_bwd(x, p[name], s, dz)
-        _, grads[name] = dw_bwd(st.op(x), p[name], s, dz)
+        dx, _ = dw_bwd(x, p[name], s, dz, dil)
+        _, grads[name] = dw_bwd(st.op(x), p[name], s, dz, dil)
     else:
         grads[name] = np.einsum("bhwo,bhwi->oi", dz, st.op(x))
         dx = dz @ st.op(p[name])
@@ -229,12 +238,13 @@ def _unit_bwd(p, name, kind, s, dy, tape, grads, st=PLAIN, add=None):
 
 
 def _chain(cfg, b, c, which):
-    """Units of the proj ('p') or main branch: (name, kind, stride, relu)."""
+    """Units of the proj ('p') or main branch: (name, kind, stride, relu, dilation)."""
     out = []
+    d = dilation(cfg, c)
     cl = [u for u in convs(cfg, b, c) if u[0].startswith(which)]
     for i, (name, kind, _, _, _, s) in enumerate(cl):
         relu = kind == "pw" and (which == "p" or i == len(cl) - 1 or name in ("m_pw1", "x_pw1", "x_pw2"))
-        out.append((name, kind, s, relu))
+        out.append((name, kind, s, relu, d if kind == "dw" else 1))
     return out
 
 
@@ -247,14 +257,14 @@ def block_fwd(cfg, b, c, p, x, st=PLAIN):
         xp = xm = x
     tapes = {"p": [], main_key: []}
     h = xm
-    for name, kind, stride, relu in _chain(cfg, b, c, main_key):
-        h, t = _unit_fwd(p, name, kind, stride, relu, h, st)
+    for name, kind, stride, relu, dil in _chain(cfg, b, c, main_key):
+        h, t = _unit_fwd(p, name, kind, stride, relu, h, st, dil)
         tapes[main_key].append(t)
     main = h
     if s == 2:
         h = xp
-        for name, kind, stride, relu in _chain(cfg, b, c, "p"):
-            h, t = _unit_fwd(p, name, kind, stride, relu, h, st)
+        for name, kind, stride, relu, dil in _chain(cfg, b, c, "p"):
+            h, t = _unit_fwd(p, name, kind, stride, relu, h, st, dil)
             tapes["p"].append(t)
         xp = h
     return np.concatenate([xp, main], axis=-1), tapes
@@ -268,8 +278,8 @@ def block_bwd(cfg, b, c, p, tapes, dy, st=PLAIN):
     grads = {}
     h = d_main
     chain = _chain(cfg, b, c, main_key)
-    for (name, kind, stride, relu), t in zip(reversed(chain), reversed(tapes[main_key])):
-        h = _unit_bwd(p, name, kind, stride, h, t, grads, st)
+    for (name, kind, stride, relu, dil), t in zip(reversed(chain), reversed(tapes[main_key])):
+        h = _unit_bwd(p, name, kind, stride, h, t, grads, st, dil=dil)
     if s == 1:
         dx = np.zeros(d_proj.shape[:-1] + (2 * cp,))
         dx[..., 0::2] = d_proj
@@ -277,9 +287,9 @@ def block_bwd(cfg, b, c, p, tapes, dy, st=PLAIN):
         return dx, grads
     g = d_proj
     pchain = list(zip(reversed(_chain(cfg, b, c, "p")), reversed(tapes["p"])))
-    for i, ((name, kind, stride, relu), t) in enumerate(pchain):
+    for i, ((name, kind, stride, relu, dil), t) in enumerate(pchain):
         last = i == len(pchain) - 1     # the proj branch's first unit: add the main branch's dx
-        g = _unit_bwd(p, name, kind, stride, g, t, grads, st, add=h if last else None)
+        g = _unit_bwd(p, name, kind, stride, g, t, grads, st, add=h if last else None, dil=dil)
     return g, grads
 
 

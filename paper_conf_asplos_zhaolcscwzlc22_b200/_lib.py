@@ -10,7 +10,7 @@ if not os.path.exists(LIB_PATH):
                       "`python -m paper_conf_asplos_zhaolcscwzlc22_b200.build` (no CPU fallback exists)")
 lib = C.CDLL(LIB_PATH)
 
-ABI_VERSION = 3
+ABI_VERSION = 4
 SYNC = {"csp": 0, "inorder": 1, "asp": 2, "bsp": 3, "serial": 4}  # naspipe_sync (include/naspipe.h)
 FAMILY = {"mlp": 0, "transformer": 1, "spos": 2}
 DTYPE = {"fp32": 0, "bf16": 1}
@@ -37,7 +37,7 @@ class _SpecStruct(C.Structure):
                 ("image_hw", C.c_int32), ("num_classes", C.c_int32), ("stem_channels", C.c_int32),
                 ("head_channels", C.c_int32), ("n_cnn_stages", C.c_int32), ("stage_repeats", _i32p),
                 ("stage_channels", _i32p), ("choice_kernel", _i32p), ("choice_xception", _i32p),
-                ("sync_policy", C.c_int32), ("bulk_size", C.c_int32)]
+                ("sync_policy", C.c_int32), ("bulk_size", C.c_int32), ("choice_dilation", _i32p)]
 
 
 class _BatchStruct(C.Structure):
@@ -130,7 +130,7 @@ class Spec:
         s.d_model, s.seq_len = cfg.get("d_model", 0), cfg.get("seq_len", 0)
         self._keep = []
         for name in ("choice_heads", "choice_ffn", "stage_of_block", "cost_fwd", "cost_bwd", "stage_repeats",
-                     "stage_channels", "choice_kernel", "choice_xception"):
+                     "stage_channels", "choice_kernel", "choice_xception", "choice_dilation"):
             if cfg.get(name) is not None:
                 arr, ptr = _i32(np.asarray(cfg[name]).ravel())
                 self._keep.append(arr)

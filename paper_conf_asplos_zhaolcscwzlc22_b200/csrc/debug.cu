@@ -105,11 +105,11 @@ int naspipe_debug_ln_bwd(const float* dy, const float* x, const float* mean, con
 
 
 int naspipe_debug_dw(const void* x, const float* w, void* z, const void* dz, const void* add, void* dx,
-                     float* dwsum, int B, int H, int C, int k, int S, void* stream) {
+                     float* dwsum, int B, int H, int C, int k, int S, int dil, void* stream) {
   return dguard([&] {
     cudaStream_t s = (cudaStream_t)stream;
-    if (x && z) dw_fwd(s, (const bf16*)x, w, (bf16*)z, B, H, C, k, S);
-    if (dz && dx) dw_dgrad(s, (const bf16*)dz, w, (const bf16*)add, (bf16*)dx, B, H, C, k, S);
+    if (x && z) dw_fwd(s, (const bf16*)x, w, (bf16*)z, B, H, C, k, S, dil);
+    if (dz && dx) dw_dgrad(s, (const bf16*)dz, w, (const bf16*)add, (bf16*)dx, B, H, C, k, S, dil);
     if (dz && x && dwsum) {
       unsigned long long* acc = nullptr;
       int* ticket = nullptr;
@@ -118,7 +118,7 @@ int naspipe_debug_dw(const void* x, const float* w, void* z, const void* dz, con
       cudaMemsetAsync(acc, 0, ((size_t)C * k * k + 1) * 8, s);
       cudaMemsetAsync(ticket, 0, 4, s);
       cudaMemsetAsync(dwsum, 0, (size_t)C * k * k * 4, s);
-      dw_wgrad_sgd(s, (const bf16*)dz, (const bf16*)x, acc, ticket, dwsum, -1.0f, B, H, C, k, S);  // 0 + sum
+      dw_wgrad_sgd(s, (const bf16*)dz, (const bf16*)x, acc, ticket, dwsum, -1.0f, B, H, C, k, S, dil);  // 0 + sum
       cudaStreamSynchronize(s);
       cudaFree(acc);
       cudaFree(ticket);

@@ -354,7 +354,7 @@ class SposFamily : public Family {
       cv += 2 * zplane;
       st += 2 * u.cout;
       if (u.dw) {  // the depthwise conv adds the BatchNorm sums of its output itself (fused bn_stats)
-        dw_fwd(s, h, Pm + u.off_w, r.z, B_, u.H_in, u.cin, u.k, u.stride, acc_f_);
+        dw_fwd(s, h, Pm + u.off_w, r.z, B_, u.H_in, u.cin, u.k, u.stride, u.dil, acc_f_);
         counters.launches++;
       } else {
         GemmEpiParams e;  // the GEMM epilogue adds the BatchNorm sums of z (fused bn_stats)
@@ -406,7 +406,7 @@ class SposFamily : public Family {
     const bf16* dz = dz_[ring_];
     if (dst) {
       if (u.dw) {
-        dw_dgrad(s, dz, Pm + u.off_w, add, dst, B_, u.H_in, u.cin, u.k, u.stride);
+        dw_dgrad(s, dz, Pm + u.off_w, add, dst, B_, u.H_in, u.cin, u.k, u.stride, u.dil);
         counters.launches++;
       } else {
         NP_REQUIRE(add == nullptr, NASPIPE_EINTERNAL, "pw dgrad with an addend");
@@ -418,7 +418,7 @@ class SposFamily : public Family {
     cudaEventRecord(ev_dg_[ring_], s);
     cudaStreamWaitEvent(side_, ev_dg_[ring_], 0);
     if (u.dw) {
-      dw_wgrad_sgd(side_, dz, r.x, acc_w_, tick_ + 2, Um + u.off_w, lr_, B_, u.H_in, u.cin, u.k, u.stride);
+      dw_wgrad_sgd(side_, dz, r.x, acc_w_, tick_ + 2, Um + u.off_w, lr_, B_, u.H_in, u.cin, u.k, u.stride, u.dil);
       counters.launches += 1;
     } else {
       GemmEpiParams e;

@@ -157,18 +157,19 @@ void bn_bwd_apply(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P
                   unsigned long long* acc, int* ticket, int relu, bf16* dz);
 // acc holds 2C sums + the sticky overflow flag acc[2C] (fixpoint.cuh; checked at drain)
 bool bn_fix_overflow(const unsigned long long* acc, int C);
-// depthwise k x k (k in {3,5,7}), stride S, pad k/2; w fp32 [C][k][k]; H = input height = width.
+// depthwise k x k (k in {3,5,7}), stride S, dilation dil (1 or 2), pad dil*(k/2); w fp32 [C][k][k];
+// H = input height = width.
 // dw_fwd: x2 -> x2; dw_dgrad: bf16 (+ bf16 add); dw_wgrad reads the hi plane of x.
 // stats != nullptr: also add the BatchNorm sums of the stored z to it (bn_stats fused)
-void dw_fwd(cudaStream_t s, const bf16* x, const float* w, bf16* z, int B, int H, int C, int k, int S,
+void dw_fwd(cudaStream_t s, const bf16* x, const float* w, bf16* z, int B, int H, int C, int k, int S, int dil,
             unsigned long long* stats = nullptr);
 void dw_dgrad(cudaStream_t s, const bf16* dz, const float* w, const bf16* add, bf16* dx, int B, int H, int C, int k,
-              int S);
+              int S, int dil);
 int dw_wgrad_blocks(int B, int H, int C, int k, int S);
 // weight gradient of a depthwise conv with the SGD WRITE fused: w -= lr * sum over the batch
 // (acc [C*k*k + 1] and ticket zero between uses, fixpoint.cuh; w = master or BSP accumulator)
 void dw_wgrad_sgd(cudaStream_t s, const bf16* dz, const bf16* x, unsigned long long* acc, int* ticket, float* w,
-                  float lr, int B, int H, int C, int k, int S);
+                  float lr, int B, int H, int C, int k, int S, int dil);
 // channel split of a stride-1 block input [P, 2Ch] (x2): out[:, i] = x[:, 2i] (ld ldo, planes
 // oplane apart), xm[:, i] = x[:, 2i+1]; merge is its (plain bf16) backward
 void chan_split(cudaStream_t s, const bf16* x, int P, int Ch, bf16* out, int ldo, size_t oplane, bf16* xm);

@@ -75,6 +75,8 @@ Spec::Spec(const naspipe_supernet_spec* s) {
     chans.assign(raw.stage_channels, raw.stage_channels + raw.n_cnn_stages);
     kern.assign(raw.choice_kernel, raw.choice_kernel + n);
     xcep.assign(raw.choice_xception, raw.choice_xception + n);
+    if (raw.choice_dilation) dil.assign(raw.choice_dilation, raw.choice_dilation + n);
+    else dil.assign(n, 1);
     int total = 0, prev = raw.stem_channels;
     NP_REQUIRE(raw.stem_channels >= 16 && raw.stem_channels % 16 == 0, NASPIPE_EINVAL, "stem_channels %d (%%16)",
                raw.stem_channels);
@@ -91,9 +93,10 @@ Spec::Spec(const naspipe_supernet_spec* s) {
     NP_REQUIRE(raw.num_classes >= 2 && raw.head_channels >= 16 && raw.head_channels % 16 == 0, NASPIPE_EINVAL,
                "num_classes %d / head_channels %d (%%16)", raw.num_classes, raw.head_channels);
     for (int c = 0; c < n; ++c)
-      NP_REQUIRE((kern[c] == 3 || kern[c] == 5 || kern[c] == 7) && (xcep[c] == 0 || (xcep[c] == 1 && kern[c] == 3)),
-                 NASPIPE_EINVAL, "choice %d: kernel %d xception %d (k in {3,5,7}; Xception uses k=3)", c, kern[c],
-                 xcep[c]);
+      NP_REQUIRE((kern[c] == 3 || kern[c] == 5 || kern[c] == 7) && (xcep[c] == 0 || xcep[c] == 1) &&
+                     (dil[c] == 1 || dil[c] == 2),
+                 NASPIPE_EINVAL, "choice %d: kernel %d xception %d dilation %d (k in {3,5,7}, dilation 1 or 2)", c,
+                 kern[c], xcep[c], dil[c]);
   }
   if (raw.stage_of_block) {
     stage_of_block.assign(raw.stage_of_block, raw.stage_of_block + m);
@@ -114,7 +117,7 @@ Spec::Spec(const naspipe_supernet_spec* s) {
 Spec::Spec(const Spec& o)
     : raw(o.raw), heads(o.heads), ffn(o.ffn), stage_of_block(o.stage_of_block),
       cost_fwd(o.cost_fwd), cost_bwd(o.cost_bwd), reps(o.reps), chans(o.chans), kern(o.kern),
-      xcep(o.xcep), has_partition(o.has_partition), has_costs(o.has_costs) {
+      xcep(o.xcep), dil(o.dil), has_partition(o.has_partition), has_costs(o.has_costs) {
   repoint();
 }
 
@@ -128,6 +131,7 @@ void Spec::repoint() {
   raw.stage_channels = chans.empty() ? nullptr : chans.data();
   raw.choice_kernel = kern.empty() ? nullptr : kern.data();
   raw.choice_xception = xcep.empty() ? nullptr : xcep.data();
+  raw.choice_dilation = dil.empty() ? nullptr : dil.data();
 }
 
 size_t Spec::sample_elems() const {
@@ -176,12 +180,13 @@ int Spec::spos_last_hw() const { return raw.image_hw >> (1 + (int)reps.size()); 
 
 std::vector<SposConv> Spec::spos_convs(int b, int c) const {
   const SposDims d = spos_dims(b);
-  const int k = kern[c];
+  const int k = kern[c], dl = dil[c];
   std::vector<SposConv> L;
   // (branch, dw, cin, cout, k, stride, relu, H_in, H_out)
   auto add = [&](int br, int dw, int ci, int co, int kk, int s, int relu, int hin) {
     SposConv u{};
     u.branch = br; u.dw = dw; u.cin = ci; u.cout = co; u.k = kk; u.stride = s; u.relu = relu;
+    u.dil = dw ? dl : 1;
     u.H_in = hin; u.H_out = hin / s;
     L.push_back(u);
   };
@@ -195,11 +200,11 @@ std::vector<SposConv> Spec::spos_convs(int b, int c) const {
     add(1, 1, d.mid, d.mid, k, s, 0, H);
     add(1, 0, d.mid, d.outm, 1, 1, 1, Ho);
   } else {
-    add(1, 1, d.inp, d.inp, 3, s, 0, H);
+    add(1, 1, d.inp, d.inp, k, s, 0, H);
     add(1, 0, d.inp, d.mid, 1, 1, 1, Ho);
-    add(1, 1, d.mid, d.mid, 3, 1, 0, Ho);
+    add(1, 1, d.mid, d.mid, k, 1, 0, Ho);
     add(1, 0, d.mid, d.mid, 1, 1, 1, Ho);
-    add(1, 1, d.mid, d.mid, 3, 1, 0, Ho);
+    add(1, 1, d.mid, d.mid, k, 1, 0, Ho);
     add(1, 0, d.mid, d.outm, 1, 1, 1, Ho);
   }
   size_t off = 0, off16 = 0;

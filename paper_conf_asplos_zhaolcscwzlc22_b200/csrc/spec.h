@@ -35,6 +35,7 @@ struct SposConv {
   int branch;   // 0 = proj (stride-2 blocks), 1 = main
   int dw;       // 1 = depthwise k x k, 0 = pointwise
   int cin, cout, k, stride;
+  int dil;      // dw: dilation (1, or 2 for Table 5's Dil Conv; reading A36)
   int relu;     // ReLU after the BN
   int H_in, H_out;
   size_t off_w, off_g, off_b;  // offsets in the packed fp32 vector
@@ -44,7 +45,7 @@ struct SposConv {
 struct Spec {
   naspipe_supernet_spec raw{};  // scalar fields; pointer fields re-pointed into vectors below
   std::vector<int32_t> heads, ffn, stage_of_block, cost_fwd, cost_bwd;
-  std::vector<int32_t> reps, chans, kern, xcep;  // SPOS
+  std::vector<int32_t> reps, chans, kern, xcep, dil;  // SPOS
   bool has_partition = false, has_costs = false;
 
   explicit Spec(const naspipe_supernet_spec* s);

@@ -488,15 +488,16 @@ __device__ __forceinline__ void stage_dw_weights(float* ws, const float* w, int 
   __syncthreads();
 }
 
-// dx[b,ih,iw,c] = sum_{u,v} dz[b,oh,ow,c] w[c,u,v] with oh*S + u - PAD = ih (+ add[b,ih,iw,c])
-template <int K>
+// dx[b,ih,iw,c] = sum_{u,v} dz[b,oh,ow,c] w[c,u,v] with oh*S + u*DIL - PAD = ih (+ add[b,ih,iw,c]),
+// PAD = DIL*(K/2) (DIL = 2: Table 5's dilated convs, reading A36)
+template <int K, int DIL>
 __global__ void dw_dgrad_kernel(const bf16* __restrict__ dz, const float* __restrict__ w, const bf16* __restrict__ add,
                                 bf16* __restrict__ dx, int B, int H, int C, int S) {
   extern __shared__ float ws[];
   ptx::pdl_wait();
   stage_dw_weights<K>(ws, w, C);
-  constexpr int PAD = K / 2;
-  const int Ho = (H + 2 * PAD - K) / S + 1;
+  constexpr int PAD = DIL * (K / 2), KE = DIL * (K - 1) + 1;
+  const int Ho = (H + 2 * PAD - KE) / S + 1;
   const int G = C / 8;
   const size_t items = (size_t)B * H * H * G;
   for (size_t it = blockIdx.x * (size_t)blockDim.x + threadIdx.x; it < items; it += (size_t)gridDim.x * blockDim.x) {
@@ -508,13 +509,13 @@ __global__ void dw_dgrad_kernel(const bf16* __restrict__ dz, const float* __rest
     float acc[8] = {};
 #pragma unroll
     for (int u = 0; u < K; ++u) {
-      const int t = ih + PAD - u;
+      const int t = ih + PAD - u * DIL;
       if (t < 0 || t % S) continue;
       const int oh = t / S;
       if (oh >= Ho) continue;
 #pragma unroll
       for (int v = 0; v < K; ++v) {
-        const int q = iw + PAD - v;
+        const int q = iw + PAD - v * DIL;
         if (q < 0 || q % S) continue;
         const int ow = q / S;
         if (ow >= Ho) continue;
@@ -536,7 +537,8 @@ __global__ void dw_dgrad_kernel(const bf16* __restrict__ dz, const float* __rest
 }
 
 // ---------------------------------------------------------------- depthwise conv, shared-memory tiles
-// Correlation out[b,oh,ow,c] = sum_{u,v} in[b, oh*S+u-PAD, ow*S+v-PAD, c] w'[c,u,v] (+ add),
+// Correlation out[b,oh,ow,c] = sum_{u,v} in[b, oh*S+u*DIL-PAD, ow*S+v*DIL-PAD, c] w'[c,u,v] (+ add),
+// PAD = DIL*(K/2), KE = DIL*(K-1)+1 the dilated extent,
 // w' = w (forward) or w flipped in u and v (FLIP: the stride-1 input gradient).  A CTA owns
 // a tile of DT_H output rows x TW columns x CPG groups of 8 channels: the input halo is
 // staged in shared memory once (16-byte loads, fp32), each thread keeps one channel's k x k
@@ -544,15 +546,15 @@ __global__ void dw_dgrad_kernel(const bf16* __restrict__ dz, const float* __rest
 // staged value feeds up to DT_H outputs).  X2: bf16x2 input/output (forward), else bf16.
 constexpr int DT_H = 8;
 
-template <int K, int S, bool X2, bool FLIP>
+template <int K, int S, int DIL, bool X2, bool FLIP>
 __global__ void __launch_bounds__(TPB) dw_tile_kernel(const bf16* __restrict__ in, const float* __restrict__ w,
                                                     const bf16* __restrict__ add, bf16* __restrict__ out, int B,
                                                     int H, int C, int TW, unsigned long long* stats) {
-  constexpr int PAD = K / 2, IH = (DT_H - 1) * S + K;
+  constexpr int PAD = DIL * (K / 2), KE = DIL * (K - 1) + 1, IH = (DT_H - 1) * S + KE;
   extern __shared__ float tile[];  // [CPG][IH][IW][8]
   ptx::pdl_wait();
-  const int Ho = (H + 2 * PAD - K) / S + 1;
-  const int CPG = TPB / (8 * TW), IW = (TW - 1) * S + K;
+  const int Ho = (H + 2 * PAD - KE) / S + 1;
+  const int CPG = TPB / (8 * TW), IW = (TW - 1) * S + KE;
   const int tiles_h = (Ho + DT_H - 1) / DT_H, tiles_w = (Ho + TW - 1) / TW;
   int t = blockIdx.x;
   const int tw = t % tiles_w;
@@ -594,11 +596,11 @@ __global__ void __launch_bounds__(TPB) dw_tile_kernel(const bf16* __restrict__ i
   for (int ir = 0; ir < IH; ++ir) {
 #pragma unroll
     for (int v = 0; v < K; ++v) {
-      const float x = tb[((size_t)ir * IW + v) * 8];
+      const float x = tb[((size_t)ir * IW + v * DIL) * 8];
 #pragma unroll
       for (int r = 0; r < DT_H; ++r) {
-        const int u = ir - r * S;
-        if (u >= 0 && u < K) acc[r] = __fmaf_rn(x, wr[u][v], acc[r]);
+        const int t = ir - r * S;  // = u * DIL (compile-time after unrolling)
+        if (t >= 0 && t % DIL == 0 && t / DIL < K) acc[r] = __fmaf_rn(x, wr[t / DIL][v], acc[r]);
       }
     }
   }
@@ -660,15 +662,15 @@ __global__ void __launch_bounds__(TPB) dw_tile_kernel(const bf16* __restrict__ i
 // layout; fixpoint.cuh: bitwise independent of the CTA order).  The last CTA (ticket) applies
 // the SGD WRITE w -= lr * total (w = the master, or the bulk accumulator under BSP) and clears
 // acc: one launch instead of partials + a fixed-order summing SGD kernel.
-template <int K, int S>
+template <int K, int S, int DIL>
 __global__ void __launch_bounds__(TPB) dw_wgrad_kernel(const bf16* __restrict__ dz, const bf16* __restrict__ x,
                                                        unsigned long long* gacc, int* ticket, float* w, float lr,
                                                        int B, int H, int C, int TW, int NP) {
-  constexpr int PAD = K / 2, IH = (DT_H - 1) * S + K, K2 = K * K;
+  constexpr int PAD = DIL * (K / 2), KE = DIL * (K - 1) + 1, IH = (DT_H - 1) * S + KE, K2 = K * K;
   extern __shared__ float tile[];  // [CPG][IH][IW][8]; later [TPB][K2] for the column sums
   ptx::pdl_wait();
-  const int Ho = (H + 2 * PAD - K) / S + 1;
-  const int CPG = TPB / (8 * TW), IW = (TW - 1) * S + K;
+  const int Ho = (H + 2 * PAD - KE) / S + 1;
+  const int CPG = TPB / (8 * TW), IW = (TW - 1) * S + KE;
   const int tiles_h = (Ho + DT_H - 1) / DT_H, tiles_w = (Ho + TW - 1) / TW;
   const int tw = blockIdx.x % tiles_w, p = blockIdx.x / tiles_w;
   const int cg0 = blockIdx.y * CPG;
@@ -704,11 +706,11 @@ __global__ void __launch_bounds__(TPB) dw_wgrad_kernel(const bf16* __restrict__ 
     for (int ir = 0; ir < IH; ++ir) {
 #pragma unroll
       for (int v = 0; v < K; ++v) {
-        const float xv = tb[((size_t)ir * IW + v) * 8];
+        const float xv = tb[((size_t)ir * IW + v * DIL) * 8];
 #pragma unroll
         for (int r = 0; r < DT_H; ++r) {
-          const int u = ir - r * S;
-          if (u >= 0 && u < K) acc[u][v] = __fmaf_rn(g[r], xv, acc[u][v]);
+          const int t = ir - r * S;  // = u * DIL
+          if (t >= 0 && t % DIL == 0 && t / DIL < K) acc[t / DIL][v] = __fmaf_rn(g[r], xv, acc[t / DIL][v]);
         }
       }
     }
@@ -1094,46 +1096,52 @@ bool bn_fix_overflow(const unsigned long long* acc, int C) {
   return v != 0;
 }
 
-#define DW_DISPATCH(K, EXPR) \
-  switch (K) {               \
-    case 3: { constexpr int KK = 3; EXPR; break; } \
-    case 5: { constexpr int KK = 5; EXPR; break; } \
-    case 7: { constexpr int KK = 7; EXPR; break; } \
-    default: NP_REQUIRE(false, NASPIPE_EINVAL, "depthwise kernel %d", K); \
+// (kernel size, dilation) -> constexpr KK, DD
+#define DW_DISPATCH(K, D, EXPR)                                                        \
+  switch ((K) * 4 + (D)) {                                                             \
+    case 13: { constexpr int KK = 3, DD = 1; EXPR; break; }                            \
+    case 21: { constexpr int KK = 5, DD = 1; EXPR; break; }                            \
+    case 29: { constexpr int KK = 7, DD = 1; EXPR; break; }                            \
+    case 14: { constexpr int KK = 3, DD = 2; EXPR; break; }                            \
+    case 22: { constexpr int KK = 5, DD = 2; EXPR; break; }                            \
+    case 30: { constexpr int KK = 7, DD = 2; EXPR; break; }                            \
+    default: NP_REQUIRE(false, NASPIPE_EINVAL, "depthwise kernel %d dilation %d", K, D); \
   }
 
 // tile width: the smallest of 8 / 16 / 32 columns covering min(Ho, 32)
 static int dw_tw(int Ho) { return Ho <= 8 ? 8 : (Ho <= 16 ? 16 : 32); }
 
-template <int K, int S, bool X2, bool FLIP>
+template <int K, int S, int DIL, bool X2, bool FLIP>
 static void dw_tile(cudaStream_t s, const bf16* in, const float* w, const bf16* add, bf16* out, int B, int H, int C,
                     unsigned long long* stats = nullptr) {
+  constexpr int KE = DIL * (K - 1) + 1;
   const int Ho = (H - 1) / S + 1, TW = dw_tw(Ho), CPG = TPB / (8 * TW);
-  const int IH = (DT_H - 1) * S + K, IW = (TW - 1) * S + K;
+  const int IH = (DT_H - 1) * S + KE, IW = (TW - 1) * S + KE;
   const size_t sm = (size_t)CPG * IH * IW * 8 * sizeof(float);
   const int gx = B * ((Ho + DT_H - 1) / DT_H) * ((Ho + TW - 1) / TW), gy = (C / 8 + CPG - 1) / CPG;
-  set_smem(dw_tile_kernel<K, S, X2, FLIP>, sm);
-  launch_pdl(dw_tile_kernel<K, S, X2, FLIP>, dim3(gx, gy), dim3(TPB), sm, s, in, w, add, out, B, H, C, TW, stats);
+  set_smem(dw_tile_kernel<K, S, DIL, X2, FLIP>, sm);
+  launch_pdl(dw_tile_kernel<K, S, DIL, X2, FLIP>, dim3(gx, gy), dim3(TPB), sm, s, in, w, add, out, B, H, C, TW, stats);
 }
 
-void dw_fwd(cudaStream_t s, const bf16* x, const float* w, bf16* z, int B, int H, int C, int k, int S,
+void dw_fwd(cudaStream_t s, const bf16* x, const float* w, bf16* z, int B, int H, int C, int k, int S, int dil,
             unsigned long long* stats) {
   NP_REQUIRE(C % 8 == 0 && (S == 1 || S == 2), NASPIPE_EINVAL, "dw_fwd C=%d S=%d", C, S);
-  if (S == 1) { DW_DISPATCH(k, (dw_tile<KK, 1, true, false>(s, x, w, nullptr, z, B, H, C, stats))); }
-  else { DW_DISPATCH(k, (dw_tile<KK, 2, true, false>(s, x, w, nullptr, z, B, H, C, stats))); }
+  if (S == 1) { DW_DISPATCH(k, dil, (dw_tile<KK, 1, DD, true, false>(s, x, w, nullptr, z, B, H, C, stats))); }
+  else { DW_DISPATCH(k, dil, (dw_tile<KK, 2, DD, true, false>(s, x, w, nullptr, z, B, H, C, stats))); }
   check_launch("dw_fwd");
 }
 
 void dw_dgrad(cudaStream_t s, const bf16* dz, const float* w, const bf16* add, bf16* dx, int B, int H, int C, int k,
-              int S) {
+              int S, int dil) {
   if (S == 1) {  // the input gradient of a stride-1 conv is the correlation with the flipped kernel
-    DW_DISPATCH(k, (dw_tile<KK, 1, false, true>(s, dz, w, add, dx, B, H, C)));
+    DW_DISPATCH(k, dil, (dw_tile<KK, 1, DD, false, true>(s, dz, w, add, dx, B, H, C)));
   } else {
     const size_t items = (size_t)B * H * H * (C / 8);
     const size_t sm = (size_t)C * k * k * sizeof(float);
-    DW_DISPATCH(k, {
-      set_smem(dw_dgrad_kernel<KK>, sm);
-      launch_pdl(dw_dgrad_kernel<KK>, dim3(gs_grid(dw_dgrad_kernel<KK>, items, sm)), dim3(TPB), sm, s, dz, w, add, dx, B, H, C, S);
+    DW_DISPATCH(k, dil, {
+      set_smem(dw_dgrad_kernel<KK, DD>, sm);
+      launch_pdl(dw_dgrad_kernel<KK, DD>, dim3(gs_grid(dw_dgrad_kernel<KK, DD>, items, sm)), dim3(TPB), sm, s, dz, w,
+                 add, dx, B, H, C, S);
     });
   }
   check_launch("dw_dgrad");
@@ -1158,26 +1166,27 @@ int dw_wgrad_blocks(int B, int H, int C, int k, int S) {  // grid size (diagnost
 }
 
 void dw_wgrad_sgd(cudaStream_t s, const bf16* dz, const bf16* x, unsigned long long* acc, int* ticket, float* w,
-                  float lr, int B, int H, int C, int k, int S) {
+                  float lr, int B, int H, int C, int k, int S, int dil) {
   NP_REQUIRE(C % 8 == 0 && C / 8 <= TPB, NASPIPE_EINVAL, "dw_wgrad C=%d", C);
   NP_REQUIRE(S == 1 || S == 2, NASPIPE_EINVAL, "dw_wgrad stride %d", S);
   int TW, NP, gy, tiles_w;
   dw_wgrad_grid(B, H, C, k, S, TW, NP, gy, tiles_w);
   const int CPG = TPB / (8 * TW);
-  auto smem = [&](int K) {
-    const int IH = (DT_H - 1) * S + K, IW = (TW - 1) * S + K;
+  auto smem = [&](int K, int D) {
+    const int KE = D * (K - 1) + 1, IH = (DT_H - 1) * S + KE, IW = (TW - 1) * S + KE;
     return std::max((size_t)CPG * IH * IW * 8, (size_t)TPB * K * K) * sizeof(float);
   };
   const dim3 grid(tiles_w * NP, gy);
-#define DW_WG(KK, SS)                                                                                  \
-  {                                                                                                    \
-    set_smem(dw_wgrad_kernel<KK, SS>, smem(KK));                                                       \
-    launch_pdl(dw_wgrad_kernel<KK, SS>, grid, dim3(TPB), smem(KK), s, dz, x, acc, ticket, w, lr, B, H, C, TW, NP); \
+#define DW_WG(KK, SS, DD)                                                                                        \
+  {                                                                                                              \
+    set_smem(dw_wgrad_kernel<KK, SS, DD>, smem(KK, DD));                                                         \
+    launch_pdl(dw_wgrad_kernel<KK, SS, DD>, grid, dim3(TPB), smem(KK, DD), s, dz, x, acc, ticket, w, lr, B, H, C, TW, \
+               NP);                                                                                              \
   }
   if (S == 1) {
-    DW_DISPATCH(k, DW_WG(KK, 1));
+    DW_DISPATCH(k, dil, DW_WG(KK, 1, DD));
   } else {
-    DW_DISPATCH(k, DW_WG(KK, 2));
+    DW_DISPATCH(k, dil, DW_WG(KK, 2, DD));
   }
 #undef DW_WG
   check_launch("dw_wgrad");

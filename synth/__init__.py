@@ -62,6 +62,20 @@ CONFIGS = {
                  stage_repeats=[4, 4, 8, 4], stage_channels=[64, 160, 320, 640], stem_channels=16,
                  head_channels=1024, choice_kernel=[3, 5, 7, 3], choice_xception=[0, 0, 0, 1],
                  lr=0.001, compute_dtype="bf16", n_stages=8, n_subnets=256),
+    # CV.c3 analog (Table 1: 32 choice blocks x 12 layers per block) over Table 5's CV
+    # op types: Shuffle/Xception (separable) x k 3/5/7 x dilation 1/2 (A36);
+    # same stages and image size as configs[1].
+    "cv_c3": dict(family="spos", n_blocks=32, n_choices=12, batch=64, image_hw=224, num_classes=1000,
+                  stage_repeats=[8, 8, 8, 8], stage_channels=[64, 160, 320, 640], stem_channels=16,
+                  head_channels=1024, choice_kernel=[3, 5, 7] * 4, choice_xception=[0] * 6 + [1] * 6,
+                  choice_dilation=[1, 1, 1, 2, 2, 2] * 2,
+                  lr=0.001, compute_dtype="bf16", n_stages=8, n_subnets=256),
+    # small SPOS supernet with dilated candidates (parity tests of A36)
+    "tiny_spos_dil": dict(family="spos", n_blocks=5, n_choices=4, batch=4, image_hw=64, num_classes=10,
+                          stage_repeats=[1, 2, 1, 1], stage_channels=[32, 64, 96, 128], stem_channels=16,
+                          head_channels=64, choice_kernel=[3, 7, 5, 3], choice_xception=[0, 0, 1, 1],
+                          choice_dilation=[2, 2, 2, 1], lr=0.001, compute_dtype="bf16", n_stages=2,
+                          n_subnets=8),
     # small SPOS supernet for parity tests: every channel count a multiple of 16
     "tiny_spos": dict(family="spos", n_blocks=5, n_choices=4, batch=4, image_hw=64, num_classes=10,
                       stage_repeats=[1, 2, 1, 1], stage_channels=[32, 64, 96, 128], stem_channels=16,

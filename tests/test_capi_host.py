@@ -23,7 +23,7 @@ def test_exports_every_declared_symbol():
     for name in sorted(declared):
         assert hasattr(npipe.lib, name), name
     assert declared == set(npipe.EXPORTED_SYMBOLS)
-    assert npipe.naspipe_abi_version() == 3
+    assert npipe.naspipe_abi_version() == 4
 
 
 @pytest.mark.parametrize("name", ["toy", "tiny_transformer", "transformer"])
@@ -41,10 +41,11 @@ def test_init_params_match_shared_hash(name):
         assert np.array_equal(got.view(np.uint32), ref.view(np.uint32)), (b, c)
 
 
-@pytest.mark.parametrize("name", ["tiny_spos", "spos"])
+@pytest.mark.parametrize("name", ["tiny_spos", "spos", "tiny_spos_dil", "cv_c3"])
 def test_spos_layout_and_init_match_oracle(name):
     """SPOS candidates: packed sizes and counter-hash values equal the oracle's layout
-    (oracle/spos.py layout) for every candidate kind (stride 1/2, Shuffle k=3/5/7, Xception)."""
+    (oracle/spos.py layout) for every candidate kind (stride 1/2, Shuffle k=3/5/7, Xception
+    k=3/5/7, dilation 1/2)."""
     cfg = synth.get_config(name)
     spec = npipe.Spec(cfg)
     n, m = cfg["n_choices"], cfg["n_blocks"]
@@ -52,7 +53,7 @@ def test_spos_layout_and_init_match_oracle(name):
         for c in range(n):
             segs = [(int(np.prod(s)), kind, fan) for _, s, kind, fan in train.candidate_layout(cfg, b, c)]
             assert npipe.naspipe_param_count(spec, b, c) == sum(s for s, _, _ in segs), (b, c)
-            if name == "spos" and b not in (0, 1, m - 1):
+            if name in ("spos", "cv_c3") and b not in (0, 1, m - 1):
                 continue
             got = npipe.naspipe_init_params(spec, b, c)
             ref = synth.init_packed(cfg["init_seed"], b * n + c, segs)
@@ -68,7 +69,8 @@ def test_spos_spec_validation():
     cfg = synth.get_config("tiny_spos")
     for bad in (dict(stage_repeats=[1, 2, 1, 2]), dict(stage_channels=[32, 64, 80, 128]),
                 dict(choice_kernel=[3, 5, 4, 3]), dict(image_hw=48), dict(head_channels=60),
-                dict(choice_xception=[0, 0, 1, 1])):
+                dict(choice_xception=[0, 0, 2, 1]), dict(choice_dilation=[1, 3, 1, 1]),
+                dict(choice_dilation=[1, 0, 1, 1])):
         with pytest.raises(npipe.NaspipeError):
             npipe.naspipe_default_costs(npipe.Spec(dict(cfg, **bad)))
     cf, cb = npipe.naspipe_default_costs(npipe.Spec(synth.get_config("spos")))

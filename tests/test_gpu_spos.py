@@ -76,6 +76,58 @@ def test_tiny_spos_bitwise_across_runs_and_stage_counts():
         _check_trace(cfg, choices, D, tr)
 
 
+@pytest.mark.parametrize("N", [1, 8])
+def test_tiny_spos_dilated_parity(N):
+    """Dilated depthwise candidates (Table 5's Dil Conv; reading A36): Shuffle k 3/7
+    and Xception k 5 at dilation 2, Xception k 3 at dilation 1; every (block, choice) trained
+    when N = 8 (two rounds of the cyclic assignment)."""
+    cfg = synth.get_config("tiny_spos_dil")
+    m, n = cfg["n_blocks"], cfg["n_choices"]
+    choices = np.array([[(c + b) % n for b in range(m)] for c in range(N)], dtype=np.int32)
+    cfg, gpu, floor, losses, ref_loss, trace, stats = _run("tiny_spos_dil", choices)
+    pm.check(gpu, 1e-3, pm.UPD_SPOS)
+    np.testing.assert_allclose(losses, ref_loss, rtol=1e-2)
+    _check_trace(cfg, choices, 2, trace)
+
+
+def test_cv_c3_full_size_one_step_against_oracle_samples():
+    """The CV.c3 analog (Table 1: 32 choice blocks x 12 choices over Table 5's op types,
+    dilation included; reading A36) at full size, one subnet, against the fp64 oracle
+    (tests/golden/cv_c3_fullsize_1steps.npz, tools/make_multistep_golden.py, oracle/ only).
+
+    This supernet is ill-conditioned at initialisation (deep BatchNorm chains over nearly
+    constant channels at 7 x 7): the SAME oracle with its stored tensors rounded to fp32 (the
+    paper's precision) or the way this path stores them (bf16x2, A28) already moves the
+    parameters far from fp64 after one step (DESIGN.md A37).  Bars: losses rtol 1e-2;
+    per-tensor A15 <= max(1e-3, 1.5 x the bf16x2-storage oracle's A15 at the same samples).
+    The dilated kernels themselves are pinned at these shapes in test_gpu_spos_kernels.py and
+    end to end at 1e-3 on tiny_spos_dil above."""
+    gold = load_gold("cv_c3_fullsize_1steps.npz")
+    cfg = synth.get_config("cv_c3")
+    fl16 = pm.golden_floor(cfg, gold, load_gold("cv_c3_fullsize_1steps_bf16x2.npz"), 1)
+    fl32 = pm.golden_floor(cfg, gold, load_gold("cv_c3_fullsize_1steps_fp32.npz"), 1)
+    cfg, h, got_of, losses = run_fullsize("cv_c3", gold, 1)
+    sm = pm.sampled_errors(cfg, gold, 1, got_of)
+    npipe.naspipe_destroy(h)
+    print(f"cv_c3 full size, 1 step: {pm.fmt(sm)}; oracle floors bf16x2 {fl16} fp32 {fl32}; "
+          f"loss {losses} vs {gold['losses'][:1]}")
+    np.testing.assert_allclose(losses, gold["losses"][:1], rtol=1e-2)
+    assert sm["a15"] <= max(1e-3, 1.5 * fl16["a15"]), (sm["a15"], fl16)
+
+
+def test_cv_c3_full_size_bitwise_across_stage_counts():
+    """CV.c3 analog at full size: 3 subnets at D = 1 and D = 4, parameters and losses bitwise
+    equal (Def.1, Table 3)."""
+    cfg = synth.get_config("cv_c3")
+    choices = synth.sample_choices(3, cfg["n_blocks"], cfg["n_choices"])
+    batches = [synth.make_batch(cfg, y) for y in range(3)]
+    base, base_loss, _, _ = run_engine(cfg, choices, batches, D=1)
+    p, l, _, _ = run_engine(cfg, choices, batches, D=4, where=npipe.BATCH_DEVICE)
+    assert np.array_equal(l.view(np.uint32), base_loss.view(np.uint32))
+    for k in base:
+        assert np.array_equal(p[k].view(np.uint32), base[k].view(np.uint32)), k
+
+
 def test_spos_full_size_one_step():
     """configs[1] at full size (B = 64, 224 x 224, 20 blocks) in the bench's launch
     configuration (one stage), one subnet, against the plain fp64 oracle (A15 <= 1e-3,

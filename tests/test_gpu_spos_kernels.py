@@ -20,7 +20,7 @@ pytestmark = pytest.mark.gpu
 npipe = pytest.importorskip("paper_conf_asplos_zhaolcscwzlc22_b200")
 L = npipe.lib
 _vp, _i = C.c_void_p, C.c_int
-L.naspipe_debug_dw.argtypes = [_vp] * 7 + [_i] * 5 + [_vp]
+L.naspipe_debug_dw.argtypes = [_vp] * 7 + [_i] * 6 + [_vp]
 L.naspipe_debug_bn_fwd.argtypes = [_vp, _i, _i, _vp, _vp, _i, _vp, _i, C.c_size_t, _vp, _vp, _vp]
 L.naspipe_debug_bn_bwd.argtypes = [_vp, _i, _vp, _i, _i, _vp, _vp, _vp, _vp, _i, _vp, _vp, _vp, C.c_float, _i, _vp]
 L.naspipe_debug_chan_split.argtypes = [_vp, _i, _i, _vp, _i, C.c_size_t, _vp, _vp]
@@ -73,39 +73,46 @@ def _check_bf16(got, ref):
     assert np.mean(np.abs(got - r16) <= ulp + 1e-30) >= 0.99
 
 
-def _dw_ref(x, w, s):
+def _dw_ref(x, w, s, d=1):
     B, H, _, Cc = x.shape
     k = w.shape[1]
-    p = k // 2
-    Ho = (H + 2 * p - k) // s + 1
+    p = d * (k // 2)
+    Ho = (H + 2 * p - d * (k - 1) - 1) // s + 1
     xp = np.pad(x, ((0, 0), (p, p), (p, p), (0, 0)))
     y = np.zeros((B, Ho, Ho, Cc))
     for u in range(k):
         for v in range(k):
-            y += xp[:, u:u + s * (Ho - 1) + 1:s, v:v + s * (Ho - 1) + 1:s, :] * w[:, u, v]
+            y += xp[:, u * d:u * d + s * (Ho - 1) + 1:s, v * d:v * d + s * (Ho - 1) + 1:s, :] * w[:, u, v]
     return y
 
 
-def _dw_bwd_ref(x, w, s, dz):
+def _dw_bwd_ref(x, w, s, dz, d=1):
     k = w.shape[1]
-    p = k // 2
+    p = d * (k // 2)
     B, Ho, _, Cc = dz.shape
     xp = np.pad(x, ((0, 0), (p, p), (p, p), (0, 0)))
     dxp = np.zeros_like(xp)
     dw = np.zeros_like(w)
     for u in range(k):
         for v in range(k):
-            sl = (slice(None), slice(u, u + s * (Ho - 1) + 1, s), slice(v, v + s * (Ho - 1) + 1, s), slice(None))
+            sl = (slice(None), slice(u * d, u * d + s * (Ho - 1) + 1, s), slice(v * d, v * d + s * (Ho - 1) + 1, s),
+                  slice(None))
             dxp[sl] += dz * w[:, u, v]
             dw[:, u, v] = np.sum(dz * xp[sl], axis=(0, 1, 2))
     H = x.shape[1]
     return dxp[:, p:p + H, p:p + H, :], dw
 
 
-@pytest.mark.parametrize("B,H,Cc,k,s", [(2, 9, 16, 3, 1), (3, 8, 48, 5, 2), (2, 14, 32, 7, 1), (1, 7, 640, 3, 1),
-                                        (4, 6, 320, 7, 2), (64, 112, 16, 3, 2)])
-def test_depthwise_fwd_dgrad_wgrad(B, H, Cc, k, s):
-    rng = np.random.default_rng(B * 100 + H + Cc + k)
+@pytest.mark.parametrize("B,H,Cc,k,s,d", [(2, 9, 16, 3, 1, 1), (3, 8, 48, 5, 2, 1), (2, 14, 32, 7, 1, 1),
+                                          (1, 7, 640, 3, 1, 1), (4, 6, 320, 7, 2, 1), (64, 112, 16, 3, 2, 1),
+                                          (2, 9, 16, 3, 1, 2), (3, 8, 48, 5, 2, 2), (2, 14, 32, 7, 1, 2),
+                                          (4, 6, 320, 7, 2, 2), (2, 37, 24, 5, 1, 2), (2, 40, 64, 3, 2, 2),
+                                          # the CV.c3 analog's full-size dilated shapes (synth cv_c3)
+                                          (64, 112, 16, 5, 2, 2), (64, 112, 16, 7, 2, 2), (64, 56, 32, 7, 1, 2),
+                                          (64, 28, 80, 5, 1, 2), (64, 14, 160, 3, 1, 2), (64, 7, 320, 7, 1, 2)])
+def test_depthwise_fwd_dgrad_wgrad(B, H, Cc, k, s, d):
+    """Depthwise conv kernels (dilation d: Table 5's Dil Conv, reading A36) vs explicit tap loops."""
+    rng = np.random.default_rng(B * 100 + H + Cc + k + 7 * d)
     xd, x = _x2(rng.standard_normal((B, H, H, Cc)))
     x_hi = _f64(xd[0])
     w = (rng.standard_normal((Cc, k, k)) / k).astype(np.float32)
@@ -118,21 +125,21 @@ def test_depthwise_fwd_dgrad_wgrad(B, H, Cc, k, s):
     dws = torch.empty((Cc, k, k), dtype=torch.float32, device="cuda")
     outs = []
     for _ in range(2):
-        _ok(L.naspipe_debug_dw(_p(xd), _p(wd), _p(z), _p(dzd), _p(addd), _p(dx), _p(dws), B, H, Cc, k, s, None))
+        _ok(L.naspipe_debug_dw(_p(xd), _p(wd), _p(z), _p(dzd), _p(addd), _p(dx), _p(dws), B, H, Cc, k, s, d, None))
         torch.cuda.synchronize()
         outs.append((z.clone(), dx.clone(), dws.clone()))
     for a, b in zip(outs[0], outs[1]):
         assert torch.equal(a, b)
     if B * H * H > 100000:   # full-size block 0: check the reductions on a sample of channels
-        ch = [0, 7, 15]
+        ch = [0, 7, 15, Cc - 1]
         x, x_hi, dz, add, w64 = x[..., ch], x_hi[..., ch], dz[..., ch], add[..., ch], w[ch].astype(np.float64)
         got_z, got_dx, got_dw = _v2(z)[..., ch], _f64(dx)[..., ch], _f64(dws)[ch]
     else:
         w64 = w.astype(np.float64)
         got_z, got_dx, got_dw = _v2(z), _f64(dx), _f64(dws)
-    _check_x2(got_z, _dw_ref(x, w64, s))
-    rdx, _ = _dw_bwd_ref(x, w64, s, dz)
-    _, rdw = _dw_bwd_ref(x_hi, w64, s, dz)     # the weight gradient reads the hi plane
+    _check_x2(got_z, _dw_ref(x, w64, s, d))
+    rdx, _ = _dw_bwd_ref(x, w64, s, dz, d)
+    _, rdw = _dw_bwd_ref(x_hi, w64, s, dz, d)     # the weight gradient reads the hi plane
     _check_bf16(got_dx, rdx + add)
     assert np.max(np.abs(got_dw - rdw)) / np.max(np.abs(rdw)) <= 1e-5
 

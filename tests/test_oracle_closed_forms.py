@@ -278,11 +278,12 @@ def test_spos_stride1_xception_relu_placement():
         np.testing.assert_allclose(y[0, :, :, 16 + j].ravel(), q * (PAT[j % 4] > 0), rtol=0, atol=1e-12)
 
 
-def _torch_unit(x, w, kind, s, g, bb, relu):
+def _torch_unit(x, w, kind, s, g, bb, relu, dil=1):
     X = torch.tensor(x).permute(0, 3, 1, 2)
     W = torch.tensor(w)
     if kind == "dw":
-        z = torch.nn.functional.conv2d(X, W[:, None], stride=s, padding=w.shape[1] // 2, groups=w.shape[0])
+        z = torch.nn.functional.conv2d(X, W[:, None], stride=s, padding=dil * (w.shape[1] // 2), dilation=dil,
+                                       groups=w.shape[0])
     else:
         z = torch.nn.functional.conv2d(X, W[:, :, None, None])
     y = torch.nn.functional.batch_norm(z, None, None, torch.tensor(g), torch.tensor(bb), training=True, eps=1e-5)
@@ -291,19 +292,40 @@ def _torch_unit(x, w, kind, s, g, bb, relu):
     return y.permute(0, 2, 3, 1).numpy()
 
 
-@pytest.mark.parametrize("kind,k,s,relu", [("dw", 3, 1, False), ("dw", 5, 2, False), ("dw", 7, 1, False),
-                                           ("pw", 1, 1, True), ("pw", 1, 1, False)])
-def test_spos_unit_matches_torch(kind, k, s, relu):
-    """conv -> training-mode BN (biased variance, eps 1e-5) [-> ReLU] against torch.nn.functional."""
-    rng = np.random.default_rng(k * 7 + s)
+@pytest.mark.parametrize("kind,k,s,relu,dil", [("dw", 3, 1, False, 1), ("dw", 5, 2, False, 1), ("dw", 7, 1, False, 1),
+                                               ("pw", 1, 1, True, 1), ("pw", 1, 1, False, 1), ("dw", 3, 1, False, 2),
+                                               ("dw", 5, 2, False, 2), ("dw", 7, 1, False, 2)])
+def test_spos_unit_matches_torch(kind, k, s, relu, dil):
+    """conv (dilation dil: Table 5's Dil Conv, reading A36) -> training-mode BN (biased
+    variance, eps 1e-5) [-> ReLU] against torch.nn.functional."""
+    rng = np.random.default_rng(k * 7 + s + 31 * dil)
     C = 6
     x = rng.standard_normal((3, 9, 9, C))
     w = rng.standard_normal((C, k, k)) if kind == "dw" else rng.standard_normal((C + 2, C))
     co = w.shape[0]
     g, bb = 1 + 0.3 * rng.standard_normal(co), 0.3 * rng.standard_normal(co)
     p = {"u": w, "u_g": g, "u_b": bb}
-    y, _ = spos._unit_fwd(p, "u", kind, s, relu, x)
-    np.testing.assert_allclose(y, _torch_unit(x, w, kind, s, g, bb, relu), rtol=1e-11, atol=1e-11)
+    y, _ = spos._unit_fwd(p, "u", kind, s, relu, x, dil=dil)
+    np.testing.assert_allclose(y, _torch_unit(x, w, kind, s, g, bb, relu, dil), rtol=1e-11, atol=1e-11)
+
+
+@pytest.mark.parametrize("k,s,dil", [(3, 1, 2), (5, 2, 2), (7, 1, 2), (3, 2, 1)])
+def test_spos_depthwise_backward_matches_torch_autograd(k, s, dil):
+    """dw_bwd's input and weight gradients (dilated and not) against torch autograd of conv2d."""
+    rng = np.random.default_rng(100 * k + 10 * s + dil)
+    C = 5
+    x = rng.standard_normal((2, 11, 11, C))
+    w = rng.standard_normal((C, k, k))
+    y = spos.dw_fwd(x, w, s, dil)
+    dy = rng.standard_normal(y.shape)
+    dx, dw = spos.dw_bwd(x, w, s, dy, dil)
+    X = torch.tensor(x).permute(0, 3, 1, 2).requires_grad_()
+    W = torch.tensor(w)[:, None].requires_grad_()
+    Y = torch.nn.functional.conv2d(X, W, stride=s, padding=dil * (k // 2), dilation=dil, groups=C)
+    np.testing.assert_allclose(Y.detach().permute(0, 2, 3, 1).numpy(), y, rtol=1e-11, atol=1e-11)
+    Y.backward(torch.tensor(dy).permute(0, 3, 1, 2))
+    np.testing.assert_allclose(X.grad.permute(0, 2, 3, 1).numpy(), dx, rtol=1e-11, atol=1e-11)
+    np.testing.assert_allclose(W.grad[:, 0].numpy(), dw, rtol=1e-11, atol=1e-11)
 
 
 def test_head_ce_zero_classifier_is_ln_classes():

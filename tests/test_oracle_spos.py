@@ -14,11 +14,11 @@ import synth
 from oracle import spos, train
 
 
-def _dw_loops(x, w, s):
+def _dw_loops(x, w, s, d=1):
     B, H, W, C = x.shape
     k = w.shape[1]
-    p = k // 2
-    Ho, Wo = (H + 2 * p - k) // s + 1, (W + 2 * p - k) // s + 1
+    p = d * (k // 2)
+    Ho, Wo = (H + 2 * p - d * (k - 1) - 1) // s + 1, (W + 2 * p - d * (k - 1) - 1) // s + 1
     y = np.zeros((B, Ho, Wo, C))
     for b in range(B):
         for i in range(Ho):
@@ -27,19 +27,36 @@ def _dw_loops(x, w, s):
                     acc = 0.0
                     for u in range(k):
                         for v in range(k):
-                            ii, jj = i * s + u - p, j * s + v - p
+                            ii, jj = i * s + u * d - p, j * s + v * d - p
                             if 0 <= ii < H and 0 <= jj < W:
                                 acc += x[b, ii, jj, c] * w[c, u, v]
                     y[b, i, j, c] = acc
     return y
 
 
-@pytest.mark.parametrize("k,s", [(3, 1), (5, 2), (7, 1), (3, 2)])
-def test_depthwise_matches_loops(k, s):
-    rng = np.random.default_rng(k * 10 + s)
-    x = rng.standard_normal((2, 6, 6, 3))
+@pytest.mark.parametrize("k,s,d", [(3, 1, 1), (5, 2, 1), (7, 1, 1), (3, 2, 1), (3, 1, 2), (5, 2, 2), (7, 1, 2)])
+def test_depthwise_matches_loops(k, s, d):
+    rng = np.random.default_rng(k * 10 + s + 100 * d)
+    x = rng.standard_normal((2, 7, 7, 3))
     w = rng.standard_normal((3, k, k))
-    np.testing.assert_allclose(spos.dw_fwd(x, w, s), _dw_loops(x, w, s), rtol=1e-12, atol=1e-12)
+    y = spos.dw_fwd(x, w, s, d)
+    assert y.shape == (2, (7 - 1) // s + 1, (7 - 1) // s + 1, 3)   # "same" padding for every dilation
+    np.testing.assert_allclose(y, _dw_loops(x, w, s, d), rtol=1e-12, atol=1e-12)
+
+
+def test_dilated_depthwise_special_cases():
+    """Dilation 2 of a k x k kernel = the (2k-1) x (2k-1) kernel with zeros between the taps;
+    a kernel whose only nonzero tap is the centre is the identity for every dilation."""
+    rng = np.random.default_rng(3)
+    x = rng.standard_normal((2, 9, 9, 4))
+    w = rng.standard_normal((4, 3, 3))
+    wz = np.zeros((4, 5, 5))
+    wz[:, ::2, ::2] = w
+    for s in (1, 2):
+        np.testing.assert_allclose(spos.dw_fwd(x, w, s, 2), spos.dw_fwd(x, wz, s, 1), rtol=1e-13, atol=1e-13)
+    delta = np.zeros((4, 5, 5))
+    delta[:, 2, 2] = 1.0
+    np.testing.assert_allclose(spos.dw_fwd(x, delta, 1, 2), x, rtol=1e-14)
 
 
 def test_depthwise_special_cases():
@@ -82,6 +99,8 @@ def test_batchnorm_closed_form():
 MINI = dict(family="spos", n_blocks=2, n_choices=4, batch=2, image_hw=16, num_classes=5,
             stage_repeats=[2], stage_channels=[8], stem_channels=4, head_channels=6,
             choice_kernel=[3, 5, 7, 3], choice_xception=[0, 0, 0, 1], lr=0.01, init_seed=2)
+# the dilated choices of Table 5 (reading A36): Shuffle 3/5 and Xception 3/5 at dilation 2
+MINI_DIL = dict(MINI, choice_kernel=[3, 5, 3, 5], choice_xception=[0, 0, 1, 1], choice_dilation=[2, 2, 2, 2])
 
 
 def _check_fd(f, analytic, arr, rng, n=6, eps=1e-6):
@@ -98,9 +117,11 @@ def _check_fd(f, analytic, arr, rng, n=6, eps=1e-6):
         assert abs(num - analytic[i]) <= 1e-5 * max(abs(num), abs(analytic[i])) + 1e-7, (i, num, analytic[i])
 
 
+@pytest.mark.parametrize("cfg", [MINI, MINI_DIL], ids=["plain", "dilated"])
 @pytest.mark.parametrize("b", [0, 1])          # block 0: stride 2 (proj branch), block 1: stride 1
-@pytest.mark.parametrize("c", [0, 1, 2, 3])    # Shuffle 3/5/7, Xception
-def test_block_fd(b, c):
+@pytest.mark.parametrize("c", [0, 1, 2, 3])    # Shuffle 3/5/7, Xception (MINI_DIL: dilated Shuffle/Xception 3/5)
+def test_block_fd(b, c, cfg):
+    MINI = cfg
     rng = np.random.default_rng(10 * b + c)
     s, inp, mid, out, cout, H = spos.block_dims(MINI, b)
     p = {}
