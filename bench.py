@@ -355,13 +355,16 @@ def plan_bound_ms(cfg, npipe, choices, D, busy_us):
     return npipe.naspipe_plan(s, D, choices).makespan() / 1000.0
 
 
-def algorithmic_work(cfg, st, steps):
+def algorithmic_work(cfg, st, steps, choices=None):
     """(work per step, unit, peak key) of the whole step for fraction 2: transformer = GEMM
-    flops (library counter) + attention flops (12 B S^2 d per block, fwd + bwd); SPOS = none
-    beyond the counted BatchNorm bytes (its other kernels' bytes are not counted: the
-    fraction is then a lower bound)."""
+    flops (library counter) + attention flops (12 B S^2 d per attention block, fwd + bwd; the
+    NLP conv ops of A38 count their GEMMs only); SPOS = none beyond the counted BatchNorm
+    bytes (its other kernels' bytes are not counted: the fraction is then a lower bound)."""
     if cfg["family"] == "transformer":
-        att = 12.0 * cfg["batch"] * cfg["seq_len"] ** 2 * cfg["d_model"] * cfg["n_blocks"]
+        ops = np.asarray(cfg.get("choice_op", [0] * cfg["n_choices"]))
+        n_att = (float(np.mean(np.sum(ops[np.asarray(choices)] == 0, axis=1))) if choices is not None
+                 else float(np.sum(ops == 0)) / len(ops) * cfg["n_blocks"])
+        att = 12.0 * cfg["batch"] * cfg["seq_len"] ** 2 * cfg["d_model"] * n_att
         return st["gemm_flops"] / steps + att, "flop", "bf16_sustained"
     return None, None, None
 
@@ -369,7 +372,8 @@ def algorithmic_work(cfg, st, steps):
 def workload_config(args, cfg, world):
     names = {"transformer": "configs[2] transformer", "large_transformer": "configs[3] large_transformer",
              "toy": "configs[0] toy", "spos": "configs[1] SPOS CNN",
-             "cv_c3": "CV.c3 analog (Table 1: 32 blocks x 12 choices, Table 5 ops incl. dilated)"}
+             "cv_c3": "CV.c3 analog (Table 1: 32 blocks x 12 choices, Table 5 ops incl. dilated)",
+             "nlp_c3": "NLP.c3 analog (Table 1: 48 blocks x 24 choices, Table 5 NLP ops)"}
     c = {"workload": names.get(args.workload, args.workload) if not args.n_choices
          else f"configs[4] sweep n={args.n_choices}",
          "n_blocks": cfg["n_blocks"], "n_choices": cfg["n_choices"], "batch": cfg["batch"],
@@ -379,6 +383,8 @@ def workload_config(args, cfg, world):
          "l2": "working set > L2 (active weights + activations per step >> 126 MB)"}
     if cfg["family"] == "transformer":
         c.update(seq_len=cfg["seq_len"], d_model=cfg["d_model"], heads=cfg["choice_heads"], ffn=cfg["choice_ffn"])
+        if "choice_op" in cfg:
+            c["op"] = cfg["choice_op"]
     if cfg["family"] == "spos":
         c.update(image_hw=cfg["image_hw"], stage_repeats=cfg["stage_repeats"], stage_channels=cfg["stage_channels"],
                  choice_kernel=cfg["choice_kernel"], choice_xception=cfg["choice_xception"],
@@ -434,7 +440,8 @@ def main():
         sec = {"configs[2] transformer": secondary(args, "transformer"),
                "configs[3] large_transformer (budget 3x, context switching)":
                    secondary(args, "large_transformer", ["--budget-x", "3", "--no-repro"], steps=min(args.steps, 12)),
-               "CV.c3 analog (32 x 12, dilated candidates)": secondary(args, "cv_c3", ["--no-repro"])}
+               "CV.c3 analog (32 x 12, dilated candidates)": secondary(args, "cv_c3", ["--no-repro"]),
+               "NLP.c3 analog (48 x 24, Table 5 NLP ops)": secondary(args, "nlp_c3", ["--no-repro"])}
 
     import torch
     import torch.distributed as dist
@@ -577,7 +584,7 @@ def main():
             "note": "algorithmic GEMM flops / GEMM device time (CUPTI) / sustained bf16 peak; SPOS counts one "
                     "bf16 product per 3-pass bf16x2 GEMM"}
         busy = gather(busy_us)
-        w_step, w_unit, w_peak = algorithmic_work(cfg, {"gemm_flops": gflops}, args.steps)
+        w_step, w_unit, w_peak = algorithmic_work(cfg, {"gemm_flops": gflops}, args.steps, timed_choices)
         e2e_hw = None
         if w_step is not None:
             e2e_hw = (w_step * 1e-12) / (D * pk[w_peak] * (ms / args.steps / 1000))

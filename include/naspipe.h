@@ -184,6 +184,10 @@ typedef struct {
   int32_t bulk_size;
   /* ABI 4: per-choice depthwise dilation (SPOS_CNN; NULL = 1) */
   const int32_t* choice_dilation;
+  /* ABI 4: per-choice token mixer (TRANSFORMER; NULL = all attention): 0 multi-head attention,
+   * 1 Conv 3x1, 2 Sep Conv 7x1, 3 Light Conv 5x1 (heads = its weight-sharing heads H) --
+   * Table 5's NLP ops; internals: DESIGN.md A38, oracle/transformer.py */
+  const int32_t* choice_op;
 } naspipe_supernet_spec;
 
 /* naspipe_batch.where */

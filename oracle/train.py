@@ -62,7 +62,7 @@ def mse_loss(y, t):
 def _block_fwd(cfg, p, x, c):
     if cfg["family"] == "mlp":
         return mlp.forward(p, x)
-    return transformer.forward(p, x, cfg["choice_heads"][c])
+    return transformer.forward(p, x, cfg["choice_heads"][c], transformer.op_of(cfg, c))
 
 
 def _block_bwd(cfg, p, tape, dy):

@@ -37,7 +37,7 @@ class _SpecStruct(C.Structure):
                 ("image_hw", C.c_int32), ("num_classes", C.c_int32), ("stem_channels", C.c_int32),
                 ("head_channels", C.c_int32), ("n_cnn_stages", C.c_int32), ("stage_repeats", _i32p),
                 ("stage_channels", _i32p), ("choice_kernel", _i32p), ("choice_xception", _i32p),
-                ("sync_policy", C.c_int32), ("bulk_size", C.c_int32), ("choice_dilation", _i32p)]
+                ("sync_policy", C.c_int32), ("bulk_size", C.c_int32), ("choice_dilation", _i32p), ("choice_op", _i32p)]
 
 
 class _BatchStruct(C.Structure):
@@ -130,7 +130,7 @@ class Spec:
         s.d_model, s.seq_len = cfg.get("d_model", 0), cfg.get("seq_len", 0)
         self._keep = []
         for name in ("choice_heads", "choice_ffn", "stage_of_block", "cost_fwd", "cost_bwd", "stage_repeats",
-                     "stage_channels", "choice_kernel", "choice_xception", "choice_dilation"):
+                     "stage_channels", "choice_kernel", "choice_xception", "choice_dilation", "choice_op"):
             if cfg.get(name) is not None:
                 arr, ptr = _i32(np.asarray(cfg[name]).ravel())
                 self._keep.append(arr)

@@ -201,13 +201,25 @@ class TfFamily : public Family {
     gb_[1] = A.alloc<float>(Td);
     // split-K workspace (side stream only): the largest splits * M * N of the wgrad GEMMs
     ws_elems_ = 0;
+    bool any_conv3 = false, any_taps = false;
     for (int c = 0; c < n; ++c) {
       const int f = spec.ffn[c], T = T_, d = d_;
-      const int shp[4][3] = {{d, f, T}, {f, d, T}, {d, d, T}, {3 * d, d, T}};
+      const int shp[5][3] = {{d, f, T}, {f, d, T}, {d, d, T}, {3 * d, d, T}, {d, 3 * d, T}};
       for (auto& q : shp)
         ws_elems_ = std::max(ws_elems_, (size_t)gemm_splitk_factor(q[0], q[1], q[2]) * q[0] * q[1]);
+      any_conv3 |= spec.op[c] == TF_CONV3;
+      any_taps |= spec.op[c] == TF_SEPCONV7 || spec.op[c] == TF_LIGHTCONV5;
     }
     ws_ = A.alloc<float>(ws_elems_);
+    // NLP op families (reading A38): Conv 3x1's column gradient, the sequence-conv weight
+    // gradient partials (side stream only) and its arrival ticket
+    if (any_conv3) dcols_ = A.alloc<float>(3 * Td);
+    if (any_taps) {  // fixed-point totals [d * 7] + the overflow flag (reading A33)
+      sc_acc_ = A.alloc<unsigned long long>((size_t)d_ * 7 + 1);
+      cudaMemset(sc_acc_, 0, ((size_t)d_ * 7 + 1) * 8);
+      sc_tick_ = A.alloc<int>(1);
+      cudaMemset(sc_tick_, 0, sizeof(int));
+    }
     csb_ = colsum_blocks(T_);
     lnb_ = ln_bwd_blocks(T_);
     for (int p = 0; p < 2; ++p) {
@@ -234,11 +246,19 @@ class TfFamily : public Family {
     cudaStreamDestroy(side_);
   }
 
+  void check_after_drain() override {
+    if (!sc_acc_) return;
+    unsigned long long flag = 0;
+    cudaMemcpy(&flag, sc_acc_ + (size_t)d_ * 7, 8, cudaMemcpyDeviceToHost);
+    NP_REQUIRE(flag == 0, NASPIPE_EINTERNAL,
+               "sequence-conv weight-gradient fixed-point overflow (a partial outside the 64-bit range, seqconv.cu)");
+  }
+
   void bind(int j, int c, float* w32, bf16* w16) override {
     w32_[(size_t)j * spec_.n() + c] = w32;
     w16_[(size_t)j * spec_.n() + c] = w16;
   }
-  size_t shadow_elems(int, int c) const override { return 4 * (size_t)d_ * d_ + 2 * (size_t)d_ * spec_.ffn[c]; }
+  size_t shadow_elems(int, int c) const override { return spec_.tf_offsets(c).sh_total; }
   float* master(int j, int c) override { return w32_[(size_t)j * spec_.n() + c]; }
 
   void refresh_shadow(int j, int c, cudaStream_t s) override {
@@ -246,10 +266,10 @@ class TfFamily : public Family {
     const size_t d = d_, f = spec_.ffn[c];
     float* p = master(j, c);
     bf16* w = w16_[(size_t)j * spec_.n() + c];
-    f32_to_bf16(s, p + o.Wqkv, w, 3 * d * d);
-    f32_to_bf16(s, p + o.Wo, w + 3 * d * d, d * d);
-    f32_to_bf16(s, p + o.W1, w + 4 * d * d, f * d);
-    f32_to_bf16(s, p + o.W2, w + 4 * d * d + f * d, d * f);
+    if (o.n_Win) f32_to_bf16(s, p + o.Win, w + o.sh_Win, o.n_Win);
+    f32_to_bf16(s, p + o.Wo, w + o.sh_Wo, o.n_Wo);
+    f32_to_bf16(s, p + o.W1, w + o.sh_W1, f * d);
+    f32_to_bf16(s, p + o.W2, w + o.sh_W2, d * f);
   }
 
   void forward(int slot, const int32_t* ch, const void* x_in, void* x_out, cudaStream_t s) override {
@@ -334,19 +354,36 @@ class TfFamily : public Family {
     const int d = d_, f = spec_.ffn[c], h = spec_.heads[c], T = T_;
     float* P = master(j, c);
     bf16* W = w16_[(size_t)j * spec_.n() + c];
-    const bf16 *Wqkv = W, *Wo = W + 3 * (size_t)d * d, *W1 = W + 4 * (size_t)d * d,
-               *W2 = W1 + (size_t)f * d;
+    const bf16 *Win = W + o.sh_Win, *Wo = W + o.sh_Wo, *W1 = W + o.sh_W1, *W2 = W + o.sh_W2;
     ln_fwd(s, t.xin, P + o.ln1g, P + o.ln1b, t.a, t.mean1, t.rstd1, T, d);
-    GemmEpiParams e1;
-    e1.bias = P + o.bqkv;
-    e1.out = t.qkv;
-    gemm(s, T, 3 * d, d, t.a, false, d, Wqkv, false, d, EPI_BIAS_BF16, e1);
-    attn_fwd(s, t.qkv, t.o, t.lse, B_, S_, d, h);
+    // token mixer (attention, or one of Table 5's NLP convolutions, reading A38); its output
+    // projection adds the bias and the residual: x1 = x + M(a)
+    const bf16* mo = t.o;  // input of the output projection
+    int mo_k = d;
+    if (o.op == TF_ATTN) {
+      GemmEpiParams e1;
+      e1.bias = P + o.bin;
+      e1.out = t.qkv;
+      gemm(s, T, 3 * d, d, t.a, false, d, Win, false, d, EPI_BIAS_BF16, e1);
+      attn_fwd(s, t.qkv, t.o, t.lse, B_, S_, d, h);
+    } else if (o.op == TF_CONV3) {
+      conv3_cols(s, t.a, t.qkv, T, S_, d);  // [T, 3d] columns (t.qkv holds 3 T d)
+      mo = t.qkv;
+      mo_k = 3 * d;
+    } else if (o.op == TF_SEPCONV7) {
+      seqconv(s, t.a, P + o.taps, 0, 7, false, false, t.o, T, S_, d);
+    } else {  // Light Conv 5x1: v = a Wi^T + bi (in t.qkv), l = LightConv(v)
+      GemmEpiParams e1;
+      e1.bias = P + o.bin;
+      e1.out = t.qkv;
+      gemm(s, T, d, d, t.a, false, d, Win, false, d, EPI_BIAS_BF16, e1);
+      seqconv(s, t.qkv, P + o.taps, h, 5, false, false, t.o, T, S_, d);
+    }
     GemmEpiParams e2;
     e2.bias = P + o.bo;
     e2.resid = t.xin;
     e2.out = t.x1;
-    gemm(s, T, d, d, t.o, false, d, Wo, false, d, EPI_BIAS_RESID_F32, e2);
+    gemm(s, T, d, mo_k, mo, false, mo_k, Wo, false, mo_k, EPI_BIAS_RESID_F32, e2);
     ln_fwd(s, t.x1, P + o.ln2g, P + o.ln2b, t.a2, t.mean2, t.rstd2, T, d);
     GemmEpiParams e3;
     e3.bias = P + o.b1;
@@ -369,7 +406,7 @@ class TfFamily : public Family {
     const int d = d_, f = spec_.ffn[c], h = spec_.heads[c], T = T_;
     float* P = master(j, c);
     bf16* W = w16_[(size_t)j * spec_.n() + c];
-    bf16 *Wqkv = W, *Wo = W + 3 * (size_t)d * d, *W1 = W + 4 * (size_t)d * d, *W2 = W1 + (size_t)f * d;
+    bf16 *Win = W + o.sh_Win, *Wo = W + o.sh_Wo, *W1 = W + o.sh_W1, *W2 = W + o.sh_W2;
     float* U = upd(j, c);  // SGD WRITE target (P in place; the BSP accumulator, no shadow refresh)
     const bool inplace = in_place(j, c);
     auto sgd_ep = [&](float* w32, bf16* w16) {
@@ -395,31 +432,76 @@ class TfFamily : public Family {
     cudaStreamWaitEvent(side_, ev_da2_, 0);
     gemm(side_, f, d, T, dz_[p], true, f, t.a2, true, d, EPI_SGD, sgd_ep(U + o.W1, W1), true);  // W1 -= lr dz^T a2
     ln_bwd(s, da_, t.x1, t.mean2, t.rstd2, P + o.ln2g, dy, dx1_, dx1_16_[p], p_g2_[p], p_b2_[p], p_dbo_[p], T, d);
-    // ---- attention half
-    e = GemmEpiParams();
-    e.out = do16_;
-    gemm(s, T, d, d, dx1_16_[p], false, d, Wo, true, d, EPI_BF16, e);        // do = dx1 Wo
-    cudaEventRecord(ev_do_, s);
-    cudaStreamWaitEvent(side_, ev_do_, 0);
-    gemm(side_, d, d, T, dx1_16_[p], true, d, t.o, true, d, EPI_SGD, sgd_ep(U + o.Wo, Wo), true);  // Wo -= lr dx1^T o
-    attn_bwd(s, t.qkv, t.o, t.lse, do16_, dqkv_[p], B_, S_, d, h);
-    e = GemmEpiParams();
-    e.out = da_;
-    gemm(s, T, d, 3 * d, dqkv_[p], false, 3 * d, Wqkv, true, d, EPI_F32, e);  // da = dqkv Wqkv
-    cudaEventRecord(ev_da_, s);
-    cudaStreamWaitEvent(side_, ev_da_, 0);
-    colsum_bf16(side_, dqkv_[p], p_dbqkv_[p], T, 3 * d);
-    gemm(side_, 3 * d, d, T, dqkv_[p], true, 3 * d, t.a, true, d, EPI_SGD, sgd_ep(U + o.Wqkv, Wqkv), true);
+    // ---- mixer half (da = dM/da into da_; every weight gradient on the side stream after the
+    // dgrad that read the pre-update weight, reading A4)
+    int nl = 0;  // non-GEMM launches of the mixer half
+    if (o.op == TF_ATTN) {
+      e = GemmEpiParams();
+      e.out = do16_;
+      gemm(s, T, d, d, dx1_16_[p], false, d, Wo, true, d, EPI_BF16, e);        // do = dx1 Wo
+      cudaEventRecord(ev_do_, s);
+      cudaStreamWaitEvent(side_, ev_do_, 0);
+      gemm(side_, d, d, T, dx1_16_[p], true, d, t.o, true, d, EPI_SGD, sgd_ep(U + o.Wo, Wo), true);  // Wo -= lr dx1^T o
+      attn_bwd(s, t.qkv, t.o, t.lse, do16_, dqkv_[p], B_, S_, d, h);
+      e = GemmEpiParams();
+      e.out = da_;
+      gemm(s, T, d, 3 * d, dqkv_[p], false, 3 * d, Win, true, d, EPI_F32, e);  // da = dqkv Wqkv
+      cudaEventRecord(ev_da_, s);
+      cudaStreamWaitEvent(side_, ev_da_, 0);
+      colsum_bf16(side_, dqkv_[p], p_dbqkv_[p], T, 3 * d);
+      gemm(side_, 3 * d, d, T, dqkv_[p], true, 3 * d, t.a, true, d, EPI_SGD, sgd_ep(U + o.Win, Win), true);
+      nl = 2;
+    } else if (o.op == TF_CONV3) {
+      e = GemmEpiParams();
+      e.out = dcols_;
+      gemm(s, T, 3 * d, d, dx1_16_[p], false, d, Wo, true, 3 * d, EPI_F32, e);  // dcols = dx1 Wc
+      cudaEventRecord(ev_do_, s);
+      cudaStreamWaitEvent(side_, ev_do_, 0);
+      gemm(side_, d, 3 * d, T, dx1_16_[p], true, d, t.qkv, true, 3 * d, EPI_SGD, sgd_ep(U + o.Wo, Wo), true);
+      conv3_cols_bwd(s, dcols_, da_, T, S_, d);                                 // da = cols'(dcols)
+      nl = 1;
+    } else if (o.op == TF_SEPCONV7) {
+      bf16* ds = dqkv_[p];  // parity buffer: the side stream reads it
+      e = GemmEpiParams();
+      e.out = ds;
+      gemm(s, T, d, d, dx1_16_[p], false, d, Wo, true, d, EPI_BF16, e);        // ds = dx1 Wp
+      cudaEventRecord(ev_do_, s);
+      cudaStreamWaitEvent(side_, ev_do_, 0);
+      gemm(side_, d, d, T, dx1_16_[p], true, d, t.o, true, d, EPI_SGD, sgd_ep(U + o.Wo, Wo), true);  // Wp -= lr dx1^T s
+      seqconv(s, ds, P + o.taps, 0, 7, true, true, da_, T, S_, d);              // da = DW'(ds)
+      cudaEventRecord(ev_da_, s);
+      cudaStreamWaitEvent(side_, ev_da_, 0);
+      seqconv_wgrad_sgd(side_, ds, t.a, sc_acc_, sc_acc_ + (size_t)d * 7, sc_tick_, P + o.taps, U + o.taps, 0, 7, lr_, T, S_, d);
+      nl = 2;
+    } else {  // Light Conv 5x1
+      bf16 *dl = dqkv_[p], *dv = dqkv_[p] + (size_t)T * d;
+      e = GemmEpiParams();
+      e.out = dl;
+      gemm(s, T, d, d, dx1_16_[p], false, d, Wo, true, d, EPI_BF16, e);        // dl = dx1 Wo
+      cudaEventRecord(ev_do_, s);
+      cudaStreamWaitEvent(side_, ev_do_, 0);
+      gemm(side_, d, d, T, dx1_16_[p], true, d, t.o, true, d, EPI_SGD, sgd_ep(U + o.Wo, Wo), true);  // Wo -= lr dx1^T l
+      seqconv(s, dl, P + o.taps, h, 5, true, false, dv, T, S_, d);              // dv = LightConv'(dl)
+      e = GemmEpiParams();
+      e.out = da_;
+      gemm(s, T, d, d, dv, false, d, Win, true, d, EPI_F32, e);                 // da = dv Wi
+      cudaEventRecord(ev_da_, s);
+      cudaStreamWaitEvent(side_, ev_da_, 0);
+      seqconv_wgrad_sgd(side_, dl, t.qkv, sc_acc_, sc_acc_ + (size_t)d * 7, sc_tick_, P + o.taps, U + o.taps, h, 5, lr_, T, S_, d);
+      colsum_bf16(side_, dv, p_dbqkv_[p], T, d);
+      gemm(side_, d, d, T, dv, true, d, t.a, true, d, EPI_SGD, sgd_ep(U + o.Win, Win), true);  // Wi -= lr dv^T a
+      nl = 3;
+    }
     // bias / LN2 updates (all their partials are complete)
     SgdJobs j1{};
     j1.lr = lr_;
     j1.job[0] = {U + o.b2, p_db2_[p], db2_nblk, d};
     j1.job[1] = {U + o.b1, p_db1_[p], csb_, f};
     j1.job[2] = {U + o.bo, p_dbo_[p], lnb_, d};
-    j1.job[3] = {U + o.bqkv, p_dbqkv_[p], csb_, 3 * d};
-    j1.job[4] = {U + o.ln2g, p_g2_[p], lnb_, d};
-    j1.job[5] = {U + o.ln2b, p_b2_[p], lnb_, d};
-    j1.count = 6;
+    j1.job[3] = {U + o.ln2g, p_g2_[p], lnb_, d};
+    j1.job[4] = {U + o.ln2b, p_b2_[p], lnb_, d};
+    j1.count = 5;
+    if (o.n_bin) j1.job[j1.count++] = {U + o.bin, p_dbqkv_[p], csb_, (int)o.n_bin};
     sgd_multi(side_, j1);
     cudaEventRecord(ev_done_[p], side_);
     // LN1 backward: dx = dx1 + LN1'(da); its bf16 copy / column partials feed block j-1 and
@@ -433,7 +515,7 @@ class TfFamily : public Family {
     j2.job[1] = {U + o.ln1b, p_b1_, lnb_, d};
     j2.count = 2;
     sgd_multi(s, j2);
-    counters.launches += 7;
+    counters.launches += 5 + nl;
   }
 
   const Spec& spec_;
@@ -448,6 +530,9 @@ class TfFamily : public Family {
   float* ry_ = nullptr;   // recomputed block output (discarded)
   bf16 *dy16_[2], *dz_[2], *dx1_16_[2], *dqkv_[2], *do16_;
   float *da_, *dx1_, *gb_[2], *ws_ = nullptr;
+  float* dcols_ = nullptr;
+  unsigned long long* sc_acc_ = nullptr;
+  int* sc_tick_ = nullptr;
   size_t ws_elems_ = 0;
   float *p_db2_[2], *p_db1_[2], *p_dbo_[2], *p_dbqkv_[2], *p_g2_[2], *p_b2_[2], *p_g1_, *p_b1_;
   cudaStream_t side_ = nullptr;

@@ -170,6 +170,20 @@ int dw_wgrad_blocks(int B, int H, int C, int k, int S);
 // (acc [C*k*k + 1] and ticket zero between uses, fixpoint.cuh; w = master or BSP accumulator)
 void dw_wgrad_sgd(cudaStream_t s, const bf16* dz, const bf16* x, unsigned long long* acc, int* ticket, float* w,
                   float lr, int B, int H, int C, int k, int S, int dil);
+// ---- NLP op families (seqconv.cu; Table 5, reading A38).  x, dy: bf16 [T = B*S, d].
+// seqconv: depthwise conv along each sequence of S rows, taps w [d][k] (H == 0) or
+// softmax(Wl[H][k]) shared by d/H channels (Light Conv); flip = the input gradient; out bf16 or f32.
+void seqconv(cudaStream_t s, const bf16* x, const float* w, int H, int k, bool flip, bool out_f32, void* out, int T,
+             int S, int d);
+// weight gradient + SGD WRITE (wupd -= lr * g; Light Conv through the softmax Jacobian, wread =
+// the weights the forward used); acc [d*k] fixed-point totals and ticket zero between uses,
+// flag = sticky overflow flag (fixpoint.cuh)
+void seqconv_wgrad_sgd(cudaStream_t s, const bf16* dy, const bf16* x, unsigned long long* acc,
+                       unsigned long long* flag, int* ticket, const float* wread, float* wupd, int H, int k, float lr,
+                       int T, int S, int d);
+// Conv 3x1 im2col: cols [T][3d], cols[t][u*d+i] = x[t+u-1][i] inside the sequence; and its adjoint (f32)
+void conv3_cols(cudaStream_t s, const bf16* x, bf16* cols, int T, int S, int d);
+void conv3_cols_bwd(cudaStream_t s, const float* dcols, float* dx, int T, int S, int d);
 // channel split of a stride-1 block input [P, 2Ch] (x2): out[:, i] = x[:, 2i] (ld ldo, planes
 // oplane apart), xm[:, i] = x[:, 2i+1]; merge is its (plain bf16) backward
 void chan_split(cudaStream_t s, const bf16* x, int P, int Ch, bf16* out, int ldo, size_t oplane, bf16* xm);

@@ -58,11 +58,15 @@ Spec::Spec(const naspipe_supernet_spec* s) {
     NP_REQUIRE(raw.choice_heads && raw.choice_ffn, NASPIPE_EINVAL, "choice_heads/choice_ffn NULL");
     heads.assign(raw.choice_heads, raw.choice_heads + n);
     ffn.assign(raw.choice_ffn, raw.choice_ffn + n);
+    if (raw.choice_op) op.assign(raw.choice_op, raw.choice_op + n);
+    else op.assign(n, TF_ATTN);
     for (int c = 0; c < n; ++c) {
+      NP_REQUIRE(op[c] >= TF_ATTN && op[c] <= TF_LIGHTCONV5, NASPIPE_EINVAL, "choice_op[%d]=%d (0..3)", c, op[c]);
       NP_REQUIRE(heads[c] >= 1 && raw.d_model % heads[c] == 0, NASPIPE_EINVAL,
                  "heads[%d]=%d must divide d_model", c, heads[c]);
       const int hd = raw.d_model / heads[c];
-      NP_REQUIRE(hd % 16 == 0 && hd <= 128, NASPIPE_EINVAL, "head dim %d must be 16..128, %%16", hd);
+      NP_REQUIRE(op[c] != TF_ATTN || (hd % 16 == 0 && hd <= 128), NASPIPE_EINVAL,
+                 "head dim %d must be 16..128, %%16", hd);
       NP_REQUIRE(ffn[c] >= 16 && ffn[c] % 16 == 0, NASPIPE_EINVAL, "ffn[%d]=%d must be a multiple of 16",
                  c, ffn[c]);
     }
@@ -115,7 +119,7 @@ Spec::Spec(const naspipe_supernet_spec* s) {
 }
 
 Spec::Spec(const Spec& o)
-    : raw(o.raw), heads(o.heads), ffn(o.ffn), stage_of_block(o.stage_of_block),
+    : raw(o.raw), heads(o.heads), ffn(o.ffn), op(o.op), stage_of_block(o.stage_of_block),
       cost_fwd(o.cost_fwd), cost_bwd(o.cost_bwd), reps(o.reps), chans(o.chans), kern(o.kern),
       xcep(o.xcep), dil(o.dil), has_partition(o.has_partition), has_costs(o.has_costs) {
   repoint();
@@ -124,6 +128,7 @@ Spec::Spec(const Spec& o)
 void Spec::repoint() {
   raw.choice_heads = heads.empty() ? nullptr : heads.data();
   raw.choice_ffn = ffn.empty() ? nullptr : ffn.data();
+  raw.choice_op = op.empty() ? nullptr : op.data();
   raw.stage_of_block = has_partition ? stage_of_block.data() : nullptr;
   raw.cost_fwd = has_costs ? cost_fwd.data() : nullptr;
   raw.cost_bwd = has_costs ? cost_bwd.data() : nullptr;
@@ -250,17 +255,42 @@ void Spec::init_frozen(int part, float* dst) const {
 int Spec::rows() const { return family() == NASPIPE_MLP ? raw.batch : raw.batch * raw.seq_len; }
 
 TfOffsets Spec::tf_offsets(int c) const {
-  const size_t d = raw.d_model, f = ffn[c];
+  const size_t d = raw.d_model, f = ffn[c], H = heads[c];
   TfOffsets o{};
+  o.op = op[c];
   size_t off = 0;
   auto take = [&](size_t n) { size_t r = off; off += n; return r; };
-  o.Wqkv = take(3 * d * d); o.bqkv = take(3 * d);
-  o.Wo = take(d * d); o.bo = take(d);
+  switch (o.op) {  // packing order of oracle/transformer.py mixer_layout
+    case TF_ATTN:
+      o.n_Win = 3 * d * d; o.Win = take(o.n_Win); o.n_bin = 3 * d; o.bin = take(o.n_bin);
+      o.taps = off;
+      o.n_Wo = d * d; o.wo_in = (int)d; o.Wo = take(o.n_Wo); o.bo = take(d);
+      break;
+    case TF_CONV3:
+      o.Win = o.bin = o.taps = off;
+      o.n_Wo = 3 * d * d; o.wo_in = 3 * (int)d; o.Wo = take(o.n_Wo); o.bo = take(d);
+      break;
+    case TF_SEPCONV7:
+      o.Win = o.bin = off;
+      o.taps_rows = (int)d; o.taps_k = 7; o.n_taps = 7 * d; o.taps = take(o.n_taps);
+      o.n_Wo = d * d; o.wo_in = (int)d; o.Wo = take(o.n_Wo); o.bo = take(d);
+      break;
+    default:  // TF_LIGHTCONV5
+      o.n_Win = d * d; o.Win = take(o.n_Win); o.n_bin = d; o.bin = take(o.n_bin);
+      o.taps_rows = (int)H; o.taps_k = 5; o.n_taps = 5 * H; o.taps = take(o.n_taps);
+      o.n_Wo = d * d; o.wo_in = (int)d; o.Wo = take(o.n_Wo); o.bo = take(d);
+      break;
+  }
   o.ln1g = take(d); o.ln1b = take(d);
   o.W1 = take(f * d); o.b1 = take(f);
   o.W2 = take(d * f); o.b2 = take(d);
   o.ln2g = take(d); o.ln2b = take(d);
   o.total = off;
+  o.sh_Win = 0;
+  o.sh_Wo = o.n_Win;
+  o.sh_W1 = o.sh_Wo + o.n_Wo;
+  o.sh_W2 = o.sh_W1 + f * d;
+  o.sh_total = o.sh_W2 + d * f;
   return o;
 }
 
@@ -282,10 +312,13 @@ std::vector<Segment> Spec::segments(int b, int c) const {
   }
   const TfOffsets o = tf_offsets(c);
   const size_t d = raw.d_model, f = ffn[c];
-  s.push_back({o.Wqkv, 3 * d * d, 0, (int)d});
-  s.push_back({o.bqkv, 3 * d, 0, (int)d});
-  s.push_back({o.Wo, d * d, 0, (int)d});
-  s.push_back({o.bo, d, 0, (int)d});
+  if (o.n_Win) {
+    s.push_back({o.Win, o.n_Win, 0, (int)d});
+    s.push_back({o.bin, o.n_bin, 0, (int)d});
+  }
+  if (o.n_taps) s.push_back({o.taps, o.n_taps, 0, o.taps_k});
+  s.push_back({o.Wo, o.n_Wo, 0, o.wo_in});
+  s.push_back({o.bo, d, 0, o.wo_in});
   s.push_back({o.ln1g, d, 1, 0});
   s.push_back({o.ln1b, d, 2, 0});
   s.push_back({o.W1, f * d, 0, (int)d});
@@ -342,7 +375,10 @@ void Spec::default_costs(int32_t* cf, int32_t* cb) const {
       } else {
         const double d = raw.d_model, f = ffn[c], T = (double)raw.batch * raw.seq_len,
                      S = raw.seq_len;
-        flops = 2.0 * T * (4.0 * d * d + 2.0 * d * f) + 4.0 * T * S * d;
+        const int opc = op[c];
+        const double mix = opc == TF_ATTN ? 4.0 * d * d : opc == TF_CONV3 ? 3.0 * d * d
+                         : opc == TF_SEPCONV7 ? d * d + 7.0 * d : 2.0 * d * d + 5.0 * d;
+        flops = 2.0 * T * (mix + 2.0 * d * f) + (opc == TF_ATTN ? 4.0 * T * S * d : 0.0);
         bytes = 2.0 * T * (12.0 * d + 3.0 * f) + 2.0 * P;
       }
       const double tf = std::max(flops / peak, bytes / bw) * 1e6;

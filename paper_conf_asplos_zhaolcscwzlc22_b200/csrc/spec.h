@@ -22,8 +22,19 @@ struct Segment {
 
 // Offsets (in floats) of the transformer candidate tensors in the packed vector
 // (packing order of include/naspipe.h).
+// Transformer-family candidate (oracle/transformer.py layout).  The token mixer (reading A38)
+// is op: 0 attention (Win = Wqkv [3d,d], bin = bqkv, Wo [d,d], bo), 1 Conv 3x1 (Wo = Wc [d,3d],
+// bo = bc), 2 Sep Conv 7x1 (taps = Wd [d,7], Wo = Wp [d,d], bo = bp), 3 Light Conv 5x1 (Win = Wi
+// [d,d], bin = bi, taps = Wl [H,5], Wo [d,d], bo).  Unused roles have size 0 (offset = next).
+// The bf16 shadow holds Win at sh_Win, Wo at sh_Wo, then W1, W2 (sh_total elements).
+enum TfOp { TF_ATTN = 0, TF_CONV3 = 1, TF_SEPCONV7 = 2, TF_LIGHTCONV5 = 3 };
 struct TfOffsets {
-  size_t Wqkv, bqkv, Wo, bo, ln1g, ln1b, W1, b1, W2, b2, ln2g, ln2b, total;
+  int op;
+  size_t Win, bin, taps, Wo, bo, ln1g, ln1b, W1, b1, W2, b2, ln2g, ln2b, total;
+  size_t n_Win, n_bin, n_taps, n_Wo;  // element counts of the mixer matrices / bias / taps
+  int taps_k, taps_rows;       // taps: [taps_rows][taps_k]
+  int wo_in;                   // Wo's input width (d, or 3d for Conv 3x1)
+  size_t sh_Win, sh_Wo, sh_W1, sh_W2, sh_total;
 };
 
 // SPOS block geometry (SURVEY §8c "C2 SPOS candidate"; oracle/spos.py block_dims).
@@ -44,7 +55,7 @@ struct SposConv {
 
 struct Spec {
   naspipe_supernet_spec raw{};  // scalar fields; pointer fields re-pointed into vectors below
-  std::vector<int32_t> heads, ffn, stage_of_block, cost_fwd, cost_bwd;
+  std::vector<int32_t> heads, ffn, op, stage_of_block, cost_fwd, cost_bwd;
   std::vector<int32_t> reps, chans, kern, xcep, dil;  // SPOS
   bool has_partition = false, has_costs = false;
 

@@ -48,6 +48,20 @@ CONFIGS = {
                               choice_heads=[16] * 4 + [32] * 4,
                               choice_ffn=[4096, 8192, 12288, 16384] * 2,
                               lr=0.01, compute_dtype="bf16", n_stages=8, n_subnets=64),
+    # NLP.c3 analog (Table 1: 48 choice blocks x 24 layers per block) over Table 5's
+    # NLP ops (reading A38): {8/16-head attention, Conv 3x1, Sep Conv 7x1, Light
+    # Conv 5x1 with 8/16 weight-sharing heads} x FFN {1024, 2048, 3072}; d, seq and batch of
+    # configs[2].
+    "nlp_c3": dict(family="transformer", n_blocks=48, n_choices=24, batch=32, d_model=1024, seq_len=128,
+                   choice_op=[op for op in (0, 1, 2, 3) for _ in range(6)],
+                   choice_heads=[h for _ in range(4) for h in (8, 16) for _ in range(3)],
+                   choice_ffn=[f for _ in range(8) for f in (1024, 2048, 3072)],
+                   lr=0.01, compute_dtype="bf16", n_stages=8, n_subnets=256),
+    # small supernet with every NLP op (parity tests of A38): Conv 3x1, Sep Conv 7x1, Light
+    # Conv 5x1 (H = 4), attention
+    "tiny_nlp": dict(family="transformer", n_blocks=4, n_choices=4, batch=2, d_model=192, seq_len=128,
+                     choice_op=[1, 2, 3, 0], choice_heads=[3, 2, 4, 3], choice_ffn=[320, 384, 192, 256],
+                     lr=0.01, compute_dtype="bf16", n_stages=2, n_subnets=8),
     # Small transformer used by the parity tests: several GEMM tiles in every dimension
     # and ragged tails (d=192 is 1.5 x 128; f=320 is 2.5 x 128), seq 128 like the real one.
     "tiny_transformer": dict(family="transformer", n_blocks=4, n_choices=3, batch=2,

@@ -26,16 +26,20 @@ def test_exports_every_declared_symbol():
     assert npipe.naspipe_abi_version() == 4
 
 
-@pytest.mark.parametrize("name", ["toy", "tiny_transformer", "transformer"])
+@pytest.mark.parametrize("name", ["toy", "tiny_transformer", "transformer", "tiny_nlp", "nlp_c3"])
 def test_init_params_match_shared_hash(name):
+    """Packed sizes and counter-hash init equal the oracle's layout (nlp: every op, A38)."""
     cfg = synth.get_config(name)
     spec = npipe.Spec(cfg)
     n = cfg["n_choices"]
-    for (b, c) in [(0, 0), (1, n - 1), (cfg["n_blocks"] - 1, n // 2)]:
+    pairs = [(0, 0), (1, n - 1), (cfg["n_blocks"] - 1, n // 2)]
+    if name in ("tiny_nlp", "nlp_c3"):
+        pairs += [(2, c) for c in range(n)]
+    for (b, c) in pairs:
         got = npipe.naspipe_init_params(spec, b, c)
         segs = [(int(np.prod(s)), kind, fan) for _, s, kind, fan in train.candidate_layout(cfg, b, c)]
         assert npipe.naspipe_param_count(spec, b, c) == sum(s for s, _, _ in segs)
-        if name == "transformer" and (b, c) != (0, 0):
+        if name in ("transformer", "nlp_c3") and (b, c) not in ((0, 0), (2, 6), (2, 12), (2, 18)):
             continue  # one full-size candidate is enough (12.6 M floats)
         ref = synth.init_packed(cfg["init_seed"], b * n + c, segs)
         assert np.array_equal(got.view(np.uint32), ref.view(np.uint32)), (b, c)
@@ -63,6 +67,17 @@ def test_spos_layout_and_init_match_oracle(name):
         ref = fz[key]["w"].ravel().astype(np.float32)
         got = npipe.naspipe_init_frozen(spec, part, ref.size)
         assert np.array_equal(got.view(np.uint32), ref.view(np.uint32)), key
+
+
+def test_nlp_op_spec_validation():
+    cfg = synth.get_config("tiny_nlp")
+    for bad in (dict(choice_op=[1, 2, 4, 0]), dict(choice_op=[1, 2, -1, 0]), dict(choice_heads=[3, 2, 5, 3])):
+        with pytest.raises(npipe.NaspipeError):
+            npipe.naspipe_default_costs(npipe.Spec(dict(cfg, **bad)))
+    # Light Conv heads need not give a 16-multiple head dim (only attention does): H = 12, d/H = 16
+    npipe.naspipe_default_costs(npipe.Spec(dict(cfg, choice_heads=[3, 2, 12, 3])))
+    cf, cb = npipe.naspipe_default_costs(npipe.Spec(synth.get_config("nlp_c3")))
+    assert (cf >= 1).all() and (cb > cf).all()
 
 
 def test_spos_spec_validation():

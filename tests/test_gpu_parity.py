@@ -124,6 +124,32 @@ def test_tiny_transformer_bitwise_across_runs_and_stage_counts():
             assert np.array_equal(p[k].view(np.uint32), base[k].view(np.uint32)), (D, k)
 
 
+@pytest.mark.parametrize("N,tol", [(1, 1e-3), (8, 1e-3), (100, 1e-2)])
+def test_tiny_nlp_ops_parity(N, tol):
+    """Table 5's NLP ops (Conv 3x1, Sep Conv 7x1, Light Conv 5x1, attention; reading A38) as
+    candidates of one supernet: subnets cycle the choices so every (block, op) is trained."""
+    cfg = synth.get_config("tiny_nlp")
+    m, n = cfg["n_blocks"], cfg["n_choices"]
+    choices = np.array([[(y + b) % n for b in range(m)] for y in range(N)], dtype=np.int32)
+    batches = [synth.make_batch(cfg, y) for y in range(N)]
+    theta0, ref, ref_loss = _oracle(cfg, choices, batches)
+    params, losses, trace, _ = run_engine(cfg, choices, batches, D=2)
+    sm = param_errors(cfg, params, ref, theta0)
+    pm.check(sm, tol, pm.UPD_BF16 if N <= 8 else None)
+    np.testing.assert_allclose(losses, ref_loss, rtol=1e-2)
+    _check_trace(cfg, choices, 2, trace)
+
+
+def test_tiny_nlp_ops_bitwise_across_stage_counts():
+    cfg, choices, batches = _workload("tiny_nlp", 10)
+    base, base_loss, _, _ = run_engine(cfg, choices, batches, D=1)
+    for D, where in ((1, npipe.BATCH_HOST), (2, npipe.BATCH_DEVICE), (4, npipe.BATCH_HOST)):
+        p, l, _, _ = run_engine(cfg, choices, batches, D=D, where=where)
+        assert np.array_equal(l.view(np.uint32), base_loss.view(np.uint32)), D
+        for k in base:
+            assert np.array_equal(p[k].view(np.uint32), base[k].view(np.uint32)), (D, k)
+
+
 def test_null_kernels_and_errors():
     cfg, choices, batches = _workload("toy", 6)
     spec = npipe.Spec(cfg, flags=FLAGS | npipe.FLAG_NULL_KERNELS)
