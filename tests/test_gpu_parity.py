@@ -221,3 +221,20 @@ def test_transformer_full_size_against_oracle_samples(steps, tol):
     print(f"configs[2] full size, {steps} steps: {pm.fmt(sm)}; losses {losses[-2:]} vs {gold['losses'][steps - 2:steps]}")
     pm.check(sm, tol, pm.UPD_BF16 if steps == 1 else None)
     np.testing.assert_allclose(losses, gold["losses"][:steps], rtol=1e-2)
+
+
+def test_nlp_c3_full_size_one_step_against_oracle_samples():
+    """The NLP.c3 analog (Table 1: 48 blocks x 24 choices over Table 5's NLP ops,
+    reading A38; d = 1024, S = 128, B = 32) at full size in the bench's launch configuration:
+    one subnet against sampled outputs of the fp64 oracle (tests/golden/nlp_c3_fullsize_1steps.npz,
+    tools/make_multistep_golden.py, oracle/ only): per-tensor A15 <= 1e-3, the update bars,
+    loss rtol 1e-2."""
+    gold = load_gold("nlp_c3_fullsize_1steps.npz")
+    cfg, h, got_of, losses = run_fullsize("nlp_c3", gold, 1)
+    sm = pm.sampled_errors(cfg, gold, 1, got_of)
+    npipe.naspipe_destroy(h)
+    ops = np.asarray(cfg["choice_op"])[gold["choices"][0]]
+    print(f"nlp_c3 full size, 1 step (ops used {np.bincount(ops, minlength=4).tolist()}): {pm.fmt(sm)}; "
+          f"loss {losses} vs {gold['losses'][:1]}")
+    pm.check(sm, 1e-3, pm.UPD_BF16)
+    np.testing.assert_allclose(losses, gold["losses"][:1], rtol=1e-2)
