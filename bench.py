@@ -67,6 +67,8 @@ def parse():
                     help="HBM weight budget per stage as a multiple of one subnet's mean stage slice "
                          "(0 = all candidates resident; P:L337 uses ~3)")
     ap.add_argument("--n-choices", type=int, default=0, help="override n (search-space sweep, configs[4])")
+    ap.add_argument("--virtual-stages", type=int, default=1,
+                    help="N = 1: pipeline stages on the one GPU (CSP across concurrently running stage streams)")
     ap.add_argument("--lookahead", type=int, default=0, help="residency prefetch depth L in tasks (0 = 2, P:L156)")
     return ap.parse_args()
 
@@ -464,7 +466,7 @@ def main():
 
     def create(sp):
         if world == 1:
-            return npipe.naspipe_create(sp, 1)
+            return npipe.naspipe_create(sp, args.virtual_stages)
         if args.transport == "nccl":
             ids = [None]
             if rank == 0:
@@ -590,7 +592,8 @@ def main():
             e2e_hw = (w_step * 1e-12) / (D * pk[w_peak] * (ms / args.steps / 1000))
         elif fam == "spos":
             e2e_hw = (roofline["algorithmic_bytes_per_step"] * 1e-9) / (D * pk["hbm"] * (ms / args.steps / 1000))
-        plan_ms = plan_bound_ms(cfg, npipe, timed_choices, D, [b for b in busy]) if args.sync == "csp" else None
+        plan_ms = (plan_bound_ms(cfg, npipe, timed_choices, D, [b for b in busy])
+                   if args.sync == "csp" and args.virtual_stages == 1 else None)
         fractions = {"kernel": roofline["frac"],
                      "end_to_end_vs_hardware": e2e_hw,
                      "end_to_end_vs_hardware_note": ("(GEMM + attention flops) / (D x sustained bf16 peak x step time)"
