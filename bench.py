@@ -382,7 +382,10 @@ def workload_config(args, cfg, world):
          "stages": world, "parallelism": f"pp{world}" if world > 1 else "single stage",
          "activation_recompute": bool(getattr(args, "recompute", False)),
          "sync_policy": getattr(args, "sync", "csp"),
-         "l2": "working set > L2 (active weights + activations per step >> 126 MB)"}
+         "l2": "working set > L2 (active weights + activations per step >> 126 MB)",
+         # reduction-order / launch tuning knobs in effect (empty = the library defaults):
+         # bitwise comparisons carry their reduction configuration
+         "env_knobs": {k: v for k, v in sorted(os.environ.items()) if k.startswith("NASPIPE_")}}
     if cfg["family"] == "transformer":
         c.update(seq_len=cfg["seq_len"], d_model=cfg["d_model"], heads=cfg["choice_heads"], ffn=cfg["choice_ffn"])
         if "choice_op" in cfg:

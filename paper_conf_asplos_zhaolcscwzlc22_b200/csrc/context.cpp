@@ -64,18 +64,22 @@ CandidateStore::CandidateStore(const Spec& spec, const Planner& planner, int K, 
       CU(cudaEventCreateWithFlags(&stage_free_[i], cudaEventDisableTiming));
       CU(cudaEventCreateWithFlags(&staged_[i], cudaEventDisableTiming));
     }
-    // keep freed blocks in the stream-ordered pool: loads reuse evicted memory
-    cudaMemPool_t pool;
-    CU(cudaDeviceGetDefaultMemPool(&pool, dev));
+    // a private stream-ordered pool (the device's default pool and stream 0 are
+    // left alone) that keeps freed blocks: loads reuse evicted memory
+    cudaMemPoolProps props{};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = dev;
+    CU(cudaMemPoolCreate(&pool_, &props));
     uint64_t thr = UINT64_MAX;
-    CU(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
+    CU(cudaMemPoolSetAttribute(pool_, cudaMemPoolAttrReleaseThreshold, &thr));
     // reserve the pool up front (fp32 masters + bf16 shadows of a full budget, plus the
     // in-flight loads/evictions) so no load pays for growing the pool mid-run
     void* reserve = nullptr;
     const size_t rbytes = (size_t)(2.0 * (double)budget_);
-    if (cudaMallocAsync(&reserve, rbytes, 0) == cudaSuccess) {
-      cudaFreeAsync(reserve, 0);
-      cudaStreamSynchronize(0);
+    if (cudaMallocFromPoolAsync(&reserve, rbytes, pool_, evict_) == cudaSuccess) {
+      cudaFreeAsync(reserve, evict_);
+      cudaStreamSynchronize(evict_);
     } else {
       cudaGetLastError();  // not fatal: the pool grows on demand
     }
@@ -121,8 +125,8 @@ CandidateStore::~CandidateStore() {
   if (wb_) cudaStreamSynchronize(wb_);  // write-backs into the stash have landed
   for (auto& cd : cands_) {
     if (cd.stash) cudaFreeHost(cd.stash);
-    if (managed() && cd.w32) cudaFree(cd.w32);
-    if (managed() && cd.w16) cudaFree(cd.w16);
+    if (managed() && cd.w32) cudaFreeAsync(cd.w32, evict_);
+    if (managed() && cd.w16) cudaFreeAsync(cd.w16, evict_);
     if (cd.ready) cudaEventDestroy(cd.ready);
     if (cd.last_use) cudaEventDestroy(cd.last_use);
     if (cd.wb_done) cudaEventDestroy(cd.wb_done);
@@ -132,6 +136,7 @@ CandidateStore::~CandidateStore() {
     cudaStreamSynchronize(evict_);
     cudaStreamDestroy(evict_);
   }
+  if (pool_) cudaMemPoolDestroy(pool_);
   if (shadow_) {
     cudaStreamSynchronize(shadow_);
     cudaStreamDestroy(shadow_);
@@ -164,8 +169,8 @@ bool CandidateStore::ready() const { return !managed() || belady_->can_decide();
 
 void CandidateStore::load(Cand& cd, cudaStream_t copy) {
   CU(cudaStreamWaitEvent(copy, cd.wb_done, 0));  // a reload reads the written-back stash
-  CU(cudaMallocAsync(reinterpret_cast<void**>(&cd.w32), cd.n32 * 4, copy));
-  if (cd.n16) CU(cudaMallocAsync(reinterpret_cast<void**>(&cd.w16), cd.n16 * 2, copy));
+  CU(cudaMallocFromPoolAsync(reinterpret_cast<void**>(&cd.w32), cd.n32 * 4, pool_, copy));
+  if (cd.n16) CU(cudaMallocFromPoolAsync(reinterpret_cast<void**>(&cd.w16), cd.n16 * 2, pool_, copy));
   CU(cudaMemcpyAsync(cd.w32, cd.stash, cd.n32 * 4, cudaMemcpyHostToDevice, copy));
   fam_->bind(cd.j, cd.c, cd.w32, cd.w16);
   // the bf16 shadow is a kernel: on its own stream, so the copy stream's next H2D does not

@@ -62,6 +62,7 @@ class CandidateStore {
   std::vector<ResidencyEvent> log;
 
  private:
+  cudaMemPool_t pool_ = nullptr;  // private pool of the managed candidates (context switching)
   struct Cand {
     int j = -1, c = -1;  // local block, choice
     size_t n32 = 0, n16 = 0;
