@@ -434,6 +434,8 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if os.environ.get("NASPIPE_BENCH_SHARE_GPU"):  # test only: every rank on GPU 0 (1-GPU boxes)
+        local = 0
     cfg = synth.get_config(args.workload) if args.n_choices == 0 else synth.sweep_config(args.n_choices)
     if args.impl == "reference":
         run_reference(args, cfg, rank, world)
@@ -454,7 +456,10 @@ def main():
 
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if os.environ.get("NASPIPE_BENCH_SHARE_GPU"):  # NCCL refuses two ranks on one GPU
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     D = world
     m, n, B = cfg["n_blocks"], cfg["n_choices"], cfg["batch"]
     total = args.warmup + 4 * args.steps
@@ -492,7 +497,7 @@ def main():
     def reduce(v, op="max"):
         if world == 1:
             return v
-        t = torch.tensor([v], device="cuda", dtype=torch.float64)
+        t = torch.tensor([v], device="cpu" if dist.get_backend() == "gloo" else "cuda", dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX if op == "max" else dist.ReduceOp.SUM)
         return float(t.item())
 
