@@ -54,6 +54,25 @@ int naspipe_debug_gemm_x2(int M, int N, int K, const void* A_hi, const void* A_l
                           const void* B_lo, int ldb, void* out_hi, void* out_lo, void* stream);
 int naspipe_debug_chan_merge(const void* dproj, int ldp, const void* dm, int P, int Ch, void* dx, void* stream);
 int naspipe_debug_stem(const float* x, const float* w, void* z, int B, int H, int C0, void* stream);
+/* Input gradient with the fused BatchNorm-backward reduction (bn_bwd_reduce fused into its
+ * producer): kind 0 / 2 = stride-1 / stride-2 depthwise dx = dw'(dz) (w fp32 [C][k][k], dx
+ * [B,H,H,C], dz [B,Ho,Ho,C]),
+ * kind 1 = 1x1-conv dx = dz W on the tcgen05 GEMM (EPI_BNBWD; dz bf16 [P][Cout], w16 bf16
+ * [Cout][C], P = B*H*H).  dx is the output gradient of the unit z (x2 [P][C]) -> BN(mean,
+ * rstd, g, b) [-> ReLU]: sums[2][C] = (sum dy', sum dy' xh) over the stored dx. */
+/* bn_apply folded into the depthwise consumer (BnApplyIn): the unit zin (x2 [B,H,H,C]) ->
+ * BN(g, b) [-> ReLU] -> depthwise k x k stride S dilation dil (w fp32 [C][k][k]).  Stored path:
+ * bn_stats, bn_apply -> y, dw_fwd(y) -> out_ref (x2 [B,Ho,Ho,C]) and the weight gradient
+ * dwsum_ref[C*k*k] = sum dz * y_hi; folded path: bn_stats, dw_fwd_bn -> out (and the published
+ * meta[4][C] = mean, rstd, g, b), dw_wgrad with BN on load -> dwsum.  mean_ref / rstd_ref [C]
+ * are bn_apply's. */
+int naspipe_debug_dw_bn_fold(const void* zin, int B, int H, int C, const float* g, const float* b, int relu,
+                             const float* w, int k, int S, int dil, const void* dz, void* out_ref, void* out,
+                             float* dwsum_ref, float* dwsum, float* meta, float* mean_ref, float* rstd_ref,
+                             void* stream);
+int naspipe_debug_bnb_fused(int kind, const void* dz, const float* w, const void* w16, void* dx, int B, int H, int C,
+                            int Cout, int k, int dil, const void* z, const float* mean, const float* rstd,
+                            const float* g, const float* b, int relu, float* sums, void* stream);
 
 #if defined(__GNUC__)
 #pragma GCC visibility pop

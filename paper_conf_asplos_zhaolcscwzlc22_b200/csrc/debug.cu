@@ -173,6 +173,99 @@ int naspipe_debug_bn_bwd(const void* dy, int lddy, const void* z, int P, int C, 
   });
 }
 
+int naspipe_debug_dw_bn_fold(const void* zin, int B, int H, int C, const float* g, const float* b, int relu,
+                             const float* w, int k, int S, int dil, const void* dz, void* out_ref, void* out,
+                             float* dwsum_ref, float* dwsum, float* meta, float* mean_ref, float* rstd_ref,
+                             void* stream) {
+  return dguard([&] {
+    cudaStream_t s = (cudaStream_t)stream;
+    const int P = B * H * H;
+    const size_t n = (size_t)P * C;
+    unsigned long long *acc = nullptr, *acc2 = nullptr, *wacc = nullptr;
+    int* tick = nullptr;
+    bf16* y = nullptr;
+    NP_REQUIRE(cudaMalloc(&acc, (2 * (size_t)C + 1) * 8) == cudaSuccess && cudaMalloc(&acc2, (2 * (size_t)C + 1) * 8) == cudaSuccess &&
+                   cudaMalloc(&wacc, ((size_t)C * k * k + 1) * 8) == cudaSuccess && cudaMalloc(&tick, 16) == cudaSuccess &&
+                   cudaMalloc(&y, 2 * n * sizeof(bf16)) == cudaSuccess,
+               NASPIPE_ENOMEM, "malloc");
+    cudaMemsetAsync(acc, 0, (2 * (size_t)C + 1) * 8, s);
+    cudaMemsetAsync(acc2, 0, (2 * (size_t)C + 1) * 8, s);
+    cudaMemsetAsync(wacc, 0, ((size_t)C * k * k + 1) * 8, s);
+    cudaMemsetAsync(tick, 0, 16, s);
+    cudaMemsetAsync(dwsum_ref, 0, (size_t)C * k * k * 4, s);
+    cudaMemsetAsync(dwsum, 0, (size_t)C * k * k * 4, s);
+    // stored path
+    bn_stats(s, (const bf16*)zin, P, C, acc);
+    bn_apply(s, (const bf16*)zin, P, C, acc, tick, mean_ref, rstd_ref, g, b, relu, y, C, n);
+    dw_fwd(s, y, w, (bf16*)out_ref, B, H, C, k, S, dil, acc2);
+    cudaMemsetAsync(acc2, 0, (2 * (size_t)C + 1) * 8, s);
+    dw_wgrad_sgd(s, (const bf16*)dz, y, wacc, tick + 1, dwsum_ref, -1.0f, B, H, C, k, S, dil);  // 0 + sum
+    // folded path
+    BnApplyIn xin;
+    xin.z = (const bf16*)zin;
+    xin.zplane = n;
+    xin.P = P;
+    xin.acc = acc;
+    xin.ticket = tick + 2;
+    xin.mean = meta;
+    xin.rstd = meta + C;
+    xin.g = g;
+    xin.b = b;
+    xin.gsnap = meta + 2 * C;
+    xin.bsnap = meta + 3 * C;
+    xin.relu = relu;
+    bn_stats(s, (const bf16*)zin, P, C, acc);
+    dw_fwd_bn(s, xin, w, (bf16*)out, B, H, C, k, S, dil, acc2);
+    dw_wgrad_sgd(s, (const bf16*)dz, nullptr, wacc, tick + 1, dwsum, -1.0f, B, H, C, k, S, dil, &xin);
+    cudaStreamSynchronize(s);
+    std::vector<unsigned long long> h(2 * (size_t)C);
+    cudaMemcpy(h.data(), acc, h.size() * 8, cudaMemcpyDeviceToHost);
+    for (auto v : h) NP_REQUIRE(v == 0, NASPIPE_EINTERNAL, "dw_fwd_bn left its input sums uncleared");
+    cudaFree(acc);
+    cudaFree(acc2);
+    cudaFree(wacc);
+    cudaFree(tick);
+    cudaFree(y);
+  });
+}
+
+int naspipe_debug_bnb_fused(int kind, const void* dz, const float* w, const void* w16, void* dx, int B, int H, int C,
+                            int Cout, int k, int dil, const void* z, const float* mean, const float* rstd,
+                            const float* g, const float* b, int relu, float* sums, void* stream) {
+  return dguard([&] {
+    cudaStream_t s = (cudaStream_t)stream;
+    const int P = B * H * H;
+    unsigned long long* acc = nullptr;
+    NP_REQUIRE(cudaMalloc(&acc, (2 * (size_t)C + 1) * 8) == cudaSuccess, NASPIPE_ENOMEM, "malloc");
+    cudaMemsetAsync(acc, 0, (2 * (size_t)C + 1) * 8, s);
+    BnBwdFuse f;
+    f.z = (const bf16*)z;
+    f.zplane = (size_t)P * C;
+    f.mean = mean;
+    f.rstd = rstd;
+    f.g = g;
+    f.b = b;
+    f.relu = relu;
+    f.acc = acc;
+    if (kind == 0 || kind == 2) {
+      dw_dgrad(s, (const bf16*)dz, w, nullptr, (bf16*)dx, B, H, C, k, kind == 2 ? 2 : 1, dil, f);
+    } else {
+      GemmEpiParams e;
+      e.out = dx;
+      e.bnb = f;
+      gemm_bf16_tc(s, P, C, Cout, (const bf16*)dz, false, Cout, (const bf16*)w16, true, C, EPI_BNBWD, e);
+    }
+    cudaStreamSynchronize(s);
+    std::vector<unsigned long long> h(2 * (size_t)C + 1);
+    cudaMemcpy(h.data(), acc, h.size() * 8, cudaMemcpyDeviceToHost);
+    NP_REQUIRE(h[2 * (size_t)C] == 0, NASPIPE_EINTERNAL, "fixed-point overflow flag set");
+    std::vector<float> fs(2 * (size_t)C);
+    for (size_t i = 0; i < fs.size(); ++i) fs[i] = (float)((double)(long long)h[i] / 1099511627776.0);
+    cudaMemcpy(sums, fs.data(), fs.size() * 4, cudaMemcpyHostToDevice);
+    cudaFree(acc);
+  });
+}
+
 int naspipe_debug_chan_split(const void* x, int P, int Ch, void* out, int ldo, size_t oplane, void* xm,
                              void* stream) {
   return dguard([&] { chan_split((cudaStream_t)stream, (const bf16*)x, P, Ch, (bf16*)out, ldo, oplane, (bf16*)xm); });

@@ -13,6 +13,7 @@
 // deterministic split-K over the pixels, refreshing W's hi/lo planes), depthwise convs and
 // BatchNorm on CUDA cores (spos.cu).
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 
 #include "family.h"
@@ -22,9 +23,11 @@ namespace naspipe {
 namespace {
 
 struct UnitRec {  // forward stash of one unit of (slot, block)
-  const bf16* x;  // unit input (hi plane; bf16x2)
+  const bf16* x;  // unit input (hi plane; bf16x2); nullptr when xbn.z is set
   bf16* z;        // conv output (bf16x2, contiguous)
-  float *mean, *rstd;
+  float *mean, *rstd;  // [C] each, then the g, b snapshots [C] each (published when the
+                       // unit's bn_apply is folded into its depthwise consumer)
+  BnApplyIn xbn;  // depthwise unit whose input is the previous unit's BN applied on load
 };
 
 class SposFamily : public Family {
@@ -56,7 +59,7 @@ class SposFamily : public Family {
           const SposConv& u = L[i];
           const size_t po = P(u.H_out), pi = P(u.H_in);
           need += 2 * po * u.cout * (last_of_branch(L, i) ? 1 : 2);
-          st += 2 * (size_t)u.cout;
+          st += 4 * (size_t)u.cout;
           dz_max = std::max(dz_max, po * u.cout);
           g_max = std::max({g_max, pi * u.cin, po * u.cout});
           C_max = std::max(C_max, (size_t)u.cout);
@@ -101,11 +104,14 @@ class SposFamily : public Family {
     // and zero everywhere, so every flag position starts (and, flags aside, stays) zero
     acc_f_ = A.alloc<unsigned long long>(2 * C_max + 1);
     acc_b_ = A.alloc<unsigned long long>(2 * C_max + 1);
-    tick_ = A.alloc<int>(3);  // bn_apply, bn_bwd_apply, dw weight gradient (side stream)
+    acc_f2_ = A.alloc<unsigned long long>(2 * C_max + 1);
+    // bn_apply, bn_bwd_apply, dw weight gradient (side stream), depthwise conv with BN on load
+    tick_ = A.alloc<int>(4);
     cudaMemset(acc_f_, 0, (2 * C_max + 1) * 8);
     cudaMemset(acc_b_, 0, (2 * C_max + 1) * 8);
+    cudaMemset(acc_f2_, 0, (2 * C_max + 1) * 8);
     C_max_ = (int)C_max;
-    cudaMemset(tick_, 0, 3 * sizeof(int));
+    cudaMemset(tick_, 0, 4 * sizeof(int));
     dwk_max_ = dwk_max;
     acc_w_ = A.alloc<unsigned long long>(dwk_max + 1);
     cudaMemset(acc_w_, 0, (dwk_max + 1) * 8);
@@ -182,7 +188,8 @@ class SposFamily : public Family {
       const int Po = (int)P(H / 2);
       spos_stem_conv(s, static_cast<const float*>(x_in), w_stem_, stem_z_, B_, H, C0);
       t_bn_stats(s, stem_z_, Po, C0, stem_mean_, stem_rstd_);
-      t_bn_apply(s, stem_z_, Po, C0, stem_mean_, stem_rstd_, ones_s_, zeros_s_, 1, stem_y_[slot], C0, (size_t)Po * C0);
+      t_bn_apply(s, stem_z_, Po, C0, stem_mean_, stem_rstd_, ones_s_, zeros_s_, 1, stem_y_[slot], C0, (size_t)Po * C0,
+                 acc_f_);
       counters.launches += 3;
       x = stem_y_[slot];
     }
@@ -234,7 +241,7 @@ class SposFamily : public Family {
     const bf16* xo = static_cast<const bf16*>(out);
     e.stats = acc_f_;  // fused bn_stats
     gemm_x2(s, PL, Ch, Cl, xo, xo + (size_t)PL * Cl, Cl, wh16_, wh16_ + (size_t)Ch * Cl, Cl, e);
-    t_bn_apply(s, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, 1, rh_, Ch, (size_t)PL * Ch);
+    t_bn_apply(s, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, 1, rh_, Ch, (size_t)PL * Ch, acc_f_);
     gap_pool(s, rh_, B_, HW, Ch, gap_);
     fc_ce(s, gap_, wf_, static_cast<const int*>(target), B_, Ch, ncls, logits_, dlogits_, loss_per_);
     ce_mean(s, loss_per_, B_, loss_dst);
@@ -251,7 +258,7 @@ class SposFamily : public Family {
   void check_after_drain() override {
     bool bad = false;  // a flag at acc[2C] of any use; the accumulators are zero elsewhere after a drain
     std::vector<unsigned long long> h(2 * (size_t)C_max_ + 1);
-    for (const unsigned long long* a : {acc_f_, acc_b_}) {
+    for (const unsigned long long* a : {acc_f_, acc_b_, acc_f2_}) {
       cudaMemcpy(h.data(), a, h.size() * 8, cudaMemcpyDeviceToHost);
       for (auto v : h) bad |= v != 0;
     }
@@ -298,9 +305,9 @@ class SposFamily : public Family {
     if (timer) timer->end(s, 4.0 * Pp * C);
   }
   void t_bn_apply(cudaStream_t s, const bf16* z, int Pp, int C, float* mean, float* rstd, const float* g,
-                  const float* b, int relu, bf16* y, int ldy, size_t yplane) {
+                  const float* b, int relu, bf16* y, int ldy, size_t yplane, unsigned long long* acc) {
     if (timer) timer->begin(s);
-    bn_apply(s, z, Pp, C, acc_f_, tick_, mean, rstd, g, b, relu, y, ldy, yplane);
+    bn_apply(s, z, Pp, C, acc, tick_, mean, rstd, g, b, relu, y, ldy, yplane);
     if (timer) timer->end(s, 8.0 * Pp * C);
   }
   void t_bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int Pp, int C, const float* mean,
@@ -342,6 +349,7 @@ class SposFamily : public Family {
     }
     const bf16* h = nullptr;
     size_t hplane = 0;
+    BnApplyIn pend;  // the previous unit's BN, folded into this depthwise conv's input load
     for (size_t i = 0; i < L.size(); ++i) {
       const SposConv& u = L[i];
       if (i == 0 || L[i - 1].branch != u.branch) {
@@ -350,11 +358,21 @@ class SposFamily : public Family {
       }
       const int Po = (int)P(u.H_out);
       const size_t zplane = (size_t)Po * u.cout;
-      UnitRec r{h, cv, st, st + u.cout};
+      UnitRec r{h, cv, st, st + u.cout, BnApplyIn()};
       cv += 2 * zplane;
-      st += 2 * u.cout;
-      if (u.dw) {  // the depthwise conv adds the BatchNorm sums of its output itself (fused bn_stats)
-        dw_fwd(s, h, Pm + u.off_w, r.z, B_, u.H_in, u.cin, u.k, u.stride, u.dil, acc_f_);
+      st += 4 * u.cout;
+      // the depthwise conv adds the BatchNorm sums of its output itself (fused bn_stats); with
+      // its input's BN applied on load it reads acc_f_ and so adds its own sums to acc_f2_
+      unsigned long long* zacc = acc_f_;
+      if (u.dw && pend.z != nullptr) {
+        r.x = nullptr;
+        r.xbn = pend;
+        zacc = acc_f2_;
+        dw_fwd_bn(s, pend, Pm + u.off_w, r.z, B_, u.H_in, u.cin, u.k, u.stride, u.dil, zacc);
+        counters.launches++;
+        pend = BnApplyIn();
+      } else if (u.dw) {
+        dw_fwd(s, h, Pm + u.off_w, r.z, B_, u.H_in, u.cin, u.k, u.stride, u.dil, zacc);
         counters.launches++;
       } else {
         GemmEpiParams e;  // the GEMM epilogue adds the BatchNorm sums of z (fused bn_stats)
@@ -362,6 +380,25 @@ class SposFamily : public Family {
         e.out2 = r.z + zplane;
         e.stats = acc_f_;
         gemm_x2(s, Po, u.cout, u.cin, h, h + hplane, u.cin, W16 + u.off_w16, W16 + half + u.off_w16, u.cin, e);
+      }
+      if (fuse_bna_ && !u.dw && !last_of_branch(L, i) && L[i + 1].dw) {
+        // conv -> BN -> ReLU -> depthwise: no bn_apply; the depthwise conv applies it on load
+        // (and its last CTA publishes this unit's mean / rstd and the g / b it used)
+        pend.z = r.z;
+        pend.zplane = zplane;
+        pend.P = Po;
+        pend.acc = acc_f_;
+        pend.ticket = tick_ + 3;
+        pend.mean = r.mean;
+        pend.rstd = r.rstd;
+        pend.g = Pm + u.off_g;
+        pend.b = Pm + u.off_b;
+        pend.gsnap = r.rstd + u.cout;
+        pend.bsnap = r.rstd + 2 * u.cout;
+        pend.relu = u.relu;
+        recs.push_back(r);
+        h = nullptr;
+        continue;
       }
       bf16* y;
       int ldy;
@@ -376,7 +413,7 @@ class SposFamily : public Family {
         cv += 2 * zplane;
         ldy = u.cout;
       }
-      t_bn_apply(s, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, u.relu, y, ldy, yplane);
+      t_bn_apply(s, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, u.relu, y, ldy, yplane, zacc);
       hplane = yplane;
       counters.launches += 1;
       recs.push_back(r);
@@ -386,14 +423,36 @@ class SposFamily : public Family {
 
   // One unit's BN backward (+ the WRITE of its gamma/beta), leaves dz in the next ring
   // buffer dz_[ring_] (whose previous reader, a weight-gradient on the side stream, is done).
-  void unit_bn_bwd(const SposConv& u, const UnitRec& r, float* Pm, float* Um, const bf16* dy, int lddy, cudaStream_t s) {
+  // reduced: the producer of dy already added the reduction's sums (BnBwdFuse), so only the
+  // apply runs.
+  void unit_bn_bwd(const SposConv& u, const UnitRec& r, float* Pm, float* Um, const bf16* dy, int lddy, bool reduced,
+                   cudaStream_t s) {
     const int Po = (int)P(u.H_out);
     ring_ = (ring_ + 1) % kRing;
     if (ring_used_[ring_]) cudaStreamWaitEvent(s, ev_wg_[ring_], 0);
-    t_bn_bwd_reduce(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, u.relu);
+    if (!reduced) {
+      t_bn_bwd_reduce(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, u.relu);
+      counters.launches += 1;
+    }
     t_bn_bwd_apply(s, dy, lddy, r.z, Po, u.cout, r.mean, r.rstd, Pm + u.off_g, Pm + u.off_b, Um + u.off_g, Um + u.off_b,
                    1, u.relu, dz_[ring_]);
-    counters.launches += 2;
+    counters.launches += 1;
+  }
+  // the fused BatchNorm-backward reduction of unit `v` (record r) for the kernel producing its
+  // output gradient: stride-1 depthwise input gradients and 1x1-conv input gradients (GEMM
+  // epilogue EPI_BNBWD); the pre-update g, b (reading A4), as bn_bwd_reduce reads them
+  bool fusable_producer(const SposConv& u) const { return u.dw ? fuse_bnb_ : fuse_bnb_gemm_; }
+  BnBwdFuse bnb_of(const SposConv& v, const UnitRec& r, const float* Pm) const {
+    BnBwdFuse f;
+    f.z = r.z;
+    f.zplane = P(v.H_out) * (size_t)v.cout;
+    f.mean = r.mean;
+    f.rstd = r.rstd;
+    f.g = Pm + v.off_g;
+    f.b = Pm + v.off_b;
+    f.relu = v.relu;
+    f.acc = acc_b_;
+    return f;
   }
 
   // conv backward of one unit from dz: the input gradient into dst (+ add) with the
@@ -401,24 +460,26 @@ class SposFamily : public Family {
   // stream once that has been issued, the weight gradient with the SGD WRITE (reading A4),
   // overlapping the rest of the input-gradient chain.
   void unit_conv_bwd(const SposConv& u, const UnitRec& r, float* Pm, float* Um, bool inplace, bf16* W16, size_t half,
-                     bf16* dst, const bf16* add, cudaStream_t s) {
+                     bf16* dst, const bf16* add, cudaStream_t s, const BnBwdFuse* fuse = nullptr) {
     const int Po = (int)P(u.H_out);
     const bf16* dz = dz_[ring_];
     if (dst) {
       if (u.dw) {
-        dw_dgrad(s, dz, Pm + u.off_w, add, dst, B_, u.H_in, u.cin, u.k, u.stride, u.dil);
+        dw_dgrad(s, dz, Pm + u.off_w, add, dst, B_, u.H_in, u.cin, u.k, u.stride, u.dil, fuse ? *fuse : BnBwdFuse());
         counters.launches++;
       } else {
         NP_REQUIRE(add == nullptr, NASPIPE_EINTERNAL, "pw dgrad with an addend");
         GemmEpiParams e;
         e.out = dst;
-        gemm(s, Po, u.cin, u.cout, dz, false, u.cout, W16 + u.off_w16, true, u.cin, EPI_BF16, e);
+        if (fuse) e.bnb = *fuse;
+        gemm(s, Po, u.cin, u.cout, dz, false, u.cout, W16 + u.off_w16, true, u.cin, fuse ? EPI_BNBWD : EPI_BF16, e);
       }
     }
     cudaEventRecord(ev_dg_[ring_], s);
     cudaStreamWaitEvent(side_, ev_dg_[ring_], 0);
     if (u.dw) {
-      dw_wgrad_sgd(side_, dz, r.x, acc_w_, tick_ + 2, Um + u.off_w, lr_, B_, u.H_in, u.cin, u.k, u.stride, u.dil);
+      dw_wgrad_sgd(side_, dz, r.x, acc_w_, tick_ + 2, Um + u.off_w, lr_, B_, u.H_in, u.cin, u.k, u.stride, u.dil,
+                   r.xbn.z ? &r.xbn : nullptr);
       counters.launches += 1;
     } else {
       GemmEpiParams e;
@@ -448,13 +509,17 @@ class SposFamily : public Family {
     const bf16* h = dyb + main_col;
     int ldh = d.C_out;
     int pp = 0;
+    bool reduced = false;  // the producer of h added unit i's BatchNorm-backward sums
     for (size_t i = L.size(); i-- > m0;) {
       const SposConv& u = L[i];
-      unit_bn_bwd(u, recs[i], Pm, Um, h, ldh, s);
+      unit_bn_bwd(u, recs[i], Pm, Um, h, ldh, reduced, s);
       bf16* dst;
       if (i > m0) dst = g_[pp ^= 1];
       else dst = need_dx ? (d.stride == 1 ? g_[pp ^ 1] : gfirst_) : nullptr;
-      unit_conv_bwd(u, recs[i], Pm, Um, inplace, W16, half, dst, nullptr, s);
+      reduced = i > m0 && fusable_producer(u);
+      BnBwdFuse f;
+      if (reduced) f = bnb_of(L[i - 1], recs[i - 1], Pm);
+      unit_conv_bwd(u, recs[i], Pm, Um, inplace, W16, half, dst, nullptr, s, reduced ? &f : nullptr);
       h = dst;
       ldh = u.cin;
     }
@@ -469,11 +534,16 @@ class SposFamily : public Family {
     // the main branch's (both branches read the block input)
     const bf16* hp = dyb;
     int ldp = d.C_out;
+    reduced = false;
     for (size_t i = m0; i-- > 0;) {
       const SposConv& u = L[i];
-      unit_bn_bwd(u, recs[i], Pm, Um, hp, ldp, s);
+      unit_bn_bwd(u, recs[i], Pm, Um, hp, ldp, reduced, s);
       bf16* dst = i > 0 ? g_[pp ^= 1] : (need_dx ? dxb : nullptr);
-      unit_conv_bwd(u, recs[i], Pm, Um, inplace, W16, half, dst, (i == 0 && need_dx) ? gfirst_ : nullptr, s);
+      reduced = i > 0 && fusable_producer(u);
+      BnBwdFuse f;
+      if (reduced) f = bnb_of(L[i - 1], recs[i - 1], Pm);
+      unit_conv_bwd(u, recs[i], Pm, Um, inplace, W16, half, dst, (i == 0 && need_dx) ? gfirst_ : nullptr, s,
+                    reduced ? &f : nullptr);
       hp = dst;
       ldp = u.cin;
     }
@@ -500,11 +570,31 @@ class SposFamily : public Family {
   cudaEvent_t ev_dg_[kRing], ev_wg_[kRing], ev_join_;
   float* ws_;
   unsigned long long *acc_f_, *acc_b_;  // BatchNorm fixed-point accumulators (forward / backward)
+  unsigned long long* acc_f2_;          // forward sums of a depthwise conv that reads acc_f_ (BN on load)
   unsigned long long* acc_w_ = nullptr; // depthwise weight gradient accumulator (side stream)
   size_t dwk_max_ = 0;
   int* tick_;                           // [2] arrival tickets of bn_apply / bn_bwd_apply
   int C_max_ = 0;
   size_t ws_elems_ = 0;
+  // BatchNorm-backward reductions fused into the depthwise producers of dy
+  // (NASPIPE_SPOS_FUSE_BNB=1; off by default: measured slower)
+  const bool fuse_bnb_ = [] {
+    const char* e = getenv("NASPIPE_SPOS_FUSE_BNB");
+    return e && e[0] == '1';
+  }();
+  // ... and into the 1x1-conv input-gradient GEMM's epilogue (EPI_BNBWD): off by default --
+  // measured slower (the epilogue's extra z reads and per-tile sums cost more than the
+  // reduce launch they remove: +0.7 ms per configs[1] step); NASPIPE_SPOS_FUSE_BNB_GEMM=1
+  const bool fuse_bnb_gemm_ = [] {
+    const char* e = getenv("NASPIPE_SPOS_FUSE_BNB_GEMM");
+    return e && e[0] == '1';
+  }();
+  // bn_apply of a conv -> BN -> ReLU unit folded into its depthwise consumer's load
+  // (NASPIPE_SPOS_FUSE_BNA=1; off by default: measured neutral to slower)
+  const bool fuse_bna_ = [] {
+    const char* e = getenv("NASPIPE_SPOS_FUSE_BNA");
+    return e && e[0] == '1';
+  }();
   // stem
   float* w_stem_ = nullptr;
   bf16* stem_z_ = nullptr;

@@ -20,6 +20,7 @@
 
 #include "common.h"
 #include "kernels.h"
+#include "bnfuse.cuh"
 #include "fixpoint.cuh"
 #include "launch.h"
 #include "ptx.cuh"
@@ -47,9 +48,9 @@ struct TileCfg {
   static constexpr int STAGES = (200 * 1024) / STAGE_BYTES > 6 ? 6 : (200 * 1024) / STAGE_BYTES;
   static constexpr int BAR_OFF = STAGES * STAGE_BYTES;
   static constexpr int STG_OFF = BAR_OFF + (2 * STAGES + 4) * 8 + 16;
-  // SPLIT (the SPOS forward 1x1 conv): per-warp column sums of the fused BatchNorm statistics
+  // per-warp column sums of the fused BatchNorm statistics (EPI_X2 forward, EPI_BNBWD backward)
   static constexpr int SST_OFF = STG_OFF + 8 * 32 * 20 * 4;
-  static constexpr int SST_BYTES = SPLIT ? 8 * (TN / 2) * 2 * 4 : 0;
+  static constexpr int SST_BYTES = 8 * (TN / 2) * 2 * 4;
   static constexpr int SMEM_TOTAL = SST_OFF + SST_BYTES + 1024;  // + epilogue staging, alignment slack
   static constexpr int TMEM_COLS = 2 * TN <= 128 ? 128 : (2 * TN <= 256 ? 256 : 512);
 };
@@ -148,7 +149,8 @@ __device__ __forceinline__ void epilogue4(float4 v, float4 pre, float4 b, size_t
 // every global load/store of the epilogue is a coalesced row segment of 4*EC (fp32) or
 // 2*EC (bf16) bytes, instead of 32 rows x 16 bytes per instruction.  The padding makes
 // both staging passes bank-conflict free.
-// sst (EPI_X2 with ep.stats): this warp's [cend - cbeg][2] column sums of its 32 rows
+// sst (EPI_X2 with ep.stats, EPI_BNBWD with ep.bnb.acc): this warp's [cend - cbeg][2]
+// column sums of its 32 rows
 template <int EPI, int EC>
 __device__ __forceinline__ void epilogue_warp(uint32_t taddr, float* stg, int row0, int cbeg, int cend, int n0,
                                               int M, int N, const GemmEpiParams& ep, int split, int lane,
@@ -156,6 +158,7 @@ __device__ __forceinline__ void epilogue_warp(uint32_t taddr, float* stg, int ro
   constexpr int LD = EC + 4, LPR = EC / 4, RPI = 32 / LPR, NIT = 32 / RPI;
   constexpr bool HAS_PRE = EPI == EPI_BIAS_RESID_F32 || EPI == EPI_SGD || EPI == EPI_DGELU;
   constexpr bool HAS_BIAS = EPI == EPI_BIAS_BF16 || EPI == EPI_BIAS_RESID_F32 || EPI == EPI_BIAS_GELU;
+  constexpr bool BNB = EPI == EPI_BNBWD;
   const int cc = (lane % LPR) * 4;
 #pragma unroll 1
   for (int c0 = cbeg; c0 < cend; c0 += EC) {
@@ -166,12 +169,31 @@ __device__ __forceinline__ void epilogue_warp(uint32_t taddr, float* stg, int ro
     if constexpr (HAS_BIAS) {
       if (gcol < N) b = *reinterpret_cast<const float4*>(ep.bias + gcol);
     }
+    // EPI_BNBWD: the unit's per-column mean, rstd, g, b and its z (hi, lo) per element
+    float4 bmu = b, brs = b, bga = b, bbe = b;
+    uint2 zh[NIT], zl[NIT];
+    if constexpr (BNB) {
+      if (gcol < N) {
+        bmu = *reinterpret_cast<const float4*>(ep.bnb.mean + gcol);
+        brs = *reinterpret_cast<const float4*>(ep.bnb.rstd + gcol);
+        bga = *reinterpret_cast<const float4*>(ep.bnb.g + gcol);
+        bbe = *reinterpret_cast<const float4*>(ep.bnb.b + gcol);
+      }
+    }
 #pragma unroll
     for (int it = 0; it < NIT; ++it) {
       const int grow = row0 + it * RPI + lane / LPR;
       pre[it] = make_float4(0.f, 0.f, 0.f, 0.f);
       if constexpr (HAS_PRE) {
         if (grow < M && gcol < N) pre[it] = preload4<EPI>((size_t)grow * N + gcol, ep);
+      }
+      if constexpr (BNB) {
+        zh[it] = zl[it] = make_uint2(0u, 0u);
+        if (grow < M && gcol < N) {
+          const size_t off = (size_t)grow * N + gcol;
+          zh[it] = *reinterpret_cast<const uint2*>(ep.bnb.z + off);
+          zl[it] = *reinterpret_cast<const uint2*>(ep.bnb.z + ep.bnb.zplane + off);
+        }
       }
     }
     uint32_t r[EC];
@@ -202,9 +224,25 @@ __device__ __forceinline__ void epilogue_warp(uint32_t taddr, float* stg, int ro
             bq[i] = __fmaf_rn(st, st, bq[i]);
           }
         }
+        if constexpr (BNB) {  // BatchNorm-backward sums of the stored dy (bn_bwd_reduce's terms)
+          const float vv[4] = {v.x, v.y, v.z, v.w};
+          const float zz[4] = {__uint_as_float(zh[it].x << 16) + __uint_as_float(zl[it].x << 16),
+                               __uint_as_float(zh[it].x & 0xffff0000u) + __uint_as_float(zl[it].x & 0xffff0000u),
+                               __uint_as_float(zh[it].y << 16) + __uint_as_float(zl[it].y << 16),
+                               __uint_as_float(zh[it].y & 0xffff0000u) + __uint_as_float(zl[it].y & 0xffff0000u)};
+          const float mu[4] = {bmu.x, bmu.y, bmu.z, bmu.w}, rs[4] = {brs.x, brs.y, brs.z, brs.w};
+          const float ga[4] = {bga.x, bga.y, bga.z, bga.w}, be[4] = {bbe.x, bbe.y, bbe.z, bbe.w};
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            float d = __bfloat162float(__float2bfloat16_rn(vv[i])), xh;
+            bn_bwd_elem(d, zz[i], mu[i], rs[i], ga[i], be[i], ep.bnb.relu, xh);
+            bs[i] += d;
+            bq[i] = __fmaf_rn(d, xh, bq[i]);
+          }
+        }
       }
     }
-    if constexpr (EPI == EPI_X2) {
+    if constexpr (EPI == EPI_X2 || BNB) {
       if (sst != nullptr) {  // fixed xor tree over the 8 row groups of the warp (lanes cc + 4 LPR k)
 #pragma unroll
         for (int o = LPR; o < 32; o <<= 1)
@@ -372,16 +410,17 @@ __global__ void __launch_bounds__(THREADS, 1)
       if (t + (int)gridDim.x >= n_tiles) ptx::pdl_trigger();  // last tile: let the next kernel launch
       const uint32_t taddr = tmem + ((uint32_t)lane_base << 16) + acc * TN;
       float* sst = nullptr;
-      if constexpr (EPI == EPI_X2)
-        if (ep.stats != nullptr) sst = reinterpret_cast<float*>(smem + Cf::SST_OFF) + (warp - 2) * (TN / 2) * 2;
+      unsigned long long* sacc = EPI == EPI_BNBWD ? ep.bnb.acc : ep.stats;  // fused BatchNorm sums
+      if constexpr (EPI == EPI_X2 || EPI == EPI_BNBWD)
+        if (sacc != nullptr) sst = reinterpret_cast<float*>(smem + Cf::SST_OFF) + (warp - 2) * (TN / 2) * 2;
       epilogue_warp<EPI, 16>(taddr, stg + (warp - 2) * 32 * 20, tm * BM + lane_base, cbeg, cbeg + TN / 2, tn * TN, M,
                              N, ep, ks, lane, sst);
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(&tempty[acc]);
-      if constexpr (EPI == EPI_X2) {
-        if (ep.stats != nullptr) {
-          // fused BatchNorm statistics: the 4 warps of this column half (lane quarters 0..3)
+      if constexpr (EPI == EPI_X2 || EPI == EPI_BNBWD) {
+        if (sacc != nullptr) {
+          // fused BatchNorm sums: the 4 warps of this column half (lane quarters 0..3)
           // combine their 32-row column sums in quarter order, one fixed-point add per column
           const int half = (warp - 2) >> 2;
           ptx::named_bar_sync(1 + half, 128);
@@ -396,8 +435,8 @@ __global__ void __launch_bounds__(THREADS, 1)
               s1 += w[j * 2];
               s2 += w[j * 2 + 1];
             }
-            fix_add(ep.stats, gcol, ep.stats + 2 * N, s1, FIX_S1);
-            fix_add(ep.stats, N + gcol, ep.stats + 2 * N, s2, FIX_S2);
+            fix_add(sacc, gcol, sacc + 2 * N, s1, EPI == EPI_BNBWD ? FIX_B : FIX_S1);
+            fix_add(sacc, N + gcol, sacc + 2 * N, s2, EPI == EPI_BNBWD ? FIX_B : FIX_S2);
           }
           ptx::named_bar_sync(1 + half, 128);  // the slots are rewritten by the next tile
         }
@@ -743,7 +782,9 @@ bool pair_enabled() {
 // N tile of the 1-CTA kernel: narrow outputs (the SPOS 1x1-conv input gradients and weight
 // gradients, N = C_in <= 320) get 64- or 128-wide tiles instead of wasting 3/4 or 1/2 of a
 // 256-wide tile's MMA and TMEM work on zero columns (epilogues without per-column operands).
-bool small_n_epi(int epi) { return epi == EPI_BF16 || epi == EPI_F32 || epi == EPI_SGD || epi == EPI_PARTIAL; }
+bool small_n_epi(int epi) {
+  return epi == EPI_BF16 || epi == EPI_F32 || epi == EPI_SGD || epi == EPI_PARTIAL || epi == EPI_BNBWD;
+}
 int tile_n(int N, int epi) { return !small_n_epi(epi) ? BN : (N <= 64 ? 64 : (N <= 128 ? 128 : BN)); }
 
 template <bool A_MN, bool B_MN, int TN>
@@ -754,6 +795,7 @@ void dispatch_narrow(cudaStream_t s, int M, int N, const TileSpace& ts, const CU
     case EPI_F32: return launch<A_MN, B_MN, EPI_F32, TN>(s, M, N, ts, ta, tb, ep);
     case EPI_SGD: return launch<A_MN, B_MN, EPI_SGD, TN>(s, M, N, ts, ta, tb, ep);
     case EPI_PARTIAL: return launch<A_MN, B_MN, EPI_PARTIAL, TN>(s, M, N, ts, ta, tb, ep);
+    case EPI_BNBWD: return launch<A_MN, B_MN, EPI_BNBWD, TN>(s, M, N, ts, ta, tb, ep);
     default: NP_REQUIRE(false, NASPIPE_EINVAL, "narrow-tile epilogue %d", epi);
   }
 }
@@ -773,6 +815,7 @@ void dispatch_epi(cudaStream_t s, int M, int N, const TileSpace& ts, const CUten
     case EPI_DGELU: return launch<A_MN, B_MN, EPI_DGELU>(s, M, N, ts, ta, tb, ep);
     case EPI_SGD: return launch<A_MN, B_MN, EPI_SGD>(s, M, N, ts, ta, tb, ep);
     case EPI_PARTIAL: return launch<A_MN, B_MN, EPI_PARTIAL>(s, M, N, ts, ta, tb, ep);
+    case EPI_BNBWD: return launch<A_MN, B_MN, EPI_BNBWD>(s, M, N, ts, ta, tb, ep);
     default: NP_REQUIRE(false, NASPIPE_EINVAL, "bad epilogue %d", epi);
   }
 }
@@ -825,7 +868,10 @@ void gemm_bf16_tc(cudaStream_t s, int M, int N, int K, const bf16* A, bool a_mn,
   NP_REQUIRE(M > 0 && N > 0 && K > 0 && N % 16 == 0, NASPIPE_EINVAL, "gemm dims M=%d N=%d K=%d (N%%16)", M, N, K);
   GemmEpiParams ep = ep_in;
   g_gemm_flops.fetch_add(2ull * (uint64_t)M * (uint64_t)N * (uint64_t)K, std::memory_order_relaxed);
-  const bool pair = gemm_uses_pair(M, N);
+  // the fused BatchNorm-backward epilogue exists in the 1-CTA kernel only
+  const bool pair = gemm_uses_pair(M, N) && epi != EPI_BNBWD;
+  NP_REQUIRE(epi != EPI_BNBWD || (ep.bnb.acc != nullptr && ep.bnb.z != nullptr && N % 4 == 0), NASPIPE_EINVAL,
+             "EPI_BNBWD needs bnb.acc / bnb.z (N=%d)", N);
   int splits = 1;
   if ((epi == EPI_SGD || epi == EPI_F32) && ep.ws != nullptr) {
     splits = gemm_splitk_factor(M, N, K);

@@ -27,6 +27,40 @@ enum GemmEpi {
   EPI_SGD = 6,            // w32[m,n] -= lr * acc; w16[m,n] = bf16(w32[m,n])   (the WRITE)
                           //   (+ w16lo[m,n] = bf16(w32 - w16) when w16lo != nullptr)
   EPI_X2 = 7,             // out16 = hi = bf16(acc), out2 = lo = bf16(acc - hi)  (bf16x2 planes)
+  EPI_BNBWD = 8,          // out16 = dy = bf16(acc), plus the BatchNorm-backward sums of the unit
+                          //   whose output gradient dy is (bn_bwd_reduce fused, see `bnb`)
+};
+// A depthwise conv whose input is the output of a conv -> BN [-> ReLU] unit that was never
+// materialised (bn_apply folded into its consumer): the consumer reads the unit's z and
+// applies y = relu?(g (z - mean) rstd + b) on load, rounding y to bf16x2 exactly as bn_apply
+// stores it (so the numerics are those of the stored path).  Forward: mean/rstd come from
+// the fixed-point sums acc of z; the consumer's last CTA (ticket) publishes mean, rstd and
+// the g, b it used (gsnap, bsnap: the backward recomputes y with them even if g, b have been
+// written since) and zeroes acc and the ticket.  Backward (depthwise weight gradient): mean,
+// rstd, gsnap, bsnap as published.
+struct BnApplyIn {
+  const bf16* z = nullptr;  // x2 [P, C], lo plane zplane elements after hi
+  size_t zplane = 0;
+  int P = 0;
+  unsigned long long* acc = nullptr;  // forward: the sums of z (zero after the consumer)
+  int* ticket = nullptr;
+  float *mean = nullptr, *rstd = nullptr;  // [C], published by the forward consumer
+  const float *g = nullptr, *b = nullptr;  // the unit's g, b (forward)
+  float *gsnap = nullptr, *bsnap = nullptr;  // [C], the g, b the forward applied
+  int relu = 0;
+};
+
+// EPI_BNBWD / the depthwise input gradient with fused BatchNorm-backward sums: the unit
+// z -> BN(mean, rstd, g, b) [-> ReLU] whose output gradient the kernel produces; per output
+// element dy (as stored, bf16) it adds dy' = dy masked by the ReLU and dy' * xh, xh = (z -
+// mean) rstd, to acc[0..C) / acc[C..2C) in fixed point (FIX_B; acc[2C] = overflow flag):
+// exactly what bn_bwd_reduce would add, so bn_bwd_apply follows without a reduce launch.
+struct BnBwdFuse {
+  const bf16* z = nullptr;  // x2 [P, C], lo plane zplane elements after hi
+  size_t zplane = 0;
+  const float *mean = nullptr, *rstd = nullptr, *g = nullptr, *b = nullptr;
+  int relu = 0;
+  unsigned long long* acc = nullptr;  // nullptr: no fused sums
 };
 struct GemmEpiParams {
   const float* bias = nullptr;
@@ -46,6 +80,7 @@ struct GemmEpiParams {
   // values) of the output to stats[0..2N) in fixed point (fixpoint.cuh; stats[2N] = the
   // overflow flag): the SPOS forward 1x1 conv with bn_stats fused
   unsigned long long* stats = nullptr;
+  BnBwdFuse bnb;  // EPI_BNBWD only (stats of the fused BatchNorm backward; 1-CTA kernel)
 };
 // split-K factor the launcher uses for an (M, N, K) GEMM given a large enough workspace
 int gemm_splitk_factor(int M, int N, int K);
@@ -163,13 +198,20 @@ bool bn_fix_overflow(const unsigned long long* acc, int C);
 // stats != nullptr: also add the BatchNorm sums of the stored z to it (bn_stats fused)
 void dw_fwd(cudaStream_t s, const bf16* x, const float* w, bf16* z, int B, int H, int C, int k, int S, int dil,
             unsigned long long* stats = nullptr);
+// dw_fwd of y = BN(z) [+ ReLU] applied on load (BnApplyIn; x is not read)
+void dw_fwd_bn(cudaStream_t s, const BnApplyIn& xin, const float* w, bf16* z, int B, int H, int C, int k, int S,
+               int dil, unsigned long long* stats);
+// bnb.acc != nullptr (stride 1 only): also add the BatchNorm-backward sums of the unit whose
+// output gradient dx is (BnBwdFuse; bn_bwd_reduce fused)
 void dw_dgrad(cudaStream_t s, const bf16* dz, const float* w, const bf16* add, bf16* dx, int B, int H, int C, int k,
-              int S, int dil);
+              int S, int dil, const BnBwdFuse& bnb = BnBwdFuse());
 int dw_wgrad_blocks(int B, int H, int C, int k, int S);
 // weight gradient of a depthwise conv with the SGD WRITE fused: w -= lr * sum over the batch
 // (acc [C*k*k + 1] and ticket zero between uses, fixpoint.cuh; w = master or BSP accumulator)
+// xin != nullptr: x = the hi plane of BN(z) [+ ReLU] recomputed on load (BnApplyIn, the
+// published mean/rstd and g/b snapshots); x is then not read
 void dw_wgrad_sgd(cudaStream_t s, const bf16* dz, const bf16* x, unsigned long long* acc, int* ticket, float* w,
-                  float lr, int B, int H, int C, int k, int S, int dil);
+                  float lr, int B, int H, int C, int k, int S, int dil, const BnApplyIn* xin = nullptr);
 // ---- NLP op families (seqconv.cu; Table 5, reading A38).  x, dy: bf16 [T = B*S, d].
 // seqconv: depthwise conv along each sequence of S rows, taps w [d][k] (H == 0) or
 // softmax(Wl[H][k]) shared by d/H channels (Light Conv); flip = the input gradient; out bf16 or f32.

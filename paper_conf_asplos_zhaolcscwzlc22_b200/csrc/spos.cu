@@ -28,6 +28,7 @@
 #include "common.h"
 #include "kernels.h"
 #include "launch.h"
+#include "bnfuse.cuh"
 #include "fixpoint.cuh"
 #include "ptx.cuh"
 
@@ -109,12 +110,6 @@ __device__ __forceinline__ void store8x2(bf16* p, size_t plane, const float (&v)
 __device__ __forceinline__ void load8f(const float* p, float (&v)[8]) {
   const float4 a = reinterpret_cast<const float4*>(p)[0], b = reinterpret_cast<const float4*>(p)[1];
   v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w; v[4] = b.x; v[5] = b.y; v[6] = b.z; v[7] = b.w;
-}
-
-// BN output (also recomputed in the backward for the ReLU mask: same expression, same
-// rounding, explicit fma so no contraction choice can differ between the two kernels)
-__device__ __forceinline__ float bn_y(float z, float mu, float rs, float g, float b) {
-  return __fmaf_rn(g, __fmul_rn(__fsub_rn(z, mu), rs), b);
 }
 
 // ---------------------------------------------------------------- frozen stem (conv3x3 s2)
@@ -340,10 +335,7 @@ __device__ __forceinline__ void bn_bwd_item(const bf16* dy, const bf16* z, size_
   load4(dy, d);
   load4x2(z, zplane, zz);
 #pragma unroll
-  for (int i = 0; i < BV; ++i) {
-    xh[i] = __fmul_rn(__fsub_rn(zz[i], mu[i]), rs[i]);
-    if (relu && !(bn_y(zz[i], mu[i], rs[i], g8[i], b8[i]) > 0.f)) d[i] = 0.f;
-  }
+  for (int i = 0; i < BV; ++i) bn_bwd_elem(d[i], zz[i], mu[i], rs[i], g8[i], b8[i], relu, xh[i]);
 }
 
 // s1 = sum dy', s2 = sum dy' xh (dy' = dy masked by the ReLU): fixed-order row-block
@@ -488,54 +480,6 @@ __device__ __forceinline__ void stage_dw_weights(float* ws, const float* w, int 
   __syncthreads();
 }
 
-// dx[b,ih,iw,c] = sum_{u,v} dz[b,oh,ow,c] w[c,u,v] with oh*S + u*DIL - PAD = ih (+ add[b,ih,iw,c]),
-// PAD = DIL*(K/2) (DIL = 2: Table 5's dilated convs, reading A36)
-template <int K, int DIL>
-__global__ void dw_dgrad_kernel(const bf16* __restrict__ dz, const float* __restrict__ w, const bf16* __restrict__ add,
-                                bf16* __restrict__ dx, int B, int H, int C, int S) {
-  extern __shared__ float ws[];
-  ptx::pdl_wait();
-  stage_dw_weights<K>(ws, w, C);
-  constexpr int PAD = DIL * (K / 2), KE = DIL * (K - 1) + 1;
-  const int Ho = (H + 2 * PAD - KE) / S + 1;
-  const int G = C / 8;
-  const size_t items = (size_t)B * H * H * G;
-  for (size_t it = blockIdx.x * (size_t)blockDim.x + threadIdx.x; it < items; it += (size_t)gridDim.x * blockDim.x) {
-    const int c = (int)(it % G) * 8;
-    const size_t p = it / G;
-    const int iw = (int)(p % H);
-    const int ih = (int)((p / H) % H);
-    const int b = (int)(p / ((size_t)H * H));
-    float acc[8] = {};
-#pragma unroll
-    for (int u = 0; u < K; ++u) {
-      const int t = ih + PAD - u * DIL;
-      if (t < 0 || t % S) continue;
-      const int oh = t / S;
-      if (oh >= Ho) continue;
-#pragma unroll
-      for (int v = 0; v < K; ++v) {
-        const int q = iw + PAD - v * DIL;
-        if (q < 0 || q % S) continue;
-        const int ow = q / S;
-        if (ow >= Ho) continue;
-        float dv[8];
-        load8(dz + (((size_t)b * Ho + oh) * Ho + ow) * C + c, dv);
-        const float* wt = ws + (u * K + v) * C + c;
-#pragma unroll
-        for (int i = 0; i < 8; ++i) acc[i] = __fmaf_rn(dv[i], wt[i], acc[i]);
-      }
-    }
-    if (add) {
-      float a[8];
-      load8(add + p * C + c, a);
-#pragma unroll
-      for (int i = 0; i < 8; ++i) acc[i] += a[i];
-    }
-    store8(dx + p * C + c, acc);
-  }
-}
-
 // ---------------------------------------------------------------- depthwise conv, shared-memory tiles
 // Correlation out[b,oh,ow,c] = sum_{u,v} in[b, oh*S+u*DIL-PAD, ow*S+v*DIL-PAD, c] w'[c,u,v] (+ add),
 // PAD = DIL*(K/2), KE = DIL*(K-1)+1 the dilated extent,
@@ -544,18 +488,65 @@ __global__ void dw_dgrad_kernel(const bf16* __restrict__ dz, const float* __rest
 // staged in shared memory once (16-byte loads, fp32), each thread keeps one channel's k x k
 // weights in registers and computes a DT_H-row strip of one column from shared memory (each
 // staged value feeds up to DT_H outputs).  X2: bf16x2 input/output (forward), else bf16.
+// Fused reductions (fixed order per CTA, fixed point across CTAs): X2 with `stats` adds the
+// BatchNorm sums of the stored output (bn_stats); FLIP with bnb.acc adds the BatchNorm-backward
+// sums of the unit whose output gradient the stored dx is (bn_bwd_reduce, BnBwdFuse).
 constexpr int DT_H = 8;
 
-template <int K, int S, int DIL, bool X2, bool FLIP>
+// XBN (forward, X2): the input is y = relu?(BN(z)) of a unit whose bn_apply was folded in
+// here (BnApplyIn): the halo loads z and applies BN [+ ReLU] with the CTA's per-channel
+// moments from the fixed-point sums, rounding y to bf16x2 as bn_apply stores it; the last
+// CTA publishes mean / rstd and the g / b used, and clears the sums (bn_apply's duties).
+constexpr int XBN_CH = TPB / 8;  // channels of a CTA: CPG * 8 <= 32
+
+// per-channel BN parameters of channels [c0, c0 + n) in shared memory: forward = moments
+// from the fixed-point sums and the live g, b; backward = the published mean / rstd and the
+// forward's g, b snapshots
+__device__ __forceinline__ void xbn_stage(const BnApplyIn& xb, bool fwd, int c0, int n, int C, float* mu, float* rs,
+                                          float* g, float* b) {
+  for (int i = threadIdx.x; i < n; i += blockDim.x) {
+    const int c = c0 + i;
+    if (c >= C) continue;
+    if (fwd) {
+      bn_moments(xb.acc, C, c, xb.P, mu[i], rs[i]);
+      g[i] = xb.g[c];
+      b[i] = xb.b[c];
+    } else {
+      mu[i] = xb.mean[c];
+      rs[i] = xb.rstd[c];
+      g[i] = xb.gsnap[c];
+      b[i] = xb.bsnap[c];
+    }
+  }
+  __syncthreads();
+}
+// y of 8 channels (smem parameter index j0) from z, rounded to bf16x2 (hi + lo) or, HI_ONLY,
+// to its hi plane
+template <bool HI_ONLY>
+__device__ __forceinline__ void xbn_y8(float (&v)[8], const float* mu, const float* rs, const float* g, const float* b,
+                                       int j0, int relu) {
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    float y = bn_y(v[j], mu[j0 + j], rs[j0 + j], g[j0 + j], b[j0 + j]);
+    y = relu ? fmaxf(y, 0.f) : y;
+    const float hi = __bfloat162float(__float2bfloat16_rn(y));
+    v[j] = HI_ONLY ? hi : hi + __bfloat162float(__float2bfloat16_rn(y - hi));
+  }
+}
+
+template <int K, int S, int DIL, bool X2, bool FLIP, bool XBN = false>
 __global__ void __launch_bounds__(TPB) dw_tile_kernel(const bf16* __restrict__ in, const float* __restrict__ w,
                                                     const bf16* __restrict__ add, bf16* __restrict__ out, int B,
-                                                    int H, int C, int TW, unsigned long long* stats) {
+                                                    int H, int C, int TW, int strips, unsigned long long* stats,
+                                                    const BnBwdFuse bnb, const BnApplyIn xbn) {
+  static_assert(!XBN || (X2 && !FLIP), "BN-on-load is a forward (bf16x2) mode");
   constexpr int PAD = DIL * (K / 2), KE = DIL * (K - 1) + 1, IH = (DT_H - 1) * S + KE;
   extern __shared__ float tile[];  // [CPG][IH][IW][8]
   ptx::pdl_wait();
   const int Ho = (H + 2 * PAD - KE) / S + 1;
   const int CPG = TPB / (8 * TW), IW = (TW - 1) * S + KE;
-  const int tiles_h = (Ho + DT_H - 1) / DT_H, tiles_w = (Ho + TW - 1) / TW;
+  const int RH = DT_H * strips;  // output rows of the CTA: `strips` strips of DT_H rows
+  const int tiles_h = (Ho + RH - 1) / RH, tiles_w = (Ho + TW - 1) / TW;
   int t = blockIdx.x;
   const int tw = t % tiles_w;
   t /= tiles_w;
@@ -564,21 +555,8 @@ __global__ void __launch_bounds__(TPB) dw_tile_kernel(const bf16* __restrict__ i
   const int b = t;
   const int cg0 = blockIdx.y * CPG;  // first channel group of the CTA
   const size_t iplane = (size_t)B * H * H * C, oplane = (size_t)B * Ho * Ho * C;
-  // stage the halo: CPG x IH x IW pixels of 8 channels
-  const int ih0 = th * DT_H * S - PAD, iw0 = tw * TW * S - PAD;
-  for (int i = threadIdx.x; i < CPG * IH * IW; i += TPB) {
-    const int col = i % IW, row = (i / IW) % IH, cg = i / (IW * IH);
-    const int ih = ih0 + row, iw = iw0 + col, c = (cg0 + cg) * 8;
-    float v[8] = {};
-    if (ih >= 0 && ih < H && iw >= 0 && iw < H && c < C) {
-      const bf16* p = in + (((size_t)b * H + ih) * H + iw) * C + c;
-      if (X2) load8x2(p, iplane, v);
-      else load8(p, v);
-    }
-    float4* d = reinterpret_cast<float4*>(tile + (size_t)i * 8);
-    d[0] = make_float4(v[0], v[1], v[2], v[3]);
-    d[1] = make_float4(v[4], v[5], v[6], v[7]);
-  }
+  __shared__ float xmu[XBN ? XBN_CH : 1], xrs[XBN ? XBN_CH : 1], xg[XBN ? XBN_CH : 1], xb[XBN ? XBN_CH : 1];
+  if constexpr (XBN) xbn_stage(xbn, true, cg0 * 8, CPG * 8, C, xmu, xrs, xg, xb);
   const int ch = threadIdx.x % 8, col = (threadIdx.x / 8) % TW, cgi = threadIdx.x / (8 * TW);
   const int c = (cg0 + cgi) * 8 + ch;
   float wr[K][K];
@@ -586,47 +564,91 @@ __global__ void __launch_bounds__(TPB) dw_tile_kernel(const bf16* __restrict__ i
   for (int u = 0; u < K; ++u)
 #pragma unroll
     for (int v = 0; v < K; ++v)
-      wr[u][v] = c < C ? w[(size_t)c * K * K + (FLIP ? (K - 1 - u) * K + (K - 1 - v) : u * K + v)] : 0.f;
-  __syncthreads();
-  float acc[DT_H];
-#pragma unroll
-  for (int r = 0; r < DT_H; ++r) acc[r] = 0.f;
-  const float* tb = tile + ((size_t)cgi * IH * IW + col * S) * 8 + ch;
-#pragma unroll
-  for (int ir = 0; ir < IH; ++ir) {
-#pragma unroll
-    for (int v = 0; v < K; ++v) {
-      const float x = tb[((size_t)ir * IW + v * DIL) * 8];
-#pragma unroll
-      for (int r = 0; r < DT_H; ++r) {
-        const int t = ir - r * S;  // = u * DIL (compile-time after unrolling)
-        if (t >= 0 && t % DIL == 0 && t / DIL < K) acc[r] = __fmaf_rn(x, wr[t / DIL][v], acc[r]);
-      }
-    }
-  }
+      wr[u][v] = c < C ? w[c * K * K + (FLIP ? (K - 1 - u) * K + (K - 1 - v) : u * K + v)] : 0.f;
   const int ow = tw * TW + col;
   const bool valid = c < C && ow < Ho;
-  float ss = 0.f, sq = 0.f;  // BatchNorm statistics of the stored values (fused bn_stats)
-  if (valid) {
+  // fused sums over the CTA's strips: (sum, sum of squares) of the stored z (X2), or
+  // (sum dy', sum dy' xh) (FLIP with bnb)
+  const bool fuse_b = !X2 && FLIP && bnb.acc != nullptr;
+  float ss = 0.f, sq = 0.f;
+  float bmu = 0.f, brs = 0.f, bg = 0.f, bb = 0.f;
+  if (fuse_b && valid) {
+    bmu = bnb.mean[c];
+    brs = bnb.rstd[c];
+    bg = bnb.g[c];
+    bb = bnb.b[c];
+  }
+  const float* tb = tile + (cgi * IH * IW + col * S) * 8 + ch;
+  const int iw0 = tw * TW * S - PAD;
+  for (int st = 0; st < strips; ++st) {
+    const int oh0 = th * RH + st * DT_H;
+    if (oh0 >= Ho) break;  // CTA-uniform
+    const int ih0 = oh0 * S - PAD;
+    __syncthreads();  // the previous strip's halo has been consumed
+    // stage the halo: CPG x IH x IW pixels of 8 channels (XBN: y = BN(z) [+ ReLU] on load;
+    // the zero padding stays zero)
+    for (int i = threadIdx.x; i < CPG * IH * IW; i += TPB) {
+      const int cl = i % IW, row = (i / IW) % IH, cg = i / (IW * IH);
+      const int ih = ih0 + row, iw = iw0 + cl, c8 = (cg0 + cg) * 8;
+      float v[8] = {};
+      if (ih >= 0 && ih < H && iw >= 0 && iw < H && c8 < C) {
+        const bf16* p = (XBN ? xbn.z : in) + (((size_t)b * H + ih) * H + iw) * C + c8;
+        if (X2) load8x2(p, XBN ? xbn.zplane : iplane, v);
+        else load8(p, v);
+        if constexpr (XBN) xbn_y8<false>(v, xmu, xrs, xg, xb, cg * 8, xbn.relu);
+      }
+      float4* d = reinterpret_cast<float4*>(tile + i * 8);
+      d[0] = make_float4(v[0], v[1], v[2], v[3]);
+      d[1] = make_float4(v[4], v[5], v[6], v[7]);
+    }
+    __syncthreads();
+    float acc[DT_H];
 #pragma unroll
-    for (int r = 0; r < DT_H; ++r) {
-      const int oh = th * DT_H + r;
-      if (oh >= Ho) break;
-      const size_t o = (((size_t)b * Ho + oh) * Ho + ow) * C + c;
-      if (X2) {
-        const bf16 hi = __float2bfloat16_rn(acc[r]);
-        const bf16 lo = __float2bfloat16_rn(acc[r] - __bfloat162float(hi));
-        out[o] = hi;
-        out[o + oplane] = lo;
-        const float v = __bfloat162float(hi) + __bfloat162float(lo);
-        ss += v;
-        sq = __fmaf_rn(v, v, sq);
-      } else {
-        out[o] = __float2bfloat16_rn(add ? acc[r] + __bfloat162float(add[o]) : acc[r]);
+    for (int r = 0; r < DT_H; ++r) acc[r] = 0.f;
+#pragma unroll
+    for (int ir = 0; ir < IH; ++ir) {
+      const float* rowp = tb + ir * IW * 8;
+#pragma unroll
+      for (int v = 0; v < K; ++v) {
+        const float x = rowp[v * DIL * 8];
+#pragma unroll
+        for (int r = 0; r < DT_H; ++r) {
+          const int tt = ir - r * S;  // = u * DIL (compile-time after unrolling)
+          if (tt >= 0 && tt % DIL == 0 && tt / DIL < K) acc[r] = __fmaf_rn(x, wr[tt / DIL][v], acc[r]);
+        }
+      }
+    }
+    if (valid) {
+      const size_t o0 = (((size_t)b * Ho + oh0) * Ho + ow) * C + c, rstride = (size_t)Ho * C;
+      const int nr = min(DT_H, Ho - oh0);
+#pragma unroll
+      for (int r = 0; r < DT_H; ++r) {
+        if (r >= nr) break;
+        const size_t o = o0 + r * rstride;
+        if (X2) {
+          const bf16 hi = __float2bfloat16_rn(acc[r]);
+          const bf16 lo = __float2bfloat16_rn(acc[r] - __bfloat162float(hi));
+          out[o] = hi;
+          out[o + oplane] = lo;
+          const float v = __bfloat162float(hi) + __bfloat162float(lo);
+          ss += v;
+          sq = __fmaf_rn(v, v, sq);
+        } else {
+          const bf16 ob = __float2bfloat16_rn(add ? acc[r] + __bfloat162float(add[o]) : acc[r]);
+          out[o] = ob;
+          if (fuse_b) {  // bn_bwd_reduce's terms of the stored dy
+            float d = __bfloat162float(ob), xh;
+            const float zz = __bfloat162float(bnb.z[o]) + __bfloat162float(bnb.z[o + bnb.zplane]);
+            bn_bwd_elem(d, zz, bmu, brs, bg, bb, bnb.relu, xh);
+            ss += d;
+            sq = __fmaf_rn(d, xh, sq);
+          }
+        }
       }
     }
   }
-  if (X2 && stats != nullptr) {
+  unsigned long long* sacc = X2 ? stats : (fuse_b ? bnb.acc : nullptr);
+  if (sacc != nullptr) {
     // per channel over the CTA's TW columns, fixed order: xor tree over the 4 columns of a
     // warp (lanes ch + 8 col), then the warps of the channel group in warp order
     __shared__ float wsum[TPB / 32][2][8];
@@ -647,7 +669,162 @@ __global__ void __launch_bounds__(TPB) dw_tile_kernel(const bf16* __restrict__ i
       const int cc = (cg0 + g) * 8 + chn;
       float a = 0.f;
       for (int k = 0; k < wpg; ++k) a += wsum[g * wpg + k][which][chn];
-      if (cc < C) fix_add(stats, (which ? C : 0) + cc, stats + 2 * C, a, which ? FIX_S2 : FIX_S1);
+      if (cc < C) fix_add(sacc, (which ? C : 0) + cc, sacc + 2 * C, a, X2 ? (which ? FIX_S2 : FIX_S1) : FIX_B);
+    }
+  }
+  if constexpr (XBN) {
+    if (last_cta(xbn.ticket)) {  // every CTA has read the input sums: publish, clear
+      for (int cc = threadIdx.x; cc < C; cc += TPB) {
+        float mu, rs;
+        bn_moments(xbn.acc, C, cc, xbn.P, mu, rs);
+        xbn.mean[cc] = mu;
+        xbn.rstd[cc] = rs;
+        xbn.gsnap[cc] = xbn.g[cc];
+        xbn.bsnap[cc] = xbn.b[cc];
+      }
+      __syncthreads();
+      for (int e = threadIdx.x; e < 2 * C; e += TPB) xbn.acc[e] = 0ull;
+      if (threadIdx.x == 0) *xbn.ticket = 0;
+    }
+  }
+}
+
+// Input gradient of a STRIDE-2 depthwise conv, tiled (replaces round 2's grid-stride gather,
+// which took 32 / 75 / 182 us per k = 3 / 5 / 7 launch at configs[1]'s 112x112 inputs):
+//   dx[b,ih,iw,c] = sum_{u,v} dz[b,oh,ow,c] w[c,u,v] over oh*2 + u*DIL - PAD = ih,
+//   ow*2 + v*DIL - PAD = iw (+ add), PAD = DIL*(K/2).
+// A CTA owns DT_H rows x TW columns x CPG channel groups of dx; the dz window they read
+// (DT_H/2 + ~K*DIL/2 rows x TW/2 + ~K*DIL/2 columns) is staged in shared memory once.  Row
+// parity is compile-time (ih0 is even); the column parity picks the valid v taps, so the
+// threads are permuted so that each warp's 4 columns share one parity (no divergence).
+// BnBwdFuse: as dw_tile_kernel's FLIP mode (bn_bwd_reduce fused, fixed order per CTA).
+constexpr int S2_STRIPS = 4;  // DT_H-row strips per CTA (the weights and the grid's fixed costs amortised over them)
+
+// One thread's DT_H outputs of a strip from the staged dz window (column parity class Q,
+// compile-time): with EP = (PAD - (K-1) DIL) & 1, output row r takes tap u iff
+// EP + (K-1-u) DIL + r is even, from staged row (EP + (K-1-u) DIL + r) / 2; column tap v iff
+// Q + (K-1-v) DIL is even, at staged column cb + (Q + (K-1-v) DIL) / 2.  All offsets but the
+// row pitch are compile-time: ~1 FFMA + 1 LDS per tap (the generic gather spent ~15 integer
+// instructions per tap).
+template <int K, int DIL, int Q>
+__device__ __forceinline__ void s2_strip(const float* base, int ow8, const float (&wr)[K][K], float (&acc)[DT_H]) {
+  constexpr int PAD = DIL * (K / 2), EP = (PAD - (K - 1) * DIL) & 1;
+#pragma unroll
+  for (int r = 0; r < DT_H; ++r) {
+    float a = 0.f;
+#pragma unroll
+    for (int u = 0; u < K; ++u) {
+      if (((EP + (K - 1 - u) * DIL + r) & 1) != 0) continue;
+      const float* row = base + ((EP + (K - 1 - u) * DIL + r) >> 1) * ow8;
+#pragma unroll
+      for (int v = 0; v < K; ++v) {
+        if (((Q + (K - 1 - v) * DIL) & 1) != 0) continue;
+        a = __fmaf_rn(row[((Q + (K - 1 - v) * DIL) >> 1) * 8], wr[u][v], a);
+      }
+    }
+    acc[r] = a;
+  }
+}
+
+template <int K, int DIL>
+__global__ void __launch_bounds__(TPB) dw_dgrad_s2_kernel(const bf16* __restrict__ dz, const float* __restrict__ w,
+                                                        const bf16* __restrict__ add, bf16* __restrict__ dx, int B,
+                                                        int H, int C, int TW, const BnBwdFuse bnb) {
+  constexpr int PAD = DIL * (K / 2), KE = DIL * (K - 1) + 1, OH = DT_H / 2 + (KE + 1) / 2 + 1;
+  constexpr int RH = DT_H * S2_STRIPS, EP = (PAD - (K - 1) * DIL) & 1;
+  extern __shared__ float tile[];  // [CPG][OH][OW][8]
+  ptx::pdl_wait();
+  const int Ho = (H + 2 * PAD - KE) / 2 + 1;
+  const int CPG = TPB / (8 * TW), OW = TW / 2 + (KE + 1) / 2 + 1;
+  const int tiles_h = (H + RH - 1) / RH, tiles_w = (H + TW - 1) / TW;
+  int t = blockIdx.x;
+  const int tw = t % tiles_w;
+  t /= tiles_w;
+  const int th = t % tiles_h;
+  const int b = t / tiles_h;
+  const int cg0 = blockIdx.y * CPG;
+  const int iw0 = tw * TW;  // even
+  const int ow0 = (iw0 + PAD - (K - 1) * DIL) >> 1;  // first dz column the tile reads (floor; may be < 0)
+  // thread -> (channel, column, channel group); columns permuted so a warp's 4 share a parity
+  const int ch = threadIdx.x % 8, ci = (threadIdx.x / 8) % TW, cgi = threadIdx.x / (8 * TW);
+  const int col = (ci & ~7) + 2 * (ci & 3) + ((ci >> 2) & 1);
+  const int c = (cg0 + cgi) * 8 + ch;
+  float wr[K][K];
+#pragma unroll
+  for (int u = 0; u < K; ++u)
+#pragma unroll
+    for (int v = 0; v < K; ++v) wr[u][v] = c < C ? w[c * K * K + u * K + v] : 0.f;
+  const int iw = iw0 + col;
+  const int cc = EP + col;  // staged column of tap v: (cc + (K-1-v) DIL) / 2
+  const float* base = tile + (cgi * OH * OW + (cc >> 1)) * 8 + ch;
+  const int ow8 = OW * 8;
+  const bool fuse_b = bnb.acc != nullptr;
+  const bool valid = c < C && iw < H;
+  float ss = 0.f, sq = 0.f, bmu = 0.f, brs = 0.f, bg = 0.f, bb = 0.f;
+  if (fuse_b && valid) {
+    bmu = bnb.mean[c];
+    brs = bnb.rstd[c];
+    bg = bnb.g[c];
+    bb = bnb.b[c];
+  }
+  const size_t rstride = (size_t)H * C;
+  for (int st = 0; st < S2_STRIPS; ++st) {
+    const int ih0 = th * RH + st * DT_H;  // even
+    if (ih0 >= H) break;  // CTA-uniform
+    const int oh0 = (ih0 + PAD - (K - 1) * DIL) >> 1;  // first dz row the strip reads (floor)
+    __syncthreads();  // the previous strip's window has been consumed
+    for (int i = threadIdx.x; i < CPG * OH * OW; i += TPB) {
+      const int cl = i % OW, row = (i / OW) % OH, cg = i / (OW * OH);
+      const int oh = oh0 + row, ow = ow0 + cl, c8 = (cg0 + cg) * 8;
+      float v[8] = {};
+      if (oh >= 0 && oh < Ho && ow >= 0 && ow < Ho && c8 < C) load8(dz + (((size_t)b * Ho + oh) * Ho + ow) * C + c8, v);
+      float4* d = reinterpret_cast<float4*>(tile + i * 8);
+      d[0] = make_float4(v[0], v[1], v[2], v[3]);
+      d[1] = make_float4(v[4], v[5], v[6], v[7]);
+    }
+    __syncthreads();
+    float acc[DT_H];
+    if (cc & 1) s2_strip<K, DIL, 1>(base, ow8, wr, acc);  // warp-uniform
+    else s2_strip<K, DIL, 0>(base, ow8, wr, acc);
+    if (valid) {
+      const size_t o0 = (((size_t)b * H + ih0) * H + iw) * C + c;
+      const int nr = min(DT_H, H - ih0);
+#pragma unroll
+      for (int r = 0; r < DT_H; ++r) {
+        if (r >= nr) break;
+        const size_t o = o0 + r * rstride;
+        const bf16 ob = __float2bfloat16_rn(add ? acc[r] + __bfloat162float(add[o]) : acc[r]);
+        dx[o] = ob;
+        if (fuse_b) {
+          float d = __bfloat162float(ob), xh;
+          const float zz = __bfloat162float(bnb.z[o]) + __bfloat162float(bnb.z[o + bnb.zplane]);
+          bn_bwd_elem(d, zz, bmu, brs, bg, bb, bnb.relu, xh);
+          ss += d;
+          sq = __fmaf_rn(d, xh, sq);
+        }
+      }
+    }
+  }
+  if (fuse_b) {  // per channel: xor tree over the warp's 4 columns, then its warps in warp order
+    __shared__ float wsum[TPB / 32][2][8];
+#pragma unroll
+    for (int o = 8; o < 32; o <<= 1) {
+      ss += __shfl_xor_sync(0xffffffffu, ss, o);
+      sq += __shfl_xor_sync(0xffffffffu, sq, o);
+    }
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (lane < 8) {
+      wsum[warp][0][lane] = ss;
+      wsum[warp][1][lane] = sq;
+    }
+    __syncthreads();
+    const int wpg = TW / 4;
+    if (threadIdx.x < CPG * 16) {
+      const int g = threadIdx.x / 16, which = (threadIdx.x / 8) & 1, chn = threadIdx.x & 7;
+      const int c2 = (cg0 + g) * 8 + chn;
+      float a = 0.f;
+      for (int k = 0; k < wpg; ++k) a += wsum[g * wpg + k][which][chn];
+      if (c2 < C) fix_add(bnb.acc, (which ? C : 0) + c2, bnb.acc + 2 * C, a, FIX_B);
     }
   }
 }
@@ -662,10 +839,12 @@ __global__ void __launch_bounds__(TPB) dw_tile_kernel(const bf16* __restrict__ i
 // layout; fixpoint.cuh: bitwise independent of the CTA order).  The last CTA (ticket) applies
 // the SGD WRITE w -= lr * total (w = the master, or the bulk accumulator under BSP) and clears
 // acc: one launch instead of partials + a fixed-order summing SGD kernel.
-template <int K, int S, int DIL>
+// XBN: x = the hi plane of relu?(BN(z)) recomputed on load from the published mean / rstd
+// and the forward's g / b snapshots (BnApplyIn; bn_apply was folded into the forward conv).
+template <int K, int S, int DIL, bool XBN = false>
 __global__ void __launch_bounds__(TPB) dw_wgrad_kernel(const bf16* __restrict__ dz, const bf16* __restrict__ x,
                                                        unsigned long long* gacc, int* ticket, float* w, float lr,
-                                                       int B, int H, int C, int TW, int NP) {
+                                                       int B, int H, int C, int TW, int NP, const BnApplyIn xbn) {
   constexpr int PAD = DIL * (K / 2), KE = DIL * (K - 1) + 1, IH = (DT_H - 1) * S + KE, K2 = K * K;
   extern __shared__ float tile[];  // [CPG][IH][IW][8]; later [TPB][K2] for the column sums
   ptx::pdl_wait();
@@ -676,6 +855,8 @@ __global__ void __launch_bounds__(TPB) dw_wgrad_kernel(const bf16* __restrict__ 
   const int cg0 = blockIdx.y * CPG;
   const int ch = threadIdx.x % 8, col = (threadIdx.x / 8) % TW, cgi = threadIdx.x / (8 * TW);
   const int c = (cg0 + cgi) * 8 + ch, ow = tw * TW + col;
+  __shared__ float xmu[XBN ? XBN_CH : 1], xrs[XBN ? XBN_CH : 1], xg[XBN ? XBN_CH : 1], xb[XBN ? XBN_CH : 1];
+  if constexpr (XBN) xbn_stage(xbn, false, cg0 * 8, CPG * 8, C, xmu, xrs, xg, xb);
   float acc[K][K];
 #pragma unroll
   for (int u = 0; u < K; ++u)
@@ -689,7 +870,15 @@ __global__ void __launch_bounds__(TPB) dw_wgrad_kernel(const bf16* __restrict__ 
       const int cl = i % IW, row = (i / IW) % IH, cg = i / (IW * IH);
       const int ih = ih0 + row, iw = iw0 + cl, cc = (cg0 + cg) * 8;
       float v[8] = {};
-      if (ih >= 0 && ih < H && iw >= 0 && iw < H && cc < C) load8(x + (((size_t)b * H + ih) * H + iw) * C + cc, v);
+      if (ih >= 0 && ih < H && iw >= 0 && iw < H && cc < C) {
+        const size_t o = (((size_t)b * H + ih) * H + iw) * C + cc;
+        if constexpr (XBN) {
+          load8x2(xbn.z + o, xbn.zplane, v);
+          xbn_y8<true>(v, xmu, xrs, xg, xb, cg * 8, xbn.relu);
+        } else {
+          load8(x + o, v);
+        }
+      }
       float4* d = reinterpret_cast<float4*>(tile + (size_t)i * 8);
       d[0] = make_float4(v[0], v[1], v[2], v[3]);
       d[1] = make_float4(v[4], v[5], v[6], v[7]);
@@ -1001,7 +1190,7 @@ static int ew_waves() {
 // NASPIPE_MAX_CTAS_PER_SM (tuning): cap the resident-CTA count used for the grid sizes below
 // resident CTAs per SM of `kern` at `smem` dynamic bytes, cached per (kernel address, smem)
 // -- a static per template instantiation was shared by kernels of the same type (e.g. the
-// dw_dgrad_kernel<K> of different K); guarded: engines may be created from
+// dw_tile_kernel<K> of different K); guarded: engines may be created from
 // several host threads
 template <typename Kern>
 static int occupancy(Kern kern, size_t smem) {
@@ -1108,19 +1297,39 @@ bool bn_fix_overflow(const unsigned long long* acc, int C) {
     default: NP_REQUIRE(false, NASPIPE_EINVAL, "depthwise kernel %d dilation %d", K, D); \
   }
 
+// DT_H-row strips per depthwise CTA: NASPIPE_DW_STRIPS (1 / 2 / 4; default 0 = by grid size)
+static int dw_strips() {
+  static const int v = [] {
+    const char* e = getenv("NASPIPE_DW_STRIPS");
+    return e ? std::max(0, std::min(4, atoi(e))) : 0;
+  }();
+  return v;
+}
+
 // tile width: the smallest of 8 / 16 / 32 columns covering min(Ho, 32)
 static int dw_tw(int Ho) { return Ho <= 8 ? 8 : (Ho <= 16 ? 16 : 32); }
 
-template <int K, int S, int DIL, bool X2, bool FLIP>
+template <int K, int S, int DIL, bool X2, bool FLIP, bool XBN = false>
 static void dw_tile(cudaStream_t s, const bf16* in, const float* w, const bf16* add, bf16* out, int B, int H, int C,
-                    unsigned long long* stats = nullptr) {
+                    unsigned long long* stats = nullptr, const BnBwdFuse& bnb = BnBwdFuse(),
+                    const BnApplyIn& xbn = BnApplyIn()) {
   constexpr int KE = DIL * (K - 1) + 1;
   const int Ho = (H - 1) / S + 1, TW = dw_tw(Ho), CPG = TPB / (8 * TW);
   const int IH = (DT_H - 1) * S + KE, IW = (TW - 1) * S + KE;
   const size_t sm = (size_t)CPG * IH * IW * 8 * sizeof(float);
-  const int gx = B * ((Ho + DT_H - 1) / DT_H) * ((Ho + TW - 1) / TW), gy = (C / 8 + CPG - 1) / CPG;
-  set_smem(dw_tile_kernel<K, S, DIL, X2, FLIP>, sm);
-  launch_pdl(dw_tile_kernel<K, S, DIL, X2, FLIP>, dim3(gx, gy), dim3(TPB), sm, s, in, w, add, out, B, H, C, TW, stats);
+  auto kern = dw_tile_kernel<K, S, DIL, X2, FLIP, XBN>;
+  set_smem(kern, sm);
+  // strips of DT_H rows per CTA: as many (<= 4) as keep >= 2 waves of resident CTAs (the
+  // weights, the halo setup and the reductions amortised over more outputs per CTA)
+  const int tiles_w = (Ho + TW - 1) / TW, gy = (C / 8 + CPG - 1) / CPG, rows = (Ho + DT_H - 1) / DT_H;
+  int strips = dw_strips();
+  if (strips <= 0) {
+    const long wave = (long)num_sms() * occupancy(kern, sm);
+    strips = 1;
+    while (strips < 4 && (long)B * ((rows + 2 * strips - 1) / (2 * strips)) * tiles_w * gy >= 2 * wave) strips *= 2;
+  }
+  const int gx = B * ((Ho + DT_H * strips - 1) / (DT_H * strips)) * tiles_w;
+  launch_pdl(kern, dim3(gx, gy), dim3(TPB), sm, s, in, w, add, out, B, H, C, TW, strips, stats, bnb, xbn);
 }
 
 void dw_fwd(cudaStream_t s, const bf16* x, const float* w, bf16* z, int B, int H, int C, int k, int S, int dil,
@@ -1131,18 +1340,35 @@ void dw_fwd(cudaStream_t s, const bf16* x, const float* w, bf16* z, int B, int H
   check_launch("dw_fwd");
 }
 
+void dw_fwd_bn(cudaStream_t s, const BnApplyIn& xin, const float* w, bf16* z, int B, int H, int C, int k, int S,
+               int dil, unsigned long long* stats) {
+  NP_REQUIRE(C % 8 == 0 && (S == 1 || S == 2) && xin.P == B * H * H && xin.acc && xin.ticket && xin.mean &&
+                 xin.gsnap && stats != xin.acc,
+             NASPIPE_EINVAL, "dw_fwd_bn C=%d S=%d P=%d", C, S, xin.P);
+  if (S == 1) { DW_DISPATCH(k, dil, (dw_tile<KK, 1, DD, true, false, true>(s, nullptr, w, nullptr, z, B, H, C, stats, BnBwdFuse(), xin))); }
+  else { DW_DISPATCH(k, dil, (dw_tile<KK, 2, DD, true, false, true>(s, nullptr, w, nullptr, z, B, H, C, stats, BnBwdFuse(), xin))); }
+  check_launch("dw_fwd_bn");
+}
+
+template <int K, int DIL>
+static void dw_dgrad_s2(cudaStream_t s, const bf16* dz, const float* w, const bf16* add, bf16* dx, int B, int H, int C,
+                        const BnBwdFuse& bnb) {
+  constexpr int KE = DIL * (K - 1) + 1, OH = DT_H / 2 + (KE + 1) / 2 + 1;
+  const int TW = dw_tw(H), CPG = TPB / (8 * TW);
+  const int RH = DT_H * S2_STRIPS;
+  const int gx = B * ((H + RH - 1) / RH) * ((H + TW - 1) / TW), gy = (C / 8 + CPG - 1) / CPG;
+  const size_t sm = (size_t)CPG * OH * (TW / 2 + (KE + 1) / 2 + 1) * 8 * sizeof(float);
+  set_smem(dw_dgrad_s2_kernel<K, DIL>, sm);
+  launch_pdl(dw_dgrad_s2_kernel<K, DIL>, dim3(gx, gy), dim3(TPB), sm, s, dz, w, add, dx, B, H, C, TW, bnb);
+}
+
 void dw_dgrad(cudaStream_t s, const bf16* dz, const float* w, const bf16* add, bf16* dx, int B, int H, int C, int k,
-              int S, int dil) {
+              int S, int dil, const BnBwdFuse& bnb) {
+  NP_REQUIRE(C % 8 == 0 && (S == 1 || S == 2), NASPIPE_EINVAL, "dw_dgrad C=%d S=%d", C, S);
   if (S == 1) {  // the input gradient of a stride-1 conv is the correlation with the flipped kernel
-    DW_DISPATCH(k, dil, (dw_tile<KK, 1, DD, false, true>(s, dz, w, add, dx, B, H, C)));
+    DW_DISPATCH(k, dil, (dw_tile<KK, 1, DD, false, true>(s, dz, w, add, dx, B, H, C, nullptr, bnb)));
   } else {
-    const size_t items = (size_t)B * H * H * (C / 8);
-    const size_t sm = (size_t)C * k * k * sizeof(float);
-    DW_DISPATCH(k, dil, {
-      set_smem(dw_dgrad_kernel<KK, DD>, sm);
-      launch_pdl(dw_dgrad_kernel<KK, DD>, dim3(gs_grid(dw_dgrad_kernel<KK, DD>, items, sm)), dim3(TPB), sm, s, dz, w,
-                 add, dx, B, H, C, S);
-    });
+    DW_DISPATCH(k, dil, (dw_dgrad_s2<KK, DD>(s, dz, w, add, dx, B, H, C, bnb)));
   }
   check_launch("dw_dgrad");
 }
@@ -1166,7 +1392,7 @@ int dw_wgrad_blocks(int B, int H, int C, int k, int S) {  // grid size (diagnost
 }
 
 void dw_wgrad_sgd(cudaStream_t s, const bf16* dz, const bf16* x, unsigned long long* acc, int* ticket, float* w,
-                  float lr, int B, int H, int C, int k, int S, int dil) {
+                  float lr, int B, int H, int C, int k, int S, int dil, const BnApplyIn* xin) {
   NP_REQUIRE(C % 8 == 0 && C / 8 <= TPB, NASPIPE_EINVAL, "dw_wgrad C=%d", C);
   NP_REQUIRE(S == 1 || S == 2, NASPIPE_EINVAL, "dw_wgrad stride %d", S);
   int TW, NP, gy, tiles_w;
@@ -1177,18 +1403,22 @@ void dw_wgrad_sgd(cudaStream_t s, const bf16* dz, const bf16* x, unsigned long l
     return std::max((size_t)CPG * IH * IW * 8, (size_t)TPB * K * K) * sizeof(float);
   };
   const dim3 grid(tiles_w * NP, gy);
-#define DW_WG(KK, SS, DD)                                                                                        \
+  const BnApplyIn xb = xin ? *xin : BnApplyIn();
+#define DW_WG1(KK, SS, DD, XB)                                                                                     \
   {                                                                                                              \
-    set_smem(dw_wgrad_kernel<KK, SS, DD>, smem(KK, DD));                                                         \
-    launch_pdl(dw_wgrad_kernel<KK, SS, DD>, grid, dim3(TPB), smem(KK, DD), s, dz, x, acc, ticket, w, lr, B, H, C, TW, \
-               NP);                                                                                              \
+    set_smem(dw_wgrad_kernel<KK, SS, DD, XB>, smem(KK, DD));                                                     \
+    launch_pdl(dw_wgrad_kernel<KK, SS, DD, XB>, grid, dim3(TPB), smem(KK, DD), s, dz, x, acc, ticket, w, lr, B, H, C, \
+               TW, NP, xb);                                                                                      \
   }
+#define DW_WG(KK, SS, DD) \
+  if (xin) DW_WG1(KK, SS, DD, true) else DW_WG1(KK, SS, DD, false)
   if (S == 1) {
     DW_DISPATCH(k, dil, DW_WG(KK, 1, DD));
   } else {
     DW_DISPATCH(k, dil, DW_WG(KK, 2, DD));
   }
 #undef DW_WG
+#undef DW_WG1
   check_launch("dw_wgrad");
 }
 

@@ -27,6 +27,8 @@ L.naspipe_debug_chan_split.argtypes = [_vp, _i, _i, _vp, _i, C.c_size_t, _vp, _v
 L.naspipe_debug_gemm_x2.argtypes = [_i, _i, _i, _vp, _vp, _i, _vp, _vp, _i, _vp, _vp, _vp]
 L.naspipe_debug_chan_merge.argtypes = [_vp, _i, _vp, _i, _i, _vp, _vp]
 L.naspipe_debug_stem.argtypes = [_vp, _vp, _vp, _i, _i, _i, _vp]
+L.naspipe_debug_dw_bn_fold.argtypes = [_vp, _i, _i, _i, _vp, _vp, _i, _vp, _i, _i, _i] + [_vp] * 9
+L.naspipe_debug_bnb_fused.argtypes = [_i, _vp, _vp, _vp, _vp] + [_i] * 6 + [_vp] * 5 + [_i, _vp, _vp]
 
 
 def _ok(rc):
@@ -199,6 +201,96 @@ def test_batchnorm_fwd_bwd(P, Cc, relu):
     np.testing.assert_allclose(_f64(g2), g - lr * s[Cc:].astype(np.float32), rtol=1e-6, atol=1e-7)
     np.testing.assert_allclose(_f64(b2), b - lr * s[:Cc].astype(np.float32), rtol=1e-6, atol=1e-7)
     _check_bf16(_f64(dz), rdz)
+
+
+@pytest.mark.parametrize("B,H,Cc,k,s,d,relu", [(2, 9, 16, 3, 1, 1, 1), (3, 8, 48, 5, 2, 1, 1), (2, 14, 32, 7, 1, 2, 0),
+                                             (64, 56, 32, 3, 1, 1, 1), (64, 112, 32, 5, 2, 1, 1),
+                                             (64, 7, 320, 7, 1, 1, 1), (64, 14, 160, 3, 2, 2, 1)])
+def test_bn_apply_folded_into_depthwise_is_bitwise_the_stored_path(B, H, Cc, k, s, d, relu):
+    """conv -> BN -> ReLU -> depthwise with bn_apply folded into the depthwise conv's load
+    (BnApplyIn): the conv output, the weight gradient (BN recomputed on load) and the
+    published mean / rstd are BITWISE those of the stored path (bn_apply -> y -> dw_fwd); the
+    published g, b snapshots are the forward's; and the result matches explicit loops."""
+    rng = np.random.default_rng(B + H + Cc + k + s + d)
+    zd, z = _x2(rng.standard_normal((B, H, H, Cc)) * rng.uniform(0.5, 2.0, Cc) + rng.uniform(-1, 1, Cc))
+    g = rng.uniform(0.5, 1.5, Cc).astype(np.float32)
+    b = rng.uniform(-0.3, 0.3, Cc).astype(np.float32)
+    gd, bd = torch.from_numpy(g).cuda(), torch.from_numpy(b).cuda()
+    w = (rng.standard_normal((Cc, k, k)) / k).astype(np.float32)
+    wd = torch.from_numpy(w).cuda()
+    Ho = (H - 1) // s + 1
+    dzd, dz = _bf(rng.standard_normal((B, Ho, Ho, Cc)))
+    out_ref = torch.empty((2, B, Ho, Ho, Cc), dtype=torch.bfloat16, device="cuda")
+    out = torch.empty_like(out_ref)
+    dws_ref = torch.empty((Cc, k, k), device="cuda")
+    dws = torch.empty_like(dws_ref)
+    meta = torch.empty(4 * Cc, device="cuda")
+    mean_ref, rstd_ref = torch.empty(Cc, device="cuda"), torch.empty(Cc, device="cuda")
+    _ok(L.naspipe_debug_dw_bn_fold(_p(zd), B, H, Cc, _p(gd), _p(bd), relu, _p(wd), k, s, d, _p(dzd), _p(out_ref),
+                                   _p(out), _p(dws_ref), _p(dws), _p(meta), _p(mean_ref), _p(rstd_ref), None))
+    torch.cuda.synchronize()
+    assert torch.equal(out, out_ref)
+    assert torch.equal(dws, dws_ref)
+    assert torch.equal(meta[:Cc], mean_ref) and torch.equal(meta[Cc:2 * Cc], rstd_ref)
+    assert torch.equal(meta[2 * Cc:3 * Cc], gd) and torch.equal(meta[3 * Cc:], bd)
+    if B * H * H <= 20000:  # and the composition against explicit loops (fp64 on the stored y)
+        ry, _, _, _ = _bn_ref(z.reshape(-1, Cc), g.astype(np.float64), b.astype(np.float64), relu)
+        _check_x2(_v2(out), _dw_ref(ry.reshape(z.shape), w.astype(np.float64), s, d), tol=1e-4)
+
+
+@pytest.mark.parametrize("kind,B,H,Cc,Cout,k,dil,relu", [
+    (0, 2, 9, 16, 0, 3, 1, 1), (0, 3, 14, 32, 0, 7, 1, 0), (0, 2, 37, 24, 0, 5, 2, 1), (0, 64, 56, 32, 0, 3, 1, 1),
+    (0, 64, 7, 320, 0, 7, 2, 1), (2, 3, 9, 16, 0, 3, 1, 1), (2, 2, 14, 48, 0, 7, 2, 0), (2, 64, 112, 32, 0, 7, 1, 1),
+    (2, 64, 14, 160, 0, 5, 1, 1),
+    (1, 2, 9, 16, 48, 0, 0, 0), (1, 3, 13, 80, 160, 0, 0, 1), (1, 64, 14, 160, 320, 0, 0, 0),
+    (1, 64, 7, 320, 640, 0, 0, 1), (1, 64, 56, 32, 32, 0, 0, 0)])
+def test_bn_backward_sums_fused_into_input_gradient(kind, B, H, Cc, Cout, k, dil, relu):
+    """bn_bwd_reduce fused into the producer of dy (stride-1 / stride-2 depthwise dgrad, 1x1-conv dgrad
+    epilogue EPI_BNBWD): dx as the plain kernels compute it, and (sum dy', sum dy' xh) of the
+    STORED dx against an fp64 reference on the same values (unit z -> BN -> ReLU?)."""
+    rng = np.random.default_rng(1000 * kind + B + H + Cc + k)
+    P = B * H * H
+    if kind in (0, 2):
+        w = (rng.standard_normal((Cc, k, k)) / k).astype(np.float32)
+        wd, w16d = torch.from_numpy(w).cuda(), None
+        Ho = H if kind == 0 else (H - 1) // 2 + 1
+        dzd, dz = _bf(rng.standard_normal((B, Ho, Ho, Cc)))
+    else:
+        w16d, w16 = _bf(rng.standard_normal((Cout, Cc)) / np.sqrt(Cout))
+        wd = None
+        dzd, dz = _bf(rng.standard_normal((P, Cout)))
+    zd, z = _x2(rng.standard_normal((P, Cc)) * rng.uniform(0.5, 2.0, Cc) + rng.uniform(-1, 1, Cc))
+    mu = z.mean(axis=0).astype(np.float32)
+    rs = (1.0 / np.sqrt(z.var(axis=0) + 1e-5)).astype(np.float32)
+    g = rng.uniform(0.5, 1.5, Cc).astype(np.float32)
+    b = rng.uniform(-0.3, 0.3, Cc).astype(np.float32)
+    md, rd, gd, bd = (torch.from_numpy(a).cuda() for a in (mu, rs, g, b))
+    dx = torch.empty((P, Cc), dtype=torch.bfloat16, device="cuda")
+    sums = torch.empty(2 * Cc, device="cuda")
+    outs = []
+    for _ in range(2):
+        _ok(L.naspipe_debug_bnb_fused(kind, _p(dzd), _p(wd), _p(w16d), _p(dx), B, H, Cc, Cout, k, dil, _p(zd), _p(md),
+                                      _p(rd), _p(gd), _p(bd), relu, _p(sums), None))
+        torch.cuda.synchronize()
+        outs.append((dx.clone(), sums.clone()))
+    assert torch.equal(outs[0][0], outs[1][0]) and torch.equal(outs[0][1], outs[1][1])
+    if kind in (0, 2):
+        rdx, _ = _dw_bwd_ref(np.zeros((B, H, H, Cc)), w.astype(np.float64), 1 if kind == 0 else 2, dz, dil)
+        rdx = rdx.reshape(P, Cc)
+    else:
+        rdx = dz @ w16
+    got = _f64(dx)
+    _check_bf16(got, rdx)
+    # the sums are taken over the stored dx (bf16); xh and the ReLU mask as the kernel forms
+    # them (fp32 xh = (z - mean) rstd, y = fma(g, xh, b): the sign of the exact g xh + b)
+    xh32 = ((z.astype(np.float32) - mu) * rs).astype(np.float32)
+    xh = xh32.astype(np.float64)
+    d = got * ((g.astype(np.float64) * xh + b) > 0) if relu else got
+    s1, s2 = d.sum(axis=0), (d * xh).sum(axis=0)
+    s = _f64(sums)
+    a1, a2 = np.abs(d).sum(axis=0), np.abs(d * xh).sum(axis=0)
+    assert np.all(np.abs(s[:Cc] - s1) <= 1e-5 * a1 + 1e-9)
+    assert np.all(np.abs(s[Cc:] - s2) <= 1e-5 * a2 + 1e-9)
 
 
 @pytest.mark.parametrize("P,Ch", [(7, 16), (3136, 320), (1000, 80)])
