@@ -166,8 +166,44 @@ __global__ void __launch_bounds__(128, 1) attn_fwd_tc_kernel(const __grid_consta
   }
 }
 
+// Di = rowsum(dO o O) of the CTA's 128 query rows into sDi, coalesced: a warp reads LPR = HD/8
+// lanes x 16 bytes per row (RPI rows per load instruction, every load of the warp's rows in
+// flight at once), each lane sums its 8 products in column order, then a fixed xor tree over
+// the row's LPR lanes (bitwise deterministic).  (A thread-per-row loop left ~25 % of the
+// backward's stall samples on these loads: 4 dependent round trips of uncoalesced rows.)
+template <int HD, int NWARPS>
+__device__ __forceinline__ void attn_di_rows(const bf16* __restrict__ dout, const bf16* __restrict__ o, int b, int hh,
+                                             int d, float* sDi) {
+  constexpr int LPR = HD / 8, RPI = 32 / LPR, ROWS = AS / NWARPS, IT = ROWS / RPI;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int sub = lane / LPR, cl = (lane % LPR) * 8;
+  uint4 a[IT], q[IT];
+#pragma unroll
+  for (int it = 0; it < IT; ++it) {
+    const int row = warp * ROWS + it * RPI + sub;
+    const size_t off = ((size_t)b * AS + row) * d + hh * HD + cl;
+    a[it] = *reinterpret_cast<const uint4*>(dout + off);
+    q[it] = *reinterpret_cast<const uint4*>(o + off);
+  }
+#pragma unroll
+  for (int it = 0; it < IT; ++it) {
+    const uint32_t aw[4] = {a[it].x, a[it].y, a[it].z, a[it].w}, qw[4] = {q[it].x, q[it].y, q[it].z, q[it].w};
+    float di = 0.f;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      di = fmaf(__uint_as_float(aw[i] << 16), __uint_as_float(qw[i] << 16), di);
+      di = fmaf(__uint_as_float(aw[i] & 0xffff0000u), __uint_as_float(qw[i] & 0xffff0000u), di);
+    }
+#pragma unroll
+    for (int off = LPR / 2; off >= 1; off >>= 1) di += __shfl_xor_sync(0xffffffffu, di, off);
+    if (lane % LPR == 0) sDi[warp * ROWS + it * RPI + sub] = di;
+  }
+}
+
+// 8 warps: warps w and w + 4 share TMEM lane quarter w % 4 (query / key rows 32 (w % 4) ..)
+// and split the columns of the softmax phase and of the gradient epilogue in halves.
 template <int HD>
-__global__ void __launch_bounds__(128, 1) attn_bwd_tc_kernel(const __grid_constant__ CUtensorMap tq,
+__global__ void __launch_bounds__(256, 1) attn_bwd_tc_kernel(const __grid_constant__ CUtensorMap tq,
                                                               const __grid_constant__ CUtensorMap tdo,
                                                               const bf16* __restrict__ o, const float* __restrict__ lse,
                                                               const bf16* __restrict__ dout, bf16* __restrict__ dqkv,
@@ -182,8 +218,10 @@ __global__ void __launch_bounds__(128, 1) attn_bwd_tc_kernel(const __grid_consta
   uint8_t* sdS = sP + 2 * TILE;     // [128 q][128 k]
   uint64_t* bar = reinterpret_cast<uint64_t*>(sdS + 2 * TILE);  // [0] TMA, [1] S + dP, [2] gradients
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bar + 3);
+  float* sDi = reinterpret_cast<float*>(bar + 4);  // [128]
   const int bh = blockIdx.x, b = bh / h, hh = bh % h;
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, r = threadIdx.x;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int r = 32 * (warp & 3) + lane, hf = warp >> 2;  // TMEM lane (row) and column half
   if (threadIdx.x == 0) {
     ptx::tma_prefetch(&tq);
     ptx::tma_prefetch(&tdo);
@@ -217,28 +255,17 @@ __global__ void __launch_bounds__(128, 1) attn_bwd_tc_kernel(const __grid_consta
     }
     __syncwarp();
   }
-  // Di = rowsum(dO o O) (fp32, column order) while the MMAs run
-  const bf16* drow = dout + ((size_t)b * AS + r) * d + hh * HD;
-  const bf16* orow = o + ((size_t)b * AS + r) * d + hh * HD;
-  float di = 0.f;
-#pragma unroll 4
-  for (int c = 0; c < HD; c += 8) {
-    const uint4 a = *reinterpret_cast<const uint4*>(drow + c);
-    const uint4 q = *reinterpret_cast<const uint4*>(orow + c);
-    const uint32_t aw[4] = {a.x, a.y, a.z, a.w}, qw[4] = {q.x, q.y, q.z, q.w};
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      di = fmaf(__uint_as_float(aw[i] << 16), __uint_as_float(qw[i] << 16), di);
-      di = fmaf(__uint_as_float(aw[i] & 0xffff0000u), __uint_as_float(qw[i] & 0xffff0000u), di);
-    }
-  }
+  // Di = rowsum(dO o O) while the MMAs run
+  attn_di_rows<HD, 8>(dout, o, b, hh, d, sDi);
   const float l2 = lse[(size_t)bh * AS + r] * LOG2E;
   const float scale = 1.f / sqrtf((float)HD), sl2 = LOG2E * scale;
+  __syncthreads();
+  const float di = sDi[r];
   ptx::mbar_wait(&bar[1], 0);
   ptx::tc_fence_after();
-  const uint32_t trow = tmem + ((uint32_t)(warp * 32) << 16);
+  const uint32_t trow = tmem + ((uint32_t)(32 * (warp & 3)) << 16);
 #pragma unroll
-  for (int c0 = 0; c0 < AS; c0 += 32) {
+  for (int c0 = hf * (AS / 2); c0 < hf * (AS / 2) + AS / 2; c0 += 32) {
     uint32_t s[32], dp[32];
     ptx::tmem_ld32(trow + c0, s);
     ptx::tmem_ld32(trow + 128 + c0, dp);
@@ -281,7 +308,7 @@ __global__ void __launch_bounds__(128, 1) attn_bwd_tc_kernel(const __grid_consta
   bf16* krow = qrow + d;
   bf16* vrow = qrow + 2 * d;
 #pragma unroll
-  for (int c0 = 0; c0 < HD; c0 += 32) {
+  for (int c0 = hf * (HD / 2); c0 < hf * (HD / 2) + HD / 2; c0 += 32) {
     uint32_t dv[32], dk[32], dq[32];
     ptx::tmem_ld32(trow + c0, dv);
     ptx::tmem_ld32(trow + HD + c0, dk);
@@ -331,6 +358,7 @@ __global__ void __launch_bounds__(128, 2) attn_bwd_tc64_kernel(const __grid_cons
   uint8_t* sB = sdO + TILE;  // [128 q][128 k]: P, then dS
   uint64_t* bar = reinterpret_cast<uint64_t*>(sB + 2 * TILE);  // [0] TMA, [1] S + dP, [2] dV, [3] dK + dQ
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bar + 4);
+  float* sDi = reinterpret_cast<float*>(bar + 5);  // [128]
   const int bh = blockIdx.x, b = bh / h, hh = bh % h;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, r = threadIdx.x;
   if (threadIdx.x == 0) {
@@ -364,20 +392,9 @@ __global__ void __launch_bounds__(128, 2) attn_bwd_tc64_kernel(const __grid_cons
     }
     __syncwarp();
   }
-  const bf16* drow = dout + ((size_t)b * AS + r) * d + hh * HD;
-  const bf16* orow = o + ((size_t)b * AS + r) * d + hh * HD;
-  float di = 0.f;
-#pragma unroll 4
-  for (int c = 0; c < HD; c += 8) {
-    const uint4 a = *reinterpret_cast<const uint4*>(drow + c);
-    const uint4 q = *reinterpret_cast<const uint4*>(orow + c);
-    const uint32_t aw[4] = {a.x, a.y, a.z, a.w}, qw[4] = {q.x, q.y, q.z, q.w};
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      di = fmaf(__uint_as_float(aw[i] << 16), __uint_as_float(qw[i] << 16), di);
-      di = fmaf(__uint_as_float(aw[i] & 0xffff0000u), __uint_as_float(qw[i] & 0xffff0000u), di);
-    }
-  }
+  attn_di_rows<HD, 4>(dout, o, b, hh, d, sDi);
+  __syncthreads();
+  const float di = sDi[r];
   const float l2 = lse[(size_t)bh * AS + r] * LOG2E;
   const float scale = 1.f / sqrtf((float)HD), sl2 = LOG2E * scale;
   ptx::mbar_wait(&bar[1], 0);
@@ -518,13 +535,13 @@ void attn_bwd_tc(cudaStream_t s, const bf16* qkv, const bf16* o, const float* ls
   const CUtensorMap tq = tma_map_bf16(qkv, 3 * (uint64_t)d, (uint64_t)B * S, 3 * (uint64_t)d, 128);
   const CUtensorMap tdo = tma_map_bf16(dout, (uint64_t)d, (uint64_t)B * S, (uint64_t)d, 128);
   if (hd == 64) {  // one P/dS buffer, two CTAs per SM
-    const int smem = 6 * TILE + 1024 + 64;
+    const int smem = 6 * TILE + 1024 + 64 + 512;
     set_smem_attr(attn_bwd_tc64_kernel, smem);
     launch_pdl(attn_bwd_tc64_kernel, dim3(B * h), dim3(128), smem, s, tq, tdo, o, lse, dout, dqkv, d, h);
   } else {
-    const int smem = 12 * TILE + 1024 + 64;
+    const int smem = 12 * TILE + 1024 + 64 + 512;
     set_smem_attr(attn_bwd_tc_kernel<128>, smem);
-    launch_pdl(attn_bwd_tc_kernel<128>, dim3(B * h), dim3(128), smem, s, tq, tdo, o, lse, dout, dqkv, d, h);
+    launch_pdl(attn_bwd_tc_kernel<128>, dim3(B * h), dim3(256), smem, s, tq, tdo, o, lse, dout, dqkv, d, h);
   }
   const cudaError_t e = cudaGetLastError();
   NP_REQUIRE(e == cudaSuccess, NASPIPE_ECUDA, "attn_bwd_tc: %s", cudaGetErrorString(e));
