@@ -70,6 +70,9 @@ def parse():
     ap.add_argument("--virtual-stages", type=int, default=1,
                     help="N = 1: pipeline stages on the one GPU (CSP across concurrently running stage streams)")
     ap.add_argument("--lookahead", type=int, default=0, help="residency prefetch depth L in tasks (0 = 2, P:L156)")
+    ap.add_argument("--timed", action="store_true",
+                    help="N = 1: the timing-driven executor (NASPIPE_FLAG_TIMED: Alg.1 on observed completions, "
+                         "Alg.3's predictor scored) instead of the planned one")
     return ap.parse_args()
 
 
@@ -382,6 +385,8 @@ def workload_config(args, cfg, world):
          "stages": world, "parallelism": f"pp{world}" if world > 1 else "single stage",
          "activation_recompute": bool(getattr(args, "recompute", False)),
          "sync_policy": getattr(args, "sync", "csp"),
+         "executor": "timing-driven (Alg.1 on observed completions)" if getattr(args, "timed", False) else "planned",
+         "virtual_stages": getattr(args, "virtual_stages", 1),
          "l2": "working set > L2 (active weights + activations per step >> 126 MB)",
          # reduction-order / launch tuning knobs in effect (empty = the library defaults):
          # bitwise comparisons carry their reduction configuration
@@ -469,8 +474,9 @@ def main():
     dev_pool = [(torch.from_numpy(x).cuda(), torch.from_numpy(t).cuda()) for x, t in pool]
     host_pool = [(torch.from_numpy(x).pin_memory(), torch.from_numpy(t).pin_memory()) for x, t in pool]
     budget = stage_budget(cfg, D, args.budget_x, npipe) if args.budget_x > 0 else 0
+    assert not (args.timed and world > 1), "--timed: one process (stages on this GPU via --virtual-stages)"
     spec = npipe.Spec(cfg, hbm_weight_budget_bytes=budget, lookahead=args.lookahead, sync=args.sync,
-                      flags=npipe.FLAG_RECOMPUTE if args.recompute else 0)
+                      flags=(npipe.FLAG_RECOMPUTE if args.recompute else 0) | (npipe.FLAG_TIMED if args.timed else 0))
 
     def create(sp):
         if world == 1:
@@ -628,6 +634,7 @@ def main():
         e2e = {"value": args.steps * B / (ms2 / 1000), "unit": "samples/s",
                "h2d_bytes_per_step": x.numel() * x.element_size() + t.numel() * t.element_size(),
                "d2h_bytes_per_step": 4}
+    timed_stats = npipe.naspipe_get_timed_stats(h) if args.timed else None
     losses = npipe.naspipe_get_losses(h, state["y"]) if rank == world - 1 else None
     loss_ok = bool(losses is None or np.all(np.isfinite(losses)))
     loss_ok = reduce(0.0 if loss_ok else 1.0) == 0.0
@@ -689,6 +696,9 @@ def main():
                                            "(profiles/*pcie*; tools/pcie_bw.py)"} if budget else None,
            "p2p_GBps": (s1["p2p_bytes"] - s0["p2p_bytes"]) / (ms / 1000) / 1e9 if world > 1 else None,
            "loss_finite": loss_ok, "bit_repro": repro}
+    if timed_stats is not None:
+        out["timed_executor"] = dict(timed_stats, note="all timed regions of this run (value, CUPTI, e2e); Alg.3 "
+                                     "hits = predictions equal to the stage's next forward")
     if sec is not None:
         out["secondary"] = sec
     print(json.dumps(out))

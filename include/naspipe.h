@@ -105,6 +105,20 @@ typedef enum { NASPIPE_FP32 = 0, NASPIPE_BF16 = 1 } naspipe_dtype; /* compute dt
  * planned and issued at naspipe_drain (the mirrored plan is computed over the submitted
  * stream). */
 #define NASPIPE_FLAG_MIRROR 32
+/* Timing-driven execution (Alg.1 P:L170-197 run on OBSERVED completions,
+ * Alg.3's predictor P:L239-273 evaluated online; reading A39): instead of walking
+ * the logical-time plan, the host polls each stage's running task (a CUDA event) and, the
+ * moment a stage is free, picks its next task by Alg.1 + Alg.2 with the state it observes:
+ * the lowest-id backward whose output gradient has arrived, else the lowest-id queued forward
+ * whose input has arrived and whose candidates' previous users have finished their backward
+ * on this stage (Def.2), stage 0 admitting y < (lowest unfinished id) + W.  At every backward
+ * start the stage runs Alg.3's prediction of its next forward (Alg.2 on its queue with the
+ * starting backward counted finished); naspipe_get_timed_stats reports how often it was right.
+ * The schedule depends on kernel timing (it is not unique); the numerics do not (CSP): results
+ * are bitwise those of the planned executor.  naspipe_create only, CSP with strict
+ * backward-first, every candidate resident, no mirroring (EINVAL otherwise).  Tasks run at
+ * naspipe_drain over the submitted stream; the trace's t is microseconds since that drain. */
+#define NASPIPE_FLAG_TIMED 64
 
 /*
  * Supernet specification.  naspipe_create deep-copies it and every array it points to.
@@ -286,6 +300,12 @@ int naspipe_set_timing(naspipe_t* h, int on);
 
 /* Residency trace: 4 int64 per event (stage, task index, op 0=LOAD/1=EVICT, uid=b*n+c). */
 int naspipe_get_residency_trace(naspipe_t* h, int64_t* dst, size_t cap, size_t* n);
+
+/* NASPIPE_FLAG_TIMED engines: dst[0] tasks issued by the timing-driven executor, [1] backward
+ * starts, [2] Alg.3 predictions made at those starts (a queued forward was admissible), [3]
+ * predictions equal to the forward the stage actually ran next, [4] host decision-loop
+ * wall time (ms), [5] reserved.  Zeros for other engines. */
+int naspipe_get_timed_stats(naspipe_t* h, double* dst6);
 
 void naspipe_destroy(naspipe_t* h); /* implies drain; NULL is a no-op */
 

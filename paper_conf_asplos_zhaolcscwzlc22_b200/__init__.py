@@ -12,5 +12,5 @@ from ._lib import (  # noqa: F401
     naspipe_init_params, naspipe_init_frozen, naspipe_nccl_unique_id, naspipe_param_count, naspipe_partition,
     naspipe_plan, naspipe_plan_mirrored, naspipe_set_params, naspipe_set_timing, naspipe_submit, lib, BATCH_HOST, BATCH_DEVICE,
     BATCH_SYNTHETIC, FLAG_TRACE, FLAG_VERSION_CHECK, FLAG_NULL_KERNELS, FLAG_TIMING, FLAG_RECOMPUTE, FLAG_MIRROR,
-    STATS_FIELDS, EXPORTED_SYMBOLS,
+    FLAG_TIMED, naspipe_get_timed_stats, TIMED_FIELDS, STATS_FIELDS, EXPORTED_SYMBOLS,
 )

@@ -16,6 +16,7 @@ FAMILY = {"mlp": 0, "transformer": 1, "spos": 2}
 DTYPE = {"fp32": 0, "bf16": 1}
 BATCH_HOST, BATCH_DEVICE, BATCH_SYNTHETIC = 0, 1, 2
 FLAG_TRACE, FLAG_VERSION_CHECK, FLAG_NULL_KERNELS, FLAG_TIMING, FLAG_RECOMPUTE, FLAG_MIRROR = 1, 2, 4, 8, 16, 32
+FLAG_TIMED = 64
 STATS_FIELDS = ["tasks", "kernel_launches", "h2d_bytes", "d2h_bytes", "p2p_bytes", "makespan_ticks",
                 "dominant_launches", "dominant_flops", "dominant_ms", "res_loads", "res_evicts",
                 "writebacks", "version_checks", "gemm_flops", "gemm_launches", "r15"]
@@ -66,6 +67,7 @@ _sig("naspipe_get_trace", C.c_int, [C.c_void_p, _i64p, C.c_size_t, C.POINTER(C.c
 _sig("naspipe_get_stats", C.c_int, [C.c_void_p, C.POINTER(C.c_double)])
 _sig("naspipe_set_timing", C.c_int, [C.c_void_p, C.c_int])
 _sig("naspipe_get_residency_trace", C.c_int, [C.c_void_p, _i64p, C.c_size_t, C.POINTER(C.c_size_t)])
+_sig("naspipe_get_timed_stats", C.c_int, [C.c_void_p, C.POINTER(C.c_double)])
 _sig("naspipe_destroy", None, [C.c_void_p])
 _sig("naspipe_param_count", C.c_int, [_SP, C.c_int32, C.c_int32, C.POINTER(C.c_size_t)])
 _sig("naspipe_default_costs", C.c_int, [_SP, _i32p, _i32p])
@@ -97,7 +99,8 @@ EXPORTED_SYMBOLS = [
     "naspipe_plan_makespan", "naspipe_plan_deps", "naspipe_plan_residency", "naspipe_plan_destroy",
     "naspipe_plan_comm_schedule", "naspipe_plan_idle", "naspipe_plan_mirrored",
     "naspipe_nccl_unique_id", "naspipe_last_error", "naspipe_abi_version",
-    "naspipe_create_rank_peer", "naspipe_peer_export", "naspipe_peer_connect", "naspipe_set_pdl"]
+    "naspipe_create_rank_peer", "naspipe_peer_export", "naspipe_peer_connect", "naspipe_set_pdl",
+    "naspipe_get_timed_stats"]
 
 
 class NaspipeError(RuntimeError):
@@ -300,6 +303,17 @@ def naspipe_get_stats(h: Handle) -> dict:
     out = (C.c_double * 16)()
     _check(lib.naspipe_get_stats(h.ptr, out))
     return dict(zip(STATS_FIELDS, list(out)))
+
+
+TIMED_FIELDS = ("tasks", "backwards", "predictions", "hits", "host_ms", "reserved")
+
+
+def naspipe_get_timed_stats(h: Handle) -> dict:
+    """Timing-driven executor (FLAG_TIMED) counters: tasks issued, backward starts, Alg.3
+    predictions made at them, predictions that were the stage's next forward, host loop ms."""
+    out = (C.c_double * 6)()
+    _check(lib.naspipe_get_timed_stats(h.ptr, out))
+    return dict(zip(TIMED_FIELDS, list(out)))
 
 
 def naspipe_set_timing(h: Handle, on: bool) -> None:

@@ -339,6 +339,8 @@ int naspipe_get_stats(naspipe_t* h, double* dst16) { return ENGINE_CALL(h, e.get
 
 int naspipe_set_timing(naspipe_t* h, int on) { return ENGINE_CALL(h, e.set_timing(on != 0)); }
 
+int naspipe_get_timed_stats(naspipe_t* h, double* dst6) { return ENGINE_CALL(h, e.get_timed_stats(dst6)); }
+
 int naspipe_get_residency_trace(naspipe_t* h, int64_t* dst, size_t cap, size_t* n) {
   return ENGINE_CALL(h, e.get_residency_trace(dst, cap, n));
 }

@@ -11,6 +11,10 @@
 #include <cstring>
 
 #include "engine.h"
+
+#include <chrono>
+#include <set>
+#include <thread>
 #include "launch.h"
 #include "mirror.h"
 
@@ -120,8 +124,13 @@ std::unique_ptr<Engine> Engine::create_local(const Spec& spec, int D) {
   NP_REQUIRE(!mirror || (spec.raw.sync_policy == NASPIPE_SYNC_CSP && spec.raw.bwd_policy == 0 &&
                          spec.raw.hbm_weight_budget_bytes == 0 && !(spec.raw.flags & NASPIPE_FLAG_RECOMPUTE)),
              NASPIPE_EINVAL, "layer mirroring: CSP, strict backward-first, all candidates resident, no recompute");
+  const bool timed = (spec.raw.flags & NASPIPE_FLAG_TIMED) != 0;
+  NP_REQUIRE(!timed || (spec.raw.sync_policy == NASPIPE_SYNC_CSP && spec.raw.bwd_policy == 0 &&
+                        spec.raw.hbm_weight_budget_bytes == 0 && !mirror),
+             NASPIPE_EINVAL, "timing-driven execution: CSP, strict backward-first, all candidates resident, no mirroring");
   std::unique_ptr<Engine> e(new Engine(spec, D));
   e->mirror_ = mirror;
+  e->timed_ = timed;
   e->st_.resize(D);
   e->stage_sizes();
   for (int K = 0; K < D; ++K) e->setup_stage(K, (cur + K) % ndev, true);
@@ -137,6 +146,13 @@ std::unique_ptr<Engine> Engine::create_local(const Spec& spec, int D) {
       CU(cudaSetDevice(e->st_[K].dev));
       CU(cudaStreamCreateWithFlags(&e->push_[K], cudaStreamNonBlocking));
       CU(cudaEventCreateWithFlags(&e->ev_wrote_[K], cudaEventDisableTiming));
+    }
+  }
+  if (timed) {
+    e->ev_run_.resize(D);
+    for (int K = 0; K < D; ++K) {
+      CU(cudaSetDevice(e->st_[K].dev));
+      CU(cudaEventCreateWithFlags(&e->ev_run_[K], cudaEventDisableTiming));
     }
   }
   CU(cudaSetDevice(cur));
@@ -456,12 +472,12 @@ int64_t Engine::submit(const int32_t* choice, const naspipe_batch* batch) {
     NP_REQUIRE(choice[b] >= 0 && choice[b] < spec_.n(), NASPIPE_EINVAL, "choice[%d]=%d outside [0,%d)", b,
                choice[b], spec_.n());
   if (drained_) {
-    planner_.reopen();
+    if (!mirror_ && !timed_) planner_.reopen();  // those two schedule at drain, not through the plan
     drained_ = false;
   }
   const int64_t y = planner_.add_subnet(choice);
   batches_.push_back({*batch});
-  if (mirror_) return y;  // planned and issued at drain (drain_mirrored)
+  if (mirror_ || timed_) return y;  // scheduled and issued at drain (drain_mirrored / drain_timed)
   planner_.advance();
   feed_stores();
   issue_planned();
@@ -470,7 +486,8 @@ int64_t Engine::submit(const int32_t* choice, const naspipe_batch* batch) {
 
 void Engine::drain() {
   if (!drained_ && mirror_) drain_mirrored();
-  if (!drained_ && !mirror_) {
+  if (!drained_ && timed_) drain_timed();
+  if (!drained_ && !mirror_ && !timed_) {
     planner_.finalize();
     planner_.advance();
     NP_REQUIRE(planner_.done(), NASPIPE_EINTERNAL, "planner did not finish");
@@ -588,6 +605,118 @@ void Engine::issue_mirrored(const Task& t) {
     CU(cudaEventRecord(ev_push_[key], push_[t.K]));
     mwriter_[key] = t.K;
   }
+}
+
+// ------------------------------------------------------------------------------ timing-driven execution
+// Alg.1 + Alg.2 on observed completions (NASPIPE_FLAG_TIMED, reading A39): the
+// host keeps, per stage, the forward queue (input arrived), the backward queue (output
+// gradient arrived) and the finished set, learns of completions by polling each stage's
+// running task, and gives a free stage its next task at once: the lowest-id queued backward,
+// else the lowest-id queued forward admissible under Def.2 (every block's previous user
+// dep[y][b] has finished its backward, i.e. its WRITE, on this stage).  Stage 0 admits y <
+// (lowest id unfinished on stage 0) + W (reading A7).  Alg.3 (its backward
+// branch, reading A10): when B(x, K) starts, Alg.2 over K's queue with x counted finished
+// predicts the forward K runs next (the context to prefetch); it is scored against what K
+// actually runs next.  Every realised order is a CSP schedule, so the numerics are those of
+// the planned executor, bitwise.
+void Engine::drain_timed() {
+  const int64_t N = planner_.n_subnets(), base = tbase_;
+  if (N == base) return;
+  const auto t0 = std::chrono::steady_clock::now();
+  auto us_now = [&] {
+    return (int64_t)std::chrono::duration_cast<std::chrono::microseconds>(std::chrono::steady_clock::now() - t0).count();
+  };
+  std::vector<std::set<int64_t>> fq(D_), bq(D_);
+  std::vector<std::vector<uint8_t>> fin(D_, std::vector<uint8_t>((size_t)(N - base), 0));
+  std::vector<int64_t> wm(D_, base);  // lowest id not finished on stage K
+  struct Run {
+    bool on = false;
+    int kind = 0;
+    int64_t y = 0;
+  };
+  std::vector<Run> run(D_);
+  std::vector<int64_t> pred(D_, -1);     // pending Alg.3 prediction per stage (-1: none)
+  std::vector<uint8_t> pending(D_, 0);   // a backward started and K has not run its next task yet
+  auto finished = [&](int K, int64_t x, int64_t extra) { return x < base || x == extra || fin[K][x - base]; };
+  auto admissible = [&](int K, int64_t y, int64_t extra) {
+    for (int b : planner_.blocks_of(K))
+      if (!finished(K, planner_.dep(y, b), extra)) return false;
+    return true;
+  };
+  int64_t next_src = base, done = 0;
+  const int64_t total = 2 * (N - base) * D_;
+  while (done < total) {
+    bool progress = false;
+    for (int K = 0; K < D_; ++K) {  // completions
+      if (!run[K].on) continue;
+      const cudaError_t q = cudaEventQuery(ev_run_[K]);
+      if (q == cudaErrorNotReady) continue;
+      CU(q);
+      const int64_t y = run[K].y;
+      if (run[K].kind == 0) {
+        if (K < D_ - 1) fq[K + 1].insert(y);
+        else bq[K].insert(y);  // the loss ran inside F(y, D-1)
+      } else {
+        fin[K][y - base] = 1;
+        while (wm[K] < N && fin[K][wm[K] - base]) ++wm[K];
+        if (K > 0) bq[K - 1].insert(y);
+      }
+      run[K].on = false;
+      ++done;
+      progress = true;
+    }
+    while (next_src < N && next_src < wm[0] + W_) fq[0].insert(next_src++);  // stage-0 window
+    for (int K = 0; K < D_; ++K) {  // decisions of the free stages
+      if (run[K].on) continue;
+      Task t{0, K, -1, 0};
+      if (!bq[K].empty()) {
+        t.kind = 1;
+        t.y = *bq[K].begin();
+        bq[K].erase(bq[K].begin());
+      } else {
+        for (int64_t y : fq[K])
+          if (admissible(K, y, -1)) {
+            t.kind = 0;
+            t.y = y;
+            break;
+          }
+        if (t.kind == 0) fq[K].erase(t.y);
+      }
+      if (t.kind < 0) continue;
+      if (pending[K]) {  // score the prediction made at the previous backward's start
+        if (pred[K] >= 0 && t.kind == 0 && t.y == pred[K]) tstat_[3] += 1;
+        pending[K] = 0;
+      }
+      if (t.kind == 1) {  // Alg.3: predict K's next forward with t.y counted finished
+        tstat_[1] += 1;
+        pred[K] = -1;
+        for (int64_t y : fq[K])
+          if (admissible(K, y, t.y)) {
+            pred[K] = y;
+            break;
+          }
+        if (pred[K] >= 0) tstat_[2] += 1;
+        pending[K] = 1;
+      }
+      t.t = us_now();
+      issue(t);
+      ++issued_;
+      CU(cudaSetDevice(st_[K].dev));
+      CU(cudaEventRecord(ev_run_[K], st_[K].comp));
+      run[K] = {true, t.kind, t.y};
+      tstat_[0] += 1;
+      progress = true;
+    }
+    if (!progress) std::this_thread::yield();
+  }
+  tstat_[4] += (double)us_now() / 1e3;
+  tbase_ = N;
+  issued_ = 0;
+}
+
+void Engine::get_timed_stats(double* o) {
+  NP_REQUIRE(o, NASPIPE_EINVAL, "dst NULL");
+  std::copy(tstat_, tstat_ + 6, o);
 }
 
 void Engine::version_check(const Task& t) {

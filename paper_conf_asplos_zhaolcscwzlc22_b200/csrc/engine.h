@@ -58,6 +58,7 @@ class Engine {
   void get_losses(float* dst, int64_t n);
   void get_trace(int64_t* dst, size_t cap, size_t* n);
   void get_stats(double* dst16);
+  void get_timed_stats(double* dst6);
   void set_timing(bool on);
   void get_residency_trace(int64_t* dst, size_t cap, size_t* n);
   void shutdown();
@@ -77,6 +78,7 @@ class Engine {
   void issue(const Task& t);
   void issue_forward(StageRt& st, int64_t y, int slot);
   void drain_mirrored();
+  void drain_timed();
   void issue_mirrored(const Task& t);
   void issue_backward(StageRt& st, int64_t y, int slot);
   void version_check(const Task& t);
@@ -97,6 +99,12 @@ class Engine {
   std::vector<cudaEvent_t> ev_push_;   // per candidate: its last push to the other stages
   std::vector<cudaStream_t> push_;     // per stage
   std::vector<cudaEvent_t> ev_wrote_;  // per stage: the backward whose WRITEs are pushed
+  // timing-driven execution (NASPIPE_FLAG_TIMED): one running task per stage, observed
+  // through ev_run_[K]; subnets [tbase_, N) run at the next drain
+  bool timed_ = false;
+  int64_t tbase_ = 0;
+  std::vector<cudaEvent_t> ev_run_;
+  double tstat_[6] = {0, 0, 0, 0, 0, 0};
   std::vector<BatchRec> batches_;
   std::vector<int32_t> stage_choice_;  // scratch
   size_t issued_ = 0;
