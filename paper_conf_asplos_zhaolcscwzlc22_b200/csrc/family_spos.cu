@@ -110,6 +110,20 @@ class SposFamily : public Family {
     cudaMemset(acc_f_, 0, (2 * C_max + 1) * 8);
     cudaMemset(acc_b_, 0, (2 * C_max + 1) * 8);
     cudaMemset(acc_f2_, 0, (2 * C_max + 1) * 8);
+    // ticket-free BatchNorm (kernels.h BnWrite note): rings of 3 accumulators per direction;
+    // the fused-producer experiments keep the ticket path
+    tfree_ = !fuse_bna_ && !fuse_bnb_ && !fuse_bnb_gemm_ && !getenv("NASPIPE_BN_TICKETS");  // A/B knob
+    if (tfree_)
+      for (int i = 0; i < 3; ++i) {
+        ringF_[i] = A.alloc<unsigned long long>(2 * C_max + 1);
+        ringB_[i] = A.alloc<unsigned long long>(2 * C_max + 1);
+        cudaMemset(ringF_[i], 0, (2 * C_max + 1) * 8);
+        cudaMemset(ringB_[i], 0, (2 * C_max + 1) * 8);
+      }
+    if (tfree_) {
+      acc_f_ = ringF_[0];
+      acc_b_ = ringB_[0];
+    }
     C_max_ = (int)C_max;
     cudaMemset(tick_, 0, 4 * sizeof(int));
     dwk_max_ = dwk_max;
@@ -214,6 +228,11 @@ class SposFamily : public Family {
       block_bwd(j, c, k, g, out, need_dx, s);
       g = out;
     }
+    if (tfree_ && bpend_.acc != nullptr) {  // the task's last deferred gamma / beta WRITE
+      bn_write_flush(s, bpend_);
+      bpend_ = BnWrite();
+      counters.launches++;
+    }
     // the task ends when its weight updates have landed (the next task may read them)
     cudaEventRecord(ev_join_, side_);
     cudaStreamWaitEvent(s, ev_join_, 0);
@@ -258,7 +277,18 @@ class SposFamily : public Family {
   void check_after_drain() override {
     bool bad = false;  // a flag at acc[2C] of any use; the accumulators are zero elsewhere after a drain
     std::vector<unsigned long long> h(2 * (size_t)C_max_ + 1);
-    for (const unsigned long long* a : {acc_f_, acc_b_, acc_f2_}) {
+    std::vector<unsigned long long*> accs = {acc_f_, acc_b_, acc_f2_};
+    if (tfree_) {
+      // the last forward use's slot is cleared by the next use's apply: check its flag, clear it here
+      unsigned long long* last = ringF_[(fu_ + 2) % 3];
+      unsigned long long flag = 0;
+      cudaMemcpy(&flag, last + fprev_n_, 8, cudaMemcpyDeviceToHost);
+      bad |= flag != 0;
+      cudaMemset(last, 0, ((size_t)fprev_n_ + 1) * 8);
+      fprev_n_ = 0;
+      accs = {ringF_[0], ringF_[1], ringF_[2], ringB_[0], ringB_[1], ringB_[2], acc_f2_};
+    }
+    for (const unsigned long long* a : accs) {
       cudaMemcpy(h.data(), a, h.size() * 8, cudaMemcpyDeviceToHost);
       for (auto v : h) bad |= v != 0;
     }
@@ -307,7 +337,13 @@ class SposFamily : public Family {
   void t_bn_apply(cudaStream_t s, const bf16* z, int Pp, int C, float* mean, float* rstd, const float* g,
                   const float* b, int relu, bf16* y, int ldy, size_t yplane, unsigned long long* acc) {
     if (timer) timer->begin(s);
-    bn_apply(s, z, Pp, C, acc, tick_, mean, rstd, g, b, relu, y, ldy, yplane);
+    if (tfree_) {  // acc == ringF_[fu_ % 3]; zero the previous use's slot
+      bn_apply(s, z, Pp, C, acc, nullptr, mean, rstd, g, b, relu, y, ldy, yplane, ringF_[(fu_ + 2) % 3], fprev_n_);
+      fprev_n_ = 2 * C;
+      acc_f_ = ringF_[++fu_ % 3];
+    } else {
+      bn_apply(s, z, Pp, C, acc, tick_, mean, rstd, g, b, relu, y, ldy, yplane);
+    }
     if (timer) timer->end(s, 8.0 * Pp * C);
   }
   void t_bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int Pp, int C, const float* mean,
@@ -320,7 +356,20 @@ class SposFamily : public Family {
                       const float* rstd, const float* g, const float* b, float* gu, float* bu, int update, int relu,
                       bf16* dz) {
     if (timer) timer->begin(s);
-    bn_bwd_apply(s, dy, lddy, z, Pp, C, mean, rstd, g, b, gu, bu, lr_, update, acc_b_, tick_ + 1, relu, dz);
+    if (tfree_) {  // acc_b_ == ringB_[bu_ % 3]; the previous use's WRITE is performed by this launch
+      bn_bwd_apply(s, dy, lddy, z, Pp, C, mean, rstd, g, b, gu, bu, lr_, update, acc_b_, nullptr, relu, dz, bpend_);
+      bpend_.gu = gu;
+      bpend_.bu = bu;
+      bpend_.g = g;
+      bpend_.b = b;
+      bpend_.acc = acc_b_;
+      bpend_.C = C;
+      bpend_.update = update;
+      bpend_.lr = lr_;
+      acc_b_ = ringB_[++bu_ % 3];
+    } else {
+      bn_bwd_apply(s, dy, lddy, z, Pp, C, mean, rstd, g, b, gu, bu, lr_, update, acc_b_, tick_ + 1, relu, dz);
+    }
     if (timer) timer->end(s, 8.0 * Pp * C);
   }
 
@@ -571,6 +620,12 @@ class SposFamily : public Family {
   float* ws_;
   unsigned long long *acc_f_, *acc_b_;  // BatchNorm fixed-point accumulators (forward / backward)
   unsigned long long* acc_f2_;          // forward sums of a depthwise conv that reads acc_f_ (BN on load)
+  // ticket-free mode: acc_f_ / acc_b_ point at ring slot fu_ % 3 / bu_ % 3 of the next use
+  bool tfree_ = false;
+  unsigned long long *ringF_[3] = {}, *ringB_[3] = {};
+  int64_t fu_ = 0, bu_ = 0;
+  int fprev_n_ = 0;  // 2 C of the previous forward use (its slot is zeroed by the next apply)
+  BnWrite bpend_;    // the backward WRITE deferred to the next apply (or the task's flush)
   unsigned long long* acc_w_ = nullptr; // depthwise weight gradient accumulator (side stream)
   size_t dwk_max_ = 0;
   int* tick_;                           // [2] arrival tickets of bn_apply / bn_bwd_apply

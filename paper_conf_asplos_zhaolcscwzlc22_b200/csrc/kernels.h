@@ -175,12 +175,30 @@ void spos_stem_conv(cudaStream_t s, const float* x, const float* w, bf16* z, int
 // order, no finalize launch.  The consumer kernel (bn_apply / bn_bwd_apply) derives the
 // per-channel results from acc in every CTA; its last CTA (ticket: an int, 0 between uses)
 // publishes them and zeroes acc and the ticket.
+// Ticket-free ("ring") mode of the apply kernels (ticket == nullptr): the producers of
+// consecutive BatchNorm uses add into a ring of 3 accumulators, so the apply kernel of use u
+// needs no arrival ticket (round 2: the last-CTA ticket, its fences and the serial tail cost
+// ~2 us per launch): CTA 0 publishes mean / rstd itself and zeroes `clear` [0, clear_n) -- the
+// ring slot of use u-1, whose reader has finished and whose next producer (use u+2) runs
+// after this kernel.  The backward's gamma / beta WRITE of use u cannot be done inside its own
+// apply (other CTAs still read the pre-update values), so it is deferred: CTA 0 of the NEXT
+// backward apply performs use u-1's WRITE (`prev`) and zeroes its slot, and bn_write_flush
+// performs the task's last one.
+struct BnWrite {
+  float *gu = nullptr, *bu = nullptr;        // the WRITE targets (g, b in place; the BSP accumulator)
+  const float *g = nullptr, *b = nullptr;    // the values the update starts from when gu == g / bu == b
+  unsigned long long* acc = nullptr;         // the use's sums (nullptr: nothing pending); zeroed after
+  int C = 0, update = 0;
+  float lr = 0.f;
+};
+void bn_write_flush(cudaStream_t s, const BnWrite& w);
 // acc <- (sum z, sum z^2) of z (x2) over its P rows
 void bn_stats(cudaStream_t s, const bf16* z, int P, int C, unsigned long long* acc);
 // y[p*ldy + c] = relu?(g (z - mean) rstd + b) with mean, rstd from acc; z x2 (plane P*C), y
 // x2 (planes yplane apart); writes mean, rstd [C] (for the backward), clears acc
 void bn_apply(cudaStream_t s, const bf16* z, int P, int C, unsigned long long* acc, int* ticket, float* mean,
-              float* rstd, const float* g, const float* b, int relu, bf16* y, int ldy, size_t yplane);
+              float* rstd, const float* g, const float* b, int relu, bf16* y, int ldy, size_t yplane,
+              unsigned long long* clear = nullptr, int clear_n = 0);
 // acc <- (s1 = sum dy', s2 = sum dy' xh) (dy' = dy masked by the ReLU of the forward)
 void bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
                    const float* rstd, const float* g, const float* b, int relu, unsigned long long* acc);
@@ -189,7 +207,7 @@ void bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int 
 // A30); clears acc
 void bn_bwd_apply(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
                   const float* rstd, const float* g, const float* b, float* gu, float* bu, float lr, int update,
-                  unsigned long long* acc, int* ticket, int relu, bf16* dz);
+                  unsigned long long* acc, int* ticket, int relu, bf16* dz, const BnWrite& prev = BnWrite());
 // acc holds 2C sums + the sticky overflow flag acc[2C] (fixpoint.cuh; checked at drain)
 bool bn_fix_overflow(const unsigned long long* acc, int C);
 // depthwise k x k (k in {3,5,7}), stride S, dilation dil (1 or 2), pad dil*(k/2); w fp32 [C][k][k];

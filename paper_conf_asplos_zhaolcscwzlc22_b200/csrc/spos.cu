@@ -235,12 +235,23 @@ __global__ void bn_stats_kernel(const bf16* __restrict__ z, int P, int C, int ro
 // group's per-channel parameters in registers and strides over pixels.
 __device__ __forceinline__ int ew_lanes(int C) { return TPB / (C / 8); }
 
+template <int U>  // pixels in flight per thread
 __device__ __forceinline__ void bn_apply_body(const bf16* __restrict__ z, int P, int C, const unsigned long long* acc,
                                               const float* __restrict__ gam, const float* __restrict__ bet, int relu,
-                                              bf16* __restrict__ y, int ldy, size_t yplane) {
+                                              bf16* __restrict__ y, int ldy, size_t yplane, float* mean = nullptr,
+                                              float* rstd = nullptr, unsigned long long* clear = nullptr,
+                                              int clear_n = 0) {
   // the CTA derives every channel's moments once (fp64, from the fixed-point totals)
   __shared__ float smu[2048], srs[2048];  // C <= 8 TPB = 2048 (host check)
-  for (int cc = threadIdx.x; cc < C; cc += blockDim.x) bn_moments(acc, C, cc, P, smu[cc], srs[cc]);
+  for (int cc = threadIdx.x; cc < C; cc += blockDim.x) {
+    bn_moments(acc, C, cc, P, smu[cc], srs[cc]);
+    if (mean != nullptr && blockIdx.x == 0) {  // ring mode: CTA 0 publishes (same values in every CTA)
+      mean[cc] = smu[cc];
+      rstd[cc] = srs[cc];
+    }
+  }
+  if (clear != nullptr && blockIdx.x == 0)
+    for (int e = threadIdx.x; e < clear_n; e += blockDim.x) clear[e] = 0ull;
   __syncthreads();
   const int G = C / 8, lanes = ew_lanes(C);
   const int pl = threadIdx.x / G, c = (threadIdx.x % G) * 8;
@@ -256,12 +267,12 @@ __device__ __forceinline__ void bn_apply_body(const bf16* __restrict__ z, int P,
   const size_t zplane = (size_t)P * C;
   const int step = gridDim.x * lanes;
   int p = blockIdx.x * lanes + pl;
-  for (; p + step < P; p += 2 * step) {  // two pixels in flight
-    float v[2][8];
-    load8x2(z + (size_t)p * C + c, zplane, v[0]);
-    load8x2(z + (size_t)(p + step) * C + c, zplane, v[1]);
+  for (; p + (U - 1) * step < P; p += U * step) {  // U pixels in flight
+    float v[U][8];
 #pragma unroll
-    for (int u = 0; u < 2; ++u) {
+    for (int u = 0; u < U; ++u) load8x2(z + (size_t)(p + u * step) * C + c, zplane, v[u]);
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
         const float o = bn_y(v[u][i], mu[i], rs[i], g8[i], b8[i]);
@@ -282,12 +293,17 @@ __device__ __forceinline__ void bn_apply_body(const bf16* __restrict__ z, int P,
   }
 }
 
+template <int U>
 __global__ void bn_apply_kernel(const bf16* __restrict__ z, int P, int C, unsigned long long* acc, int* ticket,
                                 float* __restrict__ mean, float* __restrict__ rstd, const float* __restrict__ gam,
                                 const float* __restrict__ bet, int relu, bf16* __restrict__ y, int ldy,
-                                size_t yplane) {
+                                size_t yplane, unsigned long long* clear, int clear_n) {
   ptx::pdl_wait();
-  bn_apply_body(z, P, C, acc, gam, bet, relu, y, ldy, yplane);
+  if (ticket == nullptr) {  // ring mode (kernels.h BnWrite note): no ticket, no fence, no serial tail
+    bn_apply_body<U>(z, P, C, acc, gam, bet, relu, y, ldy, yplane, mean, rstd, clear, clear_n);
+    return;
+  }
+  bn_apply_body<U>(z, P, C, acc, gam, bet, relu, y, ldy, yplane);
   if (last_cta(ticket)) {  // every CTA has read the totals: publish mean / rstd, clear
     for (int c = threadIdx.x; c < C; c += blockDim.x) {
       float mu, rs;
@@ -396,6 +412,7 @@ __global__ void bn_bwd_reduce_kernel(const bf16* __restrict__ dy, int lddy, cons
   }
 }
 
+template <int U>  // pixels in flight per thread
 __device__ __forceinline__ void bn_bwd_apply_body(const bf16* __restrict__ dy, int lddy, const bf16* __restrict__ z,
                                                   int P, int C, const float* __restrict__ mean,
                                                   const float* __restrict__ rstd, const float* __restrict__ gam,
@@ -424,14 +441,14 @@ __device__ __forceinline__ void bn_bwd_apply_body(const bf16* __restrict__ dy, i
   const size_t zplane = (size_t)P * C;
   const int step = gridDim.x * lanes;
   int p = blockIdx.x * lanes + pl;
-  for (; p + step < P; p += 2 * step) {  // two pixels in flight
-    float d[2][BV], xh[2][BV];
+  for (; p + (U - 1) * step < P; p += U * step) {  // U pixels in flight
+    float d[U][BV], xh[U][BV];
 #pragma unroll
-    for (int u = 0; u < 2; ++u)
+    for (int u = 0; u < U; ++u)
       bn_bwd_item(dy + (size_t)(p + u * step) * lddy + c, z + (size_t)(p + u * step) * C + c, zplane, mu, rs, g8, b8,
                   relu, d[u], xh[u]);
 #pragma unroll
-    for (int u = 0; u < 2; ++u) {
+    for (int u = 0; u < U; ++u) {
 #pragma unroll
       for (int i = 0; i < BV; ++i) d[u][i] = rs[i] * g8[i] * (d[u][i] - m1[i] - xh[u][i] * m2[i]);
       store4(dz + (size_t)(p + u * step) * C + c, d[u]);
@@ -450,12 +467,37 @@ __device__ __forceinline__ void bn_bwd_apply_body(const bf16* __restrict__ dy, i
 // gradient uses the weights before the WRITE); the last CTA -- after every CTA has read
 // g, b -- applies the WRITE g -= lr s2, b -= lr s1 (into gu/bu: g/b in place, the bulk
 // accumulator under BSP) and clears acc and the ticket.
+// the deferred WRITE of a previous use (ring mode): g -= lr s2, b -= lr s1, then zero its sums
+__device__ __forceinline__ void bn_write(const BnWrite& w) {
+  if (w.acc == nullptr) return;
+  if (w.update)
+    for (int c = threadIdx.x; c < w.C; c += blockDim.x) {
+      const float f1 = (float)fix_get(w.acc, c, FIX_B), f2 = (float)fix_get(w.acc, w.C + c, FIX_B);
+      w.gu[c] = (w.gu == w.g ? w.g[c] : w.gu[c]) - w.lr * f2;
+      w.bu[c] = (w.bu == w.b ? w.b[c] : w.bu[c]) - w.lr * f1;
+    }
+  __syncthreads();  // every thread has read the sums
+  for (int e = threadIdx.x; e < 2 * w.C; e += blockDim.x) w.acc[e] = 0ull;
+}
+
+__global__ void bn_write_kernel(const BnWrite w) {
+  ptx::pdl_wait();
+  bn_write(w);
+}
+
+template <int U>
 __global__ void bn_bwd_apply_kernel(const bf16* __restrict__ dy, int lddy, const bf16* __restrict__ z, int P, int C,
                                     const float* __restrict__ mean, const float* __restrict__ rstd, const float* gam,
                                     const float* bet, float* gamu, float* betu, float lr, int update,
-                                    unsigned long long* acc, int* ticket, int relu, bf16* __restrict__ dz) {
+                                    unsigned long long* acc, int* ticket, int relu, bf16* __restrict__ dz,
+                                    const BnWrite prev) {
   ptx::pdl_wait();
-  bn_bwd_apply_body(dy, lddy, z, P, C, mean, rstd, gam, bet, acc, relu, dz);
+  if (ticket == nullptr) {  // ring mode: CTA 0 first performs the previous use's deferred WRITE
+    if (blockIdx.x == 0) bn_write(prev);
+    bn_bwd_apply_body<U>(dy, lddy, z, P, C, mean, rstd, gam, bet, acc, relu, dz);
+    return;
+  }
+  bn_bwd_apply_body<U>(dy, lddy, z, P, C, mean, rstd, gam, bet, acc, relu, dz);
   if (last_cta(ticket)) {
     if (update)
       for (int c = threadIdx.x; c < C; c += blockDim.x) {
@@ -1240,6 +1282,15 @@ static int red_blocks(int P, int C, int vec = 8, int target = 0) {
   return (P + r - 1) / r;
 }
 
+// pixels in flight per thread in the BatchNorm apply kernels: NASPIPE_BN_UNROLL (2 or 4)
+static int bn_unroll() {
+  static const int v = [] {
+    const char* e = getenv("NASPIPE_BN_UNROLL");
+    return (e && atoi(e) == 4) ? 4 : 2;
+  }();
+  return v;
+}
+
 void bn_stats(cudaStream_t s, const bf16* z, int P, int C, unsigned long long* acc) {
   NP_REQUIRE(C % 8 == 0 && C / 8 <= TPB, NASPIPE_EINVAL, "bn_stats C=%d", C);
   const size_t sm = red_smem(C);
@@ -1249,10 +1300,15 @@ void bn_stats(cudaStream_t s, const bf16* z, int P, int C, unsigned long long* a
 }
 
 void bn_apply(cudaStream_t s, const bf16* z, int P, int C, unsigned long long* acc, int* ticket, float* mean,
-              float* rstd, const float* g, const float* b, int relu, bf16* y, int ldy, size_t yplane) {
+              float* rstd, const float* g, const float* b, int relu, bf16* y, int ldy, size_t yplane,
+              unsigned long long* clear, int clear_n) {
   NP_REQUIRE(C % 8 == 0 && C / 8 <= TPB, NASPIPE_EINVAL, "bn_apply C=%d", C);
-  launch_pdl(bn_apply_kernel, dim3(ew_grid(bn_apply_kernel, P, C)), dim3(TPB), 0, s, z, P, C, acc, ticket, mean, rstd,
-             g, b, relu, y, ldy, yplane);
+  if (bn_unroll() == 4)
+    launch_pdl(bn_apply_kernel<4>, dim3(ew_grid(bn_apply_kernel<4>, P, C)), dim3(TPB), 0, s, z, P, C, acc, ticket, mean,
+               rstd, g, b, relu, y, ldy, yplane, clear, clear_n);
+  else
+    launch_pdl(bn_apply_kernel<2>, dim3(ew_grid(bn_apply_kernel<2>, P, C)), dim3(TPB), 0, s, z, P, C, acc, ticket, mean,
+               rstd, g, b, relu, y, ldy, yplane, clear, clear_n);
   check_launch("bn_apply");
 }
 
@@ -1272,11 +1328,21 @@ void bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int 
 
 void bn_bwd_apply(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int P, int C, const float* mean,
                   const float* rstd, const float* g, const float* b, float* gu, float* bu, float lr, int update,
-                  unsigned long long* acc, int* ticket, int relu, bf16* dz) {
+                  unsigned long long* acc, int* ticket, int relu, bf16* dz, const BnWrite& prev) {
   NP_REQUIRE(C % 8 == 0 && C / BV <= TPB, NASPIPE_EINVAL, "bn_bwd_apply C=%d", C);
-  launch_pdl(bn_bwd_apply_kernel, dim3(ew_grid(bn_bwd_apply_kernel, P, C, BV)), dim3(TPB), 0, s, dy, lddy, z, P, C, mean,
-             rstd, g, b, gu, bu, lr, update, acc, ticket, relu, dz);
+  if (bn_unroll() == 4)
+    launch_pdl(bn_bwd_apply_kernel<4>, dim3(ew_grid(bn_bwd_apply_kernel<4>, P, C, BV)), dim3(TPB), 0, s, dy, lddy, z, P,
+               C, mean, rstd, g, b, gu, bu, lr, update, acc, ticket, relu, dz, prev);
+  else
+    launch_pdl(bn_bwd_apply_kernel<2>, dim3(ew_grid(bn_bwd_apply_kernel<2>, P, C, BV)), dim3(TPB), 0, s, dy, lddy, z, P,
+               C, mean, rstd, g, b, gu, bu, lr, update, acc, ticket, relu, dz, prev);
   check_launch("bn_bwd_apply");
+}
+
+void bn_write_flush(cudaStream_t s, const BnWrite& w) {
+  if (w.acc == nullptr) return;
+  launch_pdl(bn_write_kernel, dim3(1), dim3(TPB), 0, s, w);
+  check_launch("bn_write_flush");
 }
 
 bool bn_fix_overflow(const unsigned long long* acc, int C) {

@@ -56,8 +56,21 @@ def main():
             a = agg.setdefault(n, [0, 0.0])
             a[0] += 1
             a[1] += e["dur"]
+        durs = {}
+        for e in v:
+            n = e["name"].replace("(anonymous namespace)::", "").replace("void ", "").split("(")[0][-70:]
+            durs.setdefault(n, []).append((e["dur"], str(e.get("args", {}).get("grid", ""))))
         for n, (c, t) in sorted(agg.items(), key=lambda kv: -kv[1][1]):
-            print(f"    {t / K:8.1f} us {c / K:6.1f}x  {t / c:7.2f} us/launch  {n}")
+            d = sorted(x for x, _ in durs[n])
+            q = lambda f: d[min(len(d) - 1, int(f * len(d)))]  # noqa: E731
+            print(f"    {t / K:8.1f} us {c / K:6.1f}x  {t / c:7.2f} us/launch  [min {d[0]:.1f} p50 {q(0.5):.1f} "
+                  f"p90 {q(0.9):.1f} max {d[-1]:.1f}]  {n}")
+            if os.environ.get("KT_GRIDS") and ("bn_" in n or "dw_" in n):
+                by = {}
+                for x, g in durs[n]:
+                    by.setdefault(g, []).append(x)
+                for g, xs in sorted(by.items(), key=lambda kv: -sum(kv[1])):
+                    print(f"        grid {g}: {len(xs) / K:.1f}x  mean {sum(xs) / len(xs):.1f} us")
     npipe.naspipe_destroy(h)
 
 
