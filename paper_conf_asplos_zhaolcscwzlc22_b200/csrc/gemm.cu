@@ -401,6 +401,7 @@ __global__ void __launch_bounds__(THREADS, 1)
     const int lane_base = 32 * (warp & 3);
     const int cbeg = ((warp - 2) >> 2) * (TN / 2);
     int it = 0;
+    float run1 = 0.f, run2 = 0.f;  // fused BatchNorm sums of this thread's column over the CTA's tiles
     for (int t = blockIdx.x; t < n_tiles; t += gridDim.x, ++it) {
       int tm, tn, ks;
       ts.decode(t, tm, tn, ks);
@@ -425,9 +426,13 @@ __global__ void __launch_bounds__(THREADS, 1)
           const int half = (warp - 2) >> 2;
           ptx::named_bar_sync(1 + half, 128);
           const float* base = reinterpret_cast<const float*>(smem + Cf::SST_OFF) + half * 4 * (TN / 2) * 2;
-          for (int j = (warp & 3) * 32 + lane; j < TN / 2; j += 128) {
-            const int gcol = tn * TN + cbeg + j;
-            if (gcol >= N) continue;
+          // TN / 2 <= 128: thread (warp & 3, lane) owns column j of the half.  The CTA's tiles of
+          // one column block are summed in tile order in registers and added in fixed point
+          // once, when the next tile of the CTA is in another column block or there is none
+          // (a per-tile add put #tiles atomics -- 1568 on a 200704-row 1x1 conv -- on each address)
+          const int j = (warp & 3) * 32 + lane;
+          const int gcol = tn * TN + cbeg + j;
+          if (j < TN / 2 && gcol < N) {
             float s1 = 0.f, s2 = 0.f;
 #pragma unroll
             for (int q = 0; q < 4; ++q) {  // quarter q is warp 2 + 4 half + ((q + 2) & 3)
@@ -435,8 +440,18 @@ __global__ void __launch_bounds__(THREADS, 1)
               s1 += w[j * 2];
               s2 += w[j * 2 + 1];
             }
-            fix_add(sacc, gcol, sacc + 2 * N, s1, EPI == EPI_BNBWD ? FIX_B : FIX_S1);
-            fix_add(sacc, N + gcol, sacc + 2 * N, s2, EPI == EPI_BNBWD ? FIX_B : FIX_S2);
+            run1 += s1;
+            run2 += s2;
+            int tn_next = -1;
+            if (t + (int)gridDim.x < n_tiles) {
+              int tm2, ks2;
+              ts.decode(t + (int)gridDim.x, tm2, tn_next, ks2);
+            }
+            if (tn_next != tn) {
+              fix_add(sacc, gcol, sacc + 2 * N, run1, EPI == EPI_BNBWD ? FIX_B : FIX_S1);
+              fix_add(sacc, N + gcol, sacc + 2 * N, run2, EPI == EPI_BNBWD ? FIX_B : FIX_S2);
+              run1 = run2 = 0.f;
+            }
           }
           ptx::named_bar_sync(1 + half, 128);  // the slots are rewritten by the next tile
         }
@@ -575,6 +590,7 @@ __global__ void __launch_bounds__(THREADS, 1)
     const int lane_base = 32 * (warp & 3);
     const int cbeg = ((warp - 2) >> 2) * (TN / 2);
     int it = 0;
+    float run1 = 0.f, run2 = 0.f;  // fused BatchNorm sums of this thread's column over the CTA's tiles
     for (int t = pair; t < n_tiles; t += n_pairs, ++it) {
       int tm, tn, ks;
       ts.decode(t, tm, tn, ks);

@@ -58,10 +58,22 @@ constexpr float BN_EPS = 1e-5f;
 
 // Row blocking of the per-channel reductions: a function of (P, C) only (deterministic),
 // about RED_CTAS blocks, each a multiple of the kernel's row lanes RP = TPB / (C/8).
+// Each row lane handles at least NASPIPE_RED_MIN_ITERS rows (default 8; measured 1 / 4 / 8 / 16 /
+// 32: 6.47 / 6.35 / 6.33 / 6.59 / 7.06 ms per configs[1] step): small tensors
+// (the 7x7 / 14x14 stages, P = 3136 / 12544) otherwise spread a few rows over ~700 CTAs, each
+// paying the shared-memory reduction and 2C fixed-point atomics on the same 2C addresses.
+static int red_min_iters() {
+  static const int v = [] {
+    const char* e = getenv("NASPIPE_RED_MIN_ITERS");
+    return e ? std::max(1, atoi(e)) : 8;
+  }();
+  return v;
+}
 inline int red_rows(int P, int C, int vec = 8, int target = 0) {
   const int rp = TPB / (C / vec);
   if (target <= 0) target = red_ctas();
   int rows = (P + target - 1) / target;
+  rows = std::max(rows, rp * red_min_iters());
   rows = ((rows + rp - 1) / rp) * rp;
   return rows < rp ? rp : rows;
 }
