@@ -349,7 +349,7 @@ void Engine::setup_stage(int K, int dev, bool local) {
   st.dev = dev;
   st.local = local;
   CU(cudaSetDevice(dev));
-  CU(cudaStreamCreateWithFlags(&st.comp, cudaStreamNonBlocking));
+  CU(create_stream(&st.comp, true));
   CU(cudaStreamCreateWithFlags(&st.copy, cudaStreamNonBlocking));
   st.arena = std::make_unique<DevArena>(dev);
   std::vector<int> blocks = planner_.blocks_of(K);

@@ -10,6 +10,7 @@
 #include <cstring>
 
 #include "family.h"
+#include "launch.h"
 
 namespace naspipe {
 
@@ -235,7 +236,7 @@ class TfFamily : public Family {
     spec_base_ = &spec;
     n_choices_ = spec.n();
     mse_part_ = A.alloc<float>(mse_blocks(spec.batch_elems()));
-    cudaStreamCreateWithFlags(&side_, cudaStreamNonBlocking);
+    create_stream(&side_, false);
     for (auto* e : {&ev_dz_, &ev_da2_, &ev_do_, &ev_da_, &ev_done_[0], &ev_done_[1], &ev_join_})
       cudaEventCreateWithFlags(e, cudaEventDisableTiming);
   }

@@ -17,6 +17,7 @@
 #include <cstring>
 
 #include "family.h"
+#include "launch.h"
 
 namespace naspipe {
 
@@ -88,7 +89,7 @@ class SposFamily : public Family {
         if (j < nb - 1) act_[k] = A.alloc<bf16>(spec.act_bytes(blocks[j] + 1) / 2);
       }
     for (auto& d : dz_) d = A.alloc<bf16>(dz_max);
-    cudaStreamCreateWithFlags(&side_, cudaStreamNonBlocking);
+    create_stream(&side_, false);
     for (int i = 0; i < kRing; ++i) {
       cudaEventCreateWithFlags(&ev_dg_[i], cudaEventDisableTiming);
       cudaEventCreateWithFlags(&ev_wg_[i], cudaEventDisableTiming);

@@ -24,6 +24,24 @@ namespace naspipe {
 //   flags between kernels (the same cross-stream pattern).
 // The CTA-pair GEMM's early triggers (NASPIPE_PAIR_TRIGGER=1) also still hang
 // tools/hangtest.sh and stay off.
+// Stream priorities: a stage's compute stream (the task's critical chain) gets the highest
+// priority, the families' side streams (weight gradients, hidden behind that chain) the
+// lowest, so the block scheduler prefers the critical chain's CTAs when both streams have
+// work.  NASPIPE_STREAM_PRIO=0: default priorities for both (A/B).
+inline bool stream_prio_on() {
+  static const bool v = [] {
+    const char* e = getenv("NASPIPE_STREAM_PRIO");
+    return !(e && e[0] == '0');
+  }();
+  return v;
+}
+inline cudaError_t create_stream(cudaStream_t* s, bool critical) {
+  int lo = 0, hi = 0;
+  if (!stream_prio_on() || cudaDeviceGetStreamPriorityRange(&lo, &hi) != cudaSuccess)
+    return cudaStreamCreateWithFlags(s, cudaStreamNonBlocking);
+  return cudaStreamCreateWithPriority(s, cudaStreamNonBlocking, critical ? hi : lo);
+}
+
 inline std::atomic<int>& pdl_suppressors() {
   static std::atomic<int> n{0};
   return n;

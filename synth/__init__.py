@@ -57,6 +57,26 @@ CONFIGS = {
                    choice_heads=[h for _ in range(4) for h in (8, 16) for _ in range(3)],
                    choice_ffn=[f for _ in range(8) for f in (1024, 2048, 3072)],
                    lr=0.01, compute_dtype="bf16", n_stages=8, n_subnets=256),
+    # The other Table 1 NLP spaces (48 choice blocks x 96 / 72 / 48 layers), executed
+    # (round 2): each layer a distinct (Table 5 op, heads, FFN width) combination over the
+    # NLP.c3 op set; NLP.c2 fits all-resident in HBM (~18e9 params x 6 B), c1 / c0 run with
+    # context switching (bench --budget-x).
+    "nlp_c2": dict(family="transformer", n_blocks=48, n_choices=48, batch=32, d_model=1024, seq_len=128,
+                   choice_op=[op for op in (0, 1, 2, 3) for _ in range(12)],
+                   choice_heads=[h for _ in range(4) for h in (8, 16) for _ in range(6)],
+                   choice_ffn=[f for _ in range(8) for f in (512, 1024, 1536, 2048, 3072, 4096)],
+                   lr=0.01, compute_dtype="bf16", n_stages=8, n_subnets=256),
+    "nlp_c1": dict(family="transformer", n_blocks=48, n_choices=72, batch=32, d_model=1024, seq_len=128,
+                   choice_op=[op for op in (0, 1, 2, 3) for _ in range(18)],
+                   choice_heads=[h for _ in range(4) for h in (8, 16) for _ in range(9)],
+                   choice_ffn=[f for _ in range(8) for f in (512, 768, 1024, 1536, 2048, 2560, 3072, 3584, 4096)],
+                   lr=0.01, compute_dtype="bf16", n_stages=8, n_subnets=256),
+    "nlp_c0": dict(family="transformer", n_blocks=48, n_choices=96, batch=32, d_model=1024, seq_len=128,
+                   choice_op=[op for op in (0, 1, 2, 3) for _ in range(24)],
+                   choice_heads=[h for _ in range(4) for h in (8, 16) for _ in range(12)],
+                   choice_ffn=[f for _ in range(8) for f in (256, 512, 768, 1024, 1280, 1536, 2048, 2560,
+                                                            3072, 3328, 3584, 4096)],
+                   lr=0.01, compute_dtype="bf16", n_stages=8, n_subnets=256),
     # small supernet with every NLP op (parity tests of A38): Conv 3x1, Sep Conv 7x1, Light
     # Conv 5x1 (H = 4), attention
     "tiny_nlp": dict(family="transformer", n_blocks=4, n_choices=4, batch=2, d_model=192, seq_len=128,
@@ -83,6 +103,19 @@ CONFIGS = {
                   stage_repeats=[8, 8, 8, 8], stage_channels=[64, 160, 320, 640], stem_channels=16,
                   head_channels=1024, choice_kernel=[3, 5, 7] * 4, choice_xception=[0] * 6 + [1] * 6,
                   choice_dilation=[1, 1, 1, 2, 2, 2] * 2,
+                  lr=0.001, compute_dtype="bf16", n_stages=8, n_subnets=256),
+    # The other Table 1 CV spaces (32 choice blocks x 24 / 48 layers), executed
+    # (round 2): CV.c3's 12 op types (Shuffle / Xception x k 3/5/7 x dilation 1/2), each
+    # present 2 / 4 times as separately trained candidates.
+    "cv_c2": dict(family="spos", n_blocks=32, n_choices=24, batch=64, image_hw=224, num_classes=1000,
+                  stage_repeats=[8, 8, 8, 8], stage_channels=[64, 160, 320, 640], stem_channels=16,
+                  head_channels=1024, choice_kernel=[3, 5, 7] * 8, choice_xception=([0] * 6 + [1] * 6) * 2,
+                  choice_dilation=[1, 1, 1, 2, 2, 2] * 4,
+                  lr=0.001, compute_dtype="bf16", n_stages=8, n_subnets=256),
+    "cv_c1": dict(family="spos", n_blocks=32, n_choices=48, batch=64, image_hw=224, num_classes=1000,
+                  stage_repeats=[8, 8, 8, 8], stage_channels=[64, 160, 320, 640], stem_channels=16,
+                  head_channels=1024, choice_kernel=[3, 5, 7] * 16, choice_xception=([0] * 6 + [1] * 6) * 4,
+                  choice_dilation=[1, 1, 1, 2, 2, 2] * 8,
                   lr=0.001, compute_dtype="bf16", n_stages=8, n_subnets=256),
     # small SPOS supernet with dilated candidates (parity tests of A36)
     "tiny_spos_dil": dict(family="spos", n_blocks=5, n_choices=4, batch=4, image_hw=64, num_classes=10,

@@ -69,6 +69,26 @@ def test_spos_layout_and_init_match_oracle(name):
         assert np.array_equal(got.view(np.uint32), ref.view(np.uint32)), key
 
 
+@pytest.mark.parametrize("name,m,n", [("nlp_c0", 48, 96), ("nlp_c1", 48, 72), ("nlp_c2", 48, 48), ("nlp_c3", 48, 24),
+                                      ("cv_c1", 32, 48), ("cv_c2", 32, 24), ("cv_c3", 32, 12)])
+def test_table1_space_configs(name, m, n):
+    """Table 1's spaces as executable configs: m blocks x n candidates, every
+    NLP candidate a distinct (op, heads, FFN) combination over Table 5's NLP ops, every CV
+    candidate one of CV.c3's 12 op types; the library accepts every candidate and its packed
+    size equals the oracle's layout (candidates of block 0 and the last block)."""
+    cfg = synth.get_config(name)
+    assert (cfg["n_blocks"], cfg["n_choices"]) == (m, n)
+    keys = sorted(k for k in cfg if k.startswith("choice_"))
+    assert all(len(cfg[k]) == n for k in keys)
+    kinds = set(zip(*[cfg[k] for k in keys]))
+    assert len(kinds) == (n if cfg["family"] == "transformer" else 12)
+    spec = npipe.Spec(cfg)
+    for b in (0, m - 1):
+        for c in range(n):
+            segs = [int(np.prod(s)) for _, s, _, _ in train.candidate_layout(cfg, b, c)]
+            assert npipe.naspipe_param_count(spec, b, c) == sum(segs), (b, c)
+
+
 def test_nlp_op_spec_validation():
     cfg = synth.get_config("tiny_nlp")
     for bad in (dict(choice_op=[1, 2, 4, 0]), dict(choice_op=[1, 2, -1, 0]), dict(choice_heads=[3, 2, 5, 3])):
