@@ -282,8 +282,7 @@ def secondary(args, workload, extra=(), steps=None):
 
 
 # ------------------------------------------------------------------------------ CUPTI kernel times
-KERNEL_FAMILIES = {"spos": ("bn_stats", "bn_finalize", "bn_apply", "bn_bwd_reduce", "bn_bwd_finalize",
-                            "bn_bwd_apply"),
+KERNEL_FAMILIES = {"spos": ("bn_stats", "bn_apply", "bn_bwd_reduce", "bn_bwd_apply", "bn_write"),
                    "transformer": ("gemm_tc", "gemm_pair")}
 
 

@@ -1281,11 +1281,21 @@ static int gs_grid(Kern kern, size_t items, size_t smem = 0) {
   const size_t g = (items + TPB - 1) / TPB;
   return (int)std::min<size_t>(std::max<size_t>(g, 1), (size_t)num_sms() * occ * gs_waves());
 }
+// minimum pixels per thread of the BatchNorm elementwise kernels (NASPIPE_EW_MIN_PIX, default
+// 1 = one wave whatever the size): every CTA derives all C channels' moments first, so a
+// full wave of CTAs over a 7x7 tensor mostly repeats that prologue
+static int ew_min_pix() {
+  static const int v = [] {
+    const char* e = getenv("NASPIPE_EW_MIN_PIX");
+    return e ? std::max(1, atoi(e)) : 1;
+  }();
+  return v;
+}
 template <typename Kern>
 static int ew_grid(Kern kern, int P, int C, int vec = 8) {
   const int occ = occupancy(kern, 0);
-  const int lanes = TPB / (C / vec);
-  return std::max(1, std::min((P + lanes - 1) / lanes, num_sms() * occ * ew_waves()));
+  const int lanes = TPB / (C / vec), per = lanes * ew_min_pix();
+  return std::max(1, std::min((P + per - 1) / per, num_sms() * occ * ew_waves()));
 }
 
 static size_t red_smem(int C, int vec = 8) { return (size_t)(TPB / (C / vec)) * 2 * C * sizeof(float); }
