@@ -237,6 +237,7 @@ class TfFamily : public Family {
     n_choices_ = spec.n();
     mse_part_ = A.alloc<float>(mse_blocks(spec.batch_elems()));
     create_stream(&side_, false);
+    if (side_stream_sms() > 0) gemm_set_stream_cap(side_, side_stream_sms());
     for (auto* e : {&ev_dz_, &ev_da2_, &ev_do_, &ev_da_, &ev_done_[0], &ev_done_[1], &ev_join_})
       cudaEventCreateWithFlags(e, cudaEventDisableTiming);
   }

@@ -90,6 +90,7 @@ class SposFamily : public Family {
       }
     for (auto& d : dz_) d = A.alloc<bf16>(dz_max);
     create_stream(&side_, false);
+    if (side_stream_sms() > 0) gemm_set_stream_cap(side_, side_stream_sms());
     for (int i = 0; i < kRing; ++i) {
       cudaEventCreateWithFlags(&ev_dg_[i], cudaEventDisableTiming);
       cudaEventCreateWithFlags(&ev_wg_[i], cudaEventDisableTiming);

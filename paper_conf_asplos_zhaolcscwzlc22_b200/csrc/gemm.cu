@@ -17,6 +17,7 @@
 #include <atomic>
 #include <cstdlib>
 #include <mutex>
+#include <vector>
 
 #include "common.h"
 #include "kernels.h"
@@ -702,6 +703,15 @@ std::atomic<uint64_t> g_gemm_launches{0};
 std::atomic<uint64_t> g_gemm_flops{0};  // algorithmic 2*M*N*K of every GEMM call (bf16x2: one product)
 
 
+std::mutex g_cap_mu;
+std::vector<std::pair<cudaStream_t, int>> g_caps;  // per-stream CTA caps (a handful of side streams)
+int stream_cap(cudaStream_t s) {
+  std::lock_guard<std::mutex> lk(g_cap_mu);
+  for (const auto& c : g_caps)
+    if (c.first == s) return c.second;
+  return 0;
+}
+
 template <bool A_MN, bool B_MN, int EPI, int TN = BN, bool SPLIT = false>
 void launch(cudaStream_t s, int M, int N, const TileSpace& ts, const CUtensorMap& ta, const CUtensorMap& tb,
             const GemmEpiParams& ep, const CUtensorMap* ta2 = nullptr, const CUtensorMap* tb2 = nullptr) {
@@ -715,7 +725,8 @@ void launch(cudaStream_t s, int M, int N, const TileSpace& ts, const CUtensorMap
     configured |= 1u << dev;
   }
   const int tiles = ts.MT * ts.NT * ts.splits;
-  const int grid = std::min(tiles, num_sms());
+  const int cap = stream_cap(s);
+  const int grid = std::min(tiles, cap > 0 ? std::min(cap, num_sms()) : num_sms());
   launch_pdl(kern, dim3(grid), dim3(THREADS), SMEM, s, ta, tb, ta2 ? *ta2 : ta, tb2 ? *tb2 : tb, M, N, ts, ep);
   g_gemm_launches.fetch_add(1, std::memory_order_relaxed);
 }
@@ -733,7 +744,8 @@ void launch_pair(cudaStream_t s, int M, int N, const TileSpace& ts, const CUtens
     configured |= 1u << dev;
   }
   const int tiles = ts.MT * ts.NT * ts.splits;
-  const int pairs = std::min(tiles, num_sms() / 2);
+  const int cap = stream_cap(s);
+  const int pairs = std::min(tiles, (cap > 0 ? std::min(cap, num_sms()) : num_sms()) / 2);
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3(2 * pairs);
   cfg.blockDim = dim3(THREADS);
@@ -850,6 +862,24 @@ int num_sms() {
 
 CUtensorMap tma_map_bf16(const bf16* base, uint64_t inner, uint64_t outer, uint64_t ld, uint32_t box_outer) {
   return make_map(base, inner, outer, ld, box_outer);
+}
+
+void gemm_set_stream_cap(cudaStream_t s, int max_ctas) {
+  std::lock_guard<std::mutex> lk(g_cap_mu);
+  for (auto& c : g_caps)
+    if (c.first == s) {
+      c.second = max_ctas;
+      return;
+    }
+  g_caps.emplace_back(s, max_ctas);
+}
+
+int side_stream_sms() {
+  static const int v = [] {
+    const char* e = getenv("NASPIPE_SIDE_SMS");
+    return e ? std::max(0, atoi(e)) : 0;
+  }();
+  return v;
 }
 
 uint64_t gemm_launch_count() { return g_gemm_launches.load(); }

@@ -82,6 +82,12 @@ struct GemmEpiParams {
   unsigned long long* stats = nullptr;
   BnBwdFuse bnb;  // EPI_BNBWD only (stats of the fused BatchNorm backward; 1-CTA kernel)
 };
+// Cap on the CTAs (CTA pairs: 2 per pair) of every GEMM launched on stream s (0 = all SMs).
+// The families cap their weight-gradient side streams (NASPIPE_SIDE_SMS), so the persistent
+// wgrad GEMMs leave SMs to the stage stream's critical chain; results are unchanged (tiles
+// are assigned statically and computed independently of the grid).
+void gemm_set_stream_cap(cudaStream_t s, int max_ctas);
+int side_stream_sms();  // NASPIPE_SIDE_SMS (0 = no cap)
 // split-K factor the launcher uses for an (M, N, K) GEMM given a large enough workspace
 int gemm_splitk_factor(int M, int N, int K);
 void gemm_bf16_tc(cudaStream_t s, int M, int N, int K, const bf16* A, bool a_mn, int lda, const bf16* B,
