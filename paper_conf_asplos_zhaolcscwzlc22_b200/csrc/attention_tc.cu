@@ -54,8 +54,11 @@ __device__ __forceinline__ uint8_t* align1024(uint8_t* p) {
   return reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(p) + 1023) & ~uintptr_t(1023));
 }
 
+// 8 warps: warps w and w + 4 share TMEM lane quarter w % 4 (query rows 32 (w % 4) ..) and
+// split the 128 key columns (softmax) and the HD output columns in halves; the row maximum
+// and sum combine the two halves through shared memory (sum = half 0 + half 1, fixed order).
 template <int HD>
-__global__ void __launch_bounds__(128, 1) attn_fwd_tc_kernel(const __grid_constant__ CUtensorMap tq, bf16* __restrict__ o,
+__global__ void __launch_bounds__(256, 1) attn_fwd_tc_kernel(const __grid_constant__ CUtensorMap tq, bf16* __restrict__ o,
                                                               float* __restrict__ lse, int d, int h) {
   constexpr int NCH = HD / 64;
   extern __shared__ uint8_t smem_raw[];
@@ -65,8 +68,10 @@ __global__ void __launch_bounds__(128, 1) attn_fwd_tc_kernel(const __grid_consta
   uint8_t* sP = sV + NCH * TILE;  // [128 q][128 k], two tiles
   uint64_t* bar = reinterpret_cast<uint64_t*>(sP + 2 * TILE);  // [0] TMA, [1] S, [2] O
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bar + 3);
+  float* xch = reinterpret_cast<float*>(bar + 4);  // [2 halves][2 (max, sum)][128 rows]
   const int bh = blockIdx.x, b = bh / h, hh = bh % h;
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, r = threadIdx.x;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int r = 32 * (warp & 3) + lane, hf = warp >> 2;  // TMEM lane (query row), column half
   if (threadIdx.x == 0) {
     ptx::tma_prefetch(&tq);
     for (int i = 0; i < 3; ++i) ptx::mbar_init(&bar[i], 1);
@@ -97,20 +102,24 @@ __global__ void __launch_bounds__(128, 1) attn_fwd_tc_kernel(const __grid_consta
   }
   ptx::mbar_wait(&bar[1], 0);
   ptx::tc_fence_after();
-  const uint32_t trow = tmem + ((uint32_t)(warp * 32) << 16);
+  const uint32_t trow = tmem + ((uint32_t)(32 * (warp & 3)) << 16);
   const float sl2 = LOG2E / sqrtf((float)HD);
+  const int k0 = hf * (AS / 2);  // this warp's key columns [k0, k0 + 64)
   float mx = -INFINITY;
 #pragma unroll
-  for (int c0 = 0; c0 < AS; c0 += 32) {
+  for (int c0 = k0; c0 < k0 + AS / 2; c0 += 32) {
     uint32_t v[32];
     ptx::tmem_ld32(trow + c0, v);
     ptx::tmem_ld_wait();
 #pragma unroll
     for (int i = 0; i < 32; ++i) mx = fmaxf(mx, __uint_as_float(v[i]));
   }
+  xch[hf * 256 + r] = mx;
+  __syncthreads();
+  mx = fmaxf(xch[r], xch[256 + r]);
   float sum = 0.f;
 #pragma unroll
-  for (int c0 = 0; c0 < AS; c0 += 32) {
+  for (int c0 = k0; c0 < k0 + AS / 2; c0 += 32) {
     uint32_t v[32];
     ptx::tmem_ld32(trow + c0, v);
     ptx::tmem_ld_wait();
@@ -125,10 +134,12 @@ __global__ void __launch_bounds__(128, 1) attn_fwd_tc_kernel(const __grid_consta
       st_sw128(sP, r, c0 + 8 * q, p);
     }
   }
+  xch[hf * 256 + 128 + r] = sum;
   fence_proxy_async();  // P (generic-proxy stores) visible to the tensor core (async proxy)
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
+  sum = xch[128 + r] + xch[256 + 128 + r];  // half 0 + half 1
   if (warp == 0) {  // lane 0 issues; lanes 1-31 wait at the __syncwarp, not spinning on an mbarrier
     if (lane == 0) {
       constexpr uint32_t idesc = ptx::umma_idesc_bf16(128, HD, 0, 1);  // A = P K-major, B = V MN-major
@@ -143,7 +154,7 @@ __global__ void __launch_bounds__(128, 1) attn_fwd_tc_kernel(const __grid_consta
   const float inv = 1.f / sum;
   bf16* orow = o + ((size_t)b * AS + r) * d + hh * HD;
 #pragma unroll
-  for (int c0 = 0; c0 < HD; c0 += 32) {
+  for (int c0 = hf * (HD / 2); c0 < hf * (HD / 2) + HD / 2; c0 += 32) {
     uint32_t v[32];
     ptx::tmem_ld32(trow + 128 + c0, v);
     ptx::tmem_ld_wait();
@@ -157,7 +168,7 @@ __global__ void __launch_bounds__(128, 1) attn_fwd_tc_kernel(const __grid_consta
       *reinterpret_cast<uint4*>(orow + c0 + 8 * q) = w;
     }
   }
-  lse[(size_t)bh * AS + r] = mx * sl2 * 0.6931471805599453f + logf(sum);
+  if (hf == 0) lse[(size_t)bh * AS + r] = mx * sl2 * 0.6931471805599453f + logf(sum);
   ptx::tc_fence_before();
   __syncthreads();
   if (warp == 0) {
@@ -517,13 +528,13 @@ void attn_fwd_tc(cudaStream_t s, const bf16* qkv, bf16* o, float* lse, int B, in
   const int hd = d / h;
   const CUtensorMap tq = tma_map_bf16(qkv, 3 * (uint64_t)d, (uint64_t)B * S, 3 * (uint64_t)d, 128);
   if (hd == 64) {
-    const int smem = 5 * TILE + 1024 + 64;
+    const int smem = 5 * TILE + 1024 + 64 + 2048;
     set_smem_attr(attn_fwd_tc_kernel<64>, smem);
-    launch_pdl(attn_fwd_tc_kernel<64>, dim3(B * h), dim3(128), smem, s, tq, o, lse, d, h);
+    launch_pdl(attn_fwd_tc_kernel<64>, dim3(B * h), dim3(256), smem, s, tq, o, lse, d, h);
   } else {
-    const int smem = 8 * TILE + 1024 + 64;
+    const int smem = 8 * TILE + 1024 + 64 + 2048;
     set_smem_attr(attn_fwd_tc_kernel<128>, smem);
-    launch_pdl(attn_fwd_tc_kernel<128>, dim3(B * h), dim3(128), smem, s, tq, o, lse, d, h);
+    launch_pdl(attn_fwd_tc_kernel<128>, dim3(B * h), dim3(256), smem, s, tq, o, lse, d, h);
   }
   const cudaError_t e = cudaGetLastError();
   NP_REQUIRE(e == cudaSuccess, NASPIPE_ECUDA, "attn_fwd_tc: %s", cudaGetErrorString(e));
