@@ -109,15 +109,21 @@ def dilation(cfg, c):
 
 
 def convs(cfg, b, c):
-    """Ordered conv list of candidate (b, c): (name, kind 'pw'|'dw', cin, cout, k, stride).
+    """Ordered conv list of candidate (b, c): (name, kind 'pw'|'dw'|'cv', cin, cout, k, stride).
     Every depthwise conv of the candidate uses its kernel size k = choice_kernel[c] (the
-    Xception choice of the default configs has k = 3) and its dilation (dilation())."""
+    Xception choice of the default configs has k = 3) and its dilation (dilation()).
+    choice_xception[c] == 2 is Table 5's dense "Conv 3x3" (reading A40): the Shuffle
+    block with its depthwise k x k conv replaced by a DENSE k x k conv over the mid channels
+    ('cv': mid -> mid, stride s, pad k // 2, no bias, BN, no ReLU, dilation 1); the stride-2
+    proj branch stays depthwise."""
     s, inp, mid, out, _, _ = block_dims(cfg, b)
     k = cfg["choice_kernel"][c]
     L = []
     if s == 2:
         L += [("p_dw", "dw", inp, inp, k, 2), ("p_pw", "pw", inp, inp, 1, 1)]
-    if not cfg["choice_xception"][c]:
+    if cfg["choice_xception"][c] == 2:
+        L += [("m_pw1", "pw", inp, mid, 1, 1), ("m_cv", "cv", mid, mid, k, s), ("m_pw2", "pw", mid, out, 1, 1)]
+    elif not cfg["choice_xception"][c]:
         L += [("m_pw1", "pw", inp, mid, 1, 1), ("m_dw", "dw", mid, mid, k, s), ("m_pw2", "pw", mid, out, 1, 1)]
     else:
         L += [("x_dw1", "dw", inp, inp, k, s), ("x_pw1", "pw", inp, mid, 1, 1), ("x_dw2", "dw", mid, mid, k, 1),
@@ -130,6 +136,8 @@ def layout(cfg, b, c):
     for name, kind, cin, cout, k, _ in convs(cfg, b, c):
         if kind == "pw":
             out.append((name, (cout, cin), "uniform", cin))
+        elif kind == "cv":
+            out.append((name, (cout, k, k, cin), "uniform", k * k * cin))
         else:
             out.append((name, (cout, k, k), "uniform", k * k))
         out.append((name + "_g", (cout,), "ones", 0))
@@ -194,6 +202,23 @@ def conv_fwd(x, w, s):
     return y
 
 
+def conv_bwd(x, w, s, dy):
+    """Gradients of conv_fwd (pad k // 2, stride s): dx = sum over taps of the transposed
+    correlation of dy with w, dw[o, u, v, i] = sum over (b, oh, ow) of dy[.., o] xpad[.., i]."""
+    k = w.shape[1]
+    p = k // 2
+    xp = pad_hw(x, p)
+    B, Ho, Wo, _ = dy.shape
+    dxp = np.zeros_like(xp)
+    dw = np.zeros_like(w)
+    for u in range(k):
+        for v in range(k):
+            sl = (slice(None), slice(u, u + s * (Ho - 1) + 1, s), slice(v, v + s * (Wo - 1) + 1, s), slice(None))
+            dxp[sl] += dy @ w[:, u, v, :]
+            dw[:, u, v, :] = np.einsum("bhwo,bhwi->oi", dy, xp[sl])
+    return dxp[:, p:p + x.shape[1], p:p + x.shape[2], :], dw
+
+
 def bn_fwd(x, g, b):
     mu = x.mean(axis=(0, 1, 2))
     var = ((x - mu) ** 2).mean(axis=(0, 1, 2))
@@ -212,7 +237,13 @@ def bn_bwd(dy, g, cache):
 # ------------------------------------------------------------------ conv -> BN [-> ReLU] unit
 def _unit_fwd(p, name, kind, s, relu, x, st=PLAIN, dil=1):
     w = p[name]
-    z = st.f(dw_fwd(x, w, s, dil) if kind == "dw" else x @ st.w(w).T)
+    if kind == "dw":
+        z = dw_fwd(x, w, s, dil)
+    elif kind == "cv":
+        z = conv_fwd(x, st.w(w), s)
+    else:
+        z = x @ st.w(w).T
+    z = st.f(z)
     y, cb = bn_fwd(z, p[name + "_g"], p[name + "_b"])
     if relu:
         y = np.maximum(y, 0.0)
@@ -231,6 +262,9 @@ def _unit_bwd(p, name, kind, s, dy, tape, grads, st=PLAIN, add=None, dil=1):
     if kind == "dw":
         dx, _ = dw_bwd(x, p[name], s, dz, dil)
         _, grads[name] = dw_bwd(st.op(x), p[name], s, dz, dil)
+    elif kind == "cv":
+        dx, _ = conv_bwd(x, st.op(p[name]), s, dz)
+        _, grads[name] = conv_bwd(st.op(x), p[name], s, dz)
     else:
         grads[name] = np.einsum("bhwo,bhwi->oi", dz, st.op(x))
         dx = dz @ st.op(p[name])
@@ -250,7 +284,7 @@ def _chain(cfg, b, c, which):
 
 def block_fwd(cfg, b, c, p, x, st=PLAIN):
     s = block_dims(cfg, b)[0]
-    main_key = "x" if cfg["choice_xception"][c] else "m"
+    main_key = "x" if cfg["choice_xception"][c] == 1 else "m"
     if s == 1:
         xp, xm = x[..., 0::2], x[..., 1::2]
     else:
@@ -272,7 +306,7 @@ def block_fwd(cfg, b, c, p, x, st=PLAIN):
 
 def block_bwd(cfg, b, c, p, tapes, dy, st=PLAIN):
     s, inp = block_dims(cfg, b)[:2]
-    main_key = "x" if cfg["choice_xception"][c] else "m"
+    main_key = "x" if cfg["choice_xception"][c] == 1 else "m"
     cp = inp if s == 2 else dy.shape[-1] // 2
     d_proj, d_main = dy[..., :cp], dy[..., cp:]
     grads = {}

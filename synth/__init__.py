@@ -117,6 +117,12 @@ CONFIGS = {
                   head_channels=1024, choice_kernel=[3, 5, 7] * 16, choice_xception=([0] * 6 + [1] * 6) * 4,
                   choice_dilation=[1, 1, 1, 2, 2, 2] * 8,
                   lr=0.001, compute_dtype="bf16", n_stages=8, n_subnets=256),
+    # small SPOS supernet with Table 5's dense "Conv 3x3" candidates (choice_xception 2, reading
+    # A40) beside Shuffle 5 and Xception 3 (parity tests)
+    "tiny_spos_dense": dict(family="spos", n_blocks=5, n_choices=4, batch=4, image_hw=64, num_classes=10,
+                            stage_repeats=[1, 2, 1, 1], stage_channels=[32, 64, 96, 128], stem_channels=16,
+                            head_channels=64, choice_kernel=[3, 5, 3, 3], choice_xception=[2, 0, 1, 2],
+                            lr=0.001, compute_dtype="bf16", n_stages=2, n_subnets=8),
     # small SPOS supernet with dilated candidates (parity tests of A36)
     "tiny_spos_dil": dict(family="spos", n_blocks=5, n_choices=4, batch=4, image_hw=64, num_classes=10,
                           stage_repeats=[1, 2, 1, 1], stage_channels=[32, 64, 96, 128], stem_channels=16,

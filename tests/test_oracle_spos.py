@@ -87,6 +87,50 @@ def test_dense_conv_matches_loops():
     np.testing.assert_allclose(y, ref, rtol=1e-12)
 
 
+@pytest.mark.parametrize("k,s", [(3, 1), (3, 2), (5, 1), (5, 2)])
+def test_dense_conv_fwd_bwd_match_torch(k, s):
+    """conv_fwd / conv_bwd (the dense Conv 3x3 candidate, reading A40) against PyTorch's
+    conv2d (NCHW, padding k // 2) and its autograd gradients, fp64."""
+    torch = pytest.importorskip("torch")
+    rng = np.random.default_rng(10 * k + s)
+    x = rng.standard_normal((2, 10, 10, 8))
+    w = rng.standard_normal((6, k, k, 8))
+    y = spos.conv_fwd(x, w, s)
+    xt = torch.tensor(x.transpose(0, 3, 1, 2), requires_grad=True)
+    wt = torch.tensor(w.transpose(0, 3, 1, 2), requires_grad=True)
+    yt = torch.nn.functional.conv2d(xt, wt, stride=s, padding=k // 2)
+    np.testing.assert_allclose(y, yt.detach().numpy().transpose(0, 2, 3, 1), rtol=1e-12, atol=1e-12)
+    dy = rng.standard_normal(y.shape)
+    yt.backward(torch.tensor(dy.transpose(0, 3, 1, 2)))
+    dx, dw = spos.conv_bwd(x, w, s, dy)
+    np.testing.assert_allclose(dx, xt.grad.numpy().transpose(0, 2, 3, 1), rtol=1e-12, atol=1e-12)
+    np.testing.assert_allclose(dw, wt.grad.numpy().transpose(0, 2, 3, 1), rtol=1e-12, atol=1e-12)
+
+
+def test_dense_candidate_structure():
+    """The dense candidate is the Shuffle block with its depthwise conv replaced: same units,
+    the mid conv dense [mid, k, k, mid] (fan-in k k mid); a centred identity kernel (w[o, 1, 1, i]
+    = delta_oi) makes it reproduce the Shuffle block with a centred-delta depthwise kernel."""
+    b, c_dense, c_shuf = 1, 0, 2          # MINI_DENSE: c 0 = dense k 3, c 2 = Shuffle k 3
+    ld = spos.layout(MINI_DENSE, b, c_dense)
+    ls = spos.layout(MINI_DENSE, b, c_shuf)
+    assert [n for n, *_ in ld] == [n.replace("m_dw", "m_cv") for n, *_ in ls]
+    s, inp, mid, out, cout, H = spos.block_dims(MINI_DENSE, b)
+    assert dict((n, (sh, f)) for n, sh, _, f in ld)["m_cv"] == ((mid, 3, 3, mid), 9 * mid)
+    rng = np.random.default_rng(3)
+    ps = {n: (rng.standard_normal(sh) if kind == "uniform" else (np.ones(sh) if kind == "ones" else np.zeros(sh)))
+          for n, sh, kind, _ in ls}
+    ps["m_dw"] = np.zeros((mid, 3, 3))
+    ps["m_dw"][:, 1, 1] = 1.0
+    pd = {n.replace("m_dw", "m_cv"): v for n, v in ps.items()}
+    pd["m_cv"] = np.zeros((mid, 3, 3, mid))
+    pd["m_cv"][:, 1, 1, :] = np.eye(mid)
+    x = rng.standard_normal((2, H, H, cout))
+    ys, _ = spos.block_fwd(MINI_DENSE, b, c_shuf, ps, x)
+    yd, _ = spos.block_fwd(MINI_DENSE, b, c_dense, pd, x)
+    np.testing.assert_allclose(yd, ys, rtol=1e-12, atol=1e-12)
+
+
 def test_batchnorm_closed_form():
     rng = np.random.default_rng(2)
     x = rng.standard_normal((3, 4, 4, 5)) * 3 + 2
@@ -101,6 +145,8 @@ MINI = dict(family="spos", n_blocks=2, n_choices=4, batch=2, image_hw=16, num_cl
             choice_kernel=[3, 5, 7, 3], choice_xception=[0, 0, 0, 1], lr=0.01, init_seed=2)
 # the dilated choices of Table 5 (reading A36): Shuffle 3/5 and Xception 3/5 at dilation 2
 MINI_DIL = dict(MINI, choice_kernel=[3, 5, 3, 5], choice_xception=[0, 0, 1, 1], choice_dilation=[2, 2, 2, 2])
+# Table 5's dense "Conv 3x3" (reading A40): the Shuffle block with a dense k x k mid conv
+MINI_DENSE = dict(MINI, choice_kernel=[3, 5, 3, 3], choice_xception=[2, 2, 0, 1])
 
 
 def _check_fd(f, analytic, arr, rng, n=6, eps=1e-6):
@@ -117,7 +163,7 @@ def _check_fd(f, analytic, arr, rng, n=6, eps=1e-6):
         assert abs(num - analytic[i]) <= 1e-5 * max(abs(num), abs(analytic[i])) + 1e-7, (i, num, analytic[i])
 
 
-@pytest.mark.parametrize("cfg", [MINI, MINI_DIL], ids=["plain", "dilated"])
+@pytest.mark.parametrize("cfg", [MINI, MINI_DIL, MINI_DENSE], ids=["plain", "dilated", "dense"])
 @pytest.mark.parametrize("b", [0, 1])          # block 0: stride 2 (proj branch), block 1: stride 1
 @pytest.mark.parametrize("c", [0, 1, 2, 3])    # Shuffle 3/5/7, Xception (MINI_DIL: dilated Shuffle/Xception 3/5)
 def test_block_fd(b, c, cfg):
