@@ -382,7 +382,8 @@ def workload_config(args, cfg, world):
              "nlp_c1": "NLP.c1 analog (Table 1: 48 blocks x 72 choices, Table 5 NLP ops)",
              "nlp_c0": "NLP.c0 analog (Table 1: 48 blocks x 96 choices, Table 5 NLP ops)",
              "cv_c2": "CV.c2 analog (Table 1: 32 blocks x 24 choices, Table 5 ops incl. dilated)",
-             "cv_c1": "CV.c1 analog (Table 1: 32 blocks x 48 choices, Table 5 ops incl. dilated)"}
+             "cv_c1": "CV.c1 analog (Table 1: 32 blocks x 48 choices, Table 5 ops incl. dilated)",
+             "spos_dense": "configs[1] geometry with Table 5's dense Conv 3x3 candidate (A40)"}
     c = {"workload": names.get(args.workload, args.workload) if not args.n_choices
          else f"configs[4] sweep n={args.n_choices}",
          "n_blocks": cfg["n_blocks"], "n_choices": cfg["n_choices"], "batch": cfg["batch"],

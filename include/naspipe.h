@@ -153,7 +153,10 @@ typedef enum { NASPIPE_FP32 = 0, NASPIPE_BF16 = 1 } naspipe_dtype; /* compute dt
  *                 stage has stride 2, inp = C_prev, mid = C/2, out = C - C_prev; the
  *                 others stride 1 with inp = mid = out = C/2 (channel split).
  *   choice_kernel[n] (3, 5 or 7): the k of every depthwise conv of choice n;
- *   choice_xception[n] (0 = Shuffle, 1 = Xception); choice_dilation[n] (ABI 4; 1 or 2,
+ *   choice_xception[n] (0 = Shuffle, 1 = Xception, 2 = Table 5's dense "Conv 3x3", P:L447:
+ *                 the Shuffle block with its depthwise conv replaced by a dense 3x3 conv over
+ *                 the mid channels, weights [mid][3][3][mid], k 3 and dilation 1 only;
+ *                 DESIGN.md A40); choice_dilation[n] (ABI 4; 1 or 2,
  *                 NULL = all 1): dilation of choice n's depthwise convs, pad dilation*(k/2)
  *                 (Table 5's "Dil Conv 3x3"; A36)
  *   Frozen stem/head/FC weights use the counter hash with uids m*n + {0, 1, 2}, fan_in

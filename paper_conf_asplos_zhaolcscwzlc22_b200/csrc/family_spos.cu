@@ -44,7 +44,7 @@ class SposFamily : public Family {
     w16_.assign((size_t)nb * n, nullptr);
     plans_.resize((size_t)nb * n);
     dims_.resize(nb);
-    size_t stash_max = 0, stats_max = 0, dz_max = 0, g_max = 0, blk_max = 0, dwk_max = 0, C_max = 0;
+    size_t stash_max = 0, stats_max = 0, dz_max = 0, g_max = 0, blk_max = 0, dwk_max = 0, C_max = 0, dcols_max = 0;
     ws_elems_ = 0;
     for (int j = 0; j < nb; ++j) {
       const int b = blocks[j];
@@ -60,13 +60,18 @@ class SposFamily : public Family {
           const SposConv& u = L[i];
           const size_t po = P(u.H_out), pi = P(u.H_in);
           need += 2 * po * u.cout * (last_of_branch(L, i) ? 1 : 2);
+          if (u.dw == 2) {  // dense conv: its x2 columns stay in the stash for the weight gradient
+            need += 2 * po * (size_t)u.gemm_k();
+            dcols_max = std::max(dcols_max, po * (size_t)u.gemm_k());
+          }
           st += 4 * (size_t)u.cout;
           dz_max = std::max(dz_max, po * u.cout);
           g_max = std::max({g_max, pi * u.cin, po * u.cout});
           C_max = std::max(C_max, (size_t)u.cout);
-          if (u.dw) dwk_max = std::max(dwk_max, (size_t)u.cout * u.k * u.k);
+          if (u.dw == 1) dwk_max = std::max(dwk_max, (size_t)u.cout * u.k * u.k);
           else
-            ws_elems_ = std::max(ws_elems_, (size_t)gemm_splitk_factor(u.cout, u.cin, (int)po) * u.cout * u.cin);
+            ws_elems_ = std::max(ws_elems_, (size_t)gemm_splitk_factor(u.cout, u.gemm_k(), (int)po) * u.cout *
+                                                u.gemm_k());
         }
         stash_max = std::max(stash_max, need);
         stats_max = std::max(stats_max, st);
@@ -132,6 +137,7 @@ class SposFamily : public Family {
     acc_w_ = A.alloc<unsigned long long>(dwk_max + 1);
     cudaMemset(acc_w_, 0, (dwk_max + 1) * 8);
     ws_ = A.alloc<float>(std::max<size_t>(ws_elems_, 4));
+    if (dcols_max) dcols_ = A.alloc<float>(dcols_max);  // dense conv input-gradient columns (fp32)
     if (first_) {
       std::vector<float> h(spec.frozen_count(0));
       spec.init_frozen(0, h.data());
@@ -193,7 +199,7 @@ class SposFamily : public Family {
     bf16* w = w16_[(size_t)j * spec_.n() + c];
     const size_t half = shadow_elems(j, c) / 2;
     for (const SposConv& u : plans_[(size_t)j * spec_.n() + c])
-      if (!u.dw) f32_to_bf16x2(s, p + u.off_w, w + u.off_w16, w + half + u.off_w16, (size_t)u.cout * u.cin);
+      if (u.dw != 1) f32_to_bf16x2(s, p + u.off_w, w + u.off_w16, w + half + u.off_w16, u.weights());
   }
 
   void forward(int slot, const int32_t* ch, const void* x_in, void* x_out, cudaStream_t s) override {
@@ -415,16 +421,29 @@ class SposFamily : public Family {
       // the depthwise conv adds the BatchNorm sums of its output itself (fused bn_stats); with
       // its input's BN applied on load it reads acc_f_ and so adds its own sums to acc_f2_
       unsigned long long* zacc = acc_f_;
-      if (u.dw && pend.z != nullptr) {
+      if (u.dw == 1 && pend.z != nullptr) {
         r.x = nullptr;
         r.xbn = pend;
         zacc = acc_f2_;
         dw_fwd_bn(s, pend, Pm + u.off_w, r.z, B_, u.H_in, u.cin, u.k, u.stride, u.dil, zacc);
         counters.launches++;
         pend = BnApplyIn();
-      } else if (u.dw) {
+      } else if (u.dw == 1) {
         dw_fwd(s, h, Pm + u.off_w, r.z, B_, u.H_in, u.cin, u.k, u.stride, u.dil, zacc);
         counters.launches++;
+      } else if (u.dw == 2) {  // dense k x k (reading A40): x2 columns, 3-pass GEMM over K = k k cin
+        const int gk = u.gemm_k();
+        const size_t cplane = (size_t)Po * gk;
+        bf16* cols = cv;
+        cv += 2 * cplane;
+        im2col_x2(s, h, hplane, B_, u.H_in, u.cin, u.k, u.stride, cols, cplane);
+        counters.launches++;
+        r.x = cols;  // the weight gradient reads the columns' hi plane
+        GemmEpiParams e;  // the GEMM epilogue adds the BatchNorm sums of z (fused bn_stats)
+        e.out = r.z;
+        e.out2 = r.z + zplane;
+        e.stats = acc_f_;
+        gemm_x2(s, Po, u.cout, gk, cols, cols + cplane, gk, W16 + u.off_w16, W16 + half + u.off_w16, gk, e);
       } else {
         GemmEpiParams e;  // the GEMM epilogue adds the BatchNorm sums of z (fused bn_stats)
         e.out = r.z;
@@ -432,7 +451,7 @@ class SposFamily : public Family {
         e.stats = acc_f_;
         gemm_x2(s, Po, u.cout, u.cin, h, h + hplane, u.cin, W16 + u.off_w16, W16 + half + u.off_w16, u.cin, e);
       }
-      if (fuse_bna_ && !u.dw && !last_of_branch(L, i) && L[i + 1].dw) {
+      if (fuse_bna_ && u.dw == 0 && !last_of_branch(L, i) && L[i + 1].dw == 1) {
         // conv -> BN -> ReLU -> depthwise: no bn_apply; the depthwise conv applies it on load
         // (and its last CTA publishes this unit's mean / rstd and the g / b it used)
         pend.z = r.z;
@@ -492,7 +511,9 @@ class SposFamily : public Family {
   // the fused BatchNorm-backward reduction of unit `v` (record r) for the kernel producing its
   // output gradient: stride-1 depthwise input gradients and 1x1-conv input gradients (GEMM
   // epilogue EPI_BNBWD); the pre-update g, b (reading A4), as bn_bwd_reduce reads them
-  bool fusable_producer(const SposConv& u) const { return u.dw ? fuse_bnb_ : fuse_bnb_gemm_; }
+  bool fusable_producer(const SposConv& u) const {
+    return u.dw == 1 ? fuse_bnb_ : (u.dw == 0 ? fuse_bnb_gemm_ : false);
+  }
   BnBwdFuse bnb_of(const SposConv& v, const UnitRec& r, const float* Pm) const {
     BnBwdFuse f;
     f.z = r.z;
@@ -515,8 +536,14 @@ class SposFamily : public Family {
     const int Po = (int)P(u.H_out);
     const bf16* dz = dz_[ring_];
     if (dst) {
-      if (u.dw) {
+      if (u.dw == 1) {
         dw_dgrad(s, dz, Pm + u.off_w, add, dst, B_, u.H_in, u.cin, u.k, u.stride, u.dil, fuse ? *fuse : BnBwdFuse());
+        counters.launches++;
+      } else if (u.dw == 2) {  // dense: dcols = dz W (fp32), then the fixed-order column adjoint
+        GemmEpiParams e;
+        e.out = dcols_;
+        gemm(s, Po, u.gemm_k(), u.cout, dz, false, u.cout, W16 + u.off_w16, true, u.gemm_k(), EPI_F32, e);
+        col2im(s, dcols_, B_, u.H_in, u.cin, u.k, u.stride, add, dst);
         counters.launches++;
       } else {
         NP_REQUIRE(add == nullptr, NASPIPE_EINTERNAL, "pw dgrad with an addend");
@@ -528,7 +555,7 @@ class SposFamily : public Family {
     }
     cudaEventRecord(ev_dg_[ring_], s);
     cudaStreamWaitEvent(side_, ev_dg_[ring_], 0);
-    if (u.dw) {
+    if (u.dw == 1) {
       dw_wgrad_sgd(side_, dz, r.x, acc_w_, tick_ + 2, Um + u.off_w, lr_, B_, u.H_in, u.cin, u.k, u.stride, u.dil,
                    r.xbn.z ? &r.xbn : nullptr);
       counters.launches += 1;
@@ -538,7 +565,7 @@ class SposFamily : public Family {
       e.w16 = inplace ? W16 + u.off_w16 : nullptr;
       e.w16lo = inplace ? W16 + half + u.off_w16 : nullptr;
       e.lr = lr_;
-      gemm(side_, u.cout, u.cin, Po, dz, true, u.cout, r.x, true, u.cin, EPI_SGD, e, true);
+      gemm(side_, u.cout, u.gemm_k(), Po, dz, true, u.cout, r.x, true, u.gemm_k(), EPI_SGD, e, true);
     }
     cudaEventRecord(ev_wg_[ring_], side_);
     ring_used_[ring_] = true;
@@ -620,6 +647,7 @@ class SposFamily : public Family {
   cudaStream_t side_ = nullptr;  // weight gradients + SGD of the backward
   cudaEvent_t ev_dg_[kRing], ev_wg_[kRing], ev_join_;
   float* ws_;
+  float* dcols_ = nullptr;  // dense conv: fp32 input-gradient columns (stage stream)
   unsigned long long *acc_f_, *acc_b_;  // BatchNorm fixed-point accumulators (forward / backward)
   unsigned long long* acc_f2_;          // forward sums of a depthwise conv that reads acc_f_ (BN on load)
   // ticket-free mode: acc_f_ / acc_b_ point at ring slot fu_ % 3 / bu_ % 3 of the next use

@@ -230,6 +230,13 @@ void dw_fwd_bn(cudaStream_t s, const BnApplyIn& xin, const float* w, bf16* z, in
 void dw_dgrad(cudaStream_t s, const bf16* dz, const float* w, const bf16* add, bf16* dx, int B, int H, int C, int k,
               int S, int dil, const BnBwdFuse& bnb = BnBwdFuse());
 int dw_wgrad_blocks(int B, int H, int C, int k, int S);
+// Dense k x k conv (Table 5's Conv 3x3; reading A40) as GEMMs over explicit columns:
+// cols [B*Ho*Ho][k*k*C] (column (u*k + v)*C + c = x[b, oh*S + u - k/2, ow*S + v - k/2, c],
+// zero outside), x2 planes (hi plane, lo plane cplane elements later); and its adjoint
+// dx[b, ih, iw, c] = sum over (u, v) in order of dcols (fp32) (+ add), rounded to bf16.
+void im2col_x2(cudaStream_t s, const bf16* x, size_t xplane, int B, int H, int C, int k, int S, bf16* cols,
+               size_t cplane);
+void col2im(cudaStream_t s, const float* dcols, int B, int H, int C, int k, int S, const bf16* add, bf16* dx);
 // weight gradient of a depthwise conv with the SGD WRITE fused: w -= lr * sum over the batch
 // (acc [C*k*k + 1] and ticket zero between uses, fixpoint.cuh; w = master or BSP accumulator)
 // xin != nullptr: x = the hi plane of BN(z) [+ ReLU] recomputed on load (BnApplyIn, the

@@ -97,10 +97,12 @@ Spec::Spec(const naspipe_supernet_spec* s) {
     NP_REQUIRE(raw.num_classes >= 2 && raw.head_channels >= 16 && raw.head_channels % 16 == 0, NASPIPE_EINVAL,
                "num_classes %d / head_channels %d (%%16)", raw.num_classes, raw.head_channels);
     for (int c = 0; c < n; ++c)
-      NP_REQUIRE((kern[c] == 3 || kern[c] == 5 || kern[c] == 7) && (xcep[c] == 0 || xcep[c] == 1) &&
-                     (dil[c] == 1 || dil[c] == 2),
-                 NASPIPE_EINVAL, "choice %d: kernel %d xception %d dilation %d (k in {3,5,7}, dilation 1 or 2)", c,
-                 kern[c], xcep[c], dil[c]);
+      NP_REQUIRE((kern[c] == 3 || kern[c] == 5 || kern[c] == 7) && (xcep[c] >= 0 && xcep[c] <= 2) &&
+                     (dil[c] == 1 || dil[c] == 2) && (xcep[c] != 2 || (kern[c] == 3 && dil[c] == 1)),
+                 NASPIPE_EINVAL,
+                 "choice %d: kernel %d xception %d dilation %d (k in {3,5,7}, dilation 1 or 2; the dense "
+                 "Conv 3x3 (xception 2) takes k 3, dilation 1)",
+                 c, kern[c], xcep[c], dil[c]);
   }
   if (raw.stage_of_block) {
     stage_of_block.assign(raw.stage_of_block, raw.stage_of_block + m);
@@ -191,7 +193,7 @@ std::vector<SposConv> Spec::spos_convs(int b, int c) const {
   auto add = [&](int br, int dw, int ci, int co, int kk, int s, int relu, int hin) {
     SposConv u{};
     u.branch = br; u.dw = dw; u.cin = ci; u.cout = co; u.k = kk; u.stride = s; u.relu = relu;
-    u.dil = dw ? dl : 1;
+    u.dil = dw == 1 ? dl : 1;
     u.H_in = hin; u.H_out = hin / s;
     L.push_back(u);
   };
@@ -200,7 +202,11 @@ std::vector<SposConv> Spec::spos_convs(int b, int c) const {
     add(0, 1, d.inp, d.inp, k, 2, 0, H);
     add(0, 0, d.inp, d.inp, 1, 1, 1, Ho);
   }
-  if (!xcep[c]) {
+  if (xcep[c] == 2) {  // dense Conv 3x3 in place of the depthwise conv (reading A40)
+    add(1, 0, d.inp, d.mid, 1, 1, 1, H);
+    add(1, 2, d.mid, d.mid, k, s, 0, H);
+    add(1, 0, d.mid, d.outm, 1, 1, 1, Ho);
+  } else if (!xcep[c]) {
     add(1, 0, d.inp, d.mid, 1, 1, 1, H);
     add(1, 1, d.mid, d.mid, k, s, 0, H);
     add(1, 0, d.mid, d.outm, 1, 1, 1, Ho);
@@ -215,14 +221,14 @@ std::vector<SposConv> Spec::spos_convs(int b, int c) const {
   size_t off = 0, off16 = 0;
   for (auto& u : L) {
     u.off_w = off;
-    const size_t nw = u.dw ? (size_t)u.cout * u.k * u.k : (size_t)u.cout * u.cin;
+    const size_t nw = u.weights();
     off += nw;
     u.off_g = off;
     off += u.cout;
     u.off_b = off;
     off += u.cout;
     u.off_w16 = off16;
-    if (!u.dw) off16 += nw;
+    if (u.dw != 1) off16 += nw;
   }
   return L;
 }
@@ -231,7 +237,7 @@ std::vector<SposConv> Spec::spos_convs(int b, int c) const {
 size_t Spec::spos_shadow_elems(int b, int c) const {
   size_t t = 0;
   for (auto& u : spos_convs(b, c))
-    if (!u.dw) t += (size_t)u.cout * u.cin;
+    if (u.dw != 1) t += u.weights();
   return 2 * t;
 }
 
@@ -298,7 +304,7 @@ std::vector<Segment> Spec::segments(int b, int c) const {
   std::vector<Segment> s;
   if (family() == NASPIPE_SPOS_CNN) {
     for (auto& u : spos_convs(b, c)) {
-      s.push_back({u.off_w, u.off_g - u.off_w, 0, u.dw ? u.k * u.k : u.cin});
+      s.push_back({u.off_w, u.off_g - u.off_w, 0, u.dw == 1 ? u.k * u.k : u.gemm_k()});
       s.push_back({u.off_g, (size_t)u.cout, 1, 0});
       s.push_back({u.off_b, (size_t)u.cout, 2, 0});
     }
@@ -369,7 +375,7 @@ void Spec::default_costs(int32_t* cf, int32_t* cb) const {
         flops = bytes = 0;
         for (auto& u : spos_convs(b, c)) {
           const double Pin = (double)B() * u.H_in * u.H_in, Pout = (double)B() * u.H_out * u.H_out;
-          flops += u.dw ? 2.0 * Pout * u.cout * u.k * u.k : 2.0 * Pout * u.cin * u.cout;
+          flops += u.dw == 1 ? 2.0 * Pout * u.cout * u.k * u.k : 2.0 * Pout * u.gemm_k() * u.cout;
           bytes += 2.0 * (Pin * u.cin + 4.0 * Pout * u.cout);
         }
       } else {

@@ -44,13 +44,18 @@ struct SposDims {
 // One conv -> BN [-> ReLU] unit of a SPOS candidate, in packing order.
 struct SposConv {
   int branch;   // 0 = proj (stride-2 blocks), 1 = main
-  int dw;       // 1 = depthwise k x k, 0 = pointwise
+  int dw;       // 1 = depthwise k x k, 0 = pointwise, 2 = dense k x k (Table 5's Conv 3x3; reading A40)
   int cin, cout, k, stride;
   int dil;      // dw: dilation (1, or 2 for Table 5's Dil Conv; reading A36)
   int relu;     // ReLU after the BN
   int H_in, H_out;
   size_t off_w, off_g, off_b;  // offsets in the packed fp32 vector
-  size_t off_w16;              // pw: offset of the bf16 GEMM operand in the shadow
+  size_t off_w16;              // pw / dense: offset of the bf16 GEMM operand in the shadow
+  // GEMM K of a pointwise / dense unit (dense: over the k x k x cin columns) and weight count
+  int gemm_k() const { return dw == 2 ? k * k * cin : cin; }
+  size_t weights() const {
+    return dw == 1 ? (size_t)cout * k * k : (dw == 2 ? (size_t)cout * k * k * cin : (size_t)cout * cin);
+  }
 };
 
 struct Spec {

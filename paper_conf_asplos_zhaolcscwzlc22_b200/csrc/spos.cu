@@ -983,6 +983,68 @@ __global__ void __launch_bounds__(TPB) dw_wgrad_kernel(const bf16* __restrict__ 
 }
 
 
+// ---------------------------------------------------------------- dense k x k conv: columns
+// thread = (output pixel, tap, 8-channel group): one 16-byte hi and lo copy (exact)
+__global__ void im2col_x2_kernel(const bf16* __restrict__ x, size_t xplane, int B, int H, int C, int k, int S,
+                                 bf16* __restrict__ cols, size_t cplane) {
+  ptx::pdl_wait();
+  const int Ho = (H - 1) / S + 1, pad = k / 2, G = C / 8, K = k * k * C;
+  const size_t items = (size_t)B * Ho * Ho * k * k * G;
+  for (size_t it = blockIdx.x * (size_t)blockDim.x + threadIdx.x; it < items; it += (size_t)gridDim.x * blockDim.x) {
+    const int g = (int)(it % G);
+    const int tap = (int)((it / G) % (k * k));
+    const size_t po = it / ((size_t)G * k * k);
+    const int ow = (int)(po % Ho), oh = (int)((po / Ho) % Ho), b = (int)(po / ((size_t)Ho * Ho));
+    const int ih = oh * S + tap / k - pad, iw = ow * S + tap % k - pad;
+    uint4 hi = make_uint4(0u, 0u, 0u, 0u), lo = hi;
+    if (ih >= 0 && ih < H && iw >= 0 && iw < H) {
+      const size_t o = (((size_t)b * H + ih) * H + iw) * C + 8 * g;
+      hi = *reinterpret_cast<const uint4*>(x + o);
+      lo = *reinterpret_cast<const uint4*>(x + xplane + o);
+    }
+    const size_t d = po * K + (size_t)tap * C + 8 * g;
+    *reinterpret_cast<uint4*>(cols + d) = hi;
+    *reinterpret_cast<uint4*>(cols + cplane + d) = lo;
+  }
+}
+
+// thread = (input pixel, 8-channel group): the taps that read it, in (u, v) order, fp32
+__global__ void col2im_kernel(const float* __restrict__ dcols, int B, int H, int C, int k, int S,
+                              const bf16* __restrict__ add, bf16* __restrict__ dx) {
+  ptx::pdl_wait();
+  const int Ho = (H - 1) / S + 1, pad = k / 2, G = C / 8, K = k * k * C;
+  const size_t items = (size_t)B * H * H * G;
+  for (size_t it = blockIdx.x * (size_t)blockDim.x + threadIdx.x; it < items; it += (size_t)gridDim.x * blockDim.x) {
+    const int g = (int)(it % G);
+    const size_t pi = it / G;
+    const int iw = (int)(pi % H), ih = (int)((pi / H) % H), b = (int)(pi / ((size_t)H * H));
+    float acc[8] = {};
+    for (int u = 0; u < k; ++u) {
+      const int t = ih + pad - u;
+      if (t < 0 || t % S) continue;
+      const int oh = t / S;
+      if (oh >= Ho) continue;
+      for (int v = 0; v < k; ++v) {
+        const int q = iw + pad - v;
+        if (q < 0 || q % S) continue;
+        const int ow = q / S;
+        if (ow >= Ho) continue;
+        float dv[8];
+        load8f(dcols + (((size_t)b * Ho + oh) * Ho + ow) * K + (size_t)(u * k + v) * C + 8 * g, dv);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) acc[i] += dv[i];
+      }
+    }
+    if (add) {
+      float a[8];
+      load8(add + pi * C + 8 * g, a);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) acc[i] += a[i];
+    }
+    store8(dx + pi * C + 8 * g, acc);
+  }
+}
+
 // ---------------------------------------------------------------- channel split / merge
 // stride-1 block input x [P, 2Ch]: out[:, i] = x[:, 2i] (passed through, ld ldo), xm[:, i] = x[:, 2i+1]
 // (all three bf16x2; x and xm planes P*2Ch and P*Ch apart, out's planes oplane apart)
@@ -1508,6 +1570,23 @@ void dw_wgrad_sgd(cudaStream_t s, const bf16* dz, const bf16* x, unsigned long l
 #undef DW_WG
 #undef DW_WG1
   check_launch("dw_wgrad");
+}
+
+void im2col_x2(cudaStream_t s, const bf16* x, size_t xplane, int B, int H, int C, int k, int S, bf16* cols,
+               size_t cplane) {
+  NP_REQUIRE(C % 8 == 0 && (S == 1 || S == 2) && (k % 2) == 1, NASPIPE_EINVAL, "im2col C=%d k=%d S=%d", C, k, S);
+  const int Ho = (H - 1) / S + 1;
+  const size_t items = (size_t)B * Ho * Ho * k * k * (C / 8);
+  launch_pdl(im2col_x2_kernel, dim3(gs_grid(im2col_x2_kernel, items)), dim3(TPB), 0, s, x, xplane, B, H, C, k, S, cols,
+             cplane);
+  check_launch("im2col_x2");
+}
+
+void col2im(cudaStream_t s, const float* dcols, int B, int H, int C, int k, int S, const bf16* add, bf16* dx) {
+  NP_REQUIRE(C % 8 == 0 && (S == 1 || S == 2) && (k % 2) == 1, NASPIPE_EINVAL, "col2im C=%d k=%d S=%d", C, k, S);
+  const size_t items = (size_t)B * H * H * (C / 8);
+  launch_pdl(col2im_kernel, dim3(gs_grid(col2im_kernel, items)), dim3(TPB), 0, s, dcols, B, H, C, k, S, add, dx);
+  check_launch("col2im");
 }
 
 void chan_split(cudaStream_t s, const bf16* x, int P, int Ch, bf16* out, int ldo, size_t oplane, bf16* xm) {

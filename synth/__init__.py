@@ -117,6 +117,12 @@ CONFIGS = {
                   head_channels=1024, choice_kernel=[3, 5, 7] * 16, choice_xception=([0] * 6 + [1] * 6) * 4,
                   choice_dilation=[1, 1, 1, 2, 2, 2] * 8,
                   lr=0.001, compute_dtype="bf16", n_stages=8, n_subnets=256),
+    # configs[1] with Table 5's dense "Conv 3x3" (reading A40) in place of Shuffle 3: the CV
+    # op set {Conv 3x3, Sep Conv 5x5 (Shuffle 5), Shuffle 7, Xception} at full size
+    "spos_dense": dict(family="spos", n_blocks=20, n_choices=4, batch=64, image_hw=224, num_classes=1000,
+                       stage_repeats=[4, 4, 8, 4], stage_channels=[64, 160, 320, 640], stem_channels=16,
+                       head_channels=1024, choice_kernel=[3, 5, 7, 3], choice_xception=[2, 0, 0, 1],
+                       lr=0.001, compute_dtype="bf16", n_stages=8, n_subnets=256),
     # small SPOS supernet with Table 5's dense "Conv 3x3" candidates (choice_xception 2, reading
     # A40) beside Shuffle 5 and Xception 3 (parity tests)
     "tiny_spos_dense": dict(family="spos", n_blocks=5, n_choices=4, batch=4, image_hw=64, num_classes=10,

@@ -45,7 +45,7 @@ def test_init_params_match_shared_hash(name):
         assert np.array_equal(got.view(np.uint32), ref.view(np.uint32)), (b, c)
 
 
-@pytest.mark.parametrize("name", ["tiny_spos", "spos", "tiny_spos_dil", "cv_c3"])
+@pytest.mark.parametrize("name", ["tiny_spos", "spos", "tiny_spos_dil", "cv_c3", "tiny_spos_dense"])
 def test_spos_layout_and_init_match_oracle(name):
     """SPOS candidates: packed sizes and counter-hash values equal the oracle's layout
     (oracle/spos.py layout) for every candidate kind (stride 1/2, Shuffle k=3/5/7, Xception
@@ -104,7 +104,9 @@ def test_spos_spec_validation():
     cfg = synth.get_config("tiny_spos")
     for bad in (dict(stage_repeats=[1, 2, 1, 2]), dict(stage_channels=[32, 64, 80, 128]),
                 dict(choice_kernel=[3, 5, 4, 3]), dict(image_hw=48), dict(head_channels=60),
-                dict(choice_xception=[0, 0, 2, 1]), dict(choice_dilation=[1, 3, 1, 1]),
+                dict(choice_xception=[0, 0, 3, 1]), dict(choice_dilation=[1, 3, 1, 1]),
+                # the dense Conv 3x3 (xception 2, reading A40) takes k 3 and dilation 1 only
+                dict(choice_xception=[0, 2, 0, 1]), dict(choice_xception=[2, 0, 0, 1], choice_dilation=[2, 1, 1, 1]),
                 dict(choice_dilation=[1, 0, 1, 1])):
         with pytest.raises(npipe.NaspipeError):
             npipe.naspipe_default_costs(npipe.Spec(dict(cfg, **bad)))

@@ -76,6 +76,34 @@ def test_tiny_spos_bitwise_across_runs_and_stage_counts():
         _check_trace(cfg, choices, D, tr)
 
 
+@pytest.mark.parametrize("N", [1, 8, 100])
+def test_tiny_spos_dense_parity(N):
+    """Table 5's dense Conv 3x3 candidate (reading A40: the Shuffle block with a dense
+    3x3 mid conv; explicit x2 columns, 3-pass tcgen05 GEMM forward, fp32 column gradient +
+    fixed-order adjoint, split-K weight gradient with the SGD WRITE) beside Shuffle 5 and
+    Xception 3; every (block, choice) trained when N >= 4 (cyclic assignment)."""
+    cfg = synth.get_config("tiny_spos_dense")
+    m, n = cfg["n_blocks"], cfg["n_choices"]
+    choices = np.array([[(c + b) % n for b in range(m)] for c in range(N)], dtype=np.int32)
+    cfg, gpu, floor, losses, ref_loss, trace, stats = _run("tiny_spos_dense", choices)
+    pm.check(gpu, 1e-3 if N <= 8 else 1e-2, pm.UPD_SPOS if N <= 8 else None)
+    np.testing.assert_allclose(losses, ref_loss, rtol=1e-2)
+    _check_trace(cfg, choices, 2, trace)
+    assert stats["version_checks"] == 2 * N * m
+
+
+def test_tiny_spos_dense_bitwise_across_stage_counts():
+    cfg = synth.get_config("tiny_spos_dense")
+    choices = synth.sample_choices(10, cfg["n_blocks"], cfg["n_choices"])
+    batches = [synth.make_batch(cfg, y) for y in range(10)]
+    base, base_loss, _, _ = run_engine(cfg, choices, batches, D=1)
+    for D in (1, 2, 4):
+        p, l, tr, _ = run_engine(cfg, choices, batches, D=D)
+        assert np.array_equal(l.view(np.uint32), base_loss.view(np.uint32)), D
+        for k in base:
+            assert np.array_equal(p[k].view(np.uint32), base[k].view(np.uint32)), (D, k)
+
+
 @pytest.mark.parametrize("N", [1, 8])
 def test_tiny_spos_dilated_parity(N):
     """Dilated depthwise candidates (Table 5's Dil Conv; reading A36): Shuffle k 3/7
