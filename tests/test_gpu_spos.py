@@ -14,6 +14,9 @@ Bars (BASELINE.json north_star; A15, A28, A29), all against the plain 
 tiny_spos covers every candidate kind (Shuffle k = 3/5/7, Xception; stride 1 and 2),
 ragged BN row blocks (P = 4096, 1024, 256, 64, 16 pixels) and the frozen stem/head.
 """
+import json
+import os
+
 import numpy as np
 import pytest
 
@@ -169,6 +172,30 @@ def test_spos_full_size_one_step():
     sm = pm.errors(cfg, params, ref, theta0)
     print(f"full-size one step: {pm.fmt(sm)} loss {losses[0]:.6f} vs {ref_loss[0]:.6f}")
     pm.check(sm, 1e-3, pm.UPD_SPOS)
+    np.testing.assert_allclose(losses, ref_loss, rtol=1e-2)
+
+
+def test_spos_dense_full_size_one_step():
+    """configs[1] geometry with the dense Conv 3x3 candidate (A40) at full size, a subnet that
+    uses it in every block (choice 0), one step against the fp64 oracle.  Bars: update bars,
+    loss rtol 1e-2, per-tensor A15 <= max(1e-3, 1.5 x the storage floor): block 0's dense
+    weight gradient sums 200704 products of the bf16-stored dz (zero-mean after the BatchNorm
+    backward) with ReLU outputs (positive mean), a cancelling sum, so the path's bf16 backward
+    storage (A28) alone moves that tensor by 1.1e-3 (the oracle with the path's storage,
+    tests/golden/spos_dense_fullsize_1step_floor.json from tools/make_dense_floor.py; the
+    fp32-storage oracle: 9.5e-5) -- the reading A37 bar of the CV.c3 analog."""
+    cfg = synth.get_config("spos_dense")
+    choices = np.zeros((1, cfg["n_blocks"]), dtype=np.int32)
+    batches = [synth.make_batch(cfg, 0)]
+    theta0 = train.initial_theta(cfg)
+    ref, ref_loss = train.train_sequential(cfg, theta0, choices, batches)
+    params, losses, _, _ = run_engine(cfg, choices, batches, D=1)
+    sm = pm.errors(cfg, params, ref, theta0)
+    floor = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "spos_dense_fullsize_1step_floor.json")))
+    bar = max(1e-3, 1.5 * floor["bf16x2"]["a15_tensor"])
+    print(f"dense full-size one step: {pm.fmt(sm)} loss {losses[0]:.6f} vs {ref_loss[0]:.6f}; "
+          f"storage floor {floor['bf16x2']['a15_tensor']:.2e} (fp32 {floor['fp32']['a15_tensor']:.2e}), bar {bar:.2e}")
+    pm.check(sm, bar, pm.UPD_SPOS)
     np.testing.assert_allclose(losses, ref_loss, rtol=1e-2)
 
 
