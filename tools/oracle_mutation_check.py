@@ -12,13 +12,19 @@ muts = [
  ("oracle/spos.py", "return np.concatenate([xp, main], axis=-1), tapes", "return np.concatenate([main, xp], axis=-1), tapes", "concat order"),
  ("oracle/spos.py", "relu = kind == \"pw\" and (which == \"p\" or i == len(cl) - 1 or name in (\"m_pw1\", \"x_pw1\", \"x_pw2\"))", "relu = (kind == \"pw\" and (which == \"p\" or i == len(cl) - 1 or name in (\"x_pw1\", \"x_pw2\"))) or name == \"m_dw\"", "ReLU moved pw1->dw"),
  ("oracle/spos.py", "loss = float(np.mean(lse - logits[np.arange(B), labels]))", "loss = float(np.mean(lse - logits[np.arange(B), labels])) * 1.01", "CE scale"),
+ # the dense Conv 3x3 candidate (reading A40), caught by tests/test_oracle_spos.py's pins
+ ("oracle/spos.py", "y += xp[:, u:u + s * (Ho - 1) + 1:s, v:v + s * (Wo - 1) + 1:s, :] @ w[:, u, v, :].T", "y += xp[:, u:u + s * (Ho - 1) + 1:s, v:v + s * (Wo - 1) + 1:s, :] @ w[:, v, u, :].T", "dense taps transposed", "tests/test_oracle_spos.py"),
+ ("oracle/spos.py", "            dxp[sl] += dy @ w[:, u, v, :]", "            dxp[sl] += dy @ w[:, k - 1 - u, k - 1 - v, :]", "dense dgrad flipped", "tests/test_oracle_spos.py"),
+ ("oracle/spos.py", "        L += [(\"m_pw1\", \"pw\", inp, mid, 1, 1), (\"m_cv\", \"cv\", mid, mid, k, s), (\"m_pw2\", \"pw\", mid, out, 1, 1)]", "        L += [(\"m_pw1\", \"pw\", inp, mid, 1, 1), (\"m_cv\", \"cv\", mid, mid, k, 1), (\"m_pw2\", \"pw\", mid, out, 1, 1)]", "dense stride ignored", "tests/test_oracle_spos.py"),
 ]
-for f, a, b, what in muts:
+for m in muts:
+    f, a, b, what = m[:4]
+    test = m[4] if len(m) > 4 else "tests/test_oracle_closed_forms.py"
     src = open(f).read()
     assert a in src, (f, a)
     open(f, "w").write(src.replace(a, b))
     try:
-        r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "tests/test_oracle_closed_forms.py"], capture_output=True, text=True)
+        r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", test], capture_output=True, text=True)
         last = r.stdout.strip().splitlines()[-1]
         print(f"{what:22s} -> {'CAUGHT' if r.returncode else 'MISSED'}: {last}")
     finally:
