@@ -70,6 +70,11 @@ int naspipe_debug_dw_bn_fold(const void* zin, int B, int H, int C, const float* 
                              const float* w, int k, int S, int dil, const void* dz, void* out_ref, void* out,
                              float* dwsum_ref, float* dwsum, float* meta, float* mean_ref, float* rstd_ref,
                              void* stream);
+/* Dense k x k conv columns (A40): cols x2 [B*Ho*Ho][k*k*C] (hi plane then lo plane) of x x2
+ * [B,H,H,C] (if x && cols); dx bf16 [B,H,H,C] = col2im(dcols fp32 [B*Ho*Ho][k*k*C]) (+ add)
+ * (if dcols && dx). */
+int naspipe_debug_dense_cols(const void* x, void* cols, const float* dcols, const void* add, void* dx, int B, int H,
+                             int C, int k, int S, void* stream);
 int naspipe_debug_bnb_fused(int kind, const void* dz, const float* w, const void* w16, void* dx, int B, int H, int C,
                             int Cout, int k, int dil, const void* z, const float* mean, const float* rstd,
                             const float* g, const float* b, int relu, float* sums, void* stream);

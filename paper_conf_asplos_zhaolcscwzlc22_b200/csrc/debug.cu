@@ -173,6 +173,17 @@ int naspipe_debug_bn_bwd(const void* dy, int lddy, const void* z, int P, int C, 
   });
 }
 
+int naspipe_debug_dense_cols(const void* x, void* cols, const float* dcols, const void* add, void* dx, int B, int H,
+                             int C, int k, int S, void* stream) {
+  return dguard([&] {
+    cudaStream_t s = (cudaStream_t)stream;
+    const int Ho = (H - 1) / S + 1;
+    if (x && cols)
+      im2col_x2(s, (const bf16*)x, (size_t)B * H * H * C, B, H, C, k, S, (bf16*)cols, (size_t)B * Ho * Ho * k * k * C);
+    if (dcols && dx) col2im(s, dcols, B, H, C, k, S, (const bf16*)add, (bf16*)dx);
+  });
+}
+
 int naspipe_debug_dw_bn_fold(const void* zin, int B, int H, int C, const float* g, const float* b, int relu,
                              const float* w, int k, int S, int dil, const void* dz, void* out_ref, void* out,
                              float* dwsum_ref, float* dwsum, float* meta, float* mean_ref, float* rstd_ref,

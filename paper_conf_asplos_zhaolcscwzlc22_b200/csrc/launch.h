@@ -24,14 +24,15 @@ namespace naspipe {
 //   flags between kernels (the same cross-stream pattern).
 // The CTA-pair GEMM's early triggers (NASPIPE_PAIR_TRIGGER=1) also still hang
 // tools/hangtest.sh and stay off.
-// Stream priorities: a stage's compute stream (the task's critical chain) gets the highest
-// priority, the families' side streams (weight gradients, hidden behind that chain) the
-// lowest, so the block scheduler prefers the critical chain's CTAs when both streams have
-// work.  NASPIPE_STREAM_PRIO=0: default priorities for both (A/B).
+// Stream priorities (NASPIPE_STREAM_PRIO=1; OFF by default): a stage's compute stream (the
+// task's critical chain) at the highest priority, the families' side streams (weight
+// gradients) at the lowest.  Measured neutral on configs[1] / configs[2]
+// (profiles/r2_ab2/), and with it the configs[3] context-switching bench HUNG (killed after
+// 900 s; 86 s without, same box) -- root cause not found, so the default stays off.
 inline bool stream_prio_on() {
   static const bool v = [] {
     const char* e = getenv("NASPIPE_STREAM_PRIO");
-    return !(e && e[0] == '0');
+    return e && e[0] == '1';
   }();
   return v;
 }

@@ -42,7 +42,7 @@ NEAR_STATIC = 1e-2
 
 
 def structurally_static(cfg, name):
-    return cfg["family"] == "spos" and (("_dw" in name and name.endswith("_b"))
+    return cfg["family"] == "spos" and ((("_dw" in name or name == "m_cv_b") and name.endswith("_b"))
                                         or name in ("m_pw1_g", "x_pw1_g", "x_pw2_g"))
 
 

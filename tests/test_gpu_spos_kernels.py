@@ -28,6 +28,7 @@ L.naspipe_debug_gemm_x2.argtypes = [_i, _i, _i, _vp, _vp, _i, _vp, _vp, _i, _vp,
 L.naspipe_debug_chan_merge.argtypes = [_vp, _i, _vp, _i, _i, _vp, _vp]
 L.naspipe_debug_stem.argtypes = [_vp, _vp, _vp, _i, _i, _i, _vp]
 L.naspipe_debug_dw_bn_fold.argtypes = [_vp, _i, _i, _i, _vp, _vp, _i, _vp, _i, _i, _i] + [_vp] * 9
+L.naspipe_debug_dense_cols.argtypes = [_vp] * 5 + [_i] * 5 + [_vp]
 L.naspipe_debug_bnb_fused.argtypes = [_i, _vp, _vp, _vp, _vp] + [_i] * 6 + [_vp] * 5 + [_i, _vp, _vp]
 
 
@@ -291,6 +292,42 @@ def test_bn_backward_sums_fused_into_input_gradient(kind, B, H, Cc, Cout, k, dil
     a1, a2 = np.abs(d).sum(axis=0), np.abs(d * xh).sum(axis=0)
     assert np.all(np.abs(s[:Cc] - s1) <= 1e-5 * a1 + 1e-9)
     assert np.all(np.abs(s[Cc:] - s2) <= 1e-5 * a2 + 1e-9)
+
+
+@pytest.mark.parametrize("B,H,Cc,k,s", [(2, 9, 16, 3, 1), (3, 8, 24, 3, 2), (2, 12, 8, 5, 2), (64, 56, 32, 3, 1),
+                                        (64, 112, 32, 3, 2)])
+def test_dense_conv_columns_and_adjoint(B, H, Cc, k, s):
+    """The dense Conv 3x3 columns (A40): im2col of the x2 planes bitwise equal to the
+    definition (exact copies, zero padding), and col2im = the exact adjoint of im2col on the
+    fp32 column gradient (the sum over the taps that read an input, fp64 reference) + add,
+    rounded to bf16."""
+    rng = np.random.default_rng(B + H + Cc + k + s)
+    xd, _ = _x2(rng.standard_normal((B, H, H, Cc)))
+    Ho = (H - 1) // s + 1
+    K = k * k * Cc
+    cols = torch.empty((2, B * Ho * Ho, K), dtype=torch.bfloat16, device="cuda")
+    dcols_h = rng.standard_normal((B * Ho * Ho, K)).astype(np.float32)
+    dcols = torch.from_numpy(dcols_h).cuda()
+    addd, add = _bf(rng.standard_normal((B, H, H, Cc)))
+    dx = torch.empty((B, H, H, Cc), dtype=torch.bfloat16, device="cuda")
+    _ok(L.naspipe_debug_dense_cols(_p(xd), _p(cols), _p(dcols), _p(addd), _p(dx), B, H, Cc, k, s, None))
+    torch.cuda.synchronize()
+    p = k // 2
+    xp = torch.nn.functional.pad(xd.float().permute(0, 1, 4, 2, 3), (p, p, p, p))  # [2, B, C, H+2p, H+2p]
+    ref = torch.empty((2, B, Ho, Ho, k, k, Cc), device="cuda")
+    for u in range(k):
+        for v in range(k):
+            ref[:, :, :, :, u, v, :] = xp[:, :, :, u:u + s * (Ho - 1) + 1:s, v:v + s * (Ho - 1) + 1:s].permute(0, 1, 3, 4, 2)
+    assert torch.equal(cols.float().reshape(2, B, Ho, Ho, k, k, Cc), ref)
+    if B * H * H * Cc > 2_000_000:
+        return  # the adjoint on the small shapes (fp64 reference below)
+    dc = dcols_h.astype(np.float64).reshape(B, Ho, Ho, k, k, Cc)
+    rdx = np.zeros((B, H + 2 * p, H + 2 * p, Cc))
+    for u in range(k):
+        for v in range(k):
+            rdx[:, u:u + s * (Ho - 1) + 1:s, v:v + s * (Ho - 1) + 1:s, :] += dc[:, :, :, u, v, :]
+    rdx = rdx[:, p:p + H, p:p + H, :] + add
+    _check_bf16(_f64(dx), rdx)
 
 
 @pytest.mark.parametrize("P,Ch", [(7, 16), (3136, 320), (1000, 80)])

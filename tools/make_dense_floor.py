@@ -30,7 +30,8 @@ def main():
     for st in ("fp32", "bf16x2"):
         got, _ = train.train_sequential(dict(cfg, storage=st), theta0, choices, batches)
         e = pm.errors(cfg, got, ref, theta0)
-        out[st] = {"a15_tensor": float(e["a15"]), "a15_candidate": float(e["a15_cand"]), "upd": {k: float(v) for k, v in e["upd"].items()}, "fmt": pm.fmt(e)}
+        out[st] = {"a15_tensor": float(e["a15"]), "a15_candidate": float(e["a15_cand"]), "upd": {k: float(v) for k, v in e["upd"].items()},
+                   "static": float(e["static"]), "fmt": pm.fmt(e)}
         print(st, pm.fmt(e), flush=True)
     with open(os.path.join(ROOT, "tests", "golden", "spos_dense_fullsize_1step_floor.json"), "w") as f:
         json.dump(out, f, indent=1)
