@@ -1457,7 +1457,23 @@ static int dw_strips() {
 }
 
 // tile width: the smallest of 8 / 16 / 32 columns covering min(Ho, 32)
-static int dw_tw(int Ho) { return Ho <= 8 ? 8 : (Ho <= 16 ? 16 : 32); }
+// NASPIPE_DW_TW (8 / 16 / 32; 0 = by size): tile width of the depthwise kernels.  A CTA covers
+// TW columns x (256 / (8 TW)) groups of 8 channels, so narrower tiles read more of each
+// pixel's channels (whole 32-byte sectors) at the cost of more halo columns.
+static int dw_tw_knob() {
+  static const int v = [] {
+    const char* e = getenv("NASPIPE_DW_TW");
+    const int t = e ? atoi(e) : 0;
+    return (t == 8 || t == 16 || t == 32) ? t : 0;
+  }();
+  return v;
+}
+// default: 8 columns up to Ho = 8, else 16 (measured on configs[1]: 16-wide tiles 6.284 ms
+// per step, 32-wide (for Ho > 16) 6.322, 8-wide 6.356; profiles/r2_ab2/README.md)
+static int dw_tw(int Ho) {
+  const int t = Ho <= 8 ? 8 : 16;
+  return dw_tw_knob() ? std::min(dw_tw_knob(), Ho <= 8 ? 8 : (Ho <= 16 ? 16 : 32)) : t;
+}
 
 template <int K, int S, int DIL, bool X2, bool FLIP, bool XBN = false>
 static void dw_tile(cudaStream_t s, const bf16* in, const float* w, const bf16* add, bf16* out, int B, int H, int C,
