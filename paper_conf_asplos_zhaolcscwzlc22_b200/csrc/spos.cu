@@ -369,6 +369,7 @@ __device__ __forceinline__ void bn_bwd_item(const bf16* dy, const bf16* z, size_
 // s1 = sum dy', s2 = sum dy' xh (dy' = dy masked by the ReLU): fixed-order row-block
 // partials added to acc[2C] in fixed point (see bn_stats_kernel).  Thread (r, g): rows r,
 // r + RP, ... of its block, channels [4g, 4g+4); RP = TPB / (C/4).
+template <int UR>  // rows in flight per lane (the sums stay in row order whatever UR)
 __global__ void bn_bwd_reduce_kernel(const bf16* __restrict__ dy, int lddy, const bf16* __restrict__ z, int P, int C,
                                      const float* __restrict__ mean, const float* __restrict__ rstd,
                                      const float* __restrict__ gam, const float* __restrict__ bet, int relu,
@@ -387,14 +388,14 @@ __global__ void bn_bwd_reduce_kernel(const bf16* __restrict__ dy, int lddy, cons
     load4f(bet + BV * g, b8);
     float s1[BV] = {}, s2[BV] = {};
     int row = row0 + r;
-    for (; row + 3 * RP < row1; row += 4 * RP) {  // 4 rows in flight
-      float d[4][BV], xh[4][BV];
+    for (; row + (UR - 1) * RP < row1; row += UR * RP) {  // UR rows in flight
+      float d[UR][BV], xh[UR][BV];
 #pragma unroll
-      for (int u = 0; u < 4; ++u)
+      for (int u = 0; u < UR; ++u)
         bn_bwd_item(dy + (size_t)(row + u * RP) * lddy + BV * g, z + (size_t)(row + u * RP) * C + BV * g, zplane, mu,
                     rs, g8, b8, relu, d[u], xh[u]);
 #pragma unroll
-      for (int u = 0; u < 4; ++u)
+      for (int u = 0; u < UR; ++u)
 #pragma unroll
         for (int i = 0; i < BV; ++i) {
           s1[i] += d[u][i];
@@ -1400,13 +1401,19 @@ void bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int 
                    const float* rstd, const float* g, const float* b, int relu, unsigned long long* acc) {
   NP_REQUIRE(C % 8 == 0 && C / BV <= TPB, NASPIPE_EINVAL, "bn_bwd C=%d", C);
   const size_t sm = red_smem(C, BV);
-  set_smem(bn_bwd_reduce_kernel, sm);
+  // rows in flight per lane: NASPIPE_BNR_UNROLL (4 or 8; the sums are bitwise the same)
+  static const int ur = [] {
+    const char* e = getenv("NASPIPE_BNR_UNROLL");
+    return (e && atoi(e) == 8) ? 8 : 4;
+  }();
+  auto kern = ur == 8 ? bn_bwd_reduce_kernel<8> : bn_bwd_reduce_kernel<4>;
+  set_smem(kern, sm);
   // one wave of resident CTAs (the fixed-point totals do not depend on the row blocking's
   // summation order only through the partials, which are a function of (P, C) and this
   // occupancy-derived target, itself fixed per build and device)
-  const int target = num_sms() * occupancy(bn_bwd_reduce_kernel, sm);
-  launch_pdl(bn_bwd_reduce_kernel, dim3(red_blocks(P, C, BV, target)), dim3(TPB), sm, s, dy, lddy, z, P, C, mean, rstd,
-             g, b, relu, red_rows(P, C, BV, target), acc);
+  const int target = num_sms() * occupancy(bn_bwd_reduce_kernel<4>, sm);
+  launch_pdl(kern, dim3(red_blocks(P, C, BV, target)), dim3(TPB), sm, s, dy, lddy, z, P, C, mean, rstd, g, b, relu,
+             red_rows(P, C, BV, target), acc);
   check_launch("bn_bwd_reduce");
 }
 
