@@ -589,18 +589,18 @@ __device__ __forceinline__ void xbn_y8(float (&v)[8], const float* mu, const flo
   }
 }
 
-template <int K, int S, int DIL, bool X2, bool FLIP, bool XBN = false>
+template <int K, int S, int DIL, bool X2, bool FLIP, bool XBN = false, int DH = DT_H>
 __global__ void __launch_bounds__(TPB) dw_tile_kernel(const bf16* __restrict__ in, const float* __restrict__ w,
                                                     const bf16* __restrict__ add, bf16* __restrict__ out, int B,
                                                     int H, int C, int TW, int strips, unsigned long long* stats,
                                                     const BnBwdFuse bnb, const BnApplyIn xbn) {
   static_assert(!XBN || (X2 && !FLIP), "BN-on-load is a forward (bf16x2) mode");
-  constexpr int PAD = DIL * (K / 2), KE = DIL * (K - 1) + 1, IH = (DT_H - 1) * S + KE;
+  constexpr int PAD = DIL * (K / 2), KE = DIL * (K - 1) + 1, IH = (DH - 1) * S + KE;
   extern __shared__ float tile[];  // [CPG][IH][IW][8]
   ptx::pdl_wait();
   const int Ho = (H + 2 * PAD - KE) / S + 1;
   const int CPG = TPB / (8 * TW), IW = (TW - 1) * S + KE;
-  const int RH = DT_H * strips;  // output rows of the CTA: `strips` strips of DT_H rows
+  const int RH = DH * strips;  // output rows of the CTA: `strips` strips of DH rows
   const int tiles_h = (Ho + RH - 1) / RH, tiles_w = (Ho + TW - 1) / TW;
   int t = blockIdx.x;
   const int tw = t % tiles_w;
@@ -636,7 +636,7 @@ __global__ void __launch_bounds__(TPB) dw_tile_kernel(const bf16* __restrict__ i
   const float* tb = tile + (cgi * IH * IW + col * S) * 8 + ch;
   const int iw0 = tw * TW * S - PAD;
   for (int st = 0; st < strips; ++st) {
-    const int oh0 = th * RH + st * DT_H;
+    const int oh0 = th * RH + st * DH;
     if (oh0 >= Ho) break;  // CTA-uniform
     const int ih0 = oh0 * S - PAD;
     __syncthreads();  // the previous strip's halo has been consumed
@@ -657,9 +657,9 @@ __global__ void __launch_bounds__(TPB) dw_tile_kernel(const bf16* __restrict__ i
       d[1] = make_float4(v[4], v[5], v[6], v[7]);
     }
     __syncthreads();
-    float acc[DT_H];
+    float acc[DH];
 #pragma unroll
-    for (int r = 0; r < DT_H; ++r) acc[r] = 0.f;
+    for (int r = 0; r < DH; ++r) acc[r] = 0.f;
 #pragma unroll
     for (int ir = 0; ir < IH; ++ir) {
       const float* rowp = tb + ir * IW * 8;
@@ -667,7 +667,7 @@ __global__ void __launch_bounds__(TPB) dw_tile_kernel(const bf16* __restrict__ i
       for (int v = 0; v < K; ++v) {
         const float x = rowp[v * DIL * 8];
 #pragma unroll
-        for (int r = 0; r < DT_H; ++r) {
+        for (int r = 0; r < DH; ++r) {
           const int tt = ir - r * S;  // = u * DIL (compile-time after unrolling)
           if (tt >= 0 && tt % DIL == 0 && tt / DIL < K) acc[r] = __fmaf_rn(x, wr[tt / DIL][v], acc[r]);
         }
@@ -675,9 +675,9 @@ __global__ void __launch_bounds__(TPB) dw_tile_kernel(const bf16* __restrict__ i
     }
     if (valid) {
       const size_t o0 = (((size_t)b * Ho + oh0) * Ho + ow) * C + c, rstride = (size_t)Ho * C;
-      const int nr = min(DT_H, Ho - oh0);
+      const int nr = min(DH, Ho - oh0);
 #pragma unroll
-      for (int r = 0; r < DT_H; ++r) {
+      for (int r = 0; r < DH; ++r) {
         if (r >= nr) break;
         const size_t o = o0 + r * rstride;
         if (X2) {
@@ -1482,27 +1482,43 @@ static int dw_tw(int Ho) {
   return dw_tw_knob() ? std::min(dw_tw_knob(), Ho <= 8 ? 8 : (Ho <= 16 ? 16 : 32)) : t;
 }
 
-template <int K, int S, int DIL, bool X2, bool FLIP, bool XBN = false>
-static void dw_tile(cudaStream_t s, const bf16* in, const float* w, const bf16* add, bf16* out, int B, int H, int C,
-                    unsigned long long* stats = nullptr, const BnBwdFuse& bnb = BnBwdFuse(),
-                    const BnApplyIn& xbn = BnApplyIn()) {
+// rows per depthwise strip of dw_tile: NASPIPE_DW_DH (8 or 16; default 8)
+static int dw_dh() {
+  static const int v = [] {
+    const char* e = getenv("NASPIPE_DW_DH");
+    return (e && atoi(e) == 16) ? 16 : 8;
+  }();
+  return v;
+}
+
+template <int K, int S, int DIL, bool X2, bool FLIP, bool XBN, int DH>
+static void dw_tile_dh(cudaStream_t s, const bf16* in, const float* w, const bf16* add, bf16* out, int B, int H, int C,
+                       unsigned long long* stats, const BnBwdFuse& bnb, const BnApplyIn& xbn) {
   constexpr int KE = DIL * (K - 1) + 1;
   const int Ho = (H - 1) / S + 1, TW = dw_tw(Ho), CPG = TPB / (8 * TW);
-  const int IH = (DT_H - 1) * S + KE, IW = (TW - 1) * S + KE;
+  const int IH = (DH - 1) * S + KE, IW = (TW - 1) * S + KE;
   const size_t sm = (size_t)CPG * IH * IW * 8 * sizeof(float);
-  auto kern = dw_tile_kernel<K, S, DIL, X2, FLIP, XBN>;
+  auto kern = dw_tile_kernel<K, S, DIL, X2, FLIP, XBN, DH>;
   set_smem(kern, sm);
-  // strips of DT_H rows per CTA: as many (<= 4) as keep >= 2 waves of resident CTAs (the
+  // strips of DH rows per CTA: as many (<= 4) as keep >= 2 waves of resident CTAs (the
   // weights, the halo setup and the reductions amortised over more outputs per CTA)
-  const int tiles_w = (Ho + TW - 1) / TW, gy = (C / 8 + CPG - 1) / CPG, rows = (Ho + DT_H - 1) / DT_H;
+  const int tiles_w = (Ho + TW - 1) / TW, gy = (C / 8 + CPG - 1) / CPG, rows = (Ho + DH - 1) / DH;
   int strips = dw_strips();
   if (strips <= 0) {
     const long wave = (long)num_sms() * occupancy(kern, sm);
     strips = 1;
     while (strips < 4 && (long)B * ((rows + 2 * strips - 1) / (2 * strips)) * tiles_w * gy >= 2 * wave) strips *= 2;
   }
-  const int gx = B * ((Ho + DT_H * strips - 1) / (DT_H * strips)) * tiles_w;
+  const int gx = B * ((Ho + DH * strips - 1) / (DH * strips)) * tiles_w;
   launch_pdl(kern, dim3(gx, gy), dim3(TPB), sm, s, in, w, add, out, B, H, C, TW, strips, stats, bnb, xbn);
+}
+
+template <int K, int S, int DIL, bool X2, bool FLIP, bool XBN = false>
+static void dw_tile(cudaStream_t s, const bf16* in, const float* w, const bf16* add, bf16* out, int B, int H, int C,
+                    unsigned long long* stats = nullptr, const BnBwdFuse& bnb = BnBwdFuse(),
+                    const BnApplyIn& xbn = BnApplyIn()) {
+  if (dw_dh() == 16) dw_tile_dh<K, S, DIL, X2, FLIP, XBN, 16>(s, in, w, add, out, B, H, C, stats, bnb, xbn);
+  else dw_tile_dh<K, S, DIL, X2, FLIP, XBN, DT_H>(s, in, w, add, out, B, H, C, stats, bnb, xbn);
 }
 
 void dw_fwd(cudaStream_t s, const bf16* x, const float* w, bf16* z, int B, int H, int C, int k, int S, int dil,
