@@ -611,6 +611,10 @@ def main():
             e2e_hw = (w_step * 1e-12) / (D * pk[w_peak] * (ms / args.steps / 1000))
         elif fam == "spos":
             e2e_hw = (roofline["algorithmic_bytes_per_step"] * 1e-9) / (D * pk["hbm"] * (ms / args.steps / 1000))
+        # every kernel's algorithmic HBM bytes (stats all_bytes, counted by the library at each
+        # launch) over the value region: the whole step against the HBM roofline
+        all_b = reduce(s1["all_bytes"] - s0["all_bytes"], "sum") / args.steps
+        e2e_all = (all_b / (D * pk["hbm"] * 1e9 * (ms / args.steps / 1000))) if all_b > 0 else None
         plan_ms = (plan_bound_ms(cfg, npipe, timed_choices, D, [b for b in busy])
                    if args.sync == "csp" and args.virtual_stages == 1 else None)
         fractions = {"kernel": roofline["frac"],
@@ -619,6 +623,11 @@ def main():
                                                      if fam == "transformer" else
                                                      "BatchNorm algorithmic bytes only / (D x HBM peak x step time): "
                                                      "a lower bound (the conv kernels' bytes are not counted)"),
+                     "end_to_end_all_kernels_vs_hbm": e2e_all,
+                     "all_kernels_bytes_per_step": all_b if all_b > 0 else None,
+                     "end_to_end_all_kernels_note": ("every SPOS kernel's algorithmic HBM bytes (each tensor read / "
+                                                     "written once per launch at its stored width) / (D x HBM peak x "
+                                                     "step time)") if e2e_all else None,
                      "end_to_end_vs_csp_plan": (plan_ms / ms) if plan_ms else None,
                      "csp_plan_ms": plan_ms, "measured_ms": ms, "busy_ms_per_rank": [b / 1000 for b in busy]}
         top = sorted(per.items(), key=lambda kv: -kv[1][1])[:14]

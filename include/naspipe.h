@@ -292,7 +292,9 @@ int naspipe_get_trace(naspipe_t* h, int64_t* dst, size_t cap_tasks, size_t* n_ta
  * kernels; both counted whether or not TIMING is on), [8] dominant-kernel ms (TIMING flag
  * only), [9] residency loads, [10] residency evicts, [11] writebacks, [12] version checks
  * passed, [13] algorithmic flops of every tcgen05 GEMM launched by this process,
- * [14] tcgen05 GEMM launches of this process, [15] reserved. */
+ * [14] tcgen05 GEMM launches of this process, [15] algorithmic HBM bytes of every kernel
+ * the families launched (SPOS: each tensor read / written once per launch at its stored
+ * width; 0 for the other families). */
 int naspipe_get_stats(naspipe_t* h, double* dst16);
 
 /* Turn the dominant-kernel CUDA-event timing (stats [6..8]) on or off for the work submitted

@@ -19,7 +19,7 @@ FLAG_TRACE, FLAG_VERSION_CHECK, FLAG_NULL_KERNELS, FLAG_TIMING, FLAG_RECOMPUTE, 
 FLAG_TIMED = 64
 STATS_FIELDS = ["tasks", "kernel_launches", "h2d_bytes", "d2h_bytes", "p2p_bytes", "makespan_ticks",
                 "dominant_launches", "dominant_flops", "dominant_ms", "res_loads", "res_evicts",
-                "writebacks", "version_checks", "gemm_flops", "gemm_launches", "r15"]
+                "writebacks", "version_checks", "gemm_flops", "gemm_launches", "all_bytes"]
 
 _i32p = C.POINTER(C.c_int32)
 _i64p = C.POINTER(C.c_int64)

@@ -967,6 +967,10 @@ void Engine::get_stats(double* o) {
   o[7] = timer_.flops;
   o[8] = timer_.ms;
   o[12] = (double)version_checks_;
+  double fbytes = 0;
+  for (auto& st : st_)
+    if (st.local && st.fam) fbytes += st.fam->counters.bytes;
+  o[15] = fbytes;
   o[13] = (double)gemm_flop_count();
   o[14] = (double)gemm_launch_count();
 }

@@ -42,6 +42,9 @@ struct KernelTimer {
 
 struct FamilyCounters {
   uint64_t launches = 0;
+  // algorithmic HBM bytes of every kernel the family launched (SPOS: each tensor read and
+  // written once per launch at its stored width; stats [15], the whole-step roofline)
+  double bytes = 0;
 };
 
 class Family {

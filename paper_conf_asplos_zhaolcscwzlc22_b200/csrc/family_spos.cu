@@ -209,6 +209,7 @@ class SposFamily : public Family {
       const int H = spec_.raw.image_hw, C0 = spec_.raw.stem_channels;
       const int Po = (int)P(H / 2);
       spos_stem_conv(s, static_cast<const float*>(x_in), w_stem_, stem_z_, B_, H, C0);
+      counters.bytes += 4.0 * 3 * (double)P(H) + 4.0 * Po * C0;  // fp32 image in, z x2 out
       t_bn_stats(s, stem_z_, Po, C0, stem_mean_, stem_rstd_);
       t_bn_apply(s, stem_z_, Po, C0, stem_mean_, stem_rstd_, ones_s_, zeros_s_, 1, stem_y_[slot], C0, (size_t)Po * C0,
                  acc_f_);
@@ -268,17 +269,21 @@ class SposFamily : public Family {
     const bf16* xo = static_cast<const bf16*>(out);
     e.stats = acc_f_;  // fused bn_stats
     gemm_x2(s, PL, Ch, Cl, xo, xo + (size_t)PL * Cl, Cl, wh16_, wh16_ + (size_t)Ch * Cl, Cl, e);
+    counters.bytes += 4.0 * PL * Cl + 4.0 * PL * Ch;
     t_bn_apply(s, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, 1, rh_, Ch, (size_t)PL * Ch, acc_f_);
     gap_pool(s, rh_, B_, HW, Ch, gap_);
+    counters.bytes += 4.0 * PL * Ch;
     fc_ce(s, gap_, wf_, static_cast<const int*>(target), B_, Ch, ncls, logits_, dlogits_, loss_per_);
     ce_mean(s, loss_per_, B_, loss_dst);
     fc_dgap(s, dlogits_, wf_, B_, Ch, ncls, dgap_);
     head_bcast(s, dgap_, B_, HW, Ch, rh_);  // dr overwrites r (the mask is recomputed from z)
+    counters.bytes += 2.0 * PL * Ch;
     t_bn_bwd_reduce(s, rh_, Ch, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, 1);
     t_bn_bwd_apply(s, rh_, Ch, zh_, PL, Ch, hmean_, hrstd_, ones_, zeros_, ones_, zeros_, 0, 1, dzh_);
     e = GemmEpiParams();
     e.out = dy;
     gemm(s, PL, Cl, Ch, dzh_, false, Ch, wh16_, true, Cl, EPI_BF16, e);
+    counters.bytes += 2.0 * PL * Ch + 2.0 * PL * Cl;
     counters.launches += 9;
   }
 
@@ -341,6 +346,7 @@ class SposFamily : public Family {
     if (timer) timer->begin(s);
     bn_stats(s, z, Pp, C, acc_f_);
     if (timer) timer->end(s, 4.0 * Pp * C);
+    counters.bytes += 4.0 * Pp * C;
   }
   void t_bn_apply(cudaStream_t s, const bf16* z, int Pp, int C, float* mean, float* rstd, const float* g,
                   const float* b, int relu, bf16* y, int ldy, size_t yplane, unsigned long long* acc) {
@@ -353,12 +359,14 @@ class SposFamily : public Family {
       bn_apply(s, z, Pp, C, acc, tick_, mean, rstd, g, b, relu, y, ldy, yplane);
     }
     if (timer) timer->end(s, 8.0 * Pp * C);
+    counters.bytes += 8.0 * Pp * C;
   }
   void t_bn_bwd_reduce(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int Pp, int C, const float* mean,
                        const float* rstd, const float* g, const float* b, int relu) {
     if (timer) timer->begin(s);
     bn_bwd_reduce(s, dy, lddy, z, Pp, C, mean, rstd, g, b, relu, acc_b_);
     if (timer) timer->end(s, 6.0 * Pp * C);
+    counters.bytes += 6.0 * Pp * C;
   }
   void t_bn_bwd_apply(cudaStream_t s, const bf16* dy, int lddy, const bf16* z, int Pp, int C, const float* mean,
                       const float* rstd, const float* g, const float* b, float* gu, float* bu, int update, int relu,
@@ -379,6 +387,7 @@ class SposFamily : public Family {
       bn_bwd_apply(s, dy, lddy, z, Pp, C, mean, rstd, g, b, gu, bu, lr_, update, acc_b_, tick_ + 1, relu, dz);
     }
     if (timer) timer->end(s, 8.0 * Pp * C);
+    counters.bytes += 8.0 * Pp * C;
   }
 
   void block_fwd(int j, int c, size_t k, const bf16* x, bf16* out, cudaStream_t s) {
@@ -400,6 +409,7 @@ class SposFamily : public Family {
       main_plane = P(d.H_in) * (d.C_out / 2);
       cv += 2 * main_plane;
       chan_split(s, x, (int)P(d.H_in), d.C_out / 2, out, d.C_out, oplane, xm);
+      counters.bytes += 8.0 * P(d.H_in) * d.C_out;
       counters.launches++;
       main_in = xm;
       main_col = d.C_out / 2;
@@ -426,10 +436,12 @@ class SposFamily : public Family {
         r.xbn = pend;
         zacc = acc_f2_;
         dw_fwd_bn(s, pend, Pm + u.off_w, r.z, B_, u.H_in, u.cin, u.k, u.stride, u.dil, zacc);
+        counters.bytes += 4.0 * P(u.H_in) * u.cin + 4.0 * Po * u.cout;
         counters.launches++;
         pend = BnApplyIn();
       } else if (u.dw == 1) {
         dw_fwd(s, h, Pm + u.off_w, r.z, B_, u.H_in, u.cin, u.k, u.stride, u.dil, zacc);
+        counters.bytes += 4.0 * P(u.H_in) * u.cin + 4.0 * Po * u.cout;
         counters.launches++;
       } else if (u.dw == 2) {  // dense k x k (reading A40): x2 columns, 3-pass GEMM over K = k k cin
         const int gk = u.gemm_k();
@@ -437,6 +449,7 @@ class SposFamily : public Family {
         bf16* cols = cv;
         cv += 2 * cplane;
         im2col_x2(s, h, hplane, B_, u.H_in, u.cin, u.k, u.stride, cols, cplane);
+        counters.bytes += 4.0 * P(u.H_in) * u.cin + 4.0 * (double)cplane;
         counters.launches++;
         r.x = cols;  // the weight gradient reads the columns' hi plane
         GemmEpiParams e;  // the GEMM epilogue adds the BatchNorm sums of z (fused bn_stats)
@@ -444,12 +457,14 @@ class SposFamily : public Family {
         e.out2 = r.z + zplane;
         e.stats = acc_f_;
         gemm_x2(s, Po, u.cout, gk, cols, cols + cplane, gk, W16 + u.off_w16, W16 + half + u.off_w16, gk, e);
+        counters.bytes += 4.0 * (double)cplane + 4.0 * Po * u.cout;
       } else {
         GemmEpiParams e;  // the GEMM epilogue adds the BatchNorm sums of z (fused bn_stats)
         e.out = r.z;
         e.out2 = r.z + zplane;
         e.stats = acc_f_;
         gemm_x2(s, Po, u.cout, u.cin, h, h + hplane, u.cin, W16 + u.off_w16, W16 + half + u.off_w16, u.cin, e);
+        counters.bytes += 4.0 * Po * u.cin + 4.0 * Po * u.cout;
       }
       if (fuse_bna_ && u.dw == 0 && !last_of_branch(L, i) && L[i + 1].dw == 1) {
         // conv -> BN -> ReLU -> depthwise: no bn_apply; the depthwise conv applies it on load
@@ -538,12 +553,14 @@ class SposFamily : public Family {
     if (dst) {
       if (u.dw == 1) {
         dw_dgrad(s, dz, Pm + u.off_w, add, dst, B_, u.H_in, u.cin, u.k, u.stride, u.dil, fuse ? *fuse : BnBwdFuse());
+        counters.bytes += 2.0 * Po * u.cout + 2.0 * P(u.H_in) * u.cin * (add ? 2 : 1);
         counters.launches++;
       } else if (u.dw == 2) {  // dense: dcols = dz W (fp32), then the fixed-order column adjoint
         GemmEpiParams e;
         e.out = dcols_;
         gemm(s, Po, u.gemm_k(), u.cout, dz, false, u.cout, W16 + u.off_w16, true, u.gemm_k(), EPI_F32, e);
         col2im(s, dcols_, B_, u.H_in, u.cin, u.k, u.stride, add, dst);
+        counters.bytes += 2.0 * Po * u.cout + 8.0 * Po * u.gemm_k() + 2.0 * P(u.H_in) * u.cin * (add ? 2 : 1);
         counters.launches++;
       } else {
         NP_REQUIRE(add == nullptr, NASPIPE_EINTERNAL, "pw dgrad with an addend");
@@ -551,11 +568,13 @@ class SposFamily : public Family {
         e.out = dst;
         if (fuse) e.bnb = *fuse;
         gemm(s, Po, u.cin, u.cout, dz, false, u.cout, W16 + u.off_w16, true, u.cin, fuse ? EPI_BNBWD : EPI_BF16, e);
+        counters.bytes += 2.0 * Po * u.cout + 2.0 * Po * u.cin;
       }
     }
     cudaEventRecord(ev_dg_[ring_], s);
     cudaStreamWaitEvent(side_, ev_dg_[ring_], 0);
     if (u.dw == 1) {
+      counters.bytes += 2.0 * Po * u.cout + (r.xbn.z ? 4.0 : 2.0) * P(u.H_in) * u.cin;
       dw_wgrad_sgd(side_, dz, r.x, acc_w_, tick_ + 2, Um + u.off_w, lr_, B_, u.H_in, u.cin, u.k, u.stride, u.dil,
                    r.xbn.z ? &r.xbn : nullptr);
       counters.launches += 1;
@@ -565,6 +584,7 @@ class SposFamily : public Family {
       e.w16 = inplace ? W16 + u.off_w16 : nullptr;
       e.w16lo = inplace ? W16 + half + u.off_w16 : nullptr;
       e.lr = lr_;
+      counters.bytes += 2.0 * Po * u.cout + 2.0 * Po * u.gemm_k();
       gemm(side_, u.cout, u.gemm_k(), Po, dz, true, u.cout, r.x, true, u.gemm_k(), EPI_SGD, e, true);
     }
     cudaEventRecord(ev_wg_[ring_], side_);
@@ -604,6 +624,7 @@ class SposFamily : public Family {
     if (d.stride == 1) {
       if (need_dx) {
         chan_merge(s, dyb, d.C_out, h, (int)P(d.H_in), d.C_out / 2, dxb);
+        counters.bytes += 4.0 * P(d.H_in) * d.C_out;
         counters.launches++;
       }
       return;
